@@ -1,0 +1,329 @@
+#!/usr/bin/env python
+"""Benchmark of the BTED hot path (BASELINE.json metric) on B200.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config resnet18] [--impl ours|reference]
+
+A step = one pass of the whole hot path (Algorithm 2, PAPER.md:152-156:
+sample the batches, gather, Gram, m greedy select/deflate steps per batch,
+union, merge TED) over the synthetic AutoTVM conv2d pool of the config.
+Weak scaling: every rank runs cfg.B batches of M points per step
+(B_total = N_gpus * cfg.B), then the winners are all-gathered and merged.
+value = batch selections per second, whole job = steps * B_total * m / time
+(the merge TED's selections are NOT counted; its time is).
+
+Timing: W >= 3 untimed warm-up steps; barrier + cuda synchronize; CUDA events
+on the library's stream around exactly K steps; max over ranks.  Inputs are
+larger than L2 (K = 4 M^2 bytes = 1 GiB per batch at M = 16384, vs 126 MB L2).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "BTED selected points/sec and deflate-step HBM GB/s vs roofline at 1/2/4/8 B200"
+UNIT = "points/s"
+K2_NAME = "deflate_rescore_kernel"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="resnet18")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cpu-budget-s", type=float, default=15.0)
+    return ap.parse_args()
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            j = json.load(f)
+        return float(j["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs: torch copy, read+write bytes)"
+    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+# ------------------------------------------------------------------ clocks
+class Clocks:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                       "--format=csv,noheader,nounits", "-lms", "200"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+        time.sleep(0.3)
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        self.f.flush()
+        self.f.seek(0)
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in self.f.read().splitlines():
+            c = [x.strip() for x in line.split(",")]
+            if len(c) < 9:
+                continue
+            try:
+                sm.append(float(c[1]))
+                smax.append(float(c[2]))
+            except ValueError:
+                continue
+            for n, v in zip(names, c[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        os.unlink(self.f.name)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------ CPU oracle timing
+def oracle_points_per_s(Xb: np.ndarray, gamma: float, mu: float, m: int, budget_s: float):
+    """The fp64 oracle (oracle/ted_dense.c, all host cores) on one full batch:
+    Gram + as many of the m greedy steps as fit in ~budget_s; the m-step TED
+    time is extrapolated from the measured per-step time."""
+    from oracle import dense
+    t0 = time.perf_counter()
+    K = dense.gram(Xb, gamma)
+    t_gram = time.perf_counter() - t0
+    steps, t_steps = 0, 0.0
+    while steps < m and (steps == 0 or t_steps < budget_s):
+        t1 = time.perf_counter()
+        # one greedy step of Alg. 1 on the current (in-place deflated) K
+        dense.ted_on_matrix(K, mu, 1)
+        t_steps += time.perf_counter() - t1
+        steps += 1
+    del K
+    t_ted = t_gram + m * (t_steps / steps)
+    return m / t_ted, t_gram, t_steps / steps, steps, dense.num_threads()
+
+
+def bench_reference(args):
+    """--impl reference: the oracle IS the reference arm (no reference code exists)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    from oracle.sampling import sample_batches
+    from synth import config_pool
+    X, gamma, cfg = config_pool(args.config)
+    mu = float(np.float32(cfg["mu"]))
+    V = sample_batches(X.shape[0], cfg["M"], 1, cfg["seed"])[0]
+    Xb = X[V]
+    budget = max(1.0, min(args.cpu_budget_s, 10.0))
+    vals, times = [], []
+    for it in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        v, tg, ts, n, cores = oracle_points_per_s(Xb, gamma, mu, cfg["m"], budget_s=budget / 4)
+        if it >= args.warmup:
+            vals.append(v)
+            times.append(time.perf_counter() - t0)
+    value = float(statistics.median(vals))
+    sample = (f"per step: oracle Gram of batch 0 (N={cfg['M']}, d={cfg['d']}) + {n} of {cfg['m']} greedy "
+              f"steps; points/s extrapolated to the full {cfg['m']}-step TED (batch selections only)")
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * float(np.mean(times)),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": workload_config(args.config, cfg, gamma, 1),
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def workload_config(name, cfg, gamma, world):
+    return {"workload": f"{name}: BTED on the AutoTVM conv2d knob pool of {cfg['workload']} "
+                        f"(P={cfg['pool']} configs, d={cfg['d']}), B={cfg['B'] * world} batches of "
+                        f"M={cfg['M']}, m={cfg['m']}, mu={cfg['mu']}, RBF gamma={gamma:.6g} (median heuristic)",
+            "pool": cfg["pool"], "M": cfg["M"], "d": cfg["d"], "m": cfg["m"], "B": cfg["B"] * world,
+            "batches_per_gpu": cfg["B"], "mu": cfg["mu"], "seed": cfg["seed"],
+            "l2": "inputs larger than L2: K = 4*M^2 bytes per batch (1 GiB at M=16384) >> 126 MB",
+            "parallelism": f"batch round-robin over {world} GPU(s)" if world > 1 else "1 GPU"}
+
+
+# ------------------------------------------------------------------ ours
+def bench_ours(args):
+    import torch
+    import paper_conf_date_sunbg021_b200 as bt
+    from paper_conf_date_sunbg021_b200 import _lib as L
+    from paper_conf_date_sunbg021_b200.dist import TorchComm, run_batches_dp
+    from synth import config_pool
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    comm = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+        comm = TorchComm()
+
+    X, gamma, cfg = config_pool(args.config)
+    mu = float(np.float32(cfg["mu"]))
+    M, m, d, P = cfg["M"], cfg["m"], cfg["d"], X.shape[0]
+    B = cfg["B"] * world
+    stream = torch.cuda.Stream(dev)
+    X_dev = torch.from_numpy(X).to(dev)
+    torch.cuda.synchronize()
+    pool = bt.CandidateSet(X_dev, gamma, num_batches=B, seed=cfg["seed"], device=local,
+                           flags=L.BTED_FLAG_TIMING, stream=stream.cuda_stream)
+
+    def step():
+        if world == 1:
+            return pool.run_batches(M, m, mu, want_batches=False)[0]
+        with torch.cuda.stream(stream):
+            return run_batches_dp(pool.ctx, M, m, mu, B, comm, dev)[0]
+
+    def barrier():
+        if world > 1:
+            torch.distributed.barrier()
+
+    def max_over_ranks(v: float) -> float:
+        if world == 1:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        return float(t.item())
+
+    for _ in range(args.warmup):
+        step()
+    L.bted_reset_stats(pool.ctx)
+    clocks = Clocks(local)
+    clocks.start()
+    l0 = bt.bted_kernel_launches()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier()
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for _ in range(args.steps):
+        sel = step()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    launches = bt.bted_kernel_launches() - l0
+    ms = max_over_ranks(e0.elapsed_time(e1))
+    clk = clocks.stop()
+    stats = L.bted_get_stats(pool.ctx)
+    value = args.steps * B * m / (ms / 1e3)
+
+    # roofline of the dominant kernel K2 (fused deflate + rescore), live events
+    peak, peak_src = peaks()
+    k2_avg_ms = stats["k2_ms"] / max(stats["k2_launches"], 1)
+    alg_bytes = 8.0 * M * M                       # fp32 read + write of K per launch (8 N^2)
+    achieved = alg_bytes / (k2_avg_ms / 1e3) / 1e9
+    traffic = None
+    tj = os.path.join(ROOT, "profiles", "k2_traffic.json")
+    if os.path.exists(tj):
+        with open(tj) as f:
+            tjd = json.load(f)
+        if tjd.get("M") == M:
+            traffic = tjd.get("dram_bytes_per_launch")
+
+    # end to end through the public API with HOST buffers (pinned), per step:
+    # H2D of the pool, the whole BTED, D2H of the result
+    e2e = None
+    if not args.no_e2e:
+        Xh = torch.from_numpy(X).pin_memory()
+        ctx2 = bt.CandidateSet(Xh.numpy(), gamma, num_batches=B, seed=cfg["seed"], device=local,
+                               stream=stream.cuda_stream)
+        for _ in range(max(1, args.warmup)):
+            L.bted_update(ctx2.ctx, Xh.data_ptr())
+            if world == 1:
+                ctx2.run_batches(M, m, mu, want_batches=False)
+            else:
+                with torch.cuda.stream(stream):
+                    run_batches_dp(ctx2.ctx, M, m, mu, B, comm, dev)
+        barrier()
+        torch.cuda.synchronize()
+        f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        f0.record(stream)
+        for _ in range(args.steps):
+            L.bted_update(ctx2.ctx, Xh.data_ptr())
+            if world == 1:
+                ctx2.run_batches(M, m, mu, want_batches=False)
+            else:
+                with torch.cuda.stream(stream):
+                    run_batches_dp(ctx2.ctx, M, m, mu, B, comm, dev)
+        f1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ems = max_over_ranks(f0.elapsed_time(f1))
+        ctx2.close()
+        e2e = {"value": args.steps * B * m / (ems / 1e3), "unit": UNIT,
+               "h2d_bytes_per_step": int(P * d * 4),
+               "d2h_bytes_per_step": int(8 * m + 4 + 8 * m + 4 + 4)}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        from oracle.sampling import sample_batches
+        V = sample_batches(P, M, 1, cfg["seed"])[0]
+        v, tg, ts, n, cores = oracle_points_per_s(X[V], gamma, mu, m, args.cpu_budget_s)
+        cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": (f"batch 0 (N={M}): fp64 Gram ({tg:.2f} s) + {n} of {m} greedy steps "
+                          f"({ts:.3f} s/step) with the dense C/OpenMP oracle; points/s of the full "
+                          f"{m}-step TED extrapolated from those")}
+
+    pool.close()
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": workload_config(args.config, cfg, gamma, world),
+                "roofline": {"bound": "hbm", "kernel": K2_NAME, "achieved": achieved, "peak": peak,
+                             "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
+                             "frac_of_8TBs": achieved / 8000.0, "peak_source": peak_src,
+                             "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": k2_avg_ms,
+                             "launches_timed": stats["k2_launches"],
+                             "k2_share_of_step": (stats["k2_ms"] / ms) if ms > 0 else None,
+                             "k1_ms_per_batch": stats["k1_ms"] / max(stats["teds"], 1)},
+                "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
+                "final_selection_head": [int(x) for x in sel[:8]]}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+def main():
+    args = parse()
+    if args.warmup < 3:
+        print("warning: --warmup < 3 violates the timing rules; using 3", file=sys.stderr)
+        args.warmup = 3
+    if args.impl == "reference":
+        bench_reference(args)
+    else:
+        bench_ours(args)
+
+
+if __name__ == "__main__":
+    main()

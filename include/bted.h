@@ -1,0 +1,218 @@
+/*
+ * bted.h -- C ABI of the B200-native BTED hot path (libbted.so).
+ *
+ * Batch Transductive Experimental Design, Sun, Bai, Geng, Yu, "Deep Neural
+ * Network Hardware Deployment Optimization via Advanced Active Learning",
+ * DATE 2021.  Citations are to /root/reference/PAPER.md (line, section).
+ *
+ *   TED(V, mu, m)         Algorithm 1, PAPER.md:134-148 (Sec. III-A)
+ *   BTED(V, mu, M, m, B)  Algorithm 2, PAPER.md:152-156 (Sec. III-A)
+ *
+ * Readings of the paper adopted by this library:
+ *   k(v1,v2) = exp(-gamma ||v1-v2||^2) (RBF; PAPER.md:130 says "Euclidean
+ *   distance", which is ill-posed for TED); the argmax of Alg.1 l.3 runs over
+ *   not-yet-selected points; ties go to the lowest index; l.5 deflates the
+ *   whole matrix; indices are returned in selection order.
+ *
+ * Conventions for every entry point:
+ *   - All pointers are plain host pointers unless a parameter says "device".
+ *     Output buffers are caller-allocated; the library never keeps a caller
+ *     pointer after return, except a device X adopted with x_on_device = 1,
+ *     which must outlive the context.
+ *   - Feature matrices are row-major fp32, N rows x d columns, contiguous.
+ *   - Every call returns a bted_status; no C++ exception crosses the ABI.
+ *     On error the outputs are unspecified and bted_last_error() returns a
+ *     thread-local description.  After a CUDA error the context is poisoned
+ *     (BTED_ESTATE on later calls).
+ *   - A context is not thread-safe; distinct contexts may be used from
+ *     distinct threads.  All work of a context runs on its CUDA stream.
+ *   - There is no CPU fallback: without a usable sm_100 device every compute
+ *     entry point fails with BTED_ECUDA.
+ */
+#ifndef BTED_H_
+#define BTED_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct bted_ctx bted_ctx;    /* opaque; owns the device memory of one candidate set */
+
+typedef enum {
+    BTED_KERNEL_RBF = 0,     /* k(x,y) = exp(-gamma ||x-y||^2)          (reading A1) */
+    BTED_KERNEL_LINEAR = 1   /* k(x,y) = x.y  -- test-only (closed-form pin C8)    */
+} bted_kernel;
+
+typedef enum {
+    BTED_OK = 0,
+    BTED_EINVAL = 1,         /* invalid argument (see each call)                    */
+    BTED_ENOMEM = 2,         /* device or host allocation failed                    */
+    BTED_ECUDA = 3,          /* CUDA runtime error / no usable device               */
+    BTED_ENCCL = 4,          /* reserved for collective failures                    */
+    BTED_ENUMERIC = 5,       /* NaN score or non-positive k(v,v)+mu during a run    */
+    BTED_ESTATE = 6          /* context poisoned by an earlier CUDA error           */
+} bted_status;
+
+/* flags */
+#define BTED_FLAG_NO_GRAPH 1u   /* launch the m-step loop eagerly (debug / profiling) */
+#define BTED_FLAG_TIMING   2u   /* record CUDA events around K1 and the K2 loop of every batch
+                                   TED on the ctx stream; read with bted_get_stats()          */
+
+typedef struct {
+    float     gamma;         /* RBF bandwidth, > 0 and finite (ignored for LINEAR)      */
+    int32_t   device;        /* CUDA device ordinal; -1 = the calling thread's current  */
+    int32_t   num_batches;   /* B of Algorithm 2 (bted_run_batches), >= 1              */
+    uint64_t  seed;          /* batch sampling seed (Alg. 2 l.2, reading A10)          */
+    int32_t   x_on_device;   /* 1: X is a device pointer on `device` (adopted, not copied) */
+    uint32_t  flags;         /* BTED_FLAG_*                                           */
+    uintptr_t stream;        /* cudaStream_t to run on; 0 = a stream owned by the ctx  */
+} bted_params;
+
+/* Fill *p with defaults: gamma 1, device -1, num_batches 1, seed 0, host X,
+ * flags 0, own stream. */
+void bted_default_params(bted_params* p);
+
+/*
+ * bted_create -- a candidate set V ("the input un-sampled set V").
+ *   X: N x d row-major fp32 features (Def. 1), host pointer (copied
+ *      to the device) or, with params->x_on_device, a device pointer (adopted).
+ *   N: 1 <= N < 2^31.  d: 1 <= d <= 64.  All X finite.  gamma > 0 for RBF.
+ *   Nothing N x N is allocated here (a pool may have 2^20 rows).
+ *   Errors: EINVAL (bad sizes, non-finite X or gamma), ENOMEM, ECUDA.
+ */
+bted_status bted_create(const float* X, int64_t N, int32_t d, bted_kernel kernel,
+                        const bted_params* params, bted_ctx** out);
+
+/*
+ * bted_select -- TED(V, mu, m), Algorithm 1 on all N rows.
+ *   Builds K = K_VV (l.1), then m times: score_v = ||K_v||^2/(k(v,v)+mu) over
+ *   unselected v, x = argmax (lowest index on ties), X = X u x, and
+ *   K = K - K_x K_x^T/(k(x,x)+mu) (l.3-5; the deflation after the m-th pick is
+ *   skipped because it cannot change X).
+ *   out_idx   [m] row indices in selection order (host).
+ *   out_score [m] nullable: fp32 score of each pick at the step it was taken.
+ *   Idempotent: each call restarts from the fresh Gram matrix.  Allocates
+ *   2 N^2 fp32 (ping-pong K) on first use at this N.
+ *   Errors: EINVAL (m < 1, m > N, mu <= 0 or non-finite), ENOMEM, ECUDA,
+ *   ENUMERIC, ESTATE.
+ */
+bted_status bted_select(bted_ctx* ctx, int32_t m, float mu,
+                        int64_t* out_idx, float* out_score);
+
+/*
+ * bted_run_batches -- BTED(V, mu, M, m, B), Algorithm 2
+ * with V = the ctx's rows (the pool) and B = params.num_batches:
+ *   l.1-4  for b in 0..B-1: V_b = bted_sample_batches(P, M, B, seed)[b];
+ *          X_b = V_b[TED(X[V_b], mu, m)]
+ *   l.5    X_U = sorted unique(X_0 u ... u X_{B-1})
+ *   l.6    X = X_U[TED(X[X_U], mu, min(m, |X_U|))]   (fresh Gram of X_U)
+ *   M: m <= M <= N (N = pool rows, < 2^32).  All steps run on the device;
+ *   only the |X_U| count and the results cross to the host.
+ *   out_idx [m] pool row indices of X in selection order; *out_count =
+ *   min(m, |X_U|).  out_batch_idx nullable [B*m]: row b = X_b in selection
+ *   order.
+ *   Errors: as bted_select, plus EINVAL for M < m or M > N.
+ */
+bted_status bted_run_batches(bted_ctx* pool, int64_t M, int32_t m, float mu,
+                             int64_t* out_idx, int32_t* out_count,
+                             int64_t* out_batch_idx);
+
+/*
+ * bted_batch_teds -- Algorithm 2 lines 1-4 only, for the batches
+ * b = b_begin, b_begin + b_step, ... < B (round-robin sharding of the
+ * batches over processes/GPUs).  Writes X_b (pool indices, selection order)
+ * to out_winners[k*m .. k*m+m-1] for the k-th batch it runs.
+ *   out_winners: host pointer, or a device pointer on the ctx's device when
+ *   winners_on_device = 1 (e.g. a torch tensor that is then all-gathered).
+ */
+bted_status bted_batch_teds(bted_ctx* pool, int64_t M, int32_t m, float mu,
+                            int32_t b_begin, int32_t b_step,
+                            int64_t* out_winners, int32_t winners_on_device);
+
+/*
+ * bted_merge -- Algorithm 2 lines 5-6: X_U = sorted unique(winners[0..n)),
+ * then TED(X[X_U], mu, min(m, |X_U|)) on a fresh Gram matrix of X_U.
+ *   winners: n pool indices (host, or device with winners_on_device = 1);
+ *   negative entries are padding and ignored (e.g. the fill of an
+ *   all-gather over ranks with unequal batch counts).
+ *   out_idx [m] host; *out_count = min(m, |X_U|).
+ */
+bted_status bted_merge(bted_ctx* pool, const int64_t* winners, int64_t n,
+                       int32_t winners_on_device, int32_t m, float mu,
+                       int64_t* out_idx, int32_t* out_count);
+
+/*
+ * bted_sample_batches -- Algorithm 2 line 2 draws (reading A10): for each b,
+ * the M indices i in [0, P) with the smallest
+ *   key_b(i) = (splitmix64(splitmix64(seed + b*0xD1B54A32D192ED03) + i)
+ *               & 0xFFFFFFFF00000000) | i,
+ * in ascending order of i.  Computed on the
+ * current CUDA device.  out: host [B*M].  1 <= M <= P < 2^32, B >= 1.
+ */
+bted_status bted_sample_batches(int64_t P, int64_t M, int32_t B, uint64_t seed,
+                                int64_t* out);
+
+/* ---------------- row-sharded TED (one oversized batch over P GPUs) -------------
+ * A shard context owns rows [row0, row1) of the N x N matrix K of the full
+ * candidate set X (X is replicated: N x d).  The per-step exchange is done by
+ * the caller between calls (torch.distributed / NCCL), all on the shard's
+ * stream, so the loop can be captured in a CUDA graph:
+ *   bted_shard_gram(t=0)  -> keys[0] holds this shard's best key
+ *   all-reduce(keys[t], MAX)                      (8 bytes)
+ *   bted_shard_pivot_column(t) -> col = K[row0:row1, s_t]
+ *   all-gather(col) -> pivot (N floats, = row s_t of K by bit-symmetry)
+ *   bted_shard_step(t+1, pivot) -> keys[t+1]
+ * keys: device u64 [m] owned by the caller, zeroed before t = 0.  A key packs
+ * (score bits + 1) << 32 | (0xFFFFFFFF - index); 0 = no candidate.
+ */
+bted_status bted_shard_create(const float* X, int64_t N, int32_t d, bted_kernel kernel,
+                              int64_t row0, int64_t row1, const bted_params* params,
+                              bted_ctx** out);
+bted_status bted_shard_gram(bted_ctx* shard, float mu, uint64_t* keys_dev);
+bted_status bted_shard_step(bted_ctx* shard, int32_t t, float mu, const float* pivot_dev,
+                            uint64_t* keys_dev);
+bted_status bted_shard_pivot_column(bted_ctx* shard, int32_t t, const uint64_t* keys_dev,
+                                    float* col_dev);
+/* Leading dimension (floats) a pivot buffer must have: pivot_dev[N..ld) must be 0. */
+int64_t     bted_shard_ld(const bted_ctx* shard);
+/* Sticky device error flag of the shard (BTED_ENUMERIC if a NaN score was seen). */
+bted_status bted_shard_check(bted_ctx* shard);
+
+/*
+ * bted_update -- replace the features of a ctx (same N, d) for the next call:
+ * a pool of the same shape (e.g. the next tuning node).  Host X is copied
+ * H2D asynchronously on the ctx stream (pinned memory makes it a DMA; the
+ * caller keeps X alive until its next call on this ctx returns); a device X
+ * (x_on_device = 1) is copied D2D.  Errors: EINVAL, ECUDA, ESTATE.
+ */
+bted_status bted_update(bted_ctx* ctx, const float* X, int32_t x_on_device);
+
+/* Accumulated device timings of the TEDs run by a ctx (BTED_FLAG_TIMING):
+ * k1_ms = transpose + Gram (Alg. 1 l.1 + first l.3), k2_ms = the fused
+ * deflate/rescore loop (k2_launches launches of the K2 kernel), measured
+ * with CUDA events on the ctx stream.  Merge TEDs are not included. */
+typedef struct {
+    uint64_t teds;
+    uint64_t k2_launches;
+    double   k1_ms;
+    double   k2_ms;
+} bted_stats;
+bted_status bted_get_stats(bted_ctx* ctx, bted_stats* out);
+bted_status bted_reset_stats(bted_ctx* ctx);
+
+/* ---------------- introspection ---------------- */
+void        bted_destroy(bted_ctx* ctx);
+const char* bted_status_string(bted_status s);
+const char* bted_last_error(void);
+/* Number of kernels this library launched since load (all contexts). */
+uint64_t    bted_kernel_launches(void);
+/* Debug: copy the current fp32 K (rows x ld) of ctx's last select to host.
+ * Only valid with BTED_FLAG_NO_GRAPH runs or after bted_select returns. */
+bted_status bted_debug_copy_K(bted_ctx* ctx, int32_t which, float* out, int64_t* ld_out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BTED_H_ */

@@ -1,0 +1,841 @@
+// bted.cu -- TED engine (Alg. 1), BTED scheduler (Alg. 2) and the C ABI of
+// include/bted.h.  PAPER.md:134-156.  Built into libbted.so for sm_100a.
+//
+// Per TED (bted_select / every batch of bted_run_batches) the device runs
+//   transpose X -> XT, zero keys/sel, K1 gram_rownorm (l.1 + first l.3),
+//   then m-1 times K2 deflate_rescore (l.5 + next l.3) on ping-pong K buffers,
+// captured once per (X, N, d, m, mu, gamma) into a CUDA graph.  The pivot
+// of step t is read ON THE DEVICE from keys[t-1]; the host sees only the
+// m packed keys at the end (no per-step host round trip).
+#include <cub/cub.cuh>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <list>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/bted.h"
+#include "kernels.cuh"
+#include "sample.cuh"
+
+namespace {
+
+thread_local std::string g_last_error;
+std::atomic<uint64_t> g_launches{0};
+
+void set_error(const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_last_error = buf;
+}
+
+struct CudaError {
+    cudaError_t e;
+    const char* what;
+};
+
+#define CK(expr)                                                         \
+    do {                                                                 \
+        cudaError_t _e = (expr);                                         \
+        if (_e != cudaSuccess) throw CudaError{_e, #expr};               \
+    } while (0)
+#define LAUNCHED(n) g_launches.fetch_add((n), std::memory_order_relaxed)
+
+constexpr int kK1Rows = 16, kK1Threads = 256;
+constexpr int kK2Rows = 2, kK2Unroll = 4, kK2Threads = 256;
+constexpr int kRowsPerK2Cta = (kK2Threads / 32) * kK2Rows;
+
+inline int64_t round_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
+inline int64_t ld_for(int64_t N) { return round_up(N, 32); }
+inline uint32_t fbits(float f) { uint32_t u; std::memcpy(&u, &f, 4); return u; }
+
+template <class T>
+void grow(T*& p, size_t& cap, size_t n) {
+    if (n <= cap) return;
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    CK(cudaMalloc(&p, sizeof(T) * n));
+    cap = n;
+}
+
+// ------------------------------------------------------------------ TED engine
+struct GraphKey {
+    const float* X;
+    int64_t N;
+    int32_t d, m, kernel, part;   // part 0 = head (transpose, K1), 1 = loop (m-1 x K2)
+    uint32_t mu, gamma;
+    const void* keys;
+    bool operator==(const GraphKey& o) const {
+        return X == o.X && N == o.N && d == o.d && m == o.m && kernel == o.kernel && part == o.part &&
+               mu == o.mu && gamma == o.gamma && keys == o.keys;
+    }
+};
+
+struct Stats {
+    uint64_t teds = 0, k2_launches = 0;
+    double k1_ms = 0, k2_ms = 0;
+};
+
+struct Ted {
+    cudaStream_t stream = nullptr;
+    float* K[2] = {nullptr, nullptr};
+    size_t kcap[2] = {0, 0};
+    float* XT = nullptr;
+    size_t xtcap = 0;
+    uint8_t* sel = nullptr;
+    size_t selcap = 0;
+    unsigned long long* keys = nullptr;
+    size_t keyscap = 0;
+    int* err = nullptr;
+    size_t errcap = 0;
+    std::list<std::pair<GraphKey, cudaGraphExec_t>> graphs;   // LRU
+    int64_t last_rows = 0, last_ld = 0;
+    int last_buf = 0;
+    // timing (BTED_FLAG_TIMING): events recorded on the stream around the
+    // head and loop graphs of each TED, read back at the next host sync.
+    bool timing = false;
+    struct Slot { cudaEvent_t e[3]; int32_t m; };
+    std::vector<Slot> slots;
+    size_t used = 0;
+    Stats stats;
+
+    void release() {
+        for (auto& g : graphs) cudaGraphExecDestroy(g.second);
+        graphs.clear();
+        for (int b = 0; b < 2; ++b) if (K[b]) cudaFree(K[b]);
+        if (XT) cudaFree(XT);
+        if (sel) cudaFree(sel);
+        if (keys) cudaFree(keys);
+        if (err) cudaFree(err);
+        for (auto& sl : slots) for (auto e : sl.e) cudaEventDestroy(e);
+        slots.clear();
+        K[0] = K[1] = nullptr; XT = nullptr; sel = nullptr; keys = nullptr; err = nullptr;
+    }
+
+    // Buffers for a band of `rows` rows of an N x N problem.
+    // Any reallocation invalidates the captured graphs (they hold raw pointers).
+    void reserve(int64_t rows, int64_t N, int32_t d, int32_t m) {
+        const int64_t ld = ld_for(N);
+        const void* before[5] = {K[0], K[1], XT, sel, keys};
+        grow(K[0], kcap[0], (size_t)(rows * ld));
+        if (m > 1) grow(K[1], kcap[1], (size_t)(rows * ld));
+        grow(XT, xtcap, (size_t)(d * ld));
+        grow(sel, selcap, (size_t)rows);
+        grow(keys, keyscap, (size_t)std::max(m, 1));
+        if (!err) { grow(err, errcap, 1); CK(cudaMemsetAsync(err, 0, sizeof(int), stream)); }
+        const void* after[5] = {K[0], K[1], XT, sel, keys};
+        if (std::memcmp(before, after, sizeof before) != 0) {
+            for (auto& g : graphs) cudaGraphExecDestroy(g.second);
+            graphs.clear();
+        }
+    }
+
+    Slot* next_slot(int32_t m) {
+        if (used == slots.size()) {
+            Slot sl{};
+            for (auto& e : sl.e) CK(cudaEventCreate(&e));
+            slots.push_back(sl);
+        }
+        Slot* sl = &slots[used++];
+        sl->m = m;
+        return sl;
+    }
+
+    // after a host sync of `stream`: fold the recorded TEDs into stats
+    void collect() {
+        for (size_t i = 0; i < used; ++i) {
+            float a = 0, b = 0;
+            CK(cudaEventElapsedTime(&a, slots[i].e[0], slots[i].e[1]));
+            stats.k1_ms += a;
+            if (slots[i].m > 1) {
+                CK(cudaEventElapsedTime(&b, slots[i].e[1], slots[i].e[2]));
+                stats.k2_ms += b;
+                stats.k2_launches += (uint64_t)(slots[i].m - 1);
+            }
+            stats.teds += 1;
+        }
+        used = 0;
+    }
+};
+
+void launch_transpose(Ted& T, const float* X, int64_t N, int32_t d) {
+    const int64_t ld = ld_for(N);
+    bted::transpose_pad_kernel<<<(unsigned)((ld + 255) / 256), 256, 0, T.stream>>>(X, (int32_t)N, d, T.XT, ld);
+    LAUNCHED(1);
+}
+
+void launch_gram(Ted& T, int64_t N, int32_t d, int64_t row0, int64_t rows, float gamma, int kernel,
+                 float mu, unsigned long long* key_out) {
+    const int64_t ld = ld_for(N);
+    const unsigned grid = (unsigned)((rows + kK1Rows - 1) / kK1Rows);
+    const size_t smem = sizeof(float) * kK1Rows * d;
+    bted::gram_rownorm_kernel<kK1Rows, kK1Threads><<<grid, kK1Threads, smem, T.stream>>>(
+        T.XT, ld, d, (int32_t)N, (int32_t)row0, (int32_t)rows, gamma, kernel == BTED_KERNEL_LINEAR ? 1 : 0,
+        T.K[0], mu, key_out, T.err);
+    LAUNCHED(1);
+}
+
+void launch_step(Ted& T, int64_t N, int64_t row0, int64_t rows, int32_t t, float mu, const float* pivot,
+                 unsigned long long* keys) {
+    const int64_t ld = ld_for(N);
+    const unsigned grid = (unsigned)((rows + kRowsPerK2Cta - 1) / kRowsPerK2Cta);
+    bted::deflate_rescore_kernel<kK2Rows, kK2Unroll, kK2Threads><<<grid, kK2Threads, 0, T.stream>>>(
+        T.K[(t - 1) & 1], T.K[t & 1], ld, (int32_t)row0, (int32_t)rows, pivot, keys, t, mu, T.sel, T.err);
+    LAUNCHED(1);
+}
+
+// Alg. 1 l.1 + first l.3: XT, zero keys/sel, K1.  (2 kernels)
+void enqueue_head(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
+                  unsigned long long* keys) {
+    launch_transpose(T, X, N, d);
+    CK(cudaMemsetAsync(keys, 0, sizeof(unsigned long long) * m, T.stream));
+    CK(cudaMemsetAsync(T.sel, 0, (size_t)N, T.stream));
+    launch_gram(T, N, d, 0, N, gamma, kernel, mu, keys);
+}
+// Alg. 1 l.2-6 loop: m-1 fused deflate + rescore steps.  (m-1 kernels)
+void enqueue_loop(Ted& T, int64_t N, int32_t m, float mu, unsigned long long* keys) {
+    for (int32_t t = 1; t < m; ++t) launch_step(T, N, 0, N, t, mu, nullptr, keys);
+}
+
+template <class F>
+void graph_run(Ted& T, const GraphKey& key, uint64_t nkernels, F&& enqueue) {
+    for (auto it = T.graphs.begin(); it != T.graphs.end(); ++it) {
+        if (it->first == key) {
+            T.graphs.splice(T.graphs.begin(), T.graphs, it);
+            CK(cudaGraphLaunch(it->second, T.stream));
+            LAUNCHED(nkernels);
+            return;
+        }
+    }
+    cudaGraph_t g = nullptr;
+    CK(cudaStreamBeginCapture(T.stream, cudaStreamCaptureModeThreadLocal));
+    const uint64_t before = g_launches.load();
+    try {
+        enqueue();
+    } catch (...) {
+        cudaStreamEndCapture(T.stream, &g);
+        if (g) cudaGraphDestroy(g);
+        throw;
+    }
+    g_launches.store(before);   // captured launches run below, counted there
+    CK(cudaStreamEndCapture(T.stream, &g));
+    cudaGraphExec_t ex = nullptr;
+    cudaError_t e = cudaGraphInstantiate(&ex, g, 0);
+    cudaGraphDestroy(g);
+    CK(e);
+    T.graphs.emplace_front(key, ex);
+    while (T.graphs.size() > 16) {
+        cudaGraphExecDestroy(T.graphs.back().second);
+        T.graphs.pop_back();
+    }
+    CK(cudaGraphLaunch(ex, T.stream));
+    LAUNCHED(nkernels);
+}
+
+// Run one TED (graph-cached unless no_graph); results stay on the device.
+void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
+             unsigned long long* keys, bool no_graph, bool time_it = true) {
+    T.reserve(N, N, d, m);
+    T.last_rows = N;
+    T.last_ld = ld_for(N);
+    T.last_buf = (m - 1) & 1;
+    Ted::Slot* sl = (T.timing && time_it) ? T.next_slot(m) : nullptr;
+    if (sl) CK(cudaEventRecord(sl->e[0], T.stream));
+    if (no_graph) {
+        enqueue_head(T, X, N, d, gamma, kernel, m, mu, keys);
+    } else {
+        GraphKey key{X, N, d, m, kernel, 0, fbits(mu), fbits(gamma), keys};
+        graph_run(T, key, 2, [&] { enqueue_head(T, X, N, d, gamma, kernel, m, mu, keys); });
+    }
+    if (sl) CK(cudaEventRecord(sl->e[1], T.stream));
+    if (m > 1) {
+        if (no_graph) {
+            enqueue_loop(T, N, m, mu, keys);
+        } else {
+            GraphKey key{X, N, d, m, kernel, 1, fbits(mu), fbits(gamma), keys};
+            graph_run(T, key, (uint64_t)(m - 1), [&] { enqueue_loop(T, N, m, mu, keys); });
+        }
+    }
+    if (sl) CK(cudaEventRecord(sl->e[2], T.stream));
+}
+
+bool all_finite(const float* X, int64_t n) {
+    for (int64_t i = 0; i < n; ++i)
+        if (!std::isfinite(X[i])) return false;
+    return true;
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------ context
+struct bted_ctx {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    bted_kernel kernel = BTED_KERNEL_RBF;
+    bted_params params{};
+    int64_t N = 0;
+    int32_t d = 0;
+    float* X = nullptr;       // device N x d
+    bool own_X = false;
+    bool poisoned = false;
+    // shard
+    bool is_shard = false;
+    int64_t row0 = 0, row1 = 0;
+    Ted ted;
+    // batches (Alg. 2)
+    Ted bted_engine;          // the M x M batch TEDs and the merge TED
+    uint64_t* skeys = nullptr; size_t skeyscap = 0;
+    uint64_t* skeys2 = nullptr; size_t skeys2cap = 0;
+    uint32_t* sidx = nullptr; size_t sidxcap = 0;
+    uint32_t* sidx2 = nullptr; size_t sidx2cap = 0;
+    float* Xb = nullptr; size_t xbcap = 0;
+    int64_t* winners = nullptr; size_t winnerscap = 0;
+    uint32_t* u32a = nullptr; size_t u32acap = 0;
+    uint32_t* u32b = nullptr; size_t u32bcap = 0;
+    int* count_dev = nullptr; size_t countcap = 0;
+    unsigned long long* mkeys = nullptr; size_t mkeyscap = 0;
+    void* cub_tmp = nullptr; size_t cub_cap = 0;
+    int64_t* out_dev = nullptr; size_t outcap = 0;
+    // host staging (pinned)
+    unsigned long long* hkeys = nullptr; size_t hkeyscap = 0;
+    int* herr = nullptr;
+};
+
+namespace {
+
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        cudaGetDevice(&prev);
+        if (prev != dev) cudaSetDevice(dev);
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        cudaGetDevice(&cur);
+        if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+void host_grow(unsigned long long*& p, size_t& cap, size_t n) {
+    if (n <= cap) return;
+    if (p) cudaFreeHost(p);
+    p = nullptr;
+    cap = 0;
+    CK(cudaMallocHost(&p, sizeof(unsigned long long) * n));
+    cap = n;
+}
+
+template <class F>
+bted_status guarded(bted_ctx* ctx, F&& f) {
+    if (!ctx) { set_error("null context"); return BTED_EINVAL; }
+    if (ctx->poisoned) { set_error("context poisoned by an earlier CUDA error"); return BTED_ESTATE; }
+    try {
+        DeviceGuard dg(ctx->device);
+        return f();
+    } catch (const CudaError& e) {
+        ctx->poisoned = true;
+        set_error("CUDA error %s (%s) in %s", cudaGetErrorName(e.e), cudaGetErrorString(e.e), e.what);
+        cudaGetLastError();
+        return e.e == cudaErrorMemoryAllocation ? BTED_ENOMEM : BTED_ECUDA;
+    } catch (const std::bad_alloc&) {
+        set_error("host allocation failed");
+        return BTED_ENOMEM;
+    }
+}
+
+// Decode m packed keys on the host; checks the sticky error flag.
+bted_status finish_keys(bted_ctx* ctx, Ted& T, const unsigned long long* keys_dev, int32_t m,
+                        int64_t* out_idx, float* out_score, const int64_t* map_dev = nullptr) {
+    host_grow(ctx->hkeys, ctx->hkeyscap, (size_t)m + 1);
+    CK(cudaMemcpyAsync(ctx->hkeys, keys_dev, sizeof(unsigned long long) * m, cudaMemcpyDeviceToHost, T.stream));
+    CK(cudaMemcpyAsync(ctx->herr, T.err, sizeof(int), cudaMemcpyDeviceToHost, T.stream));
+    if (map_dev) CK(cudaMemcpyAsync(out_idx, map_dev, sizeof(int64_t) * m, cudaMemcpyDeviceToHost, T.stream));
+    CK(cudaStreamSynchronize(T.stream));
+    T.collect();
+    if (*ctx->herr) {
+        CK(cudaMemsetAsync(T.err, 0, sizeof(int), T.stream));
+        set_error("non-finite score or non-positive k(v,v)+mu during TED");
+        return BTED_ENUMERIC;
+    }
+    for (int32_t t = 0; t < m; ++t) {
+        const unsigned long long k = ctx->hkeys[t];
+        if (k == 0ull) { set_error("no candidate at step %d (internal)", t); return BTED_ENUMERIC; }
+        if (!map_dev) out_idx[t] = (int64_t)(0xFFFFFFFFu - (uint32_t)(k & 0xFFFFFFFFull));
+        if (out_score) {
+            uint32_t b = (uint32_t)(k >> 32) - 1u;
+            std::memcpy(&out_score[t], &b, 4);
+        }
+    }
+    return BTED_OK;
+}
+
+bted_status validate_params(const bted_params* p, bted_kernel kernel) {
+    if (!p) { set_error("null params"); return BTED_EINVAL; }
+    if (kernel != BTED_KERNEL_RBF && kernel != BTED_KERNEL_LINEAR) { set_error("bad kernel"); return BTED_EINVAL; }
+    if (kernel == BTED_KERNEL_RBF && !(p->gamma > 0.f && std::isfinite(p->gamma))) {
+        set_error("gamma must be > 0 and finite"); return BTED_EINVAL;
+    }
+    if (p->num_batches < 1) { set_error("num_batches must be >= 1"); return BTED_EINVAL; }
+    return BTED_OK;
+}
+
+bted_status create_common(const float* X, int64_t N, int32_t d, bted_kernel kernel, const bted_params* params,
+                          int64_t row0, int64_t row1, bool shard, bted_ctx** out) {
+    if (!out) { set_error("null out"); return BTED_EINVAL; }
+    *out = nullptr;
+    if (bted_status s = validate_params(params, kernel)) return s;
+    if (!X || N < 1 || N >= (int64_t)INT32_MAX || d < 1 || d > 64) {
+        set_error("need X != NULL, 1 <= N < 2^31, 1 <= d <= 64"); return BTED_EINVAL;
+    }
+    if (shard && !(0 <= row0 && row0 < row1 && row1 <= N)) { set_error("need 0 <= row0 < row1 <= N"); return BTED_EINVAL; }
+    if (!params->x_on_device && !all_finite(X, N * d)) { set_error("X has non-finite entries"); return BTED_EINVAL; }
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess || ndev < 1) {
+        cudaGetLastError();
+        set_error("no CUDA device available (%s): libbted has no CPU fallback", cudaGetErrorString(e));
+        return BTED_ECUDA;
+    }
+    bted_ctx* ctx = new (std::nothrow) bted_ctx();
+    if (!ctx) { set_error("host allocation failed"); return BTED_ENOMEM; }
+    ctx->params = *params;
+    ctx->kernel = kernel;
+    ctx->N = N;
+    ctx->d = d;
+    ctx->is_shard = shard;
+    ctx->row0 = shard ? row0 : 0;
+    ctx->row1 = shard ? row1 : N;
+    int dev = params->device;
+    if (dev < 0) cudaGetDevice(&dev);
+    ctx->device = dev;
+    bted_status st = guarded(ctx, [&]() -> bted_status {
+        cudaDeviceProp prop;
+        CK(cudaGetDeviceProperties(&prop, ctx->device));
+        if (prop.major < 10) {
+            set_error("device %d is sm_%d%d; libbted is built for sm_100a only", ctx->device, prop.major, prop.minor);
+            return BTED_ECUDA;
+        }
+        if (params->stream) {
+            ctx->stream = reinterpret_cast<cudaStream_t>(params->stream);
+        } else {
+            CK(cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking));
+            ctx->own_stream = true;
+        }
+        ctx->ted.stream = ctx->stream;
+        ctx->bted_engine.stream = ctx->stream;
+        ctx->ted.timing = ctx->bted_engine.timing = (params->flags & BTED_FLAG_TIMING) != 0;
+        CK(cudaMallocHost(&ctx->herr, sizeof(int)));
+        if (params->x_on_device) {
+            ctx->X = const_cast<float*>(X);
+        } else {
+            CK(cudaMalloc(&ctx->X, sizeof(float) * N * d));
+            ctx->own_X = true;
+            CK(cudaMemcpyAsync(ctx->X, X, sizeof(float) * N * d, cudaMemcpyHostToDevice, ctx->stream));
+            CK(cudaStreamSynchronize(ctx->stream));
+        }
+        return BTED_OK;
+    });
+    if (st != BTED_OK) {
+        bted_destroy(ctx);
+        return st;
+    }
+    *out = ctx;
+    return BTED_OK;
+}
+
+bool mu_ok(float mu) { return mu > 0.f && std::isfinite(mu); }
+
+// cub temp storage: grow to what the largest call needs.
+void cub_reserve(bted_ctx* ctx, size_t bytes) {
+    if (bytes <= ctx->cub_cap) return;
+    if (ctx->cub_tmp) cudaFree(ctx->cub_tmp);
+    ctx->cub_tmp = nullptr;
+    ctx->cub_cap = 0;
+    CK(cudaMalloc(&ctx->cub_tmp, bytes));
+    ctx->cub_cap = bytes;
+}
+
+int bits_for(uint64_t maxval) {
+    int b = 1;
+    while (b < 64 && (maxval >> b) != 0) ++b;
+    return b;
+}
+
+// Alg. 2 l.2 on the device: sidx[0..M) = sorted V_b.  P = pool rows.
+void sample_batch(bted_ctx* ctx, cudaStream_t st, int64_t P, int64_t M, int32_t b, uint64_t seed) {
+    grow(ctx->skeys, ctx->skeyscap, (size_t)P);
+    grow(ctx->skeys2, ctx->skeys2cap, (size_t)P);
+    grow(ctx->sidx, ctx->sidxcap, (size_t)M);
+    grow(ctx->sidx2, ctx->sidx2cap, (size_t)M);
+    const uint64_t hb = bted::splitmix64(seed + (uint64_t)b * bted::kBatchStride);
+    const unsigned g = (unsigned)std::min<int64_t>((P + 255) / 256, 148 * 16);
+    bted::batch_keys_kernel<<<g, 256, 0, st>>>((uint64_t)P, hb, ctx->skeys);
+    LAUNCHED(1);
+    size_t need = 0, need2 = 0;
+    CK(cub::DeviceRadixSort::SortKeys(nullptr, need, ctx->skeys, ctx->skeys2, (int)P, 0, 64, st));
+    CK(cub::DeviceRadixSort::SortKeys(nullptr, need2, ctx->sidx2, ctx->sidx, (int)M, 0, bits_for(P), st));
+    cub_reserve(ctx, std::max(need, need2));
+    size_t cap = ctx->cub_cap;
+    CK(cub::DeviceRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->skeys, ctx->skeys2, (int)P, 0, 64, st));
+    const unsigned gm = (unsigned)std::min<int64_t>((M + 255) / 256, 148 * 16);
+    bted::low_half_kernel<<<gm, 256, 0, st>>>(ctx->skeys2, M, ctx->sidx2);
+    LAUNCHED(1);
+    cap = ctx->cub_cap;
+    CK(cub::DeviceRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->sidx2, ctx->sidx, (int)M, 0, bits_for(P), st));
+}
+
+void gather(bted_ctx* ctx, cudaStream_t st, const uint32_t* idx, int64_t M) {
+    grow(ctx->Xb, ctx->xbcap, (size_t)(M * ctx->d));
+    const int64_t total = M * ctx->d;
+    const unsigned g = (unsigned)std::min<int64_t>((total + 255) / 256, 148 * 32);
+    bted::gather_rows_kernel<<<g, 256, 0, st>>>(ctx->X, ctx->d, idx, M, ctx->Xb);
+    LAUNCHED(1);
+}
+
+// Alg. 2 l.1-4 for batches b_begin, b_begin+b_step, ... ; winners on device.
+int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_begin, int32_t b_step) {
+    const int32_t B = ctx->params.num_batches;
+    int nb = 0;
+    for (int32_t b = b_begin; b < B; b += b_step) ++nb;
+    grow(ctx->winners, ctx->winnerscap, (size_t)std::max(nb, 1) * m);
+    grow(ctx->mkeys, ctx->mkeyscap, (size_t)m);
+    cudaStream_t st = ctx->stream;
+    const bool no_graph = (ctx->params.flags & BTED_FLAG_NO_GRAPH) != 0;
+    int k = 0;
+    for (int32_t b = b_begin; b < B; b += b_step, ++k) {
+        sample_batch(ctx, st, ctx->N, M, b, ctx->params.seed);
+        gather(ctx, st, ctx->sidx, M);
+        run_ted(ctx->bted_engine, ctx->Xb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->mkeys, no_graph);
+        bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->mkeys, m, ctx->sidx, ctx->winners + (size_t)k * m);
+        LAUNCHED(1);
+    }
+    return nb;
+}
+
+// Alg. 2 l.5-6 on device winners[0..n): returns count, out_idx host [count].
+bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, int32_t m, float mu,
+                         int64_t* out_idx, int32_t* out_count) {
+    cudaStream_t st = ctx->stream;
+    grow(ctx->u32a, ctx->u32acap, (size_t)n);
+    grow(ctx->u32b, ctx->u32bcap, (size_t)n);
+    grow(ctx->count_dev, ctx->countcap, 1);
+    const unsigned g = (unsigned)std::min<int64_t>((n + 255) / 256, 1024);
+    bted::i64_to_u32_kernel<<<g, 256, 0, st>>>(winners_dev, n, ctx->u32a);
+    LAUNCHED(1);
+    size_t need = 0, need2 = 0;
+    const int nbits = 32;   // padding (0xFFFFFFFF) must sort last
+    CK(cub::DeviceRadixSort::SortKeys(nullptr, need, ctx->u32a, ctx->u32b, (int)n, 0, nbits, st));
+    CK(cub::DeviceSelect::Unique(nullptr, need2, ctx->u32b, ctx->u32a, ctx->count_dev, (int)n, st));
+    cub_reserve(ctx, std::max(need, need2));
+    size_t cap = ctx->cub_cap;
+    CK(cub::DeviceRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->u32a, ctx->u32b, (int)n, 0, nbits, st));
+    cap = ctx->cub_cap;
+    CK(cub::DeviceSelect::Unique(ctx->cub_tmp, cap, ctx->u32b, ctx->u32a, ctx->count_dev, (int)n, st));
+    bted::drop_pad_kernel<<<1, 1, 0, st>>>(ctx->u32a, ctx->count_dev);
+    LAUNCHED(1);
+    int nu = 0;
+    CK(cudaMemcpyAsync(&nu, ctx->count_dev, sizeof(int), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));                        // |X_U| sizes the merge TED
+    ctx->bted_engine.collect();
+    if (nu < 1) { set_error("empty union"); return BTED_ENUMERIC; }
+    const int32_t mm = std::min<int32_t>(m, nu);          // reading A12
+    gather(ctx, st, ctx->u32a, nu);                       // X[X_U] (A13: fresh Gram)
+    grow(ctx->mkeys, ctx->mkeyscap, (size_t)mm);
+    grow(ctx->out_dev, ctx->outcap, (size_t)mm);
+    // the merge is tiny (|X_U| <= B m) and its size varies: run it eagerly
+    run_ted(ctx->bted_engine, ctx->Xb, nu, ctx->d, ctx->params.gamma, ctx->kernel, mm, mu, ctx->mkeys,
+            true, /*time_it=*/false);
+    bted::map_winners_kernel<<<(mm + 127) / 128, 128, 0, st>>>(ctx->mkeys, mm, ctx->u32a, ctx->out_dev);
+    LAUNCHED(1);
+    bted_status s = finish_keys(ctx, ctx->bted_engine, ctx->mkeys, mm, out_idx, nullptr, ctx->out_dev);
+    if (s == BTED_OK) *out_count = mm;
+    return s;
+}
+
+}  // namespace
+
+// ======================================================================= ABI
+extern "C" {
+
+void bted_default_params(bted_params* p) {
+    if (!p) return;
+    std::memset(p, 0, sizeof *p);
+    p->gamma = 1.0f;
+    p->device = -1;
+    p->num_batches = 1;
+}
+
+bted_status bted_create(const float* X, int64_t N, int32_t d, bted_kernel kernel, const bted_params* params,
+                        bted_ctx** out) {
+    return create_common(X, N, d, kernel, params, 0, N, false, out);
+}
+
+bted_status bted_shard_create(const float* X, int64_t N, int32_t d, bted_kernel kernel, int64_t row0,
+                              int64_t row1, const bted_params* params, bted_ctx** out) {
+    return create_common(X, N, d, kernel, params, row0, row1, true, out);
+}
+
+bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, float* out_score) {
+    if (!ctx || !out_idx) { set_error("null argument"); return BTED_EINVAL; }
+    if (ctx->is_shard) { set_error("bted_select on a shard context"); return BTED_EINVAL; }
+    if (m < 1 || m > ctx->N || !mu_ok(mu)) { set_error("need 1 <= m <= N and mu > 0 finite"); return BTED_EINVAL; }
+    return guarded(ctx, [&]() -> bted_status {
+        Ted& T = ctx->ted;
+        T.reserve(ctx->N, ctx->N, ctx->d, m);
+        run_ted(T, ctx->X, ctx->N, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, T.keys,
+                (ctx->params.flags & BTED_FLAG_NO_GRAPH) != 0);
+        return finish_keys(ctx, T, T.keys, m, out_idx, out_score);
+    });
+}
+
+bted_status bted_batch_teds(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_begin, int32_t b_step,
+                            int64_t* out_winners, int32_t winners_on_device) {
+    if (!ctx || !out_winners) { set_error("null argument"); return BTED_EINVAL; }
+    if (ctx->is_shard) { set_error("batch TEDs on a shard context"); return BTED_EINVAL; }
+    if (m < 1 || M < m || M > ctx->N || !mu_ok(mu) || b_begin < 0 || b_step < 1) {
+        set_error("need 1 <= m <= M <= N, mu > 0, b_begin >= 0, b_step >= 1"); return BTED_EINVAL;
+    }
+    return guarded(ctx, [&]() -> bted_status {
+        const int nb = run_batch_range(ctx, M, m, mu, b_begin, b_step);
+        const size_t bytes = sizeof(int64_t) * (size_t)nb * m;
+        if (nb > 0)
+            CK(cudaMemcpyAsync(out_winners, ctx->winners, bytes,
+                               winners_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, ctx->stream));
+        *ctx->herr = 0;
+        if (nb > 0)
+            CK(cudaMemcpyAsync(ctx->herr, ctx->bted_engine.err, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        ctx->bted_engine.collect();
+        if (nb > 0 && *ctx->herr) {
+            CK(cudaMemsetAsync(ctx->bted_engine.err, 0, sizeof(int), ctx->stream));
+            set_error("non-finite score during a batch TED");
+            return BTED_ENUMERIC;
+        }
+        return BTED_OK;
+    });
+}
+
+bted_status bted_merge(bted_ctx* ctx, const int64_t* winners, int64_t n, int32_t winners_on_device, int32_t m,
+                       float mu, int64_t* out_idx, int32_t* out_count) {
+    if (!ctx || !winners || !out_idx || !out_count) { set_error("null argument"); return BTED_EINVAL; }
+    if (ctx->is_shard) { set_error("merge on a shard context"); return BTED_EINVAL; }
+    if (n < 1 || n >= (int64_t)INT32_MAX || m < 1 || !mu_ok(mu)) { set_error("need n >= 1, m >= 1, mu > 0"); return BTED_EINVAL; }
+    if (!winners_on_device) {
+        for (int64_t i = 0; i < n; ++i)
+            if (winners[i] >= ctx->N) { set_error("winner index out of range"); return BTED_EINVAL; }
+    }
+    return guarded(ctx, [&]() -> bted_status {
+        grow(ctx->winners, ctx->winnerscap, (size_t)n);
+        if (winners != ctx->winners)
+            CK(cudaMemcpyAsync(ctx->winners, winners, sizeof(int64_t) * n,
+                               winners_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, ctx->stream));
+        return merge_device(ctx, ctx->winners, n, m, mu, out_idx, out_count);
+    });
+}
+
+bted_status bted_run_batches(bted_ctx* ctx, int64_t M, int32_t m, float mu, int64_t* out_idx, int32_t* out_count,
+                             int64_t* out_batch_idx) {
+    if (!ctx || !out_idx || !out_count) { set_error("null argument"); return BTED_EINVAL; }
+    if (ctx->is_shard) { set_error("run_batches on a shard context"); return BTED_EINVAL; }
+    if (m < 1 || M < m || M > ctx->N || !mu_ok(mu)) { set_error("need 1 <= m <= M <= N and mu > 0"); return BTED_EINVAL; }
+    return guarded(ctx, [&]() -> bted_status {
+        const int nb = run_batch_range(ctx, M, m, mu, 0, 1);
+        if (out_batch_idx)
+            CK(cudaMemcpyAsync(out_batch_idx, ctx->winners, sizeof(int64_t) * (size_t)nb * m,
+                               cudaMemcpyDeviceToHost, ctx->stream));
+        return merge_device(ctx, ctx->winners, (int64_t)nb * m, m, mu, out_idx, out_count);
+    });
+}
+
+bted_status bted_sample_batches(int64_t P, int64_t M, int32_t B, uint64_t seed, int64_t* out) {
+    if (!out || M < 1 || M > P || P >= (int64_t)INT32_MAX || B < 1) {
+        set_error("need 1 <= M <= P < 2^31, B >= 1, out != NULL"); return BTED_EINVAL;
+    }
+    // a scratch context with no features: only the sampling buffers are used
+    bted_params p;
+    bted_default_params(&p);
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev < 1) {
+        cudaGetLastError();
+        set_error("no CUDA device available: libbted has no CPU fallback");
+        return BTED_ECUDA;
+    }
+    bted_ctx* ctx = new (std::nothrow) bted_ctx();
+    if (!ctx) return BTED_ENOMEM;
+    cudaGetDevice(&ctx->device);
+    ctx->params = p;
+    bted_status st = guarded(ctx, [&]() -> bted_status {
+        CK(cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking));
+        ctx->own_stream = true;
+        int64_t* dout = nullptr;
+        CK(cudaMalloc(&dout, sizeof(int64_t) * (size_t)M));
+        for (int32_t b = 0; b < B; ++b) {
+            sample_batch(ctx, ctx->stream, P, M, b, seed);
+            const unsigned g = (unsigned)std::min<int64_t>((M + 255) / 256, 1024);
+            bted::u32_to_i64_kernel<<<g, 256, 0, ctx->stream>>>(ctx->sidx, M, dout);
+            LAUNCHED(1);
+            CK(cudaMemcpyAsync(out + (size_t)b * M, dout, sizeof(int64_t) * (size_t)M, cudaMemcpyDeviceToHost,
+                               ctx->stream));
+        }
+        CK(cudaStreamSynchronize(ctx->stream));
+        cudaFree(dout);
+        return BTED_OK;
+    });
+    bted_destroy(ctx);
+    return st;
+}
+
+// ------------------------------------------------------------------ shards
+bted_status bted_shard_gram(bted_ctx* ctx, float mu, uint64_t* keys_dev) {
+    if (!ctx || !keys_dev || !ctx->is_shard || !mu_ok(mu)) { set_error("bad shard_gram arguments"); return BTED_EINVAL; }
+    return guarded(ctx, [&]() -> bted_status {
+        Ted& T = ctx->ted;
+        const int64_t rows = ctx->row1 - ctx->row0;
+        T.reserve(rows, ctx->N, ctx->d, 2);
+        T.last_rows = rows;
+        T.last_ld = ld_for(ctx->N);
+        T.last_buf = 0;
+        launch_transpose(T, ctx->X, ctx->N, ctx->d);
+        CK(cudaMemsetAsync(T.sel, 0, (size_t)rows, T.stream));
+        launch_gram(T, ctx->N, ctx->d, ctx->row0, rows, ctx->params.gamma, ctx->kernel, mu,
+                    reinterpret_cast<unsigned long long*>(keys_dev));
+        return BTED_OK;
+    });
+}
+
+bted_status bted_shard_step(bted_ctx* ctx, int32_t t, float mu, const float* pivot_dev, uint64_t* keys_dev) {
+    if (!ctx || !keys_dev || !pivot_dev || !ctx->is_shard || t < 1 || !mu_ok(mu)) {
+        set_error("bad shard_step arguments"); return BTED_EINVAL;
+    }
+    return guarded(ctx, [&]() -> bted_status {
+        Ted& T = ctx->ted;
+        const int64_t rows = ctx->row1 - ctx->row0;
+        launch_step(T, ctx->N, ctx->row0, rows, t, mu, pivot_dev, reinterpret_cast<unsigned long long*>(keys_dev));
+        T.last_buf = t & 1;
+        return BTED_OK;
+    });
+}
+
+bted_status bted_shard_pivot_column(bted_ctx* ctx, int32_t t, const uint64_t* keys_dev, float* col_dev) {
+    if (!ctx || !keys_dev || !col_dev || !ctx->is_shard || t < 0) { set_error("bad pivot_column arguments"); return BTED_EINVAL; }
+    return guarded(ctx, [&]() -> bted_status {
+        Ted& T = ctx->ted;
+        const int32_t rows = (int32_t)(ctx->row1 - ctx->row0);
+        const unsigned g = (unsigned)std::min<int64_t>((rows + 255) / 256, 1024);
+        bted::pivot_column_kernel<<<g, 256, 0, T.stream>>>(T.K[t & 1], ld_for(ctx->N), rows,
+                                                           reinterpret_cast<const unsigned long long*>(keys_dev), t,
+                                                           col_dev);
+        LAUNCHED(1);
+        return BTED_OK;
+    });
+}
+
+int64_t bted_shard_ld(const bted_ctx* ctx) { return ctx ? ld_for(ctx->N) : 0; }
+
+bted_status bted_shard_check(bted_ctx* ctx) {
+    return guarded(ctx, [&]() -> bted_status {
+        if (!ctx->ted.err) return BTED_OK;
+        CK(cudaMemcpyAsync(ctx->herr, ctx->ted.err, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        if (*ctx->herr) { set_error("non-finite score in a shard step"); return BTED_ENUMERIC; }
+        return BTED_OK;
+    });
+}
+
+bted_status bted_update(bted_ctx* ctx, const float* X, int32_t x_on_device) {
+    if (!ctx || !X) { set_error("null argument"); return BTED_EINVAL; }
+    if (!x_on_device && !all_finite(X, ctx->N * ctx->d)) { set_error("X has non-finite entries"); return BTED_EINVAL; }
+    return guarded(ctx, [&]() -> bted_status {
+        if (!ctx->own_X) {
+            CK(cudaMalloc(&ctx->X, sizeof(float) * ctx->N * ctx->d));
+            ctx->own_X = true;
+        }
+        CK(cudaMemcpyAsync(ctx->X, X, sizeof(float) * ctx->N * ctx->d,
+                           x_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, ctx->stream));
+        // no sync: later work of this ctx is ordered after the copy on its stream;
+        // the caller must keep a host X alive until the next call returns
+        return BTED_OK;
+    });
+}
+
+bted_status bted_get_stats(bted_ctx* ctx, bted_stats* out) {
+    if (!ctx || !out) { set_error("null argument"); return BTED_EINVAL; }
+    const Stats& a = ctx->ted.stats;
+    const Stats& b = ctx->bted_engine.stats;
+    out->teds = a.teds + b.teds;
+    out->k2_launches = a.k2_launches + b.k2_launches;
+    out->k1_ms = a.k1_ms + b.k1_ms;
+    out->k2_ms = a.k2_ms + b.k2_ms;
+    return BTED_OK;
+}
+
+bted_status bted_reset_stats(bted_ctx* ctx) {
+    if (!ctx) { set_error("null argument"); return BTED_EINVAL; }
+    ctx->ted.stats = Stats{};
+    ctx->bted_engine.stats = Stats{};
+    return BTED_OK;
+}
+
+// ------------------------------------------------------------------ misc
+void bted_destroy(bted_ctx* ctx) {
+    if (!ctx) return;
+    {
+        DeviceGuard dg(ctx->device);
+        if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+        ctx->ted.release();
+        ctx->bted_engine.release();
+        void* bufs[] = {ctx->skeys, ctx->skeys2, ctx->sidx, ctx->sidx2, ctx->Xb, ctx->winners, ctx->u32a,
+                        ctx->u32b, ctx->count_dev, ctx->mkeys, ctx->cub_tmp, ctx->out_dev};
+        for (void* b : bufs) if (b) cudaFree(b);
+        if (ctx->own_X && ctx->X) cudaFree(ctx->X);
+        if (ctx->hkeys) cudaFreeHost(ctx->hkeys);
+        if (ctx->herr) cudaFreeHost(ctx->herr);
+        if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
+        cudaGetLastError();
+    }
+    delete ctx;
+}
+
+const char* bted_status_string(bted_status s) {
+    switch (s) {
+        case BTED_OK: return "BTED_OK";
+        case BTED_EINVAL: return "BTED_EINVAL";
+        case BTED_ENOMEM: return "BTED_ENOMEM";
+        case BTED_ECUDA: return "BTED_ECUDA";
+        case BTED_ENCCL: return "BTED_ENCCL";
+        case BTED_ENUMERIC: return "BTED_ENUMERIC";
+        case BTED_ESTATE: return "BTED_ESTATE";
+    }
+    return "BTED_UNKNOWN";
+}
+
+const char* bted_last_error(void) { return g_last_error.c_str(); }
+
+uint64_t bted_kernel_launches(void) { return g_launches.load(); }
+
+bted_status bted_debug_copy_K(bted_ctx* ctx, int32_t which, float* out, int64_t* ld_out) {
+    if (!ctx || !out) { set_error("null argument"); return BTED_EINVAL; }
+    return guarded(ctx, [&]() -> bted_status {
+        Ted& T = which == 1 ? ctx->bted_engine : ctx->ted;
+        if (!T.K[T.last_buf] || T.last_rows == 0) { set_error("no K yet"); return BTED_ESTATE; }
+        CK(cudaMemcpyAsync(out, T.K[T.last_buf], sizeof(float) * T.last_rows * T.last_ld, cudaMemcpyDeviceToHost,
+                           T.stream));
+        CK(cudaStreamSynchronize(T.stream));
+        if (ld_out) *ld_out = T.last_ld;
+        return BTED_OK;
+    });
+}
+
+}  // extern "C"

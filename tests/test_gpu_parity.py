@@ -1,0 +1,269 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle on the
+same seeded inputs.  Needs a B200 (sm_100a).  Protocol: tests/parity.py."""
+import numpy as np
+import pytest
+from scipy.spatial.distance import cdist
+
+import paper_conf_date_sunbg021_b200 as bt
+from paper_conf_date_sunbg021_b200 import _lib as L
+from oracle import dense, literal
+from oracle.sampling import sample_batches as oracle_sample_batches
+from synth import KnobSpace, WORKLOADS, make_pool, uniform_pool, median_gamma, config_pool
+from tests.parity import check_ted, ulp32
+
+pytestmark = pytest.mark.gpu
+MU = float(np.float32(0.1))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _gpu(need_gpu):
+    yield
+
+
+def knob(N, d=16, seed=3, wl="resnet18_layer1"):
+    _, X = make_pool(KnobSpace(WORKLOADS[wl], d), N, seed)
+    return X
+
+
+def ld_of(N):
+    return (N + 31) // 32 * 32
+
+
+# ------------------------------------------------------------------ K1 Gram
+@pytest.mark.parametrize("N,pool", [(1000, "knob"), (777, "uniform"), (64, "knob")])
+def test_gram_entries_bitsymmetric_and_within_ulp_bound(N, pool):
+    X = knob(N) if pool == "knob" else uniform_pool(N, 16, 4)
+    g = median_gamma(X, 1)
+    with bt.CandidateSet(X, g) as cs:
+        idx, sc = cs.select(1, MU)
+        K = cs.debug_K(N)
+    assert K.shape == (N, ld_of(N))
+    K32 = K[:, :N].astype(np.float64)
+    assert np.all(K[:, N:] == 0.0)                        # zero padding invariant
+    assert np.array_equal(K[:, :N], K[:, :N].T)           # bit-symmetric (C1, C6)
+    assert np.all(np.diag(K) == 1.0)                      # k(v,v) = 1 exactly
+    d2 = cdist(X.astype(np.float64), X.astype(np.float64), "sqeuclidean")
+    K64 = np.exp(-float(g) * d2)
+    bound = 6.0 * ulp32(K64) * (1.0 + float(g) * d2)
+    assert np.all(np.abs(K32 - K64) <= bound), np.max(np.abs(K32 - K64) / ulp32(K64))
+    # first pick = argmax of fp64 first scores (C1 + l.3)
+    s64 = (K64 * K64).sum(0) / (1.0 + MU)
+    assert abs(float(sc[0]) - s64[idx[0]]) <= 1e-5 * s64[idx[0]]
+
+
+# ------------------------------------------------------------------ K2 step
+def test_one_deflation_step_vs_fp64_and_selected_column():
+    N = 1200
+    X = knob(N, seed=9)
+    g = median_gamma(X, 2)
+    with bt.CandidateSet(X, g) as cs:
+        _ = cs.select(1, MU)
+        K0 = cs.debug_K(N)[:, :N].astype(np.float64)
+        idx, _ = cs.select(2, MU)
+        K1 = cs.debug_K(N)[:, :N].astype(np.float64)
+        _ = cs.select(9, MU)
+        K8 = cs.debug_K(N)
+    s = int(idx[0])
+    c = K0[s, s] + MU
+    prod = np.outer(K0[:, s], K0[s, :]) / c
+    ref = K0 - prod                                        # one fp64 step from the GPU's own K0
+    tol = 3.0 * ulp32(np.maximum(np.abs(K0), np.abs(prod))) + 1e-30
+    assert np.all(np.abs(K1 - ref) <= tol)
+    # C5: the selected column scales by mu / (k(s,s) + mu)
+    np.testing.assert_allclose(K1[:, s], K0[:, s] * MU / c, rtol=2e-6, atol=1e-30)
+    assert np.array_equal(K1, K1.T)
+    assert np.array_equal(K8[:, :N], K8[:, :N].T)           # still bit-symmetric after 8 steps
+
+
+# ------------------------------------------------------------------ TED parity
+def _ted_parity(X, g, m, label, use_dense=True):
+    with bt.CandidateSet(X, g) as cs:
+        idx, sc = cs.select(m, MU)
+        idx2, sc2 = cs.select(m, MU)
+    assert np.array_equal(idx, idx2) and np.array_equal(sc.view(np.uint32), sc2.view(np.uint32))  # deterministic
+    tr = dense.ted(X, g, MU, m, forced=idx) if use_dense else literal.ted(X, g, MU, m, forced=idx)
+    near = check_ted(idx, sc, tr, label)
+    free = dense.ted(X, g, MU, m) if use_dense else literal.ted(X, g, MU, m)
+    if min(free.gap) > 1e-6:
+        assert idx.tolist() == free.idx, f"{label}: free-running selection differs"
+    return near
+
+
+def test_ted_parity_toy_config():
+    X, g, cfg = config_pool("toy")
+    _ted_parity(X, g, cfg["m"], "toy", use_dense=False)
+
+
+@pytest.mark.parametrize("N,pool,m", [(257, "knob", 64), (1000, "uniform", 64), (2049, "knob12", 48),
+                                      (4096, "knob", 64), (4096, "uniform", 64)])
+def test_ted_parity_multi_tile_ragged(N, pool, m):
+    if pool == "knob":
+        X = knob(N, seed=N)
+    elif pool == "knob12":
+        X = knob(N, d=12, seed=N)
+    else:
+        X = uniform_pool(N, 16, N)
+    g = median_gamma(X, N)
+    _ted_parity(X, g, m, f"{pool}-{N}")
+
+
+def test_ted_parity_bench_size_resnet18_batch():
+    """The bench workload (resnet18 config: one batch of N = 16384 from the
+    2^20-row pool, m = 64), checked at every step against the dense C oracle."""
+    X, g, cfg = config_pool("resnet18")
+    V = oracle_sample_batches(X.shape[0], cfg["M"], 1, cfg["seed"])[0]
+    Xb = X[V]
+    with bt.CandidateSet(X, g, num_batches=1, seed=cfg["seed"]) as pool:
+        sel, bidx = pool.run_batches(cfg["M"], cfg["m"], MU)
+    with bt.CandidateSet(Xb, g) as cs:
+        idx, sc = cs.select(cfg["m"], MU)
+    # the batch TED inside run_batches is the same TED as select on X[V_b]
+    assert np.array_equal(V[idx], bidx[0])
+    tr = dense.ted(Xb, g, MU, cfg["m"], forced=idx)
+    check_ted(idx, sc, tr, "resnet18-16384")
+    assert set(sel.tolist()) == set(bidx[0].tolist())      # C10: B = 1 merge keeps the set
+
+
+# ------------------------------------------------------------------ edge cases
+def test_single_point_and_full_permutation():
+    X = knob(1)
+    with bt.CandidateSet(X, 1.0) as cs:
+        idx, sc = cs.select(1, MU)
+    assert idx.tolist() == [0] and sc[0] == np.float32(np.float32(1.0) / np.float32(1.0 + MU)) or \
+        abs(sc[0] - 1 / (1 + MU)) < 1e-6
+    X = knob(100, d=12, seed=5)                              # has exact duplicates
+    g = median_gamma(X, 5)
+    with bt.CandidateSet(X, g) as cs:
+        idx, sc = cs.select(100, MU)
+    assert sorted(idx.tolist()) == list(range(100))          # C7: m = N is a permutation
+
+
+def test_identity_kernel_ties_lowest_index():
+    X = (np.arange(40, dtype=np.float32) * 100.0)[:, None]  # K = I exactly in fp32
+    with bt.CandidateSet(X, 1.0) as cs:
+        idx, sc = cs.select(10, MU)
+    assert idx.tolist() == list(range(10))                   # C9 + reading A5
+    assert np.all(sc == np.float32(1.0) / np.float32(np.float32(1.0) + np.float32(MU)))
+
+
+def test_exact_duplicates_tie_to_lowest_index():
+    X = knob(300, seed=2)
+    X = np.concatenate([X, X[:50]], axis=0)                  # rows 300..349 duplicate rows 0..49
+    g = median_gamma(X, 3)
+    with bt.CandidateSet(X, g) as cs:
+        idx, sc = cs.select(40, MU)
+    for s in idx:
+        assert s < 300 or (s - 300) in idx[: list(idx).index(s)], "duplicate chosen before its twin"
+    tr = dense.ted(X, g, MU, 40, forced=idx)
+    check_ted(idx, sc, tr, "dups")
+
+
+def test_linear_kernel_closed_form_c8():
+    rng = np.random.default_rng(8)
+    X = (rng.standard_normal((300, 6)) * 0.5).astype(np.float32)
+    with bt.CandidateSet(X, 1.0, kernel=L.BTED_KERNEL_LINEAR) as cs:
+        idx, sc = cs.select(6, MU)
+        K5 = cs.debug_K(300)[:, :300].astype(np.float64)
+    Xd = X.astype(np.float64)
+    XS = Xd[idx[:5]]
+    ref = MU * Xd @ np.linalg.inv(MU * np.eye(6) + XS.T @ XS) @ Xd.T
+    assert np.max(np.abs(K5 - ref)) < 2e-5 * np.abs(Xd @ Xd.T).max()
+    tr = literal.ted_on_matrix(literal.linear_kernel(X), MU, 6, forced=idx)
+    check_ted(idx, sc, tr, "linear")
+
+
+def test_invalid_arguments_fail_loudly():
+    X = knob(50)
+    with bt.CandidateSet(X, 0.5) as cs:
+        for m, mu in [(0, MU), (51, MU), (5, 0.0), (5, float("nan"))]:
+            with pytest.raises(bt.BtedError) as e:
+                cs.select(m, mu)
+            assert e.value.status == 1
+    bad = X.copy()
+    bad[3, 2] = np.nan
+    with pytest.raises(bt.BtedError):
+        bt.CandidateSet(bad, 0.5)
+    with pytest.raises(bt.BtedError):
+        bt.CandidateSet(X, -1.0)
+
+
+# ------------------------------------------------------------------ Alg. 2
+@pytest.mark.parametrize("P,M,B,seed", [(1 << 20, 16384, 2, 5), (777, 777, 2, 1), (1000, 1, 3, 9),
+                                        (50000, 2048, 4, 3)])
+def test_sampling_bit_exact_vs_oracle_sampler(P, M, B, seed):
+    gpu = bt.bted_sample_batches(P, M, B, seed)
+    ref = oracle_sample_batches(P, M, B, seed)
+    assert np.array_equal(gpu, ref)
+
+
+def _positions(V, pool_idx):
+    pos = np.searchsorted(V, pool_idx)
+    assert np.array_equal(V[pos], pool_idx)
+    return pos
+
+
+def test_bted_parity_vs_oracle():
+    P, M, B, m, seed = 60000, 2048, 4, 32, 3
+    space = KnobSpace(WORKLOADS["vgg16_conv1_1"], 16)
+    _, X = make_pool(space, P, 77)
+    g = median_gamma(X, 77)
+    with bt.CandidateSet(X, g, num_batches=B, seed=seed) as pool:
+        sel, bidx = pool.run_batches(M, m, MU)
+    batches = oracle_sample_batches(P, M, B, seed)
+    for b in range(B):
+        Vb = batches[b]
+        pos = _positions(Vb, bidx[b])
+        tr = dense.ted(X[Vb], g, MU, m, forced=pos)
+        check_ted(pos, [], tr, f"batch{b}")
+    XU = np.unique(bidx)                                     # Alg. 2 l.5
+    assert set(sel.tolist()) <= set(XU.tolist()) and len(sel) == min(m, len(XU))
+    mpos = _positions(XU, sel)
+    trm = literal.ted(X[XU], g, MU, len(sel), forced=mpos)   # l.6 on a fresh Gram of X_U
+    check_ted(mpos, [], trm, "merge")
+
+
+def test_round_robin_batches_then_merge_equals_run_batches():
+    P, M, B, m, seed = 30000, 1024, 5, 16, 11
+    X = knob(P, seed=4)
+    g = median_gamma(X, 4)
+    with bt.CandidateSet(X, g, num_batches=B, seed=seed) as pool:
+        sel, bidx = pool.run_batches(M, m, MU)
+        w0 = np.empty(3 * m, np.int64)
+        w1 = np.full(3 * m, -1, np.int64)                    # rank 1 has 2 batches: padded like an all-gather
+        pool.batch_teds(M, m, MU, 0, 2, w0)
+        pool.batch_teds(M, m, MU, 1, 2, w1)
+        assert np.array_equal(w0.reshape(3, m), bidx[0::2]) and np.array_equal(w1[: 2 * m].reshape(2, m), bidx[1::2])
+        sel2 = pool.merge(np.concatenate([w0, w1]), 6 * m, m, MU)
+    assert np.array_equal(sel, sel2)
+
+
+def test_merge_smaller_than_m():
+    X = knob(500, seed=6)
+    g = median_gamma(X, 6)
+    with bt.CandidateSet(X, g) as pool:
+        out = pool.merge(np.array([5, 9, 5, 100, -1, 9]), 6, 8, MU)
+    assert sorted(out.tolist()) == [5, 9, 100]               # A12: select all of X_U
+
+
+# ------------------------------------------------------------------ sharded
+@pytest.mark.parametrize("N,P", [(3000, 2), (3001, 3), (1024, 4)])
+def test_row_sharded_loopback_bit_identical(N, P):
+    import torch
+    from paper_conf_date_sunbg021_b200.dist import sharded_select_loopback
+    X = knob(N, seed=N + P)
+    g = median_gamma(X, P)
+    with bt.CandidateSet(X, g) as cs:
+        idx, sc = cs.select(24, MU)
+    dev = torch.device("cuda", 0)
+    st = torch.cuda.Stream(dev)
+    sidx, ssc = sharded_select_loopback(X, g, P, 24, MU, dev, st)
+    assert np.array_equal(sidx, idx)
+    assert np.array_equal(ssc.view(np.uint32), sc.view(np.uint32))
+
+
+def test_launch_counter_counts_kernels():
+    X = knob(300)
+    before = bt.bted_kernel_launches()
+    with bt.CandidateSet(X, 0.3) as cs:
+        cs.select(10, MU)
+    assert bt.bted_kernel_launches() - before == 11          # transpose + K1 + 9 x K2
