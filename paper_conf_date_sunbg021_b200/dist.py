@@ -17,11 +17,14 @@ Two ways Algorithm 2 spreads over GPUs (DESIGN.md
    (every row's reduction order depends on N only), so the selection is
    bit-identical to `bted_select` for any number of shards.
 
-Every step of the method runs in libbted.so's kernels; this module only
-moves buffers between them (the `comm` object) and owns no arithmetic.
+Every step of the method runs in libbted.so's kernels (the `LibShard` /
+`LibPool` backends below); this module only moves buffers between them
+through the `comm` object and owns no arithmetic.  The backends are
+injectable so the exchange protocol itself is covered by CPU (gloo) tests.
 """
 from __future__ import annotations
 
+import contextlib
 import math
 
 import numpy as np
@@ -54,36 +57,81 @@ def band(N: int, P: int, r: int):
     return min(N, r * B), min(N, (r + 1) * B), B
 
 
+def _stream_ctx(stream):
+    return torch.cuda.stream(stream) if stream is not None else contextlib.nullcontext()
+
+
 # ------------------------------------------------------- 1. batch round-robin
-def run_batches_dp(pool_ctx: int, M: int, m: int, mu: float, B: int, comm, device: torch.device):
-    """Alg. 2 over `comm.world` ranks.  Returns (X pool indices, per-rank winners)."""
+class LibPool:
+    """Backend of run_batches_dp: a pool ctx of libbted.so."""
+
+    def __init__(self, ctx: int):
+        self.ctx = ctx
+
+    def batch_teds(self, M, m, mu, b_begin, b_step, out: torch.Tensor):
+        L.bted_batch_teds(self.ctx, M, m, mu, b_begin, b_step, out.data_ptr(), winners_on_device=out.is_cuda)
+
+    def merge(self, winners: torch.Tensor, m, mu):
+        if winners.is_cuda:
+            torch.cuda.current_stream(winners.device).synchronize()
+            return L.bted_merge(self.ctx, winners.data_ptr(), winners.numel(), m, mu, winners_on_device=True)
+        return L.bted_merge(self.ctx, winners.numpy(), winners.numel(), m, mu)
+
+
+def run_batches_dp(pool, M: int, m: int, mu: float, B: int, comm, device: torch.device):
+    """Alg. 2 over `comm.world` ranks.  pool: LibPool or a pool ctx handle.
+    Returns (X pool indices, this rank's winners with -1 padding)."""
+    if isinstance(pool, int):
+        pool = LibPool(pool)
     G, r = comm.world, comm.rank
     nb_max = math.ceil(B / G)
     nb_local = len(range(r, B, G))
     win = torch.full((nb_max * m,), -1, dtype=torch.int64, device=device)
     if nb_local:
-        L.bted_batch_teds(pool_ctx, M, m, mu, r, G, win.data_ptr(), winners_on_device=True)
+        pool.batch_teds(M, m, mu, r, G, win)         # l.1-4 for b = r, r+G, ...
     allw = torch.empty((G * nb_max * m,), dtype=torch.int64, device=device)
-    comm.allgather_(allw, win)                       # Alg. 2 l.5 exchange (padding = -1)
-    torch.cuda.current_stream(device).synchronize()
-    sel = L.bted_merge(pool_ctx, allw.data_ptr(), allw.numel(), m, mu, winners_on_device=True)
-    return sel, win
+    comm.allgather_(allw, win)                       # l.5 exchange (padding = -1)
+    return pool.merge(allw, m, mu), win              # l.5 union + l.6 merge TED
 
 
 # ------------------------------------------------------- 2. row-sharded TED
-class ShardedTed:
-    """TED on N rows with this rank's band of K (rows [row0, row1))."""
+class LibShard:
+    """Backend of ShardedTed: a shard ctx of libbted.so (rows [row0, row1))."""
 
-    def __init__(self, X, N: int, d: int, gamma: float, comm, device: torch.device, stream: torch.cuda.Stream,
-                 kernel: int = L.BTED_KERNEL_RBF):
-        self.N, self.d, self.comm, self.device, self.stream = int(N), int(d), comm, device, stream
-        self.row0, self.row1, self.bandB = band(self.N, comm.world, comm.rank)
+    def __init__(self, X, N, d, gamma, row0, row1, device: torch.device, stream, kernel=L.BTED_KERNEL_RBF):
+        on_dev = isinstance(X, int)
         p = L.default_params(gamma=gamma, device=device.index, stream=stream.cuda_stream,
-                             x_on_device=1 if isinstance(X, int) else 0)
-        self.ctx = L.bted_shard_create(X, N, d, kernel, self.row0, self.row1, p)
+                             x_on_device=1 if on_dev else 0)
+        self.ctx = L.bted_shard_create(X, N, d, kernel, row0, row1, p)
         self.ld = L.bted_shard_ld(self.ctx)
-        width = max(self.ld, comm.world * self.bandB)
-        with torch.cuda.stream(stream):
+
+    def gram(self, mu, keys: torch.Tensor):
+        L.bted_shard_gram(self.ctx, mu, keys.data_ptr())
+
+    def pivot_column(self, t, keys: torch.Tensor, col: torch.Tensor):
+        L.bted_shard_pivot_column(self.ctx, t, keys.data_ptr(), col.data_ptr())
+
+    def step(self, t, mu, pivot: torch.Tensor, keys: torch.Tensor):
+        L.bted_shard_step(self.ctx, t, mu, pivot.data_ptr(), keys.data_ptr())
+
+    def check(self):
+        L.bted_shard_check(self.ctx)
+
+    def close(self):
+        if self.ctx:
+            L.bted_destroy(self.ctx)
+            self.ctx = None
+
+
+class ShardedTed:
+    """TED (Alg. 1) on N rows with this rank's band of K.  `backend` runs the
+    band's kernels (LibShard on a GPU); `comm` does the two per-step exchanges."""
+
+    def __init__(self, backend, N: int, comm, device: torch.device, stream=None):
+        self.be, self.N, self.comm, self.device, self.stream = backend, int(N), comm, device, stream
+        self.row0, self.row1, self.bandB = band(self.N, comm.world, comm.rank)
+        width = max(getattr(backend, "ld", self.N), comm.world * self.bandB)
+        with _stream_ctx(stream):
             self.pivot = torch.zeros(width, dtype=torch.float32, device=device)
             self.col = torch.zeros(self.bandB, dtype=torch.float32, device=device)
 
@@ -91,66 +139,52 @@ class ShardedTed:
         if not (1 <= m <= self.N):
             raise ValueError("need 1 <= m <= N")
         P = self.comm.world
-        with torch.cuda.stream(self.stream):
+        with _stream_ctx(self.stream):
             keys = torch.zeros(m, dtype=torch.int64, device=self.device)
-            kp = keys.data_ptr()
-            L.bted_shard_gram(self.ctx, mu, kp)                   # l.1 + first l.3 on the band
-            self.comm.allreduce_max_(keys[0:1])                   # global argmax s_1
+            self.be.gram(mu, keys)                                # l.1 + first l.3 on the band
+            self.comm.allreduce_max_(keys[0:1])                   # global argmax s_1 (8 B)
             gathered = self.pivot[: P * self.bandB]
             for t in range(1, m):
-                L.bted_shard_pivot_column(self.ctx, t - 1, kp, self.col.data_ptr())
-                self.comm.allgather_(gathered, self.col)          # column s_t == row s_t
-                L.bted_shard_step(self.ctx, t, mu, self.pivot.data_ptr(), kp)   # l.5 + next l.3
-                self.comm.allreduce_max_(keys[t:t + 1])
+                self.be.pivot_column(t - 1, keys, self.col)       # K[band, s_t]
+                self.comm.allgather_(gathered, self.col)          # column s_t == row s_t (4N B)
+                self.be.step(t, mu, self.pivot, keys)             # l.5 + next l.3 on the band
+                self.comm.allreduce_max_(keys[t:t + 1])           # s_{t+1}
             host = keys.cpu().numpy().view(np.uint64)
-        L.bted_shard_check(self.ctx)
+        self.be.check()
         return L.decode_keys(host)
-
-    def close(self):
-        if getattr(self, "ctx", None):
-            L.bted_destroy(self.ctx)
-            self.ctx = None
-
-    def __del__(self):
-        try:
-            self.close()
-        except Exception:
-            pass
 
 
 # ------------------------------------------------ loopback (P shards, 1 GPU)
 def sharded_select_loopback(X: np.ndarray, gamma: float, P: int, m: int, mu: float, device: torch.device,
                             stream: torch.cuda.Stream, kernel: int = L.BTED_KERNEL_RBF):
     """The ShardedTed exchange with P logical shards on ONE GPU; the two
-    collectives are emulated by device copies / a max.  Exercises the sharded
-    control flow and its bit-identity without a second GPU."""
+    collectives are emulated by a device copy and a max.  Exercises the
+    sharded kernels and their bit-identity without a second GPU."""
     N, d = X.shape
-    ctxs, bands = [], []
-    p = L.default_params(gamma=gamma, device=device.index, stream=stream.cuda_stream)
+    shards = []
     try:
         for r in range(P):
             r0, r1, Bw = band(N, P, r)
-            ctxs.append(L.bted_shard_create(X, N, d, kernel, r0, r1, p))
-            bands.append((r0, r1))
-        ld = L.bted_shard_ld(ctxs[0])
+            shards.append(LibShard(X, N, d, gamma, r0, r1, device, stream, kernel))
+        ld = shards[0].ld
         with torch.cuda.stream(stream):
             keys = torch.zeros((P, m), dtype=torch.int64, device=device)
             pivot = torch.zeros(max(ld, P * Bw), dtype=torch.float32, device=device)
             cols = torch.zeros((P, Bw), dtype=torch.float32, device=device)
             for r in range(P):
-                L.bted_shard_gram(ctxs[r], mu, keys[r].data_ptr())
+                shards[r].gram(mu, keys[r])
             keys[:, 0] = keys[:, 0].max()
             for t in range(1, m):
                 for r in range(P):
-                    L.bted_shard_pivot_column(ctxs[r], t - 1, keys[r].data_ptr(), cols[r].data_ptr())
+                    shards[r].pivot_column(t - 1, keys[r], cols[r])
                 pivot[: P * Bw].copy_(cols.reshape(-1))
                 for r in range(P):
-                    L.bted_shard_step(ctxs[r], t, mu, pivot.data_ptr(), keys[r].data_ptr())
+                    shards[r].step(t, mu, pivot, keys[r])
                 keys[:, t] = keys[:, t].max()
             host = keys[0].cpu().numpy().view(np.uint64)
-        for c in ctxs:
-            L.bted_shard_check(c)
+        for s in shards:
+            s.check()
         return L.decode_keys(host)
     finally:
-        for c in ctxs:
-            L.bted_destroy(c)
+        for s in shards:
+            s.close()
