@@ -52,7 +52,7 @@ struct CudaError {
 #define LAUNCHED(n) g_launches.fetch_add((n), std::memory_order_relaxed)
 
 constexpr int kK1Rows = 16, kK1Threads = 256;
-constexpr int kK2Rows = 2, kK2Unroll = 4, kK2Threads = 256;
+constexpr int kK2Rows = 1, kK2Unroll = 4, kK2Threads = 256;
 constexpr int kRowsPerK2Cta = (kK2Threads / 32) * kK2Rows;
 
 inline int64_t round_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }

@@ -203,13 +203,39 @@ gram_rownorm_kernel(const float* __restrict__ XT, int64_t ld, int32_t d, int32_t
 }
 
 // ---------------------------------------------------------------------------
+// 256-bit global accesses (sm_100: LDG.E.256 / STG.E.256).  A lane moves 8
+// consecutive fp32 per instruction; K streams with L1 no-allocate loads and
+// evict-first (.cs) stores, the pivot row with plain cached loads (L2-hot).
+struct f8 { float v[8]; };
+__device__ __forceinline__ f8 ld8_stream(const float* p) {
+    f8 r;
+    asm volatile("ld.global.nc.L1::no_allocate.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=f"(r.v[0]), "=f"(r.v[1]), "=f"(r.v[2]), "=f"(r.v[3]), "=f"(r.v[4]), "=f"(r.v[5]),
+                   "=f"(r.v[6]), "=f"(r.v[7]) : "l"(p));
+    return r;
+}
+__device__ __forceinline__ f8 ld8_keep(const float* p) {
+    f8 r;
+    asm volatile("ld.global.nc.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=f"(r.v[0]), "=f"(r.v[1]), "=f"(r.v[2]), "=f"(r.v[3]), "=f"(r.v[4]), "=f"(r.v[5]),
+                   "=f"(r.v[6]), "=f"(r.v[7]) : "l"(p));
+    return r;
+}
+__device__ __forceinline__ void st8_stream(float* p, const f8& r) {
+    asm volatile("st.global.cs.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};"
+                 :: "l"(p), "f"(r.v[0]), "f"(r.v[1]), "f"(r.v[2]), "f"(r.v[3]), "f"(r.v[4]), "f"(r.v[5]),
+                    "f"(r.v[6]), "f"(r.v[7]) : "memory");
+}
+
+// ---------------------------------------------------------------------------
 // K2: Alg. 1 l.5 at step t (pivot s_t = keys[t-1]) fused with l.3 of step
 // t+1: K_out = K_in - K_in[:,s] K_in[s,:] / (K_in[s,s] + mu), new row norms,
 // scores, and the packed argmax into keys[t].  One warp owns kRows rows at a
-// time; lanes stride the row's float4 column groups (kUnroll groups in
-// flight per row).  The pivot row p (= column s by symmetry) is read through
-// L2 once per kRows rows; K is streamed with evict-first loads/stores.
-// Ping-pong buffers (K_in != K_out) make the pivot row read-only.
+// time; lane l covers the 8-float column groups l, l+32, ... (kUnroll groups
+// in flight per row, 256-bit loads).  The pivot row p (= column s by
+// symmetry) is read through L2 once per kRows rows.  Ping-pong buffers
+// (K_in != K_out) make the pivot row read-only during the sweep.
+// Chosen by scripts/k2_variants.cu (profiles/r1/k2_variants.txt).
 template <int kRows, int kUnroll, int kThreads>
 __global__ void __launch_bounds__(kThreads)
 deflate_rescore_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, int64_t ld,
@@ -224,7 +250,7 @@ deflate_rescore_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, 
         sel[(int32_t)s - row0] = 1;
     const int w = threadIdx.x / kWarp, l = threadIdx.x % kWarp;
     const int lrow0 = (blockIdx.x * kWarps + w) * kRows;
-    const int64_t nvec = ld >> 2;
+    const int64_t nvec = ld >> 3;
 
     float a[kRows], acc[kRows];
     const float* kin[kRows];
@@ -241,45 +267,39 @@ deflate_rescore_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, 
     if (any) {
         int64_t v = l;
         for (; v + (kUnroll - 1) * kWarp < nvec; v += kUnroll * kWarp) {
-            float4 pv[kUnroll], kv[kUnroll][kRows];
+            f8 pv[kUnroll], kv[kUnroll][kRows];
 #pragma unroll
             for (int u = 0; u < kUnroll; ++u) {
-                pv[u] = ld_keep(p + ((v + u * kWarp) << 2));
+                pv[u] = ld8_keep(p + ((v + u * kWarp) << 3));
 #pragma unroll
-                for (int r = 0; r < kRows; ++r) kv[u][r] = ld_stream(kin[r] + ((v + u * kWarp) << 2));
+                for (int r = 0; r < kRows; ++r) kv[u][r] = ld8_stream(kin[r] + ((v + u * kWarp) << 3));
             }
 #pragma unroll
             for (int u = 0; u < kUnroll; ++u) {
 #pragma unroll
                 for (int r = 0; r < kRows; ++r) {
-                    float4 o;
-                    o.x = deflate1(kv[u][r].x, a[r], pv[u].x, inv_c);
-                    o.y = deflate1(kv[u][r].y, a[r], pv[u].y, inv_c);
-                    o.z = deflate1(kv[u][r].z, a[r], pv[u].z, inv_c);
-                    o.w = deflate1(kv[u][r].w, a[r], pv[u].w, inv_c);
-                    acc[r] = __fmaf_rn(o.x, o.x, acc[r]);
-                    acc[r] = __fmaf_rn(o.y, o.y, acc[r]);
-                    acc[r] = __fmaf_rn(o.z, o.z, acc[r]);
-                    acc[r] = __fmaf_rn(o.w, o.w, acc[r]);
-                    if (lrow0 + r < nrows) st_stream(kout[r] + ((v + u * kWarp) << 2), o);
+                    f8 o;
+#pragma unroll
+                    for (int c = 0; c < 8; ++c) {
+                        o.v[c] = deflate1(kv[u][r].v[c], a[r], pv[u].v[c], inv_c);
+                        acc[r] = __fmaf_rn(o.v[c], o.v[c], acc[r]);
+                    }
+                    if (lrow0 + r < nrows) st8_stream(kout[r] + ((v + u * kWarp) << 3), o);
                 }
             }
         }
         for (; v < nvec; v += kWarp) {                  // ragged tail of the row
-            const float4 pv = ld_keep(p + (v << 2));
+            const f8 pv = ld8_keep(p + (v << 3));
 #pragma unroll
             for (int r = 0; r < kRows; ++r) {
-                const float4 kv = ld_stream(kin[r] + (v << 2));
-                float4 o;
-                o.x = deflate1(kv.x, a[r], pv.x, inv_c);
-                o.y = deflate1(kv.y, a[r], pv.y, inv_c);
-                o.z = deflate1(kv.z, a[r], pv.z, inv_c);
-                o.w = deflate1(kv.w, a[r], pv.w, inv_c);
-                acc[r] = __fmaf_rn(o.x, o.x, acc[r]);
-                acc[r] = __fmaf_rn(o.y, o.y, acc[r]);
-                acc[r] = __fmaf_rn(o.z, o.z, acc[r]);
-                acc[r] = __fmaf_rn(o.w, o.w, acc[r]);
-                if (lrow0 + r < nrows) st_stream(kout[r] + (v << 2), o);
+                const f8 kv = ld8_stream(kin[r] + (v << 3));
+                f8 o;
+#pragma unroll
+                for (int c = 0; c < 8; ++c) {
+                    o.v[c] = deflate1(kv.v[c], a[r], pv.v[c], inv_c);
+                    acc[r] = __fmaf_rn(o.v[c], o.v[c], acc[r]);
+                }
+                if (lrow0 + r < nrows) st8_stream(kout[r] + (v << 3), o);
             }
         }
     }
