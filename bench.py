@@ -33,7 +33,8 @@ import numpy as np  # noqa: E402
 
 METRIC = "BTED selected points/sec and deflate-step HBM GB/s vs roofline at 1/2/4/8 B200"
 UNIT = "points/s"
-K2_NAME = "deflate_rescore_kernel"
+K2_NAME = {"dense": "deflate_rescore_kernel",
+           "packed": "deflate_packed_kernel (+ packed_pivot_kernel, per step)"}
 
 
 def parse():
@@ -46,6 +47,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
+    ap.add_argument("--layout", default="packed", choices=["packed", "dense"],
+                    help="K storage: packed upper-triangular tiles (4 N^2 B/step) or dense (8 N^2 B/step)")
     return ap.parse_args()
 
 
@@ -196,8 +199,9 @@ def bench_ours(args):
     stream = torch.cuda.Stream(dev)
     X_dev = torch.from_numpy(X).to(dev)
     torch.cuda.synchronize()
+    lay_flag = L.BTED_FLAG_DENSE if args.layout == "dense" else 0
     pool = bt.CandidateSet(X_dev, gamma, num_batches=B, seed=cfg["seed"], device=local,
-                           flags=L.BTED_FLAG_TIMING, stream=stream.cuda_stream)
+                           flags=L.BTED_FLAG_TIMING | lay_flag, stream=stream.cuda_stream)
 
     def step():
         if world == 1:
@@ -240,14 +244,16 @@ def bench_ours(args):
     # roofline of the dominant kernel K2 (fused deflate + rescore), live events
     peak, peak_src = peaks()
     k2_avg_ms = stats["k2_ms"] / max(stats["k2_launches"], 1)
-    alg_bytes = 8.0 * M * M                       # fp32 read + write of K per launch (8 N^2)
+    # algorithmic bytes per step: fp32 read + write of K = 8 N^2 (dense) or of
+    # its upper triangle = 4 N^2 (packed; report against 4 N^2)
+    alg_bytes = (8.0 if args.layout == "dense" else 4.0) * M * M
     achieved = alg_bytes / (k2_avg_ms / 1e3) / 1e9
     traffic = None
     tj = os.path.join(ROOT, "profiles", "k2_traffic.json")
     if os.path.exists(tj):
         with open(tj) as f:
             tjd = json.load(f)
-        if tjd.get("M") == M:
+        if tjd.get("M") == M and tjd.get("layout", "dense") == args.layout:
             traffic = tjd.get("dram_bytes_per_launch")
 
     # end to end through the public API with HOST buffers (pinned), per step:
@@ -256,7 +262,7 @@ def bench_ours(args):
     if not args.no_e2e:
         Xh = torch.from_numpy(X).pin_memory()
         ctx2 = bt.CandidateSet(Xh.numpy(), gamma, num_batches=B, seed=cfg["seed"], device=local,
-                               stream=stream.cuda_stream)
+                               flags=lay_flag, stream=stream.cuda_stream)
         for _ in range(max(1, args.warmup)):
             L.bted_update(ctx2.ctx, Xh.data_ptr())
             if world == 1:
@@ -300,7 +306,8 @@ def bench_ours(args):
                 "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
                 "config": workload_config(args.config, cfg, gamma, world),
-                "roofline": {"bound": "hbm", "kernel": K2_NAME, "achieved": achieved, "peak": peak,
+                "layout": args.layout,
+                "roofline": {"bound": "hbm", "kernel": K2_NAME[args.layout], "achieved": achieved, "peak": peak,
                              "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
                              "frac_of_8TBs": achieved / 8000.0, "peak_source": peak_src,
                              "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": k2_avg_ms,

@@ -57,6 +57,9 @@ typedef enum {
 
 /* flags */
 #define BTED_FLAG_NO_GRAPH 1u   /* launch the m-step loop eagerly (debug / profiling) */
+#define BTED_FLAG_DENSE    4u   /* store K densely (N x ld, 8 N^2 bytes per step) instead of the
+                                   default packed upper-triangular tiles (4 N^2 bytes per step;
+                                   used when d <= 32).  Shard contexts are always dense. */
 #define BTED_FLAG_TIMING   2u   /* record CUDA events around K1 and the K2 loop of every batch
                                    TED on the ctx stream; read with bted_get_stats()          */
 
@@ -208,8 +211,9 @@ const char* bted_status_string(bted_status s);
 const char* bted_last_error(void);
 /* Number of kernels this library launched since load (all contexts). */
 uint64_t    bted_kernel_launches(void);
-/* Debug: copy the current fp32 K (rows x ld) of ctx's last select to host.
- * Only valid with BTED_FLAG_NO_GRAPH runs or after bted_select returns. */
+/* Debug: copy the fp32 K of the last TED run by ctx (which = 0: bted_select,
+ * 1: the last batch / merge TED) to host as a dense rows x ld matrix (packed
+ * storage is unpacked), i.e. K after the m-1 deflations of that run. */
 bted_status bted_debug_copy_K(bted_ctx* ctx, int32_t which, float* out, int64_t* ld_out);
 
 #ifdef __cplusplus

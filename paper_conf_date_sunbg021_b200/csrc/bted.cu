@@ -24,6 +24,7 @@
 #include "../../include/bted.h"
 #include "kernels.cuh"
 #include "sample.cuh"
+#include "packed.cuh"
 
 namespace {
 
@@ -74,10 +75,12 @@ struct GraphKey {
     const float* X;
     int64_t N;
     int32_t d, m, kernel, part;   // part 0 = head (transpose, K1), 1 = loop (m-1 x K2)
+    int32_t packed;
     uint32_t mu, gamma;
     const void* keys;
     bool operator==(const GraphKey& o) const {
         return X == o.X && N == o.N && d == o.d && m == o.m && kernel == o.kernel && part == o.part &&
+               packed == o.packed &&
                mu == o.mu && gamma == o.gamma && keys == o.keys;
     }
 };
@@ -99,9 +102,18 @@ struct Ted {
     size_t keyscap = 0;
     int* err = nullptr;
     size_t errcap = 0;
+    // packed-symmetric layout (packed.cuh): partials, arrival counters, pivot row
+    float* P = nullptr;
+    size_t pcap = 0;
+    unsigned int* cnt = nullptr;
+    size_t cntcap = 0;
+    float* piv = nullptr;
+    size_t pivcap = 0;
     std::list<std::pair<GraphKey, cudaGraphExec_t>> graphs;   // LRU
     int64_t last_rows = 0, last_ld = 0;
     int last_buf = 0;
+    bool last_packed = false;
+    int32_t last_nT = 0;
     // timing (BTED_FLAG_TIMING): events recorded on the stream around the
     // head and loop graphs of each TED, read back at the next host sync.
     bool timing = false;
@@ -118,9 +130,34 @@ struct Ted {
         if (sel) cudaFree(sel);
         if (keys) cudaFree(keys);
         if (err) cudaFree(err);
+        if (P) cudaFree(P);
+        if (cnt) cudaFree(cnt);
+        if (piv) cudaFree(piv);
         for (auto& sl : slots) for (auto e : sl.e) cudaEventDestroy(e);
         slots.clear();
         K[0] = K[1] = nullptr; XT = nullptr; sel = nullptr; keys = nullptr; err = nullptr;
+        P = nullptr; cnt = nullptr; piv = nullptr;
+    }
+
+    // Buffers of the packed layout for an N-point TED.
+    void reserve_packed(int64_t N, int32_t m) {
+        const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
+        const size_t tiles = (size_t)bted::pk::num_tiles(nT) * bted::pk::T * bted::pk::T;
+        const size_t NP = (size_t)nT * bted::pk::T;
+        const void* before[8] = {K[0], K[1], sel, keys, P, cnt, piv, XT};
+        grow(K[0], kcap[0], tiles);
+        if (m > 1) grow(K[1], kcap[1], tiles);
+        grow(sel, selcap, NP);
+        grow(keys, keyscap, (size_t)std::max(m, 1));
+        grow(P, pcap, (size_t)nT * NP);
+        grow(cnt, cntcap, 2 * (size_t)nT);
+        grow(piv, pivcap, NP);
+        if (!err) { grow(err, errcap, 1); CK(cudaMemsetAsync(err, 0, sizeof(int), stream)); }
+        const void* after[8] = {K[0], K[1], sel, keys, P, cnt, piv, XT};
+        if (std::memcmp(before, after, sizeof before) != 0) {
+            for (auto& g : graphs) cudaGraphExecDestroy(g.second);
+            graphs.clear();
+        }
     }
 
     // Buffers for a band of `rows` rows of an N x N problem.
@@ -195,6 +232,53 @@ void launch_step(Ted& T, int64_t N, int64_t row0, int64_t rows, int32_t t, float
     LAUNCHED(1);
 }
 
+// ---- packed layout (packed.cuh) ----
+int g_num_sms = 0;
+int num_sms() {
+    if (!g_num_sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
+        if (g_num_sms <= 0) g_num_sms = 148;
+    }
+    return g_num_sms;
+}
+constexpr size_t kK2pSmem = (size_t)bted::pk::kStages * bted::pk::kTileBytes + 2 * bted::pk::kStages * sizeof(uint64_t);
+
+// Alg. 1 l.1 + first l.3 on the packed tiles.  (1 kernel)
+void enqueue_head_packed(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m,
+                         float mu, unsigned long long* keys) {
+    const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
+    CK(cudaMemsetAsync(keys, 0, sizeof(unsigned long long) * m, T.stream));
+    CK(cudaMemsetAsync(T.sel, 0, (size_t)nT * bted::pk::T, T.stream));
+    CK(cudaMemsetAsync(T.cnt, 0, sizeof(unsigned int) * 2 * nT, T.stream));
+    const int64_t tiles = bted::pk::num_tiles(nT);
+    const unsigned grid = (unsigned)std::min<int64_t>(tiles, (int64_t)num_sms() * 2);
+    const int lin = kernel == BTED_KERNEL_LINEAR ? 1 : 0;
+    if (d <= 16)
+        bted::pk::gram_packed_kernel<16><<<grid, bted::pk::kConsumers, 0, T.stream>>>(
+            X, (int32_t)N, d, gamma, lin, T.K[0], nT, T.P, T.cnt, mu, keys, T.err);
+    else
+        bted::pk::gram_packed_kernel<32><<<grid, bted::pk::kConsumers, 0, T.stream>>>(
+            X, (int32_t)N, d, gamma, lin, T.K[0], nT, T.P, T.cnt, mu, keys, T.err);
+    LAUNCHED(1);
+}
+
+// Alg. 1 l.2-6 loop on the packed tiles: per step, pivot-row extraction + K2p.  (2(m-1) kernels)
+void enqueue_loop_packed(Ted& T, int64_t N, int32_t m, float mu, unsigned long long* keys) {
+    const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
+    const int64_t tiles = bted::pk::num_tiles(nT);
+    const unsigned grid = (unsigned)std::min<int64_t>(tiles, (int64_t)num_sms());
+    const unsigned pgrid = (unsigned)std::min<int64_t>(((int64_t)nT * bted::pk::T + 255) / 256, 1024);
+    for (int32_t t = 1; t < m; ++t) {
+        const float* Kin = T.K[(t - 1) & 1];
+        bted::pk::packed_pivot_kernel<<<pgrid, 256, 0, T.stream>>>(Kin, nT, keys, t - 1, T.piv);
+        bted::pk::deflate_packed_kernel<<<grid, bted::pk::kConsumers + 32, kK2pSmem, T.stream>>>(
+            Kin, T.K[t & 1], nT, (int32_t)N, T.piv, T.P, T.cnt + (size_t)(t & 1) * nT, keys, t, mu, T.sel, T.err);
+        LAUNCHED(2);
+    }
+}
+
 // Alg. 1 l.1 + first l.3: XT, zero keys/sel, K1.  (2 kernels)
 void enqueue_head(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
                   unsigned long long* keys) {
@@ -244,27 +328,54 @@ void graph_run(Ted& T, const GraphKey& key, uint64_t nkernels, F&& enqueue) {
 }
 
 // Run one TED (graph-cached unless no_graph); results stay on the device.
+void ensure_packed_attrs() {
+    static bool done = false;
+    if (!done) {
+        CK(cudaFuncSetAttribute(bted::pk::deflate_packed_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)kK2pSmem));
+        done = true;
+    }
+}
+
+// packed layout unless the caller asks for dense or d is too wide for K1p
+bool use_packed(uint32_t flags, int32_t d) { return !(flags & BTED_FLAG_DENSE) && d <= 32; }
+
 void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
-             unsigned long long* keys, bool no_graph, bool time_it = true) {
-    T.reserve(N, N, d, m);
+             unsigned long long* keys, bool no_graph, bool time_it = true, bool packed = false) {
+    if (packed) {
+        ensure_packed_attrs();
+        T.reserve_packed(N, m);
+        T.last_nT = (int32_t)((N + bted::pk::T - 1) / bted::pk::T);
+    } else {
+        T.reserve(N, N, d, m);
+    }
+    T.last_packed = packed;
     T.last_rows = N;
     T.last_ld = ld_for(N);
     T.last_buf = (m - 1) & 1;
     Ted::Slot* sl = (T.timing && time_it) ? T.next_slot(m) : nullptr;
     if (sl) CK(cudaEventRecord(sl->e[0], T.stream));
+    auto head = [&] {
+        if (packed) enqueue_head_packed(T, X, N, d, gamma, kernel, m, mu, keys);
+        else enqueue_head(T, X, N, d, gamma, kernel, m, mu, keys);
+    };
+    auto loop = [&] {
+        if (packed) enqueue_loop_packed(T, N, m, mu, keys);
+        else enqueue_loop(T, N, m, mu, keys);
+    };
     if (no_graph) {
-        enqueue_head(T, X, N, d, gamma, kernel, m, mu, keys);
+        head();
     } else {
-        GraphKey key{X, N, d, m, kernel, 0, fbits(mu), fbits(gamma), keys};
-        graph_run(T, key, 2, [&] { enqueue_head(T, X, N, d, gamma, kernel, m, mu, keys); });
+        GraphKey key{X, N, d, m, kernel, 0, packed ? 1 : 0, fbits(mu), fbits(gamma), keys};
+        graph_run(T, key, packed ? 1 : 2, head);
     }
     if (sl) CK(cudaEventRecord(sl->e[1], T.stream));
     if (m > 1) {
         if (no_graph) {
-            enqueue_loop(T, N, m, mu, keys);
+            loop();
         } else {
-            GraphKey key{X, N, d, m, kernel, 1, fbits(mu), fbits(gamma), keys};
-            graph_run(T, key, (uint64_t)(m - 1), [&] { enqueue_loop(T, N, m, mu, keys); });
+            GraphKey key{X, N, d, m, kernel, 1, packed ? 1 : 0, fbits(mu), fbits(gamma), keys};
+            graph_run(T, key, (uint64_t)(m - 1) * (packed ? 2 : 1), loop);
         }
     }
     if (sl) CK(cudaEventRecord(sl->e[2], T.stream));
@@ -517,7 +628,8 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
     for (int32_t b = b_begin; b < B; b += b_step, ++k) {
         sample_batch(ctx, st, ctx->N, M, b, ctx->params.seed);
         gather(ctx, st, ctx->sidx, M);
-        run_ted(ctx->bted_engine, ctx->Xb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->mkeys, no_graph);
+        run_ted(ctx->bted_engine, ctx->Xb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->mkeys, no_graph,
+                true, use_packed(ctx->params.flags, ctx->d));
         bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->mkeys, m, ctx->sidx, ctx->winners + (size_t)k * m);
         LAUNCHED(1);
     }
@@ -556,7 +668,7 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
     grow(ctx->out_dev, ctx->outcap, (size_t)mm);
     // the merge is tiny (|X_U| <= B m) and its size varies: run it eagerly
     run_ted(ctx->bted_engine, ctx->Xb, nu, ctx->d, ctx->params.gamma, ctx->kernel, mm, mu, ctx->mkeys,
-            true, /*time_it=*/false);
+            true, /*time_it=*/false, use_packed(ctx->params.flags, ctx->d));
     bted::map_winners_kernel<<<(mm + 127) / 128, 128, 0, st>>>(ctx->mkeys, mm, ctx->u32a, ctx->out_dev);
     LAUNCHED(1);
     bted_status s = finish_keys(ctx, ctx->bted_engine, ctx->mkeys, mm, out_idx, nullptr, ctx->out_dev);
@@ -595,7 +707,7 @@ bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, fl
         Ted& T = ctx->ted;
         T.reserve(ctx->N, ctx->N, ctx->d, m);
         run_ted(T, ctx->X, ctx->N, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, T.keys,
-                (ctx->params.flags & BTED_FLAG_NO_GRAPH) != 0);
+                (ctx->params.flags & BTED_FLAG_NO_GRAPH) != 0, true, use_packed(ctx->params.flags, ctx->d));
         return finish_keys(ctx, T, T.keys, m, out_idx, out_score);
     });
 }
@@ -830,10 +942,26 @@ bted_status bted_debug_copy_K(bted_ctx* ctx, int32_t which, float* out, int64_t*
     return guarded(ctx, [&]() -> bted_status {
         Ted& T = which == 1 ? ctx->bted_engine : ctx->ted;
         if (!T.K[T.last_buf] || T.last_rows == 0) { set_error("no K yet"); return BTED_ESTATE; }
-        CK(cudaMemcpyAsync(out, T.K[T.last_buf], sizeof(float) * T.last_rows * T.last_ld, cudaMemcpyDeviceToHost,
-                           T.stream));
-        CK(cudaStreamSynchronize(T.stream));
-        if (ld_out) *ld_out = T.last_ld;
+        const int64_t rows = T.last_rows, ld = T.last_ld;
+        if (!T.last_packed) {
+            CK(cudaMemcpyAsync(out, T.K[T.last_buf], sizeof(float) * rows * ld, cudaMemcpyDeviceToHost, T.stream));
+            CK(cudaStreamSynchronize(T.stream));
+        } else {
+            // unpack the upper-triangular tiles into the dense rows x ld view
+            const int nT = T.last_nT, TT = bted::pk::T;
+            const size_t n = (size_t)bted::pk::num_tiles(nT) * TT * TT;
+            std::vector<float> h(n);
+            CK(cudaMemcpyAsync(h.data(), T.K[T.last_buf], sizeof(float) * n, cudaMemcpyDeviceToHost, T.stream));
+            CK(cudaStreamSynchronize(T.stream));
+            std::memset(out, 0, sizeof(float) * rows * ld);
+            for (int64_t i = 0; i < rows; ++i)
+                for (int64_t j = 0; j < rows; ++j) {
+                    const int I = (int)(i / TT), J = (int)(j / TT), r = (int)(i % TT), c = (int)(j % TT);
+                    out[i * ld + j] = I <= J ? h[(size_t)bted::pk::tile_offset(I, J, nT) * TT * TT + r * TT + c]
+                                             : h[(size_t)bted::pk::tile_offset(J, I, nT) * TT * TT + c * TT + r];
+                }
+        }
+        if (ld_out) *ld_out = ld;
         return BTED_OK;
     });
 }

@@ -31,10 +31,11 @@ def ld_of(N):
 
 # ------------------------------------------------------------------ K1 Gram
 @pytest.mark.parametrize("N,pool", [(1000, "knob"), (777, "uniform"), (64, "knob")])
-def test_gram_entries_bitsymmetric_and_within_ulp_bound(N, pool):
+@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+def test_gram_entries_bitsymmetric_and_within_ulp_bound(N, pool, flags):
     X = knob(N) if pool == "knob" else uniform_pool(N, 16, 4)
     g = median_gamma(X, 1)
-    with bt.CandidateSet(X, g) as cs:
+    with bt.CandidateSet(X, g, flags=flags) as cs:
         idx, sc = cs.select(1, MU)
         K = cs.debug_K(N)
     assert K.shape == (N, ld_of(N))
@@ -52,11 +53,12 @@ def test_gram_entries_bitsymmetric_and_within_ulp_bound(N, pool):
 
 
 # ------------------------------------------------------------------ K2 step
-def test_one_deflation_step_vs_fp64_and_selected_column():
+@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+def test_one_deflation_step_vs_fp64_and_selected_column(flags):
     N = 1200
     X = knob(N, seed=9)
     g = median_gamma(X, 2)
-    with bt.CandidateSet(X, g) as cs:
+    with bt.CandidateSet(X, g, flags=flags) as cs:
         _ = cs.select(1, MU)
         K0 = cs.debug_K(N)[:, :N].astype(np.float64)
         idx, _ = cs.select(2, MU)
@@ -76,8 +78,8 @@ def test_one_deflation_step_vs_fp64_and_selected_column():
 
 
 # ------------------------------------------------------------------ TED parity
-def _ted_parity(X, g, m, label, use_dense=True):
-    with bt.CandidateSet(X, g) as cs:
+def _ted_parity(X, g, m, label, use_dense=True, flags=0):
+    with bt.CandidateSet(X, g, flags=flags) as cs:
         idx, sc = cs.select(m, MU)
         idx2, sc2 = cs.select(m, MU)
     assert np.array_equal(idx, idx2) and np.array_equal(sc.view(np.uint32), sc2.view(np.uint32))  # deterministic
@@ -89,14 +91,16 @@ def _ted_parity(X, g, m, label, use_dense=True):
     return near
 
 
-def test_ted_parity_toy_config():
+@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+def test_ted_parity_toy_config(flags):
     X, g, cfg = config_pool("toy")
-    _ted_parity(X, g, cfg["m"], "toy", use_dense=False)
+    _ted_parity(X, g, cfg["m"], "toy", use_dense=False, flags=flags)
 
 
 @pytest.mark.parametrize("N,pool,m", [(257, "knob", 64), (1000, "uniform", 64), (2049, "knob12", 48),
                                       (4096, "knob", 64), (4096, "uniform", 64)])
-def test_ted_parity_multi_tile_ragged(N, pool, m):
+@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+def test_ted_parity_multi_tile_ragged(N, pool, m, flags):
     if pool == "knob":
         X = knob(N, seed=N)
     elif pool == "knob12":
@@ -104,18 +108,19 @@ def test_ted_parity_multi_tile_ragged(N, pool, m):
     else:
         X = uniform_pool(N, 16, N)
     g = median_gamma(X, N)
-    _ted_parity(X, g, m, f"{pool}-{N}")
+    _ted_parity(X, g, m, f"{pool}-{N}", flags=flags)
 
 
-def test_ted_parity_bench_size_resnet18_batch():
+@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+def test_ted_parity_bench_size_resnet18_batch(flags):
     """The bench workload (resnet18 config: one batch of N = 16384 from the
     2^20-row pool, m = 64), checked at every step against the dense C oracle."""
     X, g, cfg = config_pool("resnet18")
     V = oracle_sample_batches(X.shape[0], cfg["M"], 1, cfg["seed"])[0]
     Xb = X[V]
-    with bt.CandidateSet(X, g, num_batches=1, seed=cfg["seed"]) as pool:
+    with bt.CandidateSet(X, g, num_batches=1, seed=cfg["seed"], flags=flags) as pool:
         sel, bidx = pool.run_batches(cfg["M"], cfg["m"], MU)
-    with bt.CandidateSet(Xb, g) as cs:
+    with bt.CandidateSet(Xb, g, flags=flags) as cs:
         idx, sc = cs.select(cfg["m"], MU)
     # the batch TED inside run_batches is the same TED as select on X[V_b]
     assert np.array_equal(V[idx], bidx[0])
@@ -125,32 +130,35 @@ def test_ted_parity_bench_size_resnet18_batch():
 
 
 # ------------------------------------------------------------------ edge cases
-def test_single_point_and_full_permutation():
+@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+def test_single_point_and_full_permutation(flags):
     X = knob(1)
-    with bt.CandidateSet(X, 1.0) as cs:
+    with bt.CandidateSet(X, 1.0, flags=flags) as cs:
         idx, sc = cs.select(1, MU)
     assert idx.tolist() == [0] and sc[0] == np.float32(np.float32(1.0) / np.float32(1.0 + MU)) or \
         abs(sc[0] - 1 / (1 + MU)) < 1e-6
     X = knob(100, d=12, seed=5)                              # has exact duplicates
     g = median_gamma(X, 5)
-    with bt.CandidateSet(X, g) as cs:
+    with bt.CandidateSet(X, g, flags=flags) as cs:
         idx, sc = cs.select(100, MU)
     assert sorted(idx.tolist()) == list(range(100))          # C7: m = N is a permutation
 
 
-def test_identity_kernel_ties_lowest_index():
+@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+def test_identity_kernel_ties_lowest_index(flags):
     X = (np.arange(40, dtype=np.float32) * 100.0)[:, None]  # K = I exactly in fp32
-    with bt.CandidateSet(X, 1.0) as cs:
+    with bt.CandidateSet(X, 1.0, flags=flags) as cs:
         idx, sc = cs.select(10, MU)
     assert idx.tolist() == list(range(10))                   # C9 + reading A5
     assert np.all(sc == np.float32(1.0) / np.float32(np.float32(1.0) + np.float32(MU)))
 
 
-def test_exact_duplicates_tie_to_lowest_index():
+@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+def test_exact_duplicates_tie_to_lowest_index(flags):
     X = knob(300, seed=2)
     X = np.concatenate([X, X[:50]], axis=0)                  # rows 300..349 duplicate rows 0..49
     g = median_gamma(X, 3)
-    with bt.CandidateSet(X, g) as cs:
+    with bt.CandidateSet(X, g, flags=flags) as cs:
         idx, sc = cs.select(40, MU)
     for s in idx:
         assert s < 300 or (s - 300) in idx[: list(idx).index(s)], "duplicate chosen before its twin"
@@ -158,10 +166,11 @@ def test_exact_duplicates_tie_to_lowest_index():
     check_ted(idx, sc, tr, "dups")
 
 
-def test_linear_kernel_closed_form_c8():
+@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+def test_linear_kernel_closed_form_c8(flags):
     rng = np.random.default_rng(8)
     X = (rng.standard_normal((300, 6)) * 0.5).astype(np.float32)
-    with bt.CandidateSet(X, 1.0, kernel=L.BTED_KERNEL_LINEAR) as cs:
+    with bt.CandidateSet(X, 1.0, kernel=L.BTED_KERNEL_LINEAR, flags=flags) as cs:
         idx, sc = cs.select(6, MU)
         K5 = cs.debug_K(300)[:, :300].astype(np.float64)
     Xd = X.astype(np.float64)
@@ -202,12 +211,13 @@ def _positions(V, pool_idx):
     return pos
 
 
-def test_bted_parity_vs_oracle():
+@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+def test_bted_parity_vs_oracle(flags):
     P, M, B, m, seed = 60000, 2048, 4, 32, 3
     space = KnobSpace(WORKLOADS["vgg16_conv1_1"], 16)
     _, X = make_pool(space, P, 77)
     g = median_gamma(X, 77)
-    with bt.CandidateSet(X, g, num_batches=B, seed=seed) as pool:
+    with bt.CandidateSet(X, g, num_batches=B, seed=seed, flags=flags) as pool:
         sel, bidx = pool.run_batches(M, m, MU)
     batches = oracle_sample_batches(P, M, B, seed)
     for b in range(B):
@@ -222,11 +232,12 @@ def test_bted_parity_vs_oracle():
     check_ted(mpos, [], trm, "merge")
 
 
-def test_round_robin_batches_then_merge_equals_run_batches():
+@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+def test_round_robin_batches_then_merge_equals_run_batches(flags):
     P, M, B, m, seed = 30000, 1024, 5, 16, 11
     X = knob(P, seed=4)
     g = median_gamma(X, 4)
-    with bt.CandidateSet(X, g, num_batches=B, seed=seed) as pool:
+    with bt.CandidateSet(X, g, num_batches=B, seed=seed, flags=flags) as pool:
         sel, bidx = pool.run_batches(M, m, MU)
         w0 = np.empty(3 * m, np.int64)
         w1 = np.full(3 * m, -1, np.int64)                    # rank 1 has 2 batches: padded like an all-gather
@@ -252,7 +263,7 @@ def test_row_sharded_loopback_bit_identical(N, P):
     from paper_conf_date_sunbg021_b200.dist import sharded_select_loopback
     X = knob(N, seed=N + P)
     g = median_gamma(X, P)
-    with bt.CandidateSet(X, g) as cs:
+    with bt.CandidateSet(X, g, flags=L.BTED_FLAG_DENSE) as cs:     # shards are dense
         idx, sc = cs.select(24, MU)
     dev = torch.device("cuda", 0)
     st = torch.cuda.Stream(dev)
@@ -264,6 +275,32 @@ def test_row_sharded_loopback_bit_identical(N, P):
 def test_launch_counter_counts_kernels():
     X = knob(300)
     before = bt.bted_kernel_launches()
-    with bt.CandidateSet(X, 0.3) as cs:
+    with bt.CandidateSet(X, 0.3, flags=L.BTED_FLAG_DENSE) as cs:
         cs.select(10, MU)
     assert bt.bted_kernel_launches() - before == 11          # transpose + K1 + 9 x K2
+    before = bt.bted_kernel_launches()
+    with bt.CandidateSet(X, 0.3) as cs:
+        cs.select(10, MU)
+    assert bt.bted_kernel_launches() - before == 19          # K1p + 9 x (pivot + K2p)
+
+
+# ------------------------------------------------------------------ packed vs dense layout
+@pytest.mark.parametrize("N,d,m", [(1000, 16, 40), (4099, 16, 64), (300, 12, 300), (129, 30, 20)])
+def test_packed_layout_matches_dense(N, d, m):
+    """Packed-symmetric storage (N4) computes every element of K bitwise like
+    the dense layout; only the norm summation order differs."""
+    X = knob(N, d=16, seed=N)[:, :d] if d <= 16 else uniform_pool(N, d, N)
+    g = median_gamma(X, d)
+    with bt.CandidateSet(X, g, flags=L.BTED_FLAG_DENSE) as cd, bt.CandidateSet(X, g) as cp:
+        i_d, s_d = cd.select(m, MU)
+        i_p, s_p = cp.select(m, MU)
+        tr = dense.ted(X, g, MU, m, forced=i_p)
+        check_ted(i_p, s_p, tr, f"packed-{N}")
+        if np.array_equal(i_d, i_p):
+            np.testing.assert_allclose(s_p, s_d, rtol=2e-6)
+            Kd, Kp = cd.debug_K(N), cp.debug_K(N)
+            assert np.array_equal(Kd[:, :N], Kp[:, :N])      # same pivots -> bitwise equal K
+            assert np.all(Kp[:, N:] == 0)
+        else:                                                  # only legitimate near-ties may differ
+            k = int(np.argmax(i_d != i_p))
+            assert tr.gap[k] <= 1e-5
