@@ -34,7 +34,7 @@ import numpy as np  # noqa: E402
 METRIC = "BTED selected points/sec and deflate-step HBM GB/s vs roofline at 1/2/4/8 B200"
 UNIT = "points/s"
 K2_NAME = {"dense": "deflate_rescore_kernel",
-           "packed": "deflate_packed_kernel (+ packed_pivot_kernel, per step)"}
+           "packed": "deflate_packed_kernel (+ finalize_packed_kernel, per step)"}
 
 
 def parse():

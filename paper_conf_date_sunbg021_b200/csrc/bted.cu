@@ -102,13 +102,9 @@ struct Ted {
     size_t keyscap = 0;
     int* err = nullptr;
     size_t errcap = 0;
-    // packed-symmetric layout (packed.cuh): partials, arrival counters, pivot row
+    // packed-symmetric layout (packed.cuh): per-tile norm partials [nT][nT*T]
     float* P = nullptr;
     size_t pcap = 0;
-    unsigned int* cnt = nullptr;
-    size_t cntcap = 0;
-    float* piv = nullptr;
-    size_t pivcap = 0;
     std::list<std::pair<GraphKey, cudaGraphExec_t>> graphs;   // LRU
     int64_t last_rows = 0, last_ld = 0;
     int last_buf = 0;
@@ -131,12 +127,10 @@ struct Ted {
         if (keys) cudaFree(keys);
         if (err) cudaFree(err);
         if (P) cudaFree(P);
-        if (cnt) cudaFree(cnt);
-        if (piv) cudaFree(piv);
         for (auto& sl : slots) for (auto e : sl.e) cudaEventDestroy(e);
         slots.clear();
         K[0] = K[1] = nullptr; XT = nullptr; sel = nullptr; keys = nullptr; err = nullptr;
-        P = nullptr; cnt = nullptr; piv = nullptr;
+        P = nullptr;
     }
 
     // Buffers of the packed layout for an N-point TED.
@@ -144,16 +138,14 @@ struct Ted {
         const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
         const size_t tiles = (size_t)bted::pk::num_tiles(nT) * bted::pk::T * bted::pk::T;
         const size_t NP = (size_t)nT * bted::pk::T;
-        const void* before[8] = {K[0], K[1], sel, keys, P, cnt, piv, XT};
+        const void* before[5] = {K[0], K[1], sel, keys, P};
         grow(K[0], kcap[0], tiles);
         if (m > 1) grow(K[1], kcap[1], tiles);
         grow(sel, selcap, NP);
         grow(keys, keyscap, (size_t)std::max(m, 1));
         grow(P, pcap, (size_t)nT * NP);
-        grow(cnt, cntcap, 2 * (size_t)nT);
-        grow(piv, pivcap, NP);
         if (!err) { grow(err, errcap, 1); CK(cudaMemsetAsync(err, 0, sizeof(int), stream)); }
-        const void* after[8] = {K[0], K[1], sel, keys, P, cnt, piv, XT};
+        const void* after[5] = {K[0], K[1], sel, keys, P};
         if (std::memcmp(before, after, sizeof before) != 0) {
             for (auto& g : graphs) cudaGraphExecDestroy(g.second);
             graphs.clear();
@@ -243,38 +235,42 @@ int num_sms() {
     }
     return g_num_sms;
 }
-constexpr size_t kK2pSmem = (size_t)bted::pk::kStages * bted::pk::kTileBytes + 2 * bted::pk::kStages * sizeof(uint64_t);
+constexpr size_t kK2pSmem = (size_t)bted::pk::kStages * bted::pk::kTileBytes +
+                            2 * (size_t)bted::pk::kGroups * bted::pk::T * sizeof(float) +
+                            2 * bted::pk::kStages * sizeof(uint64_t);
 
-// Alg. 1 l.1 + first l.3 on the packed tiles.  (1 kernel)
+// Alg. 1 l.1 + first l.3 on the packed tiles.  (2 kernels: K1p, fin)
 void enqueue_head_packed(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m,
                          float mu, unsigned long long* keys) {
     const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
     CK(cudaMemsetAsync(keys, 0, sizeof(unsigned long long) * m, T.stream));
     CK(cudaMemsetAsync(T.sel, 0, (size_t)nT * bted::pk::T, T.stream));
-    CK(cudaMemsetAsync(T.cnt, 0, sizeof(unsigned int) * 2 * nT, T.stream));
     const int64_t tiles = bted::pk::num_tiles(nT);
     const unsigned grid = (unsigned)std::min<int64_t>(tiles, (int64_t)num_sms() * 2);
     const int lin = kernel == BTED_KERNEL_LINEAR ? 1 : 0;
     if (d <= 16)
         bted::pk::gram_packed_kernel<16><<<grid, bted::pk::kConsumers, 0, T.stream>>>(
-            X, (int32_t)N, d, gamma, lin, T.K[0], nT, T.P, T.cnt, mu, keys, T.err);
+            X, (int32_t)N, d, gamma, lin, T.K[0], nT, T.P);
     else
         bted::pk::gram_packed_kernel<32><<<grid, bted::pk::kConsumers, 0, T.stream>>>(
-            X, (int32_t)N, d, gamma, lin, T.K[0], nT, T.P, T.cnt, mu, keys, T.err);
-    LAUNCHED(1);
+            X, (int32_t)N, d, gamma, lin, T.K[0], nT, T.P);
+    bted::pk::finalize_packed_kernel<<<nT, bted::pk::T, 0, T.stream>>>(T.P, nT, (int32_t)N, T.K[0], mu, T.sel,
+                                                                       keys, 0, keys, T.err);
+    LAUNCHED(2);
 }
 
-// Alg. 1 l.2-6 loop on the packed tiles: per step, pivot-row extraction + K2p.  (2(m-1) kernels)
+// Alg. 1 l.2-6 loop on the packed tiles: per step K2p (deflate + partials) and fin.  (2(m-1) kernels)
 void enqueue_loop_packed(Ted& T, int64_t N, int32_t m, float mu, unsigned long long* keys) {
     const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
     const int64_t tiles = bted::pk::num_tiles(nT);
     const unsigned grid = (unsigned)std::min<int64_t>(tiles, (int64_t)num_sms());
-    const unsigned pgrid = (unsigned)std::min<int64_t>(((int64_t)nT * bted::pk::T + 255) / 256, 1024);
     for (int32_t t = 1; t < m; ++t) {
         const float* Kin = T.K[(t - 1) & 1];
-        bted::pk::packed_pivot_kernel<<<pgrid, 256, 0, T.stream>>>(Kin, nT, keys, t - 1, T.piv);
+        float* Kout = T.K[t & 1];
         bted::pk::deflate_packed_kernel<<<grid, bted::pk::kConsumers + 32, kK2pSmem, T.stream>>>(
-            Kin, T.K[t & 1], nT, (int32_t)N, T.piv, T.P, T.cnt + (size_t)(t & 1) * nT, keys, t, mu, T.sel, T.err);
+            Kin, Kout, nT, (int32_t)N, T.P, keys, t, mu, T.sel);
+        bted::pk::finalize_packed_kernel<<<nT, bted::pk::T, 0, T.stream>>>(T.P, nT, (int32_t)N, Kout, mu, T.sel,
+                                                                           keys, t, keys + t, T.err);
         LAUNCHED(2);
     }
 }
@@ -367,7 +363,7 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
         head();
     } else {
         GraphKey key{X, N, d, m, kernel, 0, packed ? 1 : 0, fbits(mu), fbits(gamma), keys};
-        graph_run(T, key, packed ? 1 : 2, head);
+        graph_run(T, key, 2, head);
     }
     if (sl) CK(cudaEventRecord(sl->e[1], T.stream));
     if (m > 1) {

@@ -7,20 +7,23 @@
 // (+ the diagonal tiles' duplicated halves) instead of 8 N^2:
 //
 //   K2p: tile (I,J) <- tile - p_I p_J^T / (k(s,s)+mu)  (product first, as dense)
-//        row partials   P[J][i] = sum_{j in J} K_ij^2      (i in block I)
+//        row partials    P[J][i] = sum_{j in J} K_ij^2     (i in block I)
 //        column partials P[I][j] = sum_{i in I} K_ij^2     (j in block J, I < J)
-//   and ||K_v||^2 = sum_J P[J][v] in J order (deterministic), because the
-//   (I,J) block for J < I is the transpose of the stored (J,I) tile.
+//   fin: ||K_v||^2 = sum_J P[J][v] in J order, because block (I,J), J < I, is
+//        the transpose of the stored tile (J,I); score and masked argmax.
 //
 // Every element value is bitwise the same as in the dense layout (same
-// operands, same instruction); only the norm summation order differs.
+// operands, same instruction).  Row and column partials use ONE canonical
+// 128-term summation tree (groups of 4 consecutive terms, then a
+// 32-leaf butterfly), so a row's norm does not depend on whether its
+// partials came from rows or columns of stored tiles: exact duplicate points
+// get bitwise-equal scores and tie to the lowest index (reading A5).
 //
 // K2p is a TMA pipeline: one producer warp streams tiles into a 3-stage
 // shared-memory ring with cp.async.bulk (mbarrier complete_tx), eight
-// consumer warps update them, store the new tile with 128-bit streaming
-// stores and reduce the partials.  The block of rows whose partials are
-// complete is finished (score + argmax) by the CTA that delivers its last
-// partial (a per-block arrival counter), so a step stays ONE kernel.
+// consumer warps update them and write the new tile with 128-bit streaming
+// stores.  Pivot segments (row s of K_in restricted to a tile's row/column
+// block) are read straight from K_in: no pivot-extraction kernel.
 #pragma once
 #include <cstdint>
 #include <cuda_runtime.h>
@@ -33,6 +36,7 @@ constexpr int T = 128;                 // tile edge
 constexpr int kConsumers = 256;        // 8 consumer warps
 constexpr int kStages = 3;
 constexpr int kTileBytes = T * T * 4;  // 64 KiB
+constexpr int kGroups = T / 4;         // 32 groups of 4 rows per tile
 
 __host__ __device__ __forceinline__ int64_t tile_offset(int I, int J, int nT) {
     // tiles of rows 0..I-1 precede row I: sum_{i<I} (nT - i)
@@ -42,7 +46,6 @@ __host__ __device__ __forceinline__ int64_t num_tiles(int nT) { return (int64_t)
 
 // tile linear index -> (I, J) (row-major over the upper triangle)
 __device__ __forceinline__ void tile_ij(int64_t k, int nT, int& I, int& J) {
-    // solve offset(I) <= k < offset(I+1) with offset(I) = I*nT - I(I-1)/2
     double a = 2.0 * nT + 1.0;
     int i = (int)((a - sqrt(a * a - 8.0 * (double)k)) * 0.5);
     if (i < 0) i = 0;
@@ -51,6 +54,13 @@ __device__ __forceinline__ void tile_ij(int64_t k, int nT, int& I, int& J) {
     while (i < nT - 1 && tile_offset(i + 1, i + 1, nT) <= k) ++i;
     I = i;
     J = i + (int)(k - tile_offset(i, i, nT));
+}
+
+// element (i, j) of the symmetric matrix in packed storage
+__device__ __forceinline__ int64_t packed_index(int i, int j, int nT) {
+    const int I = i / T, J = j / T;
+    return I <= J ? tile_offset(I, J, nT) * (T * T) + (int64_t)(i % T) * T + (j % T)
+                  : tile_offset(J, I, nT) * (T * T) + (int64_t)(j % T) * T + (i % T);
 }
 
 // ------------------------------------------------------------------ PTX helpers
@@ -80,119 +90,82 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 __device__ __forceinline__ void consumer_sync() {       // named barrier 1: the 256 consumer threads
     asm volatile("bar.sync 1, %0;" :: "n"(kConsumers) : "memory");
 }
-__device__ __forceinline__ float4 lds4(const float* p) { return *reinterpret_cast<const float4*>(p); }
 
-// ------------------------------------------------------------------ shared epilogue
-// Partials of one finished tile: rowp[r] (row sums over the tile's columns)
-// and, for off-diagonal tiles, colp[c].  Written to P, then the arrival
-// counters of blocks I and J are bumped; a block whose nT partials are all
-// in is finished by this CTA: g_i = sum_J P[J][i], score, masked argmax.
-struct Epi {
-    float* P;                // [nT][NP] partials
-    int64_t NP;              // nT * T
-    unsigned int* cnt;       // [nT] arrival counters (this step's parity)
-    const float* Kdiag_base; // Kout (diagonal read-back)
-    int nT, N;
-    float mu;
-    const uint8_t* sel;
-    uint32_t s;              // pivot of this step (0xFFFFFFFF for the Gram)
-    unsigned long long* key_out;
-    int* err;
+// ------------------------------------------------------------------ canonical sums
+// group of 4 consecutive terms: ((v0^2 + v1^2) + v2^2) + v3^2 with fused steps
+__device__ __forceinline__ float group4(float v0, float v1, float v2, float v3) {
+    float g = __fmul_rn(v0, v0);
+    g = __fmaf_rn(v1, v1, g);
+    g = __fmaf_rn(v2, v2, g);
+    return __fmaf_rn(v3, v3, g);
+}
+// 32-leaf butterfly over groups held by smem column (stride T): same tree as warp_sum
+__device__ __forceinline__ float tree32_smem(const float* g, int stride) {
+    float h[kGroups];
+#pragma unroll
+    for (int q = 0; q < kGroups; ++q) h[q] = g[q * stride];
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1)
+#pragma unroll
+        for (int q = 0; q < off; ++q) h[q] = __fadd_rn(h[q], h[q + off]);
+    return h[0];
+}
+
+// Per-lane state while a warp walks its 16 rows of a tile (lane l owns columns 4l..4l+3).
+struct RowWalk {
+    float cg[4];     // running group-of-4-rows sums for the lane's 4 columns
+    float rowsum;    // lane l < 16: partial of row 16w + l
 };
 
-__device__ __forceinline__ void finish_block(const Epi& e, int B, int tid, unsigned long long* red) {
-    unsigned long long key = 0ull;
-    if (tid < T) {
-        const int i = B * T + tid;
-        if (i < e.N) {
-            float g = 0.f;
-            for (int J = 0; J < e.nT; ++J) g = __fadd_rn(g, __ldcg(e.P + (int64_t)J * e.NP + i));
-            const float* dt = e.Kdiag_base + tile_offset(B, B, e.nT) * (int64_t)(T * T);
-            const float diag = __ldcg(dt + tid * T + tid);
-            const bool masked = (e.sel && e.sel[i] != 0) || (uint32_t)i == e.s;
-            key = score_key(g, diag, e.mu, (uint32_t)i, masked, e.err);
+// one row (index rr within the warp's 16) of new values o -> partials
+__device__ __forceinline__ void walk_row(RowWalk& a, int rr, int l, const float4& o, float (*colg)[T], int w,
+                                         bool want_cols) {
+    float rp = group4(o.x, o.y, o.z, o.w);
+    rp = warp_sum(rp);                                   // butterfly over the 32 groups of the row
+    if (l == rr) a.rowsum = rp;
+    if (want_cols) {
+        if ((rr & 3) == 0) {
+            a.cg[0] = __fmul_rn(o.x, o.x); a.cg[1] = __fmul_rn(o.y, o.y);
+            a.cg[2] = __fmul_rn(o.z, o.z); a.cg[3] = __fmul_rn(o.w, o.w);
+        } else {
+            a.cg[0] = __fmaf_rn(o.x, o.x, a.cg[0]); a.cg[1] = __fmaf_rn(o.y, o.y, a.cg[1]);
+            a.cg[2] = __fmaf_rn(o.z, o.z, a.cg[2]); a.cg[3] = __fmaf_rn(o.w, o.w, a.cg[3]);
+        }
+        if ((rr & 3) == 3) {                            // group (16w + rr) / 4 complete
+            const int q = 4 * w + (rr >> 2);
+            *reinterpret_cast<float4*>(&colg[q][4 * l]) = make_float4(a.cg[0], a.cg[1], a.cg[2], a.cg[3]);
         }
     }
-    key = warp_max_u64(key);
-    const int w = tid / kWarp, l = tid % kWarp;
-    if (l == 0) red[w] = key;
-    consumer_sync();
-    if (tid == 0) {
-        unsigned long long v = 0ull;
-        for (int k = 0; k < kConsumers / kWarp; ++k) v = red[k] > v ? red[k] : v;
-        if (v) atomicMax(e.key_out, v);
-    }
-    consumer_sync();
 }
 
-// After the tile's partials are stored by the consumers (all 256 threads
-// passed consumer_sync): count arrivals, finish completed blocks.
-__device__ __forceinline__ void arrive_and_finish(const Epi& e, int I, int J, int tid, int* flag,
-                                                  unsigned long long* red) {
-    __threadfence();                 // this thread's tile / partial stores are visible GPU-wide
-    consumer_sync();
-    if (tid == 0) {
-        int f = 0;
-        if (atomicAdd(e.cnt + I, 1u) == (unsigned)(e.nT - 1)) f |= 1;
-        if (I != J && atomicAdd(e.cnt + J, 1u) == (unsigned)(e.nT - 1)) f |= 2;
-        if (f) __threadfence();
-        *flag = f;
-    }
-    consumer_sync();
-    const int f = *flag;
-    if (f & 1) { if (tid == 0) e.cnt[I] = 0u; finish_block(e, I, tid, red); }
-    if (f & 2) { if (tid == 0) e.cnt[J] = 0u; finish_block(e, J, tid, red); }
-}
-
-// Consumer part common to K1p / K2p: given 16 rows x 4 columns of new
-// values per lane (row-by-row), accumulate partials.  Layout: warp w owns
-// rows 16w..16w+15 of the tile, lane l owns columns 4l..4l+3.
-struct TileAcc {
-    float col[4];
-    float rowsum;            // lane l < 16: the sum of row 16w + l after the tile
-};
-
-__device__ __forceinline__ void store_partials(const Epi& e, int I, int J, int w, int l, const TileAcc& a,
-                                               float (*colred)[T]) {
-    // row partials of rows 16w + l (l < 16) -> P[J][I*T + 16w + l]
-    if (l < 16) e.P[(int64_t)J * e.NP + (int64_t)I * T + 16 * w + l] = a.rowsum;
-    if (I != J) {
-        colred[w][4 * l + 0] = a.col[0];
-        colred[w][4 * l + 1] = a.col[1];
-        colred[w][4 * l + 2] = a.col[2];
-        colred[w][4 * l + 3] = a.col[3];
-    }
-    consumer_sync();
-    const int tid = w * kWarp + l;
-    if (I != J && tid < T) {
-        float c = 0.f;
-        for (int ww = 0; ww < kConsumers / kWarp; ++ww) c = __fadd_rn(c, colred[ww][tid]);
-        e.P[(int64_t)I * e.NP + (int64_t)J * T + tid] = c;
-    }
-    consumer_sync();
+// After all 8 warps walked the tile (and colg is complete, consumer_sync
+// done by the caller): write row partials and the column tree.
+__device__ __forceinline__ void write_partials(float* P, int64_t NP, int I, int J, int w, int l, const RowWalk& a,
+                                               float (*colg)[T], int tid) {
+    if (l < 16) P[(int64_t)J * NP + (int64_t)I * T + 16 * w + l] = a.rowsum;
+    if (I != J && tid < T) P[(int64_t)I * NP + (int64_t)J * T + tid] = tree32_smem(&colg[0][tid], T);
 }
 
 // ------------------------------------------------------------------ K1p: Gram tiles
-// Alg. 1 l.1 + first l.3 on the upper-triangular tiles.  One CTA (256
-// threads) per tile in a persistent loop.  Lane l keeps the features of its
-// 4 columns in registers (kD <= 32); the rows' features are smem broadcasts.
+// Alg. 1 l.1 on the upper-triangular tiles (+ the partials of the first l.3).
+// One CTA (256 threads) per tile in a persistent loop.  Lane l keeps the
+// features of its 4 columns in registers (kD <= 32); the rows' features
+// are smem broadcasts.
 template <int kD>
 __global__ void __launch_bounds__(kConsumers)
 gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma, int32_t linear,
-                   float* __restrict__ K, int nT, float* __restrict__ P, unsigned int* __restrict__ cnt,
-                   float mu, unsigned long long* __restrict__ key_out, int* __restrict__ err) {
+                   float* __restrict__ K, int nT, float* __restrict__ P) {
     __shared__ __align__(16) float xi[T][kD];
     __shared__ __align__(16) float xj[T][kD];
-    __shared__ float colred[kConsumers / kWarp][T];
-    __shared__ unsigned long long red[kConsumers / kWarp];
-    __shared__ int flag;
+    __shared__ __align__(16) float colg[kGroups][T];
     const int tid = threadIdx.x, w = tid / kWarp, l = tid % kWarp;
     const int64_t ntiles = num_tiles(nT);
+    const int64_t NP = (int64_t)nT * T;
     const float ng = -gamma;
-    Epi e{P, (int64_t)nT * T, cnt, K, nT, N, mu, nullptr, 0xFFFFFFFFu, key_out, err};
     for (int64_t k = blockIdx.x; k < ntiles; k += gridDim.x) {
         int I, J;
         tile_ij(k, nT, I, J);
+        consumer_sync();                                 // previous tile's smem readers are done
         for (int q = tid; q < T * kD; q += kConsumers) {
             const int r = q / kD, c = q % kD;
             const int gi = I * T + r, gj = J * T + r;
@@ -209,8 +182,7 @@ gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamm
                 y[c][q] = v.x; y[c][q + 1] = v.y; y[c][q + 2] = v.z; y[c][q + 3] = v.w;
             }
         float* tile = K + k * (int64_t)(T * T);
-        TileAcc a;
-        a.col[0] = a.col[1] = a.col[2] = a.col[3] = 0.f;
+        RowWalk a;
         a.rowsum = 0.f;
         for (int rr = 0; rr < 16; ++rr) {
             const int r = 16 * w + rr;
@@ -230,54 +202,63 @@ gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamm
             }
             float4 o;
             float* oc = &o.x;
-            float rp = 0.f;
             const bool rv = I * T + r < N;
 #pragma unroll
             for (int c = 0; c < 4; ++c) {
                 const bool cv = J * T + 4 * l + c < N;
                 const float val = linear ? acc[c] : expf(__fmul_rn(ng, acc[c]));
                 oc[c] = (rv && cv) ? val : 0.f;
-                rp = __fmaf_rn(oc[c], oc[c], rp);
-                a.col[c] = __fmaf_rn(oc[c], oc[c], a.col[c]);
             }
             st_stream(tile + r * T + 4 * l, o);
-            rp = warp_sum(rp);
-            if (l == rr) a.rowsum = rp;
+            walk_row(a, rr, l, o, colg, w, I != J);
         }
-        store_partials(e, I, J, w, l, a, colred);
-        arrive_and_finish(e, I, J, tid, &flag, red);
+        consumer_sync();
+        write_partials(P, NP, I, J, w, l, a, colg, tid);
     }
 }
 
-// ------------------------------------------------------------------ pivot extraction
-// p[j] = K[s][j] for j < nT*T, s = key_index(keys[t]) (the new pivot).
-__global__ void packed_pivot_kernel(const float* __restrict__ K, int nT, const unsigned long long* __restrict__ keys,
-                                    int32_t t, float* __restrict__ p) {
-    const uint32_t s = key_index(keys[t]);
-    const int S = (int)(s / T), rs = (int)(s % T);
+// ------------------------------------------------------------------ fin: scores + argmax
+// Alg. 1 l.3 from the partials: g_i = sum_J P[J][i] (J order), score =
+// g / (k(i,i) + mu) with the new diagonal read back from the diagonal tile,
+// masked (selected / the pivot / padding), packed key -> atomicMax(key_out).
+// One CTA of T threads per row block.
+__global__ void __launch_bounds__(T)
+finalize_packed_kernel(const float* __restrict__ P, int nT, int32_t N, const float* __restrict__ K, float mu,
+                       const uint8_t* __restrict__ sel, const unsigned long long* __restrict__ keys, int32_t t,
+                       unsigned long long* __restrict__ key_out, int* __restrict__ err) {
+    const int B = blockIdx.x, r = threadIdx.x;
     const int64_t NP = (int64_t)nT * T;
-    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < NP; j += (int64_t)gridDim.x * blockDim.x) {
-        const int J = (int)(j / T), c = (int)(j % T);
-        float v;
-        if (S <= J) v = K[tile_offset(S, J, nT) * (T * T) + rs * T + c];
-        else        v = K[tile_offset(J, S, nT) * (T * T) + c * T + rs];
-        p[j] = v;
+    const int i = B * T + r;
+    const uint32_t s = t > 0 ? key_index(keys[t - 1]) : 0xFFFFFFFFu;
+    unsigned long long key = 0ull;
+    if (i < N) {
+        float g = 0.f;
+        int J = 0;
+        for (; J + 8 <= nT; J += 8) {
+            float v[8];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) v[q] = P[(int64_t)(J + q) * NP + i];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) g = __fadd_rn(g, v[q]);
+        }
+        for (; J < nT; ++J) g = __fadd_rn(g, P[(int64_t)J * NP + i]);
+        const float diag = K[tile_offset(B, B, nT) * (T * T) + (int64_t)r * T + r];
+        const bool masked = sel[i] != 0 || (uint32_t)i == s;
+        key = score_key(g, diag, mu, (uint32_t)i, masked, err);
     }
+    cta_key_max_to<T>(key, key_out);
 }
 
 // ------------------------------------------------------------------ K2p: TMA deflate
 __global__ void __launch_bounds__(kConsumers + kWarp, 1)
 deflate_packed_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, int nT, int32_t N,
-                      const float* __restrict__ p, float* __restrict__ P, unsigned int* __restrict__ cnt,
-                      unsigned long long* __restrict__ keys, int32_t t, float mu, uint8_t* __restrict__ sel,
-                      int* __restrict__ err) {
+                      float* __restrict__ P, const unsigned long long* __restrict__ keys, int32_t t, float mu,
+                      uint8_t* __restrict__ sel) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
     float* stage = reinterpret_cast<float*>(smem_raw);                       // [kStages][T*T]
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + kStages * kTileBytes);
+    float (*colg)[kGroups][T] = reinterpret_cast<float (*)[kGroups][T]>(smem_raw + kStages * kTileBytes);  // [2]
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + kStages * kTileBytes + 2 * kGroups * T * 4);
     uint64_t* empty = full + kStages;
-    __shared__ float colred[kConsumers / kWarp][T];
-    __shared__ unsigned long long red[kConsumers / kWarp];
-    __shared__ int flag;
 
     const int tid = threadIdx.x;
     const int64_t ntiles = num_tiles(nT);
@@ -308,51 +289,54 @@ deflate_packed_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, i
 
     // ---------------- consumers
     const int w = tid / kWarp, l = tid % kWarp;
+    const int64_t NP = (int64_t)nT * T;
     const uint32_t s = key_index(keys[t - 1]);
-    const float inv_c = __frcp_rn(__fadd_rn(p[s], mu));
+    const int S = (int)(s / T), rs = (int)(s % T);
+    const float inv_c = __frcp_rn(__fadd_rn(Kin[packed_index((int)s, (int)s, nT)], mu));   // 1/(k(s,s)+mu)
     if (blockIdx.x == 0 && tid == 0 && (int32_t)s < N) sel[s] = 1;
-    Epi e{P, (int64_t)nT * T, cnt, Kout, nT, N, mu, sel, s, keys + t, err};
+    // K_in[s, B*T + c]: a contiguous row segment of tile (S,B) if S <= B, else a
+    // column of tile (B,S)
+    auto seg = [&](int B, int c) -> float {
+        return S <= B ? Kin[tile_offset(S, B, nT) * (T * T) + (int64_t)rs * T + c]
+                      : Kin[tile_offset(B, S, nT) * (T * T) + (int64_t)c * T + rs];
+    };
     int n = 0;
     for (int64_t k = blockIdx.x; k < ntiles; k += gridDim.x, ++n) {
         int I, J;
         tile_ij(k, nT, I, J);
         const int st = n % kStages;
         const uint32_t ph = (uint32_t)(n / kStages) & 1u;
-        // pivot segments: rows of block I (one per lane < 16), columns of block J
-        const float pr_l = l < 16 ? p[I * T + 16 * w + l] : 0.f;
-        const float4 pc = *reinterpret_cast<const float4*>(p + J * T + 4 * l);
+        float (*cg)[T] = colg[n & 1];
+        // pivot segments: a_i for the warp's 16 rows (lane < 16), p_j for the lane's 4 columns
+        const float pr_l = l < 16 ? seg(I, 16 * w + l) : 0.f;
+        float4 pc;
+        if (S <= J) {
+            pc = *reinterpret_cast<const float4*>(Kin + tile_offset(S, J, nT) * (T * T) + (int64_t)rs * T + 4 * l);
+        } else {
+            pc.x = seg(J, 4 * l); pc.y = seg(J, 4 * l + 1); pc.z = seg(J, 4 * l + 2); pc.w = seg(J, 4 * l + 3);
+        }
         mbar_wait(full + st, ph);
         const float* sm = stage + st * (T * T);
         float* gout = Kout + k * (int64_t)(T * T);
-        TileAcc a;
-        a.col[0] = a.col[1] = a.col[2] = a.col[3] = 0.f;
+        RowWalk a;
         a.rowsum = 0.f;
 #pragma unroll 4
         for (int rr = 0; rr < 16; ++rr) {
             const int r = 16 * w + rr;
             const float ai = __shfl_sync(0xffffffffu, pr_l, rr);
-            const float4 kv = lds4(sm + r * T + 4 * l);
+            const float4 kv = *reinterpret_cast<const float4*>(sm + r * T + 4 * l);
             float4 o;
             o.x = deflate1(kv.x, ai, pc.x, inv_c);
             o.y = deflate1(kv.y, ai, pc.y, inv_c);
             o.z = deflate1(kv.z, ai, pc.z, inv_c);
             o.w = deflate1(kv.w, ai, pc.w, inv_c);
             st_stream(gout + r * T + 4 * l, o);
-            float rp = __fmul_rn(o.x, o.x);
-            rp = __fmaf_rn(o.y, o.y, rp);
-            rp = __fmaf_rn(o.z, o.z, rp);
-            rp = __fmaf_rn(o.w, o.w, rp);
-            a.col[0] = __fmaf_rn(o.x, o.x, a.col[0]);
-            a.col[1] = __fmaf_rn(o.y, o.y, a.col[1]);
-            a.col[2] = __fmaf_rn(o.z, o.z, a.col[2]);
-            a.col[3] = __fmaf_rn(o.w, o.w, a.col[3]);
-            rp = warp_sum(rp);
-            if (l == rr) a.rowsum = rp;
+            walk_row(a, rr, l, o, cg, w, I != J);
         }
         __syncwarp();
         if (l == 0) mbar_arrive(empty + st);       // this warp is done reading the stage
-        store_partials(e, I, J, w, l, a, colred);
-        arrive_and_finish(e, I, J, tid, &flag, red);
+        consumer_sync();                           // colg of this tile complete
+        write_partials(P, NP, I, J, w, l, a, cg, tid);
     }
 }
 

@@ -281,7 +281,7 @@ def test_launch_counter_counts_kernels():
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3) as cs:
         cs.select(10, MU)
-    assert bt.bted_kernel_launches() - before == 19          # K1p + 9 x (pivot + K2p)
+    assert bt.bted_kernel_launches() - before == 20          # K1p + fin + 9 x (K2p + fin)
 
 
 # ------------------------------------------------------------------ packed vs dense layout
