@@ -60,6 +60,8 @@ typedef enum {
 #define BTED_FLAG_DENSE    4u   /* store K densely (N x ld, 8 N^2 bytes per step) instead of the
                                    default packed upper-triangular tiles (4 N^2 bytes per step;
                                    used when d <= 32).  Shard contexts are always dense. */
+#define BTED_FLAG_NO_SMALL 8u   /* never use the one-kernel cluster TED for small candidate sets
+                                   (N <= ~940: K in distributed shared memory)               */
 #define BTED_FLAG_TIMING   2u   /* record CUDA events around K1 and the K2 loop of every batch
                                    TED on the ctx stream; read with bted_get_stats()          */
 

@@ -25,6 +25,7 @@
 #include "kernels.cuh"
 #include "sample.cuh"
 #include "packed.cuh"
+#include "small.cuh"
 
 namespace {
 
@@ -254,7 +255,7 @@ void enqueue_head_packed(Ted& T, const float* X, int64_t N, int32_t d, float gam
     else
         bted::pk::gram_packed_kernel<32><<<grid, bted::pk::kConsumers, 0, T.stream>>>(
             X, (int32_t)N, d, gamma, lin, T.K[0], nT, T.P);
-    bted::pk::finalize_packed_kernel<<<nT, bted::pk::T, 0, T.stream>>>(T.P, nT, (int32_t)N, T.K[0], mu, T.sel,
+    bted::pk::finalize_packed_kernel<<<nT, bted::pk::kFinThreads, 0, T.stream>>>(T.P, nT, (int32_t)N, T.K[0], mu, T.sel,
                                                                        keys, 0, keys, T.err);
     LAUNCHED(2);
 }
@@ -269,7 +270,7 @@ void enqueue_loop_packed(Ted& T, int64_t N, int32_t m, float mu, unsigned long l
         float* Kout = T.K[t & 1];
         bted::pk::deflate_packed_kernel<<<grid, bted::pk::kConsumers + 32, kK2pSmem, T.stream>>>(
             Kin, Kout, nT, (int32_t)N, T.P, keys, t, mu, T.sel);
-        bted::pk::finalize_packed_kernel<<<nT, bted::pk::T, 0, T.stream>>>(T.P, nT, (int32_t)N, Kout, mu, T.sel,
+        bted::pk::finalize_packed_kernel<<<nT, bted::pk::kFinThreads, 0, T.stream>>>(T.P, nT, (int32_t)N, Kout, mu, T.sel,
                                                                            keys, t, keys + t, T.err);
         LAUNCHED(2);
     }
@@ -415,6 +416,9 @@ struct bted_ctx {
     unsigned long long* mkeys = nullptr; size_t mkeyscap = 0;
     void* cub_tmp = nullptr; size_t cub_cap = 0;
     int64_t* out_dev = nullptr; size_t outcap = 0;
+    uint32_t* sall = nullptr; size_t sallcap = 0;          // small-batch path: [nb][M] draws
+    float* xall = nullptr; size_t xallcap = 0;             // [nb][M][d] gathered batches
+    unsigned long long* kall = nullptr; size_t kallcap = 0; // [nb][m] keys
     // host staging (pinned)
     unsigned long long* hkeys = nullptr; size_t hkeyscap = 0;
     int* herr = nullptr;
@@ -581,7 +585,8 @@ int bits_for(uint64_t maxval) {
 }
 
 // Alg. 2 l.2 on the device: sidx[0..M) = sorted V_b.  P = pool rows.
-void sample_batch(bted_ctx* ctx, cudaStream_t st, int64_t P, int64_t M, int32_t b, uint64_t seed) {
+void sample_batch(bted_ctx* ctx, cudaStream_t st, int64_t P, int64_t M, int32_t b, uint64_t seed,
+                  uint32_t* dst = nullptr) {
     grow(ctx->skeys, ctx->skeyscap, (size_t)P);
     grow(ctx->skeys2, ctx->skeys2cap, (size_t)P);
     grow(ctx->sidx, ctx->sidxcap, (size_t)M);
@@ -592,7 +597,8 @@ void sample_batch(bted_ctx* ctx, cudaStream_t st, int64_t P, int64_t M, int32_t 
     LAUNCHED(1);
     size_t need = 0, need2 = 0;
     CK(cub::DeviceRadixSort::SortKeys(nullptr, need, ctx->skeys, ctx->skeys2, (int)P, 0, 64, st));
-    CK(cub::DeviceRadixSort::SortKeys(nullptr, need2, ctx->sidx2, ctx->sidx, (int)M, 0, bits_for(P), st));
+    if (!dst) dst = ctx->sidx;
+    CK(cub::DeviceRadixSort::SortKeys(nullptr, need2, ctx->sidx2, dst, (int)M, 0, bits_for(P), st));
     cub_reserve(ctx, std::max(need, need2));
     size_t cap = ctx->cub_cap;
     CK(cub::DeviceRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->skeys, ctx->skeys2, (int)P, 0, 64, st));
@@ -600,15 +606,68 @@ void sample_batch(bted_ctx* ctx, cudaStream_t st, int64_t P, int64_t M, int32_t 
     bted::low_half_kernel<<<gm, 256, 0, st>>>(ctx->skeys2, M, ctx->sidx2);
     LAUNCHED(1);
     cap = ctx->cub_cap;
-    CK(cub::DeviceRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->sidx2, ctx->sidx, (int)M, 0, bits_for(P), st));
+    CK(cub::DeviceRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->sidx2, dst, (int)M, 0, bits_for(P), st));
 }
 
-void gather(bted_ctx* ctx, cudaStream_t st, const uint32_t* idx, int64_t M) {
-    grow(ctx->Xb, ctx->xbcap, (size_t)(M * ctx->d));
+void gather(bted_ctx* ctx, cudaStream_t st, const uint32_t* idx, int64_t M, float* dst = nullptr) {
+    if (!dst) {
+        grow(ctx->Xb, ctx->xbcap, (size_t)(M * ctx->d));
+        dst = ctx->Xb;
+    }
     const int64_t total = M * ctx->d;
     const unsigned g = (unsigned)std::min<int64_t>((total + 255) / 256, 148 * 32);
-    bted::gather_rows_kernel<<<g, 256, 0, st>>>(ctx->X, ctx->d, idx, M, ctx->Xb);
+    bted::gather_rows_kernel<<<g, 256, 0, st>>>(ctx->X, ctx->d, idx, M, dst);
     LAUNCHED(1);
+}
+
+// ---- small TEDs: one cluster kernel per launch runs every step (small.cuh) ----
+int small_cluster_for(int64_t N) {
+    if (N < 1 || N > 4096) return 0;
+    for (int C = 1; C <= 16; C *= 2)
+        if (bted::sm::smem_bytes((int)N, C) <= bted::sm::kSmemBudget) return C;
+    return 0;
+}
+bool use_small(uint32_t flags, int64_t N) { return !(flags & BTED_FLAG_NO_SMALL) && small_cluster_for(N) > 0; }
+
+template <int C>
+void launch_small_c(const float* X, int ninst, int32_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
+                    unsigned long long* keys, int* err, cudaStream_t st) {
+    static bool attr = false;
+    if (!attr) {
+        CK(cudaFuncSetAttribute(bted::sm::ted_cluster_kernel<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)bted::sm::kSmemBudget));
+        if (C > 8) CK(cudaFuncSetAttribute(bted::sm::ted_cluster_kernel<C>,
+                                           cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+        attr = true;
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(ninst * C));
+    cfg.blockDim = dim3(bted::sm::kThreads);
+    cfg.dynamicSmemBytes = bted::sm::smem_bytes(N, C);
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = C;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    CK(cudaLaunchKernelEx(&cfg, bted::sm::ted_cluster_kernel<C>, X, N, d, gamma,
+                          (int32_t)(kernel == BTED_KERNEL_LINEAR ? 1 : 0), m, mu, keys, err));
+    LAUNCHED(1);
+}
+
+// ninst independent TEDs on X[inst][N][d] -> keys[inst][m]; err = a Ted's flag
+void launch_small(const float* X, int ninst, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
+                  unsigned long long* keys, int* err, cudaStream_t st) {
+    switch (small_cluster_for(N)) {
+        case 1: launch_small_c<1>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st); break;
+        case 2: launch_small_c<2>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st); break;
+        case 4: launch_small_c<4>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st); break;
+        case 8: launch_small_c<8>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st); break;
+        case 16: launch_small_c<16>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st); break;
+        default: throw CudaError{cudaErrorInvalidValue, "launch_small: N too large"};
+    }
 }
 
 // Alg. 2 l.1-4 for batches b_begin, b_begin+b_step, ... ; winners on device.
@@ -620,6 +679,27 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
     grow(ctx->mkeys, ctx->mkeyscap, (size_t)m);
     cudaStream_t st = ctx->stream;
     const bool no_graph = (ctx->params.flags & BTED_FLAG_NO_GRAPH) != 0;
+    if (nb > 0 && use_small(ctx->params.flags, M)) {
+        // small batches (the paper's M = 500): all batch TEDs in ONE cluster launch
+        grow(ctx->sall, ctx->sallcap, (size_t)nb * M);
+        grow(ctx->xall, ctx->xallcap, (size_t)nb * M * ctx->d);
+        grow(ctx->kall, ctx->kallcap, (size_t)nb * m);
+        Ted& T = ctx->bted_engine;
+        if (!T.err) { grow(T.err, T.errcap, 1); CK(cudaMemsetAsync(T.err, 0, sizeof(int), st)); }
+        int kk = 0;
+        for (int32_t b = b_begin; b < B; b += b_step, ++kk) {
+            sample_batch(ctx, st, ctx->N, M, b, ctx->params.seed, ctx->sall + (size_t)kk * M);
+            gather(ctx, st, ctx->sall + (size_t)kk * M, M, ctx->xall + (size_t)kk * M * ctx->d);
+        }
+        launch_small(ctx->xall, nb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->kall, T.err, st);
+        for (kk = 0; kk < nb; ++kk) {
+            bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->kall + (size_t)kk * m, m,
+                                                                     ctx->sall + (size_t)kk * M,
+                                                                     ctx->winners + (size_t)kk * m);
+            LAUNCHED(1);
+        }
+        return nb;
+    }
     int k = 0;
     for (int32_t b = b_begin; b < B; b += b_step, ++k) {
         sample_batch(ctx, st, ctx->N, M, b, ctx->params.seed);
@@ -662,9 +742,16 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
     gather(ctx, st, ctx->u32a, nu);                       // X[X_U] (A13: fresh Gram)
     grow(ctx->mkeys, ctx->mkeyscap, (size_t)mm);
     grow(ctx->out_dev, ctx->outcap, (size_t)mm);
-    // the merge is tiny (|X_U| <= B m) and its size varies: run it eagerly
-    run_ted(ctx->bted_engine, ctx->Xb, nu, ctx->d, ctx->params.gamma, ctx->kernel, mm, mu, ctx->mkeys,
-            true, /*time_it=*/false, use_packed(ctx->params.flags, ctx->d));
+    if (use_small(ctx->params.flags, nu)) {
+        // the merge is small (|X_U| <= B m): one cluster kernel runs all its steps
+        Ted& T = ctx->bted_engine;
+        if (!T.err) { grow(T.err, T.errcap, 1); CK(cudaMemsetAsync(T.err, 0, sizeof(int), st)); }
+        launch_small(ctx->Xb, 1, nu, ctx->d, ctx->params.gamma, ctx->kernel, mm, mu, ctx->mkeys, T.err, st);
+    } else {
+        // size varies with |X_U|: run it eagerly
+        run_ted(ctx->bted_engine, ctx->Xb, nu, ctx->d, ctx->params.gamma, ctx->kernel, mm, mu, ctx->mkeys,
+                true, /*time_it=*/false, use_packed(ctx->params.flags, ctx->d));
+    }
     bted::map_winners_kernel<<<(mm + 127) / 128, 128, 0, st>>>(ctx->mkeys, mm, ctx->u32a, ctx->out_dev);
     LAUNCHED(1);
     bted_status s = finish_keys(ctx, ctx->bted_engine, ctx->mkeys, mm, out_idx, nullptr, ctx->out_dev);
@@ -701,6 +788,13 @@ bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, fl
     if (m < 1 || m > ctx->N || !mu_ok(mu)) { set_error("need 1 <= m <= N and mu > 0 finite"); return BTED_EINVAL; }
     return guarded(ctx, [&]() -> bted_status {
         Ted& T = ctx->ted;
+        if (use_small(ctx->params.flags, ctx->N)) {
+            grow(T.keys, T.keyscap, (size_t)m);
+            if (!T.err) { grow(T.err, T.errcap, 1); CK(cudaMemsetAsync(T.err, 0, sizeof(int), T.stream)); }
+            launch_small(ctx->X, 1, ctx->N, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, T.keys, T.err, T.stream);
+            T.last_rows = 0;                       // K lived in shared memory only
+            return finish_keys(ctx, T, T.keys, m, out_idx, out_score);
+        }
         T.reserve(ctx->N, ctx->N, ctx->d, m);
         run_ted(T, ctx->X, ctx->N, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, T.keys,
                 (ctx->params.flags & BTED_FLAG_NO_GRAPH) != 0, true, use_packed(ctx->params.flags, ctx->d));
@@ -905,7 +999,8 @@ void bted_destroy(bted_ctx* ctx) {
         ctx->ted.release();
         ctx->bted_engine.release();
         void* bufs[] = {ctx->skeys, ctx->skeys2, ctx->sidx, ctx->sidx2, ctx->Xb, ctx->winners, ctx->u32a,
-                        ctx->u32b, ctx->count_dev, ctx->mkeys, ctx->cub_tmp, ctx->out_dev};
+                        ctx->u32b, ctx->count_dev, ctx->mkeys, ctx->cub_tmp, ctx->out_dev, ctx->sall,
+                        ctx->xall, ctx->kall};
         for (void* b : bufs) if (b) cudaFree(b);
         if (ctx->own_X && ctx->X) cudaFree(ctx->X);
         if (ctx->hkeys) cudaFreeHost(ctx->hkeys);

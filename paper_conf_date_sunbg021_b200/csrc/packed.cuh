@@ -221,32 +221,40 @@ gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamm
 // Alg. 1 l.3 from the partials: g_i = sum_J P[J][i] (J order), score =
 // g / (k(i,i) + mu) with the new diagonal read back from the diagonal tile,
 // masked (selected / the pivot / padding), packed key -> atomicMax(key_out).
-// One CTA of T threads per row block.
-__global__ void __launch_bounds__(T)
+// One CTA of kFinThreads per row block: the block's partials are staged in
+// smem by all threads (many loads in flight), then thread r < T sums row r
+// sequentially in J order.
+constexpr int kFinThreads = 512;
+constexpr int kFinChunk = 64;                 // J values staged per round (32 KiB)
+__global__ void __launch_bounds__(kFinThreads)
 finalize_packed_kernel(const float* __restrict__ P, int nT, int32_t N, const float* __restrict__ K, float mu,
                        const uint8_t* __restrict__ sel, const unsigned long long* __restrict__ keys, int32_t t,
                        unsigned long long* __restrict__ key_out, int* __restrict__ err) {
-    const int B = blockIdx.x, r = threadIdx.x;
+    __shared__ float stg[kFinChunk][T];
+    const int B = blockIdx.x, tid = threadIdx.x;
     const int64_t NP = (int64_t)nT * T;
-    const int i = B * T + r;
     const uint32_t s = t > 0 ? key_index(keys[t - 1]) : 0xFFFFFFFFu;
-    unsigned long long key = 0ull;
-    if (i < N) {
-        float g = 0.f;
-        int J = 0;
-        for (; J + 8 <= nT; J += 8) {
-            float v[8];
-#pragma unroll
-            for (int q = 0; q < 8; ++q) v[q] = P[(int64_t)(J + q) * NP + i];
-#pragma unroll
-            for (int q = 0; q < 8; ++q) g = __fadd_rn(g, v[q]);
+    float g = 0.f;
+    for (int J0 = 0; J0 < nT; J0 += kFinChunk) {
+        const int nj = min(kFinChunk, nT - J0);
+        __syncthreads();
+        for (int q = tid; q < nj * (T / 4); q += kFinThreads) {
+            const int jj = q / (T / 4), c4 = q % (T / 4);
+            *reinterpret_cast<float4*>(&stg[jj][4 * c4]) =
+                __ldcg(reinterpret_cast<const float4*>(P + (int64_t)(J0 + jj) * NP + (int64_t)B * T) + c4);
         }
-        for (; J < nT; ++J) g = __fadd_rn(g, P[(int64_t)J * NP + i]);
-        const float diag = K[tile_offset(B, B, nT) * (T * T) + (int64_t)r * T + r];
+        __syncthreads();
+        if (tid < T)
+            for (int jj = 0; jj < nj; ++jj) g = __fadd_rn(g, stg[jj][tid]);
+    }
+    unsigned long long key = 0ull;
+    const int i = B * T + tid;
+    if (tid < T && i < N) {
+        const float diag = K[tile_offset(B, B, nT) * (T * T) + (int64_t)tid * T + tid];
         const bool masked = sel[i] != 0 || (uint32_t)i == s;
         key = score_key(g, diag, mu, (uint32_t)i, masked, err);
     }
-    cta_key_max_to<T>(key, key_out);
+    cta_key_max_to<kFinThreads>(key, key_out);
 }
 
 // ------------------------------------------------------------------ K2p: TMA deflate

@@ -1,0 +1,154 @@
+// small.cuh -- whole-TED-in-one-kernel for small candidate sets (SURVEY.md
+// Sec. 8(f) N3: the paper's own workload, M = 500 points per batch, B = 10,
+// m = 64, and the |X_U| <= B m point merge TED of Alg. 2 l.6, PAPER.md:156,
+// 372-374).  At these sizes a per-step kernel launch costs more than the
+// step, so one thread-block CLUSTER runs all m steps of one TED with K held
+// in the cluster's distributed shared memory:
+//
+//   CTA r of a cluster of C owns rows [r*R, r*R+R) of K (dense, ld = N
+//   rounded to 4) in its own smem.  Per step: every CTA copies the pivot row
+//   from its owner's smem (DSMEM), cluster barrier, deflates its rows
+//   (k - (a_i p_j)/c with the same instruction as K2 -> bitwise the same
+//   elements), computes the new row norms, scores and its masked argmax
+//   key, writes the key into every CTA's slot (DSMEM), cluster barrier,
+//   each CTA reduces the C keys -> next pivot.  2 cluster barriers per step.
+//
+// Several TEDs (the B batches) run as independent clusters of one launch.
+#pragma once
+#include <cstdint>
+#include <cooperative_groups.h>
+#include <cuda_runtime.h>
+#include "kernels.cuh"
+
+namespace bted {
+namespace sm {
+
+namespace cg = cooperative_groups;
+constexpr int kThreads = 512;
+constexpr int kWarps = kThreads / 32;
+constexpr size_t kSmemBudget = 220 * 1024;
+
+__host__ __device__ __forceinline__ int ldk_for(int N) { return (N + 3) / 4 * 4; }
+__host__ __device__ __forceinline__ int rows_per(int N, int C) { return (N + C - 1) / C; }
+// dynamic smem of one CTA: band + pivot row + key slots + warp keys + sel
+__host__ __device__ __forceinline__ size_t smem_bytes(int N, int C) {
+    const size_t R = (size_t)rows_per(N, C), L = (size_t)ldk_for(N);
+    return (R * L + L) * sizeof(float) + (2 * 16 + kWarps) * sizeof(unsigned long long) + ((R + 15) / 16) * 16;
+}
+
+template <int C>
+__global__ void __launch_bounds__(kThreads, 1)
+ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float gamma, int32_t linear,
+                   int32_t m, float mu, unsigned long long* __restrict__ keys_all, int* __restrict__ err) {
+    cg::cluster_group cl = cg::this_cluster();
+    const int rank = (int)cl.block_rank();
+    const int inst = blockIdx.x / C;
+    const float* __restrict__ X = Xall + (int64_t)inst * N * d;
+    unsigned long long* keys_out = keys_all + (int64_t)inst * m;
+
+    extern __shared__ __align__(16) unsigned char smem[];
+    const int R = rows_per(N, C), L = ldk_for(N);
+    float* Kb = reinterpret_cast<float*>(smem);                 // [R][L]
+    float* piv = Kb + (size_t)R * L;                            // [L]
+    unsigned long long* kslot = reinterpret_cast<unsigned long long*>(piv + L);   // [2][16]
+    unsigned long long* wred = kslot + 32;                      // [kWarps]
+    uint8_t* sel = reinterpret_cast<uint8_t*>(wred + kWarps);   // [R]
+
+    const int tid = threadIdx.x, w = tid / 32, l = tid % 32;
+    const int r0 = rank * R;
+    const int nr = max(0, min(R, N - r0));
+    const float ng = -gamma;
+
+    // ---------------- l.1: this CTA's rows of K_VV, plus the first l.3
+    for (int q = tid; q < R; q += kThreads) sel[q] = 0;
+    unsigned long long best_local = 0ull;
+    for (int lr = w; lr < nr; lr += kWarps) {
+        const int i = r0 + lr;
+        float* row = Kb + (size_t)lr * L;
+        float acc_norm = 0.f;
+        for (int j = l; j < L; j += 32) {
+            float v = 0.f;
+            if (j < N) {
+                float a = 0.f;
+                for (int k = 0; k < d; ++k) {
+                    const float xi = X[(int64_t)i * d + k], xj = X[(int64_t)j * d + k];
+                    if (linear) a = __fmaf_rn(xi, xj, a);
+                    else { const float df = __fsub_rn(xi, xj); a = __fmaf_rn(df, df, a); }
+                }
+                v = linear ? a : expf(__fmul_rn(ng, a));
+            }
+            row[j] = v;
+            acc_norm = __fmaf_rn(v, v, acc_norm);
+        }
+        const float g = warp_sum(acc_norm);
+        if (l == 0) {
+            const unsigned long long k = score_key(g, row[i], mu, (uint32_t)i, false, err);
+            best_local = k > best_local ? k : best_local;
+        }
+    }
+    // CTA max -> every CTA's slot[0][rank] -> cluster max
+    auto exchange = [&](unsigned long long key, int parity) -> unsigned long long {
+        key = warp_max_u64(key);
+        if (l == 0) wred[w] = key;
+        __syncthreads();
+        if (tid == 0) {
+            unsigned long long v = 0ull;
+            for (int q = 0; q < kWarps; ++q) v = wred[q] > v ? wred[q] : v;
+            for (int r = 0; r < C; ++r) {
+                unsigned long long* dst = cl.map_shared_rank(kslot, r);
+                dst[parity * 16 + rank] = v;
+            }
+        }
+        cl.sync();
+        unsigned long long b = 0ull;
+        for (int r = 0; r < C; ++r) b = kslot[parity * 16 + r] > b ? kslot[parity * 16 + r] : b;
+        return b;
+    };
+    unsigned long long best = exchange(best_local, 0);
+
+    for (int t = 1; t < m; ++t) {
+        if (rank == 0 && tid == 0) keys_out[t - 1] = best;
+        const int s = (int)key_index(best);
+        if (best == 0ull) { if (tid == 0) atomicOr(err, 2); break; }
+        // pivot row K[s][:] from its owner's shared memory
+        const int owner = s / R;
+        const float* src = cl.map_shared_rank(Kb, owner) + (size_t)(s - owner * R) * L;
+        for (int j4 = tid; j4 < L / 4; j4 += kThreads)
+            reinterpret_cast<float4*>(piv)[j4] = reinterpret_cast<const float4*>(src)[j4];
+        if (owner == rank && tid == 0) sel[s - r0] = 1;
+        cl.sync();                                   // every CTA holds the pivot before rows change
+        const float inv_c = __frcp_rn(__fadd_rn(piv[s], mu));
+        best_local = 0ull;
+        for (int lr = w; lr < nr; lr += kWarps) {
+            const int i = r0 + lr;
+            float* row = Kb + (size_t)lr * L;
+            const float a = piv[i];                  // K[i][s] = K[s][i]
+            float acc_norm = 0.f;
+            for (int j4 = l; j4 < L / 4; j4 += 32) {
+                float4 kv = reinterpret_cast<float4*>(row)[j4];
+                const float4 pv = reinterpret_cast<const float4*>(piv)[j4];
+                kv.x = deflate1(kv.x, a, pv.x, inv_c);
+                kv.y = deflate1(kv.y, a, pv.y, inv_c);
+                kv.z = deflate1(kv.z, a, pv.z, inv_c);
+                kv.w = deflate1(kv.w, a, pv.w, inv_c);
+                reinterpret_cast<float4*>(row)[j4] = kv;
+                acc_norm = __fmaf_rn(kv.x, kv.x, acc_norm);
+                acc_norm = __fmaf_rn(kv.y, kv.y, acc_norm);
+                acc_norm = __fmaf_rn(kv.z, kv.z, acc_norm);
+                acc_norm = __fmaf_rn(kv.w, kv.w, acc_norm);
+            }
+            const float g = warp_sum(acc_norm);
+            if (l == 0) {
+                const bool masked = sel[lr] != 0 || i == s;
+                const unsigned long long k = score_key(g, row[i], mu, (uint32_t)i, masked, err);
+                best_local = k > best_local ? k : best_local;
+            }
+        }
+        best = exchange(best_local, t & 1);
+    }
+    if (rank == 0 && tid == 0) keys_out[m - 1] = best;
+    cl.sync();                                       // no CTA exits while others may read its smem
+}
+
+}  // namespace sm
+}  // namespace bted

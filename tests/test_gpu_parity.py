@@ -13,6 +13,12 @@ from tests.parity import check_ted, ulp32
 
 pytestmark = pytest.mark.gpu
 MU = float(np.float32(0.1))
+# engine paths: packed tiles (N4), dense rows, and "auto" (the one-kernel
+# cluster TED of small.cuh for N <= ~940, packed above)
+PACKED = L.BTED_FLAG_NO_SMALL
+DENSE = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_DENSE
+LAYOUTS = pytest.mark.parametrize("flags", [PACKED, DENSE, 0], ids=["packed", "dense", "auto"])
+LAYOUTS_K = pytest.mark.parametrize("flags", [PACKED, DENSE], ids=["packed", "dense"])   # tests reading K back
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -31,7 +37,7 @@ def ld_of(N):
 
 # ------------------------------------------------------------------ K1 Gram
 @pytest.mark.parametrize("N,pool", [(1000, "knob"), (777, "uniform"), (64, "knob")])
-@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+@LAYOUTS_K
 def test_gram_entries_bitsymmetric_and_within_ulp_bound(N, pool, flags):
     X = knob(N) if pool == "knob" else uniform_pool(N, 16, 4)
     g = median_gamma(X, 1)
@@ -53,7 +59,7 @@ def test_gram_entries_bitsymmetric_and_within_ulp_bound(N, pool, flags):
 
 
 # ------------------------------------------------------------------ K2 step
-@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+@LAYOUTS_K
 def test_one_deflation_step_vs_fp64_and_selected_column(flags):
     N = 1200
     X = knob(N, seed=9)
@@ -91,7 +97,7 @@ def _ted_parity(X, g, m, label, use_dense=True, flags=0):
     return near
 
 
-@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+@LAYOUTS
 def test_ted_parity_toy_config(flags):
     X, g, cfg = config_pool("toy")
     _ted_parity(X, g, cfg["m"], "toy", use_dense=False, flags=flags)
@@ -99,7 +105,7 @@ def test_ted_parity_toy_config(flags):
 
 @pytest.mark.parametrize("N,pool,m", [(257, "knob", 64), (1000, "uniform", 64), (2049, "knob12", 48),
                                       (4096, "knob", 64), (4096, "uniform", 64)])
-@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+@LAYOUTS
 def test_ted_parity_multi_tile_ragged(N, pool, m, flags):
     if pool == "knob":
         X = knob(N, seed=N)
@@ -111,7 +117,7 @@ def test_ted_parity_multi_tile_ragged(N, pool, m, flags):
     _ted_parity(X, g, m, f"{pool}-{N}", flags=flags)
 
 
-@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+@LAYOUTS
 def test_ted_parity_bench_size_resnet18_batch(flags):
     """The bench workload (resnet18 config: one batch of N = 16384 from the
     2^20-row pool, m = 64), checked at every step against the dense C oracle."""
@@ -130,7 +136,7 @@ def test_ted_parity_bench_size_resnet18_batch(flags):
 
 
 # ------------------------------------------------------------------ edge cases
-@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+@LAYOUTS
 def test_single_point_and_full_permutation(flags):
     X = knob(1)
     with bt.CandidateSet(X, 1.0, flags=flags) as cs:
@@ -144,7 +150,7 @@ def test_single_point_and_full_permutation(flags):
     assert sorted(idx.tolist()) == list(range(100))          # C7: m = N is a permutation
 
 
-@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+@LAYOUTS
 def test_identity_kernel_ties_lowest_index(flags):
     X = (np.arange(40, dtype=np.float32) * 100.0)[:, None]  # K = I exactly in fp32
     with bt.CandidateSet(X, 1.0, flags=flags) as cs:
@@ -153,7 +159,7 @@ def test_identity_kernel_ties_lowest_index(flags):
     assert np.all(sc == np.float32(1.0) / np.float32(np.float32(1.0) + np.float32(MU)))
 
 
-@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+@LAYOUTS
 def test_exact_duplicates_tie_to_lowest_index(flags):
     X = knob(300, seed=2)
     X = np.concatenate([X, X[:50]], axis=0)                  # rows 300..349 duplicate rows 0..49
@@ -166,7 +172,7 @@ def test_exact_duplicates_tie_to_lowest_index(flags):
     check_ted(idx, sc, tr, "dups")
 
 
-@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+@LAYOUTS_K
 def test_linear_kernel_closed_form_c8(flags):
     rng = np.random.default_rng(8)
     X = (rng.standard_normal((300, 6)) * 0.5).astype(np.float32)
@@ -211,7 +217,7 @@ def _positions(V, pool_idx):
     return pos
 
 
-@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+@LAYOUTS
 def test_bted_parity_vs_oracle(flags):
     P, M, B, m, seed = 60000, 2048, 4, 32, 3
     space = KnobSpace(WORKLOADS["vgg16_conv1_1"], 16)
@@ -232,7 +238,7 @@ def test_bted_parity_vs_oracle(flags):
     check_ted(mpos, [], trm, "merge")
 
 
-@pytest.mark.parametrize("flags", [0, L.BTED_FLAG_DENSE], ids=["packed", "dense"])
+@LAYOUTS
 def test_round_robin_batches_then_merge_equals_run_batches(flags):
     P, M, B, m, seed = 30000, 1024, 5, 16, 11
     X = knob(P, seed=4)
@@ -263,7 +269,7 @@ def test_row_sharded_loopback_bit_identical(N, P):
     from paper_conf_date_sunbg021_b200.dist import sharded_select_loopback
     X = knob(N, seed=N + P)
     g = median_gamma(X, P)
-    with bt.CandidateSet(X, g, flags=L.BTED_FLAG_DENSE) as cs:     # shards are dense
+    with bt.CandidateSet(X, g, flags=DENSE) as cs:     # shards are dense
         idx, sc = cs.select(24, MU)
     dev = torch.device("cuda", 0)
     st = torch.cuda.Stream(dev)
@@ -275,13 +281,17 @@ def test_row_sharded_loopback_bit_identical(N, P):
 def test_launch_counter_counts_kernels():
     X = knob(300)
     before = bt.bted_kernel_launches()
-    with bt.CandidateSet(X, 0.3, flags=L.BTED_FLAG_DENSE) as cs:
+    with bt.CandidateSet(X, 0.3, flags=DENSE) as cs:
         cs.select(10, MU)
     assert bt.bted_kernel_launches() - before == 11          # transpose + K1 + 9 x K2
     before = bt.bted_kernel_launches()
-    with bt.CandidateSet(X, 0.3) as cs:
+    with bt.CandidateSet(X, 0.3, flags=PACKED) as cs:
         cs.select(10, MU)
     assert bt.bted_kernel_launches() - before == 20          # K1p + fin + 9 x (K2p + fin)
+    before = bt.bted_kernel_launches()
+    with bt.CandidateSet(X, 0.3) as cs:
+        cs.select(10, MU)
+    assert bt.bted_kernel_launches() - before == 1           # the whole TED in one cluster kernel
 
 
 # ------------------------------------------------------------------ packed vs dense layout
@@ -291,7 +301,7 @@ def test_packed_layout_matches_dense(N, d, m):
     the dense layout; only the norm summation order differs."""
     X = knob(N, d=16, seed=N)[:, :d] if d <= 16 else uniform_pool(N, d, N)
     g = median_gamma(X, d)
-    with bt.CandidateSet(X, g, flags=L.BTED_FLAG_DENSE) as cd, bt.CandidateSet(X, g) as cp:
+    with bt.CandidateSet(X, g, flags=DENSE) as cd, bt.CandidateSet(X, g, flags=PACKED) as cp:
         i_d, s_d = cd.select(m, MU)
         i_p, s_p = cp.select(m, MU)
         tr = dense.ted(X, g, MU, m, forced=i_p)
@@ -304,3 +314,37 @@ def test_packed_layout_matches_dense(N, d, m):
         else:                                                  # only legitimate near-ties may differ
             k = int(np.argmax(i_d != i_p))
             assert tr.gap[k] <= 1e-5
+
+
+# ------------------------------------------------------------------ paper-scale (N3) and the cluster TED
+def test_paper_scale_bted_vs_oracle():
+    """The paper's own BTED workload: B = 10 batches of M = 500
+    points, m = 64, union of <= 640 points; batch TEDs and the merge run as
+    cluster kernels (small.cuh)."""
+    X, g, cfg = config_pool("paper")
+    B, M, m = cfg["B"], cfg["M"], cfg["m"]
+    with bt.CandidateSet(X, g, num_batches=B, seed=cfg["seed"]) as pool:
+        before = bt.bted_kernel_launches()
+        sel, bidx = pool.run_batches(M, m, MU)
+        launched = bt.bted_kernel_launches() - before
+    batches = oracle_sample_batches(X.shape[0], M, B, cfg["seed"])
+    for b in range(B):
+        pos = _positions(batches[b], bidx[b])
+        check_ted(pos, [], literal.ted(X[batches[b]], g, MU, m, forced=pos), f"paper-batch{b}")
+    XU = np.unique(bidx)
+    assert len(XU) == len(set(bidx.ravel().tolist()))
+    mpos = _positions(XU, sel)
+    check_ted(mpos, [], literal.ted(X[XU], g, MU, len(sel), forced=mpos), "paper-merge")
+    # one cluster launch for all 10 batch TEDs + one for the merge (+ sampling/gather/union kernels)
+    assert launched < 60
+
+
+@pytest.mark.parametrize("N", [1, 5, 64, 230, 231, 500, 640, 777, 940])
+def test_cluster_ted_matches_oracle_across_cluster_sizes(N):
+    X = knob(N, seed=N + 7)
+    g = median_gamma(X, N) if N > 1 else 1.0
+    m = min(N, 48)
+    with bt.CandidateSet(X, g) as cs:
+        idx, sc = cs.select(m, MU)
+    tr = literal.ted(X, g, MU, m, forced=idx)
+    check_ted(idx, sc, tr, f"cluster-{N}")
