@@ -87,6 +87,35 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
         "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
         :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
 }
+// same, with an L2 eviction-priority policy (createpolicy) for streamed data
+__device__ __forceinline__ void bulk_g2s_hint(void* dst, const void* src, uint32_t bytes, uint64_t* bar,
+                                              uint64_t policy) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+        :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(policy) : "memory");
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ float ld_hint(const float* p, uint64_t policy) {
+    float v;
+    asm volatile("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(policy));
+    return v;
+}
+__device__ __forceinline__ float4 ld4_hint(const float* p, uint64_t policy) {
+    float4 v;
+    asm volatile("ld.global.nc.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(policy));
+    return v;
+}
+
 __device__ __forceinline__ void consumer_sync() {       // named barrier 1: the 256 consumer threads
     asm volatile("bar.sync 1, %0;" :: "n"(kConsumers) : "memory");
 }
@@ -226,31 +255,46 @@ gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamm
 // sequentially in J order.
 constexpr int kFinThreads = 512;
 constexpr int kFinChunk = 64;                 // J values staged per round (32 KiB)
+constexpr int kFinSplit = 4;                  // 4 threads per row: J ranges combined in a fixed order
 __global__ void __launch_bounds__(kFinThreads)
 finalize_packed_kernel(const float* __restrict__ P, int nT, int32_t N, const float* __restrict__ K, float mu,
                        const uint8_t* __restrict__ sel, const unsigned long long* __restrict__ keys, int32_t t,
                        unsigned long long* __restrict__ key_out, int* __restrict__ err) {
     __shared__ float stg[kFinChunk][T];
+    __shared__ float part[kFinSplit][T];
     const int B = blockIdx.x, tid = threadIdx.x;
+    const int r = tid % T, q = tid / T;          // row r, quarter q of each chunk
     const int64_t NP = (int64_t)nT * T;
     const uint32_t s = t > 0 ? key_index(keys[t - 1]) : 0xFFFFFFFFu;
     float g = 0.f;
+    // g(row) = sum over chunks c of ( sum_{q} ( sequential sum of chunk c, quarter q ) )
     for (int J0 = 0; J0 < nT; J0 += kFinChunk) {
         const int nj = min(kFinChunk, nT - J0);
         __syncthreads();
-        for (int q = tid; q < nj * (T / 4); q += kFinThreads) {
-            const int jj = q / (T / 4), c4 = q % (T / 4);
+        for (int e = tid; e < nj * (T / 4); e += kFinThreads) {
+            const int jj = e / (T / 4), c4 = e % (T / 4);
             *reinterpret_cast<float4*>(&stg[jj][4 * c4]) =
                 __ldcg(reinterpret_cast<const float4*>(P + (int64_t)(J0 + jj) * NP + (int64_t)B * T) + c4);
         }
         __syncthreads();
-        if (tid < T)
-            for (int jj = 0; jj < nj; ++jj) g = __fadd_rn(g, stg[jj][tid]);
+        const int per = (nj + kFinSplit - 1) / kFinSplit;
+        const int j0 = q * per, j1 = min(nj, j0 + per);
+        float h = 0.f;
+#pragma unroll 8
+        for (int jj = j0; jj < j1; ++jj) h = __fadd_rn(h, stg[jj][r]);
+        part[q][r] = h;
+        __syncthreads();
+        if (q == 0) {
+            float c = part[0][r];
+#pragma unroll
+            for (int qq = 1; qq < kFinSplit; ++qq) c = __fadd_rn(c, part[qq][r]);
+            g = __fadd_rn(g, c);
+        }
     }
     unsigned long long key = 0ull;
-    const int i = B * T + tid;
-    if (tid < T && i < N) {
-        const float diag = K[tile_offset(B, B, nT) * (T * T) + (int64_t)tid * T + tid];
+    const int i = B * T + r;
+    if (q == 0 && i < N) {
+        const float diag = K[tile_offset(B, B, nT) * (T * T) + (int64_t)r * T + r];
         const bool masked = sel[i] != 0 || (uint32_t)i == s;
         key = score_key(g, diag, mu, (uint32_t)i, masked, err);
     }
@@ -279,6 +323,7 @@ deflate_packed_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, i
     if (tid >= kConsumers) {
         // ---------------- producer warp: one elected lane streams the tiles
         if (tid == kConsumers) {
+            const uint64_t pol = policy_evict_first();    // K streams through L2 once per step
             int n = 0;
             for (int64_t k = blockIdx.x; k < ntiles; k += gridDim.x, ++n) {
                 const int st = n % kStages;
@@ -289,7 +334,7 @@ deflate_packed_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, i
                 float* dst = stage + st * (T * T);
 #pragma unroll
                 for (int q = 0; q < 4; ++q)
-                    bulk_g2s(dst + q * (T * T / 4), src + q * (T * T / 4), kTileBytes / 4, full + st);
+                    bulk_g2s_hint(dst + q * (T * T / 4), src + q * (T * T / 4), kTileBytes / 4, full + st, pol);
             }
         }
         return;
@@ -303,11 +348,26 @@ deflate_packed_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, i
     const float inv_c = __frcp_rn(__fadd_rn(Kin[packed_index((int)s, (int)s, nT)], mu));   // 1/(k(s,s)+mu)
     if (blockIdx.x == 0 && tid == 0 && (int32_t)s < N) sel[s] = 1;
     // K_in[s, B*T + c]: a contiguous row segment of tile (S,B) if S <= B, else a
-    // column of tile (B,S)
+    // column of tile (B,S).  Read with an evict-last policy (reused by every
+    // tile of block B) and prefetched one tile ahead.
+    const uint64_t keep = policy_evict_last();
     auto seg = [&](int B, int c) -> float {
-        return S <= B ? Kin[tile_offset(S, B, nT) * (T * T) + (int64_t)rs * T + c]
-                      : Kin[tile_offset(B, S, nT) * (T * T) + (int64_t)c * T + rs];
+        return S <= B ? ld_hint(Kin + tile_offset(S, B, nT) * (T * T) + (int64_t)rs * T + c, keep)
+                      : ld_hint(Kin + tile_offset(B, S, nT) * (T * T) + (int64_t)c * T + rs, keep);
     };
+    auto load_segs = [&](int64_t k, float& pr, float4& pc) {
+        int I, J;
+        tile_ij(k, nT, I, J);
+        pr = l < 16 ? seg(I, 16 * w + l) : 0.f;        // a_i for the warp's 16 rows
+        if (S <= J) {
+            pc = ld4_hint(Kin + tile_offset(S, J, nT) * (T * T) + (int64_t)rs * T + 4 * l, keep);
+        } else {
+            pc.x = seg(J, 4 * l); pc.y = seg(J, 4 * l + 1); pc.z = seg(J, 4 * l + 2); pc.w = seg(J, 4 * l + 3);
+        }
+    };
+    float pr_next = 0.f;
+    float4 pc_next = make_float4(0.f, 0.f, 0.f, 0.f);
+    if ((int64_t)blockIdx.x < ntiles) load_segs(blockIdx.x, pr_next, pc_next);
     int n = 0;
     for (int64_t k = blockIdx.x; k < ntiles; k += gridDim.x, ++n) {
         int I, J;
@@ -315,14 +375,9 @@ deflate_packed_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, i
         const int st = n % kStages;
         const uint32_t ph = (uint32_t)(n / kStages) & 1u;
         float (*cg)[T] = colg[n & 1];
-        // pivot segments: a_i for the warp's 16 rows (lane < 16), p_j for the lane's 4 columns
-        const float pr_l = l < 16 ? seg(I, 16 * w + l) : 0.f;
-        float4 pc;
-        if (S <= J) {
-            pc = *reinterpret_cast<const float4*>(Kin + tile_offset(S, J, nT) * (T * T) + (int64_t)rs * T + 4 * l);
-        } else {
-            pc.x = seg(J, 4 * l); pc.y = seg(J, 4 * l + 1); pc.z = seg(J, 4 * l + 2); pc.w = seg(J, 4 * l + 3);
-        }
+        const float pr_l = pr_next;
+        const float4 pc = pc_next;
+        if (k + gridDim.x < ntiles) load_segs(k + gridDim.x, pr_next, pc_next);   // next tile's segments
         mbar_wait(full + st, ph);
         const float* sm = stage + st * (T * T);
         float* gout = Kout + k * (int64_t)(T * T);

@@ -7,6 +7,7 @@ OUT=gpurun_out/$TAG
 mkdir -p $OUT
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > $OUT/nvsmi.txt 2>&1
 timeout 1200 python -m pytest tests -m gpu -q $PYARGS > $OUT/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> $OUT/pytest_gpu.log
+timeout 120 python scripts/h2d_probe.py > $OUT/h2d.txt 2>&1
 timeout 300 python __graft_entry__.py smoke > $OUT/smoke.log 2>&1; echo "smoke rc=$?" >> $OUT/smoke.log
 timeout 900 python bench.py --steps 10 --warmup 3 > $OUT/bench.json 2> $OUT/bench.err; echo "bench rc=$?" >> $OUT/bench.err
 timeout 900 python bench.py --steps 10 --warmup 3 --layout dense --no-cpu-baseline > $OUT/bench_dense.json 2> $OUT/bench_dense.err
@@ -14,7 +15,7 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
     python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_launches.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:deflate_packed -s 8 -c 1 \
     -o $OUT/prof_k2p python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_k2p.log 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:gram_packed -s 4 -c 1 \
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:gram_packed -s 2 -c 1 \
     -o $OUT/prof_k1p python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_k1p.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:deflate_rescore -s 8 -c 1 \
     -o $OUT/prof_k2 python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e --layout dense > $OUT/ncu_k2.log 2>&1

@@ -1,6 +1,7 @@
 """Host->device copy rates: torch pinned copy vs the library's bted_update
 (from torch-pinned memory and from pageable numpy memory)."""
-import time
+import os, sys, time
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np
 import torch
 import paper_conf_date_sunbg021_b200 as bt
