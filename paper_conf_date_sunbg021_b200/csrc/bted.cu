@@ -236,9 +236,11 @@ int num_sms() {
     }
     return g_num_sms;
 }
-constexpr size_t kK2pSmem = (size_t)bted::pk::kStages * bted::pk::kTileBytes +
-                            2 * (size_t)bted::pk::kGroups * bted::pk::T * sizeof(float) +
-                            2 * bted::pk::kStages * sizeof(uint64_t);
+// production K2p configuration (scripts/k2p_variants.cu)
+constexpr int kK2pSub = 64;
+constexpr bool kK2pHints = false;
+#define K2P_KERNEL bted::pk::deflate_packed_kernel<kK2pSub, kK2pHints>
+constexpr size_t kK2pSmem = bted::pk::k2p_smem_bytes(kK2pSub);
 
 // Alg. 1 l.1 + first l.3 on the packed tiles.  (2 kernels: K1p, fin)
 void enqueue_head_packed(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m,
@@ -268,7 +270,7 @@ void enqueue_loop_packed(Ted& T, int64_t N, int32_t m, float mu, unsigned long l
     for (int32_t t = 1; t < m; ++t) {
         const float* Kin = T.K[(t - 1) & 1];
         float* Kout = T.K[t & 1];
-        bted::pk::deflate_packed_kernel<<<grid, bted::pk::kConsumers + 32, kK2pSmem, T.stream>>>(
+        K2P_KERNEL<<<grid, bted::pk::kConsumers + 32, kK2pSmem, T.stream>>>(
             Kin, Kout, nT, (int32_t)N, T.P, keys, t, mu, T.sel);
         bted::pk::finalize_packed_kernel<<<nT, bted::pk::kFinThreads, 0, T.stream>>>(T.P, nT, (int32_t)N, Kout, mu, T.sel,
                                                                            keys, t, keys + t, T.err);
@@ -328,7 +330,7 @@ void graph_run(Ted& T, const GraphKey& key, uint64_t nkernels, F&& enqueue) {
 void ensure_packed_attrs() {
     static bool done = false;
     if (!done) {
-        CK(cudaFuncSetAttribute(bted::pk::deflate_packed_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        CK(cudaFuncSetAttribute(K2P_KERNEL, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)kK2pSmem));
         done = true;
     }

@@ -34,7 +34,6 @@ namespace pk {
 
 constexpr int T = 128;                 // tile edge
 constexpr int kConsumers = 256;        // 8 consumer warps
-constexpr int kStages = 3;
 constexpr int kTileBytes = T * T * 4;  // 64 KiB
 constexpr int kGroups = T / 4;         // 32 groups of 4 rows per tile
 
@@ -302,39 +301,54 @@ finalize_packed_kernel(const float* __restrict__ P, int nT, int32_t N, const flo
 }
 
 // ------------------------------------------------------------------ K2p: TMA deflate
+// kSub rows of a tile per pipeline stage (kSub x 128 fp32), kStagesOf(kSub)
+// stages in a ~192 KiB ring.  kHints: evict-first policy on the streamed
+// tiles and evict-last on the pivot segments (reused by every tile of a
+// block row/column), pivot segments prefetched one tile ahead.
+__host__ __device__ constexpr int kStagesOf(int sub) { return (192 * 1024) / (sub * T * 4); }
+__host__ __device__ constexpr size_t k2p_smem_bytes(int sub) {
+    return (size_t)kStagesOf(sub) * sub * T * 4 + 2 * (size_t)kGroups * T * 4 + 2 * kStagesOf(sub) * 8;
+}
+
+template <int kSub, bool kHints>
 __global__ void __launch_bounds__(kConsumers + kWarp, 1)
 deflate_packed_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, int nT, int32_t N,
                       float* __restrict__ P, const unsigned long long* __restrict__ keys, int32_t t, float mu,
                       uint8_t* __restrict__ sel) {
+    constexpr int kS = kStagesOf(kSub);
+    constexpr int kStageFloats = kSub * T;
+    constexpr int kSubs = T / kSub;             // stages per tile
+    constexpr int kRW = kSub / 8;               // rows per warp per stage
     extern __shared__ __align__(1024) unsigned char smem_raw[];
-    float* stage = reinterpret_cast<float*>(smem_raw);                       // [kStages][T*T]
-    float (*colg)[kGroups][T] = reinterpret_cast<float (*)[kGroups][T]>(smem_raw + kStages * kTileBytes);  // [2]
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + kStages * kTileBytes + 2 * kGroups * T * 4);
-    uint64_t* empty = full + kStages;
+    float* stage = reinterpret_cast<float*>(smem_raw);                       // [kS][kSub*T]
+    float (*colg)[kGroups][T] = reinterpret_cast<float (*)[kGroups][T]>(smem_raw + (size_t)kS * kStageFloats * 4);
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + (size_t)kS * kStageFloats * 4 + 2 * kGroups * T * 4);
+    uint64_t* empty = full + kS;
 
     const int tid = threadIdx.x;
     const int64_t ntiles = num_tiles(nT);
     if (tid == 0) {
-        for (int q = 0; q < kStages; ++q) { mbar_init(full + q, 1); mbar_init(empty + q, kConsumers / kWarp); }
+        for (int q = 0; q < kS; ++q) { mbar_init(full + q, 1); mbar_init(empty + q, kConsumers / kWarp); }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
 
     if (tid >= kConsumers) {
-        // ---------------- producer warp: one elected lane streams the tiles
+        // ---------------- producer warp: one elected lane streams the tiles, kSub rows per stage
         if (tid == kConsumers) {
             const uint64_t pol = policy_evict_first();    // K streams through L2 once per step
             int n = 0;
-            for (int64_t k = blockIdx.x; k < ntiles; k += gridDim.x, ++n) {
-                const int st = n % kStages;
-                const uint32_t ph = (uint32_t)(n / kStages) & 1u;
-                mbar_wait(empty + st, ph ^ 1u);
-                mbar_expect_tx(full + st, kTileBytes);
+            for (int64_t k = blockIdx.x; k < ntiles; k += gridDim.x) {
                 const float* src = Kin + k * (int64_t)(T * T);
-                float* dst = stage + st * (T * T);
-#pragma unroll
-                for (int q = 0; q < 4; ++q)
-                    bulk_g2s_hint(dst + q * (T * T / 4), src + q * (T * T / 4), kTileBytes / 4, full + st, pol);
+                for (int sb = 0; sb < kSubs; ++sb, ++n) {
+                    const int st = n % kS;
+                    const uint32_t ph = (uint32_t)(n / kS) & 1u;
+                    mbar_wait(empty + st, ph ^ 1u);
+                    mbar_expect_tx(full + st, kStageFloats * 4);
+                    if (kHints) bulk_g2s_hint(stage + st * kStageFloats, src + sb * kStageFloats, kStageFloats * 4,
+                                              full + st, pol);
+                    else bulk_g2s(stage + st * kStageFloats, src + sb * kStageFloats, kStageFloats * 4, full + st);
+                }
             }
         }
         return;
@@ -347,20 +361,22 @@ deflate_packed_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, i
     const int S = (int)(s / T), rs = (int)(s % T);
     const float inv_c = __frcp_rn(__fadd_rn(Kin[packed_index((int)s, (int)s, nT)], mu));   // 1/(k(s,s)+mu)
     if (blockIdx.x == 0 && tid == 0 && (int32_t)s < N) sel[s] = 1;
-    // K_in[s, B*T + c]: a contiguous row segment of tile (S,B) if S <= B, else a
-    // column of tile (B,S).  Read with an evict-last policy (reused by every
-    // tile of block B) and prefetched one tile ahead.
-    const uint64_t keep = policy_evict_last();
+    // K_in[s, B*T + c]: a contiguous row segment of tile (S,B) if S <= B, else a column of tile (B,S)
+    const uint64_t keep = kHints ? policy_evict_last() : 0ull;
+    auto ldf = [&](const float* p) -> float { return kHints ? ld_hint(p, keep) : __ldg(p); };
     auto seg = [&](int B, int c) -> float {
-        return S <= B ? ld_hint(Kin + tile_offset(S, B, nT) * (T * T) + (int64_t)rs * T + c, keep)
-                      : ld_hint(Kin + tile_offset(B, S, nT) * (T * T) + (int64_t)c * T + rs, keep);
+        return S <= B ? ldf(Kin + tile_offset(S, B, nT) * (T * T) + (int64_t)rs * T + c)
+                      : ldf(Kin + tile_offset(B, S, nT) * (T * T) + (int64_t)c * T + rs);
     };
+    // the warp's 16 rows of a tile: row(l) for l < 16
+    auto my_row = [&](int q) { return (q / kRW) * kSub + w * kRW + (q % kRW); };
     auto load_segs = [&](int64_t k, float& pr, float4& pc) {
         int I, J;
         tile_ij(k, nT, I, J);
-        pr = l < 16 ? seg(I, 16 * w + l) : 0.f;        // a_i for the warp's 16 rows
+        pr = l < 16 ? seg(I, my_row(l)) : 0.f;                 // a_i for the warp's 16 rows
         if (S <= J) {
-            pc = ld4_hint(Kin + tile_offset(S, J, nT) * (T * T) + (int64_t)rs * T + 4 * l, keep);
+            const float* p = Kin + tile_offset(S, J, nT) * (T * T) + (int64_t)rs * T + 4 * l;
+            pc = kHints ? ld4_hint(p, keep) : __ldg(reinterpret_cast<const float4*>(p));
         } else {
             pc.x = seg(J, 4 * l); pc.y = seg(J, 4 * l + 1); pc.z = seg(J, 4 * l + 2); pc.w = seg(J, 4 * l + 3);
         }
@@ -368,38 +384,57 @@ deflate_packed_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, i
     float pr_next = 0.f;
     float4 pc_next = make_float4(0.f, 0.f, 0.f, 0.f);
     if ((int64_t)blockIdx.x < ntiles) load_segs(blockIdx.x, pr_next, pc_next);
-    int n = 0;
-    for (int64_t k = blockIdx.x; k < ntiles; k += gridDim.x, ++n) {
+    int n = 0, tcount = 0;
+    for (int64_t k = blockIdx.x; k < ntiles; k += gridDim.x, ++tcount) {
         int I, J;
         tile_ij(k, nT, I, J);
-        const int st = n % kStages;
-        const uint32_t ph = (uint32_t)(n / kStages) & 1u;
-        float (*cg)[T] = colg[n & 1];
+        float (*cg)[T] = colg[tcount & 1];
         const float pr_l = pr_next;
         const float4 pc = pc_next;
         if (k + gridDim.x < ntiles) load_segs(k + gridDim.x, pr_next, pc_next);   // next tile's segments
-        mbar_wait(full + st, ph);
-        const float* sm = stage + st * (T * T);
         float* gout = Kout + k * (int64_t)(T * T);
         RowWalk a;
         a.rowsum = 0.f;
-#pragma unroll 4
-        for (int rr = 0; rr < 16; ++rr) {
-            const int r = 16 * w + rr;
-            const float ai = __shfl_sync(0xffffffffu, pr_l, rr);
-            const float4 kv = *reinterpret_cast<const float4*>(sm + r * T + 4 * l);
-            float4 o;
-            o.x = deflate1(kv.x, ai, pc.x, inv_c);
-            o.y = deflate1(kv.y, ai, pc.y, inv_c);
-            o.z = deflate1(kv.z, ai, pc.z, inv_c);
-            o.w = deflate1(kv.w, ai, pc.w, inv_c);
-            st_stream(gout + r * T + 4 * l, o);
-            walk_row(a, rr, l, o, cg, w, I != J);
+        for (int sb = 0; sb < kSubs; ++sb, ++n) {
+            const int st = n % kS;
+            const uint32_t ph = (uint32_t)(n / kS) & 1u;
+            mbar_wait(full + st, ph);
+            const float* sm = stage + st * kStageFloats;
+#pragma unroll
+            for (int rr = 0; rr < kRW; ++rr) {
+                const int q = sb * kRW + rr;                       // the warp's q-th row of the tile
+                const int r = sb * kSub + w * kRW + rr;            // row within the tile
+                const float ai = __shfl_sync(0xffffffffu, pr_l, q);
+                const float4 kv = *reinterpret_cast<const float4*>(sm + (w * kRW + rr) * T + 4 * l);
+                float4 o;
+                o.x = deflate1(kv.x, ai, pc.x, inv_c);
+                o.y = deflate1(kv.y, ai, pc.y, inv_c);
+                o.z = deflate1(kv.z, ai, pc.z, inv_c);
+                o.w = deflate1(kv.w, ai, pc.w, inv_c);
+                st_stream(gout + r * T + 4 * l, o);
+                // partials: row sum via the canonical tree; column groups of 4 rows
+                float rp = group4(o.x, o.y, o.z, o.w);
+                rp = warp_sum(rp);
+                if (l == q) a.rowsum = rp;
+                if (I != J) {
+                    if ((r & 3) == 0) {
+                        a.cg[0] = __fmul_rn(o.x, o.x); a.cg[1] = __fmul_rn(o.y, o.y);
+                        a.cg[2] = __fmul_rn(o.z, o.z); a.cg[3] = __fmul_rn(o.w, o.w);
+                    } else {
+                        a.cg[0] = __fmaf_rn(o.x, o.x, a.cg[0]); a.cg[1] = __fmaf_rn(o.y, o.y, a.cg[1]);
+                        a.cg[2] = __fmaf_rn(o.z, o.z, a.cg[2]); a.cg[3] = __fmaf_rn(o.w, o.w, a.cg[3]);
+                    }
+                    if ((r & 3) == 3)
+                        *reinterpret_cast<float4*>(&cg[r >> 2][4 * l]) =
+                            make_float4(a.cg[0], a.cg[1], a.cg[2], a.cg[3]);
+                }
+            }
+            __syncwarp();
+            if (l == 0) mbar_arrive(empty + st);   // this warp is done reading the stage
         }
-        __syncwarp();
-        if (l == 0) mbar_arrive(empty + st);       // this warp is done reading the stage
         consumer_sync();                           // colg of this tile complete
-        write_partials(P, NP, I, J, w, l, a, cg, tid);
+        if (l < 16) P[(int64_t)J * NP + (int64_t)I * T + my_row(l)] = a.rowsum;
+        if (I != J && tid < T) P[(int64_t)I * NP + (int64_t)J * T + tid] = tree32_smem(&cg[0][tid], T);
     }
 }
 
