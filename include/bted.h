@@ -62,6 +62,9 @@ typedef enum {
                                    used when d <= 32).  Shard contexts are always dense. */
 #define BTED_FLAG_NO_SMALL 8u   /* never use the one-kernel cluster TED for small candidate sets
                                    (N <= ~940: K in distributed shared memory)               */
+#define BTED_FLAG_TMA     16u   /* packed layout: stream K through the persistent TMA ring
+                                   (cp.async.bulk + mbarrier) instead of the default one-CTA-per-
+                                   tile 256-bit-load kernel (which measured faster on B200)   */
 #define BTED_FLAG_TIMING   2u   /* record CUDA events around K1 and the K2 loop of every batch
                                    TED on the ctx stream; read with bted_get_stats()          */
 

@@ -114,6 +114,7 @@ struct Ted {
     // timing (BTED_FLAG_TIMING): events recorded on the stream around the
     // head and loop graphs of each TED, read back at the next host sync.
     bool timing = false;
+    bool tma = false;          // packed K2p: TMA-ring variant instead of the LDG one
     struct Slot { cudaEvent_t e[3]; int32_t m; };
     std::vector<Slot> slots;
     size_t used = 0;
@@ -236,10 +237,13 @@ int num_sms() {
     }
     return g_num_sms;
 }
-// production K2p configuration (scripts/k2p_variants.cu)
+// K2p configurations (scripts/k2p_variants.cu, profiles/r1/k2p_variants_*.txt):
+// default = one CTA per tile with 256-bit loads (k2p_ldg<4>, measured 6.40 /
+// 6.75 TB/s at N = 16384 / 32768, above cudaMemcpy D2D); BTED_FLAG_TMA = the
+// persistent TMA-ring pipeline (v8 stores, 64-row stages; 5.90 / 6.09 TB/s).
 constexpr int kK2pSub = 64;
-constexpr bool kK2pHints = false;
-#define K2P_KERNEL bted::pk::deflate_packed_kernel<kK2pSub, kK2pHints>
+#define K2P_TMA_KERNEL bted::pk::deflate_packed_v8_kernel<kK2pSub, false>
+#define K2P_LDG_KERNEL bted::pk::deflate_packed_ldg_kernel<4>
 constexpr size_t kK2pSmem = bted::pk::k2p_smem_bytes(kK2pSub);
 
 // Alg. 1 l.1 + first l.3 on the packed tiles.  (2 kernels: K1p, fin)
@@ -263,15 +267,19 @@ void enqueue_head_packed(Ted& T, const float* X, int64_t N, int32_t d, float gam
 }
 
 // Alg. 1 l.2-6 loop on the packed tiles: per step K2p (deflate + partials) and fin.  (2(m-1) kernels)
-void enqueue_loop_packed(Ted& T, int64_t N, int32_t m, float mu, unsigned long long* keys) {
+void enqueue_loop_packed(Ted& T, int64_t N, int32_t m, float mu, unsigned long long* keys, bool tma) {
     const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
     const int64_t tiles = bted::pk::num_tiles(nT);
     const unsigned grid = (unsigned)std::min<int64_t>(tiles, (int64_t)num_sms());
     for (int32_t t = 1; t < m; ++t) {
         const float* Kin = T.K[(t - 1) & 1];
         float* Kout = T.K[t & 1];
-        K2P_KERNEL<<<grid, bted::pk::kConsumers + 32, kK2pSmem, T.stream>>>(
-            Kin, Kout, nT, (int32_t)N, T.P, keys, t, mu, T.sel);
+        if (tma)
+            K2P_TMA_KERNEL<<<grid, bted::pk::kConsumers + 32, kK2pSmem, T.stream>>>(
+                Kin, Kout, nT, (int32_t)N, T.P, keys, t, mu, T.sel);
+        else
+            K2P_LDG_KERNEL<<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
+                Kin, Kout, nT, (int32_t)N, T.P, keys, t, mu, T.sel);
         bted::pk::finalize_packed_kernel<<<nT, bted::pk::kFinThreads, 0, T.stream>>>(T.P, nT, (int32_t)N, Kout, mu, T.sel,
                                                                            keys, t, keys + t, T.err);
         LAUNCHED(2);
@@ -330,7 +338,7 @@ void graph_run(Ted& T, const GraphKey& key, uint64_t nkernels, F&& enqueue) {
 void ensure_packed_attrs() {
     static bool done = false;
     if (!done) {
-        CK(cudaFuncSetAttribute(K2P_KERNEL, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        CK(cudaFuncSetAttribute(K2P_TMA_KERNEL, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)kK2pSmem));
         done = true;
     }
@@ -359,7 +367,7 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
         else enqueue_head(T, X, N, d, gamma, kernel, m, mu, keys);
     };
     auto loop = [&] {
-        if (packed) enqueue_loop_packed(T, N, m, mu, keys);
+        if (packed) enqueue_loop_packed(T, N, m, mu, keys, T.tma);
         else enqueue_loop(T, N, m, mu, keys);
     };
     if (no_graph) {
@@ -373,7 +381,7 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
         if (no_graph) {
             loop();
         } else {
-            GraphKey key{X, N, d, m, kernel, 1, packed ? 1 : 0, fbits(mu), fbits(gamma), keys};
+            GraphKey key{X, N, d, m, kernel, 1, packed ? (T.tma ? 2 : 1) : 0, fbits(mu), fbits(gamma), keys};
             graph_run(T, key, (uint64_t)(m - 1) * (packed ? 2 : 1), loop);
         }
     }
@@ -549,6 +557,7 @@ bted_status create_common(const float* X, int64_t N, int32_t d, bted_kernel kern
         ctx->ted.stream = ctx->stream;
         ctx->bted_engine.stream = ctx->stream;
         ctx->ted.timing = ctx->bted_engine.timing = (params->flags & BTED_FLAG_TIMING) != 0;
+        ctx->ted.tma = ctx->bted_engine.tma = (params->flags & BTED_FLAG_TMA) != 0;
         CK(cudaMallocHost(&ctx->herr, sizeof(int)));
         if (params->x_on_device) {
             ctx->X = const_cast<float*>(X);

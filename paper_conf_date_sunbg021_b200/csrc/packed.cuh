@@ -270,10 +270,19 @@ finalize_packed_kernel(const float* __restrict__ P, int nT, int32_t N, const flo
     for (int J0 = 0; J0 < nT; J0 += kFinChunk) {
         const int nj = min(kFinChunk, nT - J0);
         __syncthreads();
-        for (int e = tid; e < nj * (T / 4); e += kFinThreads) {
-            const int jj = e / (T / 4), c4 = e % (T / 4);
-            *reinterpret_cast<float4*>(&stg[jj][4 * c4]) =
-                __ldcg(reinterpret_cast<const float4*>(P + (int64_t)(J0 + jj) * NP + (int64_t)B * T) + c4);
+        // all loads of the chunk first (4 float4 per thread), then the smem stores
+        constexpr int kPer = kFinChunk * (T / 4) / kFinThreads;
+        float4 v[kPer];
+#pragma unroll
+        for (int u = 0; u < kPer; ++u) {
+            const int e = tid + u * kFinThreads, jj = e / (T / 4), c4 = e % (T / 4);
+            v[u] = jj < nj ? __ldcg(reinterpret_cast<const float4*>(P + (int64_t)(J0 + jj) * NP + (int64_t)B * T) + c4)
+                           : make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+#pragma unroll
+        for (int u = 0; u < kPer; ++u) {
+            const int e = tid + u * kFinThreads, jj = e / (T / 4), c4 = e % (T / 4);
+            *reinterpret_cast<float4*>(&stg[jj][4 * c4]) = v[u];
         }
         __syncthreads();
         const int per = (nj + kFinSplit - 1) / kFinSplit;
@@ -435,6 +444,244 @@ deflate_packed_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, i
         consumer_sync();                           // colg of this tile complete
         if (l < 16) P[(int64_t)J * NP + (int64_t)I * T + my_row(l)] = a.rowsum;
         if (I != J && tid < T) P[(int64_t)I * NP + (int64_t)J * T + tid] = tree32_smem(&cg[0][tid], T);
+    }
+}
+
+// 256-bit-store variant: a half-warp covers one row (lane: 8 consecutive
+// columns), rows split so each half-warp walks whole groups of 4 rows.
+template <int kSub, bool kHints>
+__global__ void __launch_bounds__(kConsumers + kWarp, 1)
+deflate_packed_v8_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, int nT, int32_t N,
+                      float* __restrict__ P, const unsigned long long* __restrict__ keys, int32_t t, float mu,
+                      uint8_t* __restrict__ sel) {
+    constexpr int kS = kStagesOf(kSub);
+    constexpr int kStageFloats = kSub * T;
+    constexpr int kSubs = T / kSub;             // stages per tile
+    constexpr int kRW = kSub / 8;               // rows per warp per stage
+    extern __shared__ __align__(1024) unsigned char smem_raw[];
+    float* stage = reinterpret_cast<float*>(smem_raw);                       // [kS][kSub*T]
+    float (*colg)[kGroups][T] = reinterpret_cast<float (*)[kGroups][T]>(smem_raw + (size_t)kS * kStageFloats * 4);
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + (size_t)kS * kStageFloats * 4 + 2 * kGroups * T * 4);
+    uint64_t* empty = full + kS;
+
+    const int tid = threadIdx.x;
+    const int64_t ntiles = num_tiles(nT);
+    if (tid == 0) {
+        for (int q = 0; q < kS; ++q) { mbar_init(full + q, 1); mbar_init(empty + q, kConsumers / kWarp); }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+
+    if (tid >= kConsumers) {
+        // ---------------- producer warp: one elected lane streams the tiles, kSub rows per stage
+        if (tid == kConsumers) {
+            const uint64_t pol = policy_evict_first();    // K streams through L2 once per step
+            int n = 0;
+            for (int64_t k = blockIdx.x; k < ntiles; k += gridDim.x) {
+                const float* src = Kin + k * (int64_t)(T * T);
+                for (int sb = 0; sb < kSubs; ++sb, ++n) {
+                    const int st = n % kS;
+                    const uint32_t ph = (uint32_t)(n / kS) & 1u;
+                    mbar_wait(empty + st, ph ^ 1u);
+                    mbar_expect_tx(full + st, kStageFloats * 4);
+                    if (kHints) bulk_g2s_hint(stage + st * kStageFloats, src + sb * kStageFloats, kStageFloats * 4,
+                                              full + st, pol);
+                    else bulk_g2s(stage + st * kStageFloats, src + sb * kStageFloats, kStageFloats * 4, full + st);
+                }
+            }
+        }
+        return;
+    }
+
+    // ---------------- consumers
+    const int w = tid / kWarp, l = tid % kWarp;
+    const int64_t NP = (int64_t)nT * T;
+    const uint32_t s = key_index(keys[t - 1]);
+    const int S = (int)(s / T), rs = (int)(s % T);
+    const float inv_c = __frcp_rn(__fadd_rn(Kin[packed_index((int)s, (int)s, nT)], mu));   // 1/(k(s,s)+mu)
+    if (blockIdx.x == 0 && tid == 0 && (int32_t)s < N) sel[s] = 1;
+    // K_in[s, B*T + c]: a contiguous row segment of tile (S,B) if S <= B, else a column of tile (B,S)
+    const uint64_t keep = kHints ? policy_evict_last() : 0ull;
+    auto ldf = [&](const float* p) -> float { return kHints ? ld_hint(p, keep) : __ldg(p); };
+    auto seg = [&](int B, int c) -> float {
+        return S <= B ? ldf(Kin + tile_offset(S, B, nT) * (T * T) + (int64_t)rs * T + c)
+                      : ldf(Kin + tile_offset(B, S, nT) * (T * T) + (int64_t)c * T + rs);
+    };
+    // the warp's 16 rows of a tile: row(l) for l < 16
+    auto my_row = [&](int q) { return (q / kRW) * kSub + w * kRW + (q % kRW); };
+    const int c8 = 8 * (l & 15);
+    auto load_segs = [&](int64_t k, float& pr, float4& pa, float4& pb) {
+        int I, J;
+        tile_ij(k, nT, I, J);
+        pr = l < 16 ? seg(I, my_row(l)) : 0.f;                 // a_i for the warp's 16 rows
+        if (S <= J) {
+            const float* p = Kin + tile_offset(S, J, nT) * (T * T) + (int64_t)rs * T + c8;
+            pa = __ldg(reinterpret_cast<const float4*>(p));
+            pb = __ldg(reinterpret_cast<const float4*>(p + 4));
+        } else {
+            pa.x = seg(J, c8); pa.y = seg(J, c8 + 1); pa.z = seg(J, c8 + 2); pa.w = seg(J, c8 + 3);
+            pb.x = seg(J, c8 + 4); pb.y = seg(J, c8 + 5); pb.z = seg(J, c8 + 6); pb.w = seg(J, c8 + 7);
+        }
+    };
+    float pr_next = 0.f;
+    float4 pa_next = make_float4(0.f, 0.f, 0.f, 0.f), pb_next = pa_next;
+    if ((int64_t)blockIdx.x < ntiles) load_segs(blockIdx.x, pr_next, pa_next, pb_next);
+    int n = 0, tcount = 0;
+    for (int64_t k = blockIdx.x; k < ntiles; k += gridDim.x, ++tcount) {
+        int I, J;
+        tile_ij(k, nT, I, J);
+        float (*cgs)[T] = colg[tcount & 1];
+        const float pr_l = pr_next;
+        const float4 pc0 = pa_next, pc1 = pb_next;
+        if (k + gridDim.x < ntiles) load_segs(k + gridDim.x, pr_next, pa_next, pb_next);   // next tile's segments
+        float* gout = Kout + k * (int64_t)(T * T);
+        float rowsum = 0.f;                         // lane l < 16: partial of the warp's row l
+        float cg[8];
+        const int hw = l >> 4, hl = l & 15;         // half-warp: rows, lane: 8 columns 8hl..8hl+7
+        for (int sb = 0; sb < kSubs; ++sb, ++n) {
+            const int st = n % kS;
+            const uint32_t ph = (uint32_t)(n / kS) & 1u;
+            mbar_wait(full + st, ph);
+            const float* sm = stage + st * kStageFloats;
+#pragma unroll
+            for (int rr = 0; rr < kRW / 2; ++rr) {
+                const int lrow = hw * (kRW / 2) + rr;              // row of the warp within the stage
+                const int q = sb * kRW + lrow;                     // the warp's q-th row of the tile
+                const int r = sb * kSub + w * kRW + lrow;          // row within the tile
+                const float ai = __shfl_sync(0xffffffffu, pr_l, q);
+                const float4 k0 = *reinterpret_cast<const float4*>(sm + (w * kRW + lrow) * T + 8 * hl);
+                const float4 k1 = *reinterpret_cast<const float4*>(sm + (w * kRW + lrow) * T + 8 * hl + 4);
+                f8 o;
+                o.v[0] = deflate1(k0.x, ai, pc0.x, inv_c); o.v[1] = deflate1(k0.y, ai, pc0.y, inv_c);
+                o.v[2] = deflate1(k0.z, ai, pc0.z, inv_c); o.v[3] = deflate1(k0.w, ai, pc0.w, inv_c);
+                o.v[4] = deflate1(k1.x, ai, pc1.x, inv_c); o.v[5] = deflate1(k1.y, ai, pc1.y, inv_c);
+                o.v[6] = deflate1(k1.z, ai, pc1.z, inv_c); o.v[7] = deflate1(k1.w, ai, pc1.w, inv_c);
+                st8_stream(gout + r * T + 8 * hl, o);
+                // canonical row tree: groups (8hl..+3), (8hl+4..+7) = groups 2hl, 2hl+1;
+                // levels 16,8,4,2 are xor 8,4,2,1 within the half-warp, level 1 is a + b
+                float ga = group4(o.v[0], o.v[1], o.v[2], o.v[3]);
+                float gb = group4(o.v[4], o.v[5], o.v[6], o.v[7]);
+#pragma unroll
+                for (int off = 8; off > 0; off >>= 1) {
+                    ga = __fadd_rn(ga, __shfl_xor_sync(0xffffffffu, ga, off));
+                    gb = __fadd_rn(gb, __shfl_xor_sync(0xffffffffu, gb, off));
+                }
+                const float rp = __fadd_rn(ga, gb);
+                // row q's sum lives in half hw; lane q (< 16) keeps it
+                const float rq0 = __shfl_sync(0xffffffffu, rp, 0);    // half 0's row
+                const float rq1 = __shfl_sync(0xffffffffu, rp, 16);   // half 1's row
+                const int q0 = sb * kRW + rr, q1 = sb * kRW + kRW / 2 + rr;
+                if (l == q0) rowsum = rq0;
+                if (l == q1) rowsum = rq1;
+                if (I != J) {
+                    if ((r & 3) == 0) {
+#pragma unroll
+                        for (int c = 0; c < 8; ++c) cg[c] = __fmul_rn(o.v[c], o.v[c]);
+                    } else {
+#pragma unroll
+                        for (int c = 0; c < 8; ++c) cg[c] = __fmaf_rn(o.v[c], o.v[c], cg[c]);
+                    }
+                    if ((r & 3) == 3) {
+                        *reinterpret_cast<float4*>(&cgs[r >> 2][8 * hl]) = make_float4(cg[0], cg[1], cg[2], cg[3]);
+                        *reinterpret_cast<float4*>(&cgs[r >> 2][8 * hl + 4]) = make_float4(cg[4], cg[5], cg[6], cg[7]);
+                    }
+                }
+            }
+            __syncwarp();
+            if (l == 0) mbar_arrive(empty + st);   // this warp is done reading the stage
+        }
+        consumer_sync();                           // colg of this tile complete
+        if (l < 16) P[(int64_t)J * NP + (int64_t)I * T + my_row(l)] = rowsum;
+        if (I != J && tid < T) P[(int64_t)I * NP + (int64_t)J * T + tid] = tree32_smem(&cgs[0][tid], T);
+    }
+}
+
+// ------------------------------------------------------------------ K2p (LDG variant)
+// One CTA (256 threads) per tile, non-persistent (the hardware scheduler
+// balances 8256+ tiles over the SMs; several CTAs per SM keep many 256-bit
+// loads in flight, like the dense K2).  Warp w owns rows 16w..16w+15; half-warp
+// h of it rows 16w+8h..+7 (two whole groups of 4 rows); lane hl owns columns
+// 8hl..8hl+7.  Same element arithmetic and canonical partial trees as the
+// TMA variant (bit-identical outputs).
+template <int kU>
+__global__ void __launch_bounds__(kConsumers)
+deflate_packed_ldg_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, int nT, int32_t N,
+                          float* __restrict__ P, const unsigned long long* __restrict__ keys, int32_t t, float mu,
+                          uint8_t* __restrict__ sel) {
+    __shared__ __align__(16) float cgs[kGroups][T];
+    const int tid = threadIdx.x, w = tid / kWarp, l = tid % kWarp;
+    const int hw = l >> 4, hl = l & 15, c8 = 8 * hl;
+    const int64_t k = blockIdx.x;
+    int I, J;
+    tile_ij(k, nT, I, J);
+    const int64_t NP = (int64_t)nT * T;
+    const uint32_t s = key_index(keys[t - 1]);
+    const int S = (int)(s / T), rs = (int)(s % T);
+    if (k == 0 && tid == 0 && (int32_t)s < N) sel[s] = 1;
+    const float inv_c = __frcp_rn(__fadd_rn(__ldg(Kin + packed_index((int)s, (int)s, nT)), mu));
+    auto seg = [&](int B, int c) -> float {
+        return S <= B ? __ldg(Kin + tile_offset(S, B, nT) * (T * T) + (int64_t)rs * T + c)
+                      : __ldg(Kin + tile_offset(B, S, nT) * (T * T) + (int64_t)c * T + rs);
+    };
+    // a_i for the half-warp's 8 rows (lane hl < 8 holds row 16w + 8hw + hl), p_j for the lane's 8 columns
+    const float pr_l = hl < 8 ? seg(I, 16 * w + 8 * hw + hl) : 0.f;
+    float pc[8];
+    if (S <= J) {
+        const float* p = Kin + tile_offset(S, J, nT) * (T * T) + (int64_t)rs * T + c8;
+        const float4 a = __ldg(reinterpret_cast<const float4*>(p)), b = __ldg(reinterpret_cast<const float4*>(p + 4));
+        pc[0] = a.x; pc[1] = a.y; pc[2] = a.z; pc[3] = a.w; pc[4] = b.x; pc[5] = b.y; pc[6] = b.z; pc[7] = b.w;
+    } else {
+#pragma unroll
+        for (int c = 0; c < 8; ++c) pc[c] = seg(J, c8 + c);
+    }
+    const float* gin = Kin + k * (int64_t)(T * T);
+    float* gout = Kout + k * (int64_t)(T * T);
+    float rowsum = 0.f;                      // lane q < 16 of the warp: the warp's row q
+    float cg[8];
+#pragma unroll
+    for (int r0 = 0; r0 < 8; r0 += kU) {
+        f8 kv[kU];
+#pragma unroll
+        for (int u = 0; u < kU; ++u) kv[u] = ld8_stream(gin + (16 * w + 8 * hw + r0 + u) * T + c8);
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int rr = r0 + u;                       // row within the half-warp's 8
+            const int r = 16 * w + 8 * hw + rr;          // row within the tile
+            const float ai = __shfl_sync(0xffffffffu, pr_l, 16 * hw + rr);
+            f8 o;
+#pragma unroll
+            for (int c = 0; c < 8; ++c) o.v[c] = deflate1(kv[u].v[c], ai, pc[c], inv_c);
+            st8_stream(gout + r * T + c8, o);
+            float ga = group4(o.v[0], o.v[1], o.v[2], o.v[3]);
+            float gb = group4(o.v[4], o.v[5], o.v[6], o.v[7]);
+#pragma unroll
+            for (int off = 8; off > 0; off >>= 1) {
+                ga = __fadd_rn(ga, __shfl_xor_sync(0xffffffffu, ga, off));
+                gb = __fadd_rn(gb, __shfl_xor_sync(0xffffffffu, gb, off));
+            }
+            const float rp = __fadd_rn(ga, gb);
+            const float rq0 = __shfl_sync(0xffffffffu, rp, 0), rq1 = __shfl_sync(0xffffffffu, rp, 16);
+            if (l == rr) rowsum = rq0;
+            if (l == 8 + rr) rowsum = rq1;
+            if (I != J) {
+                if ((rr & 3) == 0) {
+#pragma unroll
+                    for (int c = 0; c < 8; ++c) cg[c] = __fmul_rn(o.v[c], o.v[c]);
+                } else {
+#pragma unroll
+                    for (int c = 0; c < 8; ++c) cg[c] = __fmaf_rn(o.v[c], o.v[c], cg[c]);
+                }
+                if ((rr & 3) == 3) {
+                    *reinterpret_cast<float4*>(&cgs[r >> 2][c8]) = make_float4(cg[0], cg[1], cg[2], cg[3]);
+                    *reinterpret_cast<float4*>(&cgs[r >> 2][c8 + 4]) = make_float4(cg[4], cg[5], cg[6], cg[7]);
+                }
+            }
+        }
+    }
+    if (l < 16) P[(int64_t)J * NP + (int64_t)I * T + 16 * w + l] = rowsum;
+    if (I != J) {
+        __syncthreads();
+        if (tid < T) P[(int64_t)I * NP + (int64_t)J * T + tid] = tree32_smem(&cgs[0][tid], T);
     }
 }
 

@@ -29,16 +29,16 @@ __global__ void init_packed(float* K, int nT, int N) {
     }
 }
 
-template <int kSub, bool kHints>
+template <int kSub, bool kHints, bool kV8 = false>
 void launch(const float* A, float* B, int nT, int N, float* P, unsigned long long* keys, uint8_t* sel, int sms) {
+    auto kern = kV8 ? deflate_packed_v8_kernel<kSub, kHints> : deflate_packed_kernel<kSub, kHints>;
     static bool set = false;
     if (!set) {
-        CK(cudaFuncSetAttribute(deflate_packed_kernel<kSub, kHints>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)k2p_smem_bytes(kSub)));
+        CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k2p_smem_bytes(kSub)));
         set = true;
     }
     const int64_t tiles = num_tiles(nT);
-    deflate_packed_kernel<kSub, kHints><<<(unsigned)std::min<int64_t>(tiles, sms), kConsumers + 32, k2p_smem_bytes(kSub)>>>(
+    kern<<<(unsigned)std::min<int64_t>(tiles, sms), kConsumers + 32, k2p_smem_bytes(kSub)>>>(
         A, B, nT, N, P, keys, 1, 0.1f, sel);
 }
 
@@ -89,8 +89,12 @@ int main(int argc, char** argv) {
     run("k2p<128,hints>", [&] { launch<128, true>(A, B, nT, N, P, keys, sel, sms); }, true);
     run("k2p<64,nohint>", [&] { launch<64, false>(A, B, nT, N, P, keys, sel, sms); }, true);
     run("k2p<64,hints>", [&] { launch<64, true>(A, B, nT, N, P, keys, sel, sms); }, true);
-    run("k2p<32,nohint>", [&] { launch<32, false>(A, B, nT, N, P, keys, sel, sms); }, true);
-    run("k2p<32,hints>", [&] { launch<32, true>(A, B, nT, N, P, keys, sel, sms); }, true);
+    run("k2p_v8<128,nohint>", [&] { launch<128, false, true>(A, B, nT, N, P, keys, sel, sms); }, true);
+    run("k2p_v8<64,nohint>", [&] { launch<64, false, true>(A, B, nT, N, P, keys, sel, sms); }, true);
+    run("k2p_v8<64,hints>", [&] { launch<64, true, true>(A, B, nT, N, P, keys, sel, sms); }, true);
+    run("k2p_ldg<4>", [&] { deflate_packed_ldg_kernel<4><<<(unsigned)num_tiles(nT), kConsumers>>>(A, B, nT, N, P, keys, 1, 0.1f, sel); }, true);
+    run("k2p_ldg<8>", [&] { deflate_packed_ldg_kernel<8><<<(unsigned)num_tiles(nT), kConsumers>>>(A, B, nT, N, P, keys, 1, 0.1f, sel); }, true);
+    run("k2p_ldg<2>", [&] { deflate_packed_ldg_kernel<2><<<(unsigned)num_tiles(nT), kConsumers>>>(A, B, nT, N, P, keys, 1, 0.1f, sel); }, true);
     run("finalize", [&] { finalize_packed_kernel<<<nT, kFinThreads>>>(P, nT, N, B, 0.1f, sel, keys, 1, keys + 1, err); }, false);
     printf("done N=%d tiles=%lld\n", N, (long long)num_tiles(nT));
     return 0;

@@ -17,8 +17,9 @@ MU = float(np.float32(0.1))
 # cluster TED of small.cuh for N <= ~940, packed above)
 PACKED = L.BTED_FLAG_NO_SMALL
 DENSE = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_DENSE
-LAYOUTS = pytest.mark.parametrize("flags", [PACKED, DENSE, 0], ids=["packed", "dense", "auto"])
-LAYOUTS_K = pytest.mark.parametrize("flags", [PACKED, DENSE], ids=["packed", "dense"])   # tests reading K back
+PACKED_TMA = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_TMA
+LAYOUTS = pytest.mark.parametrize("flags", [PACKED, PACKED_TMA, DENSE, 0], ids=["packed", "packed-tma", "dense", "auto"])
+LAYOUTS_K = pytest.mark.parametrize("flags", [PACKED, PACKED_TMA, DENSE], ids=["packed", "packed-tma", "dense"])
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -301,9 +302,13 @@ def test_packed_layout_matches_dense(N, d, m):
     the dense layout; only the norm summation order differs."""
     X = knob(N, d=16, seed=N)[:, :d] if d <= 16 else uniform_pool(N, d, N)
     g = median_gamma(X, d)
-    with bt.CandidateSet(X, g, flags=DENSE) as cd, bt.CandidateSet(X, g, flags=PACKED) as cp:
+    with bt.CandidateSet(X, g, flags=DENSE) as cd, bt.CandidateSet(X, g, flags=PACKED) as cp, \
+            bt.CandidateSet(X, g, flags=PACKED_TMA) as ct:
         i_d, s_d = cd.select(m, MU)
         i_p, s_p = cp.select(m, MU)
+        i_t, s_t = ct.select(m, MU)
+        assert np.array_equal(i_t, i_p) and np.array_equal(s_t.view(np.uint32), s_p.view(np.uint32))
+        assert np.array_equal(ct.debug_K(N), cp.debug_K(N))       # TMA and LDG variants: same bits
         tr = dense.ted(X, g, MU, m, forced=i_p)
         check_ted(i_p, s_p, tr, f"packed-{N}")
         if np.array_equal(i_d, i_p):
