@@ -260,11 +260,13 @@ def bench_ours(args):
     # H2D of the pool, the whole BTED, D2H of the result
     e2e = None
     if not args.no_e2e:
-        Xh = torch.from_numpy(X).pin_memory()
-        ctx2 = bt.CandidateSet(Xh.numpy(), gamma, num_batches=B, seed=cfg["seed"], device=local,
+        # the pool in page-locked memory of the library's runtime (bted_host_alloc)
+        Xpin = L.PinnedArray(X.shape)
+        Xpin.array[:] = X
+        ctx2 = bt.CandidateSet(Xpin.array, gamma, num_batches=B, seed=cfg["seed"], device=local,
                                flags=lay_flag, stream=stream.cuda_stream)
         for _ in range(max(1, args.warmup)):
-            L.bted_update(ctx2.ctx, Xh.data_ptr())
+            L.bted_update(ctx2.ctx, Xpin.ptr)
             if world == 1:
                 ctx2.run_batches(M, m, mu, want_batches=False)
             else:
@@ -275,7 +277,7 @@ def bench_ours(args):
         f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         f0.record(stream)
         for _ in range(args.steps):
-            L.bted_update(ctx2.ctx, Xh.data_ptr())
+            L.bted_update(ctx2.ctx, Xpin.ptr)
             if world == 1:
                 ctx2.run_batches(M, m, mu, want_batches=False)
             else:
@@ -286,6 +288,7 @@ def bench_ours(args):
         barrier()
         ems = max_over_ranks(f0.elapsed_time(f1))
         ctx2.close()
+        Xpin.close()
         e2e = {"value": args.steps * B * m / (ems / 1e3), "unit": UNIT,
                "h2d_bytes_per_step": int(P * d * 4),
                "d2h_bytes_per_step": int(8 * m + 4 + 8 * m + 4 + 4)}

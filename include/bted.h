@@ -32,6 +32,7 @@
 #ifndef BTED_H_
 #define BTED_H_
 
+#include <stddef.h>
 #include <stdint.h>
 
 #ifdef __cplusplus
@@ -196,6 +197,16 @@ bted_status bted_shard_check(bted_ctx* shard);
  * (x_on_device = 1) is copied D2D.  Errors: EINVAL, ECUDA, ESTATE.
  */
 bted_status bted_update(bted_ctx* ctx, const float* X, int32_t x_on_device);
+
+/*
+ * bted_host_alloc / bted_host_free -- page-locked host memory from the
+ * library's CUDA runtime, for feature buffers passed to bted_create /
+ * bted_update: host->device copies from it run at DMA speed (memory pinned by
+ * another runtime instance in the process, e.g. torch's, is copied as
+ * pageable).  Errors: EINVAL, ENOMEM, ECUDA.
+ */
+bted_status bted_host_alloc(size_t bytes, void** out);
+void        bted_host_free(void* p);
 
 /* Accumulated device timings of the TEDs run by a ctx (BTED_FLAG_TIMING):
  * k1_ms = transpose + Gram (Alg. 1 l.1 + first l.3), k2_ms = the fused

@@ -70,6 +70,8 @@ _SIGS = {
     "bted_update": (ctypes.c_int, [_vp, _vp, _i32]),
     "bted_get_stats": (ctypes.c_int, [_vp, ctypes.POINTER(bted_stats)]),
     "bted_reset_stats": (ctypes.c_int, [_vp]),
+    "bted_host_alloc": (ctypes.c_int, [ctypes.c_size_t, ctypes.POINTER(_vp)]),
+    "bted_host_free": (None, [_vp]),
 }
 EXPORTS = tuple(_SIGS)
 
@@ -210,6 +212,31 @@ def bted_update(ctx: int, X, x_on_device: bool = False):
     the call, so it is first pinned by the caller or kept alive)."""
     ptr = X if isinstance(X, int) else _ptr(X)
     check(lib().bted_update(ctx, ptr, 1 if x_on_device else 0))
+
+
+class PinnedArray:
+    """A numpy view of page-locked memory from bted_host_alloc (freed on close/del)."""
+
+    def __init__(self, shape, dtype=np.float32):
+        dtype = np.dtype(dtype)
+        n = int(np.prod(shape)) * dtype.itemsize
+        p = _vp()
+        check(lib().bted_host_alloc(n, ctypes.byref(p)))
+        self.ptr = p.value
+        buf = (ctypes.c_char * n).from_address(self.ptr)
+        self.array = np.frombuffer(buf, dtype=dtype).reshape(shape)
+
+    def close(self):
+        if getattr(self, "ptr", None):
+            self.array = None
+            lib().bted_host_free(self.ptr)
+            self.ptr = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 def bted_get_stats(ctx: int) -> dict:

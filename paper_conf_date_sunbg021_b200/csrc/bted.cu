@@ -983,6 +983,22 @@ bted_status bted_update(bted_ctx* ctx, const float* X, int32_t x_on_device) {
     });
 }
 
+bted_status bted_host_alloc(size_t bytes, void** out) {
+    if (!out || bytes == 0) { set_error("need bytes > 0 and out != NULL"); return BTED_EINVAL; }
+    *out = nullptr;
+    cudaError_t e = cudaMallocHost(out, bytes);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        set_error("cudaMallocHost(%zu): %s", bytes, cudaGetErrorString(e));
+        return e == cudaErrorMemoryAllocation ? BTED_ENOMEM : BTED_ECUDA;
+    }
+    return BTED_OK;
+}
+
+void bted_host_free(void* p) {
+    if (p) cudaFreeHost(p);
+}
+
 bted_status bted_get_stats(bted_ctx* ctx, bted_stats* out) {
     if (!ctx || !out) { set_error("null argument"); return BTED_EINVAL; }
     const Stats& a = ctx->ted.stats;

@@ -596,6 +596,19 @@ deflate_packed_v8_kernel(const float* __restrict__ Kin, float* __restrict__ Kout
     }
 }
 
+// L2-priority variants for the LDG kernel: K streams evict-first, the
+// partials (nT * NP floats, read by the finalize kernel) are kept evict-last.
+__device__ __forceinline__ f8 ld8_evict_first(const float* p) {
+    f8 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::evict_first.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=f"(r.v[0]), "=f"(r.v[1]), "=f"(r.v[2]), "=f"(r.v[3]), "=f"(r.v[4]), "=f"(r.v[5]),
+                   "=f"(r.v[6]), "=f"(r.v[7]) : "l"(p));
+    return r;
+}
+__device__ __forceinline__ void st_keep(float* p, float v, uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.f32 [%0], %1, %2;" :: "l"(p), "f"(v), "l"(pol) : "memory");
+}
+
 // ------------------------------------------------------------------ K2p (LDG variant)
 // One CTA (256 threads) per tile, non-persistent (the hardware scheduler
 // balances 8256+ tiles over the SMs; several CTAs per SM keep many 256-bit
@@ -642,7 +655,7 @@ deflate_packed_ldg_kernel(const float* __restrict__ Kin, float* __restrict__ Kou
     for (int r0 = 0; r0 < 8; r0 += kU) {
         f8 kv[kU];
 #pragma unroll
-        for (int u = 0; u < kU; ++u) kv[u] = ld8_stream(gin + (16 * w + 8 * hw + r0 + u) * T + c8);
+        for (int u = 0; u < kU; ++u) kv[u] = ld8_evict_first(gin + (16 * w + 8 * hw + r0 + u) * T + c8);
 #pragma unroll
         for (int u = 0; u < kU; ++u) {
             const int rr = r0 + u;                       // row within the half-warp's 8
@@ -678,10 +691,11 @@ deflate_packed_ldg_kernel(const float* __restrict__ Kin, float* __restrict__ Kou
             }
         }
     }
-    if (l < 16) P[(int64_t)J * NP + (int64_t)I * T + 16 * w + l] = rowsum;
+    const uint64_t keep = policy_evict_last();
+    if (l < 16) st_keep(P + (int64_t)J * NP + (int64_t)I * T + 16 * w + l, rowsum, keep);
     if (I != J) {
         __syncthreads();
-        if (tid < T) P[(int64_t)I * NP + (int64_t)J * T + tid] = tree32_smem(&cgs[0][tid], T);
+        if (tid < T) st_keep(P + (int64_t)I * NP + (int64_t)J * T + tid, tree32_smem(&cgs[0][tid], T), keep);
     }
 }
 

@@ -13,7 +13,7 @@ timeout 900 python bench.py --steps 10 --warmup 3 > $OUT/bench.json 2> $OUT/benc
 timeout 900 python bench.py --steps 10 --warmup 3 --layout dense --no-cpu-baseline > $OUT/bench_dense.json 2> $OUT/bench_dense.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
     python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_launches.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:deflate_packed -s 8 -c 1 \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"deflate_packed|finalize_packed" -s 16 -c 2 \
     -o $OUT/prof_k2p python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_k2p.log 2>&1
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:gram_packed -s 2 -c 1 \
     -o $OUT/prof_k1p python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_k1p.log 2>&1

@@ -25,7 +25,10 @@ for name, fn in [("torch pinned copy_", lambda: Xd.copy_(Xh, non_blocking=True))
         torch.cuda.synchronize()
     print(f"{name}: {X.nbytes * 10 / (e0.elapsed_time(e1) / 1e3) / 1e9:.1f} GB/s")
 cs = bt.CandidateSet(X, 0.3, stream=st.cuda_stream)
-for name, ptr in [("bted_update pinned(torch)", Xh.data_ptr()), ("bted_update pageable(numpy)", X.ctypes.data)]:
+pa = L.PinnedArray(X.shape)
+pa.array[:] = X
+for name, ptr in [("bted_update pinned(torch)", Xh.data_ptr()), ("bted_update pageable(numpy)", X.ctypes.data),
+                  ("bted_update pinned(bted_host_alloc)", pa.ptr)]:
     for _ in range(3):
         L.bted_update(cs.ctx, ptr)
     torch.cuda.synchronize()
