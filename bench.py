@@ -47,6 +47,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="weak: every GPU runs the config's B batches; strong: the config's B batches are split")
     ap.add_argument("--layout", default="packed", choices=["packed", "dense"],
                     help="K storage: packed upper-triangular tiles (4 N^2 B/step) or dense (8 N^2 B/step)")
     return ap.parse_args()
@@ -163,12 +165,13 @@ def bench_reference(args):
     print(json.dumps(line), flush=True)
 
 
-def workload_config(name, cfg, gamma, world):
+def workload_config(name, cfg, gamma, world, B=None):
+    B = cfg["B"] * world if B is None else B
     return {"workload": f"{name}: BTED on the AutoTVM conv2d knob pool of {cfg['workload']} "
-                        f"(P={cfg['pool']} configs, d={cfg['d']}), B={cfg['B'] * world} batches of "
+                        f"(P={cfg['pool']} configs, d={cfg['d']}), B={B} batches of "
                         f"M={cfg['M']}, m={cfg['m']}, mu={cfg['mu']}, RBF gamma={gamma:.6g} (median heuristic)",
-            "pool": cfg["pool"], "M": cfg["M"], "d": cfg["d"], "m": cfg["m"], "B": cfg["B"] * world,
-            "batches_per_gpu": cfg["B"], "mu": cfg["mu"], "seed": cfg["seed"],
+            "pool": cfg["pool"], "M": cfg["M"], "d": cfg["d"], "m": cfg["m"], "B": B,
+            "batches_per_gpu": B / world, "mu": cfg["mu"], "seed": cfg["seed"],
             "l2": "inputs larger than L2: K = 4*M^2 bytes per batch (1 GiB at M=16384) >> 126 MB",
             "parallelism": f"batch round-robin over {world} GPU(s)" if world > 1 else "1 GPU"}
 
@@ -195,7 +198,9 @@ def bench_ours(args):
     X, gamma, cfg = config_pool(args.config)
     mu = float(np.float32(cfg["mu"]))
     M, m, d, P = cfg["M"], cfg["m"], cfg["d"], X.shape[0]
-    B = cfg["B"] * world
+    if cfg["B"] == 1 and args.config == "oversized" and world > 1:
+        return bench_sharded(args, X, gamma, cfg, comm, dev, world, rank)
+    B = cfg["B"] * world if args.scaling == "weak" else cfg["B"]
     stream = torch.cuda.Stream(dev)
     X_dev = torch.from_numpy(X).to(dev)
     torch.cuda.synchronize()
@@ -307,8 +312,8 @@ def bench_ours(args):
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-                "config": workload_config(args.config, cfg, gamma, world),
+                "scaling": args.scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": workload_config(args.config, cfg, gamma, world, B),
                 "layout": args.layout,
                 "roofline": {"bound": "hbm", "kernel": K2_NAME[args.layout], "achieved": achieved, "peak": peak,
                              "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
@@ -322,6 +327,65 @@ def bench_ours(args):
         print(json.dumps(line), flush=True)
     if world > 1:
         torch.distributed.destroy_process_group()
+
+
+def bench_sharded(args, X, gamma, cfg, comm, dev, world, rank):
+    """config 'oversized' on N > 1 GPUs: ONE batch of M points, K row-sharded
+    (dense bands) over the ranks; per step an 8-byte MAX all-reduce of the
+    packed argmax key and an all-gather of column s (= row s) -- dist.ShardedTed."""
+    import torch
+    import paper_conf_date_sunbg021_b200 as bt
+    from paper_conf_date_sunbg021_b200.dist import LibShard, ShardedTed, band
+    from oracle.sampling import sample_batches  # noqa: F401  (not used on the timed path)
+    mu = float(np.float32(cfg["mu"]))
+    M, m = cfg["M"], cfg["m"]
+    # the batch V_0 = the first draw of Alg. 2 l.2, gathered on every rank by the library
+    V = bt.bted_sample_batches(X.shape[0], M, 1, cfg["seed"])[0]
+    Xb = np.ascontiguousarray(X[V])
+    stream = torch.cuda.Stream(dev)
+    r0, r1, _ = band(M, world, rank)
+    shard = LibShard(Xb, M, cfg["d"], gamma, r0, r1, dev, stream)
+    st = ShardedTed(shard, M, comm, dev, stream)
+    for _ in range(args.warmup):
+        st.select(m, mu)
+    clocks = Clocks(int(os.environ.get("LOCAL_RANK", "0")))
+    clocks.start()
+    l0 = bt.bted_kernel_launches()
+    torch.distributed.barrier()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.steps):
+        idx, _ = st.select(m, mu)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    torch.distributed.barrier()
+    launches = bt.bted_kernel_launches() - l0
+    t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+    torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+    ms = float(t.item())
+    clk = clocks.stop()
+    shard.close()
+    peak, peak_src = peaks()
+    step_ms = ms / args.steps / max(m - 1, 1)
+    per_gpu_bytes = 8.0 * M * M / world
+    achieved = per_gpu_bytes / (step_ms / 1e3) / 1e9
+    if rank == 0:
+        line = {"metric": METRIC, "value": args.steps * m / (ms / 1e3), "unit": UNIT, "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+                "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+                "data": "synthetic", "layout": "dense-row-sharded",
+                "config": dict(workload_config(args.config, cfg, gamma, world, 1),
+                               parallelism=f"row-sharded K over {world} GPUs (NCCL all-reduce + all-gather per step)"),
+                "roofline": {"bound": "hbm", "kernel": "deflate_rescore_kernel (per-GPU band) + NCCL",
+                             "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                             "traffic": None, "peak_source": peak_src,
+                             "alg_bytes_per_launch": per_gpu_bytes, "avg_launch_ms": step_ms,
+                             "note": "per-GPU step time includes the two collectives"},
+                "cpu_baseline": None, "e2e": None, "gpu_launches": int(launches), "clocks": clk,
+                "final_selection_head": [int(x) for x in idx[:8]]}
+        print(json.dumps(line), flush=True)
+    torch.distributed.destroy_process_group()
 
 
 def main():

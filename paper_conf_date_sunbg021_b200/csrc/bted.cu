@@ -388,11 +388,6 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
     if (sl) CK(cudaEventRecord(sl->e[2], T.stream));
 }
 
-bool all_finite(const float* X, int64_t n) {
-    for (int64_t i = 0; i < n; ++i)
-        if (!std::isfinite(X[i])) return false;
-    return true;
-}
 
 }  // namespace
 
@@ -432,6 +427,7 @@ struct bted_ctx {
     // host staging (pinned)
     unsigned long long* hkeys = nullptr; size_t hkeyscap = 0;
     int* herr = nullptr;
+    int* xbad = nullptr;      // device: non-finite feature seen by finite_check_kernel
 };
 
 namespace {
@@ -476,6 +472,24 @@ bted_status guarded(bted_ctx* ctx, F&& f) {
     }
 }
 
+void launch_finite_check(bted_ctx* ctx) {
+    const int64_t n = ctx->N * ctx->d;
+    const unsigned g = (unsigned)std::min<int64_t>((n + 255) / 256, 148 * 8);
+    bted::finite_check_kernel<<<g, 256, 0, ctx->stream>>>(ctx->X, n, ctx->xbad);
+    LAUNCHED(1);
+}
+
+// a bted_update of non-finite features surfaces at the next host sync
+bool take_xbad(bted_ctx* ctx) {
+    int v = 0;
+    CK(cudaMemcpy(&v, ctx->xbad, sizeof(int), cudaMemcpyDeviceToHost));
+    if (v) {
+        CK(cudaMemset(ctx->xbad, 0, sizeof(int)));
+        set_error("X has non-finite entries (bted_update)");
+    }
+    return v != 0;
+}
+
 // Decode m packed keys on the host; checks the sticky error flag.
 bted_status finish_keys(bted_ctx* ctx, Ted& T, const unsigned long long* keys_dev, int32_t m,
                         int64_t* out_idx, float* out_score, const int64_t* map_dev = nullptr) {
@@ -485,6 +499,7 @@ bted_status finish_keys(bted_ctx* ctx, Ted& T, const unsigned long long* keys_de
     if (map_dev) CK(cudaMemcpyAsync(out_idx, map_dev, sizeof(int64_t) * m, cudaMemcpyDeviceToHost, T.stream));
     CK(cudaStreamSynchronize(T.stream));
     T.collect();
+    if (ctx->xbad && take_xbad(ctx)) return BTED_EINVAL;
     if (*ctx->herr) {
         CK(cudaMemsetAsync(T.err, 0, sizeof(int), T.stream));
         set_error("non-finite score or non-positive k(v,v)+mu during TED");
@@ -521,7 +536,6 @@ bted_status create_common(const float* X, int64_t N, int32_t d, bted_kernel kern
         set_error("need X != NULL, 1 <= N < 2^31, 1 <= d <= 64"); return BTED_EINVAL;
     }
     if (shard && !(0 <= row0 && row0 < row1 && row1 <= N)) { set_error("need 0 <= row0 < row1 <= N"); return BTED_EINVAL; }
-    if (!params->x_on_device && !all_finite(X, N * d)) { set_error("X has non-finite entries"); return BTED_EINVAL; }
     int ndev = 0;
     cudaError_t e = cudaGetDeviceCount(&ndev);
     if (e != cudaSuccess || ndev < 1) {
@@ -565,8 +579,13 @@ bted_status create_common(const float* X, int64_t N, int32_t d, bted_kernel kern
             CK(cudaMalloc(&ctx->X, sizeof(float) * N * d));
             ctx->own_X = true;
             CK(cudaMemcpyAsync(ctx->X, X, sizeof(float) * N * d, cudaMemcpyHostToDevice, ctx->stream));
-            CK(cudaStreamSynchronize(ctx->stream));
         }
+        CK(cudaMalloc(&ctx->xbad, sizeof(int)));
+        CK(cudaMemsetAsync(ctx->xbad, 0, sizeof(int), ctx->stream));
+        launch_finite_check(ctx);
+        CK(cudaMemcpyAsync(ctx->herr, ctx->xbad, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        if (*ctx->herr) { set_error("X has non-finite entries"); return BTED_EINVAL; }
         return BTED_OK;
     });
     if (st != BTED_OK) {
@@ -831,6 +850,7 @@ bted_status bted_batch_teds(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32
             CK(cudaMemcpyAsync(ctx->herr, ctx->bted_engine.err, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
         CK(cudaStreamSynchronize(ctx->stream));
         ctx->bted_engine.collect();
+        if (take_xbad(ctx)) return BTED_EINVAL;
         if (nb > 0 && *ctx->herr) {
             CK(cudaMemsetAsync(ctx->bted_engine.err, 0, sizeof(int), ctx->stream));
             set_error("non-finite score during a batch TED");
@@ -969,7 +989,6 @@ bted_status bted_shard_check(bted_ctx* ctx) {
 
 bted_status bted_update(bted_ctx* ctx, const float* X, int32_t x_on_device) {
     if (!ctx || !X) { set_error("null argument"); return BTED_EINVAL; }
-    if (!x_on_device && !all_finite(X, ctx->N * ctx->d)) { set_error("X has non-finite entries"); return BTED_EINVAL; }
     return guarded(ctx, [&]() -> bted_status {
         if (!ctx->own_X) {
             CK(cudaMalloc(&ctx->X, sizeof(float) * ctx->N * ctx->d));
@@ -978,7 +997,9 @@ bted_status bted_update(bted_ctx* ctx, const float* X, int32_t x_on_device) {
         CK(cudaMemcpyAsync(ctx->X, X, sizeof(float) * ctx->N * ctx->d,
                            x_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, ctx->stream));
         // no sync: later work of this ctx is ordered after the copy on its stream;
-        // the caller must keep a host X alive until the next call returns
+        // the caller must keep a host X alive until the next call returns.  The
+        // finiteness check runs on the device; a bad X fails the next call (EINVAL).
+        launch_finite_check(ctx);
         return BTED_OK;
     });
 }
@@ -1032,6 +1053,7 @@ void bted_destroy(bted_ctx* ctx) {
         if (ctx->own_X && ctx->X) cudaFree(ctx->X);
         if (ctx->hkeys) cudaFreeHost(ctx->hkeys);
         if (ctx->herr) cudaFreeHost(ctx->herr);
+        if (ctx->xbad) cudaFree(ctx->xbad);
         if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
         cudaGetLastError();
     }

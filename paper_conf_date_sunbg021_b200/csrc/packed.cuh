@@ -119,6 +119,25 @@ __device__ __forceinline__ void consumer_sync() {       // named barrier 1: the 
     asm volatile("bar.sync 1, %0;" :: "n"(kConsumers) : "memory");
 }
 
+// ------------------------------------------------------------------ f32x2 (sm_100 FADD2 / FFMA2)
+__device__ __forceinline__ unsigned long long pack2(float lo, float hi) {
+    return ((unsigned long long)__float_as_uint(hi) << 32) | (unsigned long long)__float_as_uint(lo);
+}
+__device__ __forceinline__ void unpack2(unsigned long long v, float& lo, float& hi) {
+    lo = __uint_as_float((unsigned)(v & 0xFFFFFFFFull));
+    hi = __uint_as_float((unsigned)(v >> 32));
+}
+__device__ __forceinline__ unsigned long long sub2(unsigned long long a, unsigned long long b) {
+    unsigned long long d;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+    return d;
+}
+__device__ __forceinline__ unsigned long long fma2(unsigned long long a, unsigned long long b, unsigned long long c) {
+    unsigned long long d;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+    return d;
+}
+
 // ------------------------------------------------------------------ canonical sums
 // group of 4 consecutive terms: ((v0^2 + v1^2) + v2^2) + v3^2 with fused steps
 __device__ __forceinline__ float group4(float v0, float v1, float v2, float v3) {
@@ -201,33 +220,41 @@ gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamm
             xj[r][c] = (gj < N && c < d) ? X[(int64_t)gj * d + c] : 0.f;
         }
         consumer_sync();
-        float y[4][kD];
+        // column features as f32x2 pairs (columns 4l,4l+1 | 4l+2,4l+3): the
+        // distance loop runs on FADD2/FFMA2 (IEEE RN per half: bitwise the
+        // same as the scalar __fsub_rn / __fmaf_rn sequence)
+        unsigned long long y01[kD], y23[kD];
 #pragma unroll
-        for (int c = 0; c < 4; ++c)
-#pragma unroll
-            for (int q = 0; q < kD; q += 4) {
-                const float4 v = *reinterpret_cast<const float4*>(&xj[4 * l + c][q]);
-                y[c][q] = v.x; y[c][q + 1] = v.y; y[c][q + 2] = v.z; y[c][q + 3] = v.w;
-            }
+        for (int q = 0; q < kD; ++q) {
+            y01[q] = pack2(xj[4 * l + 0][q], xj[4 * l + 1][q]);
+            y23[q] = pack2(xj[4 * l + 2][q], xj[4 * l + 3][q]);
+        }
         float* tile = K + k * (int64_t)(T * T);
         RowWalk a;
         a.rowsum = 0.f;
         for (int rr = 0; rr < 16; ++rr) {
             const int r = 16 * w + rr;
-            float acc[4] = {0.f, 0.f, 0.f, 0.f};
+            unsigned long long a01 = 0ull, a23 = 0ull;
 #pragma unroll
             for (int q = 0; q < kD; q += 4) {
                 const float4 xv = *reinterpret_cast<const float4*>(&xi[r][q]);
                 const float xs[4] = {xv.x, xv.y, xv.z, xv.w};
 #pragma unroll
                 for (int qq = 0; qq < 4; ++qq) {
-#pragma unroll
-                    for (int c = 0; c < 4; ++c) {
-                        if (linear) acc[c] = __fmaf_rn(xs[qq], y[c][q + qq], acc[c]);
-                        else { const float df = __fsub_rn(xs[qq], y[c][q + qq]); acc[c] = __fmaf_rn(df, df, acc[c]); }
+                    const unsigned long long xx = pack2(xs[qq], xs[qq]);
+                    if (linear) {
+                        a01 = fma2(xx, y01[q + qq], a01);
+                        a23 = fma2(xx, y23[q + qq], a23);
+                    } else {
+                        const unsigned long long d01 = sub2(xx, y01[q + qq]), d23 = sub2(xx, y23[q + qq]);
+                        a01 = fma2(d01, d01, a01);
+                        a23 = fma2(d23, d23, a23);
                     }
                 }
             }
+            float acc[4];
+            unpack2(a01, acc[0], acc[1]);
+            unpack2(a23, acc[2], acc[3]);
             float4 o;
             float* oc = &o.x;
             const bool rv = I * T + r < N;

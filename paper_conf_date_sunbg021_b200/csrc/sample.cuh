@@ -67,4 +67,13 @@ __global__ void u32_to_i64_kernel(const uint32_t* __restrict__ in, int64_t n, in
         out[j] = (int64_t)in[j];
 }
 
+// *bad = 1 if any of X[0..n) is NaN or +-inf (input validation on the device:
+// a host scan of a 2^20 x 16 pool costs ~10 ms, this ~10 us)
+__global__ void finite_check_kernel(const float* __restrict__ X, int64_t n, int* __restrict__ bad) {
+    bool ok = true;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        ok &= isfinite(X[i]);
+    if (__syncthreads_or(!ok) && threadIdx.x == 0) *bad = 1;
+}
+
 }  // namespace bted

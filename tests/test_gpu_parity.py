@@ -353,3 +353,50 @@ def test_cluster_ted_matches_oracle_across_cluster_sizes(N):
         idx, sc = cs.select(m, MU)
     tr = literal.ted(X, g, MU, m, forced=idx)
     check_ted(idx, sc, tr, f"cluster-{N}")
+
+
+# ------------------------------------------------------------------ full size: oversized batch
+def test_oversized_65536_sampled_against_closed_form():
+    """BASELINE config 'oversized': one TED on N = 65536 (d = 16, m = 64) in
+    the default (packed) layout, checked on sampled outputs one by one with
+    the matrix-free fp64 oracle (oracle/closed_form.py): P1 at EVERY step
+    (the pick's score vs its fp64 score given the same history), and at four
+    steps no sampled candidate beats the pick by more than the 1e-6 gap rule."""
+    from oracle.closed_form import ClosedForm
+    X, g, cfg = config_pool("oversized")
+    V = oracle_sample_batches(X.shape[0], cfg["M"], 1, cfg["seed"])[0]
+    Xb = X[V]
+    m = cfg["m"]
+    with bt.CandidateSet(Xb, g) as cs:
+        idx, sc = cs.select(m, MU)
+    assert len(set(idx.tolist())) == m
+    cf = ClosedForm(Xb, g, MU)
+    rng = np.random.default_rng(65536)
+    for t in range(m):
+        s64 = cf.scores([idx[t]])[0]
+        assert abs(float(sc[t]) - s64) <= 1e-5 * s64, (t, float(sc[t]), s64)          # P1
+        if t in (0, 1, 31, m - 1):
+            cand = rng.choice(cfg["M"], 384, replace=False)
+            cand = np.array([c for c in cand if c not in set(idx[:t].tolist())])
+            other = cf.scores(cand)
+            assert other.max() <= s64 * (1 + 1e-6), (t, other.max(), s64)             # sampled P2
+        cf.add(idx[t])
+
+
+def test_update_replaces_features_and_validates_on_device():
+    X1, X2 = knob(3000, seed=1), knob(3000, seed=2)
+    g = median_gamma(X1, 1)
+    with bt.CandidateSet(X2, g, num_batches=2, seed=4) as ref:
+        want = ref.run_batches(1000, 16, MU)[0]
+    with bt.CandidateSet(X1, g, num_batches=2, seed=4) as cs:
+        first = cs.run_batches(1000, 16, MU)[0]
+        L.bted_update(cs.ctx, X2)
+        assert np.array_equal(cs.run_batches(1000, 16, MU)[0], want)
+        bad = X2.copy()
+        bad[7, 3] = np.inf
+        L.bted_update(cs.ctx, bad)
+        with pytest.raises(bt.BtedError) as e:
+            cs.run_batches(1000, 16, MU)
+        assert e.value.status == 1 and "non-finite" in str(e.value)
+        L.bted_update(cs.ctx, X1)                                   # recovers
+        assert np.array_equal(cs.run_batches(1000, 16, MU)[0], first)

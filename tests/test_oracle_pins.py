@@ -257,3 +257,19 @@ def test_c_oracle_pins_directly():
     X = (np.arange(12, dtype=np.float32) * 100.0)[:, None]
     tr = dense.ted(X, 1.0, MU, 12)
     assert tr.idx == list(range(12))
+
+
+# ------------------------------------------------ matrix-free closed form (full-size sampling)
+def test_closed_form_scores_match_literal():
+    from oracle.closed_form import ClosedForm
+    X = knob_X(500, seed=31)
+    g = median_gamma(X, 31)
+    tr = ted(X, g, MU, 12, keep_scores=True)
+    cf = ClosedForm(X, g, MU)
+    rng = np.random.default_rng(0)
+    for t in range(12):
+        cand = np.unique(np.concatenate([[tr.idx[t]], rng.choice(500, 40, replace=False)]))
+        cand = np.array([c for c in cand if c not in tr.idx[:t]])
+        sc = cf.scores(cand)
+        np.testing.assert_allclose(sc, tr.scores[t][cand], rtol=1e-11)
+        cf.add(tr.idx[t])
