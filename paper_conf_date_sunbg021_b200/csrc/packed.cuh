@@ -198,80 +198,6 @@ __device__ __forceinline__ void write_partials(float* P, int64_t NP, int I, int 
 // One CTA (256 threads) per tile in a persistent loop.  Lane l keeps the
 // features of its 4 columns in registers (kD <= 32); the rows' features
 // are smem broadcasts.
-template <int kD>
-__global__ void __launch_bounds__(kConsumers)
-gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma, int32_t linear,
-                   float* __restrict__ K, int nT, float* __restrict__ P) {
-    __shared__ __align__(16) float xi[T][kD];
-    __shared__ __align__(16) float xj[T][kD];
-    __shared__ __align__(16) float colg[kGroups][T];
-    const int tid = threadIdx.x, w = tid / kWarp, l = tid % kWarp;
-    const int64_t ntiles = num_tiles(nT);
-    const int64_t NP = (int64_t)nT * T;
-    const float ng = -gamma;
-    for (int64_t k = blockIdx.x; k < ntiles; k += gridDim.x) {
-        int I, J;
-        tile_ij(k, nT, I, J);
-        consumer_sync();                                 // previous tile's smem readers are done
-        for (int q = tid; q < T * kD; q += kConsumers) {
-            const int r = q / kD, c = q % kD;
-            const int gi = I * T + r, gj = J * T + r;
-            xi[r][c] = (gi < N && c < d) ? X[(int64_t)gi * d + c] : 0.f;   // zero features add (0-0)^2 = 0
-            xj[r][c] = (gj < N && c < d) ? X[(int64_t)gj * d + c] : 0.f;
-        }
-        consumer_sync();
-        // column features as f32x2 pairs (columns 4l,4l+1 | 4l+2,4l+3): the
-        // distance loop runs on FADD2/FFMA2 (IEEE RN per half: bitwise the
-        // same as the scalar __fsub_rn / __fmaf_rn sequence)
-        unsigned long long y01[kD], y23[kD];
-#pragma unroll
-        for (int q = 0; q < kD; ++q) {
-            y01[q] = pack2(xj[4 * l + 0][q], xj[4 * l + 1][q]);
-            y23[q] = pack2(xj[4 * l + 2][q], xj[4 * l + 3][q]);
-        }
-        float* tile = K + k * (int64_t)(T * T);
-        RowWalk a;
-        a.rowsum = 0.f;
-        for (int rr = 0; rr < 16; ++rr) {
-            const int r = 16 * w + rr;
-            unsigned long long a01 = 0ull, a23 = 0ull;
-#pragma unroll
-            for (int q = 0; q < kD; q += 4) {
-                const float4 xv = *reinterpret_cast<const float4*>(&xi[r][q]);
-                const float xs[4] = {xv.x, xv.y, xv.z, xv.w};
-#pragma unroll
-                for (int qq = 0; qq < 4; ++qq) {
-                    const unsigned long long xx = pack2(xs[qq], xs[qq]);
-                    if (linear) {
-                        a01 = fma2(xx, y01[q + qq], a01);
-                        a23 = fma2(xx, y23[q + qq], a23);
-                    } else {
-                        const unsigned long long d01 = sub2(xx, y01[q + qq]), d23 = sub2(xx, y23[q + qq]);
-                        a01 = fma2(d01, d01, a01);
-                        a23 = fma2(d23, d23, a23);
-                    }
-                }
-            }
-            float acc[4];
-            unpack2(a01, acc[0], acc[1]);
-            unpack2(a23, acc[2], acc[3]);
-            float4 o;
-            float* oc = &o.x;
-            const bool rv = I * T + r < N;
-#pragma unroll
-            for (int c = 0; c < 4; ++c) {
-                const bool cv = J * T + 4 * l + c < N;
-                const float val = linear ? acc[c] : expf(__fmul_rn(ng, acc[c]));
-                oc[c] = (rv && cv) ? val : 0.f;
-            }
-            st_stream(tile + r * T + 4 * l, o);
-            walk_row(a, rr, l, o, colg, w, I != J);
-        }
-        consumer_sync();
-        write_partials(P, NP, I, J, w, l, a, colg, tid);
-    }
-}
-
 // ------------------------------------------------------------------ fin: scores + argmax
 // Alg. 1 l.3 from the partials: g_i = sum_J P[J][i] (J order), score =
 // g / (k(i,i) + mu) with the new diagonal read back from the diagonal tile,
@@ -636,6 +562,164 @@ __device__ __forceinline__ void st_keep(float* p, float v, uint64_t pol) {
     asm volatile("st.global.L2::cache_hint.f32 [%0], %1, %2;" :: "l"(p), "f"(v), "l"(pol) : "memory");
 }
 
+// ------------------------------------------------------------------ in-kernel finish
+// Row block B is complete when all nT of its partials are stored.  The CTA
+// that stores the last one (per-block arrival counter) computes the block's
+// scores: g_i = (sum_{J < nT/2} P[J][i]) + (sum_{J >= nT/2} P[J][i]), each
+// half summed sequentially in J (a fixed order: bitwise reproducible, the
+// same for every row), diag read back from tile (B,B), masked key ->
+// atomicMax.  256 threads: thread (h, r) sums half h of row r.
+struct Fin {
+    const float* P;
+    int64_t NP;
+    int nT, N;
+    const float* K;                 // K_out (diagonal read-back)
+    float mu;
+    const uint8_t* sel;
+    uint32_t s;                     // this step's pivot (excluded); 0xFFFFFFFF for the Gram
+    unsigned int* cnt;              // [nT] arrival counters of this step
+    unsigned long long* key_out;
+    int* err;
+};
+
+__device__ __forceinline__ void finish_block256(const Fin& f, int B, float (*part)[T], unsigned long long* red) {
+    const int tid = threadIdx.x, r = tid % T, h = tid / T;
+    const int half = f.nT / 2;
+    const int j0 = h ? half : 0, j1 = h ? f.nT : half;
+    const float* src = f.P + (int64_t)B * T + r;
+    float acc = 0.f;
+    int J = j0;
+    for (; J + 8 <= j1; J += 8) {
+        float v[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) v[q] = __ldcg(src + (int64_t)(J + q) * f.NP);
+#pragma unroll
+        for (int q = 0; q < 8; ++q) acc = __fadd_rn(acc, v[q]);
+    }
+    for (; J < j1; ++J) acc = __fadd_rn(acc, __ldcg(src + (int64_t)J * f.NP));
+    part[h][r] = acc;
+    __syncthreads();
+    unsigned long long key = 0ull;
+    const int i = B * T + r;
+    if (h == 0 && i < f.N) {
+        const float g = __fadd_rn(part[0][r], part[1][r]);
+        const float diag = __ldcg(f.K + tile_offset(B, B, f.nT) * (T * T) + (int64_t)r * T + r);
+        const bool masked = f.sel[i] != 0 || (uint32_t)i == f.s;
+        key = score_key(g, diag, f.mu, (uint32_t)i, masked, f.err);
+    }
+    key = warp_max_u64(key);
+    const int w = tid / kWarp, l = tid % kWarp;
+    if (l == 0) red[w] = key;
+    __syncthreads();
+    if (tid == 0) {
+        unsigned long long v = 0ull;
+        for (int q = 0; q < kConsumers / kWarp; ++q) v = red[q] > v ? red[q] : v;
+        if (v) atomicMax(f.key_out, v);
+    }
+    __syncthreads();
+}
+
+// All threads of the CTA stored their tile / partials for (I, J).  Count the
+// arrivals (one fence per CTA) and finish the blocks this CTA completed.
+__device__ __forceinline__ void arrive_finish256(const Fin& f, int I, int J, float (*part)[T],
+                                                 unsigned long long* red, int* flag) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        int v = 0;
+        if (atomicAdd(f.cnt + I, 1u) == (unsigned)(f.nT - 1)) v |= 1;
+        if (I != J && atomicAdd(f.cnt + J, 1u) == (unsigned)(f.nT - 1)) v |= 2;
+        if (v) __threadfence();
+        *flag = v;
+    }
+    __syncthreads();
+    const int v = *flag;
+    if (v & 1) { if (threadIdx.x == 0) f.cnt[I] = 0u; finish_block256(f, I, part, red); }
+    if (v & 2) { if (threadIdx.x == 0) f.cnt[J] = 0u; finish_block256(f, J, part, red); }
+}
+
+template <int kD>
+__global__ void __launch_bounds__(kConsumers)
+gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma, int32_t linear,
+                   float* __restrict__ K, int nT, float* __restrict__ P, float mu, const uint8_t* __restrict__ sel,
+                   unsigned int* __restrict__ cnt, unsigned long long* __restrict__ key_out, int* __restrict__ err) {
+    __shared__ float part[2][T];
+    __shared__ unsigned long long red[kConsumers / kWarp];
+    __shared__ int flag;
+    __shared__ __align__(16) float xi[T][kD];
+    __shared__ __align__(16) float xj[T][kD];
+    __shared__ __align__(16) float colg[kGroups][T];
+    const int tid = threadIdx.x, w = tid / kWarp, l = tid % kWarp;
+    const int64_t ntiles = num_tiles(nT);
+    const int64_t NP = (int64_t)nT * T;
+    const float ng = -gamma;
+    {
+        const int64_t k = blockIdx.x;                    // one tile per CTA
+        int I, J;
+        tile_ij(k, nT, I, J);
+        for (int q = tid; q < T * kD; q += kConsumers) {
+            const int r = q / kD, c = q % kD;
+            const int gi = I * T + r, gj = J * T + r;
+            xi[r][c] = (gi < N && c < d) ? X[(int64_t)gi * d + c] : 0.f;   // zero features add (0-0)^2 = 0
+            xj[r][c] = (gj < N && c < d) ? X[(int64_t)gj * d + c] : 0.f;
+        }
+        consumer_sync();
+        // column features as f32x2 pairs (columns 4l,4l+1 | 4l+2,4l+3): the
+        // distance loop runs on FADD2/FFMA2 (IEEE RN per half: bitwise the
+        // same as the scalar __fsub_rn / __fmaf_rn sequence)
+        unsigned long long y01[kD], y23[kD];
+#pragma unroll
+        for (int q = 0; q < kD; ++q) {
+            y01[q] = pack2(xj[4 * l + 0][q], xj[4 * l + 1][q]);
+            y23[q] = pack2(xj[4 * l + 2][q], xj[4 * l + 3][q]);
+        }
+        float* tile = K + k * (int64_t)(T * T);
+        RowWalk a;
+        a.rowsum = 0.f;
+        for (int rr = 0; rr < 16; ++rr) {
+            const int r = 16 * w + rr;
+            unsigned long long a01 = 0ull, a23 = 0ull;
+#pragma unroll
+            for (int q = 0; q < kD; q += 4) {
+                const float4 xv = *reinterpret_cast<const float4*>(&xi[r][q]);
+                const float xs[4] = {xv.x, xv.y, xv.z, xv.w};
+#pragma unroll
+                for (int qq = 0; qq < 4; ++qq) {
+                    const unsigned long long xx = pack2(xs[qq], xs[qq]);
+                    if (linear) {
+                        a01 = fma2(xx, y01[q + qq], a01);
+                        a23 = fma2(xx, y23[q + qq], a23);
+                    } else {
+                        const unsigned long long d01 = sub2(xx, y01[q + qq]), d23 = sub2(xx, y23[q + qq]);
+                        a01 = fma2(d01, d01, a01);
+                        a23 = fma2(d23, d23, a23);
+                    }
+                }
+            }
+            float acc[4];
+            unpack2(a01, acc[0], acc[1]);
+            unpack2(a23, acc[2], acc[3]);
+            float4 o;
+            float* oc = &o.x;
+            const bool rv = I * T + r < N;
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                const bool cv = J * T + 4 * l + c < N;
+                const float val = linear ? acc[c] : expf(__fmul_rn(ng, acc[c]));
+                oc[c] = (rv && cv) ? val : 0.f;
+            }
+            st_stream(tile + r * T + 4 * l, o);
+            walk_row(a, rr, l, o, colg, w, I != J);
+        }
+        consumer_sync();
+        write_partials(P, NP, I, J, w, l, a, colg, tid);
+        const Fin f{P, NP, nT, N, K, mu, sel, 0xFFFFFFFFu, cnt, key_out, err};
+        arrive_finish256(f, I, J, part, red, &flag);
+    }
+    (void)ntiles;
+}
+
+
 // ------------------------------------------------------------------ K2p (LDG variant)
 // One CTA (256 threads) per tile, non-persistent (the hardware scheduler
 // balances 8256+ tiles over the SMs; several CTAs per SM keep many 256-bit
@@ -646,9 +730,12 @@ __device__ __forceinline__ void st_keep(float* p, float v, uint64_t pol) {
 template <int kU>
 __global__ void __launch_bounds__(kConsumers)
 deflate_packed_ldg_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, int nT, int32_t N,
-                          float* __restrict__ P, const unsigned long long* __restrict__ keys, int32_t t, float mu,
-                          uint8_t* __restrict__ sel) {
+                          float* __restrict__ P, unsigned long long* __restrict__ keys, int32_t t, float mu,
+                          uint8_t* __restrict__ sel, unsigned int* __restrict__ cnt, int* __restrict__ err) {
     __shared__ __align__(16) float cgs[kGroups][T];
+    __shared__ float part[2][T];
+    __shared__ unsigned long long red[kConsumers / kWarp];
+    __shared__ int flag;
     const int tid = threadIdx.x, w = tid / kWarp, l = tid % kWarp;
     const int hw = l >> 4, hl = l & 15, c8 = 8 * hl;
     const int64_t k = blockIdx.x;
@@ -724,6 +811,8 @@ deflate_packed_ldg_kernel(const float* __restrict__ Kin, float* __restrict__ Kou
         __syncthreads();
         if (tid < T) st_keep(P + (int64_t)I * NP + (int64_t)J * T + tid, tree32_smem(&cgs[0][tid], T), keep);
     }
+    const Fin f{P, NP, nT, N, Kout, mu, sel, s, cnt, keys + t, err};
+    arrive_finish256(f, I, J, part, red, &flag);
 }
 
 }  // namespace pk

@@ -288,7 +288,11 @@ def test_launch_counter_counts_kernels():
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3, flags=PACKED) as cs:
         cs.select(10, MU)
-    assert bt.bted_kernel_launches() - before == 20          # K1p + fin + 9 x (K2p + fin)
+    assert bt.bted_kernel_launches() - before == 10          # K1p + 9 x K2p (scores finished in-kernel)
+    before = bt.bted_kernel_launches()
+    with bt.CandidateSet(X, 0.3, flags=PACKED_TMA) as cs:
+        cs.select(10, MU)
+    assert bt.bted_kernel_launches() - before == 19          # K1p + 9 x (TMA K2p + finalize)
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3) as cs:
         cs.select(10, MU)
