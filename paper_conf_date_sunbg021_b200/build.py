@@ -40,7 +40,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     cmd = [nvcc(), *NVCC_FLAGS, *SOURCES, "-o", LIB]
     res = subprocess.run(cmd, capture_output=True, text=True)
     if res.returncode != 0:
-        raise RuntimeError(f"nvcc failed ({res.returncode}):\n{res.stderr[-4000:]}")
+        errs = [ln for ln in res.stderr.splitlines() if "error" in ln.lower() or "warning" in ln.lower()]
+        raise RuntimeError(f"nvcc failed ({res.returncode}):\n" + "\n".join(errs[:40]))
     with open(os.path.join(HERE, "ptxas_info.txt"), "w") as f:
         f.write(res.stderr)
     if verbose:

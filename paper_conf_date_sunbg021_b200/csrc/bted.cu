@@ -492,7 +492,10 @@ bool take_xbad(bted_ctx* ctx) {
     int v = 0;
     CK(cudaMemcpy(&v, ctx->xbad, sizeof(int), cudaMemcpyDeviceToHost));
     if (v) {
+        // the run on the bad features may also have raised the numeric flags: clear all
         CK(cudaMemset(ctx->xbad, 0, sizeof(int)));
+        if (ctx->ted.err) CK(cudaMemset(ctx->ted.err, 0, sizeof(int)));
+        if (ctx->bted_engine.err) CK(cudaMemset(ctx->bted_engine.err, 0, sizeof(int)));
         set_error("X has non-finite entries (bted_update)");
     }
     return v != 0;

@@ -643,9 +643,7 @@ __global__ void __launch_bounds__(kConsumers)
 gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma, int32_t linear,
                    float* __restrict__ K, int nT, float* __restrict__ P, float mu, const uint8_t* __restrict__ sel,
                    unsigned int* __restrict__ cnt, unsigned long long* __restrict__ key_out, int* __restrict__ err) {
-    __shared__ float part[2][T];
-    __shared__ unsigned long long red[kConsumers / kWarp];
-    __shared__ int flag;
+
     __shared__ __align__(16) float xi[T][kD];
     __shared__ __align__(16) float xj[T][kD];
     __shared__ __align__(16) float colg[kGroups][T];
@@ -714,7 +712,10 @@ gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamm
         consumer_sync();
         write_partials(P, NP, I, J, w, l, a, colg, tid);
         const Fin f{P, NP, nT, N, K, mu, sel, 0xFFFFFFFFu, cnt, key_out, err};
-        arrive_finish256(f, I, J, part, red, &flag);
+        // xi / xj / colg are free after the row loop and the column tree: the
+        // finisher's scratch lives there (static smem stays under 48 KiB at kD = 32)
+        arrive_finish256(f, I, J, reinterpret_cast<float (*)[T]>(&xi[0][0]),
+                         reinterpret_cast<unsigned long long*>(&xj[0][0]), reinterpret_cast<int*>(&xj[T / 2][0]));
     }
     (void)ntiles;
 }

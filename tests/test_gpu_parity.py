@@ -284,19 +284,19 @@ def test_launch_counter_counts_kernels():
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3, flags=DENSE) as cs:
         cs.select(10, MU)
-    assert bt.bted_kernel_launches() - before == 11          # transpose + K1 + 9 x K2
+    assert bt.bted_kernel_launches() - before == 1 + 11      # finite check + transpose + K1 + 9 x K2
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3, flags=PACKED) as cs:
         cs.select(10, MU)
-    assert bt.bted_kernel_launches() - before == 10          # K1p + 9 x K2p (scores finished in-kernel)
+    assert bt.bted_kernel_launches() - before == 1 + 10      # finite check + K1p + 9 x K2p (finished in-kernel)
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3, flags=PACKED_TMA) as cs:
         cs.select(10, MU)
-    assert bt.bted_kernel_launches() - before == 19          # K1p + 9 x (TMA K2p + finalize)
+    assert bt.bted_kernel_launches() - before == 1 + 19      # finite check + K1p + 9 x (TMA K2p + finalize)
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3) as cs:
         cs.select(10, MU)
-    assert bt.bted_kernel_launches() - before == 1           # the whole TED in one cluster kernel
+    assert bt.bted_kernel_launches() - before == 1 + 1       # finite check + the whole TED in one cluster kernel
 
 
 # ------------------------------------------------------------------ packed vs dense layout
