@@ -103,12 +103,9 @@ struct Ted {
     size_t keyscap = 0;
     int* err = nullptr;
     size_t errcap = 0;
-    // packed-symmetric layout (packed.cuh): per-tile norm partials [nT][nT*T],
-    // per-row-block arrival counters [2][nT] (step parity)
+    // packed-symmetric layout (packed.cuh): per-tile norm partials [nT][nT*T]
     float* P = nullptr;
     size_t pcap = 0;
-    unsigned int* cnt = nullptr;
-    size_t cntcap = 0;
     std::list<std::pair<GraphKey, cudaGraphExec_t>> graphs;   // LRU
     int64_t last_rows = 0, last_ld = 0;
     int last_buf = 0;
@@ -132,11 +129,10 @@ struct Ted {
         if (keys) cudaFree(keys);
         if (err) cudaFree(err);
         if (P) cudaFree(P);
-        if (cnt) cudaFree(cnt);
         for (auto& sl : slots) for (auto e : sl.e) cudaEventDestroy(e);
         slots.clear();
         K[0] = K[1] = nullptr; XT = nullptr; sel = nullptr; keys = nullptr; err = nullptr;
-        P = nullptr; cnt = nullptr;
+        P = nullptr;
     }
 
     // Buffers of the packed layout for an N-point TED.
@@ -144,15 +140,14 @@ struct Ted {
         const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
         const size_t tiles = (size_t)bted::pk::num_tiles(nT) * bted::pk::T * bted::pk::T;
         const size_t NP = (size_t)nT * bted::pk::T;
-        const void* before[6] = {K[0], K[1], sel, keys, P, cnt};
+        const void* before[5] = {K[0], K[1], sel, keys, P};
         grow(K[0], kcap[0], tiles);
         if (m > 1) grow(K[1], kcap[1], tiles);
         grow(sel, selcap, NP);
         grow(keys, keyscap, (size_t)std::max(m, 1));
         grow(P, pcap, (size_t)nT * NP);
-        grow(cnt, cntcap, 2 * (size_t)nT);
         if (!err) { grow(err, errcap, 1); CK(cudaMemsetAsync(err, 0, sizeof(int), stream)); }
-        const void* after[6] = {K[0], K[1], sel, keys, P, cnt};
+        const void* after[5] = {K[0], K[1], sel, keys, P};
         if (std::memcmp(before, after, sizeof before) != 0) {
             for (auto& g : graphs) cudaGraphExecDestroy(g.second);
             graphs.clear();
@@ -251,23 +246,30 @@ constexpr int kK2pSub = 64;
 #define K2P_LDG_KERNEL bted::pk::deflate_packed_ldg_kernel<4>
 constexpr size_t kK2pSmem = bted::pk::k2p_smem_bytes(kK2pSub);
 
+void launch_finalize(Ted& T, int64_t N, int nT, const float* Kout, float mu, const unsigned long long* keys,
+                     int32_t t, unsigned long long* key_out) {
+    const unsigned grid = (unsigned)((int64_t)nT * bted::pk::T / bted::pk::kFinRows);
+    bted::pk::finalize_packed_kernel<<<grid, bted::pk::kFinThreads, 0, T.stream>>>(T.P, nT, (int32_t)N, Kout, mu,
+                                                                                  T.sel, keys, t, key_out, T.err);
+}
+
 // Alg. 1 l.1 + first l.3 on the packed tiles.  (2 kernels: K1p, fin)
 void enqueue_head_packed(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m,
                          float mu, unsigned long long* keys) {
     const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
     CK(cudaMemsetAsync(keys, 0, sizeof(unsigned long long) * m, T.stream));
     CK(cudaMemsetAsync(T.sel, 0, (size_t)nT * bted::pk::T, T.stream));
-    CK(cudaMemsetAsync(T.cnt, 0, sizeof(unsigned int) * 2 * nT, T.stream));
     const int64_t tiles = bted::pk::num_tiles(nT);
     const int lin = kernel == BTED_KERNEL_LINEAR ? 1 : 0;
-    // one CTA per tile; the CTA completing a row block finishes its first scores
+    // one CTA per tile, then the first scores from the partials
     if (d <= 16)
         bted::pk::gram_packed_kernel<16><<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
-            X, (int32_t)N, d, gamma, lin, T.K[0], nT, T.P, mu, T.sel, T.cnt, keys, T.err);
+            X, (int32_t)N, d, gamma, lin, T.K[0], nT, T.P);
     else
         bted::pk::gram_packed_kernel<32><<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
-            X, (int32_t)N, d, gamma, lin, T.K[0], nT, T.P, mu, T.sel, T.cnt, keys, T.err);
-    LAUNCHED(1);
+            X, (int32_t)N, d, gamma, lin, T.K[0], nT, T.P);
+    launch_finalize(T, N, nT, T.K[0], mu, keys, 0, keys);
+    LAUNCHED(2);
 }
 
 // Alg. 1 l.2-6 loop on the packed tiles: per step K2p (deflate + partials) and fin.  (2(m-1) kernels)
@@ -278,19 +280,14 @@ void enqueue_loop_packed(Ted& T, int64_t N, int32_t m, float mu, unsigned long l
     for (int32_t t = 1; t < m; ++t) {
         const float* Kin = T.K[(t - 1) & 1];
         float* Kout = T.K[t & 1];
-        if (tma) {
-            // the persistent TMA variant finishes scores in a separate kernel
+        if (tma)
             K2P_TMA_KERNEL<<<grid, bted::pk::kConsumers + 32, kK2pSmem, T.stream>>>(
                 Kin, Kout, nT, (int32_t)N, T.P, keys, t, mu, T.sel);
-            bted::pk::finalize_packed_kernel<<<nT, bted::pk::kFinThreads, 0, T.stream>>>(
-                T.P, nT, (int32_t)N, Kout, mu, T.sel, keys, t, keys + t, T.err);
-            LAUNCHED(2);
-        } else {
-            // one kernel per step: tiles + in-kernel finish of completed row blocks
+        else
             K2P_LDG_KERNEL<<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
-                Kin, Kout, nT, (int32_t)N, T.P, keys, t, mu, T.sel, T.cnt + (size_t)(t & 1) * nT, T.err);
-            LAUNCHED(1);
-        }
+                Kin, Kout, nT, (int32_t)N, T.P, keys, t, mu, T.sel);
+        launch_finalize(T, N, nT, Kout, mu, keys, t, keys + t);
+        LAUNCHED(2);
     }
 }
 
@@ -382,7 +379,7 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
         head();
     } else {
         GraphKey key{X, N, d, m, kernel, 0, packed ? 1 : 0, fbits(mu), fbits(gamma), keys};
-        graph_run(T, key, packed ? 1 : 2, head);
+        graph_run(T, key, 2, head);
     }
     if (sl) CK(cudaEventRecord(sl->e[1], T.stream));
     if (m > 1) {
@@ -390,7 +387,7 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
             loop();
         } else {
             GraphKey key{X, N, d, m, kernel, 1, packed ? (T.tma ? 2 : 1) : 0, fbits(mu), fbits(gamma), keys};
-            graph_run(T, key, (uint64_t)(m - 1) * ((packed && T.tma) ? 2 : 1), loop);
+            graph_run(T, key, (uint64_t)(m - 1) * (packed ? 2 : 1), loop);
         }
     }
     if (sl) CK(cudaEventRecord(sl->e[2], T.stream));

@@ -199,67 +199,54 @@ __device__ __forceinline__ void write_partials(float* P, int64_t NP, int I, int 
 // features of its 4 columns in registers (kD <= 32); the rows' features
 // are smem broadcasts.
 // ------------------------------------------------------------------ fin: scores + argmax
-// Alg. 1 l.3 from the partials: g_i = sum_J P[J][i] (J order), score =
-// g / (k(i,i) + mu) with the new diagonal read back from the diagonal tile,
-// masked (selected / the pivot / padding), packed key -> atomicMax(key_out).
-// One CTA of kFinThreads per row block: the block's partials are staged in
-// smem by all threads (many loads in flight), then thread r < T sums row r
-// sequentially in J order.
-constexpr int kFinThreads = 512;
-constexpr int kFinChunk = 64;                 // J values staged per round (32 KiB)
-constexpr int kFinSplit = 4;                  // 4 threads per row: J ranges combined in a fixed order
+// Alg. 1 l.3 from the partials: g_i = sum_J P[J][i], score = g / (k(i,i) + mu)
+// with the new diagonal read back from the diagonal tile, masked (selected /
+// the pivot / padding), packed key -> atomicMax(key_out).  The sum runs in a
+// fixed order that depends on nT only (the same for every row: exact
+// duplicates still tie): 8 contiguous J ranges, each summed sequentially,
+// then the 8 range sums in order.  CTA = 32 rows x 8 ranges (lane = row, so
+// every load is a coalesced 128-byte row of P); all of a thread's loads are
+// issued before its adds.
+constexpr int kFinThreads = 256;
+constexpr int kFinRows = 32;
 __global__ void __launch_bounds__(kFinThreads)
 finalize_packed_kernel(const float* __restrict__ P, int nT, int32_t N, const float* __restrict__ K, float mu,
                        const uint8_t* __restrict__ sel, const unsigned long long* __restrict__ keys, int32_t t,
                        unsigned long long* __restrict__ key_out, int* __restrict__ err) {
-    __shared__ float stg[kFinChunk][T];
-    __shared__ float part[kFinSplit][T];
-    const int B = blockIdx.x, tid = threadIdx.x;
-    const int r = tid % T, q = tid / T;          // row r, quarter q of each chunk
+    __shared__ float part[8][kFinRows];
+    const int lane = threadIdx.x % 32, w = threadIdx.x / 32;
     const int64_t NP = (int64_t)nT * T;
+    const int i = blockIdx.x * kFinRows + lane;            // row (< nT*T by construction)
     const uint32_t s = t > 0 ? key_index(keys[t - 1]) : 0xFFFFFFFFu;
-    float g = 0.f;
-    // g(row) = sum over chunks c of ( sum_{q} ( sequential sum of chunk c, quarter q ) )
-    for (int J0 = 0; J0 < nT; J0 += kFinChunk) {
-        const int nj = min(kFinChunk, nT - J0);
-        __syncthreads();
-        // all loads of the chunk first (4 float4 per thread), then the smem stores
-        constexpr int kPer = kFinChunk * (T / 4) / kFinThreads;
-        float4 v[kPer];
+    const int per = (nT + 7) / 8;
+    const int j0 = min(nT, w * per), j1 = min(nT, j0 + per);
+    const float* src = P + i;
+    float acc = 0.f;
+    int J = j0;
+    for (; J + 16 <= j1; J += 16) {
+        float v[16];
 #pragma unroll
-        for (int u = 0; u < kPer; ++u) {
-            const int e = tid + u * kFinThreads, jj = e / (T / 4), c4 = e % (T / 4);
-            v[u] = jj < nj ? __ldcg(reinterpret_cast<const float4*>(P + (int64_t)(J0 + jj) * NP + (int64_t)B * T) + c4)
-                           : make_float4(0.f, 0.f, 0.f, 0.f);
-        }
+        for (int q = 0; q < 16; ++q) v[q] = src[(int64_t)(J + q) * NP];
 #pragma unroll
-        for (int u = 0; u < kPer; ++u) {
-            const int e = tid + u * kFinThreads, jj = e / (T / 4), c4 = e % (T / 4);
-            *reinterpret_cast<float4*>(&stg[jj][4 * c4]) = v[u];
-        }
-        __syncthreads();
-        const int per = (nj + kFinSplit - 1) / kFinSplit;
-        const int j0 = q * per, j1 = min(nj, j0 + per);
-        float h = 0.f;
-#pragma unroll 8
-        for (int jj = j0; jj < j1; ++jj) h = __fadd_rn(h, stg[jj][r]);
-        part[q][r] = h;
-        __syncthreads();
-        if (q == 0) {
-            float c = part[0][r];
-#pragma unroll
-            for (int qq = 1; qq < kFinSplit; ++qq) c = __fadd_rn(c, part[qq][r]);
-            g = __fadd_rn(g, c);
-        }
+        for (int q = 0; q < 16; ++q) acc = __fadd_rn(acc, v[q]);
     }
-    unsigned long long key = 0ull;
-    const int i = B * T + r;
-    if (q == 0 && i < N) {
-        const float diag = K[tile_offset(B, B, nT) * (T * T) + (int64_t)r * T + r];
-        const bool masked = sel[i] != 0 || (uint32_t)i == s;
-        key = score_key(g, diag, mu, (uint32_t)i, masked, err);
+    for (; J < j1; ++J) acc = __fadd_rn(acc, src[(int64_t)J * NP]);
+    part[w][lane] = acc;
+    __syncthreads();
+    if (w == 0) {
+        unsigned long long key = 0ull;
+        if (i < N) {
+            float g = part[0][lane];
+#pragma unroll
+            for (int q = 1; q < 8; ++q) g = __fadd_rn(g, part[q][lane]);
+            const int B = i / T, r = i % T;
+            const float diag = K[tile_offset(B, B, nT) * (T * T) + (int64_t)r * T + r];
+            const bool masked = sel[i] != 0 || (uint32_t)i == s;
+            key = score_key(g, diag, mu, (uint32_t)i, masked, err);
+        }
+        key = warp_max_u64(key);
+        if (lane == 0 && key) atomicMax(key_out, key);
     }
-    cta_key_max_to<kFinThreads>(key, key_out);
 }
 
 // ------------------------------------------------------------------ K2p: TMA deflate
@@ -562,87 +549,10 @@ __device__ __forceinline__ void st_keep(float* p, float v, uint64_t pol) {
     asm volatile("st.global.L2::cache_hint.f32 [%0], %1, %2;" :: "l"(p), "f"(v), "l"(pol) : "memory");
 }
 
-// ------------------------------------------------------------------ in-kernel finish
-// Row block B is complete when all nT of its partials are stored.  The CTA
-// that stores the last one (per-block arrival counter) computes the block's
-// scores: g_i = (sum_{J < nT/2} P[J][i]) + (sum_{J >= nT/2} P[J][i]), each
-// half summed sequentially in J (a fixed order: bitwise reproducible, the
-// same for every row), diag read back from tile (B,B), masked key ->
-// atomicMax.  256 threads: thread (h, r) sums half h of row r.
-struct Fin {
-    const float* P;
-    int64_t NP;
-    int nT, N;
-    const float* K;                 // K_out (diagonal read-back)
-    float mu;
-    const uint8_t* sel;
-    uint32_t s;                     // this step's pivot (excluded); 0xFFFFFFFF for the Gram
-    unsigned int* cnt;              // [nT] arrival counters of this step
-    unsigned long long* key_out;
-    int* err;
-};
-
-__device__ __forceinline__ void finish_block256(const Fin& f, int B, float (*part)[T], unsigned long long* red) {
-    const int tid = threadIdx.x, r = tid % T, h = tid / T;
-    const int half = f.nT / 2;
-    const int j0 = h ? half : 0, j1 = h ? f.nT : half;
-    const float* src = f.P + (int64_t)B * T + r;
-    float acc = 0.f;
-    int J = j0;
-    for (; J + 8 <= j1; J += 8) {
-        float v[8];
-#pragma unroll
-        for (int q = 0; q < 8; ++q) v[q] = __ldcg(src + (int64_t)(J + q) * f.NP);
-#pragma unroll
-        for (int q = 0; q < 8; ++q) acc = __fadd_rn(acc, v[q]);
-    }
-    for (; J < j1; ++J) acc = __fadd_rn(acc, __ldcg(src + (int64_t)J * f.NP));
-    part[h][r] = acc;
-    __syncthreads();
-    unsigned long long key = 0ull;
-    const int i = B * T + r;
-    if (h == 0 && i < f.N) {
-        const float g = __fadd_rn(part[0][r], part[1][r]);
-        const float diag = __ldcg(f.K + tile_offset(B, B, f.nT) * (T * T) + (int64_t)r * T + r);
-        const bool masked = f.sel[i] != 0 || (uint32_t)i == f.s;
-        key = score_key(g, diag, f.mu, (uint32_t)i, masked, f.err);
-    }
-    key = warp_max_u64(key);
-    const int w = tid / kWarp, l = tid % kWarp;
-    if (l == 0) red[w] = key;
-    __syncthreads();
-    if (tid == 0) {
-        unsigned long long v = 0ull;
-        for (int q = 0; q < kConsumers / kWarp; ++q) v = red[q] > v ? red[q] : v;
-        if (v) atomicMax(f.key_out, v);
-    }
-    __syncthreads();
-}
-
-// All threads of the CTA stored their tile / partials for (I, J).  Count the
-// arrivals (one fence per CTA) and finish the blocks this CTA completed.
-__device__ __forceinline__ void arrive_finish256(const Fin& f, int I, int J, float (*part)[T],
-                                                 unsigned long long* red, int* flag) {
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();
-        int v = 0;
-        if (atomicAdd(f.cnt + I, 1u) == (unsigned)(f.nT - 1)) v |= 1;
-        if (I != J && atomicAdd(f.cnt + J, 1u) == (unsigned)(f.nT - 1)) v |= 2;
-        if (v) __threadfence();
-        *flag = v;
-    }
-    __syncthreads();
-    const int v = *flag;
-    if (v & 1) { if (threadIdx.x == 0) f.cnt[I] = 0u; finish_block256(f, I, part, red); }
-    if (v & 2) { if (threadIdx.x == 0) f.cnt[J] = 0u; finish_block256(f, J, part, red); }
-}
-
 template <int kD>
 __global__ void __launch_bounds__(kConsumers)
 gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma, int32_t linear,
-                   float* __restrict__ K, int nT, float* __restrict__ P, float mu, const uint8_t* __restrict__ sel,
-                   unsigned int* __restrict__ cnt, unsigned long long* __restrict__ key_out, int* __restrict__ err) {
+                   float* __restrict__ K, int nT, float* __restrict__ P) {
 
     __shared__ __align__(16) float xi[T][kD];
     __shared__ __align__(16) float xj[T][kD];
@@ -711,11 +621,6 @@ gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamm
         }
         consumer_sync();
         write_partials(P, NP, I, J, w, l, a, colg, tid);
-        const Fin f{P, NP, nT, N, K, mu, sel, 0xFFFFFFFFu, cnt, key_out, err};
-        // xi / xj / colg are free after the row loop and the column tree: the
-        // finisher's scratch lives there (static smem stays under 48 KiB at kD = 32)
-        arrive_finish256(f, I, J, reinterpret_cast<float (*)[T]>(&xi[0][0]),
-                         reinterpret_cast<unsigned long long*>(&xj[0][0]), reinterpret_cast<int*>(&xj[T / 2][0]));
     }
     (void)ntiles;
 }
@@ -731,12 +636,9 @@ gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamm
 template <int kU>
 __global__ void __launch_bounds__(kConsumers)
 deflate_packed_ldg_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, int nT, int32_t N,
-                          float* __restrict__ P, unsigned long long* __restrict__ keys, int32_t t, float mu,
-                          uint8_t* __restrict__ sel, unsigned int* __restrict__ cnt, int* __restrict__ err) {
+                          float* __restrict__ P, const unsigned long long* __restrict__ keys, int32_t t, float mu,
+                          uint8_t* __restrict__ sel) {
     __shared__ __align__(16) float cgs[kGroups][T];
-    __shared__ float part[2][T];
-    __shared__ unsigned long long red[kConsumers / kWarp];
-    __shared__ int flag;
     const int tid = threadIdx.x, w = tid / kWarp, l = tid % kWarp;
     const int hw = l >> 4, hl = l & 15, c8 = 8 * hl;
     const int64_t k = blockIdx.x;
@@ -812,8 +714,6 @@ deflate_packed_ldg_kernel(const float* __restrict__ Kin, float* __restrict__ Kou
         __syncthreads();
         if (tid < T) st_keep(P + (int64_t)I * NP + (int64_t)J * T + tid, tree32_smem(&cgs[0][tid], T), keep);
     }
-    const Fin f{P, NP, nT, N, Kout, mu, sel, s, cnt, keys + t, err};
-    arrive_finish256(f, I, J, part, red, &flag);
 }
 
 }  // namespace pk

@@ -95,7 +95,7 @@ int main(int argc, char** argv) {
     run("k2p_ldg<4>", [&] { deflate_packed_ldg_kernel<4><<<(unsigned)num_tiles(nT), kConsumers>>>(A, B, nT, N, P, keys, 1, 0.1f, sel); }, true);
     run("k2p_ldg<8>", [&] { deflate_packed_ldg_kernel<8><<<(unsigned)num_tiles(nT), kConsumers>>>(A, B, nT, N, P, keys, 1, 0.1f, sel); }, true);
     run("k2p_ldg<2>", [&] { deflate_packed_ldg_kernel<2><<<(unsigned)num_tiles(nT), kConsumers>>>(A, B, nT, N, P, keys, 1, 0.1f, sel); }, true);
-    run("finalize", [&] { finalize_packed_kernel<<<nT, kFinThreads>>>(P, nT, N, B, 0.1f, sel, keys, 1, keys + 1, err); }, false);
+    run("finalize", [&] { finalize_packed_kernel<<<nT * T / kFinRows, kFinThreads>>>(P, nT, N, B, 0.1f, sel, keys, 1, keys + 1, err); }, false);
     printf("done N=%d tiles=%lld\n", N, (long long)num_tiles(nT));
     return 0;
 }

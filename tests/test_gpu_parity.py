@@ -288,11 +288,11 @@ def test_launch_counter_counts_kernels():
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3, flags=PACKED) as cs:
         cs.select(10, MU)
-    assert bt.bted_kernel_launches() - before == 1 + 10      # finite check + K1p + 9 x K2p (finished in-kernel)
+    assert bt.bted_kernel_launches() - before == 1 + 20      # finite check + K1p + fin + 9 x (K2p + fin)
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3, flags=PACKED_TMA) as cs:
         cs.select(10, MU)
-    assert bt.bted_kernel_launches() - before == 1 + 19      # finite check + K1p + 9 x (TMA K2p + finalize)
+    assert bt.bted_kernel_launches() - before == 1 + 20      # finite check + K1p + fin + 9 x (TMA K2p + fin)
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3) as cs:
         cs.select(10, MU)
