@@ -66,6 +66,10 @@ typedef enum {
 #define BTED_FLAG_TMA     16u   /* packed layout: stream K through the persistent TMA ring
                                    (cp.async.bulk + mbarrier) instead of the default one-CTA-per-
                                    tile 256-bit-load kernel (which measured faster on B200)   */
+#define BTED_FLAG_IMPLICIT 32u   /* implicit deflation (N2): keep the packed Gram K read-only and
+                                   carry K^(t) = K - L L^T by its fp64 factor L; one K.l pass per
+                                   step (2 N^2 bytes, read only) + O(N m).  Same selections in
+                                   exact arithmetic; fp64 recurrences.  Packed layouts only.   */
 #define BTED_FLAG_TIMING   2u   /* record CUDA events around K1 and the K2 loop of every batch
                                    TED on the ctx stream; read with bted_get_stats()          */
 

@@ -26,6 +26,7 @@
 #include "sample.cuh"
 #include "packed.cuh"
 #include "small.cuh"
+#include "implicit.cuh"
 
 namespace {
 
@@ -106,6 +107,15 @@ struct Ted {
     // packed-symmetric layout (packed.cuh): per-tile norm partials [nT][nT*T]
     float* P = nullptr;
     size_t pcap = 0;
+    // implicit deflation (implicit.cuh): fp64 partials, factor L [NPa][m], l, n, r, h
+    double* P64 = nullptr; size_t p64cap = 0;
+    double* Lf = nullptr; size_t lfcap = 0;
+    double* ell = nullptr; size_t ellcap = 0;
+    double* nv = nullptr; size_t nvcap = 0;
+    double* rd = nullptr; size_t rdcap = 0;
+    double* Hp = nullptr; size_t hpcap = 0;
+    double* hv = nullptr; size_t hvcap = 0;
+    bool implicit = false;
     std::list<std::pair<GraphKey, cudaGraphExec_t>> graphs;   // LRU
     int64_t last_rows = 0, last_ld = 0;
     int last_buf = 0;
@@ -129,10 +139,36 @@ struct Ted {
         if (keys) cudaFree(keys);
         if (err) cudaFree(err);
         if (P) cudaFree(P);
+        for (double* q : {P64, Lf, ell, nv, rd, Hp, hv}) if (q) cudaFree(q);
+        P64 = Lf = ell = nv = rd = Hp = hv = nullptr;
         for (auto& sl : slots) for (auto e : sl.e) cudaEventDestroy(e);
         slots.clear();
         K[0] = K[1] = nullptr; XT = nullptr; sel = nullptr; keys = nullptr; err = nullptr;
         P = nullptr;
+    }
+
+    // Buffers of the implicit-deflation engine for an N-point TED.
+    void reserve_implicit(int64_t N, int32_t m) {
+        const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
+        const size_t tiles = (size_t)bted::pk::num_tiles(nT) * bted::pk::T * bted::pk::T;
+        const size_t NP = (size_t)nT * bted::pk::T, NPa = (NP + 255) / 256 * 256;
+        const void* before[10] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Hp, hv};
+        grow(K[0], kcap[0], tiles);
+        grow(sel, selcap, NPa);
+        grow(keys, keyscap, (size_t)std::max(m, 1));
+        grow(P64, p64cap, (size_t)nT * NP);
+        grow(Lf, lfcap, NPa * (size_t)m);
+        grow(ell, ellcap, NPa);
+        grow(nv, nvcap, NPa);
+        grow(rd, rdcap, NPa);
+        grow(Hp, hpcap, (NPa / 256) * (size_t)(m + 1));
+        grow(hv, hvcap, (size_t)m + 1);
+        if (!err) { grow(err, errcap, 1); CK(cudaMemsetAsync(err, 0, sizeof(int), stream)); }
+        const void* after[10] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Hp, hv};
+        if (std::memcmp(before, after, sizeof before) != 0) {
+            for (auto& g : graphs) cudaGraphExecDestroy(g.second);
+            graphs.clear();
+        }
     }
 
     // Buffers of the packed layout for an N-point TED.
@@ -291,6 +327,49 @@ void enqueue_loop_packed(Ted& T, int64_t N, int32_t m, float mu, unsigned long l
     }
 }
 
+// ---- implicit deflation (implicit.cuh) ----
+// head: K1p (the packed Gram, read-only from now on), fp64 norm pass, scores.  (3 kernels)
+void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m,
+                           float mu, unsigned long long* keys) {
+    const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
+    const int64_t NP = (int64_t)nT * bted::pk::T, NPa = (NP + 255) / 256 * 256;
+    const int64_t tiles = bted::pk::num_tiles(nT);
+    CK(cudaMemsetAsync(keys, 0, sizeof(unsigned long long) * m, T.stream));
+    CK(cudaMemsetAsync(T.sel, 0, (size_t)NPa, T.stream));
+    CK(cudaMemsetAsync(T.Lf, 0, sizeof(double) * NPa * m, T.stream));
+    const int lin = kernel == BTED_KERNEL_LINEAR ? 1 : 0;
+    float* scratch = reinterpret_cast<float*>(T.P64);      // K1p's fp32 partials are not used here
+    if (d <= 16)
+        bted::pk::gram_packed_kernel<16><<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
+            X, (int32_t)N, d, gamma, lin, T.K[0], nT, scratch);
+    else
+        bted::pk::gram_packed_kernel<32><<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
+            X, (int32_t)N, d, gamma, lin, T.K[0], nT, scratch);
+    bted::im::tile_pass_kernel<true><<<(unsigned)tiles, bted::im::kThreads, 0, T.stream>>>(
+        T.K[0], nT, nullptr, T.P64, nullptr, 0, 0, 0, nullptr);
+    bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
+        T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, m, 0, T.hv, T.nv, T.rd, T.sel, keys, 0, keys, T.err);
+    LAUNCHED(3);
+}
+
+// loop: per step the new factor column (A), q = K l over the tiles (B), scores (C).  (3(m-1) kernels)
+void enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned long long* keys) {
+    const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
+    const int64_t NP = (int64_t)nT * bted::pk::T, NPa = (NP + 255) / 256 * 256;
+    const int64_t tiles = bted::pk::num_tiles(nT);
+    const int nA = (int)(NPa / 256);
+    for (int32_t t = 1; t < m; ++t) {
+        const int32_t tp = t - 1;
+        bted::im::ell_kernel<<<nA, bted::im::kThreads, 0, T.stream>>>(T.K[0], nT, (int32_t)N, T.Lf, m, tp, T.rd, mu,
+                                                                      keys, t, T.ell, T.Hp, T.sel);
+        bted::im::tile_pass_kernel<false><<<(unsigned)tiles, bted::im::kThreads, 0, T.stream>>>(
+            T.K[0], nT, T.ell, T.P64, T.Hp, nA, tp + 1, m + 1, T.hv);
+        bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
+            T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, m, tp, T.hv, T.nv, T.rd, T.sel, keys, t, keys + t, T.err);
+        LAUNCHED(3);
+    }
+}
+
 // Alg. 1 l.1 + first l.3: XT, zero keys/sel, K1.  (2 kernels)
 void enqueue_head(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
                   unsigned long long* keys) {
@@ -354,7 +433,11 @@ bool use_packed(uint32_t flags, int32_t d) { return !(flags & BTED_FLAG_DENSE) &
 
 void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
              unsigned long long* keys, bool no_graph, bool time_it = true, bool packed = false) {
-    if (packed) {
+    const bool implicit = packed && T.implicit && m <= bted::im::kMaxM;
+    if (implicit) {
+        T.reserve_implicit(N, m);
+        T.last_nT = (int32_t)((N + bted::pk::T - 1) / bted::pk::T);
+    } else if (packed) {
         ensure_packed_attrs();
         T.reserve_packed(N, m);
         T.last_nT = (int32_t)((N + bted::pk::T - 1) / bted::pk::T);
@@ -362,32 +445,36 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
         T.reserve(N, N, d, m);
     }
     T.last_packed = packed;
-    T.last_rows = N;
+    T.last_rows = implicit ? 0 : N;          // implicit mode never materialises K^(t)
     T.last_ld = ld_for(N);
     T.last_buf = (m - 1) & 1;
     Ted::Slot* sl = (T.timing && time_it) ? T.next_slot(m) : nullptr;
     if (sl) CK(cudaEventRecord(sl->e[0], T.stream));
     auto head = [&] {
-        if (packed) enqueue_head_packed(T, X, N, d, gamma, kernel, m, mu, keys);
+        if (implicit) enqueue_head_implicit(T, X, N, d, gamma, kernel, m, mu, keys);
+        else if (packed) enqueue_head_packed(T, X, N, d, gamma, kernel, m, mu, keys);
         else enqueue_head(T, X, N, d, gamma, kernel, m, mu, keys);
     };
     auto loop = [&] {
-        if (packed) enqueue_loop_packed(T, N, m, mu, keys, T.tma);
+        if (implicit) enqueue_loop_implicit(T, N, m, mu, keys);
+        else if (packed) enqueue_loop_packed(T, N, m, mu, keys, T.tma);
         else enqueue_loop(T, N, m, mu, keys);
     };
+    const int mode = implicit ? 3 : packed ? (T.tma ? 2 : 1) : 0;
+    const uint64_t head_k = implicit ? 3 : 2, loop_k = implicit ? 3 : packed ? 2 : 1;
     if (no_graph) {
         head();
     } else {
-        GraphKey key{X, N, d, m, kernel, 0, packed ? 1 : 0, fbits(mu), fbits(gamma), keys};
-        graph_run(T, key, 2, head);
+        GraphKey key{X, N, d, m, kernel, 0, mode, fbits(mu), fbits(gamma), keys};
+        graph_run(T, key, head_k, head);
     }
     if (sl) CK(cudaEventRecord(sl->e[1], T.stream));
     if (m > 1) {
         if (no_graph) {
             loop();
         } else {
-            GraphKey key{X, N, d, m, kernel, 1, packed ? (T.tma ? 2 : 1) : 0, fbits(mu), fbits(gamma), keys};
-            graph_run(T, key, (uint64_t)(m - 1) * (packed ? 2 : 1), loop);
+            GraphKey key{X, N, d, m, kernel, 1, mode, fbits(mu), fbits(gamma), keys};
+            graph_run(T, key, (uint64_t)(m - 1) * loop_k, loop);
         }
     }
     if (sl) CK(cudaEventRecord(sl->e[2], T.stream));
@@ -580,6 +667,7 @@ bted_status create_common(const float* X, int64_t N, int32_t d, bted_kernel kern
         ctx->bted_engine.stream = ctx->stream;
         ctx->ted.timing = ctx->bted_engine.timing = (params->flags & BTED_FLAG_TIMING) != 0;
         ctx->ted.tma = ctx->bted_engine.tma = (params->flags & BTED_FLAG_TMA) != 0;
+        ctx->ted.implicit = ctx->bted_engine.implicit = (params->flags & BTED_FLAG_IMPLICIT) != 0;
         CK(cudaMallocHost(&ctx->herr, sizeof(int)));
         if (params->x_on_device) {
             ctx->X = const_cast<float*>(X);

@@ -1,0 +1,262 @@
+// implicit.cuh -- implicit deflation on the packed
+// read-only Gram matrix.
+//
+// Algorithm 1 deflates K <- K - K_:s K_s: / (K_ss + mu)
+// every step.  Written as K^(t) = K - L L^T with L = [l_1 .. l_t] (N x t),
+// l_t = K^(t-1)_:s / sqrt(K^(t-1)_ss + mu), the same selections follow from
+// K itself (never rewritten) plus the factor L:
+//
+//   R = K - L L^T (implicit),  l = R_:s / sqrt(R_ss + mu)
+//   l_i   = (K_is - sum_k L_ik L_sk) / sqrt(c)                     (kernel A)
+//   q     = K l  (one pass over the packed tiles, READ ONLY: 2 N^2 B) (kernel B)
+//   (R l)_v = q_v - sum_k L_vk h_k,  h = L^T l,  |l|^2
+//   n_v  <- n_v - 2 l_v (R l)_v + l_v^2 |l|^2      (= ||R'_:v||^2)   (kernel C)
+//   r_vv <- r_vv - l_v^2,   score_v = n_v / (r_vv + mu)
+//
+// Every accumulation is fp64 (K stays the fp32 Gram of K1p), so the
+// recurrence's cancellation costs nothing at the 1e-5 parity tolerance.  A
+// step moves 2 N^2 bytes (packed K, read once) + O(N m) instead of the
+// literal deflation's 4 N^2 (packed) / 8 N^2 (dense).  Sums run in orders
+// that depend on N only (canonical trees as in packed.cuh, fp64), so exact
+// duplicate points still tie to the lowest index.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+#include "kernels.cuh"
+#include "packed.cuh"
+
+namespace bted {
+namespace im {
+
+using pk::T;
+using pk::kGroups;
+using pk::tile_ij;
+using pk::tile_offset;
+using pk::num_tiles;
+using pk::packed_index;
+constexpr int kThreads = 256;
+constexpr int kMaxM = 256;           // factor columns held per step (m <= kMaxM)
+
+__device__ __forceinline__ double warp_sum64(double v) {
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) v = __dadd_rn(v, __shfl_xor_sync(0xffffffffu, v, off));
+    return v;
+}
+
+// ------------------------------------------------------------------ tile pass (fp64 partials)
+// kNorm: row/col partials of K_ij^2 (the initial ||K_:v||^2);  else of K_ij w_j
+// (rows) and K_ij w_i (columns): q = K w.  One CTA (256 threads) per stored
+// tile; warp w: rows 16w..16w+15, half-warp h: rows 16w+8h..+7, lane hl:
+// columns 8hl..8hl+7.  Canonical per-128 tree: groups of 4 consecutive terms
+// (sequential), then the 32-leaf butterfly.
+template <bool kNorm>
+__global__ void __launch_bounds__(kThreads)
+tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__ w, double* __restrict__ P64,
+                 const double* __restrict__ Hpart, int nHpart, int nh, int hstride, double* __restrict__ h) {
+    __shared__ double cgs[kGroups][T];                 // 32 KiB: column groups
+    __shared__ double wi[T];                           // w on the tile's rows
+    const int tid = threadIdx.x, w_ = tid / 32, l = tid % 32;
+    const int hw = l >> 4, hl = l & 15, c8 = 8 * hl;
+    const int64_t k = blockIdx.x;
+    int I, J;
+    tile_ij(k, nT, I, J);
+    const int64_t NP = (int64_t)nT * T;
+    // kernel A left per-CTA partials of h = L^T l and |l|^2: CTA 0 reduces them
+    // in CTA order for kernel C (fixed order, deterministic)
+    if (!kNorm && k == 0 && tid < nh) {
+        double a = 0.0;
+        for (int b = 0; b < nHpart; ++b) a = __dadd_rn(a, Hpart[(int64_t)b * hstride + tid]);
+        h[tid] = a;
+    }
+    double wc[8];
+    if (!kNorm) {
+        if (tid < T) wi[tid] = w[(int64_t)I * T + tid];
+#pragma unroll
+        for (int c = 0; c < 8; ++c) wc[c] = w[(int64_t)J * T + c8 + c];
+        __syncthreads();
+    }
+    const float* gin = K + k * (int64_t)(T * T);
+    double rowsum = 0.0;
+    double cg[8];
+#pragma unroll
+    for (int r0 = 0; r0 < 8; r0 += 4) {
+        f8 kv[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) kv[u] = ld8_stream(gin + (16 * w_ + 8 * hw + r0 + u) * T + c8);
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const int rr = r0 + u;
+            const int r = 16 * w_ + 8 * hw + rr;
+            double x[8];
+            const double wr = kNorm ? 0.0 : wi[r];
+#pragma unroll
+            for (int c = 0; c < 8; ++c) {
+                const double kij = (double)kv[u].v[c];
+                x[c] = kNorm ? kij : kij * wc[c];       // row term factor: K_ij * (K_ij | w_j)
+            }
+            double ga, gb;
+            if (kNorm) {
+                ga = __dmul_rn(x[0], x[0]); ga = __fma_rn(x[1], x[1], ga); ga = __fma_rn(x[2], x[2], ga); ga = __fma_rn(x[3], x[3], ga);
+                gb = __dmul_rn(x[4], x[4]); gb = __fma_rn(x[5], x[5], gb); gb = __fma_rn(x[6], x[6], gb); gb = __fma_rn(x[7], x[7], gb);
+            } else {
+                const double k0 = (double)kv[u].v[0], k1 = (double)kv[u].v[1], k2 = (double)kv[u].v[2], k3 = (double)kv[u].v[3];
+                const double k4 = (double)kv[u].v[4], k5 = (double)kv[u].v[5], k6 = (double)kv[u].v[6], k7 = (double)kv[u].v[7];
+                ga = __dmul_rn(k0, wc[0]); ga = __fma_rn(k1, wc[1], ga); ga = __fma_rn(k2, wc[2], ga); ga = __fma_rn(k3, wc[3], ga);
+                gb = __dmul_rn(k4, wc[4]); gb = __fma_rn(k5, wc[5], gb); gb = __fma_rn(k6, wc[6], gb); gb = __fma_rn(k7, wc[7], gb);
+            }
+#pragma unroll
+            for (int off = 8; off > 0; off >>= 1) {
+                ga = __dadd_rn(ga, __shfl_xor_sync(0xffffffffu, ga, off));
+                gb = __dadd_rn(gb, __shfl_xor_sync(0xffffffffu, gb, off));
+            }
+            const double rp = __dadd_rn(ga, gb);
+            const double rq0 = __shfl_sync(0xffffffffu, rp, 0), rq1 = __shfl_sync(0xffffffffu, rp, 16);
+            if (l == rr) rowsum = rq0;
+            if (l == 8 + rr) rowsum = rq1;
+            if (I != J) {
+#pragma unroll
+                for (int c = 0; c < 8; ++c) {
+                    const double kij = (double)kv[u].v[c];
+                    const double f = kNorm ? kij : wr;   // column term: K_ij * (K_ij | w_i)
+                    cg[c] = (rr & 3) == 0 ? __dmul_rn(kij, f) : __fma_rn(kij, f, cg[c]);
+                }
+                if ((rr & 3) == 3) {
+#pragma unroll
+                    for (int c = 0; c < 8; ++c) cgs[r >> 2][c8 + c] = cg[c];
+                }
+            }
+            (void)x;
+        }
+    }
+    if (l < 16) P64[(int64_t)J * NP + (int64_t)I * T + 16 * w_ + l] = rowsum;
+    if (I != J) {
+        __syncthreads();
+        if (tid < T) {
+            double hh[kGroups];
+#pragma unroll
+            for (int q = 0; q < kGroups; ++q) hh[q] = cgs[q][tid];
+#pragma unroll
+            for (int off = 16; off > 0; off >>= 1)
+#pragma unroll
+                for (int q = 0; q < off; ++q) hh[q] = __dadd_rn(hh[q], hh[q + off]);
+            P64[(int64_t)I * NP + (int64_t)J * T + tid] = hh[0];
+        }
+    }
+}
+
+// ------------------------------------------------------------------ kernel A: the new factor column
+// l_i = (K_is - sum_{k<tp} L_ik L_sk) / sqrt(r_ss + mu) for every row i (0 on
+// padding), L[:, tp] = l, ell = l; per-CTA partials of h_k = sum_i L_ik l_i
+// (k < tp) and of |l|^2 (slot tp) for the tile pass to reduce.
+__global__ void __launch_bounds__(kThreads)
+ell_kernel(const float* __restrict__ K, int nT, int32_t N, double* __restrict__ L, int32_t ldL, int32_t tp,
+           const double* __restrict__ rdiag, float mu, const unsigned long long* __restrict__ keys, int32_t t,
+           double* __restrict__ ell, double* __restrict__ Hpart, uint8_t* __restrict__ sel) {
+    __shared__ double Ls[kMaxM];
+    __shared__ double red[kThreads / 32][65];
+    const int tid = threadIdx.x, w = tid / 32, l = tid % 32;
+    const int i = blockIdx.x * kThreads + tid;         // L / ell have round_up(nT*T, 256) rows
+    const uint32_t s = key_index(keys[t - 1]);
+    if (blockIdx.x == 0 && tid == 0) sel[s] = 1;
+    for (int q = tid; q < tp; q += kThreads) Ls[q] = L[(int64_t)s * ldL + q];
+    __syncthreads();
+    const double c = __dadd_rn(rdiag[s], (double)mu);
+    double li = 0.0;
+    if (i < N) {
+        double a = (double)K[packed_index(i, (int)s, nT)];
+        const double* Li = L + (int64_t)i * ldL;
+        for (int q = 0; q < tp; ++q) a = __fma_rn(-Li[q], Ls[q], a);
+        li = __ddiv_rn(a, __dsqrt_rn(c));
+    }
+    L[(int64_t)i * ldL + tp] = li;
+    ell[i] = li;
+    // per-CTA partial sums (warp butterfly, then warps in order) of L_ik l_i and l_i^2
+    const double* Li = L + (int64_t)i * ldL;
+    for (int q = 0; q <= tp; ++q) {
+        const double x = q < tp ? __dmul_rn(Li[q], li) : __dmul_rn(li, li);
+        const double ws = warp_sum64(x);
+        if (l == 0) red[w][q & 63] = ws;
+        if ((q & 63) == 63 || q == tp) {
+            __syncthreads();
+            const int qbase = q & ~63;
+            for (int qq = tid; qq <= q - qbase; qq += kThreads) {
+                double a = 0.0;
+                for (int ww = 0; ww < kThreads / 32; ++ww) a = __dadd_rn(a, red[ww][qq]);
+                Hpart[(int64_t)blockIdx.x * (ldL + 1) + qbase + qq] = a;
+            }
+            __syncthreads();
+        }
+    }
+}
+
+// ------------------------------------------------------------------ kernel C: scores
+// t == 0 (after the norm pass): n_v = q_v (= ||K_:v||^2), r_vv = K_vv.
+// t >= 1: (R l)_v = q_v - sum_{k<tp} L_vk h_k; n_v -= 2 l_v (R l)_v - l_v^2 |l|^2;
+// r_vv -= l_v^2.  Score n_v / (r_vv + mu) rounded to fp32, masked, packed key.
+constexpr int kFinRows = 32;
+__global__ void __launch_bounds__(kThreads)
+fin64_kernel(const double* __restrict__ P64, int nT, int32_t N, const float* __restrict__ K, float mu,
+             const double* __restrict__ L, int32_t ldL, int32_t tp, const double* __restrict__ h,
+             double* __restrict__ nv, double* __restrict__ rdiag, const uint8_t* __restrict__ sel,
+             const unsigned long long* __restrict__ keys, int32_t t, unsigned long long* __restrict__ key_out,
+             int* __restrict__ err) {
+    __shared__ double part[8][kFinRows];
+    __shared__ double hs[kMaxM + 1];
+    const int lane = threadIdx.x % 32, w = threadIdx.x / 32;
+    const int64_t NP = (int64_t)nT * T;
+    const int i = blockIdx.x * kFinRows + lane;
+    if (t > 0)
+        for (int q = threadIdx.x; q <= tp; q += kThreads) hs[q] = h[q];
+    const int per = (nT + 7) / 8;
+    const int j0 = min(nT, w * per), j1 = min(nT, j0 + per);
+    const double* src = P64 + i;
+    double acc = 0.0;
+    int J = j0;
+    for (; J + 8 <= j1; J += 8) {
+        double v[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) v[q] = src[(int64_t)(J + q) * NP];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) acc = __dadd_rn(acc, v[q]);
+    }
+    for (; J < j1; ++J) acc = __dadd_rn(acc, src[(int64_t)J * NP]);
+    part[w][lane] = acc;
+    __syncthreads();
+    if (w != 0) return;
+    unsigned long long key = 0ull;
+    if (i < N) {
+        double q = part[0][lane];
+#pragma unroll
+        for (int u = 1; u < 8; ++u) q = __dadd_rn(q, part[u][lane]);
+        const uint32_t s = t > 0 ? key_index(keys[t - 1]) : 0xFFFFFFFFu;
+        double n, r;
+        if (t == 0) {
+            const int B = i / T, rr = i % T;
+            n = q;
+            r = (double)K[tile_offset(B, B, nT) * (T * T) + (int64_t)rr * T + rr];
+        } else {
+            const double* Li = L + (int64_t)i * ldL;
+            double rl = q;
+            for (int k = 0; k < tp; ++k) rl = __fma_rn(-Li[k], hs[k], rl);
+            const double lv = Li[tp];
+            n = nv[i];
+            n = __fma_rn(-2.0 * lv, rl, n);
+            n = __fma_rn(__dmul_rn(lv, lv), hs[tp], n);
+            r = __fma_rn(-lv, lv, rdiag[i]);
+        }
+        nv[i] = n;
+        rdiag[i] = r;
+        const bool masked = sel[i] != 0 || (uint32_t)i == s;
+        const float sc = (float)(__ddiv_rn(n > 0.0 ? n : 0.0, __dadd_rn(r, (double)mu)));
+        if (!(__dadd_rn(r, (double)mu) > 0.0) || !(sc >= 0.f) || !(sc <= 3.402823466e38f)) {
+            if (!masked) atomicOr(err, 1);
+        } else if (!masked) {
+            key = pack_key(sc, (uint32_t)i);
+        }
+    }
+    key = warp_max_u64(key);
+    if (lane == 0 && key) atomicMax(key_out, key);
+}
+
+}  // namespace im
+}  // namespace bted

@@ -11,6 +11,7 @@ timeout 120 python scripts/h2d_probe.py > $OUT/h2d.txt 2>&1
 timeout 300 python __graft_entry__.py smoke > $OUT/smoke.log 2>&1; echo "smoke rc=$?" >> $OUT/smoke.log
 timeout 900 python bench.py --steps 10 --warmup 3 > $OUT/bench.json 2> $OUT/bench.err; echo "bench rc=$?" >> $OUT/bench.err
 timeout 900 python bench.py --steps 10 --warmup 3 --layout dense --no-cpu-baseline > $OUT/bench_dense.json 2> $OUT/bench_dense.err
+timeout 900 python bench.py --steps 10 --warmup 3 --layout implicit --no-cpu-baseline > $OUT/bench_implicit.json 2> $OUT/bench_implicit.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
     python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_launches.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"deflate_packed|finalize_packed" -s 16 -c 2 \

@@ -18,7 +18,9 @@ MU = float(np.float32(0.1))
 PACKED = L.BTED_FLAG_NO_SMALL
 DENSE = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_DENSE
 PACKED_TMA = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_TMA
-LAYOUTS = pytest.mark.parametrize("flags", [PACKED, PACKED_TMA, DENSE, 0], ids=["packed", "packed-tma", "dense", "auto"])
+IMPLICIT = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_IMPLICIT
+LAYOUTS = pytest.mark.parametrize("flags", [PACKED, PACKED_TMA, DENSE, IMPLICIT, 0],
+                                  ids=["packed", "packed-tma", "dense", "implicit", "auto"])
 LAYOUTS_K = pytest.mark.parametrize("flags", [PACKED, PACKED_TMA, DENSE], ids=["packed", "packed-tma", "dense"])
 
 
@@ -307,7 +309,9 @@ def test_packed_layout_matches_dense(N, d, m):
     X = knob(N, d=16, seed=N)[:, :d] if d <= 16 else uniform_pool(N, d, N)
     g = median_gamma(X, d)
     with bt.CandidateSet(X, g, flags=DENSE) as cd, bt.CandidateSet(X, g, flags=PACKED) as cp, \
-            bt.CandidateSet(X, g, flags=PACKED_TMA) as ct:
+            bt.CandidateSet(X, g, flags=PACKED_TMA) as ct, bt.CandidateSet(X, g, flags=IMPLICIT) as ci:
+        i_i, s_i = ci.select(m, MU)
+        check_ted(i_i, s_i, dense.ted(X, g, MU, m, forced=i_i), f"implicit-{N}")
         i_d, s_d = cd.select(m, MU)
         i_p, s_p = cp.select(m, MU)
         i_t, s_t = ct.select(m, MU)
@@ -346,6 +350,19 @@ def test_paper_scale_bted_vs_oracle():
     check_ted(mpos, [], literal.ted(X[XU], g, MU, len(sel), forced=mpos), "paper-merge")
     # one cluster launch for all 10 batch TEDs + one for the merge (+ sampling/gather/union kernels)
     assert launched < 60
+
+
+@pytest.mark.parametrize("N,m", [(1000, 64), (4099, 64), (300, 256), (2000, 200)])
+def test_implicit_deflation_matches_oracle(N, m):
+    """N2: K read-only + fp64 factor recurrences -> same picks as the oracle."""
+    X = knob(N, seed=N + 11)
+    g = median_gamma(X, N)
+    with bt.CandidateSet(X, g, flags=IMPLICIT) as cs:
+        idx, sc = cs.select(m, MU)
+        idx2, sc2 = cs.select(m, MU)
+    assert np.array_equal(idx, idx2) and np.array_equal(sc.view(np.uint32), sc2.view(np.uint32))
+    tr = dense.ted(X, g, MU, m, forced=idx)
+    check_ted(idx, sc, tr, f"implicit-{N}")
 
 
 @pytest.mark.parametrize("N", [1, 5, 64, 230, 231, 500, 640, 777, 940])
