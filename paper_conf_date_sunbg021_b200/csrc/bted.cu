@@ -161,7 +161,7 @@ struct Ted {
         grow(ell, ellcap, NPa);
         grow(nv, nvcap, NPa);
         grow(rd, rdcap, NPa);
-        grow(Hp, hpcap, (NPa / 256) * (size_t)(m + 1));
+        grow(Hp, hpcap, (NPa / bted::im::kEllRows) * (size_t)(m + 1));
         grow(hv, hvcap, (size_t)m + 1);
         if (!err) { grow(err, errcap, 1); CK(cudaMemsetAsync(err, 0, sizeof(int), stream)); }
         const void* after[10] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Hp, hv};
@@ -357,7 +357,7 @@ void enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned long
     const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
     const int64_t NP = (int64_t)nT * bted::pk::T, NPa = (NP + 255) / 256 * 256;
     const int64_t tiles = bted::pk::num_tiles(nT);
-    const int nA = (int)(NPa / 256);
+    const int nA = (int)(NPa / bted::im::kEllRows);
     for (int32_t t = 1; t < m; ++t) {
         const int32_t tp = t - 1;
         bted::im::ell_kernel<<<nA, bted::im::kThreads, 0, T.stream>>>(T.K[0], nT, (int32_t)N, T.Lf, m, tp, T.rd, mu,

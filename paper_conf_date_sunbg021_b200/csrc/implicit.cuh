@@ -53,7 +53,10 @@ template <bool kNorm>
 __global__ void __launch_bounds__(kThreads)
 tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__ w, double* __restrict__ P64,
                  const double* __restrict__ Hpart, int nHpart, int nh, int hstride, double* __restrict__ h) {
-    __shared__ double cgs[kGroups][T];                 // 32 KiB: column groups
+    // column groups, layout [q][c][hl] (group q, lane hl, its column 8hl+c): a
+    // half-warp stores 16 consecutive doubles per c; tree thread tid reads
+    // [q][tid] and owns column 8*(tid&15) + (tid>>4).  No bank conflicts.
+    __shared__ double cgs[kGroups * T];                // 32 KiB
     __shared__ double wi[T];                           // w on the tile's rows
     const int tid = threadIdx.x, w_ = tid / 32, l = tid % 32;
     const int hw = l >> 4, hl = l & 15, c8 = 8 * hl;
@@ -63,10 +66,20 @@ tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__
     const int64_t NP = (int64_t)nT * T;
     // kernel A left per-CTA partials of h = L^T l and |l|^2: CTA 0 reduces them
     // in CTA order for kernel C (fixed order, deterministic)
-    if (!kNorm && k == 0 && tid < nh) {
+    if (!kNorm && k < nh) {
+        // CTA k reduces column k of Hpart (nHpart CTA partials): thread-strided
+        // sequential sums, then a fixed tree over the 256 threads
         double a = 0.0;
-        for (int b = 0; b < nHpart; ++b) a = __dadd_rn(a, Hpart[(int64_t)b * hstride + tid]);
-        h[tid] = a;
+        for (int b = tid; b < nHpart; b += kThreads) a = __dadd_rn(a, Hpart[(int64_t)b * hstride + k]);
+        a = warp_sum64(a);
+        if (l == 0) cgs[w_] = a;
+        __syncthreads();
+        if (tid == 0) {
+            double v = 0.0;
+            for (int q = 0; q < kThreads / 32; ++q) v = __dadd_rn(v, cgs[q]);
+            h[k] = v;
+        }
+        __syncthreads();
     }
     double wc[8];
     if (!kNorm) {
@@ -122,7 +135,7 @@ tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__
                 }
                 if ((rr & 3) == 3) {
 #pragma unroll
-                    for (int c = 0; c < 8; ++c) cgs[r >> 2][c8 + c] = cg[c];
+                    for (int c = 0; c < 8; ++c) cgs[(r >> 2) * T + c * 16 + hl] = cg[c];
                 }
             }
             (void)x;
@@ -134,12 +147,12 @@ tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__
         if (tid < T) {
             double hh[kGroups];
 #pragma unroll
-            for (int q = 0; q < kGroups; ++q) hh[q] = cgs[q][tid];
+            for (int q = 0; q < kGroups; ++q) hh[q] = cgs[q * T + tid];
 #pragma unroll
             for (int off = 16; off > 0; off >>= 1)
 #pragma unroll
                 for (int q = 0; q < off; ++q) hh[q] = __dadd_rn(hh[q], hh[q + off]);
-            P64[(int64_t)I * NP + (int64_t)J * T + tid] = hh[0];
+            P64[(int64_t)I * NP + (int64_t)J * T + 8 * (tid & 15) + (tid >> 4)] = hh[0];
         }
     }
 }
@@ -147,45 +160,60 @@ tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__
 // ------------------------------------------------------------------ kernel A: the new factor column
 // l_i = (K_is - sum_{k<tp} L_ik L_sk) / sqrt(r_ss + mu) for every row i (0 on
 // padding), L[:, tp] = l, ell = l; per-CTA partials of h_k = sum_i L_ik l_i
-// (k < tp) and of |l|^2 (slot tp) for the tile pass to reduce.
+// (k < tp) and of |l|^2 (slot tp), reduced by the tile pass.  A warp takes
+// kRowsPerWarp rows; lane j holds factor columns j, j+32, ... (kMaxM / 32).
+constexpr int kRowsPerWarp = 4;
+constexpr int kEllRows = (kThreads / 32) * kRowsPerWarp;      // 32 rows per CTA
 __global__ void __launch_bounds__(kThreads)
 ell_kernel(const float* __restrict__ K, int nT, int32_t N, double* __restrict__ L, int32_t ldL, int32_t tp,
            const double* __restrict__ rdiag, float mu, const unsigned long long* __restrict__ keys, int32_t t,
            double* __restrict__ ell, double* __restrict__ Hpart, uint8_t* __restrict__ sel) {
-    __shared__ double Ls[kMaxM];
-    __shared__ double red[kThreads / 32][65];
+    constexpr int kC = kMaxM / 32;
+    __shared__ double part[kThreads / 32][kMaxM + 1];
     const int tid = threadIdx.x, w = tid / 32, l = tid % 32;
-    const int i = blockIdx.x * kThreads + tid;         // L / ell have round_up(nT*T, 256) rows
     const uint32_t s = key_index(keys[t - 1]);
     if (blockIdx.x == 0 && tid == 0) sel[s] = 1;
-    for (int q = tid; q < tp; q += kThreads) Ls[q] = L[(int64_t)s * ldL + q];
-    __syncthreads();
-    const double c = __dadd_rn(rdiag[s], (double)mu);
-    double li = 0.0;
-    if (i < N) {
-        double a = (double)K[packed_index(i, (int)s, nT)];
-        const double* Li = L + (int64_t)i * ldL;
-        for (int q = 0; q < tp; ++q) a = __fma_rn(-Li[q], Ls[q], a);
-        li = __ddiv_rn(a, __dsqrt_rn(c));
+    const double rc = __dsqrt_rn(__dadd_rn(rdiag[s], (double)mu));
+    double ls[kC], hacc[kC], lsq = 0.0;
+#pragma unroll
+    for (int c = 0; c < kC; ++c) {
+        const int q = l + 32 * c;
+        ls[c] = q < tp ? L[(int64_t)s * ldL + q] : 0.0;
+        hacc[c] = 0.0;
     }
-    L[(int64_t)i * ldL + tp] = li;
-    ell[i] = li;
-    // per-CTA partial sums (warp butterfly, then warps in order) of L_ik l_i and l_i^2
-    const double* Li = L + (int64_t)i * ldL;
-    for (int q = 0; q <= tp; ++q) {
-        const double x = q < tp ? __dmul_rn(Li[q], li) : __dmul_rn(li, li);
-        const double ws = warp_sum64(x);
-        if (l == 0) red[w][q & 63] = ws;
-        if ((q & 63) == 63 || q == tp) {
-            __syncthreads();
-            const int qbase = q & ~63;
-            for (int qq = tid; qq <= q - qbase; qq += kThreads) {
-                double a = 0.0;
-                for (int ww = 0; ww < kThreads / 32; ++ww) a = __dadd_rn(a, red[ww][qq]);
-                Hpart[(int64_t)blockIdx.x * (ldL + 1) + qbase + qq] = a;
-            }
-            __syncthreads();
+    for (int rr = 0; rr < kRowsPerWarp; ++rr) {
+        const int i = blockIdx.x * kEllRows + w * kRowsPerWarp + rr;
+        const double* Li = L + (int64_t)i * ldL;
+        double li_q[kC];
+        double dot = 0.0;
+#pragma unroll
+        for (int c = 0; c < kC; ++c) {
+            const int q = l + 32 * c;
+            li_q[c] = q < tp ? Li[q] : 0.0;
+            dot = __fma_rn(li_q[c], ls[c], dot);
         }
+        dot = warp_sum64(dot);
+        double li = 0.0;
+        if (i < N) li = __ddiv_rn(__dsub_rn((double)K[packed_index(i, (int)s, nT)], dot), rc);
+        if (l == 0) {
+            L[(int64_t)i * ldL + tp] = li;
+            ell[i] = li;
+        }
+#pragma unroll
+        for (int c = 0; c < kC; ++c) hacc[c] = __fma_rn(li_q[c], li, hacc[c]);
+        lsq = __fma_rn(li, li, lsq);
+    }
+#pragma unroll
+    for (int c = 0; c < kC; ++c) {
+        const int q = l + 32 * c;
+        if (q < tp) part[w][q] = hacc[c];
+    }
+    if (l == 0) part[w][tp] = lsq;
+    __syncthreads();
+    for (int q = tid; q <= tp; q += kThreads) {
+        double a = 0.0;
+        for (int ww = 0; ww < kThreads / 32; ++ww) a = __dadd_rn(a, part[ww][q]);
+        Hpart[(int64_t)blockIdx.x * (ldL + 1) + q] = a;
     }
 }
 
