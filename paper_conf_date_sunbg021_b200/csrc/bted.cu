@@ -329,6 +329,17 @@ void enqueue_loop_packed(Ted& T, int64_t N, int32_t m, float mu, unsigned long l
 
 // ---- implicit deflation (implicit.cuh) ----
 // head: K1p (the packed Gram, read-only from now on), fp64 norm pass, scores.  (3 kernels)
+void ensure_implicit_attrs() {
+    static bool done = false;
+    if (!done) {
+        CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)bted::im::tile_pass_smem_bytes));
+        CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)bted::im::tile_pass_smem_bytes));
+        done = true;
+    }
+}
+
 void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m,
                            float mu, unsigned long long* keys) {
     const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
@@ -345,7 +356,7 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
     else
         bted::pk::gram_packed_kernel<32><<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
             X, (int32_t)N, d, gamma, lin, T.K[0], nT, scratch);
-    bted::im::tile_pass_kernel<true><<<(unsigned)tiles, bted::im::kThreads, 0, T.stream>>>(
+    bted::im::tile_pass_kernel<true><<<(unsigned)tiles, bted::im::kThreads, bted::im::tile_pass_smem_bytes, T.stream>>>(
         T.K[0], nT, nullptr, T.P64, nullptr, 0, 0, 0, nullptr);
     bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
         T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, m, 0, T.hv, T.nv, T.rd, T.sel, keys, 0, keys, T.err);
@@ -362,7 +373,8 @@ void enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned long
         const int32_t tp = t - 1;
         bted::im::ell_kernel<<<nA, bted::im::kThreads, 0, T.stream>>>(T.K[0], nT, (int32_t)N, T.Lf, m, tp, T.rd, mu,
                                                                       keys, t, T.ell, T.Hp, T.sel);
-        bted::im::tile_pass_kernel<false><<<(unsigned)tiles, bted::im::kThreads, 0, T.stream>>>(
+        bted::im::tile_pass_kernel<false><<<(unsigned)tiles, bted::im::kThreads, bted::im::tile_pass_smem_bytes,
+                                            T.stream>>>(
             T.K[0], nT, T.ell, T.P64, T.Hp, nA, tp + 1, m + 1, T.hv);
         bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
             T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, m, tp, T.hv, T.nv, T.rd, T.sel, keys, t, keys + t, T.err);
@@ -435,6 +447,7 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
              unsigned long long* keys, bool no_graph, bool time_it = true, bool packed = false) {
     const bool implicit = packed && T.implicit && m <= bted::im::kMaxM;
     if (implicit) {
+        ensure_implicit_attrs();
         T.reserve_implicit(N, m);
         T.last_nT = (int32_t)((N + bted::pk::T - 1) / bted::pk::T);
     } else if (packed) {

@@ -49,38 +49,45 @@ __device__ __forceinline__ double warp_sum64(double v) {
 // tile; warp w: rows 16w..16w+15, half-warp h: rows 16w+8h..+7, lane hl:
 // columns 8hl..8hl+7.  Canonical per-128 tree: groups of 4 consecutive terms
 // (sequential), then the 32-leaf butterfly.
+constexpr size_t tile_pass_smem_bytes = (size_t)(T * (kGroups + 1) + kGroups * T + T) * sizeof(double);
+
 template <bool kNorm>
 __global__ void __launch_bounds__(kThreads)
 tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__ w, double* __restrict__ P64,
                  const double* __restrict__ Hpart, int nHpart, int nh, int hstride, double* __restrict__ h) {
-    // column groups, layout [q][c][hl] (group q, lane hl, its column 8hl+c): a
-    // half-warp stores 16 consecutive doubles per c; tree thread tid reads
-    // [q][tid] and owns column 8*(tid&15) + (tid>>4).  No bank conflicts.
-    __shared__ double cgs[kGroups * T];                // 32 KiB
-    __shared__ double wi[T];                           // w on the tile's rows
+    // group sums: rows [r][q] (row stride 33: conflict-free tree reads), columns
+    // [q][c][hl] (group q, lane hl, its column 8hl+c).  Then threads 0..127 run the
+    // canonical 32-leaf tree of one row each, threads 128..255 of one column each.
+    constexpr int kRS = kGroups + 1;
+    extern __shared__ double dsm[];                    // dynamic: tile_pass_smem_bytes
+    double* rgs = dsm;                                 // [T][kRS]     33 KiB
+    double* cgs = rgs + T * kRS;                       // [kGroups*T]  32 KiB
+    double* wi = cgs + kGroups * T;                    // [T] w on the tile's rows
     const int tid = threadIdx.x, w_ = tid / 32, l = tid % 32;
     const int hw = l >> 4, hl = l & 15, c8 = 8 * hl;
+    const int nTiles = (int)num_tiles(nT);
+    const int64_t NP = (int64_t)nT * T;
+    // kernel A left per-CTA partials of h = L^T l and |l|^2: CTAs k, k + grid, ...
+    // reduce column k (thread-strided sequential sums, then a fixed tree)
+    if (!kNorm) {
+        for (int col = blockIdx.x; col < nh; col += gridDim.x) {
+            double a = 0.0;
+            for (int b = tid; b < nHpart; b += kThreads) a = __dadd_rn(a, Hpart[(int64_t)b * hstride + col]);
+            a = warp_sum64(a);
+            if (l == 0) cgs[w_] = a;
+            __syncthreads();
+            if (tid == 0) {
+                double v = 0.0;
+                for (int q = 0; q < kThreads / 32; ++q) v = __dadd_rn(v, cgs[q]);
+                h[col] = v;
+            }
+            __syncthreads();
+        }
+    }
     const int64_t k = blockIdx.x;
     int I, J;
     tile_ij(k, nT, I, J);
-    const int64_t NP = (int64_t)nT * T;
-    // kernel A left per-CTA partials of h = L^T l and |l|^2: CTA 0 reduces them
-    // in CTA order for kernel C (fixed order, deterministic)
-    if (!kNorm && k < nh) {
-        // CTA k reduces column k of Hpart (nHpart CTA partials): thread-strided
-        // sequential sums, then a fixed tree over the 256 threads
-        double a = 0.0;
-        for (int b = tid; b < nHpart; b += kThreads) a = __dadd_rn(a, Hpart[(int64_t)b * hstride + k]);
-        a = warp_sum64(a);
-        if (l == 0) cgs[w_] = a;
-        __syncthreads();
-        if (tid == 0) {
-            double v = 0.0;
-            for (int q = 0; q < kThreads / 32; ++q) v = __dadd_rn(v, cgs[q]);
-            h[k] = v;
-        }
-        __syncthreads();
-    }
+    (void)nTiles;
     double wc[8];
     if (!kNorm) {
         if (tid < T) wi[tid] = w[(int64_t)I * T + tid];
@@ -89,7 +96,6 @@ tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__
         __syncthreads();
     }
     const float* gin = K + k * (int64_t)(T * T);
-    double rowsum = 0.0;
     double cg[8];
 #pragma unroll
     for (int r0 = 0; r0 < 8; r0 += 4) {
@@ -100,59 +106,50 @@ tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__
         for (int u = 0; u < 4; ++u) {
             const int rr = r0 + u;
             const int r = 16 * w_ + 8 * hw + rr;
-            double x[8];
-            const double wr = kNorm ? 0.0 : wi[r];
+            double kd[8];
 #pragma unroll
-            for (int c = 0; c < 8; ++c) {
-                const double kij = (double)kv[u].v[c];
-                x[c] = kNorm ? kij : kij * wc[c];       // row term factor: K_ij * (K_ij | w_j)
-            }
-            double ga, gb;
-            if (kNorm) {
-                ga = __dmul_rn(x[0], x[0]); ga = __fma_rn(x[1], x[1], ga); ga = __fma_rn(x[2], x[2], ga); ga = __fma_rn(x[3], x[3], ga);
-                gb = __dmul_rn(x[4], x[4]); gb = __fma_rn(x[5], x[5], gb); gb = __fma_rn(x[6], x[6], gb); gb = __fma_rn(x[7], x[7], gb);
-            } else {
-                const double k0 = (double)kv[u].v[0], k1 = (double)kv[u].v[1], k2 = (double)kv[u].v[2], k3 = (double)kv[u].v[3];
-                const double k4 = (double)kv[u].v[4], k5 = (double)kv[u].v[5], k6 = (double)kv[u].v[6], k7 = (double)kv[u].v[7];
-                ga = __dmul_rn(k0, wc[0]); ga = __fma_rn(k1, wc[1], ga); ga = __fma_rn(k2, wc[2], ga); ga = __fma_rn(k3, wc[3], ga);
-                gb = __dmul_rn(k4, wc[4]); gb = __fma_rn(k5, wc[5], gb); gb = __fma_rn(k6, wc[6], gb); gb = __fma_rn(k7, wc[7], gb);
-            }
-#pragma unroll
-            for (int off = 8; off > 0; off >>= 1) {
-                ga = __dadd_rn(ga, __shfl_xor_sync(0xffffffffu, ga, off));
-                gb = __dadd_rn(gb, __shfl_xor_sync(0xffffffffu, gb, off));
-            }
-            const double rp = __dadd_rn(ga, gb);
-            const double rq0 = __shfl_sync(0xffffffffu, rp, 0), rq1 = __shfl_sync(0xffffffffu, rp, 16);
-            if (l == rr) rowsum = rq0;
-            if (l == 8 + rr) rowsum = rq1;
+            for (int c = 0; c < 8; ++c) kd[c] = (double)kv[u].v[c];
+            // row terms K_ij * (K_ij | w_j): two groups of 4 consecutive columns
+            const double* f = kNorm ? kd : wc;
+            double ga = __dmul_rn(kd[0], f[0]);
+            ga = __fma_rn(kd[1], f[1], ga); ga = __fma_rn(kd[2], f[2], ga); ga = __fma_rn(kd[3], f[3], ga);
+            double gb = __dmul_rn(kd[4], f[4]);
+            gb = __fma_rn(kd[5], f[5], gb); gb = __fma_rn(kd[6], f[6], gb); gb = __fma_rn(kd[7], f[7], gb);
+            rgs[r * kRS + 2 * hl] = ga;
+            rgs[r * kRS + 2 * hl + 1] = gb;
             if (I != J) {
+                // column terms K_ij * (K_ij | w_i): groups of 4 consecutive rows
+                const double wr = kNorm ? 0.0 : wi[r];
 #pragma unroll
                 for (int c = 0; c < 8; ++c) {
-                    const double kij = (double)kv[u].v[c];
-                    const double f = kNorm ? kij : wr;   // column term: K_ij * (K_ij | w_i)
-                    cg[c] = (rr & 3) == 0 ? __dmul_rn(kij, f) : __fma_rn(kij, f, cg[c]);
+                    const double g = kNorm ? kd[c] : wr;
+                    cg[c] = (rr & 3) == 0 ? __dmul_rn(kd[c], g) : __fma_rn(kd[c], g, cg[c]);
                 }
                 if ((rr & 3) == 3) {
 #pragma unroll
                     for (int c = 0; c < 8; ++c) cgs[(r >> 2) * T + c * 16 + hl] = cg[c];
                 }
             }
-            (void)x;
         }
     }
-    if (l < 16) P64[(int64_t)J * NP + (int64_t)I * T + 16 * w_ + l] = rowsum;
-    if (I != J) {
-        __syncthreads();
-        if (tid < T) {
-            double hh[kGroups];
+    __syncthreads();
+    double hh[kGroups];
+    if (tid < T) {                                      // row tid: P[J][I*T + tid]
 #pragma unroll
-            for (int q = 0; q < kGroups; ++q) hh[q] = cgs[q * T + tid];
+        for (int q = 0; q < kGroups; ++q) hh[q] = rgs[tid * kRS + q];
+    } else if (I != J) {                                // column: P[I][J*T + 8(c&15) + (c>>4)]
 #pragma unroll
-            for (int off = 16; off > 0; off >>= 1)
+        for (int q = 0; q < kGroups; ++q) hh[q] = cgs[q * T + (tid - T)];
+    }
+    if (tid < T || I != J) {
 #pragma unroll
-                for (int q = 0; q < off; ++q) hh[q] = __dadd_rn(hh[q], hh[q + off]);
-            P64[(int64_t)I * NP + (int64_t)J * T + 8 * (tid & 15) + (tid >> 4)] = hh[0];
+        for (int off = 16; off > 0; off >>= 1)
+#pragma unroll
+            for (int q = 0; q < off; ++q) hh[q] = __dadd_rn(hh[q], hh[q + off]);
+        if (tid < T) P64[(int64_t)J * NP + (int64_t)I * T + tid] = hh[0];
+        else {
+            const int c = tid - T;
+            P64[(int64_t)I * NP + (int64_t)J * T + 8 * (c & 15) + (c >> 4)] = hh[0];
         }
     }
 }
