@@ -43,6 +43,20 @@ __device__ __forceinline__ double warp_sum64(double v) {
     return v;
 }
 
+// fp32 -> fp64 with integer ops (the F2F.F64.F32 pipe is the tile pass's
+// bottleneck on B200).  Exact for zeros and normal numbers: exponent rebias
+// (+896) and mantissa shift; subnormal inputs (|x| < 2^-126) take the
+// hardware conversion (the caller checks per warp).
+__device__ __forceinline__ double f2d_int(float x) {
+    const uint32_t u = __float_as_uint(x), t = u & 0x7FFFFFFFu, sgn = u & 0x80000000u;
+    const uint32_t hi = t ? (((t >> 3) + 0x38000000u) | sgn) : sgn;
+    return __hiloint2double((int)hi, (int)(u << 29));
+}
+__device__ __forceinline__ bool is_subnormal(float x) {
+    const uint32_t t = __float_as_uint(x) & 0x7FFFFFFFu;
+    return t != 0u && t < 0x00800000u;
+}
+
 // ------------------------------------------------------------------ tile pass (fp64 partials)
 // kNorm: row/col partials of K_ij^2 (the initial ||K_:v||^2);  else of K_ij w_j
 // (rows) and K_ij w_i (columns): q = K w.  One CTA (256 threads) per stored
@@ -107,8 +121,16 @@ tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__
             const int rr = r0 + u;
             const int r = 16 * w_ + 8 * hw + rr;
             double kd[8];
+            bool sub = false;
 #pragma unroll
-            for (int c = 0; c < 8; ++c) kd[c] = (double)kv[u].v[c];
+            for (int c = 0; c < 8; ++c) sub |= is_subnormal(kv[u].v[c]);
+            if (__any_sync(0xffffffffu, sub)) {
+#pragma unroll
+                for (int c = 0; c < 8; ++c) kd[c] = (double)kv[u].v[c];
+            } else {
+#pragma unroll
+                for (int c = 0; c < 8; ++c) kd[c] = f2d_int(kv[u].v[c]);
+            }
             // row terms K_ij * (K_ij | w_j): two groups of 4 consecutive columns
             const double* f = kNorm ? kd : wc;
             double ga = __dmul_rn(kd[0], f[0]);

@@ -425,3 +425,15 @@ def test_update_replaces_features_and_validates_on_device():
         assert e.value.status == 1 and "non-finite" in str(e.value)
         L.bted_update(cs.ctx, X1)                                   # recovers
         assert np.array_equal(cs.run_batches(1000, 16, MU)[0], first)
+
+
+@pytest.mark.parametrize("flags", [IMPLICIT, PACKED, DENSE], ids=["implicit", "packed", "dense"])
+def test_subnormal_and_underflowing_kernel_values(flags):
+    """gamma large enough that many K_ij are fp32 subnormals or underflow to 0
+    (exercises the implicit tile pass's conversion fallback)."""
+    X = uniform_pool(700, 16, 70)
+    g = 30.0
+    with bt.CandidateSet(X, g, flags=flags) as cs:
+        idx, sc = cs.select(32, MU)
+    tr = dense.ted(X, g, MU, 32, forced=idx)
+    check_ted(idx, sc, tr, f"subnormal-{flags}")
