@@ -735,12 +735,15 @@ void sample_batch(bted_ctx* ctx, cudaStream_t st, int64_t P, int64_t M, int32_t 
     bted::batch_keys_kernel<<<g, 256, 0, st>>>((uint64_t)P, hb, ctx->skeys);
     LAUNCHED(1);
     size_t need = 0, need2 = 0;
-    CK(cub::DeviceRadixSort::SortKeys(nullptr, need, ctx->skeys, ctx->skeys2, (int)P, 0, 64, st));
+    // only the hash half (bits 32..63) needs sorting: the radix sort is stable
+    // and keys arrive in index order, so equal hashes stay ordered by index --
+    // the same order as the full 64-bit key
+    CK(cub::DeviceRadixSort::SortKeys(nullptr, need, ctx->skeys, ctx->skeys2, (int)P, 32, 64, st));
     if (!dst) dst = ctx->sidx;
     CK(cub::DeviceRadixSort::SortKeys(nullptr, need2, ctx->sidx2, dst, (int)M, 0, bits_for(P), st));
     cub_reserve(ctx, std::max(need, need2));
     size_t cap = ctx->cub_cap;
-    CK(cub::DeviceRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->skeys, ctx->skeys2, (int)P, 0, 64, st));
+    CK(cub::DeviceRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->skeys, ctx->skeys2, (int)P, 32, 64, st));
     const unsigned gm = (unsigned)std::min<int64_t>((M + 255) / 256, 148 * 16);
     bted::low_half_kernel<<<gm, 256, 0, st>>>(ctx->skeys2, M, ctx->sidx2);
     LAUNCHED(1);

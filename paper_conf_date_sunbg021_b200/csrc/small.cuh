@@ -41,7 +41,13 @@ __global__ void __launch_bounds__(kThreads, 1)
 ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float gamma, int32_t linear,
                    int32_t m, float mu, unsigned long long* __restrict__ keys_all, int* __restrict__ err) {
     cg::cluster_group cl = cg::this_cluster();
-    const int rank = (int)cl.block_rank();
+    const int rank = C == 1 ? 0 : (int)cl.block_rank();
+    // a cluster of one CTA needs only the CTA barrier (cluster barriers also
+    // invalidate L1)
+    auto csync = [&]() {
+        if constexpr (C == 1) __syncthreads();
+        else cl.sync();
+    };
     const int inst = blockIdx.x / C;
     const float* __restrict__ X = Xall + (int64_t)inst * N * d;
     unsigned long long* keys_out = keys_all + (int64_t)inst * m;
@@ -94,12 +100,16 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
         if (tid == 0) {
             unsigned long long v = 0ull;
             for (int q = 0; q < kWarps; ++q) v = wred[q] > v ? wred[q] : v;
-            for (int r = 0; r < C; ++r) {
-                unsigned long long* dst = cl.map_shared_rank(kslot, r);
-                dst[parity * 16 + rank] = v;
+            if constexpr (C == 1) {
+                kslot[parity * 16] = v;
+            } else {
+                for (int r = 0; r < C; ++r) {
+                    unsigned long long* dst = cl.map_shared_rank(kslot, r);
+                    dst[parity * 16 + rank] = v;
+                }
             }
         }
-        cl.sync();
+        csync();
         unsigned long long b = 0ull;
         for (int r = 0; r < C; ++r) b = kslot[parity * 16 + r] > b ? kslot[parity * 16 + r] : b;
         return b;
@@ -112,11 +122,11 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
         if (best == 0ull) { if (tid == 0) atomicOr(err, 2); break; }
         // pivot row K[s][:] from its owner's shared memory
         const int owner = s / R;
-        const float* src = cl.map_shared_rank(Kb, owner) + (size_t)(s - owner * R) * L;
+        const float* src = (C == 1 ? Kb : cl.map_shared_rank(Kb, owner)) + (size_t)(s - owner * R) * L;
         for (int j4 = tid; j4 < L / 4; j4 += kThreads)
             reinterpret_cast<float4*>(piv)[j4] = reinterpret_cast<const float4*>(src)[j4];
         if (owner == rank && tid == 0) sel[s - r0] = 1;
-        cl.sync();                                   // every CTA holds the pivot before rows change
+        csync();                                     // every CTA holds the pivot before rows change
         const float inv_c = __frcp_rn(__fadd_rn(piv[s], mu));
         best_local = 0ull;
         for (int lr = w; lr < nr; lr += kWarps) {
@@ -147,7 +157,7 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
         best = exchange(best_local, t & 1);
     }
     if (rank == 0 && tid == 0) keys_out[m - 1] = best;
-    cl.sync();                                       // no CTA exits while others may read its smem
+    csync();                                         // no CTA exits while others may read its smem
 }
 
 }  // namespace sm
