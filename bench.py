@@ -35,8 +35,7 @@ METRIC = "BTED selected points/sec and deflate-step HBM GB/s vs roofline at 1/2/
 UNIT = "points/s"
 K2_NAME = {"dense": "deflate_rescore_kernel",
            "packed": "deflate_packed_ldg_kernel (+ finalize_packed_kernel, per step)",
-           "implicit": "tile_pass_kernel (q = K l, read-only; + ell_kernel + fin64_kernel, per step)",
-           "implicit-f32": "tile_pass_kernel<fp32 groups> (q = K l, read-only; + ell_kernel + fin64_kernel)"}
+           "implicit": "tile_pass_kernel (q = K l, read-only; + ell_kernel + fin64_kernel, per step)"}
 
 
 def parse():
@@ -51,7 +50,7 @@ def parse():
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
                     help="weak: every GPU runs the config's B batches; strong: the config's B batches are split")
-    ap.add_argument("--layout", default="packed", choices=["packed", "dense", "implicit", "implicit-f32"],
+    ap.add_argument("--layout", default="packed", choices=["packed", "dense", "implicit"],
                     help="K storage: packed upper-triangular tiles (4 N^2 B/step), dense (8 N^2 B/step), "
                          "or implicit deflation on the read-only packed K (2 N^2 B/step)")
     return ap.parse_args()
@@ -207,8 +206,7 @@ def bench_ours(args):
     stream = torch.cuda.Stream(dev)
     X_dev = torch.from_numpy(X).to(dev)
     torch.cuda.synchronize()
-    lay_flag = {"dense": L.BTED_FLAG_DENSE, "packed": 0, "implicit": L.BTED_FLAG_IMPLICIT,
-                "implicit-f32": L.BTED_FLAG_IMPLICIT_F32}[args.layout]
+    lay_flag = {"dense": L.BTED_FLAG_DENSE, "packed": 0, "implicit": L.BTED_FLAG_IMPLICIT}[args.layout]
     pool = bt.CandidateSet(X_dev, gamma, num_batches=B, seed=cfg["seed"], device=local,
                            flags=L.BTED_FLAG_TIMING | lay_flag, stream=stream.cuda_stream)
 
@@ -255,7 +253,7 @@ def bench_ours(args):
     k2_avg_ms = stats["k2_ms"] / max(stats["k2_launches"], 1)
     # algorithmic bytes per step: fp32 read + write of K = 8 N^2 (dense) or of
     # its upper triangle = 4 N^2 (packed; report against 4 N^2)
-    alg_bytes = {"dense": 8.0, "packed": 4.0, "implicit": 2.0, "implicit-f32": 2.0}[args.layout] * M * M
+    alg_bytes = {"dense": 8.0, "packed": 4.0, "implicit": 2.0}[args.layout] * M * M
     achieved = alg_bytes / (k2_avg_ms / 1e3) / 1e9
     traffic = None
     tj = os.path.join(ROOT, "profiles", "k2_traffic.json")

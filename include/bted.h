@@ -70,9 +70,6 @@ typedef enum {
                                    carry K^(t) = K - L L^T by its fp64 factor L; one K.l pass per
                                    step (2 N^2 bytes, read only) + O(N m).  Same selections in
                                    exact arithmetic; fp64 recurrences.  Packed layouts only.   */
-#define BTED_FLAG_IMPLICIT_F32 64u  /* implicit deflation whose K.l pass forms products and
-                                   4-term group sums in fp32 (w split hi + lo) and only the
-                                   cross-group sums in fp64: memory-bound instead of FP64-bound */
 #define BTED_FLAG_TIMING   2u   /* record CUDA events around K1 and the K2 loop of every batch
                                    TED on the ctx stream; read with bted_get_stats()          */
 

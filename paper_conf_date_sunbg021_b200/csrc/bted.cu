@@ -116,7 +116,6 @@ struct Ted {
     double* Hp = nullptr; size_t hpcap = 0;
     double* hv = nullptr; size_t hvcap = 0;
     bool implicit = false;
-    bool implicit_f32 = false;  // tile pass: fp32 products / group sums (BTED_FLAG_IMPLICIT_F32)
     std::list<std::pair<GraphKey, cudaGraphExec_t>> graphs;   // LRU
     int64_t last_rows = 0, last_ld = 0;
     int last_buf = 0;
@@ -337,8 +336,6 @@ void ensure_implicit_attrs() {
                                 (int)bted::im::tile_pass_smem_bytes));
         CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)bted::im::tile_pass_smem_bytes));
-        CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)bted::im::tile_pass_smem_bytes));
         done = true;
     }
 }
@@ -376,14 +373,9 @@ void enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned long
         const int32_t tp = t - 1;
         bted::im::ell_kernel<<<nA, bted::im::kThreads, 0, T.stream>>>(T.K[0], nT, (int32_t)N, T.Lf, m, tp, T.rd, mu,
                                                                       keys, t, T.ell, T.Hp, T.sel);
-        if (T.implicit_f32)
-            bted::im::tile_pass_kernel<false, true><<<(unsigned)tiles, bted::im::kThreads,
-                                                      bted::im::tile_pass_smem_bytes, T.stream>>>(
-                T.K[0], nT, T.ell, T.P64, T.Hp, nA, tp + 1, m + 1, T.hv);
-        else
-            bted::im::tile_pass_kernel<false><<<(unsigned)tiles, bted::im::kThreads, bted::im::tile_pass_smem_bytes,
-                                                T.stream>>>(
-                T.K[0], nT, T.ell, T.P64, T.Hp, nA, tp + 1, m + 1, T.hv);
+        bted::im::tile_pass_kernel<false><<<(unsigned)tiles, bted::im::kThreads, bted::im::tile_pass_smem_bytes,
+                                            T.stream>>>(
+            T.K[0], nT, T.ell, T.P64, T.Hp, nA, tp + 1, m + 1, T.hv);
         bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
             T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, m, tp, T.hv, T.nv, T.rd, T.sel, keys, t, keys + t, T.err);
         LAUNCHED(3);
@@ -481,7 +473,7 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
         else if (packed) enqueue_loop_packed(T, N, m, mu, keys, T.tma);
         else enqueue_loop(T, N, m, mu, keys);
     };
-    const int mode = implicit ? (T.implicit_f32 ? 4 : 3) : packed ? (T.tma ? 2 : 1) : 0;
+    const int mode = implicit ? 3 : packed ? (T.tma ? 2 : 1) : 0;
     const uint64_t head_k = implicit ? 3 : 2, loop_k = implicit ? 3 : packed ? 2 : 1;
     if (no_graph) {
         head();
@@ -688,9 +680,7 @@ bted_status create_common(const float* X, int64_t N, int32_t d, bted_kernel kern
         ctx->bted_engine.stream = ctx->stream;
         ctx->ted.timing = ctx->bted_engine.timing = (params->flags & BTED_FLAG_TIMING) != 0;
         ctx->ted.tma = ctx->bted_engine.tma = (params->flags & BTED_FLAG_TMA) != 0;
-        ctx->ted.implicit = ctx->bted_engine.implicit =
-            (params->flags & (BTED_FLAG_IMPLICIT | BTED_FLAG_IMPLICIT_F32)) != 0;
-        ctx->ted.implicit_f32 = ctx->bted_engine.implicit_f32 = (params->flags & BTED_FLAG_IMPLICIT_F32) != 0;
+        ctx->ted.implicit = ctx->bted_engine.implicit = (params->flags & BTED_FLAG_IMPLICIT) != 0;
         CK(cudaMallocHost(&ctx->herr, sizeof(int)));
         if (params->x_on_device) {
             ctx->X = const_cast<float*>(X);

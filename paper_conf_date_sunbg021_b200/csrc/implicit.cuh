@@ -65,12 +65,7 @@ __device__ __forceinline__ bool is_subnormal(float x) {
 // (sequential), then the 32-leaf butterfly.
 constexpr size_t tile_pass_smem_bytes = (size_t)(T * (kGroups + 1) + kGroups * T + T) * sizeof(double);
 
-// kF32 (matvec only): each product K_ij * w is formed in fp32 as
-// fma(K, w_lo, fma(K, w_hi, acc)) with w = w_hi + w_lo split into two floats,
-// summed in fp32 within a group of 4 terms, and only the group sums (1/4 of
-// the terms) enter the fp64 tree: ~8x fewer FP64-pipe operations (the B200
-// FP64 pipe bounds the fp64 variant) for ~1e-7 relative group error.
-template <bool kNorm, bool kF32 = false>
+template <bool kNorm>
 __global__ void __launch_bounds__(kThreads)
 tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__ w, double* __restrict__ P64,
                  const double* __restrict__ Hpart, int nHpart, int nh, int hstride, double* __restrict__ h) {
@@ -108,18 +103,12 @@ tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__
     tile_ij(k, nT, I, J);
     (void)nTiles;
     double wc[8];
-    float whi[8], wlo[8];
     if (!kNorm) {
         if (tid < T) wi[tid] = w[(int64_t)I * T + tid];
 #pragma unroll
-        for (int c = 0; c < 8; ++c) {
-            wc[c] = w[(int64_t)J * T + c8 + c];
-            whi[c] = __double2float_rn(wc[c]);
-            wlo[c] = __double2float_rn(wc[c] - (double)whi[c]);
-        }
+        for (int c = 0; c < 8; ++c) wc[c] = w[(int64_t)J * T + c8 + c];
         __syncthreads();
     }
-    float cgf[8];
     const float* gin = K + k * (int64_t)(T * T);
     double cg[8];
 #pragma unroll
@@ -131,33 +120,6 @@ tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__
         for (int u = 0; u < 4; ++u) {
             const int rr = r0 + u;
             const int r = 16 * w_ + 8 * hw + rr;
-            if constexpr (!kNorm && kF32) {
-                const float* kf = kv[u].v;
-                float ga = __fmul_rn(kf[0], whi[0]);
-                ga = __fmaf_rn(kf[0], wlo[0], ga);
-#pragma unroll
-                for (int c = 1; c < 4; ++c) { ga = __fmaf_rn(kf[c], whi[c], ga); ga = __fmaf_rn(kf[c], wlo[c], ga); }
-                float gb = __fmul_rn(kf[4], whi[4]);
-                gb = __fmaf_rn(kf[4], wlo[4], gb);
-#pragma unroll
-                for (int c = 5; c < 8; ++c) { gb = __fmaf_rn(kf[c], whi[c], gb); gb = __fmaf_rn(kf[c], wlo[c], gb); }
-                rgs[r * kRS + 2 * hl] = (double)ga;
-                rgs[r * kRS + 2 * hl + 1] = (double)gb;
-                if (I != J) {
-                    const double wr = wi[r];
-                    const float rhi = __double2float_rn(wr), rlo = __double2float_rn(wr - (double)rhi);
-#pragma unroll
-                    for (int c = 0; c < 8; ++c) {
-                        float g = (rr & 3) == 0 ? __fmul_rn(kf[c], rhi) : __fmaf_rn(kf[c], rhi, cgf[c]);
-                        cgf[c] = __fmaf_rn(kf[c], rlo, g);
-                    }
-                    if ((rr & 3) == 3) {
-#pragma unroll
-                        for (int c = 0; c < 8; ++c) cgs[(r >> 2) * T + c * 16 + hl] = (double)cgf[c];
-                    }
-                }
-                continue;
-            }
             double kd[8];
             bool sub = false;
 #pragma unroll

@@ -19,9 +19,8 @@ PACKED = L.BTED_FLAG_NO_SMALL
 DENSE = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_DENSE
 PACKED_TMA = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_TMA
 IMPLICIT = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_IMPLICIT
-IMPLICIT32 = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_IMPLICIT_F32
-LAYOUTS = pytest.mark.parametrize("flags", [PACKED, PACKED_TMA, DENSE, IMPLICIT, IMPLICIT32, 0],
-                                  ids=["packed", "packed-tma", "dense", "implicit", "implicit-f32", "auto"])
+LAYOUTS = pytest.mark.parametrize("flags", [PACKED, PACKED_TMA, DENSE, IMPLICIT, 0],
+                                  ids=["packed", "packed-tma", "dense", "implicit", "auto"])
 LAYOUTS_K = pytest.mark.parametrize("flags", [PACKED, PACKED_TMA, DENSE], ids=["packed", "packed-tma", "dense"])
 
 
@@ -357,13 +356,12 @@ def test_paper_scale_bted_vs_oracle():
     assert launched < 60
 
 
-@pytest.mark.parametrize("flags", [IMPLICIT, IMPLICIT32], ids=["fp64", "fp32-groups"])
 @pytest.mark.parametrize("N,m", [(1000, 64), (4099, 64), (300, 256), (2000, 200)])
-def test_implicit_deflation_matches_oracle(N, m, flags):
+def test_implicit_deflation_matches_oracle(N, m):
     """N2: K read-only + fp64 factor recurrences -> same picks as the oracle."""
     X = knob(N, seed=N + 11)
     g = median_gamma(X, N)
-    with bt.CandidateSet(X, g, flags=flags) as cs:
+    with bt.CandidateSet(X, g, flags=IMPLICIT) as cs:
         idx, sc = cs.select(m, MU)
         idx2, sc2 = cs.select(m, MU)
     assert np.array_equal(idx, idx2) and np.array_equal(sc.view(np.uint32), sc2.view(np.uint32))
@@ -429,7 +427,7 @@ def test_update_replaces_features_and_validates_on_device():
         assert np.array_equal(cs.run_batches(1000, 16, MU)[0], first)
 
 
-@pytest.mark.parametrize("flags", [IMPLICIT, IMPLICIT32, PACKED, DENSE], ids=["implicit", "implicit-f32", "packed", "dense"])
+@pytest.mark.parametrize("flags", [IMPLICIT, PACKED, DENSE], ids=["implicit", "packed", "dense"])
 def test_subnormal_and_underflowing_kernel_values(flags):
     """gamma large enough that many K_ij are fp32 subnormals or underflow to 0
     (exercises the implicit tile pass's conversion fallback)."""
