@@ -1,0 +1,64 @@
+"""The multi-GPU drivers over a REAL NCCL process group (one rank: this run has
+one GPU).  Exercises dist.TorchComm's NCCL all-reduce / all-gather on CUDA
+tensors, stream ordering between them and libbted's kernels, and checks the
+results against the single-GPU entry points bit for bit."""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+import paper_conf_date_sunbg021_b200 as bt
+from paper_conf_date_sunbg021_b200 import _lib as L
+from synth import KnobSpace, WORKLOADS, make_pool, median_gamma
+
+pytestmark = pytest.mark.gpu
+MU = float(np.float32(0.1))
+
+
+@pytest.fixture(scope="module")
+def nccl_group(need_gpu):
+    import torch
+    import torch.distributed as dist
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=dev)
+    yield dev
+    dist.destroy_process_group()
+
+
+def test_sharded_ted_over_nccl_matches_dense_select(nccl_group):
+    import torch
+    from paper_conf_date_sunbg021_b200.dist import LibShard, ShardedTed, TorchComm, band
+    _, X = make_pool(KnobSpace(WORKLOADS["resnet18_layer1"], 16), 5000, 3)
+    g = median_gamma(X, 3)
+    with bt.CandidateSet(X, g, flags=L.BTED_FLAG_DENSE | L.BTED_FLAG_NO_SMALL) as cs:
+        idx, sc = cs.select(32, MU)
+    comm = TorchComm()
+    st_ = torch.cuda.Stream(nccl_group)
+    r0, r1, _ = band(5000, comm.world, comm.rank)
+    shard = LibShard(X, 5000, 16, g, r0, r1, nccl_group, st_)
+    try:
+        sidx, ssc = ShardedTed(shard, 5000, comm, nccl_group, st_).select(32, MU)
+    finally:
+        shard.close()
+    assert np.array_equal(sidx, idx)
+    assert np.array_equal(ssc.view(np.uint32), sc.view(np.uint32))
+
+
+def test_batch_round_robin_over_nccl_matches_run_batches(nccl_group):
+    import torch
+    from paper_conf_date_sunbg021_b200.dist import TorchComm, run_batches_dp
+    _, X = make_pool(KnobSpace(WORKLOADS["vgg16_conv1_1"], 16), 40000, 9)
+    g = median_gamma(X, 9)
+    st_ = torch.cuda.Stream(nccl_group)
+    with bt.CandidateSet(X, g, num_batches=3, seed=5, stream=st_.cuda_stream) as pool:
+        ref, _ = pool.run_batches(2000, 16, MU)
+        with torch.cuda.stream(st_):
+            sel, win = run_batches_dp(pool.ctx, 2000, 16, MU, 3, TorchComm(), nccl_group)
+    assert np.array_equal(sel, ref)
