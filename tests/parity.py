@@ -13,6 +13,7 @@ import numpy as np
 
 SCORE_RTOL = 1e-5
 GAP_EXACT = 1e-6
+REPORT = []          # per-call summaries; written by tests/conftest.py when BTED_PARITY_REPORT is set
 
 
 def check_ted(gpu_idx, gpu_score, trace, label=""):
@@ -23,9 +24,11 @@ def check_ted(gpu_idx, gpu_score, trace, label=""):
     assert np.array_equal(o_idx, gpu_idx), f"{label}: oracle was not forced along the GPU history"
     assert len(set(gpu_idx.tolist())) == len(gpu_idx), f"{label}: a point was selected twice"
     near = 0
+    max_rel = 0.0
     for t in range(len(gpu_idx)):
         if gpu_score is not None and len(gpu_score):
             rel = abs(gpu_score[t] - o_score[t]) / max(abs(o_score[t]), 1e-300)
+            max_rel = max(max_rel, rel)
             assert rel <= SCORE_RTOL, f"{label} P1 step {t}: gpu {gpu_score[t]!r} vs fp64 {o_score[t]!r} rel {rel:.3e}"
         if o_gap[t] > GAP_EXACT:
             assert gpu_idx[t] == o_arg[t], (f"{label} P2 step {t}: gpu picked {gpu_idx[t]}, oracle argmax {o_arg[t]}"
@@ -33,6 +36,10 @@ def check_ted(gpu_idx, gpu_score, trace, label=""):
         else:
             near += 1
             assert o_score[t] >= (1 - SCORE_RTOL) * o_max[t], f"{label} P2 near-tie step {t}"
+    gaps = np.asarray(o_gap, dtype=np.float64)
+    REPORT.append({"label": label, "steps": int(len(gpu_idx)), "max_rel_score_err": float(max_rel),
+                   "near_ties": int(near), "min_gap": float(gaps[np.isfinite(gaps)].min()) if np.isfinite(gaps).any() else None,
+                   "steps_gap_below_1e-5": int((gaps <= 1e-5).sum())})
     return near
 
 
