@@ -218,6 +218,14 @@ finalize_packed_kernel(const float* __restrict__ P, int nT, int32_t N, const flo
     const int64_t NP = (int64_t)nT * T;
     const int i = blockIdx.x * kFinRows + lane;            // row (< nT*T by construction)
     const uint32_t s = t > 0 ? key_index(keys[t - 1]) : 0xFFFFFFFFu;
+    // warp 0 fetches the row's new diagonal entry and mask up front (off the critical path)
+    float diag = 0.f;
+    bool sl = true;
+    if (w == 0 && i < N) {
+        const int B = i / T, r = i % T;
+        diag = K[tile_offset(B, B, nT) * (T * T) + (int64_t)r * T + r];
+        sl = sel[i] != 0;
+    }
     const int per = (nT + 7) / 8;
     const int j0 = min(nT, w * per), j1 = min(nT, j0 + per);
     const float* src = P + i;
@@ -239,9 +247,7 @@ finalize_packed_kernel(const float* __restrict__ P, int nT, int32_t N, const flo
             float g = part[0][lane];
 #pragma unroll
             for (int q = 1; q < 8; ++q) g = __fadd_rn(g, part[q][lane]);
-            const int B = i / T, r = i % T;
-            const float diag = K[tile_offset(B, B, nT) * (T * T) + (int64_t)r * T + r];
-            const bool masked = sel[i] != 0 || (uint32_t)i == s;
+            const bool masked = sl || (uint32_t)i == s;
             key = score_key(g, diag, mu, (uint32_t)i, masked, err);
         }
         key = warp_max_u64(key);
@@ -584,40 +590,47 @@ gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamm
         float* tile = K + k * (int64_t)(T * T);
         RowWalk a;
         a.rowsum = 0.f;
-        for (int rr = 0; rr < 16; ++rr) {
+        for (int rr = 0; rr < 16; rr += 2) {
+            // two rows at once: four independent FFMA2 chains (ILP at 2 CTAs / SM)
             const int r = 16 * w + rr;
-            unsigned long long a01 = 0ull, a23 = 0ull;
+            unsigned long long a01[2] = {0ull, 0ull}, a23[2] = {0ull, 0ull};
 #pragma unroll
             for (int q = 0; q < kD; q += 4) {
-                const float4 xv = *reinterpret_cast<const float4*>(&xi[r][q]);
-                const float xs[4] = {xv.x, xv.y, xv.z, xv.w};
 #pragma unroll
-                for (int qq = 0; qq < 4; ++qq) {
-                    const unsigned long long xx = pack2(xs[qq], xs[qq]);
-                    if (linear) {
-                        a01 = fma2(xx, y01[q + qq], a01);
-                        a23 = fma2(xx, y23[q + qq], a23);
-                    } else {
-                        const unsigned long long d01 = sub2(xx, y01[q + qq]), d23 = sub2(xx, y23[q + qq]);
-                        a01 = fma2(d01, d01, a01);
-                        a23 = fma2(d23, d23, a23);
+                for (int h = 0; h < 2; ++h) {
+                    const float4 xv = *reinterpret_cast<const float4*>(&xi[r + h][q]);
+                    const float xs[4] = {xv.x, xv.y, xv.z, xv.w};
+#pragma unroll
+                    for (int qq = 0; qq < 4; ++qq) {
+                        const unsigned long long xx = pack2(xs[qq], xs[qq]);
+                        if (linear) {
+                            a01[h] = fma2(xx, y01[q + qq], a01[h]);
+                            a23[h] = fma2(xx, y23[q + qq], a23[h]);
+                        } else {
+                            const unsigned long long d01 = sub2(xx, y01[q + qq]), d23 = sub2(xx, y23[q + qq]);
+                            a01[h] = fma2(d01, d01, a01[h]);
+                            a23[h] = fma2(d23, d23, a23[h]);
+                        }
                     }
                 }
             }
-            float acc[4];
-            unpack2(a01, acc[0], acc[1]);
-            unpack2(a23, acc[2], acc[3]);
-            float4 o;
-            float* oc = &o.x;
-            const bool rv = I * T + r < N;
 #pragma unroll
-            for (int c = 0; c < 4; ++c) {
-                const bool cv = J * T + 4 * l + c < N;
-                const float val = linear ? acc[c] : expf(__fmul_rn(ng, acc[c]));
-                oc[c] = (rv && cv) ? val : 0.f;
+            for (int h = 0; h < 2; ++h) {
+                float acc[4];
+                unpack2(a01[h], acc[0], acc[1]);
+                unpack2(a23[h], acc[2], acc[3]);
+                float4 o;
+                float* oc = &o.x;
+                const bool rv = I * T + r + h < N;
+#pragma unroll
+                for (int c = 0; c < 4; ++c) {
+                    const bool cv = J * T + 4 * l + c < N;
+                    const float val = linear ? acc[c] : expf(__fmul_rn(ng, acc[c]));
+                    oc[c] = (rv && cv) ? val : 0.f;
+                }
+                st_stream(tile + (r + h) * T + 4 * l, o);
+                walk_row(a, rr + h, l, o, colg, w, I != J);
             }
-            st_stream(tile + r * T + 4 * l, o);
-            walk_row(a, rr, l, o, colg, w, I != J);
         }
         consumer_sync();
         write_partials(P, NP, I, J, w, l, a, colg, tid);
