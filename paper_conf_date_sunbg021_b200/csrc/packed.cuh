@@ -556,7 +556,7 @@ __device__ __forceinline__ void st_keep(float* p, float v, uint64_t pol) {
 }
 
 template <int kD>
-__global__ void __launch_bounds__(kConsumers)
+__global__ void __launch_bounds__(kConsumers, (kD <= 16 ? 3 : 1))
 gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma, int32_t linear,
                    float* __restrict__ K, int nT, float* __restrict__ P) {
 
