@@ -250,18 +250,34 @@ def bench_ours(args):
 
     # roofline of the dominant kernel K2 (fused deflate + rescore), live events
     peak, peak_src = peaks()
-    k2_avg_ms = stats["k2_ms"] / max(stats["k2_launches"], 1)
-    # algorithmic bytes per step: fp32 read + write of K = 8 N^2 (dense) or of
-    # its upper triangle = 4 N^2 (packed; report against 4 N^2)
-    alg_bytes = {"dense": 8.0, "packed": 4.0, "implicit": 2.0}[args.layout] * M * M
-    achieved = alg_bytes / (k2_avg_ms / 1e3) / 1e9
     traffic = None
-    tj = os.path.join(ROOT, "profiles", "k2_traffic.json")
-    if os.path.exists(tj):
-        with open(tj) as f:
-            tjd = json.load(f)
-        if tjd.get("M") == M and tjd.get("layout", "dense") == args.layout:
-            traffic = tjd.get("dram_bytes_per_launch")
+    if stats["k2_launches"] > 0:
+        k2_avg_ms = stats["k2_ms"] / stats["k2_launches"]
+        # algorithmic bytes per step: fp32 read + write of K = 8 N^2 (dense) or of
+        # its upper triangle = 4 N^2 (packed; report against 4 N^2)
+        alg_bytes = {"dense": 8.0, "packed": 4.0, "implicit": 2.0}[args.layout] * M * M
+        achieved = alg_bytes / (k2_avg_ms / 1e3) / 1e9
+        tj = os.path.join(ROOT, "profiles", "k2_traffic.json")
+        if os.path.exists(tj):
+            with open(tj) as f:
+                tjd = json.load(f)
+            if tjd.get("M") == M and tjd.get("layout", "dense") == args.layout:
+                traffic = tjd.get("dram_bytes_per_launch")
+        roofline = {"bound": "hbm", "kernel": K2_NAME[args.layout], "achieved": achieved, "peak": peak,
+                    "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
+                    "frac_of_8TBs": achieved / 8000.0, "peak_source": peak_src,
+                    "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": k2_avg_ms,
+                    "launches_timed": stats["k2_launches"],
+                    "k2_share_of_step": (stats["k2_ms"] / ms) if ms > 0 else None,
+                    "k1_ms_per_batch": stats["k1_ms"] / max(stats["teds"], 1)}
+    else:
+        # small batches: every TED is one cluster kernel with K in distributed
+        # shared memory -- no HBM stream to hold against the HBM roofline
+        roofline = {"bound": "latency", "kernel": "ted_cluster_kernel (K in DSMEM, whole TED per launch)",
+                    "achieved": None, "peak": None, "unit": None, "frac": None, "traffic": None,
+                    "small_teds_timed": stats["small_teds"],
+                    "ms_per_small_launch": stats["small_ms"] / max(args.steps, 1),
+                    "small_share_of_step": (stats["small_ms"] / ms) if ms > 0 else None}
 
     # end to end through the public API with HOST buffers (pinned), per step:
     # H2D of the pool, the whole BTED, D2H of the result
@@ -317,13 +333,7 @@ def bench_ours(args):
                 "scaling": args.scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
                 "config": workload_config(args.config, cfg, gamma, world, B),
                 "layout": args.layout,
-                "roofline": {"bound": "hbm", "kernel": K2_NAME[args.layout], "achieved": achieved, "peak": peak,
-                             "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
-                             "frac_of_8TBs": achieved / 8000.0, "peak_source": peak_src,
-                             "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": k2_avg_ms,
-                             "launches_timed": stats["k2_launches"],
-                             "k2_share_of_step": (stats["k2_ms"] / ms) if ms > 0 else None,
-                             "k1_ms_per_batch": stats["k1_ms"] / max(stats["teds"], 1)},
+                "roofline": roofline,
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
                 "final_selection_head": [int(x) for x in sel[:8]]}
         print(json.dumps(line), flush=True)

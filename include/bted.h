@@ -221,6 +221,8 @@ typedef struct {
     uint64_t k2_launches;
     double   k1_ms;
     double   k2_ms;
+    uint64_t small_teds;     /* TEDs run whole by the cluster kernel (small N) */
+    double   small_ms;       /* their device time                              */
 } bted_stats;
 bted_status bted_get_stats(bted_ctx* ctx, bted_stats* out);
 bted_status bted_reset_stats(bted_ctx* ctx);

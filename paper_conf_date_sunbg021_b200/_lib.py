@@ -43,7 +43,8 @@ class bted_params(ctypes.Structure):
 
 class bted_stats(ctypes.Structure):
     _fields_ = [("teds", ctypes.c_uint64), ("k2_launches", ctypes.c_uint64),
-                ("k1_ms", ctypes.c_double), ("k2_ms", ctypes.c_double)]
+                ("k1_ms", ctypes.c_double), ("k2_ms", ctypes.c_double),
+                ("small_teds", ctypes.c_uint64), ("small_ms", ctypes.c_double)]
 
 
 _lib = None
@@ -243,7 +244,8 @@ class PinnedArray:
 def bted_get_stats(ctx: int) -> dict:
     st = bted_stats()
     check(lib().bted_get_stats(ctx, ctypes.byref(st)))
-    return dict(teds=st.teds, k2_launches=st.k2_launches, k1_ms=st.k1_ms, k2_ms=st.k2_ms)
+    return dict(teds=st.teds, k2_launches=st.k2_launches, k1_ms=st.k1_ms, k2_ms=st.k2_ms,
+                small_teds=st.small_teds, small_ms=st.small_ms)
 
 
 def bted_reset_stats(ctx: int):

@@ -88,8 +88,8 @@ struct GraphKey {
 };
 
 struct Stats {
-    uint64_t teds = 0, k2_launches = 0;
-    double k1_ms = 0, k2_ms = 0;
+    uint64_t teds = 0, k2_launches = 0, small_teds = 0;
+    double k1_ms = 0, k2_ms = 0, small_ms = 0;
 };
 
 struct Ted {
@@ -125,7 +125,7 @@ struct Ted {
     // head and loop graphs of each TED, read back at the next host sync.
     bool timing = false;
     bool tma = false;          // packed K2p: TMA-ring variant instead of the LDG one
-    struct Slot { cudaEvent_t e[3]; int32_t m; };
+    struct Slot { cudaEvent_t e[3]; int32_t m; int32_t small; };   // small > 0: one cluster launch of `small` TEDs
     std::vector<Slot> slots;
     size_t used = 0;
     Stats stats;
@@ -216,6 +216,7 @@ struct Ted {
         }
         Slot* sl = &slots[used++];
         sl->m = m;
+        sl->small = 0;
         return sl;
     }
 
@@ -223,6 +224,12 @@ struct Ted {
     void collect() {
         for (size_t i = 0; i < used; ++i) {
             float a = 0, b = 0;
+            if (slots[i].small > 0) {
+                CK(cudaEventElapsedTime(&a, slots[i].e[0], slots[i].e[1]));
+                stats.small_ms += a;
+                stats.small_teds += (uint64_t)slots[i].small;
+                continue;
+            }
             CK(cudaEventElapsedTime(&a, slots[i].e[0], slots[i].e[1]));
             stats.k1_ms += a;
             if (slots[i].m > 1) {
@@ -833,7 +840,10 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
             sample_batch(ctx, st, ctx->N, M, b, ctx->params.seed, ctx->sall + (size_t)kk * M);
             gather(ctx, st, ctx->sall + (size_t)kk * M, M, ctx->xall + (size_t)kk * M * ctx->d);
         }
+        Ted::Slot* sl = T.timing ? T.next_slot(m) : nullptr;
+        if (sl) { sl->small = nb; CK(cudaEventRecord(sl->e[0], st)); }
         launch_small(ctx->xall, nb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->kall, T.err, st);
+        if (sl) CK(cudaEventRecord(sl->e[1], st));
         for (kk = 0; kk < nb; ++kk) {
             bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->kall + (size_t)kk * m, m,
                                                                      ctx->sall + (size_t)kk * M,
@@ -933,7 +943,10 @@ bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, fl
         if (use_small(ctx->params.flags, ctx->N)) {
             grow(T.keys, T.keyscap, (size_t)m);
             if (!T.err) { grow(T.err, T.errcap, 1); CK(cudaMemsetAsync(T.err, 0, sizeof(int), T.stream)); }
+            Ted::Slot* sl = T.timing ? T.next_slot(m) : nullptr;
+            if (sl) { sl->small = 1; CK(cudaEventRecord(sl->e[0], T.stream)); }
             launch_small(ctx->X, 1, ctx->N, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, T.keys, T.err, T.stream);
+            if (sl) CK(cudaEventRecord(sl->e[1], T.stream));
             T.last_rows = 0;                       // K lived in shared memory only
             return finish_keys(ctx, T, T.keys, m, out_idx, out_score);
         }
@@ -1140,6 +1153,8 @@ bted_status bted_get_stats(bted_ctx* ctx, bted_stats* out) {
     out->k2_launches = a.k2_launches + b.k2_launches;
     out->k1_ms = a.k1_ms + b.k1_ms;
     out->k2_ms = a.k2_ms + b.k2_ms;
+    out->small_teds = a.small_teds + b.small_teds;
+    out->small_ms = a.small_ms + b.small_ms;
     return BTED_OK;
 }
 
