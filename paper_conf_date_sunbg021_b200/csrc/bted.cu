@@ -521,10 +521,6 @@ struct bted_ctx {
     Ted ted;
     // batches (Alg. 2)
     Ted bted_engine;          // the M x M batch TEDs and the merge TED
-    uint64_t* skeys = nullptr; size_t skeyscap = 0;
-    uint64_t* skeys2 = nullptr; size_t skeys2cap = 0;
-    uint32_t* sidx = nullptr; size_t sidxcap = 0;
-    uint32_t* sidx2 = nullptr; size_t sidx2cap = 0;
     float* Xb = nullptr; size_t xbcap = 0;
     int64_t* winners = nullptr; size_t winnerscap = 0;
     uint32_t* u32a = nullptr; size_t u32acap = 0;
@@ -533,7 +529,12 @@ struct bted_ctx {
     unsigned long long* mkeys = nullptr; size_t mkeyscap = 0;
     void* cub_tmp = nullptr; size_t cub_cap = 0;
     int64_t* out_dev = nullptr; size_t outcap = 0;
-    uint32_t* sall = nullptr; size_t sallcap = 0;          // small-batch path: [nb][M] draws
+    uint32_t* sall = nullptr; size_t sallcap = 0;          // [nb][M] draws (sorted V_b)
+    unsigned* shist = nullptr; size_t shistcap = 0;        // radix-select sampler scratch
+    int* sint = nullptr; size_t sintcap = 0;
+    uint64_t* scand = nullptr; size_t scandcap = 0;
+    uint32_t* ssel = nullptr; size_t sselcap = 0;
+    int* soff = nullptr; size_t soffcap = 0;
     float* xall = nullptr; size_t xallcap = 0;             // [nb][M][d] gathered batches
     unsigned long long* kall = nullptr; size_t kallcap = 0; // [nb][m] keys
     // host staging (pinned)
@@ -730,32 +731,41 @@ int bits_for(uint64_t maxval) {
     return b;
 }
 
-// Alg. 2 l.2 on the device: sidx[0..M) = sorted V_b.  P = pool rows.
-void sample_batch(bted_ctx* ctx, cudaStream_t st, int64_t P, int64_t M, int32_t b, uint64_t seed,
-                  uint32_t* dst = nullptr) {
-    grow(ctx->skeys, ctx->skeyscap, (size_t)P);
-    grow(ctx->skeys2, ctx->skeys2cap, (size_t)P);
-    grow(ctx->sidx, ctx->sidxcap, (size_t)M);
-    grow(ctx->sidx2, ctx->sidx2cap, (size_t)M);
-    const uint64_t hb = bted::splitmix64(seed + (uint64_t)b * bted::kBatchStride);
-    const unsigned g = (unsigned)std::min<int64_t>((P + 255) / 256, 148 * 16);
-    bted::batch_keys_kernel<<<g, 256, 0, st>>>((uint64_t)P, hb, ctx->skeys);
-    LAUNCHED(1);
-    size_t need = 0, need2 = 0;
-    // only the hash half (bits 32..63) needs sorting: the radix sort is stable
-    // and keys arrive in index order, so equal hashes stay ordered by index --
-    // the same order as the full 64-bit key
-    CK(cub::DeviceRadixSort::SortKeys(nullptr, need, ctx->skeys, ctx->skeys2, (int)P, 32, 64, st));
-    if (!dst) dst = ctx->sidx;
-    CK(cub::DeviceRadixSort::SortKeys(nullptr, need2, ctx->sidx2, dst, (int)M, 0, bits_for(P), st));
-    cub_reserve(ctx, std::max(need, need2));
+// Alg. 2 l.2 for batches b_begin, b_begin + b_step, ... (nb of them) at once:
+// out[k][0..M) = sorted V_{b_begin + k b_step}, by radix select (sample.cuh).
+void sample_batches_dev(bted_ctx* ctx, cudaStream_t st, int64_t P, int64_t M, int32_t b_begin, int32_t b_step,
+                        int nb, uint64_t seed, uint32_t* out) {
+    grow(ctx->shist, ctx->shistcap, (size_t)nb * bted::kSelBins);
+    grow(ctx->sint, ctx->sintcap, (size_t)4 * nb + 1);
+    grow(ctx->scand, ctx->scandcap, (size_t)nb * bted::kCandCap);
+    grow(ctx->ssel, ctx->sselcap, (size_t)nb * M);
+    grow(ctx->soff, ctx->soffcap, (size_t)nb + 1);
+    int* bstar = ctx->sint;
+    int* below = ctx->sint + nb;
+    unsigned* nsel = reinterpret_cast<unsigned*>(ctx->sint + 2 * nb);
+    unsigned* ncand = reinterpret_cast<unsigned*>(ctx->sint + 3 * nb);
+    CK(cudaMemsetAsync(ctx->shist, 0, sizeof(unsigned) * nb * bted::kSelBins, st));
+    CK(cudaMemsetAsync(nsel, 0, sizeof(unsigned) * 2 * nb, st));
+    const unsigned gx = (unsigned)std::max<int64_t>(1, std::min<int64_t>((P + 1023) / 1024, 64));
+    bted::sel_hist_kernel<<<dim3(gx, nb), 256, 0, st>>>((uint64_t)P, seed, b_begin, b_step, ctx->shist);
+    bted::sel_thresh_kernel<<<nb, 1024, 0, st>>>(ctx->shist, M, bstar, below);
+    bted::sel_collect_kernel<<<dim3(gx, nb), 256, 0, st>>>((uint64_t)P, seed, b_begin, b_step, M, bstar, ctx->ssel,
+                                                            nsel, ctx->scand, ncand);
+    if (!ctx->bted_engine.err) {
+        grow(ctx->bted_engine.err, ctx->bted_engine.errcap, 1);
+        CK(cudaMemsetAsync(ctx->bted_engine.err, 0, sizeof(int), st));
+    }
+    bted::sel_finish_kernel<<<nb, 1024, 0, st>>>(M, below, ctx->scand, ncand, ctx->ssel, ctx->bted_engine.err);
+    bted::seg_offsets_kernel<<<(nb + 256) / 256, 256, 0, st>>>(nb, M, ctx->soff);
+    LAUNCHED(5);
+    size_t need = 0;
+    const int nbits = bits_for((uint64_t)P);
+    CK(cub::DeviceSegmentedRadixSort::SortKeys(nullptr, need, ctx->ssel, out, (int)(nb * M), nb, ctx->soff,
+                                               ctx->soff + 1, 0, nbits, st));
+    cub_reserve(ctx, need);
     size_t cap = ctx->cub_cap;
-    CK(cub::DeviceRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->skeys, ctx->skeys2, (int)P, 32, 64, st));
-    const unsigned gm = (unsigned)std::min<int64_t>((M + 255) / 256, 148 * 16);
-    bted::low_half_kernel<<<gm, 256, 0, st>>>(ctx->skeys2, M, ctx->sidx2);
-    LAUNCHED(1);
-    cap = ctx->cub_cap;
-    CK(cub::DeviceRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->sidx2, dst, (int)M, 0, bits_for(P), st));
+    CK(cub::DeviceSegmentedRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->ssel, out, (int)(nb * M), nb, ctx->soff,
+                                               ctx->soff + 1, 0, nbits, st));
 }
 
 void gather(bted_ctx* ctx, cudaStream_t st, const uint32_t* idx, int64_t M, float* dst = nullptr) {
@@ -828,23 +838,22 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
     grow(ctx->mkeys, ctx->mkeyscap, (size_t)m);
     cudaStream_t st = ctx->stream;
     const bool no_graph = (ctx->params.flags & BTED_FLAG_NO_GRAPH) != 0;
-    if (nb > 0 && use_small(ctx->params.flags, M)) {
+    if (nb == 0) return 0;
+    // Alg. 2 l.2 for all of this call's batches at once (radix select, sorted V_b)
+    grow(ctx->sall, ctx->sallcap, (size_t)nb * M);
+    sample_batches_dev(ctx, st, ctx->N, M, b_begin, b_step, nb, ctx->params.seed, ctx->sall);
+    if (use_small(ctx->params.flags, M)) {
         // small batches (the paper's M = 500): all batch TEDs in ONE cluster launch
-        grow(ctx->sall, ctx->sallcap, (size_t)nb * M);
         grow(ctx->xall, ctx->xallcap, (size_t)nb * M * ctx->d);
         grow(ctx->kall, ctx->kallcap, (size_t)nb * m);
         Ted& T = ctx->bted_engine;
-        if (!T.err) { grow(T.err, T.errcap, 1); CK(cudaMemsetAsync(T.err, 0, sizeof(int), st)); }
-        int kk = 0;
-        for (int32_t b = b_begin; b < B; b += b_step, ++kk) {
-            sample_batch(ctx, st, ctx->N, M, b, ctx->params.seed, ctx->sall + (size_t)kk * M);
+        for (int kk = 0; kk < nb; ++kk)
             gather(ctx, st, ctx->sall + (size_t)kk * M, M, ctx->xall + (size_t)kk * M * ctx->d);
-        }
         Ted::Slot* sl = T.timing ? T.next_slot(m) : nullptr;
         if (sl) { sl->small = nb; CK(cudaEventRecord(sl->e[0], st)); }
         launch_small(ctx->xall, nb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->kall, T.err, st);
         if (sl) CK(cudaEventRecord(sl->e[1], st));
-        for (kk = 0; kk < nb; ++kk) {
+        for (int kk = 0; kk < nb; ++kk) {
             bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->kall + (size_t)kk * m, m,
                                                                      ctx->sall + (size_t)kk * M,
                                                                      ctx->winners + (size_t)kk * m);
@@ -852,13 +861,12 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
         }
         return nb;
     }
-    int k = 0;
-    for (int32_t b = b_begin; b < B; b += b_step, ++k) {
-        sample_batch(ctx, st, ctx->N, M, b, ctx->params.seed);
-        gather(ctx, st, ctx->sidx, M);
+    for (int k = 0; k < nb; ++k) {
+        const uint32_t* idx = ctx->sall + (size_t)k * M;
+        gather(ctx, st, idx, M);
         run_ted(ctx->bted_engine, ctx->Xb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->mkeys, no_graph,
                 true, use_packed(ctx->params.flags, ctx->d));
-        bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->mkeys, m, ctx->sidx, ctx->winners + (size_t)k * m);
+        bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->mkeys, m, idx, ctx->winners + (size_t)k * m);
         LAUNCHED(1);
     }
     return nb;
@@ -1038,17 +1046,18 @@ bted_status bted_sample_batches(int64_t P, int64_t M, int32_t B, uint64_t seed, 
         CK(cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking));
         ctx->own_stream = true;
         int64_t* dout = nullptr;
-        CK(cudaMalloc(&dout, sizeof(int64_t) * (size_t)M));
-        for (int32_t b = 0; b < B; ++b) {
-            sample_batch(ctx, ctx->stream, P, M, b, seed);
-            const unsigned g = (unsigned)std::min<int64_t>((M + 255) / 256, 1024);
-            bted::u32_to_i64_kernel<<<g, 256, 0, ctx->stream>>>(ctx->sidx, M, dout);
-            LAUNCHED(1);
-            CK(cudaMemcpyAsync(out + (size_t)b * M, dout, sizeof(int64_t) * (size_t)M, cudaMemcpyDeviceToHost,
-                               ctx->stream));
-        }
+        CK(cudaMalloc(&dout, sizeof(int64_t) * (size_t)M * B));
+        grow(ctx->sall, ctx->sallcap, (size_t)M * B);
+        sample_batches_dev(ctx, ctx->stream, P, M, 0, 1, B, seed, ctx->sall);
+        const unsigned g = (unsigned)std::min<int64_t>((M * B + 255) / 256, 4096);
+        bted::u32_to_i64_kernel<<<g, 256, 0, ctx->stream>>>(ctx->sall, M * B, dout);
+        LAUNCHED(1);
+        CK(cudaMemcpyAsync(out, dout, sizeof(int64_t) * (size_t)M * B, cudaMemcpyDeviceToHost, ctx->stream));
         CK(cudaStreamSynchronize(ctx->stream));
         cudaFree(dout);
+        int e = 0;
+        if (ctx->bted_engine.err) CK(cudaMemcpy(&e, ctx->bted_engine.err, sizeof(int), cudaMemcpyDeviceToHost));
+        if (e) { set_error("batch sampling candidate overflow"); return BTED_ENUMERIC; }
         return BTED_OK;
     });
     bted_destroy(ctx);
@@ -1173,9 +1182,9 @@ void bted_destroy(bted_ctx* ctx) {
         if (ctx->stream) cudaStreamSynchronize(ctx->stream);
         ctx->ted.release();
         ctx->bted_engine.release();
-        void* bufs[] = {ctx->skeys, ctx->skeys2, ctx->sidx, ctx->sidx2, ctx->Xb, ctx->winners, ctx->u32a,
+        void* bufs[] = {ctx->Xb, ctx->winners, ctx->u32a,
                         ctx->u32b, ctx->count_dev, ctx->mkeys, ctx->cub_tmp, ctx->out_dev, ctx->sall,
-                        ctx->xall, ctx->kall};
+                        ctx->xall, ctx->kall, ctx->shist, ctx->sint, ctx->scand, ctx->ssel, ctx->soff};
         for (void* b : bufs) if (b) cudaFree(b);
         if (ctx->own_X && ctx->X) cudaFree(ctx->X);
         if (ctx->hkeys) cudaFreeHost(ctx->hkeys);

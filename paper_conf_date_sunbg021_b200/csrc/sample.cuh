@@ -15,19 +15,6 @@ __host__ __device__ __forceinline__ uint64_t splitmix64(uint64_t z) {
 }
 constexpr uint64_t kBatchStride = 0xD1B54A32D192ED03ull;
 
-// key_b(i) = (splitmix64(h_b + i) & 0xFFFFFFFF00000000) | i
-__global__ void batch_keys_kernel(uint64_t P, uint64_t hb, uint64_t* __restrict__ keys) {
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < P;
-         i += (uint64_t)gridDim.x * blockDim.x)
-        keys[i] = (splitmix64(hb + i) & 0xFFFFFFFF00000000ull) | i;
-}
-
-// the M smallest keys (sorted by key) -> their indices (low halves)
-__global__ void low_half_kernel(const uint64_t* __restrict__ sorted, int64_t M, uint32_t* __restrict__ idx) {
-    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < M; j += (int64_t)gridDim.x * blockDim.x)
-        idx[j] = (uint32_t)(sorted[j] & 0xFFFFFFFFull);
-}
-
 // Xb[j][:] = X[idx[j]][:]   (X_b = X[V_b]; one thread per element)
 __global__ void gather_rows_kernel(const float* __restrict__ X, int32_t d, const uint32_t* __restrict__ idx,
                                    int64_t M, float* __restrict__ Xb) {
@@ -74,6 +61,134 @@ __global__ void finite_check_kernel(const float* __restrict__ X, int64_t n, int*
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         ok &= isfinite(X[i]);
     if (__syncthreads_or(!ok) && threadIdx.x == 0) *bad = 1;
+}
+
+// ---------------------------------------------------------------------------
+// Batch draws by radix SELECT instead of a full sort (all batches at once).
+// V_b = the M smallest key_b(i); key order = (hash32, i).  hash32 is computed on
+// the fly, nothing of size P is stored:
+//   sel_hist     histogram of the top 12 bits of hash32 per batch
+//   sel_thresh   the bin b* holding the M-th smallest key, count `below` before it
+//   sel_collect  indices in bins < b* (all selected), keys in bin b* (candidates)
+//   sel_finish   sort the candidates (bitonic, smem), keep the first M - below
+// then one segmented sort puts each V_b in ascending index order.
+constexpr int kSelBins = 4096;
+constexpr int kCandCap = 4096;
+
+__device__ __forceinline__ uint64_t batch_hash_seed(uint64_t seed, int32_t b) {
+    return splitmix64(seed + (uint64_t)b * kBatchStride);
+}
+__device__ __forceinline__ uint32_t hash32_of(uint64_t hb, uint64_t i) {
+    return (uint32_t)(splitmix64(hb + i) >> 32);
+}
+// warp-aggregated atomic increment; every lane of the warp must call it
+__device__ __forceinline__ unsigned warp_agg_inc(unsigned* ctr, bool pred) {
+    const unsigned m = __ballot_sync(0xffffffffu, pred);
+    const int lane = threadIdx.x & 31;
+    unsigned base = 0;
+    if (m) {
+        const int leader = __ffs(m) - 1;
+        if (lane == leader) base = atomicAdd(ctr, (unsigned)__popc(m));
+        base = __shfl_sync(0xffffffffu, base, leader);
+    }
+    return base + (unsigned)__popc(m & ((1u << lane) - 1u));
+}
+
+__global__ void sel_hist_kernel(uint64_t P, uint64_t seed, int32_t b_begin, int32_t b_step,
+                                unsigned* __restrict__ hist) {
+    __shared__ unsigned h[kSelBins];
+    const int k = blockIdx.y;
+    const uint64_t hb = batch_hash_seed(seed, b_begin + k * b_step);
+    for (int q = threadIdx.x; q < kSelBins; q += blockDim.x) h[q] = 0u;
+    __syncthreads();
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < P; i += (uint64_t)gridDim.x * blockDim.x)
+        atomicAdd(&h[hash32_of(hb, i) >> 20], 1u);
+    __syncthreads();
+    for (int q = threadIdx.x; q < kSelBins; q += blockDim.x)
+        if (h[q]) atomicAdd(&hist[(int64_t)k * kSelBins + q], h[q]);
+}
+
+// one CTA (1024 threads) per batch: inclusive scan of the 4096 bins, first bin
+// whose cumulative count reaches M
+__global__ void __launch_bounds__(1024)
+sel_thresh_kernel(const unsigned* __restrict__ hist, int64_t M, int* __restrict__ bstar, int* __restrict__ below) {
+    __shared__ unsigned part[1024];
+    const int k = blockIdx.x, tid = threadIdx.x;
+    const unsigned* hk = hist + (int64_t)k * kSelBins;
+    unsigned v[4], s = 0;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) { v[q] = hk[4 * tid + q]; s += v[q]; }
+    part[tid] = s;
+    __syncthreads();
+    for (int off = 1; off < 1024; off <<= 1) {           // Hillis-Steele inclusive scan
+        const unsigned a = tid >= off ? part[tid - off] : 0u;
+        __syncthreads();
+        part[tid] += a;
+        __syncthreads();
+    }
+    unsigned c = tid ? part[tid - 1] : 0u;                // count before this thread's 4 bins
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        if (c < (unsigned)M && c + v[q] >= (unsigned)M) { bstar[k] = 4 * tid + q; below[k] = (int)c; }
+        c += v[q];
+    }
+}
+
+__global__ void sel_collect_kernel(uint64_t P, uint64_t seed, int32_t b_begin, int32_t b_step, int64_t M,
+                                   const int* __restrict__ bstar, uint32_t* __restrict__ sel,
+                                   unsigned* __restrict__ nsel, uint64_t* __restrict__ cand,
+                                   unsigned* __restrict__ ncand) {
+    const int k = blockIdx.y;
+    const uint64_t hb = batch_hash_seed(seed, b_begin + k * b_step);
+    const unsigned bs = (unsigned)bstar[k];
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    const uint64_t first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t iters = (P + stride - 1) / stride;      // uniform per warp: ballots stay converged
+    for (uint64_t it = 0; it < iters; ++it) {
+        const uint64_t i = first + it * stride;
+        const bool in = i < P;
+        const uint32_t h = in ? hash32_of(hb, i) : 0xFFFFFFFFu;
+        const unsigned bin = h >> 20;
+        const bool is_sel = in && bin < bs, is_cand = in && bin == bs;
+        const unsigned ps = warp_agg_inc(nsel + k, is_sel);
+        if (is_sel) sel[(int64_t)k * M + ps] = (uint32_t)i;
+        const unsigned pc = warp_agg_inc(ncand + k, is_cand);
+        if (is_cand && pc < (unsigned)kCandCap) cand[(int64_t)k * kCandCap + pc] = ((uint64_t)h << 32) | i;
+    }
+}
+
+// one CTA (1024 threads) per batch: bitonic sort of the candidates in smem
+__global__ void __launch_bounds__(1024)
+sel_finish_kernel(int64_t M, const int* __restrict__ below, const uint64_t* __restrict__ cand,
+                  const unsigned* __restrict__ ncand, uint32_t* __restrict__ sel, int* __restrict__ err) {
+    __shared__ uint64_t s[kCandCap];
+    const int k = blockIdx.x, tid = threadIdx.x;
+    const unsigned n = ncand[k];
+    if (n > (unsigned)kCandCap) { if (tid == 0) atomicOr(err, 4); return; }
+    int np = 1;
+    while (np < (int)n) np <<= 1;
+    for (int q = tid; q < np; q += 1024) s[q] = q < (int)n ? cand[(int64_t)k * kCandCap + q] : ~0ull;
+    __syncthreads();
+    for (int size = 2; size <= np; size <<= 1)
+        for (int stride = size >> 1; stride > 0; stride >>= 1) {
+            for (int q = tid; q < np; q += 1024) {
+                const int p = q ^ stride;
+                if (p > q) {
+                    const bool up = (q & size) == 0;
+                    const uint64_t a = s[q], c = s[p];
+                    if ((a > c) == up) { s[q] = c; s[p] = a; }
+                }
+            }
+            __syncthreads();
+        }
+    const int b0 = below[k];
+    const int need = (int)M - b0;
+    for (int q = tid; q < need; q += 1024) sel[(int64_t)k * M + b0 + q] = (uint32_t)(s[q] & 0xFFFFFFFFull);
+}
+
+__global__ void seg_offsets_kernel(int nb, int64_t M, int* __restrict__ off) {
+    const int q = blockIdx.x * blockDim.x + threadIdx.x;
+    if (q <= nb) off[q] = (int)(q * M);
 }
 
 }  // namespace bted
