@@ -70,6 +70,9 @@ typedef enum {
                                    carry K^(t) = K - L L^T by its fp64 factor L; one K.l pass per
                                    step (2 N^2 bytes, read only) + O(N m).  Same selections in
                                    exact arithmetic; fp64 recurrences.  Packed layouts only.   */
+#define BTED_FLAG_NO_REFINE 128u /* disable K4: near ties (fp32 scores within 2e-5 of the best) are
+                                   otherwise re-scored exactly in fp64 from the features and the
+                                   exact argmax taken (packed / implicit engines)               */
 #define BTED_FLAG_TIMING   2u   /* record CUDA events around K1 and the K2 loop of every batch
                                    TED on the ctx stream; read with bted_get_stats()          */
 
@@ -223,6 +226,8 @@ typedef struct {
     double   k2_ms;
     uint64_t small_teds;     /* TEDs run whole by the cluster kernel (small N) */
     double   small_ms;       /* their device time                              */
+    uint64_t refined_steps;  /* K4: near-tie steps re-scored exactly in fp64   */
+    uint64_t corrected_steps;/* K4: of those, steps whose pick changed         */
 } bted_stats;
 bted_status bted_get_stats(bted_ctx* ctx, bted_stats* out);
 bted_status bted_reset_stats(bted_ctx* ctx);

@@ -19,6 +19,7 @@ BTED_FLAG_DENSE = 4
 BTED_FLAG_NO_SMALL = 8
 BTED_FLAG_TMA = 16
 BTED_FLAG_IMPLICIT = 32
+BTED_FLAG_NO_REFINE = 128
 STATUS = {0: "BTED_OK", 1: "BTED_EINVAL", 2: "BTED_ENOMEM", 3: "BTED_ECUDA", 4: "BTED_ENCCL",
           5: "BTED_ENUMERIC", 6: "BTED_ESTATE"}
 
@@ -44,7 +45,8 @@ class bted_params(ctypes.Structure):
 class bted_stats(ctypes.Structure):
     _fields_ = [("teds", ctypes.c_uint64), ("k2_launches", ctypes.c_uint64),
                 ("k1_ms", ctypes.c_double), ("k2_ms", ctypes.c_double),
-                ("small_teds", ctypes.c_uint64), ("small_ms", ctypes.c_double)]
+                ("small_teds", ctypes.c_uint64), ("small_ms", ctypes.c_double),
+                ("refined_steps", ctypes.c_uint64), ("corrected_steps", ctypes.c_uint64)]
 
 
 _lib = None
@@ -245,7 +247,8 @@ def bted_get_stats(ctx: int) -> dict:
     st = bted_stats()
     check(lib().bted_get_stats(ctx, ctypes.byref(st)))
     return dict(teds=st.teds, k2_launches=st.k2_launches, k1_ms=st.k1_ms, k2_ms=st.k2_ms,
-                small_teds=st.small_teds, small_ms=st.small_ms)
+                small_teds=st.small_teds, small_ms=st.small_ms, refined_steps=st.refined_steps,
+                corrected_steps=st.corrected_steps)
 
 
 def bted_reset_stats(ctx: int):

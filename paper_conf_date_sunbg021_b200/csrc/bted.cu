@@ -27,6 +27,7 @@
 #include "packed.cuh"
 #include "small.cuh"
 #include "implicit.cuh"
+#include "refine.cuh"
 
 namespace {
 
@@ -116,6 +117,23 @@ struct Ted {
     double* Hp = nullptr; size_t hpcap = 0;
     double* hv = nullptr; size_t hvcap = 0;
     bool implicit = false;
+    // K4 near-tie refinement (refine.cuh): per-CTA top-2 keys of every step, flags, candidates
+    bool refine = true;
+    unsigned long long* top2 = nullptr; size_t top2cap = 0;
+    int* flags = nullptr; size_t flagscap = 0;
+    uint32_t* cand = nullptr; size_t candcap = 0;
+    int* ncand = nullptr; size_t ncandcap = 0;
+    int* nflag = nullptr; size_t nflagcap = 0;
+    int32_t last_nC = 0;
+
+    void reserve_refine(int64_t NP, int32_t m) {
+        grow(top2, top2cap, (size_t)m * (size_t)(NP / 32) * 2);
+        grow(flags, flagscap, (size_t)m);
+        grow(cand, candcap, (size_t)m * bted::rf::kMaxCand);
+        grow(ncand, ncandcap, (size_t)m);
+        grow(nflag, nflagcap, 1);
+        last_nC = (int32_t)(NP / 32);
+    }
     std::list<std::pair<GraphKey, cudaGraphExec_t>> graphs;   // LRU
     int64_t last_rows = 0, last_ld = 0;
     int last_buf = 0;
@@ -141,6 +159,8 @@ struct Ted {
         if (P) cudaFree(P);
         for (double* q : {P64, Lf, ell, nv, rd, Hp, hv}) if (q) cudaFree(q);
         P64 = Lf = ell = nv = rd = Hp = hv = nullptr;
+        for (void* q : {(void*)top2, (void*)flags, (void*)cand, (void*)ncand, (void*)nflag}) if (q) cudaFree(q);
+        top2 = nullptr; flags = nullptr; cand = nullptr; ncand = nullptr; nflag = nullptr;
         for (auto& sl : slots) for (auto e : sl.e) cudaEventDestroy(e);
         slots.clear();
         K[0] = K[1] = nullptr; XT = nullptr; sel = nullptr; keys = nullptr; err = nullptr;
@@ -164,7 +184,10 @@ struct Ted {
         grow(Hp, hpcap, (NPa / bted::im::kEllRows) * (size_t)(m + 1));
         grow(hv, hvcap, (size_t)m + 1);
         if (!err) { grow(err, errcap, 1); CK(cudaMemsetAsync(err, 0, sizeof(int), stream)); }
+        const void* top2_before = top2;
+        reserve_refine((int64_t)NP, m);
         const void* after[10] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Hp, hv};
+        if (top2 != top2_before) { for (auto& g : graphs) cudaGraphExecDestroy(g.second); graphs.clear(); }
         if (std::memcmp(before, after, sizeof before) != 0) {
             for (auto& g : graphs) cudaGraphExecDestroy(g.second);
             graphs.clear();
@@ -183,6 +206,9 @@ struct Ted {
         grow(keys, keyscap, (size_t)std::max(m, 1));
         grow(P, pcap, (size_t)nT * NP);
         if (!err) { grow(err, errcap, 1); CK(cudaMemsetAsync(err, 0, sizeof(int), stream)); }
+        const void* top2_before = top2;
+        reserve_refine((int64_t)NP, m);
+        if (top2 != top2_before) { for (auto& g : graphs) cudaGraphExecDestroy(g.second); graphs.clear(); }
         const void* after[5] = {K[0], K[1], sel, keys, P};
         if (std::memcmp(before, after, sizeof before) != 0) {
             for (auto& g : graphs) cudaGraphExecDestroy(g.second);
@@ -292,8 +318,8 @@ constexpr size_t kK2pSmem = bted::pk::k2p_smem_bytes(kK2pSub);
 void launch_finalize(Ted& T, int64_t N, int nT, const float* Kout, float mu, const unsigned long long* keys,
                      int32_t t, unsigned long long* key_out) {
     const unsigned grid = (unsigned)((int64_t)nT * bted::pk::T / bted::pk::kFinRows);
-    bted::pk::finalize_packed_kernel<<<grid, bted::pk::kFinThreads, 0, T.stream>>>(T.P, nT, (int32_t)N, Kout, mu,
-                                                                                  T.sel, keys, t, key_out, T.err);
+    bted::pk::finalize_packed_kernel<<<grid, bted::pk::kFinThreads, 0, T.stream>>>(
+        T.P, nT, (int32_t)N, Kout, mu, T.sel, keys, t, key_out, T.err, T.refine ? T.top2 : nullptr);
 }
 
 // Alg. 1 l.1 + first l.3 on the packed tiles.  (2 kernels: K1p, fin)
@@ -366,7 +392,8 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
     bted::im::tile_pass_kernel<true><<<(unsigned)tiles, bted::im::kThreads, bted::im::tile_pass_smem_bytes, T.stream>>>(
         T.K[0], nT, nullptr, T.P64, nullptr, 0, 0, 0, nullptr);
     bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
-        T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, m, 0, T.hv, T.nv, T.rd, T.sel, keys, 0, keys, T.err);
+        T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, m, 0, T.hv, T.nv, T.rd, T.sel, keys, 0, keys, T.err,
+        T.refine ? T.top2 : nullptr);
     LAUNCHED(3);
 }
 
@@ -384,7 +411,8 @@ void enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned long
                                             T.stream>>>(
             T.K[0], nT, T.ell, T.P64, T.Hp, nA, tp + 1, m + 1, T.hv);
         bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
-            T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, m, tp, T.hv, T.nv, T.rd, T.sel, keys, t, keys + t, T.err);
+            T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, m, tp, T.hv, T.nv, T.rd, T.sel, keys, t, keys + t, T.err,
+            T.refine ? T.top2 : nullptr);
         LAUNCHED(3);
     }
 }
@@ -450,8 +478,13 @@ void ensure_packed_attrs() {
 // packed layout unless the caller asks for dense or d is too wide for K1p
 bool use_packed(uint32_t flags, int32_t d) { return !(flags & BTED_FLAG_DENSE) && d <= 32; }
 
+// nflag_dst: K4 near-tie count of this TED (packed / implicit engines), nullable.
+// forced_keys (host, pinned or pageable; nf entries, flagged kForced): preset
+// picks of steps 0..nf-1 (K4 re-run with a corrected prefix; eager launches).
 void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
-             unsigned long long* keys, bool no_graph, bool time_it = true, bool packed = false) {
+             unsigned long long* keys, bool no_graph, bool time_it = true, bool packed = false,
+             int* nflag_dst = nullptr, const unsigned long long* forced_keys = nullptr, int nf = 0) {
+    if (forced_keys) no_graph = true;
     const bool implicit = packed && T.implicit && m <= bted::im::kMaxM;
     if (implicit) {
         ensure_implicit_attrs();
@@ -488,6 +521,8 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
         GraphKey key{X, N, d, m, kernel, 0, mode, fbits(mu), fbits(gamma), keys};
         graph_run(T, key, head_k, head);
     }
+    if (forced_keys && nf > 0)
+        CK(cudaMemcpyAsync(keys, forced_keys, sizeof(unsigned long long) * nf, cudaMemcpyHostToDevice, T.stream));
     if (sl) CK(cudaEventRecord(sl->e[1], T.stream));
     if (m > 1) {
         if (no_graph) {
@@ -498,6 +533,11 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
         }
     }
     if (sl) CK(cudaEventRecord(sl->e[2], T.stream));
+    if (packed && T.refine && nflag_dst) {
+        bted::rf::neartie_check_kernel<<<m, 256, 0, T.stream>>>(T.top2, T.last_nC, keys, bted::rf::kTau, T.flags,
+                                                               T.cand, T.ncand, nflag_dst);
+        LAUNCHED(1);
+    }
 }
 
 
@@ -535,6 +575,17 @@ struct bted_ctx {
     uint64_t* scand = nullptr; size_t scandcap = 0;
     uint32_t* ssel = nullptr; size_t sselcap = 0;
     int* soff = nullptr; size_t soffcap = 0;
+    int* bflag = nullptr; size_t bflagcap = 0;             // K4: near ties per batch TED
+    // K4 refinement scratch
+    uint32_t* rcols = nullptr; size_t rcolscap = 0;
+    double* rG = nullptr; size_t rGcap = 0;
+    double* rA = nullptr; size_t rAcap = 0;
+    double* rW = nullptr; size_t rWcap = 0;
+    double* rpart = nullptr; size_t rpartcap = 0;
+    double* rdiag = nullptr; size_t rdiagcap = 0;
+    double* rout = nullptr; size_t routcap = 0;
+    uint32_t* ridx = nullptr; size_t ridxcap = 0;
+    uint64_t refined_steps = 0, corrected_steps = 0;
     float* xall = nullptr; size_t xallcap = 0;             // [nb][M][d] gathered batches
     unsigned long long* kall = nullptr; size_t kallcap = 0; // [nb][m] keys
     // host staging (pinned)
@@ -622,7 +673,7 @@ bted_status finish_keys(bted_ctx* ctx, Ted& T, const unsigned long long* keys_de
         return BTED_ENUMERIC;
     }
     for (int32_t t = 0; t < m; ++t) {
-        const unsigned long long k = ctx->hkeys[t];
+        const unsigned long long k = ctx->hkeys[t] & ~bted::rf::kForced;   // K4-forced picks carry a flag bit
         if (k == 0ull) { set_error("no candidate at step %d (internal)", t); return BTED_ENUMERIC; }
         if (!map_dev) out_idx[t] = (int64_t)(0xFFFFFFFFu - (uint32_t)(k & 0xFFFFFFFFull));
         if (out_score) {
@@ -689,6 +740,7 @@ bted_status create_common(const float* X, int64_t N, int32_t d, bted_kernel kern
         ctx->ted.timing = ctx->bted_engine.timing = (params->flags & BTED_FLAG_TIMING) != 0;
         ctx->ted.tma = ctx->bted_engine.tma = (params->flags & BTED_FLAG_TMA) != 0;
         ctx->ted.implicit = ctx->bted_engine.implicit = (params->flags & BTED_FLAG_IMPLICIT) != 0;
+        ctx->ted.refine = ctx->bted_engine.refine = (params->flags & BTED_FLAG_NO_REFINE) == 0;
         CK(cudaMallocHost(&ctx->herr, sizeof(int)));
         if (params->x_on_device) {
             ctx->X = const_cast<float*>(X);
@@ -779,6 +831,95 @@ void gather(bted_ctx* ctx, cudaStream_t st, const uint32_t* idx, int64_t M, floa
     LAUNCHED(1);
 }
 
+// ---- K4: near-tie refinement (refine.cuh) ----
+// fp64 closed-form scores of the candidates C after the picks S; returns the
+// exact argmax (ties: lowest index) and its score.
+void refine_step(bted_ctx* ctx, cudaStream_t st, const float* X, int64_t N, int32_t d,
+                 const std::vector<uint32_t>& S, const std::vector<uint32_t>& C, float mu, uint32_t* best,
+                 double* best_score) {
+    const int t = (int)S.size(), nc = (int)C.size(), ncol = t + nc;
+    std::vector<uint32_t> cols(S);
+    cols.insert(cols.end(), C.begin(), C.end());
+    grow(ctx->rcols, ctx->rcolscap, (size_t)ncol);
+    grow(ctx->rG, ctx->rGcap, (size_t)ncol * N);
+    grow(ctx->rA, ctx->rAcap, (size_t)std::max(1, t * t));
+    grow(ctx->rW, ctx->rWcap, (size_t)bted::rf::kMaxCand * std::max(1, t));
+    const int nblk = (int)std::min<int64_t>((N + 255) / 256, 296);
+    grow(ctx->rpart, ctx->rpartcap, (size_t)nblk * bted::rf::kMaxCand);
+    grow(ctx->rdiag, ctx->rdiagcap, (size_t)bted::rf::kMaxCand);
+    grow(ctx->rout, ctx->routcap, (size_t)bted::rf::kMaxCand + 1);
+    grow(ctx->ridx, ctx->ridxcap, 1);
+    CK(cudaMemcpyAsync(ctx->rcols, cols.data(), sizeof(uint32_t) * ncol, cudaMemcpyHostToDevice, st));
+    const int lin = ctx->kernel == BTED_KERNEL_LINEAR ? 1 : 0;
+    bted::rf::refine_cols_kernel<<<dim3((unsigned)((N + 255) / 256), (unsigned)ncol), 256, 0, st>>>(
+        X, (int32_t)N, d, (double)ctx->params.gamma, lin, ctx->rcols, ctx->rG);
+    bted::rf::refine_solve_kernel<<<1, 256, 0, st>>>(ctx->rG, (int32_t)N, ctx->rcols, t, nc, (double)mu, ctx->rA,
+                                                    ctx->rW);
+    bted::rf::refine_resid_kernel<<<nblk, 256, 0, st>>>(ctx->rG, (int32_t)N, ctx->rcols, t, nc, ctx->rW, ctx->rpart,
+                                                       ctx->rdiag);
+    bted::rf::refine_pick_kernel<<<1, 32, 0, st>>>(ctx->rpart, nblk, ctx->rdiag, ctx->rcols, t, nc, (double)mu,
+                                                  ctx->rout, ctx->ridx);
+    LAUNCHED(4);
+    double sc = 0.0;
+    CK(cudaMemcpyAsync(best, ctx->ridx, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&sc, ctx->rout + bted::rf::kMaxCand, sizeof(double), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    *best_score = sc;
+}
+
+inline unsigned long long host_pack_key(float score, uint32_t idx) {
+    uint32_t b;
+    std::memcpy(&b, &score, 4);
+    return ((unsigned long long)(b + 1u) << 32) | (unsigned long long)(0xFFFFFFFFu - idx);
+}
+
+// Resolve the near ties flagged in the last TED run by T on X (keys on the
+// device, T.flags / T.cand filled by its check kernel).  Each flagged step is
+// re-scored exactly (fp64); if the exact argmax differs from the GPU's pick,
+// the TED is re-run with the corrected prefix forced.  On return `keys` on
+// the device holds the final picks (forced ones flagged kForced) and
+// scores_out[t] (nullable) the fp32 score of each pick.
+void refine_ted(bted_ctx* ctx, Ted& T, const float* X, int64_t N, int32_t d, int32_t m, float mu,
+                unsigned long long* keys, float* scores_out) {
+    cudaStream_t st = T.stream;
+    std::vector<unsigned long long> hk(m);
+    std::vector<int> fl(m), nc(m);
+    std::vector<uint32_t> cd((size_t)m * bted::rf::kMaxCand);
+    int checked = -1;
+    for (int rounds = 0; rounds <= m; ++rounds) {
+        CK(cudaMemcpyAsync(hk.data(), keys, sizeof(unsigned long long) * m, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(fl.data(), T.flags, sizeof(int) * m, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(nc.data(), T.ncand, sizeof(int) * m, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(cd.data(), T.cand, sizeof(uint32_t) * cd.size(), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        int ts = -1;
+        for (int t = checked + 1; t < m; ++t)
+            if (fl[t] && nc[t] >= 2) { ts = t; break; }
+        if (ts < 0) break;
+        std::vector<uint32_t> S(ts), C;
+        for (int k = 0; k < ts; ++k) S[k] = 0xFFFFFFFFu - (uint32_t)(hk[k] & 0xFFFFFFFFull);
+        for (int c = 0; c < nc[ts]; ++c) C.push_back(cd[(size_t)ts * bted::rf::kMaxCand + c]);
+        std::sort(C.begin(), C.end());
+        uint32_t best = 0;
+        double bs = 0.0;
+        refine_step(ctx, st, X, N, d, S, C, mu, &best, &bs);
+        ctx->refined_steps++;
+        const uint32_t pick = 0xFFFFFFFFu - (uint32_t)(hk[ts] & 0xFFFFFFFFull);
+        checked = ts;
+        if (best == pick) continue;
+        // corrected pick: re-run with picks 0..ts forced
+        ctx->corrected_steps++;
+        std::vector<unsigned long long> forced(ts + 1);
+        for (int k = 0; k < ts; ++k) forced[k] = hk[k] | bted::rf::kForced;
+        forced[ts] = host_pack_key((float)bs, best) | bted::rf::kForced;
+        if (scores_out) scores_out[ts] = (float)bs;
+        CK(cudaMemsetAsync(T.nflag, 0, sizeof(int), st));
+        run_ted(T, X, N, d, ctx->params.gamma, ctx->kernel, m, mu, keys, true, false, true, T.nflag, forced.data(),
+                ts + 1);
+        CK(cudaStreamSynchronize(st));      // `forced` (pageable) must outlive the copy
+    }
+}
+
 // ---- small TEDs: one cluster kernel per launch runs every step (small.cuh) ----
 int small_cluster_for(int64_t N) {
     if (N < 1 || N > 4096) return 0;
@@ -861,13 +1002,38 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
         }
         return nb;
     }
+    Ted& T = ctx->bted_engine;
+    const bool packed = use_packed(ctx->params.flags, ctx->d);
+    const bool k4 = packed && T.refine;
+    if (k4) {
+        grow(ctx->bflag, ctx->bflagcap, (size_t)nb);
+        CK(cudaMemsetAsync(ctx->bflag, 0, sizeof(int) * nb, st));
+    }
     for (int k = 0; k < nb; ++k) {
         const uint32_t* idx = ctx->sall + (size_t)k * M;
         gather(ctx, st, idx, M);
-        run_ted(ctx->bted_engine, ctx->Xb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->mkeys, no_graph,
-                true, use_packed(ctx->params.flags, ctx->d));
+        run_ted(T, ctx->Xb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->mkeys, no_graph, true, packed,
+                k4 ? ctx->bflag + k : nullptr);
         bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->mkeys, m, idx, ctx->winners + (size_t)k * m);
         LAUNCHED(1);
+    }
+    if (k4) {
+        // K4: batches with near ties are re-run (deterministic) and refined
+        std::vector<int> bf(nb);
+        CK(cudaMemcpyAsync(bf.data(), ctx->bflag, sizeof(int) * nb, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        for (int k = 0; k < nb; ++k) {
+            if (!bf[k]) continue;
+            const uint32_t* idx = ctx->sall + (size_t)k * M;
+            gather(ctx, st, idx, M);
+            CK(cudaMemsetAsync(T.nflag, 0, sizeof(int), st));
+            run_ted(T, ctx->Xb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->mkeys, no_graph, false, packed,
+                    T.nflag);
+            refine_ted(ctx, T, ctx->Xb, M, ctx->d, m, mu, ctx->mkeys, nullptr);
+            bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->mkeys, m, idx,
+                                                                     ctx->winners + (size_t)k * m);
+            LAUNCHED(1);
+        }
     }
     return nb;
 }
@@ -959,9 +1125,24 @@ bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, fl
             return finish_keys(ctx, T, T.keys, m, out_idx, out_score);
         }
         T.reserve(ctx->N, ctx->N, ctx->d, m);
+        const bool packed = use_packed(ctx->params.flags, ctx->d);
+        if (packed && T.refine) {
+            T.reserve_refine(((ctx->N + bted::pk::T - 1) / bted::pk::T) * bted::pk::T, m);
+            CK(cudaMemsetAsync(T.nflag, 0, sizeof(int), T.stream));
+        }
         run_ted(T, ctx->X, ctx->N, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, T.keys,
-                (ctx->params.flags & BTED_FLAG_NO_GRAPH) != 0, true, use_packed(ctx->params.flags, ctx->d));
-        return finish_keys(ctx, T, T.keys, m, out_idx, out_score);
+                (ctx->params.flags & BTED_FLAG_NO_GRAPH) != 0, true, packed, packed ? T.nflag : nullptr);
+        std::vector<float> fixed(m, -1.f);
+        if (packed && T.refine) {
+            int nf = 0;
+            CK(cudaMemcpyAsync(&nf, T.nflag, sizeof(int), cudaMemcpyDeviceToHost, T.stream));
+            CK(cudaStreamSynchronize(T.stream));
+            if (nf > 0) refine_ted(ctx, T, ctx->X, ctx->N, ctx->d, m, mu, T.keys, fixed.data());
+        }
+        bted_status st = finish_keys(ctx, T, T.keys, m, out_idx, out_score);
+        if (st == BTED_OK && out_score)
+            for (int32_t t = 0; t < m; ++t) if (fixed[t] >= 0.f) out_score[t] = fixed[t];
+        return st;
     });
 }
 
@@ -1164,6 +1345,8 @@ bted_status bted_get_stats(bted_ctx* ctx, bted_stats* out) {
     out->k2_ms = a.k2_ms + b.k2_ms;
     out->small_teds = a.small_teds + b.small_teds;
     out->small_ms = a.small_ms + b.small_ms;
+    out->refined_steps = ctx->refined_steps;
+    out->corrected_steps = ctx->corrected_steps;
     return BTED_OK;
 }
 
@@ -1171,6 +1354,7 @@ bted_status bted_reset_stats(bted_ctx* ctx) {
     if (!ctx) { set_error("null argument"); return BTED_EINVAL; }
     ctx->ted.stats = Stats{};
     ctx->bted_engine.stats = Stats{};
+    ctx->refined_steps = ctx->corrected_steps = 0;
     return BTED_OK;
 }
 
@@ -1184,7 +1368,9 @@ void bted_destroy(bted_ctx* ctx) {
         ctx->bted_engine.release();
         void* bufs[] = {ctx->Xb, ctx->winners, ctx->u32a,
                         ctx->u32b, ctx->count_dev, ctx->mkeys, ctx->cub_tmp, ctx->out_dev, ctx->sall,
-                        ctx->xall, ctx->kall, ctx->shist, ctx->sint, ctx->scand, ctx->ssel, ctx->soff};
+                        ctx->xall, ctx->kall, ctx->shist, ctx->sint, ctx->scand, ctx->ssel, ctx->soff,
+                        ctx->bflag, ctx->rcols, ctx->rG, ctx->rA, ctx->rW, ctx->rpart, ctx->rdiag, ctx->rout,
+                        ctx->ridx};
         for (void* b : bufs) if (b) cudaFree(b);
         if (ctx->own_X && ctx->X) cudaFree(ctx->X);
         if (ctx->hkeys) cudaFreeHost(ctx->hkeys);

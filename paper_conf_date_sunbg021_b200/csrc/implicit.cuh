@@ -246,7 +246,7 @@ fin64_kernel(const double* __restrict__ P64, int nT, int32_t N, const float* __r
              const double* __restrict__ L, int32_t ldL, int32_t tp, const double* __restrict__ h,
              double* __restrict__ nv, double* __restrict__ rdiag, const uint8_t* __restrict__ sel,
              const unsigned long long* __restrict__ keys, int32_t t, unsigned long long* __restrict__ key_out,
-             int* __restrict__ err) {
+             int* __restrict__ err, unsigned long long* __restrict__ top2) {
     __shared__ double part[8][kFinRows];
     __shared__ double hs[kMaxM + 1];
     const int lane = threadIdx.x % 32, w = threadIdx.x / 32;
@@ -301,8 +301,15 @@ fin64_kernel(const double* __restrict__ P64, int nT, int32_t N, const float* __r
             key = pack_key(sc, (uint32_t)i);
         }
     }
-    key = warp_max_u64(key);
-    if (lane == 0 && key) atomicMax(key_out, key);
+    const unsigned long long k1 = warp_max_u64(key);
+    if (top2) {                                        // the CTA's best two keys (K4 near-tie check)
+        const unsigned long long k2 = warp_max_u64(key == k1 ? 0ull : key);
+        if (lane == 0) {
+            top2[((int64_t)t * gridDim.x + blockIdx.x) * 2] = k1;
+            top2[((int64_t)t * gridDim.x + blockIdx.x) * 2 + 1] = k2;
+        }
+    }
+    if (lane == 0 && k1) atomicMax(key_out, k1);
 }
 
 }  // namespace im

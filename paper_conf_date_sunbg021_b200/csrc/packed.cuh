@@ -212,7 +212,8 @@ constexpr int kFinRows = 32;
 __global__ void __launch_bounds__(kFinThreads)
 finalize_packed_kernel(const float* __restrict__ P, int nT, int32_t N, const float* __restrict__ K, float mu,
                        const uint8_t* __restrict__ sel, const unsigned long long* __restrict__ keys, int32_t t,
-                       unsigned long long* __restrict__ key_out, int* __restrict__ err) {
+                       unsigned long long* __restrict__ key_out, int* __restrict__ err,
+                       unsigned long long* __restrict__ top2) {
     __shared__ float part[8][kFinRows];
     const int lane = threadIdx.x % 32, w = threadIdx.x / 32;
     const int64_t NP = (int64_t)nT * T;
@@ -250,8 +251,15 @@ finalize_packed_kernel(const float* __restrict__ P, int nT, int32_t N, const flo
             const bool masked = sl || (uint32_t)i == s;
             key = score_key(g, diag, mu, (uint32_t)i, masked, err);
         }
-        key = warp_max_u64(key);
-        if (lane == 0 && key) atomicMax(key_out, key);
+        const unsigned long long k1 = warp_max_u64(key);
+        if (top2) {                                    // the CTA's best two keys (K4 near-tie check)
+            const unsigned long long k2 = warp_max_u64(key == k1 ? 0ull : key);
+            if (lane == 0) {
+                top2[((int64_t)t * gridDim.x + blockIdx.x) * 2] = k1;
+                top2[((int64_t)t * gridDim.x + blockIdx.x) * 2 + 1] = k2;
+            }
+        }
+        if (lane == 0 && k1) atomicMax(key_out, k1);
     }
 }
 

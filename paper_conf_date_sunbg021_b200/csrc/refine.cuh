@@ -1,0 +1,197 @@
+// refine.cuh -- K4: near-tie refinement of the greedy pick (SURVEY.md Sec.
+// 2.3 K4, Sec. 8(c) "numerics vs the 1e-6 gap rule").
+//
+// The fp32 path's scores carry ~1e-6 relative error (mostly from the fp32
+// Gram entries), so two candidates whose exact scores differ by less than a
+// few 1e-6 may be ordered wrongly.  Every finalize kernel therefore also
+// emits its CTA's top-2 keys; after a TED one check kernel finds the steps
+// whose second-best fp32 score is within tau of the best and lists all
+// candidates within tau.  For such a step the host recomputes the
+// candidates' scores in fp64 from the features -- the closed form of the
+// deflation after the selected set S (pin C2):
+//
+//   K^(S)_:c = K_:c - K_:S (K_SS + mu I)^-1 K_Sc,
+//   score_c = ||K^(S)_:c||^2 / (K^(S)_cc + mu)
+//
+// and takes the exact argmax (ties: lowest index).  If it differs from the
+// GPU's pick, the TED is re-run with the corrected prefix forced.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+#include "kernels.cuh"
+
+namespace bted {
+namespace rf {
+
+constexpr float kTau = 2e-5f;          // near-tie window, relative (>= 8x the measured fp32 error)
+constexpr int kMaxCand = 32;
+constexpr unsigned long long kForced = 1ull << 63;   // key flag of a forced (preset) pick
+
+__device__ __forceinline__ float key_score(unsigned long long k) {
+    return __uint_as_float((uint32_t)(k >> 32) - 1u);
+}
+
+// Per step t (one CTA each): reduce the finalize CTAs' (top1, top2) keys; flag
+// a near tie and list the candidates within tau of the best.
+__global__ void __launch_bounds__(256)
+neartie_check_kernel(const unsigned long long* __restrict__ top2, int nC, const unsigned long long* __restrict__ keys,
+                     float tau, int* __restrict__ flags, uint32_t* __restrict__ cand, int* __restrict__ ncand,
+                     int* __restrict__ nflag) {
+    __shared__ unsigned long long red[8];
+    __shared__ int cnt;
+    const int t = blockIdx.x, tid = threadIdx.x;
+    const unsigned long long kt = keys[t];
+    if (kt & kForced) { if (tid == 0) { flags[t] = 0; ncand[t] = 0; } return; }
+    const unsigned long long* p = top2 + (int64_t)t * nC * 2;
+    unsigned long long m1 = 0ull;
+    for (int q = tid; q < 2 * nC; q += 256) m1 = p[q] > m1 ? p[q] : m1;
+    m1 = warp_max_u64(m1);
+    if ((tid & 31) == 0) red[tid >> 5] = m1;
+    if (tid == 0) cnt = 0;
+    __syncthreads();
+    unsigned long long best = 0ull;
+    for (int q = 0; q < 8; ++q) best = red[q] > best ? red[q] : best;
+    __syncthreads();
+    unsigned long long m2 = 0ull;
+    for (int q = tid; q < 2 * nC; q += 256) if (p[q] != best && p[q] > m2) m2 = p[q];
+    m2 = warp_max_u64(m2);
+    if ((tid & 31) == 0) red[tid >> 5] = m2;
+    __syncthreads();
+    unsigned long long second = 0ull;
+    for (int q = 0; q < 8; ++q) second = red[q] > second ? red[q] : second;
+    const float s1 = key_score(best);
+    const float lim = s1 * (1.f - tau);
+    const bool near = second != 0ull && key_score(second) >= lim;
+    if (near) {
+        for (int q = tid; q < 2 * nC; q += 256) {
+            const unsigned long long k = p[q];
+            if (k != 0ull && key_score(k) >= lim) {
+                const int pos = atomicAdd(&cnt, 1);
+                if (pos < kMaxCand) cand[(int64_t)t * kMaxCand + pos] = key_index(k);
+            }
+        }
+    }
+    __syncthreads();
+    if (tid == 0) {
+        flags[t] = near ? 1 : 0;
+        ncand[t] = near ? min(cnt, kMaxCand) : 0;
+        if (near) atomicAdd(nflag, 1);
+    }
+}
+
+// G[j][i] = k(x_i, x_{cols[j]}) in fp64 (direct difference; reading A1), i < N.
+__global__ void refine_cols_kernel(const float* __restrict__ X, int32_t N, int32_t d, double gamma, int32_t linear,
+                                   const uint32_t* __restrict__ cols, double* __restrict__ G) {
+    const int j = blockIdx.y;
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= N) return;
+    const uint32_t c = cols[j];
+    double a = 0.0;
+    for (int k = 0; k < d; ++k) {
+        const double xi = (double)X[(int64_t)i * d + k], xc = (double)X[(int64_t)c * d + k];
+        if (linear) a = __fma_rn(xi, xc, a);
+        else { const double df = xi - xc; a = __fma_rn(df, df, a); }
+    }
+    G[(int64_t)j * N + i] = linear ? a : exp(-gamma * a);
+}
+
+// One CTA: A = K_SS + mu I (t x t) -> Cholesky L L^T -> W[:, c] = A^-1 K_Sc for
+// the nc candidates.  cols = [S (t) | C (nc)], G from refine_cols_kernel.
+__global__ void __launch_bounds__(256)
+refine_solve_kernel(const double* __restrict__ G, int32_t N, const uint32_t* __restrict__ cols, int t, int nc,
+                    double mu, double* __restrict__ A, double* __restrict__ W) {
+    const int tid = threadIdx.x;
+    for (int e = tid; e < t * t; e += 256) {
+        const int a = e / t, b = e % t;
+        A[e] = G[(int64_t)a * N + cols[b]] + (a == b ? mu : 0.0);
+    }
+    __syncthreads();
+    for (int k = 0; k < t; ++k) {                       // right-looking Cholesky, lower triangle
+        if (tid == 0) A[k * t + k] = sqrt(A[k * t + k]);
+        __syncthreads();
+        const double dkk = A[k * t + k];
+        for (int i = k + 1 + tid; i < t; i += 256) A[i * t + k] /= dkk;
+        __syncthreads();
+        for (int e = tid; e < (t - k - 1) * (t - k - 1); e += 256) {
+            const int i = k + 1 + e / (t - k - 1), j = k + 1 + e % (t - k - 1);
+            if (j <= i) A[i * t + j] -= A[i * t + k] * A[j * t + k];
+        }
+        __syncthreads();
+    }
+    for (int c = tid; c < nc; c += 256) {               // W[:, c] = L^-T L^-1 K_Sc
+        double* w = W + (int64_t)c * t;
+        for (int i = 0; i < t; ++i) {                   // forward
+            double v = G[(int64_t)i * N + cols[t + c]];
+            for (int k = 0; k < i; ++k) v -= A[i * t + k] * w[k];
+            w[i] = v / A[i * t + i];
+        }
+        for (int i = t - 1; i >= 0; --i) {              // backward
+            double v = w[i];
+            for (int k = i + 1; k < t; ++k) v -= A[k * t + i] * w[k];
+            w[i] = v / A[i * t + i];
+        }
+    }
+}
+
+// r_ic = K_ic - sum_k K_{i,S_k} W[k][c]; per-CTA partial sums of r_ic^2 (rows in
+// thread order, then a fixed tree) and the residual at the candidate's own row.
+__global__ void __launch_bounds__(256)
+refine_resid_kernel(const double* __restrict__ G, int32_t N, const uint32_t* __restrict__ cols, int t, int nc,
+                    const double* __restrict__ W, double* __restrict__ part, double* __restrict__ diag) {
+    __shared__ double red[8][kMaxCand];
+    const int tid = threadIdx.x;
+    double acc2[kMaxCand];
+#pragma unroll
+    for (int c = 0; c < kMaxCand; ++c) acc2[c] = 0.0;
+    for (int i = blockIdx.x * 256 + tid; i < N; i += gridDim.x * 256) {
+        double r[kMaxCand];
+#pragma unroll
+        for (int c = 0; c < kMaxCand; ++c) r[c] = c < nc ? G[(int64_t)(t + c) * N + i] : 0.0;
+        for (int k = 0; k < t; ++k) {
+            const double g = G[(int64_t)k * N + i];
+#pragma unroll
+            for (int c = 0; c < kMaxCand; ++c)
+                if (c < nc) r[c] -= g * W[(int64_t)c * t + k];
+        }
+#pragma unroll
+        for (int c = 0; c < kMaxCand; ++c) {
+            if (c < nc) {
+                acc2[c] = __fma_rn(r[c], r[c], acc2[c]);
+                if ((uint32_t)i == cols[t + c]) diag[c] = r[c];
+            }
+        }
+    }
+    for (int c = 0; c < nc; ++c) {
+        double v = acc2[c];
+        for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+        if ((tid & 31) == 0) red[tid >> 5][c] = v;
+    }
+    __syncthreads();
+    if (tid < nc) {
+        double v = 0.0;
+        for (int w = 0; w < 8; ++w) v += red[w][tid];
+        part[(int64_t)blockIdx.x * kMaxCand + tid] = v;
+    }
+}
+
+// exact scores of the candidates and their argmax (ties: lowest index)
+__global__ void refine_pick_kernel(const double* __restrict__ part, int nblocks, const double* __restrict__ diag,
+                                   const uint32_t* __restrict__ cols, int t, int nc, double mu,
+                                   double* __restrict__ out_score, uint32_t* __restrict__ out_idx) {
+    if (threadIdx.x != 0) return;
+    double bs = -1.0;
+    uint32_t bi = 0xFFFFFFFFu;
+    for (int c = 0; c < nc; ++c) {
+        double n = 0.0;
+        for (int b = 0; b < nblocks; ++b) n += part[(int64_t)b * kMaxCand + c];
+        const double sc = n / (diag[c] + mu);
+        const uint32_t idx = cols[t + c];
+        out_score[c] = sc;
+        if (sc > bs || (sc == bs && idx < bi)) { bs = sc; bi = idx; }
+    }
+    out_idx[0] = bi;
+    out_score[kMaxCand] = bs;
+}
+
+}  // namespace rf
+}  // namespace bted
