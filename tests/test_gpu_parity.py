@@ -302,11 +302,11 @@ def test_launch_counter_counts_kernels():
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3, flags=PACKED) as cs:
         cs.select(10, MU)
-    assert bt.bted_kernel_launches() - before == 1 + 20      # finite check + K1p + fin + 9 x (K2p + fin)
+    assert bt.bted_kernel_launches() - before == 1 + 20 + 1  # finite check + K1p + fin + 9 x (K2p + fin) + K4 check
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3, flags=PACKED_TMA) as cs:
         cs.select(10, MU)
-    assert bt.bted_kernel_launches() - before == 1 + 20      # finite check + K1p + fin + 9 x (TMA K2p + fin)
+    assert bt.bted_kernel_launches() - before == 1 + 20 + 1  # finite check + K1p + fin + 9 x (TMA K2p + fin) + K4
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3) as cs:
         cs.select(10, MU)
