@@ -15,4 +15,5 @@ from .knob_pools import (  # noqa: F401
     config_pool,
     CONFIGS,
     whole_model_nodes,
+    whole_model_pools,
 )

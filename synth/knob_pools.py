@@ -33,7 +33,7 @@ import numpy as np
 __all__ = [
     "ConvWorkload", "KnobSpace", "WORKLOADS", "make_pool", "uniform_pool",
     "median_gamma", "config_pool", "CONFIGS", "ordered_factorizations",
-    "whole_model_nodes", "MU",
+    "whole_model_nodes", "whole_model_pools", "MU",
 ]
 
 
@@ -234,8 +234,22 @@ CONFIGS = {
     "vgg16": dict(workload="vgg16_conv1_1", d=16, pool=1 << 20, M=32768, B=8, m=64, seed=16),
     "oversized": dict(workload="vgg16_conv1_1", d=16, pool=1 << 20, M=65536, B=1, m=64, seed=65536),
     "paper": dict(workload="vgg16_conv1_1", d=16, pool=1 << 20, M=500, B=10, m=64, seed=2021),
+    # ResNet-50 + MobileNet-v2: 40 nodes x 4 batches of 32768 (whole_model_pools)
+    "wholemodel": dict(workload="resnet50+mobilenetv2 (40 nodes)", d=16, pool=1 << 20, M=32768, B=4, m=64, seed=5000),
 }
 MU = 0.1
+
+
+def whole_model_pools(pool: int = 1 << 20, d: int = 16, nodes=None):
+    """[(node, X fp32 [P_node, d], gamma)] for the 'wholemodel' config: the first
+    20 unique conv workloads of ResNet-50 and of MobileNet-v2, pool P =
+    min(pool, |D|) each, seed = 5000 + node index."""
+    out = []
+    for k, wl in enumerate(whole_model_nodes() if nodes is None else nodes):
+        space = KnobSpace(wl, d)
+        _, X = make_pool(space, pool, 5000 + k)
+        out.append((wl, X, median_gamma(X, 5000 + k)))
+    return out
 
 
 def config_pool(name: str, pool: int | None = None):
