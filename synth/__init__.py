@@ -16,4 +16,5 @@ from .knob_pools import (  # noqa: F401
     CONFIGS,
     whole_model_nodes,
     whole_model_pools,
+    MU,
 )
