@@ -234,6 +234,8 @@ CONFIGS = {
     "vgg16": dict(workload="vgg16_conv1_1", d=16, pool=1 << 20, M=32768, B=8, m=64, seed=16),
     "oversized": dict(workload="vgg16_conv1_1", d=16, pool=1 << 20, M=65536, B=1, m=64, seed=65536),
     "paper": dict(workload="vgg16_conv1_1", d=16, pool=1 << 20, M=500, B=10, m=64, seed=2021),
+    # one un-batched TED on 131072 points (K = 34 GB packed per buffer)
+    "large": dict(workload="vgg16_conv1_1", d=16, pool=1 << 20, M=131072, B=1, m=64, seed=131072),
     # ResNet-50 + MobileNet-v2: 40 nodes x 4 batches of 32768 (whole_model_pools)
     "wholemodel": dict(workload="resnet50+mobilenetv2 (40 nodes)", d=16, pool=1 << 20, M=32768, B=4, m=64, seed=5000),
 }

@@ -491,3 +491,26 @@ def test_k4_in_batches_matches_oracle_strictly():
     for b in range(B):
         pos = _positions(batches[b], bidx[b])
         check_ted(pos, [], dense.ted(X[batches[b]], g, MU, m, forced=pos), f"k4-batch{b}", gap_exact=GAP_K4)
+
+
+def test_large_131072_sampled_against_closed_form():
+    """one un-batched TED on N = 131072 (K = 34 GB per packed
+    buffer), P1 at every step and sampled P2, as for 'oversized'."""
+    from oracle.closed_form import ClosedForm
+    X, g, cfg = config_pool("large")
+    V = oracle_sample_batches(X.shape[0], cfg["M"], 1, cfg["seed"])[0]
+    Xb = X[V]
+    m = cfg["m"]
+    with bt.CandidateSet(Xb, g) as cs:
+        idx, sc = cs.select(m, MU)
+    assert len(set(idx.tolist())) == m
+    cf = ClosedForm(Xb, g, MU)
+    rng = np.random.default_rng(131072)
+    for t in range(m):
+        s64 = cf.scores([idx[t]])[0]
+        assert abs(float(sc[t]) - s64) <= 1e-5 * s64, (t, float(sc[t]), s64)
+        if t in (0, 32, m - 1):
+            cand = rng.choice(cfg["M"], 192, replace=False)
+            cand = np.array([c for c in cand if c not in set(idx[:t].tolist())])
+            assert cf.scores(cand).max() <= s64 * (1 + 1e-6)
+        cf.add(idx[t])
