@@ -454,7 +454,7 @@ def bench_sharded(args, X, gamma, cfg, comm, dev, world, rank):
     stream = torch.cuda.Stream(dev)
     r0, r1, _ = band(M, world, rank)
     shard = LibShard(Xb, M, cfg["d"], gamma, r0, r1, dev, stream)
-    st = ShardedTed(shard, M, comm, dev, stream)
+    st = ShardedTed(shard, M, comm, dev, stream, graph=True)
     for _ in range(args.warmup):
         st.select(m, mu)
     clocks = Clocks(int(os.environ.get("LOCAL_RANK", "0")))

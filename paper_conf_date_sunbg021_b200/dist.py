@@ -125,30 +125,51 @@ class LibShard:
 
 class ShardedTed:
     """TED (Alg. 1) on N rows with this rank's band of K.  `backend` runs the
-    band's kernels (LibShard on a GPU); `comm` does the two per-step exchanges."""
+    band's kernels (LibShard on a GPU); `comm` does the two per-step exchanges.
+    With `graph=True` (GPU, a CUDA stream given) the whole m-step loop --
+    kernels AND the NCCL collectives -- is captured once per (m, mu) into a
+    CUDA graph and replayed: no per-step host work."""
 
-    def __init__(self, backend, N: int, comm, device: torch.device, stream=None):
+    def __init__(self, backend, N: int, comm, device: torch.device, stream=None, graph: bool = False):
         self.be, self.N, self.comm, self.device, self.stream = backend, int(N), comm, device, stream
         self.row0, self.row1, self.bandB = band(self.N, comm.world, comm.rank)
         width = max(getattr(backend, "ld", self.N), comm.world * self.bandB)
+        self.graph = bool(graph) and stream is not None
+        self._graphs = {}
         with _stream_ctx(stream):
             self.pivot = torch.zeros(width, dtype=torch.float32, device=device)
             self.col = torch.zeros(self.bandB, dtype=torch.float32, device=device)
 
+    def _loop(self, keys: torch.Tensor, m: int, mu: float):
+        P = self.comm.world
+        keys.zero_()
+        self.be.gram(mu, keys)                                    # l.1 + first l.3 on the band
+        self.comm.allreduce_max_(keys[0:1])                       # global argmax s_1 (8 B)
+        gathered = self.pivot[: P * self.bandB]
+        for t in range(1, m):
+            self.be.pivot_column(t - 1, keys, self.col)           # K[band, s_t]
+            self.comm.allgather_(gathered, self.col)              # column s_t == row s_t (4N B)
+            self.be.step(t, mu, self.pivot, keys)                 # l.5 + next l.3 on the band
+            self.comm.allreduce_max_(keys[t:t + 1])               # s_{t+1}
+
     def select(self, m: int, mu: float):
         if not (1 <= m <= self.N):
             raise ValueError("need 1 <= m <= N")
-        P = self.comm.world
         with _stream_ctx(self.stream):
-            keys = torch.zeros(m, dtype=torch.int64, device=self.device)
-            self.be.gram(mu, keys)                                # l.1 + first l.3 on the band
-            self.comm.allreduce_max_(keys[0:1])                   # global argmax s_1 (8 B)
-            gathered = self.pivot[: P * self.bandB]
-            for t in range(1, m):
-                self.be.pivot_column(t - 1, keys, self.col)       # K[band, s_t]
-                self.comm.allgather_(gathered, self.col)          # column s_t == row s_t (4N B)
-                self.be.step(t, mu, self.pivot, keys)             # l.5 + next l.3 on the band
-                self.comm.allreduce_max_(keys[t:t + 1])           # s_{t+1}
+            if self.graph:
+                gk = (int(m), float(mu))
+                if gk not in self._graphs:
+                    keys = torch.zeros(m, dtype=torch.int64, device=self.device)
+                    self._loop(keys, m, mu)                       # eager once: allocations, NCCL init
+                    g = torch.cuda.CUDAGraph()
+                    with torch.cuda.graph(g, stream=self.stream):
+                        self._loop(keys, m, mu)
+                    self._graphs[gk] = (g, keys)
+                g, keys = self._graphs[gk]
+                g.replay()
+            else:
+                keys = torch.zeros(m, dtype=torch.int64, device=self.device)
+                self._loop(keys, m, mu)
             host = keys.cpu().numpy().view(np.uint64)
         self.be.check()
         return L.decode_keys(host)

@@ -32,7 +32,8 @@ def nccl_group(need_gpu):
     dist.destroy_process_group()
 
 
-def test_sharded_ted_over_nccl_matches_dense_select(nccl_group):
+@pytest.mark.parametrize("graph", [False, True], ids=["eager", "cuda-graph"])
+def test_sharded_ted_over_nccl_matches_dense_select(nccl_group, graph):
     import torch
     from paper_conf_date_sunbg021_b200.dist import LibShard, ShardedTed, TorchComm, band
     _, X = make_pool(KnobSpace(WORKLOADS["resnet18_layer1"], 16), 5000, 3)
@@ -44,7 +45,10 @@ def test_sharded_ted_over_nccl_matches_dense_select(nccl_group):
     r0, r1, _ = band(5000, comm.world, comm.rank)
     shard = LibShard(X, 5000, 16, g, r0, r1, nccl_group, st_)
     try:
-        sidx, ssc = ShardedTed(shard, 5000, comm, nccl_group, st_).select(32, MU)
+        sted = ShardedTed(shard, 5000, comm, nccl_group, st_, graph=graph)
+        sidx, ssc = sted.select(32, MU)
+        sidx2, _ = sted.select(32, MU)                        # replay (graph) / rerun (eager)
+        assert np.array_equal(sidx2, sidx)
     finally:
         shard.close()
     assert np.array_equal(sidx, idx)
