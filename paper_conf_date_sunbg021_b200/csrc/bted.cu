@@ -116,6 +116,7 @@ struct Ted {
     double* rd = nullptr; size_t rdcap = 0;
     double* Hp = nullptr; size_t hpcap = 0;
     double* hv = nullptr; size_t hvcap = 0;
+    int* kflag = nullptr; size_t kflagcap = 0;   // K has a non-positive-normal entry (exact conversion)
     bool implicit = false;
     // K4 near-tie refinement (refine.cuh): per-CTA top-2 keys of every step, flags, candidates
     bool refine = true;
@@ -159,6 +160,8 @@ struct Ted {
         if (P) cudaFree(P);
         for (double* q : {P64, Lf, ell, nv, rd, Hp, hv}) if (q) cudaFree(q);
         P64 = Lf = ell = nv = rd = Hp = hv = nullptr;
+        if (kflag) cudaFree(kflag);
+        kflag = nullptr;
         for (void* q : {(void*)top2, (void*)flags, (void*)cand, (void*)ncand, (void*)nflag}) if (q) cudaFree(q);
         top2 = nullptr; flags = nullptr; cand = nullptr; ncand = nullptr; nflag = nullptr;
         for (auto& sl : slots) for (auto e : sl.e) cudaEventDestroy(e);
@@ -172,7 +175,7 @@ struct Ted {
         const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
         const size_t tiles = (size_t)bted::pk::num_tiles(nT) * bted::pk::T * bted::pk::T;
         const size_t NP = (size_t)nT * bted::pk::T, NPa = (NP + 255) / 256 * 256;
-        const void* before[10] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Hp, hv};
+        const void* before[11] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Hp, hv, kflag};
         grow(K[0], kcap[0], tiles);
         grow(sel, selcap, NPa);
         grow(keys, keyscap, (size_t)std::max(m, 1));
@@ -183,10 +186,11 @@ struct Ted {
         grow(rd, rdcap, NPa);
         grow(Hp, hpcap, (NPa / bted::im::kEllRows) * (size_t)(m + 1));
         grow(hv, hvcap, (size_t)m + 1);
+        grow(kflag, kflagcap, 1);
         if (!err) { grow(err, errcap, 1); CK(cudaMemsetAsync(err, 0, sizeof(int), stream)); }
         const void* top2_before = top2;
         reserve_refine((int64_t)NP, m);
-        const void* after[10] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Hp, hv};
+        const void* after[11] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Hp, hv, kflag};
         if (top2 != top2_before) { for (auto& g : graphs) cudaGraphExecDestroy(g.second); graphs.clear(); }
         if (std::memcmp(before, after, sizeof before) != 0) {
             for (auto& g : graphs) cudaGraphExecDestroy(g.second);
@@ -361,6 +365,10 @@ void enqueue_loop_packed(Ted& T, int64_t N, int32_t m, float mu, unsigned long l
 }
 
 // ---- implicit deflation (implicit.cuh) ----
+// persistent tile pass: kTPBlocksPerSM CTAs per SM (never more than the tiles)
+unsigned tile_pass_grid(int64_t tiles) {
+    return (unsigned)std::min<int64_t>(tiles, (int64_t)bted::im::kTPBlocksPerSM * num_sms());
+}
 // head: K1p (the packed Gram, read-only from now on), fp64 norm pass, scores.  (3 kernels)
 void ensure_implicit_attrs() {
     static bool done = false;
@@ -369,6 +377,11 @@ void ensure_implicit_attrs() {
                                 (int)bted::im::tile_pass_smem_bytes));
         CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)bted::im::tile_pass_smem_bytes));
+        // two persistent CTAs per SM need the maximum shared-memory carveout
+        CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<true>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                (int)cudaSharedmemCarveoutMaxShared));
+        CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<false>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                (int)cudaSharedmemCarveoutMaxShared));
         done = true;
     }
 }
@@ -380,7 +393,7 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
     const int64_t tiles = bted::pk::num_tiles(nT);
     CK(cudaMemsetAsync(keys, 0, sizeof(unsigned long long) * m, T.stream));
     CK(cudaMemsetAsync(T.sel, 0, (size_t)NPa, T.stream));
-    CK(cudaMemsetAsync(T.Lf, 0, sizeof(double) * NPa * m, T.stream));
+    CK(cudaMemsetAsync(T.kflag, 0, sizeof(int), T.stream));
     const int lin = kernel == BTED_KERNEL_LINEAR ? 1 : 0;
     float* scratch = reinterpret_cast<float*>(T.P64);      // K1p's fp32 partials are not used here
     if (d <= 16)
@@ -389,10 +402,10 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
     else
         bted::pk::gram_packed_kernel<32><<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
             X, (int32_t)N, d, gamma, lin, T.K[0], nT, scratch);
-    bted::im::tile_pass_kernel<true><<<(unsigned)tiles, bted::im::kThreads, bted::im::tile_pass_smem_bytes, T.stream>>>(
-        T.K[0], nT, nullptr, T.P64, nullptr, 0, 0, 0, nullptr);
+    bted::im::tile_pass_kernel<true><<<tile_pass_grid(tiles), bted::im::kTPThreads, bted::im::tile_pass_smem_bytes,
+                                       T.stream>>>(T.K[0], nT, nullptr, T.P64, nullptr, 0, 0, 0, nullptr, T.kflag);
     bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
-        T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, m, 0, T.hv, T.nv, T.rd, T.sel, keys, 0, keys, T.err,
+        T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, NPa, 0, T.hv, T.nv, T.rd, T.sel, keys, 0, keys, T.err,
         T.refine ? T.top2 : nullptr);
     LAUNCHED(3);
 }
@@ -405,13 +418,13 @@ void enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned long
     const int nA = (int)(NPa / bted::im::kEllRows);
     for (int32_t t = 1; t < m; ++t) {
         const int32_t tp = t - 1;
-        bted::im::ell_kernel<<<nA, bted::im::kThreads, 0, T.stream>>>(T.K[0], nT, (int32_t)N, T.Lf, m, tp, T.rd, mu,
-                                                                      keys, t, T.ell, T.Hp, T.sel);
-        bted::im::tile_pass_kernel<false><<<(unsigned)tiles, bted::im::kThreads, bted::im::tile_pass_smem_bytes,
-                                            T.stream>>>(
-            T.K[0], nT, T.ell, T.P64, T.Hp, nA, tp + 1, m + 1, T.hv);
+        bted::im::ell_kernel<<<nA, bted::im::kThreads, 0, T.stream>>>(T.K[0], nT, (int32_t)N, T.Lf, NPa, tp, T.rd,
+                                                                      mu, keys, t, T.ell, T.Hp, m + 1, T.sel);
+        bted::im::tile_pass_kernel<false><<<tile_pass_grid(tiles), bted::im::kTPThreads,
+                                            bted::im::tile_pass_smem_bytes, T.stream>>>(
+            T.K[0], nT, T.ell, T.P64, T.Hp, nA, tp + 1, m + 1, T.hv, T.kflag);
         bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
-            T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, m, tp, T.hv, T.nv, T.rd, T.sel, keys, t, keys + t, T.err,
+            T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, NPa, tp, T.hv, T.nv, T.rd, T.sel, keys, t, keys + t, T.err,
             T.refine ? T.top2 : nullptr);
         LAUNCHED(3);
     }
