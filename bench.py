@@ -35,7 +35,9 @@ METRIC = "BTED selected points/sec and deflate-step HBM GB/s vs roofline at 1/2/
 UNIT = "points/s"
 K2_NAME = {"dense": "deflate_rescore_kernel",
            "packed": "deflate_packed_ldg_kernel (+ finalize_packed_kernel, per step)",
-           "implicit": "tile_pass_kernel (q = K l, read-only; + ell_kernel + fin64_kernel, per step)"}
+           "implicit": "tile_pass_kernel (q = K l on the read-only packed K; per step incl. ell_kernel + fin64_kernel)"}
+LAYOUT_FLAG = {"dense": 4, "packed": 64, "implicit": 0}          # BTED_FLAG_DENSE / _LITERAL / default
+ALG_BYTES_PER_N2 = {"dense": 8.0, "packed": 4.0, "implicit": 2.0}
 
 
 def parse():
@@ -50,9 +52,9 @@ def parse():
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
                     help="weak: every GPU runs the config's B batches; strong: the config's B batches are split")
-    ap.add_argument("--layout", default="packed", choices=["packed", "dense", "implicit"],
-                    help="K storage: packed upper-triangular tiles (4 N^2 B/step), dense (8 N^2 B/step), "
-                         "or implicit deflation on the read-only packed K (2 N^2 B/step)")
+    ap.add_argument("--layout", default="implicit", choices=["packed", "dense", "implicit"],
+                    help="engine: implicit deflation on the read-only packed K (2 N^2 B/step, the default), "
+                         "literal deflation on packed upper-triangular tiles (4 N^2 B/step) or dense (8 N^2 B/step)")
     return ap.parse_args()
 
 
@@ -208,7 +210,7 @@ def bench_ours(args):
     stream = torch.cuda.Stream(dev)
     X_dev = torch.from_numpy(X).to(dev)
     torch.cuda.synchronize()
-    lay_flag = {"dense": L.BTED_FLAG_DENSE, "packed": 0, "implicit": L.BTED_FLAG_IMPLICIT}[args.layout]
+    lay_flag = LAYOUT_FLAG[args.layout]
     pool = bt.CandidateSet(X_dev, gamma, num_batches=B, seed=cfg["seed"], device=local,
                            flags=L.BTED_FLAG_TIMING | lay_flag, stream=stream.cuda_stream)
 
@@ -257,14 +259,15 @@ def bench_ours(args):
         k2_avg_ms = stats["k2_ms"] / stats["k2_launches"]
         # algorithmic bytes per step: fp32 read + write of K = 8 N^2 (dense) or of
         # its upper triangle = 4 N^2 (packed; report against 4 N^2)
-        alg_bytes = {"dense": 8.0, "packed": 4.0, "implicit": 2.0}[args.layout] * M * M
+        alg_bytes = ALG_BYTES_PER_N2[args.layout] * M * M
         achieved = alg_bytes / (k2_avg_ms / 1e3) / 1e9
         tj = os.path.join(ROOT, "profiles", "k2_traffic.json")
         if os.path.exists(tj):
             with open(tj) as f:
                 tjd = json.load(f)
-            if tjd.get("M") == M and tjd.get("layout", "dense") == args.layout:
-                traffic = tjd.get("dram_bytes_per_launch")
+            ent = tjd.get(args.layout, {})
+            if ent.get("M") == M:
+                traffic = ent.get("dram_bytes_per_launch")
         roofline = {"bound": "hbm", "kernel": K2_NAME[args.layout], "achieved": achieved, "peak": peak,
                     "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
                     "frac_of_8TBs": achieved / 8000.0, "peak_source": peak_src,
@@ -375,7 +378,8 @@ def bench_wholemodel(args, comm, dev, world, rank, local):
     for (wl, X, g), k in zip(pools, mine):
         Xd = torch.from_numpy(X).to(dev)
         ctxs.append((bt.CandidateSet(Xd, g, num_batches=B, seed=cfg["seed"] + k, device=local,
-                                     flags=L.BTED_FLAG_TIMING, stream=stream.cuda_stream), Xd))
+                                     flags=L.BTED_FLAG_TIMING | LAYOUT_FLAG[args.layout],
+                                     stream=stream.cuda_stream), Xd))
     torch.cuda.synchronize()
 
     def step():
@@ -414,7 +418,7 @@ def bench_wholemodel(args, comm, dev, world, rank, local):
         k2_n += stt["k2_launches"]
     peak, peak_src = peaks()
     k2_avg = k2_ms / max(k2_n, 1)
-    alg = 4.0 * M * M
+    alg = ALG_BYTES_PER_N2[args.layout] * M * M
     total_sel = args.steps * len(nodes) * B * m
     for cs, _ in ctxs:
         cs.close()
@@ -422,13 +426,13 @@ def bench_wholemodel(args, comm, dev, world, rank, local):
         line = {"metric": METRIC, "value": total_sel / (ms / 1e3), "unit": UNIT, "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
                 "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
-                "data": "synthetic", "layout": "packed",
+                "data": "synthetic", "layout": args.layout,
                 "config": {"workload": f"wholemodel: ResNet-50 + MobileNet-v2, {len(nodes)} conv nodes (own knob "
                                        f"pools, P = min(2^20, |D|)), B={B} x M={M}, m={m} per node",
                            "nodes": len(nodes), "B_per_node": B, "M": M, "m": m, "mu": MU,
                            "l2": "inputs larger than L2 (K = 4 M^2 bytes per batch)",
                            "parallelism": f"nodes round-robin over {world} GPU(s)"},
-                "roofline": {"bound": "hbm", "kernel": K2_NAME["packed"], "achieved": alg / (k2_avg / 1e3) / 1e9,
+                "roofline": {"bound": "hbm", "kernel": K2_NAME[args.layout], "achieved": alg / (k2_avg / 1e3) / 1e9,
                              "peak": peak, "unit": "GB/s", "frac": alg / (k2_avg / 1e3) / 1e9 / peak,
                              "traffic": None, "peak_source": peak_src, "alg_bytes_per_launch": alg,
                              "avg_launch_ms": k2_avg, "launches_timed": k2_n},

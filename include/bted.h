@@ -66,10 +66,14 @@ typedef enum {
 #define BTED_FLAG_TMA     16u   /* packed layout: stream K through the persistent TMA ring
                                    (cp.async.bulk + mbarrier) instead of the default one-CTA-per-
                                    tile 256-bit-load kernel (which measured faster on B200)   */
-#define BTED_FLAG_IMPLICIT 32u   /* implicit deflation (N2): keep the packed Gram K read-only and
-                                   carry K^(t) = K - L L^T by its fp64 factor L; one K.l pass per
-                                   step (2 N^2 bytes, read only) + O(N m).  Same selections in
-                                   exact arithmetic; fp64 recurrences.  Packed layouts only.   */
+#define BTED_FLAG_IMPLICIT 32u   /* implicit deflation (N2) -- the DEFAULT engine for packed layouts
+                                   with m <= 256 (the flag is accepted and changes nothing): keep
+                                   the packed Gram K read-only and carry K^(t) = K - L L^T by its
+                                   fp64 factor L; one K.l pass per step (2 N^2 bytes, read only)
+                                   + O(N m).  Same selections in exact arithmetic. */
+#define BTED_FLAG_LITERAL  64u   /* literal deflation (Alg. 1 l.5 as written): materialise K^(t)
+                                   every step in the packed layout (K2p, 4 N^2 bytes per step;
+                                   bted_debug_copy_K then returns K^(t)).  Implied by DENSE. */
 #define BTED_FLAG_NO_REFINE 128u /* disable K4: near ties (fp32 scores within 2e-5 of the best) are
                                    otherwise re-scored exactly in fp64 from the features and the
                                    exact argmax taken (packed / implicit engines)               */

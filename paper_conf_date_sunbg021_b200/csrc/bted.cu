@@ -752,7 +752,7 @@ bted_status create_common(const float* X, int64_t N, int32_t d, bted_kernel kern
         ctx->bted_engine.stream = ctx->stream;
         ctx->ted.timing = ctx->bted_engine.timing = (params->flags & BTED_FLAG_TIMING) != 0;
         ctx->ted.tma = ctx->bted_engine.tma = (params->flags & BTED_FLAG_TMA) != 0;
-        ctx->ted.implicit = ctx->bted_engine.implicit = (params->flags & BTED_FLAG_IMPLICIT) != 0;
+        ctx->ted.implicit = ctx->bted_engine.implicit = (params->flags & BTED_FLAG_LITERAL) == 0;
         ctx->ted.refine = ctx->bted_engine.refine = (params->flags & BTED_FLAG_NO_REFINE) == 0;
         CK(cudaMallocHost(&ctx->herr, sizeof(int)));
         if (params->x_on_device) {

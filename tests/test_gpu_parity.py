@@ -13,12 +13,13 @@ from tests.parity import check_ted, ulp32, GAP_K4
 
 pytestmark = pytest.mark.gpu
 MU = float(np.float32(0.1))
-# engine paths: packed tiles (N4), dense rows, and "auto" (the one-kernel
-# cluster TED of small.cuh for N <= ~940, packed above)
-PACKED = L.BTED_FLAG_NO_SMALL
+# engine paths: literal deflation on packed tiles (N4), dense rows, implicit
+# deflation (N2, the default), and "auto" (the one-kernel cluster TED of
+# small.cuh for N <= ~940, implicit above)
+PACKED = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_LITERAL
 DENSE = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_DENSE
-PACKED_TMA = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_TMA
-IMPLICIT = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_IMPLICIT
+PACKED_TMA = L.BTED_FLAG_NO_SMALL | L.BTED_FLAG_TMA | L.BTED_FLAG_LITERAL
+IMPLICIT = L.BTED_FLAG_NO_SMALL                              # the default engine above the cluster TED
 LAYOUTS = pytest.mark.parametrize("flags", [PACKED, PACKED_TMA, DENSE, IMPLICIT, 0],
                                   ids=["packed", "packed-tma", "dense", "implicit", "auto"])
 LAYOUTS_K = pytest.mark.parametrize("flags", [PACKED, PACKED_TMA, DENSE], ids=["packed", "packed-tma", "dense"])
@@ -307,6 +308,10 @@ def test_launch_counter_counts_kernels():
     with bt.CandidateSet(X, 0.3, flags=PACKED_TMA) as cs:
         cs.select(10, MU)
     assert bt.bted_kernel_launches() - before == 1 + 20 + 1  # finite check + K1p + fin + 9 x (TMA K2p + fin) + K4
+    before = bt.bted_kernel_launches()
+    with bt.CandidateSet(X, 0.3, flags=IMPLICIT) as cs:
+        cs.select(10, MU)
+    assert bt.bted_kernel_launches() - before == 1 + 30 + 1  # finite check + K1p + norm pass + fin + 9 x (ell + q + fin) + K4
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3) as cs:
         cs.select(10, MU)
