@@ -1,6 +1,7 @@
 """Build libbted.so (sm_100a) in-tree with nvcc.  No JIT cache, no fallback."""
 from __future__ import annotations
 
+import glob
 import os
 import subprocess
 
@@ -9,8 +10,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libbted.so")
 SOURCES = [os.path.join(CSRC, "bted.cu")]
-DEPS = SOURCES + [os.path.join(CSRC, f) for f in ("kernels.cuh", "sample.cuh")] + \
-    [os.path.join(ROOT, "include", "bted.h")]
+DEPS = SOURCES + sorted(glob.glob(os.path.join(CSRC, "*.cuh"))) + [os.path.join(ROOT, "include", "bted.h")]
 
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
