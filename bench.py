@@ -52,6 +52,8 @@ def parse():
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
                     help="weak: every GPU runs the config's B batches; strong: the config's B batches are split")
+    ap.add_argument("--persistent", action="store_true",
+                    help="implicit engine: run the m-1 steps as one persistent kernel (BTED_FLAG_PERSISTENT_LOOP)")
     ap.add_argument("--layout", default="implicit", choices=["packed", "dense", "implicit"],
                     help="engine: implicit deflation on the read-only packed K (2 N^2 B/step, the default), "
                          "literal deflation on packed upper-triangular tiles (4 N^2 B/step) or dense (8 N^2 B/step)")
@@ -210,7 +212,7 @@ def bench_ours(args):
     stream = torch.cuda.Stream(dev)
     X_dev = torch.from_numpy(X).to(dev)
     torch.cuda.synchronize()
-    lay_flag = LAYOUT_FLAG[args.layout]
+    lay_flag = LAYOUT_FLAG[args.layout] | (256 if args.persistent else 0)
     pool = bt.CandidateSet(X_dev, gamma, num_batches=B, seed=cfg["seed"], device=local,
                            flags=L.BTED_FLAG_TIMING | lay_flag, stream=stream.cuda_stream)
 

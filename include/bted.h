@@ -74,6 +74,9 @@ typedef enum {
 #define BTED_FLAG_LITERAL  64u   /* literal deflation (Alg. 1 l.5 as written): materialise K^(t)
                                    every step in the packed layout (K2p, 4 N^2 bytes per step;
                                    bted_debug_copy_K then returns K^(t)).  Implied by DENSE. */
+#define BTED_FLAG_PERSISTENT_LOOP 256u /* implicit engine: all m-1 steps in ONE cooperative persistent
+                                   kernel with grid barriers between the phases, instead of the
+                                   default three kernels per step (factor column, K.l pass, scores) */
 #define BTED_FLAG_NO_REFINE 128u /* disable K4: near ties (fp32 scores within 2e-5 of the best) are
                                    otherwise re-scored exactly in fp64 from the features and the
                                    exact argmax taken (packed / implicit engines)               */

@@ -21,6 +21,7 @@ BTED_FLAG_TMA = 16
 BTED_FLAG_IMPLICIT = 32
 BTED_FLAG_LITERAL = 64
 BTED_FLAG_NO_REFINE = 128
+BTED_FLAG_PERSISTENT_LOOP = 256
 STATUS = {0: "BTED_OK", 1: "BTED_EINVAL", 2: "BTED_ENOMEM", 3: "BTED_ECUDA", 4: "BTED_ENCCL",
           5: "BTED_ENUMERIC", 6: "BTED_ESTATE"}
 

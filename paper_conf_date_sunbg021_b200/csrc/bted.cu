@@ -16,6 +16,8 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <cstdlib>
+#include <cstdio>
 #include <list>
 #include <new>
 #include <string>
@@ -114,9 +116,13 @@ struct Ted {
     double* ell = nullptr; size_t ellcap = 0;
     double* nv = nullptr; size_t nvcap = 0;
     double* rd = nullptr; size_t rdcap = 0;
-    double* Hp = nullptr; size_t hpcap = 0;
+    double* Qc = nullptr; size_t qccap = 0;      // q = K l of every step, [m][NPa] (h from the history)
+    double* G = nullptr; size_t gcap = 0;        // L^T L, [m][m]
     double* hv = nullptr; size_t hvcap = 0;
     int* kflag = nullptr; size_t kflagcap = 0;   // K has a non-positive-normal entry (exact conversion)
+    int* bar = nullptr; size_t barcap = 0;       // dependency counters of the persistent loop kernel
+    int* tctr = nullptr; size_t tctrcap = 0;     // per-pass tile counters of the K.l passes [m]
+    bool split = true;                           // implicit: three kernels per step (else BTED_FLAG_PERSISTENT_LOOP)
     bool implicit = false;
     // K4 near-tie refinement (refine.cuh): per-CTA top-2 keys of every step, flags, candidates
     bool refine = true;
@@ -158,10 +164,14 @@ struct Ted {
         if (keys) cudaFree(keys);
         if (err) cudaFree(err);
         if (P) cudaFree(P);
-        for (double* q : {P64, Lf, ell, nv, rd, Hp, hv}) if (q) cudaFree(q);
-        P64 = Lf = ell = nv = rd = Hp = hv = nullptr;
+        for (double* q : {P64, Lf, ell, nv, rd, Qc, G, hv}) if (q) cudaFree(q);
+        P64 = Lf = ell = nv = rd = Qc = G = hv = nullptr;
         if (kflag) cudaFree(kflag);
         kflag = nullptr;
+        if (bar) cudaFree(bar);
+        bar = nullptr;
+        if (tctr) cudaFree(tctr);
+        tctr = nullptr;
         for (void* q : {(void*)top2, (void*)flags, (void*)cand, (void*)ncand, (void*)nflag}) if (q) cudaFree(q);
         top2 = nullptr; flags = nullptr; cand = nullptr; ncand = nullptr; nflag = nullptr;
         for (auto& sl : slots) for (auto e : sl.e) cudaEventDestroy(e);
@@ -175,7 +185,7 @@ struct Ted {
         const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
         const size_t tiles = (size_t)bted::pk::num_tiles(nT) * bted::pk::T * bted::pk::T;
         const size_t NP = (size_t)nT * bted::pk::T, NPa = (NP + 255) / 256 * 256;
-        const void* before[11] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Hp, hv, kflag};
+        const void* before[14] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Qc, G, hv, kflag, bar, tctr};
         grow(K[0], kcap[0], tiles);
         grow(sel, selcap, NPa);
         grow(keys, keyscap, (size_t)std::max(m, 1));
@@ -184,13 +194,16 @@ struct Ted {
         grow(ell, ellcap, NPa);
         grow(nv, nvcap, NPa);
         grow(rd, rdcap, NPa);
-        grow(Hp, hpcap, (NPa / bted::im::kEllRows) * (size_t)(m + 1));
+        grow(Qc, qccap, NPa * (size_t)m);
+        grow(G, gcap, (size_t)m * (size_t)m);
         grow(hv, hvcap, (size_t)m + 1);
         grow(kflag, kflagcap, 1);
+        grow(bar, barcap, (size_t)bted::im::loop_sync_ints(NPa / bted::im::kEllRows, m));
+        grow(tctr, tctrcap, (size_t)std::max(m, 1));
         if (!err) { grow(err, errcap, 1); CK(cudaMemsetAsync(err, 0, sizeof(int), stream)); }
         const void* top2_before = top2;
         reserve_refine((int64_t)NP, m);
-        const void* after[11] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Hp, hv, kflag};
+        const void* after[14] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Qc, G, hv, kflag, bar, tctr};
         if (top2 != top2_before) { for (auto& g : graphs) cudaGraphExecDestroy(g.second); graphs.clear(); }
         if (std::memcmp(before, after, sizeof before) != 0) {
             for (auto& g : graphs) cudaGraphExecDestroy(g.second);
@@ -382,6 +395,10 @@ void ensure_implicit_attrs() {
                                 (int)cudaSharedmemCarveoutMaxShared));
         CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<false>, cudaFuncAttributePreferredSharedMemoryCarveout,
                                 (int)cudaSharedmemCarveoutMaxShared));
+        CK(cudaFuncSetAttribute(bted::im::ted_loop_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)bted::im::tile_pass_smem_bytes));
+        CK(cudaFuncSetAttribute(bted::im::ted_loop_kernel, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                (int)cudaSharedmemCarveoutMaxShared));
         done = true;
     }
 }
@@ -394,6 +411,7 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
     CK(cudaMemsetAsync(keys, 0, sizeof(unsigned long long) * m, T.stream));
     CK(cudaMemsetAsync(T.sel, 0, (size_t)NPa, T.stream));
     CK(cudaMemsetAsync(T.kflag, 0, sizeof(int), T.stream));
+    CK(cudaMemsetAsync(T.tctr, 0, sizeof(int) * m, T.stream));
     const int lin = kernel == BTED_KERNEL_LINEAR ? 1 : 0;
     float* scratch = reinterpret_cast<float*>(T.P64);      // K1p's fp32 partials are not used here
     if (d <= 16)
@@ -403,31 +421,110 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
         bted::pk::gram_packed_kernel<32><<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
             X, (int32_t)N, d, gamma, lin, T.K[0], nT, scratch);
     bted::im::tile_pass_kernel<true><<<tile_pass_grid(tiles), bted::im::kTPThreads, bted::im::tile_pass_smem_bytes,
-                                       T.stream>>>(T.K[0], nT, nullptr, T.P64, nullptr, 0, 0, 0, nullptr, T.kflag);
+                                       T.stream>>>(T.K[0], nT, nullptr, T.P64, T.kflag, T.tctr);
     bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
         T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, NPa, 0, T.hv, T.nv, T.rd, T.sel, keys, 0, keys, T.err,
-        T.refine ? T.top2 : nullptr);
+        T.refine ? T.top2 : nullptr, T.Qc);
     LAUNCHED(3);
 }
 
-// loop: per step the new factor column (A), q = K l over the tiles (B), scores (C).  (3(m-1) kernels)
-void enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned long long* keys) {
+bool capturing(cudaStream_t st) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    cudaStreamIsCapturing(st, &cs);
+    return cs != cudaStreamCaptureStatusNone;
+}
+// Grid of the persistent loop kernel: every CTA must be resident at once (grid
+// barriers), so the grid is the measured occupancy x SMs (0: cannot run).
+int loop_kernel_grid() {
+    static int g = -1;
+    if (g < 0) {
+        int nb = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, bted::im::ted_loop_kernel, bted::im::kTPThreads,
+                                                          bted::im::tile_pass_smem_bytes) != cudaSuccess)
+            nb = 0;
+        cudaGetLastError();
+        g = std::min(nb, bted::im::kTPBlocksPerSM) * num_sms();
+    }
+    return g;
+}
+
+// loop: per step the new factor column (A), q = K l over the tiles (B), scores (C).
+// BTED_FLAG_PERSISTENT_LOOP: all m-1 steps in ONE cooperative persistent kernel (ted_loop_kernel:
+// grid barriers between the phases, the TMA producer streams across them).
+// Default (or no co-resident grid): 3(m-1) kernels.
+uint64_t enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned long long* keys) {
     const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
     const int64_t NP = (int64_t)nT * bted::pk::T, NPa = (NP + 255) / 256 * 256;
     const int64_t tiles = bted::pk::num_tiles(nT);
     const int nA = (int)(NPa / bted::im::kEllRows);
+    const int grid = T.split ? 0 : loop_kernel_grid();
+    if (grid > 0) {
+        CK(cudaMemsetAsync(T.bar, 0, sizeof(int) * bted::im::loop_sync_ints(nA, m), T.stream));
+        // BTED_TRACE=<file>: phase timestamps of every CTA and step (debug; eager runs only)
+        static const char* trace_path = std::getenv("BTED_TRACE");
+        static unsigned long long* trace = nullptr;
+        const size_t ntr = (size_t)grid * m * 8;
+        if (trace_path && !trace) CK(cudaMalloc(&trace, sizeof(unsigned long long) * ntr * 4));
+        bted::im::LoopArgs a{T.K[0], nT, (int32_t)N, T.Lf, NPa, m, mu, T.rd, T.nv, keys, T.ell, T.Qc, T.G,
+                             T.hv, T.P64, T.sel, T.err, T.refine ? T.top2 : nullptr, T.kflag,
+                             trace_path ? trace : nullptr, T.bar};
+        cudaLaunchConfig_t cfg{};
+        cfg.gridDim = dim3((unsigned)grid);
+        cfg.blockDim = dim3(bted::im::kTPThreads);
+        cfg.dynamicSmemBytes = bted::im::tile_pass_smem_bytes;
+        cfg.stream = T.stream;
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeCooperative;
+        attr[0].val.cooperative = 1;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        CK(cudaLaunchKernelEx(&cfg, bted::im::ted_loop_kernel, a));
+        LAUNCHED(1);
+        if (trace_path && !capturing(T.stream)) {
+            std::vector<unsigned long long> h(ntr);
+            CK(cudaMemcpyAsync(h.data(), trace, sizeof(unsigned long long) * ntr, cudaMemcpyDeviceToHost, T.stream));
+            CK(cudaStreamSynchronize(T.stream));
+            if (FILE* f = std::fopen(trace_path, "ab")) {
+                const int hdr[3] = {grid, m, 8};
+                std::fwrite(hdr, sizeof hdr, 1, f);
+                std::fwrite(h.data(), sizeof(unsigned long long), ntr, f);
+                std::fclose(f);
+            }
+        }
+        return 1;
+    }
+    // programmatic dependent launches: each kernel may be scheduled while its
+    // predecessor drains (the kernels order themselves with griddepcontrol)
+    cudaLaunchAttribute pdl[1];
+    pdl[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    pdl[0].val.programmaticStreamSerializationAllowed = 1;
+    auto cfg_of = [&](unsigned grid, unsigned block, size_t smem) {
+        cudaLaunchConfig_t c{};
+        c.gridDim = dim3(grid);
+        c.blockDim = dim3(block);
+        c.dynamicSmemBytes = smem;
+        c.stream = T.stream;
+        c.attrs = pdl;
+        c.numAttrs = 1;
+        return c;
+    };
+    const cudaLaunchConfig_t cA = cfg_of((unsigned)nA + 1, bted::im::kThreads, 0);      // + the h CTA
+    const cudaLaunchConfig_t cB = cfg_of(tile_pass_grid(tiles), bted::im::kTPThreads, bted::im::tile_pass_smem_bytes);
+    const cudaLaunchConfig_t cC = cfg_of((unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0);
     for (int32_t t = 1; t < m; ++t) {
         const int32_t tp = t - 1;
-        bted::im::ell_kernel<<<nA, bted::im::kThreads, 0, T.stream>>>(T.K[0], nT, (int32_t)N, T.Lf, NPa, tp, T.rd,
-                                                                      mu, keys, t, T.ell, T.Hp, m + 1, T.sel);
-        bted::im::tile_pass_kernel<false><<<tile_pass_grid(tiles), bted::im::kTPThreads,
-                                            bted::im::tile_pass_smem_bytes, T.stream>>>(
-            T.K[0], nT, T.ell, T.P64, T.Hp, nA, tp + 1, m + 1, T.hv, T.kflag);
-        bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
-            T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, NPa, tp, T.hv, T.nv, T.rd, T.sel, keys, t, keys + t, T.err,
-            T.refine ? T.top2 : nullptr);
+        CK(cudaLaunchKernelEx(&cA, bted::im::ell_kernel, (const float*)T.K[0], nT, (int32_t)N, T.Lf, NPa, tp,
+                              (const double*)T.rd, (const double*)T.nv, mu, (const unsigned long long*)keys, t, T.ell,
+                              (const double*)T.Qc, T.G, m, T.hv, T.sel));
+        CK(cudaLaunchKernelEx(&cB, bted::im::tile_pass_kernel<false>, (const float*)T.K[0], nT, (const double*)T.ell,
+                              T.P64, T.kflag, T.tctr + t));
+        CK(cudaLaunchKernelEx(&cC, bted::im::fin64_kernel, (const double*)T.P64, nT, (int32_t)N,
+                              (const float*)T.K[0], mu, (const double*)T.Lf, NPa, tp, (const double*)T.hv, T.nv, T.rd,
+                              (const uint8_t*)T.sel, (const unsigned long long*)keys, t, keys + t, T.err,
+                              T.refine ? T.top2 : nullptr, T.Qc));
         LAUNCHED(3);
     }
+    return 3 * (uint64_t)(m - 1);
 }
 
 // Alg. 1 l.1 + first l.3: XT, zero keys/sel, K1.  (2 kernels)
@@ -528,6 +625,7 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
     };
     const int mode = implicit ? 3 : packed ? (T.tma ? 2 : 1) : 0;
     const uint64_t head_k = implicit ? 3 : 2, loop_k = implicit ? 3 : packed ? 2 : 1;
+    const uint64_t loop_n = (implicit && !T.split && loop_kernel_grid() > 0) ? 1 : (uint64_t)(m - 1) * loop_k;
     if (no_graph) {
         head();
     } else {
@@ -542,7 +640,7 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
             loop();
         } else {
             GraphKey key{X, N, d, m, kernel, 1, mode, fbits(mu), fbits(gamma), keys};
-            graph_run(T, key, (uint64_t)(m - 1) * loop_k, loop);
+            graph_run(T, key, loop_n, loop);
         }
     }
     if (sl) CK(cudaEventRecord(sl->e[2], T.stream));
@@ -680,6 +778,11 @@ bted_status finish_keys(bted_ctx* ctx, Ted& T, const unsigned long long* keys_de
     CK(cudaStreamSynchronize(T.stream));
     T.collect();
     if (ctx->xbad && take_xbad(ctx)) return BTED_EINVAL;
+    if (*ctx->herr & 4) {
+        CK(cudaMemsetAsync(T.err, 0, sizeof(int), T.stream));
+        set_error("persistent TED loop: grid barrier timed out (CTAs not co-resident)");
+        return BTED_ECUDA;
+    }
     if (*ctx->herr) {
         CK(cudaMemsetAsync(T.err, 0, sizeof(int), T.stream));
         set_error("non-finite score or non-positive k(v,v)+mu during TED");
@@ -754,6 +857,7 @@ bted_status create_common(const float* X, int64_t N, int32_t d, bted_kernel kern
         ctx->ted.tma = ctx->bted_engine.tma = (params->flags & BTED_FLAG_TMA) != 0;
         ctx->ted.implicit = ctx->bted_engine.implicit = (params->flags & BTED_FLAG_LITERAL) == 0;
         ctx->ted.refine = ctx->bted_engine.refine = (params->flags & BTED_FLAG_NO_REFINE) == 0;
+        ctx->ted.split = ctx->bted_engine.split = (params->flags & BTED_FLAG_PERSISTENT_LOOP) == 0;
         CK(cudaMallocHost(&ctx->herr, sizeof(int)));
         if (params->x_on_device) {
             ctx->X = const_cast<float*>(X);

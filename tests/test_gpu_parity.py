@@ -169,7 +169,7 @@ def test_identity_kernel_ties_lowest_index(flags):
         idx, sc = cs.select(10, MU)
     assert idx.tolist() == list(range(10))                   # C9 + reading A5
     assert np.all(sc == sc[0])                               # exact ties
-    if flags & L.BTED_FLAG_IMPLICIT:                         # fp64 recurrence, rounded once to fp32
+    if flags == IMPLICIT:                                    # fp64 recurrence, rounded once to fp32
         np.testing.assert_allclose(sc, 1.0 / (1.0 + MU), rtol=1e-7)
     else:
         assert np.all(sc == np.float32(1.0) / np.float32(np.float32(1.0) + np.float32(MU)))
@@ -309,6 +309,10 @@ def test_launch_counter_counts_kernels():
         cs.select(10, MU)
     assert bt.bted_kernel_launches() - before == 1 + 20 + 1  # finite check + K1p + fin + 9 x (TMA K2p + fin) + K4
     before = bt.bted_kernel_launches()
+    with bt.CandidateSet(X, 0.3, flags=IMPLICIT | L.BTED_FLAG_PERSISTENT_LOOP) as cs:
+        cs.select(10, MU)
+    assert bt.bted_kernel_launches() - before == 1 + 4 + 1   # finite check + K1p + norm pass + fin + the loop kernel + K4
+    before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3, flags=IMPLICIT) as cs:
         cs.select(10, MU)
     assert bt.bted_kernel_launches() - before == 1 + 30 + 1  # finite check + K1p + norm pass + fin + 9 x (ell + q + fin) + K4
@@ -380,6 +384,21 @@ def test_implicit_deflation_matches_oracle(N, m):
     assert np.array_equal(idx, idx2) and np.array_equal(sc.view(np.uint32), sc2.view(np.uint32))
     tr = dense.ted(X, g, MU, m, forced=idx)
     check_ted(idx, sc, tr, f"implicit-{N}")
+
+
+@pytest.mark.parametrize("N,m", [(1000, 64), (4099, 40), (16384, 64), (1500, 256)])
+def test_persistent_loop_equals_step_kernels(N, m):
+    """The one-launch persistent loop (grid barriers) runs the same arithmetic in
+    the same order as the three-kernels-per-step loop: identical picks and score bits."""
+    X = knob(N, seed=N + 5) if N != 1500 else uniform_pool(N, 8, 77)
+    g = median_gamma(X, N)
+    with bt.CandidateSet(X, g, flags=IMPLICIT | L.BTED_FLAG_PERSISTENT_LOOP) as a, \
+            bt.CandidateSet(X, g, flags=IMPLICIT) as b:
+        ia, sa = a.select(m, MU)
+        ib, sb = b.select(m, MU)
+        ia2, sa2 = a.select(m, MU)
+    assert np.array_equal(ia, ib) and np.array_equal(sa.view(np.uint32), sb.view(np.uint32))
+    assert np.array_equal(ia, ia2) and np.array_equal(sa.view(np.uint32), sa2.view(np.uint32))
 
 
 @pytest.mark.parametrize("N", [1, 5, 64, 230, 231, 500, 640, 777, 940])
