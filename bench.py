@@ -52,6 +52,9 @@ def parse():
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
                     help="weak: every GPU runs the config's B batches; strong: the config's B batches are split")
+    ap.add_argument("--norm-mode", default="symmetric", choices=["symmetric", "literal"],
+                    help="oversized row-sharded mode: scores from the band's row norms (default) or the "
+                         "north_star's literal all-reduce(SUM) of partial column norms")
     ap.add_argument("--persistent", action="store_true",
                     help="implicit engine: run the m-1 steps as one persistent kernel (BTED_FLAG_PERSISTENT_LOOP)")
     ap.add_argument("--layout", default="implicit", choices=["packed", "dense", "implicit"],
@@ -460,7 +463,7 @@ def bench_sharded(args, X, gamma, cfg, comm, dev, world, rank):
     stream = torch.cuda.Stream(dev)
     r0, r1, _ = band(M, world, rank)
     shard = LibShard(Xb, M, cfg["d"], gamma, r0, r1, dev, stream)
-    st = ShardedTed(shard, M, comm, dev, stream, graph=True)
+    st = ShardedTed(shard, M, comm, dev, stream, graph=True, norm_mode=args.norm_mode)
     for _ in range(args.warmup):
         st.select(m, mu)
     clocks = Clocks(int(os.environ.get("LOCAL_RANK", "0")))
@@ -490,7 +493,7 @@ def bench_sharded(args, X, gamma, cfg, comm, dev, world, rank):
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
                 "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
                 "data": "synthetic", "layout": "dense-row-sharded",
-                "config": dict(workload_config(args.config, cfg, gamma, world, 1),
+                "config": dict(workload_config(args.config, cfg, gamma, world, 1), norm_mode=args.norm_mode,
                                parallelism=f"row-sharded K over {world} GPUs (NCCL all-reduce + all-gather per step)"),
                 "roofline": {"bound": "hbm", "kernel": "deflate_rescore_kernel (per-GPU band) + NCCL",
                              "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,

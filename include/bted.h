@@ -198,6 +198,28 @@ bted_status bted_shard_step(bted_ctx* shard, int32_t t, float mu, const float* p
                             uint64_t* keys_dev);
 bted_status bted_shard_pivot_column(bted_ctx* shard, int32_t t, const uint64_t* keys_dev,
                                     float* col_dev);
+/*
+ * Literal norm exchange (the north_star's "NCCL allreduce of partial column
+ * norms"; SURVEY §8(e) norm_mode 1, an ablation of the default above).  Alg. 1
+ * l.3 scores v by ||K_v||^2 of v's COLUMN; here every shard
+ * contributes the part of each column inside its band and the caller sums:
+ *   bted_shard_gram(t=0, scratch keys)           (K1 on the band; its keys unused)
+ *   bted_shard_colnorm(t=0, pivot=NULL)          -> colnorm = band column norms
+ *   all-reduce(colnorm, SUM)                     (ld floats)
+ *   bted_shard_scores(t=0, colnorm)              -> keys[0] = band's best key
+ *   all-reduce(keys[t], MAX); bted_shard_pivot_column(t) ; all-gather(col)
+ *   bted_shard_colnorm(t+1, pivot)               (l.5 on the band + column partials)
+ *   all-reduce(colnorm, SUM); bted_shard_scores(t+1, colnorm) -> keys[t+1] ...
+ * colnorm_dev: device fp32 [ld] owned by the caller (written, not read, by
+ *   bted_shard_colnorm; entries >= N are 0).  The band values are bitwise those
+ *   of bted_shard_step; the column sums differ from the row norms only in
+ *   rounding order.  Errors: EINVAL (t < 0, t > 0 without pivot/keys, bad mu),
+ *   ENOMEM, ECUDA, ESTATE.
+ */
+bted_status bted_shard_colnorm(bted_ctx* shard, int32_t t, float mu, const float* pivot_dev,
+                               const uint64_t* keys_dev, float* colnorm_dev);
+bted_status bted_shard_scores(bted_ctx* shard, int32_t t, float mu, const float* colnorm_dev,
+                              uint64_t* keys_dev);
 /* Leading dimension (floats) a pivot buffer must have: pivot_dev[N..ld) must be 0. */
 int64_t     bted_shard_ld(const bted_ctx* shard);
 /* Sticky device error flag of the shard (BTED_ENUMERIC if a NaN score was seen). */

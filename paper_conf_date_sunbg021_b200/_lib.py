@@ -66,6 +66,8 @@ _SIGS = {
     "bted_shard_gram": (ctypes.c_int, [_vp, _f32, _vp]),
     "bted_shard_step": (ctypes.c_int, [_vp, _i32, _f32, _vp, _vp]),
     "bted_shard_pivot_column": (ctypes.c_int, [_vp, _i32, _vp, _vp]),
+    "bted_shard_colnorm": (ctypes.c_int, [_vp, _i32, _f32, _vp, _vp, _vp]),
+    "bted_shard_scores": (ctypes.c_int, [_vp, _i32, _f32, _vp, _vp]),
     "bted_shard_ld": (_i64, [_vp]),
     "bted_shard_check": (ctypes.c_int, [_vp]),
     "bted_destroy": (None, [_vp]),
@@ -185,6 +187,14 @@ def bted_shard_step(ctx: int, t: int, mu: float, pivot_dev: int, keys_dev: int):
 
 def bted_shard_pivot_column(ctx: int, t: int, keys_dev: int, col_dev: int):
     check(lib().bted_shard_pivot_column(ctx, int(t), keys_dev, col_dev))
+
+
+def bted_shard_colnorm(ctx: int, t: int, mu: float, pivot_dev, keys_dev, colnorm_dev: int):
+    check(lib().bted_shard_colnorm(ctx, int(t), float(mu), pivot_dev or None, keys_dev or None, colnorm_dev))
+
+
+def bted_shard_scores(ctx: int, t: int, mu: float, colnorm_dev: int, keys_dev: int):
+    check(lib().bted_shard_scores(ctx, int(t), float(mu), colnorm_dev, keys_dev))
 
 
 def bted_shard_ld(ctx: int) -> int:

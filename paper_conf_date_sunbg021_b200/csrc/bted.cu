@@ -30,6 +30,7 @@
 #include "small.cuh"
 #include "implicit.cuh"
 #include "refine.cuh"
+#include "colnorm.cuh"
 
 namespace {
 
@@ -1402,6 +1403,49 @@ bted_status bted_shard_pivot_column(bted_ctx* ctx, int32_t t, const uint64_t* ke
         bted::pivot_column_kernel<<<g, 256, 0, T.stream>>>(T.K[t & 1], ld_for(ctx->N), rows,
                                                            reinterpret_cast<const unsigned long long*>(keys_dev), t,
                                                            col_dev);
+        LAUNCHED(1);
+        return BTED_OK;
+    });
+}
+
+bted_status bted_shard_colnorm(bted_ctx* ctx, int32_t t, float mu, const float* pivot_dev,
+                               const uint64_t* keys_dev, float* colnorm_dev) {
+    if (!ctx || !colnorm_dev || !ctx->is_shard || t < 0 || (t > 0 && (!pivot_dev || !keys_dev)) || !mu_ok(mu)) {
+        set_error("bad shard_colnorm arguments"); return BTED_EINVAL;
+    }
+    return guarded(ctx, [&]() -> bted_status {
+        Ted& T = ctx->ted;
+        const int64_t ld = ld_for(ctx->N);
+        const int32_t rows = (int32_t)(ctx->row1 - ctx->row0);
+        const int32_t nchunks = (rows + bted::kColChunk - 1) / bted::kColChunk;
+        grow(T.P, T.pcap, (size_t)nchunks * (size_t)ld);
+        const dim3 grid((unsigned)((ld + 255) / 256), (unsigned)nchunks);
+        const auto* keys = reinterpret_cast<const unsigned long long*>(keys_dev);
+        if (t == 0)
+            bted::deflate_colnorm_kernel<false><<<grid, bted::kColThreads, 0, T.stream>>>(
+                T.K[0], nullptr, ld, (int32_t)ctx->row0, rows, nullptr, nullptr, 0, mu, T.sel, T.P);
+        else
+            bted::deflate_colnorm_kernel<true><<<grid, bted::kColThreads, 0, T.stream>>>(
+                T.K[(t - 1) & 1], T.K[t & 1], ld, (int32_t)ctx->row0, rows, pivot_dev, keys, t, mu, T.sel, T.P);
+        const unsigned g2 = (unsigned)std::min<int64_t>((ld + 255) / 256, 2048);
+        bted::colnorm_reduce_kernel<<<g2, 256, 0, T.stream>>>(T.P, nchunks, ld, colnorm_dev);
+        LAUNCHED(2);
+        T.last_buf = t & 1;
+        return BTED_OK;
+    });
+}
+
+bted_status bted_shard_scores(bted_ctx* ctx, int32_t t, float mu, const float* colnorm_dev, uint64_t* keys_dev) {
+    if (!ctx || !colnorm_dev || !keys_dev || !ctx->is_shard || t < 0 || !mu_ok(mu)) {
+        set_error("bad shard_scores arguments"); return BTED_EINVAL;
+    }
+    return guarded(ctx, [&]() -> bted_status {
+        Ted& T = ctx->ted;
+        const int32_t rows = (int32_t)(ctx->row1 - ctx->row0);
+        const unsigned g = (unsigned)std::min<int64_t>((rows + 255) / 256, 1184);
+        bted::colnorm_scores_kernel<<<g, 256, 0, T.stream>>>(T.K[t & 1], ld_for(ctx->N), (int32_t)ctx->row0, rows,
+                                                             colnorm_dev, mu, T.sel,
+                                                             reinterpret_cast<unsigned long long*>(keys_dev), t, T.err);
         LAUNCHED(1);
         return BTED_OK;
     });

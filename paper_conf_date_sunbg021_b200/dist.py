@@ -16,6 +16,11 @@ Two ways Algorithm 2 spreads over GPUs (DESIGN.md
    next deflation needs.  Each rank's rows are computed exactly as on one GPU
    (every row's reduction order depends on N only), so the selection is
    bit-identical to `bted_select` for any number of shards.
+   `norm_mode="literal"` is the north_star's literal exchange instead: every
+   rank sums its band's part of each COLUMN norm (Alg. 1 l.3),
+   an all-reduce(SUM) of those N floats gives ||K_v||^2, and each rank scores
+   its own indices from it (then the same argmax all-reduce).  Same band
+   values; the scores differ from the symmetric mode only in rounding order.
 
 Every step of the method runs in libbted.so's kernels (the `LibShard` /
 `LibPool` backends below); this module only moves buffers between them
@@ -46,6 +51,9 @@ class TorchComm:
 
     def allreduce_max_(self, t: torch.Tensor):
         self.dist.all_reduce(t, op=self.dist.ReduceOp.MAX, group=self.group)
+
+    def allreduce_sum_(self, t: torch.Tensor):
+        self.dist.all_reduce(t, op=self.dist.ReduceOp.SUM, group=self.group)
 
     def allgather_(self, out: torch.Tensor, inp: torch.Tensor):
         self.dist.all_gather_into_tensor(out, inp, group=self.group)
@@ -114,6 +122,13 @@ class LibShard:
     def step(self, t, mu, pivot: torch.Tensor, keys: torch.Tensor):
         L.bted_shard_step(self.ctx, t, mu, pivot.data_ptr(), keys.data_ptr())
 
+    def colnorm(self, t, mu, pivot, keys, colnorm: torch.Tensor):
+        L.bted_shard_colnorm(self.ctx, t, mu, pivot.data_ptr() if pivot is not None else None,
+                             keys.data_ptr() if keys is not None else None, colnorm.data_ptr())
+
+    def scores(self, t, mu, colnorm: torch.Tensor, keys: torch.Tensor):
+        L.bted_shard_scores(self.ctx, t, mu, colnorm.data_ptr(), keys.data_ptr())
+
     def check(self):
         L.bted_shard_check(self.ctx)
 
@@ -130,7 +145,11 @@ class ShardedTed:
     kernels AND the NCCL collectives -- is captured once per (m, mu) into a
     CUDA graph and replayed: no per-step host work."""
 
-    def __init__(self, backend, N: int, comm, device: torch.device, stream=None, graph: bool = False):
+    def __init__(self, backend, N: int, comm, device: torch.device, stream=None, graph: bool = False,
+                 norm_mode: str = "symmetric"):
+        if norm_mode not in ("symmetric", "literal"):
+            raise ValueError("norm_mode must be 'symmetric' or 'literal'")
+        self.norm_mode = norm_mode
         self.be, self.N, self.comm, self.device, self.stream = backend, int(N), comm, device, stream
         self.row0, self.row1, self.bandB = band(self.N, comm.world, comm.rank)
         width = max(getattr(backend, "ld", self.N), comm.world * self.bandB)
@@ -139,8 +158,30 @@ class ShardedTed:
         with _stream_ctx(stream):
             self.pivot = torch.zeros(width, dtype=torch.float32, device=device)
             self.col = torch.zeros(self.bandB, dtype=torch.float32, device=device)
+            if norm_mode == "literal":
+                self.cn = torch.zeros(width, dtype=torch.float32, device=device)
+                self.scratch = torch.zeros(1, dtype=torch.int64, device=device)
+
+    def _loop_literal(self, keys: torch.Tensor, m: int, mu: float):
+        P = self.comm.world
+        keys.zero_()
+        self.be.gram(mu, self.scratch)                            # l.1 on the band
+        self.be.colnorm(0, mu, None, None, self.cn)               # band part of every column norm
+        self.comm.allreduce_sum_(self.cn)                         # ||K_v||^2 (N floats)
+        self.be.scores(0, mu, self.cn, keys)                      # l.3 for the band's own v
+        self.comm.allreduce_max_(keys[0:1])                       # s_1
+        gathered = self.pivot[: P * self.bandB]
+        for t in range(1, m):
+            self.be.pivot_column(t - 1, keys, self.col)
+            self.comm.allgather_(gathered, self.col)              # pivot row s_t (4N B)
+            self.be.colnorm(t, mu, self.pivot, keys, self.cn)     # l.5 on the band + column partials
+            self.comm.allreduce_sum_(self.cn)
+            self.be.scores(t, mu, self.cn, keys)
+            self.comm.allreduce_max_(keys[t:t + 1])               # s_{t+1}
 
     def _loop(self, keys: torch.Tensor, m: int, mu: float):
+        if self.norm_mode == "literal":
+            return self._loop_literal(keys, m, mu)
         P = self.comm.world
         keys.zero_()
         self.be.gram(mu, keys)                                    # l.1 + first l.3 on the band
@@ -177,30 +218,55 @@ class ShardedTed:
 
 # ------------------------------------------------ loopback (P shards, 1 GPU)
 def sharded_select_loopback(X: np.ndarray, gamma: float, P: int, m: int, mu: float, device: torch.device,
-                            stream: torch.cuda.Stream, kernel: int = L.BTED_KERNEL_RBF):
-    """The ShardedTed exchange with P logical shards on ONE GPU; the two
-    collectives are emulated by a device copy and a max.  Exercises the
-    sharded kernels and their bit-identity without a second GPU."""
+                            stream: torch.cuda.Stream, kernel: int = L.BTED_KERNEL_RBF,
+                            norm_mode: str = "symmetric"):
+    """The ShardedTed exchange with P logical shards on ONE GPU; the
+    collectives are emulated by a device copy, a max and (literal norm mode)
+    a sum over the shards in rank order.  Exercises the sharded kernels and
+    their bit-identity without a second GPU."""
     N, d = X.shape
+    literal = norm_mode == "literal"
     shards = []
     try:
         for r in range(P):
             r0, r1, Bw = band(N, P, r)
             shards.append(LibShard(X, N, d, gamma, r0, r1, device, stream, kernel))
         ld = shards[0].ld
+        W = max(ld, P * Bw)
         with torch.cuda.stream(stream):
             keys = torch.zeros((P, m), dtype=torch.int64, device=device)
-            pivot = torch.zeros(max(ld, P * Bw), dtype=torch.float32, device=device)
+            pivot = torch.zeros(W, dtype=torch.float32, device=device)
             cols = torch.zeros((P, Bw), dtype=torch.float32, device=device)
+            cn = torch.zeros((P, W), dtype=torch.float32, device=device)
+            scratch = torch.zeros((P, 1), dtype=torch.int64, device=device)
+
+            def scores(t):
+                tot = cn[0].clone()
+                for r in range(1, P):
+                    tot += cn[r]
+                for r in range(P):
+                    shards[r].scores(t, mu, tot, keys[r])
+
             for r in range(P):
-                shards[r].gram(mu, keys[r])
+                if literal:
+                    shards[r].gram(mu, scratch[r])
+                    shards[r].colnorm(0, mu, None, None, cn[r])
+                else:
+                    shards[r].gram(mu, keys[r])
+            if literal:
+                scores(0)
             keys[:, 0] = keys[:, 0].max()
             for t in range(1, m):
                 for r in range(P):
                     shards[r].pivot_column(t - 1, keys[r], cols[r])
                 pivot[: P * Bw].copy_(cols.reshape(-1))
                 for r in range(P):
-                    shards[r].step(t, mu, pivot, keys[r])
+                    if literal:
+                        shards[r].colnorm(t, mu, pivot, keys[r], cn[r])
+                    else:
+                        shards[r].step(t, mu, pivot, keys[r])
+                if literal:
+                    scores(t)
                 keys[:, t] = keys[:, t].max()
             host = keys[0].cpu().numpy().view(np.uint64)
         for s in shards:

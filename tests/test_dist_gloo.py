@@ -81,27 +81,48 @@ class NumpyShard:
         self.K -= np.outer(a, p) / (p[s] + mu)           # l.5 on the band
         self._key(t, keys)                                # next l.3 over unselected rows
 
+    def colnorm(self, t, mu, pivot, keys, cn):
+        """Literal norm mode: (t > 0) l.5 on the band, then the band's part of every column norm."""
+        if t > 0:
+            s = unpack_idx(int(keys[t - 1]))
+            p = pivot[: self.N].numpy().astype(np.float64)
+            if self.r0 <= s < self.r1:
+                self.sel[s - self.r0] = True
+            self.K -= np.outer(p[self.r0:self.r1], p) / (p[s] + mu)
+        cn.zero_()
+        cn[: self.N] = torch.from_numpy((self.K * self.K).sum(0))
+
+    def scores(self, t, mu, cn, keys):
+        g = cn[self.r0:self.r1].numpy().astype(np.float64)           # all-reduced column norms
+        diag = self.K[np.arange(self.r1 - self.r0), np.arange(self.r0, self.r1)]
+        score = g / (diag + mu)
+        best = 0
+        for lr in range(self.r1 - self.r0):
+            if not self.sel[lr]:
+                best = max(best, pack(score[lr], self.r0 + lr))
+        keys[t] = max(int(keys[t]), best)
+
     def check(self):
         pass
 
 
-def _shard_worker(rank, world, port, X, gamma, m, q):
+def _shard_worker(rank, world, port, X, gamma, m, q, norm_mode="symmetric"):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     from paper_conf_date_sunbg021_b200.dist import ShardedTed, TorchComm, band
     comm = TorchComm()
     r0, r1, _ = band(X.shape[0], world, rank)
-    st = ShardedTed(NumpyShard(X, gamma, r0, r1), X.shape[0], comm, torch.device("cpu"))
+    st = ShardedTed(NumpyShard(X, gamma, r0, r1), X.shape[0], comm, torch.device("cpu"), norm_mode=norm_mode)
     idx, score = st.select(m, MU)
     q.put((rank, idx.tolist(), score.tolist()))
     dist.destroy_process_group()
 
 
-def _run(world, target, *args):
+def _run(world, target, *args, **kw):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = free_port()
-    procs = [ctx.Process(target=target, args=(r, world, port, *args, q)) for r in range(world)]
+    procs = [ctx.Process(target=target, args=(r, world, port, *args, q), kwargs=kw) for r in range(world)]
     for p in procs:
         p.start()
     out = [q.get(timeout=300) for _ in procs]
@@ -120,6 +141,18 @@ def test_sharded_protocol_two_ranks_matches_oracle_and_one_rank():
     assert two[0][1] == two[1][1] == one[0][1]               # every rank decodes the same selection
     tr = literal.ted(X, g, MU, m, forced=two[0][1])
     check_ted(np.array(two[0][1]), np.array(two[0][2]), tr, "gloo-shard")
+
+
+def test_sharded_literal_column_norm_exchange_two_ranks():
+    """norm_mode='literal': all-reduce(SUM) of partial column norms (north_star), same picks."""
+    _, X = make_pool(KnobSpace(WORKLOADS["resnet18_layer1"], 16), 301, 12)
+    g = median_gamma(X, 12)
+    m = 12
+    lit = _run(2, _shard_worker, X, g, m, norm_mode="literal")
+    sym = _run(2, _shard_worker, X, g, m)
+    assert lit[0][1] == lit[1][1] == sym[0][1]
+    tr = literal.ted(X, g, MU, m, forced=lit[0][1])
+    check_ted(np.array(lit[0][1]), np.array(lit[0][2]), tr, "gloo-shard-literal")
 
 
 class NumpyPool:

@@ -55,6 +55,31 @@ def test_sharded_ted_over_nccl_matches_dense_select(nccl_group, graph):
     assert np.array_equal(ssc.view(np.uint32), sc.view(np.uint32))
 
 
+@pytest.mark.parametrize("graph", [False, True], ids=["eager", "cuda-graph"])
+def test_sharded_ted_literal_norms_over_nccl(nccl_group, graph):
+    """norm_mode='literal': the partial column norms go through a real NCCL all-reduce(SUM)."""
+    import torch
+    from oracle import literal
+    from tests.parity import check_ted
+    from paper_conf_date_sunbg021_b200.dist import LibShard, ShardedTed, TorchComm, band
+    N = 3000
+    _, X = make_pool(KnobSpace(WORKLOADS["resnet18_layer1"], 16), N, 4)
+    g = median_gamma(X, 4)
+    comm = TorchComm()
+    st_ = torch.cuda.Stream(nccl_group)
+    r0, r1, _ = band(N, comm.world, comm.rank)
+    shard = LibShard(X, N, 16, g, r0, r1, nccl_group, st_)
+    try:
+        sted = ShardedTed(shard, N, comm, nccl_group, st_, graph=graph, norm_mode="literal")
+        sidx, ssc = sted.select(24, MU)
+        sidx2, ssc2 = sted.select(24, MU)
+        assert np.array_equal(sidx2, sidx) and np.array_equal(ssc2, ssc)
+    finally:
+        shard.close()
+    tr = literal.ted(X, g, MU, 24, forced=sidx.tolist())
+    check_ted(sidx, ssc, tr, "nccl-literal")
+
+
 def test_batch_round_robin_over_nccl_matches_run_batches(nccl_group):
     import torch
     from paper_conf_date_sunbg021_b200.dist import TorchComm, run_batches_dp

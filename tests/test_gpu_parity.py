@@ -294,6 +294,26 @@ def test_row_sharded_loopback_bit_identical(N, P):
     assert np.array_equal(ssc.view(np.uint32), sc.view(np.uint32))
 
 
+@pytest.mark.parametrize("N,P", [(3001, 1), (3001, 3), (1024, 4)])
+def test_row_sharded_literal_column_norms_vs_oracle(N, P):
+    """norm_mode='literal' (north_star: all-reduce of partial column norms): the
+    band values are those of the symmetric mode; the column-norm scores pass
+    P1/P2 against the fp64 oracle along the GPU's picks."""
+    import torch
+    from paper_conf_date_sunbg021_b200.dist import sharded_select_loopback
+    X = knob(N, seed=N + 7 * P)
+    g = median_gamma(X, P)
+    dev = torch.device("cuda", 0)
+    st = torch.cuda.Stream(dev)
+    m = 24
+    lidx, lsc = sharded_select_loopback(X, g, P, m, MU, dev, st, norm_mode="literal")
+    tr = literal.ted(X, g, MU, m, forced=lidx.tolist())
+    check_ted(lidx, lsc, tr, f"literal-colnorm N={N} P={P}")
+    sidx, ssc = sharded_select_loopback(X, g, P, m, MU, dev, st)
+    assert len(set(lidx.tolist())) == m
+    np.testing.assert_allclose(lsc, ssc, rtol=1e-5)         # same numbers up to rounding order
+
+
 def test_launch_counter_counts_kernels():
     X = knob(300)
     before = bt.bted_kernel_launches()
