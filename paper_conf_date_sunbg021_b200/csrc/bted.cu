@@ -383,6 +383,27 @@ void enqueue_loop_packed(Ted& T, int64_t N, int32_t m, float mu, unsigned long l
 unsigned tile_pass_grid(int64_t tiles) {
     return (unsigned)std::min<int64_t>(tiles, (int64_t)bted::im::kTPBlocksPerSM * num_sms());
 }
+// Tiles each K.l pass pins in L2 (evict-last) for the next pass, which runs in
+// the opposite order and starts with them (implicit.cuh tp_produce).  Default
+// kL2KeepFrac = 0 of the device L2 (the serpentine order alone measured best);
+// BTED_L2_KEEP_MB overrides.
+constexpr double kL2KeepFrac = 0.0;
+int l2_keep_tiles(int64_t tiles) {
+    static int64_t bytes = -1;
+    if (bytes < 0) {
+        if (const char* e = std::getenv("BTED_L2_KEEP_MB")) {
+            bytes = (int64_t)(std::atof(e) * 1048576.0);
+        } else {
+            int dev = 0, l2 = 0;
+            cudaGetDevice(&dev);
+            if (cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev) != cudaSuccess) l2 = 0;
+            cudaGetLastError();
+            bytes = (int64_t)(kL2KeepFrac * l2);
+        }
+    }
+    const int64_t tile_bytes = (int64_t)bted::pk::T * bted::pk::T * 4;
+    return (int)std::min<int64_t>(tiles, std::max<int64_t>(0, bytes / tile_bytes));
+}
 // head: K1p (the packed Gram, read-only from now on), fp64 norm pass, scores.  (3 kernels)
 void ensure_implicit_attrs() {
     static bool done = false;
@@ -422,7 +443,8 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
         bted::pk::gram_packed_kernel<32><<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
             X, (int32_t)N, d, gamma, lin, T.K[0], nT, scratch);
     bted::im::tile_pass_kernel<true><<<tile_pass_grid(tiles), bted::im::kTPThreads, bted::im::tile_pass_smem_bytes,
-                                       T.stream>>>(T.K[0], nT, nullptr, T.P64, T.kflag, T.tctr);
+                                       T.stream>>>(T.K[0], nT, nullptr, T.P64, T.kflag, T.tctr, 0,
+                                                   l2_keep_tiles(tiles));
     bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
         T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, NPa, 0, T.hv, T.nv, T.rd, T.sel, keys, 0, keys, T.err,
         T.refine ? T.top2 : nullptr, T.Qc);
@@ -468,7 +490,7 @@ uint64_t enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned 
         if (trace_path && !trace) CK(cudaMalloc(&trace, sizeof(unsigned long long) * ntr * 4));
         bted::im::LoopArgs a{T.K[0], nT, (int32_t)N, T.Lf, NPa, m, mu, T.rd, T.nv, keys, T.ell, T.Qc, T.G,
                              T.hv, T.P64, T.sel, T.err, T.refine ? T.top2 : nullptr, T.kflag,
-                             trace_path ? trace : nullptr, T.bar};
+                             trace_path ? trace : nullptr, T.bar, l2_keep_tiles(tiles)};
         cudaLaunchConfig_t cfg{};
         cfg.gridDim = dim3((unsigned)grid);
         cfg.blockDim = dim3(bted::im::kTPThreads);
@@ -512,13 +534,14 @@ uint64_t enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned 
     const cudaLaunchConfig_t cA = cfg_of((unsigned)nA + 1, bted::im::kThreads, 0);      // + the h CTA
     const cudaLaunchConfig_t cB = cfg_of(tile_pass_grid(tiles), bted::im::kTPThreads, bted::im::tile_pass_smem_bytes);
     const cudaLaunchConfig_t cC = cfg_of((unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0);
+    const int keep = l2_keep_tiles(tiles);
     for (int32_t t = 1; t < m; ++t) {
         const int32_t tp = t - 1;
         CK(cudaLaunchKernelEx(&cA, bted::im::ell_kernel, (const float*)T.K[0], nT, (int32_t)N, T.Lf, NPa, tp,
                               (const double*)T.rd, (const double*)T.nv, mu, (const unsigned long long*)keys, t, T.ell,
                               (const double*)T.Qc, T.G, m, T.hv, T.sel));
         CK(cudaLaunchKernelEx(&cB, bted::im::tile_pass_kernel<false>, (const float*)T.K[0], nT, (const double*)T.ell,
-                              T.P64, T.kflag, T.tctr + t));
+                              T.P64, T.kflag, T.tctr + t, (int)(t & 1), t + 1 < m ? keep : 0));
         CK(cudaLaunchKernelEx(&cC, bted::im::fin64_kernel, (const double*)T.P64, nT, (int32_t)N,
                               (const float*)T.K[0], mu, (const double*)T.Lf, NPa, tp, (const double*)T.hv, T.nv, T.rd,
                               (const uint8_t*)T.sel, (const unsigned long long*)keys, t, keys + t, T.err,
