@@ -617,7 +617,8 @@ bool use_packed(uint32_t flags, int32_t d) { return !(flags & BTED_FLAG_DENSE) &
 // picks of steps 0..nf-1 (K4 re-run with a corrected prefix; eager launches).
 void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
              unsigned long long* keys, bool no_graph, bool time_it = true, bool packed = false,
-             int* nflag_dst = nullptr, const unsigned long long* forced_keys = nullptr, int nf = 0) {
+             int* nflag_dst = nullptr, const unsigned long long* forced_keys = nullptr, int nf = 0,
+             int* flags_dst = nullptr, uint32_t* cand_dst = nullptr, int* ncand_dst = nullptr) {
     if (forced_keys) no_graph = true;
     const bool implicit = packed && T.implicit && m <= bted::im::kMaxM;
     if (implicit) {
@@ -669,8 +670,12 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
     }
     if (sl) CK(cudaEventRecord(sl->e[2], T.stream));
     if (packed && T.refine && nflag_dst) {
-        bted::rf::neartie_check_kernel<<<m, 256, 0, T.stream>>>(T.top2, T.last_nC, keys, bted::rf::kTau, T.flags,
-                                                               T.cand, T.ncand, nflag_dst);
+        // K4 check; its per-step flags/candidates go to T's buffers or, for a batch
+        // TED of Alg. 2, to that batch's own slice (refined later without a re-run)
+        bted::rf::neartie_check_kernel<<<m, 256, 0, T.stream>>>(T.top2, T.last_nC, keys, bted::rf::kTau,
+                                                               flags_dst ? flags_dst : T.flags,
+                                                               cand_dst ? cand_dst : T.cand,
+                                                               ncand_dst ? ncand_dst : T.ncand, nflag_dst);
         LAUNCHED(1);
     }
 }
@@ -711,6 +716,10 @@ struct bted_ctx {
     uint32_t* ssel = nullptr; size_t sselcap = 0;
     int* soff = nullptr; size_t soffcap = 0;
     int* bflag = nullptr; size_t bflagcap = 0;             // K4: near ties per batch TED
+    unsigned long long* bkeys = nullptr; size_t bkeyscap = 0; // K4: [nb][m] keys of every batch TED
+    int* bsflags = nullptr; size_t bsflagscap = 0;           //     [nb][m] per-step near-tie flags
+    int* bncand = nullptr; size_t bncandcap = 0;             //     [nb][m] candidate counts
+    uint32_t* bcand = nullptr; size_t bcandcap = 0;          //     [nb][m][kMaxCand] candidates
     // K4 refinement scratch
     uint32_t* rcols = nullptr; size_t rcolscap = 0;
     double* rG = nullptr; size_t rGcap = 0;
@@ -1146,20 +1155,30 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
     Ted& T = ctx->bted_engine;
     const bool packed = use_packed(ctx->params.flags, ctx->d);
     const bool k4 = packed && T.refine;
+    const size_t nC = (size_t)bted::rf::kMaxCand;
     if (k4) {
         grow(ctx->bflag, ctx->bflagcap, (size_t)nb);
+        grow(ctx->bkeys, ctx->bkeyscap, (size_t)nb * m);
+        grow(ctx->bsflags, ctx->bsflagscap, (size_t)nb * m);
+        grow(ctx->bncand, ctx->bncandcap, (size_t)nb * m);
+        grow(ctx->bcand, ctx->bcandcap, (size_t)nb * m * nC);
         CK(cudaMemsetAsync(ctx->bflag, 0, sizeof(int) * nb, st));
     }
     for (int k = 0; k < nb; ++k) {
         const uint32_t* idx = ctx->sall + (size_t)k * M;
         gather(ctx, st, idx, M);
         run_ted(T, ctx->Xb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->mkeys, no_graph, true, packed,
-                k4 ? ctx->bflag + k : nullptr);
+                k4 ? ctx->bflag + k : nullptr, nullptr, 0, k4 ? ctx->bsflags + (size_t)k * m : nullptr,
+                k4 ? ctx->bcand + (size_t)k * m * nC : nullptr, k4 ? ctx->bncand + (size_t)k * m : nullptr);
+        if (k4)
+            CK(cudaMemcpyAsync(ctx->bkeys + (size_t)k * m, ctx->mkeys, sizeof(unsigned long long) * m,
+                               cudaMemcpyDeviceToDevice, st));
         bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->mkeys, m, idx, ctx->winners + (size_t)k * m);
         LAUNCHED(1);
     }
     if (k4) {
-        // K4: batches with near ties are re-run (deterministic) and refined
+        // K4: the near-tie steps of each flagged batch TED are re-scored exactly
+        // from its kept keys/flags/candidates; a TED is re-run only if a pick changes
         std::vector<int> bf(nb);
         CK(cudaMemcpyAsync(bf.data(), ctx->bflag, sizeof(int) * nb, cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
@@ -1167,9 +1186,12 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
             if (!bf[k]) continue;
             const uint32_t* idx = ctx->sall + (size_t)k * M;
             gather(ctx, st, idx, M);
-            CK(cudaMemsetAsync(T.nflag, 0, sizeof(int), st));
-            run_ted(T, ctx->Xb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->mkeys, no_graph, false, packed,
-                    T.nflag);
+            CK(cudaMemcpyAsync(ctx->mkeys, ctx->bkeys + (size_t)k * m, sizeof(unsigned long long) * m,
+                               cudaMemcpyDeviceToDevice, st));
+            CK(cudaMemcpyAsync(T.flags, ctx->bsflags + (size_t)k * m, sizeof(int) * m, cudaMemcpyDeviceToDevice, st));
+            CK(cudaMemcpyAsync(T.ncand, ctx->bncand + (size_t)k * m, sizeof(int) * m, cudaMemcpyDeviceToDevice, st));
+            CK(cudaMemcpyAsync(T.cand, ctx->bcand + (size_t)k * m * nC, sizeof(uint32_t) * m * nC,
+                               cudaMemcpyDeviceToDevice, st));
             refine_ted(ctx, T, ctx->Xb, M, ctx->d, m, mu, ctx->mkeys, nullptr);
             bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->mkeys, m, idx,
                                                                      ctx->winners + (size_t)k * m);
@@ -1554,7 +1576,7 @@ void bted_destroy(bted_ctx* ctx) {
                         ctx->u32b, ctx->count_dev, ctx->mkeys, ctx->cub_tmp, ctx->out_dev, ctx->sall,
                         ctx->xall, ctx->kall, ctx->shist, ctx->sint, ctx->scand, ctx->ssel, ctx->soff,
                         ctx->bflag, ctx->rcols, ctx->rG, ctx->rA, ctx->rW, ctx->rpart, ctx->rdiag, ctx->rout,
-                        ctx->ridx};
+                        ctx->ridx, ctx->bkeys, ctx->bsflags, ctx->bncand, ctx->bcand};
         for (void* b : bufs) if (b) cudaFree(b);
         if (ctx->own_X && ctx->X) cudaFree(ctx->X);
         if (ctx->hkeys) cudaFreeHost(ctx->hkeys);

@@ -525,16 +525,29 @@ def test_k4_strict_parity_on_long_selections(flags):
     print(f"K4: refined {total_refined} steps, corrected {total_corrected}")
 
 
-def test_k4_in_batches_matches_oracle_strictly():
-    P, M, B, m, seed = 40000, 1500, 3, 200, 17
-    X = uniform_pool(P, 8, 5)
+@pytest.mark.parametrize("flags", [PACKED, IMPLICIT], ids=["packed", "implicit"])
+def test_k4_in_batches_matches_oracle_strictly(flags):
+    """Alg. 2 batch TEDs keep their own K4 state (keys, flags, candidates per
+    batch); the flagged steps are refined after all batches without re-running
+    them, and every batch still meets P2 at the fp64 gap GAP_K4."""
+    X = uniform_pool(5000, 8, 5)
+    X = np.concatenate([X, X[::5]], axis=0)                  # exact duplicates: exact ties to refine
+    P, M, B, m, seed = X.shape[0], 1500, 4, 200, 17
     g = median_gamma(X, 5)
-    with bt.CandidateSet(X, g, num_batches=B, seed=seed, flags=PACKED) as pool:
+    with bt.CandidateSet(X, g, num_batches=B, seed=seed, flags=flags) as pool:
+        L.bted_reset_stats(pool.ctx)
+        launches = bt.bted_kernel_launches()
         sel, bidx = pool.run_batches(M, m, MU)
+        launches = bt.bted_kernel_launches() - launches
+        st = L.bted_get_stats(pool.ctx)
+        sel2, bidx2 = pool.run_batches(M, m, MU)              # deterministic
+    assert np.array_equal(sel, sel2) and np.array_equal(bidx, bidx2)
+    assert st["refined_steps"] > 0                           # the refinement path ran
     batches = oracle_sample_batches(P, M, B, seed)
     for b in range(B):
         pos = _positions(batches[b], bidx[b])
         check_ted(pos, [], dense.ted(X[batches[b]], g, MU, m, forced=pos), f"k4-batch{b}", gap_exact=GAP_K4)
+    print(f"K4 in batches: refined {st['refined_steps']}, corrected {st['corrected_steps']}, launches {launches}")
 
 
 def test_large_131072_sampled_against_closed_form():
