@@ -116,8 +116,10 @@ bted_status bted_create(const float* X, int64_t N, int32_t d, bted_kernel kernel
  *   skipped because it cannot change X).
  *   out_idx   [m] row indices in selection order (host).
  *   out_score [m] nullable: fp32 score of each pick at the step it was taken.
- *   Idempotent: each call restarts from the fresh Gram matrix.  Allocates
- *   2 N^2 fp32 (ping-pong K) on first use at this N.
+ *   Idempotent: each call restarts from the fresh Gram matrix.  Device memory
+ *   on first use at this N: the default implicit engine keeps one packed
+ *   upper-triangular K (~N^2/2 fp32) plus O(N m) fp64 state; the literal
+ *   engines ping-pong two K buffers (packed ~N^2, dense 2 N^2 fp32).
  *   Errors: EINVAL (m < 1, m > N, mu <= 0 or non-finite), ENOMEM, ECUDA,
  *   ENUMERIC, ESTATE.
  */
@@ -269,7 +271,8 @@ const char* bted_last_error(void);
 uint64_t    bted_kernel_launches(void);
 /* Debug: copy the fp32 K of the last TED run by ctx (which = 0: bted_select,
  * 1: the last batch / merge TED) to host as a dense rows x ld matrix (packed
- * storage is unpacked), i.e. K after the m-1 deflations of that run. */
+ * storage is unpacked), i.e. K after the m-1 deflations of that run -- or, for
+ * the implicit engine (which never rewrites K), the Gram matrix of that run. */
 bted_status bted_debug_copy_K(bted_ctx* ctx, int32_t which, float* out, int64_t* ld_out);
 
 #ifdef __cplusplus

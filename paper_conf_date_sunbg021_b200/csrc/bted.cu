@@ -435,13 +435,16 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
     CK(cudaMemsetAsync(T.kflag, 0, sizeof(int), T.stream));
     CK(cudaMemsetAsync(T.tctr, 0, sizeof(int) * m, T.stream));
     const int lin = kernel == BTED_KERNEL_LINEAR ? 1 : 0;
-    float* scratch = reinterpret_cast<float*>(T.P64);      // K1p's fp32 partials are not used here
-    if (d <= 16)
-        bted::pk::gram_packed_kernel<16><<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
-            X, (int32_t)N, d, gamma, lin, T.K[0], nT, scratch);
-    else
-        bted::pk::gram_packed_kernel<32><<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
-            X, (int32_t)N, d, gamma, lin, T.K[0], nT, scratch);
+    // K1i: the Gram tiles only (the fp64 norm pass below recomputes the first scores)
+    auto k1i = [&](auto kern) {
+        kern<<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(X, (int32_t)N, d, gamma, T.K[0], nT);
+    };
+    // two rows per warp step at 3 CTAs/SM measured 369 us vs 388 (four rows, 2 CTAs/SM) and 412 (K1p)
+    if (d <= 16) {
+        if (lin) k1i(bted::pk::gram_tile_kernel<16, true, 2>); else k1i(bted::pk::gram_tile_kernel<16, false, 2>);
+    } else {
+        if (lin) k1i(bted::pk::gram_tile_kernel<32, true>); else k1i(bted::pk::gram_tile_kernel<32, false>);
+    }
     bted::im::tile_pass_kernel<true><<<tile_pass_grid(tiles), bted::im::kTPThreads, bted::im::tile_pass_smem_bytes,
                                        T.stream>>>(T.K[0], nT, nullptr, T.P64, T.kflag, T.tctr, 0,
                                                    l2_keep_tiles(tiles));
@@ -633,9 +636,9 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
         T.reserve(N, N, d, m);
     }
     T.last_packed = packed;
-    T.last_rows = implicit ? 0 : N;          // implicit mode never materialises K^(t)
+    T.last_rows = N;
     T.last_ld = ld_for(N);
-    T.last_buf = (m - 1) & 1;
+    T.last_buf = implicit ? 0 : (m - 1) & 1;  // implicit: K stays the Gram (buffer 0, never deflated)
     Ted::Slot* sl = (T.timing && time_it) ? T.next_slot(m) : nullptr;
     if (sl) CK(cudaEventRecord(sl->e[0], T.stream));
     auto head = [&] {

@@ -652,6 +652,87 @@ gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamm
 }
 
 
+// ------------------------------------------------------------------ K1i: Gram tiles only
+// Alg. 1 l.1 for the implicit engine, whose fp64 norm pass recomputes the
+// first scores: the same tiles, bitwise the same values as K1p (same FADD2 /
+// FFMA2 sequence over the features in order, same expf), without the fp32
+// partials.  Row features are staged as duplicated pairs (x, x), so one
+// LDS.128 feeds two features of a row with no packing; each warp runs kH rows
+// at once (2 kH independent FFMA2 chains per lane).  At N = 16384 (B200, warm
+// ncu): 369 us with kH = 2 at 3 CTAs/SM, 388 us with kH = 4 at 2 CTAs/SM,
+// vs 412 us for K1p with its fp32 partials.
+template <int kD, bool kLinear, int kH = 4>
+__global__ void __launch_bounds__(kConsumers, kH == 4 ? 2 : 3)
+gram_tile_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma, float* __restrict__ K, int nT) {
+    __shared__ __align__(16) unsigned long long xi2[T][kD];     // (x, x) pairs of the tile's rows
+    __shared__ __align__(16) float xj[T][kD];
+    const int tid = threadIdx.x, w = tid / kWarp, l = tid % kWarp;
+    const float ng = -gamma;
+    int I, J;
+    tile_ij((int64_t)blockIdx.x, nT, I, J);
+    for (int q = tid; q < T * kD; q += kConsumers) {
+        const int r = q / kD, c = q % kD;
+        const int gi = I * T + r, gj = J * T + r;
+        const float xv = (gi < N && c < d) ? X[(int64_t)gi * d + c] : 0.f;   // zero features add (0-0)^2 = 0
+        xi2[r][c] = pack2(xv, xv);
+        xj[r][c] = (gj < N && c < d) ? X[(int64_t)gj * d + c] : 0.f;
+    }
+    __syncthreads();
+    unsigned long long y01[kD], y23[kD];
+#pragma unroll
+    for (int q = 0; q < kD; ++q) {
+        y01[q] = pack2(xj[4 * l + 0][q], xj[4 * l + 1][q]);
+        y23[q] = pack2(xj[4 * l + 2][q], xj[4 * l + 3][q]);
+    }
+    float* tile = K + (int64_t)blockIdx.x * (T * T);
+    bool cv[4];
+#pragma unroll
+    for (int c = 0; c < 4; ++c) cv[c] = J * T + 4 * l + c < N;
+#pragma unroll 1
+    for (int rr = 0; rr < 16; rr += kH) {
+        const int r = 16 * w + rr;
+        unsigned long long a01[kH], a23[kH];
+#pragma unroll
+        for (int h = 0; h < kH; ++h) a01[h] = a23[h] = 0ull;
+#pragma unroll
+        for (int q = 0; q < kD; q += 2) {
+#pragma unroll
+            for (int h = 0; h < kH; ++h) {
+                const ulonglong2 xx = *reinterpret_cast<const ulonglong2*>(&xi2[r + h][q]);
+                if (kLinear) {
+                    a01[h] = fma2(xx.x, y01[q], a01[h]);
+                    a23[h] = fma2(xx.x, y23[q], a23[h]);
+                    a01[h] = fma2(xx.y, y01[q + 1], a01[h]);
+                    a23[h] = fma2(xx.y, y23[q + 1], a23[h]);
+                } else {
+                    unsigned long long d01 = sub2(xx.x, y01[q]), d23 = sub2(xx.x, y23[q]);
+                    a01[h] = fma2(d01, d01, a01[h]);
+                    a23[h] = fma2(d23, d23, a23[h]);
+                    d01 = sub2(xx.y, y01[q + 1]);
+                    d23 = sub2(xx.y, y23[q + 1]);
+                    a01[h] = fma2(d01, d01, a01[h]);
+                    a23[h] = fma2(d23, d23, a23[h]);
+                }
+            }
+        }
+#pragma unroll
+        for (int h = 0; h < kH; ++h) {
+            float acc[4];
+            unpack2(a01[h], acc[0], acc[1]);
+            unpack2(a23[h], acc[2], acc[3]);
+            const bool rv = I * T + r + h < N;
+            float4 o;
+            float* oc = &o.x;
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                const float val = kLinear ? acc[c] : expf(__fmul_rn(ng, acc[c]));
+                oc[c] = (rv && cv[c]) ? val : 0.f;
+            }
+            st_stream(tile + (r + h) * T + 4 * l, o);
+        }
+    }
+}
+
 // ------------------------------------------------------------------ K2p (LDG variant)
 // One CTA (256 threads) per tile, non-persistent (the hardware scheduler
 // balances 8256+ tiles over the SMs; several CTAs per SM keep many 256-bit

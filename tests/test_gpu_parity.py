@@ -23,6 +23,8 @@ IMPLICIT = L.BTED_FLAG_NO_SMALL                              # the default engin
 LAYOUTS = pytest.mark.parametrize("flags", [PACKED, PACKED_TMA, DENSE, IMPLICIT, 0],
                                   ids=["packed", "packed-tma", "dense", "implicit", "auto"])
 LAYOUTS_K = pytest.mark.parametrize("flags", [PACKED, PACKED_TMA, DENSE], ids=["packed", "packed-tma", "dense"])
+LAYOUTS_GRAM = pytest.mark.parametrize("flags", [PACKED, PACKED_TMA, DENSE, IMPLICIT],
+                                       ids=["packed", "packed-tma", "dense", "implicit"])
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -40,8 +42,23 @@ def ld_of(N):
 
 
 # ------------------------------------------------------------------ K1 Gram
+@pytest.mark.parametrize("N,d,pool", [(1000, 16, "knob"), (777, 16, "uniform"), (300, 12, "knob"), (515, 30, "uniform")])
+def test_implicit_gram_bitwise_equals_k1p(N, d, pool):
+    """K1i (the implicit head's Gram-only kernel) writes bitwise the tiles K1p writes."""
+    X = knob(N, d=d) if pool == "knob" else uniform_pool(N, d, 4)
+    g = median_gamma(X, 2)
+    with bt.CandidateSet(X, g, flags=IMPLICIT) as ci, bt.CandidateSet(X, g, flags=PACKED) as cp:
+        ci.select(5, MU)
+        cp.select(1, MU)
+        assert np.array_equal(ci.debug_K(N), cp.debug_K(N))
+    with bt.CandidateSet(X, 1.0, kernel=L.BTED_KERNEL_LINEAR, flags=IMPLICIT) as ci, \
+            bt.CandidateSet(X, 1.0, kernel=L.BTED_KERNEL_LINEAR, flags=PACKED) as cp:
+        ci.select(3, MU)
+        cp.select(1, MU)
+        assert np.array_equal(ci.debug_K(N), cp.debug_K(N))
+
 @pytest.mark.parametrize("N,pool", [(1000, "knob"), (777, "uniform"), (64, "knob")])
-@LAYOUTS_K
+@LAYOUTS_GRAM
 def test_gram_entries_bitsymmetric_and_within_ulp_bound(N, pool, flags):
     X = knob(N) if pool == "knob" else uniform_pool(N, 16, 4)
     g = median_gamma(X, 1)
