@@ -1096,7 +1096,8 @@ void launch_small_c(const float* X, int ninst, int32_t N, int32_t d, float gamma
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)(ninst * C));
     cfg.blockDim = dim3(bted::sm::kThreads);
-    cfg.dynamicSmemBytes = bted::sm::smem_bytes(N, C);
+    const bool stage_x = bted::sm::smem_core(N, C) + bted::sm::smem_x(N, d) <= bted::sm::kSmemBudget;
+    cfg.dynamicSmemBytes = bted::sm::smem_core(N, C) + (stage_x ? bted::sm::smem_x(N, d) : 0);
     cfg.stream = st;
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeClusterDimension;
@@ -1106,14 +1107,21 @@ void launch_small_c(const float* X, int ninst, int32_t N, int32_t d, float gamma
     cfg.attrs = at;
     cfg.numAttrs = 1;
     CK(cudaLaunchKernelEx(&cfg, bted::sm::ted_cluster_kernel<C>, X, N, d, gamma,
-                          (int32_t)(kernel == BTED_KERNEL_LINEAR ? 1 : 0), m, mu, keys, err));
+                          (int32_t)(kernel == BTED_KERNEL_LINEAR ? 1 : 0), m, mu, keys, err, (int32_t)stage_x));
     LAUNCHED(1);
 }
 
 // ninst independent TEDs on X[inst][N][d] -> keys[inst][m]; err = a Ted's flag
 void launch_small(const float* X, int ninst, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
                   unsigned long long* keys, int* err, cudaStream_t st) {
-    switch (small_cluster_for(N)) {
+    // the smallest cluster whose CTAs also hold the staged features, if the
+    // ninst clusters still fit on the SMs at once; else the smallest that fits
+    int C = small_cluster_for(N);
+    for (int c2 = C; c2 > 0 && c2 <= 16; c2 *= 2) {
+        if ((int64_t)ninst * c2 > num_sms()) break;
+        if (bted::sm::smem_core((int)N, c2) + bted::sm::smem_x((int)N, d) <= bted::sm::kSmemBudget) { C = c2; break; }
+    }
+    switch (C) {
         case 1: launch_small_c<1>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st); break;
         case 2: launch_small_c<2>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st); break;
         case 4: launch_small_c<4>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st); break;

@@ -30,16 +30,22 @@ constexpr size_t kSmemBudget = 220 * 1024;
 
 __host__ __device__ __forceinline__ int ldk_for(int N) { return (N + 3) / 4 * 4; }
 __host__ __device__ __forceinline__ int rows_per(int N, int C) { return (N + C - 1) / C; }
+constexpr int kR = 4;                  // rows per warp iteration (independent reduction chains)
 // dynamic smem of one CTA: band + pivot row + key slots + warp keys + sel
-__host__ __device__ __forceinline__ size_t smem_bytes(int N, int C) {
+__host__ __device__ __forceinline__ size_t smem_core(int N, int C) {
     const size_t R = (size_t)rows_per(N, C), L = (size_t)ldk_for(N);
-    return (R * L + L) * sizeof(float) + (2 * 16 + kWarps) * sizeof(unsigned long long) + ((R + 15) / 16) * 16;
+    return (R * L + L) * sizeof(float) + (2 * 16 + 2 * kWarps) * sizeof(unsigned long long) + ((R + 15) / 16) * 16;
 }
+// + the features of all N points staged for the Gram phase (odd row stride d|1:
+// lanes reading different points hit different banks)
+__host__ __device__ __forceinline__ size_t smem_x(int N, int d) { return (size_t)N * (size_t)(d | 1) * sizeof(float); }
+__host__ __device__ __forceinline__ size_t smem_bytes(int N, int C) { return smem_core(N, C); }
 
 template <int C>
 __global__ void __launch_bounds__(kThreads, 1)
 ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float gamma, int32_t linear,
-                   int32_t m, float mu, unsigned long long* __restrict__ keys_all, int* __restrict__ err) {
+                   int32_t m, float mu, unsigned long long* __restrict__ keys_all, int* __restrict__ err,
+                   int32_t stage_x) {
     cg::cluster_group cl = cg::this_cluster();
     const int rank = C == 1 ? 0 : (int)cl.block_rank();
     // a cluster of one CTA needs only the CTA barrier (cluster barriers also
@@ -57,8 +63,8 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
     float* Kb = reinterpret_cast<float*>(smem);                 // [R][L]
     float* piv = Kb + (size_t)R * L;                            // [L]
     unsigned long long* kslot = reinterpret_cast<unsigned long long*>(piv + L);   // [2][16]
-    unsigned long long* wred = kslot + 32;                      // [kWarps]
-    uint8_t* sel = reinterpret_cast<uint8_t*>(wred + kWarps);   // [R]
+    unsigned long long* wred = kslot + 32;                      // [2][kWarps] (step parity)
+    uint8_t* sel = reinterpret_cast<uint8_t*>(wred + 2 * kWarps);   // [R]
 
     const int tid = threadIdx.x, w = tid / 32, l = tid % 32;
     const int r0 = rank * R;
@@ -66,53 +72,79 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
     const float ng = -gamma;
 
     // ---------------- l.1: this CTA's rows of K_VV, plus the first l.3
+    // Features from smem when they fit next to the band (stage_x), else from
+    // global; the same operands in the same order either way (bitwise the same K).
+    const float* Xf = X;
+    int xs = d;
+    if (stage_x) {
+        float* Xs = reinterpret_cast<float*>(smem + smem_core(N, C));
+        xs = d | 1;
+        for (int q = tid; q < N * d; q += kThreads) Xs[(q / d) * xs + q % d] = X[q];
+        Xf = Xs;
+    }
     for (int q = tid; q < R; q += kThreads) sel[q] = 0;
+    __syncthreads();
     unsigned long long best_local = 0ull;
-    for (int lr = w; lr < nr; lr += kWarps) {
-        const int i = r0 + lr;
-        float* row = Kb + (size_t)lr * L;
-        float acc_norm = 0.f;
+    for (int base = w; base < nr; base += kWarps * kR) {
+        float acc_norm[kR];
+#pragma unroll
+        for (int h = 0; h < kR; ++h) acc_norm[h] = 0.f;
         for (int j = l; j < L; j += 32) {
-            float v = 0.f;
-            if (j < N) {
-                float a = 0.f;
-                for (int k = 0; k < d; ++k) {
-                    const float xi = X[(int64_t)i * d + k], xj = X[(int64_t)j * d + k];
-                    if (linear) a = __fmaf_rn(xi, xj, a);
-                    else { const float df = __fsub_rn(xi, xj); a = __fmaf_rn(df, df, a); }
+#pragma unroll
+            for (int h = 0; h < kR; ++h) {
+                const int lr = base + h * kWarps;
+                if (lr >= nr) continue;
+                const int i = r0 + lr;
+                float v = 0.f;
+                if (j < N) {
+                    float a = 0.f;
+                    for (int k = 0; k < d; ++k) {
+                        const float xi = Xf[i * xs + k], xj = Xf[j * xs + k];
+                        if (linear) a = __fmaf_rn(xi, xj, a);
+                        else { const float df = __fsub_rn(xi, xj); a = __fmaf_rn(df, df, a); }
+                    }
+                    v = linear ? a : expf(__fmul_rn(ng, a));
                 }
-                v = linear ? a : expf(__fmul_rn(ng, a));
+                Kb[(size_t)lr * L + j] = v;
+                acc_norm[h] = __fmaf_rn(v, v, acc_norm[h]);
             }
-            row[j] = v;
-            acc_norm = __fmaf_rn(v, v, acc_norm);
         }
-        const float g = warp_sum(acc_norm);
+        float g[kR];
+#pragma unroll
+        for (int h = 0; h < kR; ++h) g[h] = warp_sum(acc_norm[h]);
         if (l == 0) {
-            const unsigned long long k = score_key(g, row[i], mu, (uint32_t)i, false, err);
-            best_local = k > best_local ? k : best_local;
+#pragma unroll
+            for (int h = 0; h < kR; ++h) {
+                const int lr = base + h * kWarps;
+                if (lr >= nr) continue;
+                const int i = r0 + lr;
+                const unsigned long long k = score_key(g[h], Kb[(size_t)lr * L + i], mu, (uint32_t)i, false, err);
+                best_local = k > best_local ? k : best_local;
+            }
         }
     }
     // CTA max -> every CTA's slot[0][rank] -> cluster max
+    // (one CTA: every warp reduces the kWarps slots itself after ONE barrier;
+    // the slots alternate with the step parity, so the next step's writes
+    // cannot race this step's reads)
     auto exchange = [&](unsigned long long key, int parity) -> unsigned long long {
         key = warp_max_u64(key);
-        if (l == 0) wred[w] = key;
+        unsigned long long* wr = wred + parity * kWarps;
+        if (l == 0) wr[w] = key;
         __syncthreads();
-        if (tid == 0) {
-            unsigned long long v = 0ull;
-            for (int q = 0; q < kWarps; ++q) v = wred[q] > v ? wred[q] : v;
-            if constexpr (C == 1) {
-                kslot[parity * 16] = v;
-            } else {
-                for (int r = 0; r < C; ++r) {
-                    unsigned long long* dst = cl.map_shared_rank(kslot, r);
-                    dst[parity * 16 + rank] = v;
-                }
+        unsigned long long v = warp_max_u64(l < kWarps ? wr[l] : 0ull);
+        if constexpr (C == 1) {
+            return v;
+        } else {
+            if (w == 0 && l < C) {
+                unsigned long long* dst = cl.map_shared_rank(kslot, l);
+                dst[parity * 16 + rank] = v;
             }
+            csync();
+            unsigned long long b = 0ull;
+            for (int r = 0; r < C; ++r) b = kslot[parity * 16 + r] > b ? kslot[parity * 16 + r] : b;
+            return b;
         }
-        csync();
-        unsigned long long b = 0ull;
-        for (int r = 0; r < C; ++r) b = kslot[parity * 16 + r] > b ? kslot[parity * 16 + r] : b;
-        return b;
     };
     unsigned long long best = exchange(best_local, 0);
 
@@ -129,29 +161,46 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
         csync();                                     // every CTA holds the pivot before rows change
         const float inv_c = __frcp_rn(__fadd_rn(piv[s], mu));
         best_local = 0ull;
-        for (int lr = w; lr < nr; lr += kWarps) {
-            const int i = r0 + lr;
-            float* row = Kb + (size_t)lr * L;
-            const float a = piv[i];                  // K[i][s] = K[s][i]
-            float acc_norm = 0.f;
-            for (int j4 = l; j4 < L / 4; j4 += 32) {
-                float4 kv = reinterpret_cast<float4*>(row)[j4];
-                const float4 pv = reinterpret_cast<const float4*>(piv)[j4];
-                kv.x = deflate1(kv.x, a, pv.x, inv_c);
-                kv.y = deflate1(kv.y, a, pv.y, inv_c);
-                kv.z = deflate1(kv.z, a, pv.z, inv_c);
-                kv.w = deflate1(kv.w, a, pv.w, inv_c);
-                reinterpret_cast<float4*>(row)[j4] = kv;
-                acc_norm = __fmaf_rn(kv.x, kv.x, acc_norm);
-                acc_norm = __fmaf_rn(kv.y, kv.y, acc_norm);
-                acc_norm = __fmaf_rn(kv.z, kv.z, acc_norm);
-                acc_norm = __fmaf_rn(kv.w, kv.w, acc_norm);
+        for (int base = w; base < nr; base += kWarps * kR) {
+            float acc_norm[kR], a[kR];
+#pragma unroll
+            for (int h = 0; h < kR; ++h) {
+                const int lr = base + h * kWarps;
+                acc_norm[h] = 0.f;
+                a[h] = lr < nr ? piv[r0 + lr] : 0.f;   // K[i][s] = K[s][i]
             }
-            const float g = warp_sum(acc_norm);
+            for (int j4 = l; j4 < L / 4; j4 += 32) {
+                const float4 pv = reinterpret_cast<const float4*>(piv)[j4];
+#pragma unroll
+                for (int h = 0; h < kR; ++h) {
+                    const int lr = base + h * kWarps;
+                    if (lr >= nr) continue;
+                    float4* row = reinterpret_cast<float4*>(Kb + (size_t)lr * L);
+                    float4 kv = row[j4];
+                    kv.x = deflate1(kv.x, a[h], pv.x, inv_c);
+                    kv.y = deflate1(kv.y, a[h], pv.y, inv_c);
+                    kv.z = deflate1(kv.z, a[h], pv.z, inv_c);
+                    kv.w = deflate1(kv.w, a[h], pv.w, inv_c);
+                    row[j4] = kv;
+                    acc_norm[h] = __fmaf_rn(kv.x, kv.x, acc_norm[h]);
+                    acc_norm[h] = __fmaf_rn(kv.y, kv.y, acc_norm[h]);
+                    acc_norm[h] = __fmaf_rn(kv.z, kv.z, acc_norm[h]);
+                    acc_norm[h] = __fmaf_rn(kv.w, kv.w, acc_norm[h]);
+                }
+            }
+            float g[kR];
+#pragma unroll
+            for (int h = 0; h < kR; ++h) g[h] = warp_sum(acc_norm[h]);
             if (l == 0) {
-                const bool masked = sel[lr] != 0 || i == s;
-                const unsigned long long k = score_key(g, row[i], mu, (uint32_t)i, masked, err);
-                best_local = k > best_local ? k : best_local;
+#pragma unroll
+                for (int h = 0; h < kR; ++h) {
+                    const int lr = base + h * kWarps;
+                    if (lr >= nr) continue;
+                    const int i = r0 + lr;
+                    const bool masked = sel[lr] != 0 || i == s;
+                    const unsigned long long k = score_key(g[h], Kb[(size_t)lr * L + i], mu, (uint32_t)i, masked, err);
+                    best_local = k > best_local ? k : best_local;
+                }
             }
         }
         best = exchange(best_local, t & 1);
