@@ -18,7 +18,7 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:"til
     -o $OUT/prof_imp python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_imp.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"deflate_packed|finalize_packed" -s 16 -c 2 \
     -o $OUT/prof_k2p python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e --layout packed > $OUT/ncu_k2p.log 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:gram_packed -s 2 -c 1 \
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:"gram_tile|gram_packed" -s 2 -c 1 \
     -o $OUT/prof_k1p python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_k1p.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:deflate_rescore -s 8 -c 1 \
     -o $OUT/prof_k2 python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e --layout dense > $OUT/ncu_k2.log 2>&1
