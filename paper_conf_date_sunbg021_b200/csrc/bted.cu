@@ -718,6 +718,8 @@ struct bted_ctx {
     uint64_t* scand = nullptr; size_t scandcap = 0;
     uint32_t* ssel = nullptr; size_t sselcap = 0;
     int* soff = nullptr; size_t soffcap = 0;
+    uint64_t* sks = nullptr; size_t skscap = 0;            // k* (M-th smallest key) per batch
+    unsigned* scnt = nullptr; size_t scntcap = 0;          // [nb][G] chunk counts -> offsets
     int* bflag = nullptr; size_t bflagcap = 0;             // K4: near ties per batch TED
     unsigned long long* bkeys = nullptr; size_t bkeyscap = 0; // K4: [nb][m] keys of every batch TED
     int* bsflags = nullptr; size_t bsflagscap = 0;           //     [nb][m] per-step near-tie flags
@@ -943,8 +945,6 @@ void sample_batches_dev(bted_ctx* ctx, cudaStream_t st, int64_t P, int64_t M, in
     grow(ctx->shist, ctx->shistcap, (size_t)nb * bted::kSelBins);
     grow(ctx->sint, ctx->sintcap, (size_t)4 * nb + 1);
     grow(ctx->scand, ctx->scandcap, (size_t)nb * bted::kCandCap);
-    grow(ctx->ssel, ctx->sselcap, (size_t)nb * M);
-    grow(ctx->soff, ctx->soffcap, (size_t)nb + 1);
     int* bstar = ctx->sint;
     int* below = ctx->sint + nb;
     unsigned* nsel = reinterpret_cast<unsigned*>(ctx->sint + 2 * nb);
@@ -954,23 +954,24 @@ void sample_batches_dev(bted_ctx* ctx, cudaStream_t st, int64_t P, int64_t M, in
     const unsigned gx = (unsigned)std::max<int64_t>(1, std::min<int64_t>((P + 1023) / 1024, 64));
     bted::sel_hist_kernel<<<dim3(gx, nb), 256, 0, st>>>((uint64_t)P, seed, b_begin, b_step, ctx->shist);
     bted::sel_thresh_kernel<<<nb, 1024, 0, st>>>(ctx->shist, M, bstar, below);
-    bted::sel_collect_kernel<<<dim3(gx, nb), 256, 0, st>>>((uint64_t)P, seed, b_begin, b_step, M, bstar, ctx->ssel,
+    bted::sel_collect_kernel<<<dim3(gx, nb), 256, 0, st>>>((uint64_t)P, seed, b_begin, b_step, M, bstar, nullptr,
                                                             nsel, ctx->scand, ncand);
     if (!ctx->bted_engine.err) {
         grow(ctx->bted_engine.err, ctx->bted_engine.errcap, 1);
         CK(cudaMemsetAsync(ctx->bted_engine.err, 0, sizeof(int), st));
     }
-    bted::sel_finish_kernel<<<nb, 1024, 0, st>>>(M, below, ctx->scand, ncand, ctx->ssel, ctx->bted_engine.err);
-    bted::seg_offsets_kernel<<<(nb + 256) / 256, 256, 0, st>>>(nb, M, ctx->soff);
-    LAUNCHED(5);
-    size_t need = 0;
-    const int nbits = bits_for((uint64_t)P);
-    CK(cub::DeviceSegmentedRadixSort::SortKeys(nullptr, need, ctx->ssel, out, (int)(nb * M), nb, ctx->soff,
-                                               ctx->soff + 1, 0, nbits, st));
-    cub_reserve(ctx, need);
-    size_t cap = ctx->cub_cap;
-    CK(cub::DeviceSegmentedRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->ssel, out, (int)(nb * M), nb, ctx->soff,
-                                               ctx->soff + 1, 0, nbits, st));
+    // k* per batch, then the ordered compaction (V_b ascending, no sort)
+    const int G = (int)((P + bted::kCmpChunk - 1) / bted::kCmpChunk);
+    grow(ctx->sks, ctx->skscap, (size_t)nb);
+    grow(ctx->scnt, ctx->scntcap, (size_t)nb * G);
+    bted::sel_finish_kernel<<<nb, 1024, 0, st>>>(M, below, ctx->scand, ncand, nullptr, ctx->bted_engine.err,
+                                                 ctx->sks);
+    bted::sel_count_kernel<<<dim3(G, nb), bted::kCmpThreads, 0, st>>>((uint64_t)P, seed, b_begin, b_step, ctx->sks,
+                                                                     ctx->scnt);
+    bted::sel_scan_kernel<<<nb, 1024, 0, st>>>(ctx->scnt, G);
+    bted::sel_write_kernel<<<dim3(G, nb), bted::kCmpThreads, 0, st>>>((uint64_t)P, seed, b_begin, b_step, ctx->sks,
+                                                                     ctx->scnt, M, out);
+    LAUNCHED(7);
 }
 
 void gather(bted_ctx* ctx, cudaStream_t st, const uint32_t* idx, int64_t M, float* dst = nullptr) {
@@ -1587,7 +1588,7 @@ void bted_destroy(bted_ctx* ctx) {
                         ctx->u32b, ctx->count_dev, ctx->mkeys, ctx->cub_tmp, ctx->out_dev, ctx->sall,
                         ctx->xall, ctx->kall, ctx->shist, ctx->sint, ctx->scand, ctx->ssel, ctx->soff,
                         ctx->bflag, ctx->rcols, ctx->rG, ctx->rA, ctx->rW, ctx->rpart, ctx->rdiag, ctx->rout,
-                        ctx->ridx, ctx->bkeys, ctx->bsflags, ctx->bncand, ctx->bcand};
+                        ctx->ridx, ctx->bkeys, ctx->bsflags, ctx->bncand, ctx->bcand, ctx->sks, ctx->scnt};
         for (void* b : bufs) if (b) cudaFree(b);
         if (ctx->own_X && ctx->X) cudaFree(ctx->X);
         if (ctx->hkeys) cudaFreeHost(ctx->hkeys);

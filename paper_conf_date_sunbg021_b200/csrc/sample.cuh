@@ -70,8 +70,9 @@ __global__ void finite_check_kernel(const float* __restrict__ X, int64_t n, int*
 //   sel_hist     histogram of the top 12 bits of hash32 per batch
 //   sel_thresh   the bin b* holding the M-th smallest key, count `below` before it
 //   sel_collect  indices in bins < b* (all selected), keys in bin b* (candidates)
-//   sel_finish   sort the candidates (bitonic, smem), keep the first M - below
-// then one segmented sort puts each V_b in ascending index order.
+//   sel_finish   sort the candidates (bitonic, smem): the M-th smallest key k*
+//   sel_count / sel_scan / sel_write   ordered compaction of {i : key_b(i) <= k*}:
+//                each V_b comes out in ascending index order, no sort.
 constexpr int kSelBins = 4096;
 constexpr int kCandCap = 4096;
 
@@ -150,17 +151,21 @@ __global__ void sel_collect_kernel(uint64_t P, uint64_t seed, int32_t b_begin, i
         const uint32_t h = in ? hash32_of(hb, i) : 0xFFFFFFFFu;
         const unsigned bin = h >> 20;
         const bool is_sel = in && bin < bs, is_cand = in && bin == bs;
-        const unsigned ps = warp_agg_inc(nsel + k, is_sel);
-        if (is_sel) sel[(int64_t)k * M + ps] = (uint32_t)i;
+        if (sel) {
+            const unsigned ps = warp_agg_inc(nsel + k, is_sel);
+            if (is_sel) sel[(int64_t)k * M + ps] = (uint32_t)i;
+        }
         const unsigned pc = warp_agg_inc(ncand + k, is_cand);
         if (is_cand && pc < (unsigned)kCandCap) cand[(int64_t)k * kCandCap + pc] = ((uint64_t)h << 32) | i;
     }
 }
 
 // one CTA (1024 threads) per batch: bitonic sort of the candidates in smem
+// (kstar non-null: only record the M-th smallest key per batch for the ordered compaction)
 __global__ void __launch_bounds__(1024)
 sel_finish_kernel(int64_t M, const int* __restrict__ below, const uint64_t* __restrict__ cand,
-                  const unsigned* __restrict__ ncand, uint32_t* __restrict__ sel, int* __restrict__ err) {
+                  const unsigned* __restrict__ ncand, uint32_t* __restrict__ sel, int* __restrict__ err,
+                  uint64_t* __restrict__ kstar = nullptr) {
     __shared__ uint64_t s[kCandCap];
     const int k = blockIdx.x, tid = threadIdx.x;
     const unsigned n = ncand[k];
@@ -183,7 +188,92 @@ sel_finish_kernel(int64_t M, const int* __restrict__ below, const uint64_t* __re
         }
     const int b0 = below[k];
     const int need = (int)M - b0;
+    if (kstar) {
+        if (tid == 0) kstar[k] = s[need - 1];             // the M-th smallest key of the batch
+        return;
+    }
     for (int q = tid; q < need; q += 1024) sel[(int64_t)k * M + b0 + q] = (uint32_t)(s[q] & 0xFFFFFFFFull);
+}
+
+// ---------------------------------------------------------------------------
+// Ordered compaction: V_b = {i : key_b(i) <= kstar[b]} written in ascending i
+// (no sort).  A CTA owns the index chunk [c*kCmpChunk, (c+1)*kCmpChunk).
+constexpr int kCmpThreads = 256;
+constexpr int kCmpChunk = kCmpThreads * 16;
+
+__device__ __forceinline__ bool sel_pred(uint64_t hb, uint64_t i, uint64_t P, uint64_t kstar) {
+    return i < P && ((((uint64_t)hash32_of(hb, i)) << 32) | i) <= kstar;
+}
+
+__global__ void __launch_bounds__(kCmpThreads)
+sel_count_kernel(uint64_t P, uint64_t seed, int32_t b_begin, int32_t b_step, const uint64_t* __restrict__ kstar,
+                 unsigned* __restrict__ cnt) {
+    __shared__ unsigned red[kCmpThreads / 32];
+    const int k = blockIdx.y, G = gridDim.x;
+    const uint64_t hb = batch_hash_seed(seed, b_begin + k * b_step), ks = kstar[k];
+    const uint64_t base = (uint64_t)blockIdx.x * kCmpChunk;
+    unsigned c = 0;
+#pragma unroll 4
+    for (int q = 0; q < kCmpChunk / kCmpThreads; ++q) c += sel_pred(hb, base + q * kCmpThreads + threadIdx.x, P, ks);
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) c += __shfl_xor_sync(0xffffffffu, c, off);
+    if (threadIdx.x % 32 == 0) red[threadIdx.x / 32] = c;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned t = 0;
+        for (int w = 0; w < kCmpThreads / 32; ++w) t += red[w];
+        cnt[(int64_t)k * G + blockIdx.x] = t;
+    }
+}
+
+// per batch (one CTA of 1024 threads): exclusive scan of the G chunk counts, in place
+__global__ void __launch_bounds__(1024) sel_scan_kernel(unsigned* __restrict__ cnt, int G) {
+    __shared__ unsigned part[1024];
+    unsigned* c = cnt + (int64_t)blockIdx.x * G;
+    unsigned carry = 0;
+    for (int b0 = 0; b0 < G; b0 += 1024) {
+        const int q = b0 + threadIdx.x;
+        const unsigned v = q < G ? c[q] : 0u;
+        part[threadIdx.x] = v;
+        __syncthreads();
+        for (int off = 1; off < 1024; off <<= 1) {
+            const unsigned a = threadIdx.x >= off ? part[threadIdx.x - off] : 0u;
+            __syncthreads();
+            part[threadIdx.x] += a;
+            __syncthreads();
+        }
+        if (q < G) c[q] = carry + part[threadIdx.x] - v;
+        const unsigned tot = part[1023];
+        __syncthreads();
+        carry += tot;
+    }
+}
+
+__global__ void __launch_bounds__(kCmpThreads)
+sel_write_kernel(uint64_t P, uint64_t seed, int32_t b_begin, int32_t b_step, const uint64_t* __restrict__ kstar,
+                 const unsigned* __restrict__ off, int64_t M, uint32_t* __restrict__ out) {
+    __shared__ unsigned wcount[kCmpThreads / 32];
+    const int k = blockIdx.y, G = gridDim.x, w = threadIdx.x / 32, l = threadIdx.x % 32;
+    const uint64_t hb = batch_hash_seed(seed, b_begin + k * b_step), ks = kstar[k];
+    const uint64_t base = (uint64_t)blockIdx.x * kCmpChunk;
+    unsigned pos = off[(int64_t)k * G + blockIdx.x];
+    uint32_t* o = out + (int64_t)k * M;
+    for (int q = 0; q < kCmpChunk / kCmpThreads; ++q) {
+        const uint64_t i = base + q * kCmpThreads + threadIdx.x;
+        const bool p = sel_pred(hb, i, P, ks);
+        const unsigned m = __ballot_sync(0xffffffffu, p);
+        if (l == 0) wcount[w] = __popc(m);
+        __syncthreads();
+        unsigned before = 0, tot = 0;
+#pragma unroll
+        for (int ww = 0; ww < kCmpThreads / 32; ++ww) {
+            before += ww < w ? wcount[ww] : 0u;
+            tot += wcount[ww];
+        }
+        if (p) o[pos + before + __popc(m & ((1u << l) - 1u))] = (uint32_t)i;
+        pos += tot;
+        __syncthreads();
+    }
 }
 
 __global__ void seg_offsets_kernel(int nb, int64_t M, int* __restrict__ off) {
