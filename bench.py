@@ -52,6 +52,12 @@ def parse():
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
                     help="weak: every GPU runs the config's B batches; strong: the config's B batches are split")
+    ap.add_argument("--shard-engine", default="implicit", choices=["implicit", "dense"],
+                    help="oversized config on N > 1 GPUs (or with --sharded): the tile-sharded implicit engine "
+                         "(one q all-reduce per step, ~2 N^2 / P B per GPU) or the dense row bands "
+                         "(key all-reduce + pivot all-gather per step, 8 N^2 / P B per GPU)")
+    ap.add_argument("--sharded", action="store_true",
+                    help="run the oversized config through the multi-GPU sharded driver even at one GPU")
     ap.add_argument("--norm-mode", default="symmetric", choices=["symmetric", "literal"],
                     help="oversized row-sharded mode: scores from the band's row norms (default) or the "
                          "north_star's literal all-reduce(SUM) of partial column norms")
@@ -199,8 +205,17 @@ def bench_ours(args):
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     comm = None
-    if world > 1:
+    if world > 1 or args.sharded:
         import torch.distributed as dist
+        if world == 1:                                   # --sharded on one GPU: a one-rank NCCL group
+            import socket
+            sk = socket.socket()
+            sk.bind(("127.0.0.1", 0))
+            os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+            os.environ.setdefault("MASTER_PORT", str(sk.getsockname()[1]))
+            sk.close()
+            os.environ.setdefault("RANK", "0")
+            os.environ.setdefault("WORLD_SIZE", "1")
         dist.init_process_group("nccl", device_id=dev)
         comm = TorchComm()
 
@@ -209,7 +224,7 @@ def bench_ours(args):
     X, gamma, cfg = config_pool(args.config)
     mu = float(np.float32(cfg["mu"]))
     M, m, d, P = cfg["M"], cfg["m"], cfg["d"], X.shape[0]
-    if cfg["B"] == 1 and args.config == "oversized" and world > 1:
+    if cfg["B"] == 1 and args.config == "oversized" and (world > 1 or args.sharded):
         return bench_sharded(args, X, gamma, cfg, comm, dev, world, rank)
     B = cfg["B"] * world if args.scaling == "weak" else cfg["B"]
     stream = torch.cuda.Stream(dev)
@@ -461,10 +476,19 @@ def bench_sharded(args, X, gamma, cfg, comm, dev, world, rank):
     V = bt.bted_sample_batches(X.shape[0], M, 1, cfg["seed"])[0]
     Xb = np.ascontiguousarray(X[V])
     stream = torch.cuda.Stream(dev)
-    r0, r1, _ = band(M, world, rank)
-    shard = LibShard(Xb, M, cfg["d"], gamma, r0, r1, dev, stream)
-    st = ShardedTed(shard, M, comm, dev, stream, graph=True, norm_mode=args.norm_mode)
-    for _ in range(args.warmup):
+    implicit = args.shard_engine == "implicit"
+    if implicit:
+        from paper_conf_date_sunbg021_b200.dist import LibIShard, ShardedImplicitTed
+        shard = LibIShard(Xb, M, cfg["d"], gamma, rank, world, dev, stream)
+        st = ShardedImplicitTed(shard, M, comm, dev, stream, graph=True)
+    else:
+        r0, r1, _ = band(M, world, rank)
+        shard = LibShard(Xb, M, cfg["d"], gamma, r0, r1, dev, stream)
+        st = ShardedTed(shard, M, comm, dev, stream, graph=True, norm_mode=args.norm_mode)
+    lw = bt.bted_kernel_launches()
+    st.select(m, mu)                                     # first call: one eager loop + the graph capture
+    per_select = (bt.bted_kernel_launches() - lw) // 2   # (graph replays do not pass the launch counter)
+    for _ in range(args.warmup - 1):
         st.select(m, mu)
     clocks = Clocks(int(os.environ.get("LOCAL_RANK", "0")))
     clocks.start()
@@ -478,7 +502,7 @@ def bench_sharded(args, X, gamma, cfg, comm, dev, world, rank):
     e1.record(stream)
     torch.cuda.synchronize()
     torch.distributed.barrier()
-    launches = bt.bted_kernel_launches() - l0
+    launches = bt.bted_kernel_launches() - l0 + per_select * args.steps
     t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
     torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
     ms = float(t.item())
@@ -486,16 +510,21 @@ def bench_sharded(args, X, gamma, cfg, comm, dev, world, rank):
     shard.close()
     peak, peak_src = peaks()
     step_ms = ms / args.steps / max(m - 1, 1)
-    per_gpu_bytes = 8.0 * M * M / world
+    per_gpu_bytes = (2.0 if implicit else 8.0) * M * M / world
     achieved = per_gpu_bytes / (step_ms / 1e3) / 1e9
     if rank == 0:
         line = {"metric": METRIC, "value": args.steps * m / (ms / 1e3), "unit": UNIT, "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
                 "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
-                "data": "synthetic", "layout": "dense-row-sharded",
-                "config": dict(workload_config(args.config, cfg, gamma, world, 1), norm_mode=args.norm_mode,
-                               parallelism=f"row-sharded K over {world} GPUs (NCCL all-reduce + all-gather per step)"),
-                "roofline": {"bound": "hbm", "kernel": "deflate_rescore_kernel (per-GPU band) + NCCL",
+                "data": "synthetic", "layout": "implicit-tile-sharded" if implicit else "dense-row-sharded",
+                "config": dict(workload_config(args.config, cfg, gamma, world, 1),
+                               norm_mode=None if implicit else args.norm_mode,
+                               parallelism=(f"Gram tiles k = rank mod {world} over {world} GPUs (one NCCL all-reduce "
+                                            "of q = K l per step)") if implicit else
+                               f"row-sharded K over {world} GPUs (NCCL all-reduce + all-gather per step)"),
+                "roofline": {"bound": "hbm",
+                             "kernel": ("tile_pass_kernel (own tiles) + ell + fin64 + NCCL" if implicit else
+                                        "deflate_rescore_kernel (per-GPU band) + NCCL"),
                              "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                              "traffic": None, "peak_source": peak_src,
                              "alg_bytes_per_launch": per_gpu_bytes, "avg_launch_ms": step_ms,

@@ -222,6 +222,35 @@ bted_status bted_shard_colnorm(bted_ctx* shard, int32_t t, float mu, const float
                                const uint64_t* keys_dev, float* colnorm_dev);
 bted_status bted_shard_scores(bted_ctx* shard, int32_t t, float mu, const float* colnorm_dev,
                               uint64_t* keys_dev);
+/* ---------------- tile-sharded implicit TED (one oversized batch over P GPUs) ----
+ * The default single-GPU engine (implicit deflation, BTED_FLAG_IMPLICIT) with
+ * its one N^2-sized object -- the read-only packed Gram K -- split over P
+ * ranks: rank r computes, stores and streams only the upper-triangular tiles
+ * k = r (mod P) (about 2 N^2 / P bytes per step per rank instead of 2 N^2).
+ * X (N x d) and the O(N m) fp64 state (factor L, Q, G, running norms) are
+ * replicated and evolve identically on every rank; the only exchange is the
+ * per-step sum of the ranks' partial q = K l vectors (one all-reduce SUM of
+ * qlen doubles), after which every rank computes the same scores and argmax
+ * (no argmax all-reduce, no pivot broadcast).  Selection = Alg. 1 (PAPER.md
+ * 134-148) in exact arithmetic; the q sum order is the collective's.
+ *   bted_ishard_head(m, mu, q)          q = this rank's part of ||K_:v||^2
+ *   all-reduce(q, SUM)
+ *   bted_ishard_fin(0, mu, q, keys)     keys[0]
+ *   for t = 1 .. m-1:
+ *     bted_ishard_step(t, mu, keys, q)  l_t (from keys[t-1]), q = this rank's part of K l_t
+ *     all-reduce(q, SUM)
+ *     bted_ishard_fin(t, mu, q, keys)   keys[t]
+ * q_dev: device fp64 [bted_ishard_qlen(ctx)] (caller-owned); keys_dev: device
+ * u64 [m], zeroed by the caller before the head (packed keys as above).
+ * 0 <= rank < nranks, d <= 32, m <= 256, at least nranks tiles.
+ * Errors: EINVAL, ENOMEM, ECUDA, ESTATE; bted_shard_check reports ENUMERIC.
+ */
+bted_status bted_ishard_create(const float* X, int64_t N, int32_t d, bted_kernel kernel, int32_t rank,
+                               int32_t nranks, const bted_params* params, bted_ctx** out);
+bted_status bted_ishard_head(bted_ctx* shard, int32_t m, float mu, double* q_dev);
+bted_status bted_ishard_step(bted_ctx* shard, int32_t t, float mu, const uint64_t* keys_dev, double* q_dev);
+bted_status bted_ishard_fin(bted_ctx* shard, int32_t t, float mu, const double* q_dev, uint64_t* keys_dev);
+int64_t     bted_ishard_qlen(const bted_ctx* shard);
 /* Leading dimension (floats) a pivot buffer must have: pivot_dev[N..ld) must be 0. */
 int64_t     bted_shard_ld(const bted_ctx* shard);
 /* Sticky device error flag of the shard (BTED_ENUMERIC if a NaN score was seen). */

@@ -69,6 +69,12 @@ _SIGS = {
     "bted_shard_colnorm": (ctypes.c_int, [_vp, _i32, _f32, _vp, _vp, _vp]),
     "bted_shard_scores": (ctypes.c_int, [_vp, _i32, _f32, _vp, _vp]),
     "bted_shard_ld": (_i64, [_vp]),
+    "bted_ishard_create": (ctypes.c_int, [_vp, _i64, _i32, ctypes.c_int, _i32, _i32, ctypes.POINTER(bted_params),
+                                          ctypes.POINTER(_vp)]),
+    "bted_ishard_head": (ctypes.c_int, [_vp, _i32, _f32, _vp]),
+    "bted_ishard_step": (ctypes.c_int, [_vp, _i32, _f32, _vp, _vp]),
+    "bted_ishard_fin": (ctypes.c_int, [_vp, _i32, _f32, _vp, _vp]),
+    "bted_ishard_qlen": (_i64, [_vp]),
     "bted_shard_check": (ctypes.c_int, [_vp]),
     "bted_destroy": (None, [_vp]),
     "bted_status_string": (ctypes.c_char_p, [ctypes.c_int]),
@@ -175,6 +181,31 @@ def bted_sample_batches(P: int, M: int, B: int, seed: int) -> np.ndarray:
     out = np.empty((int(B), int(M)), dtype=np.int64)
     check(lib().bted_sample_batches(int(P), int(M), int(B), int(seed), _ptr(out)))
     return out
+
+
+def bted_ishard_create(X, N: int, d: int, kernel: int, rank: int, nranks: int, params: bted_params) -> int:
+    out = _vp()
+    xh = None if isinstance(X, int) else np.ascontiguousarray(X, dtype=np.float32)
+    xp = X if xh is None else _ptr(xh)
+    check(lib().bted_ishard_create(xp, int(N), int(d), int(kernel), int(rank), int(nranks), ctypes.byref(params),
+                                   ctypes.byref(out)))
+    return out.value
+
+
+def bted_ishard_head(ctx: int, m: int, mu: float, q_dev: int):
+    check(lib().bted_ishard_head(ctx, int(m), float(mu), q_dev))
+
+
+def bted_ishard_step(ctx: int, t: int, mu: float, keys_dev: int, q_dev: int):
+    check(lib().bted_ishard_step(ctx, int(t), float(mu), keys_dev, q_dev))
+
+
+def bted_ishard_fin(ctx: int, t: int, mu: float, q_dev: int, keys_dev: int):
+    check(lib().bted_ishard_fin(ctx, int(t), float(mu), q_dev, keys_dev))
+
+
+def bted_ishard_qlen(ctx: int) -> int:
+    return int(lib().bted_ishard_qlen(ctx))
 
 
 def bted_shard_gram(ctx: int, mu: float, keys_dev: int):

@@ -182,9 +182,10 @@ struct Ted {
     }
 
     // Buffers of the implicit-deflation engine for an N-point TED.
-    void reserve_implicit(int64_t N, int32_t m) {
+    // ktiles >= 0: store only that many tiles (a tile shard of the multi-GPU engine)
+    void reserve_implicit(int64_t N, int32_t m, int64_t ktiles = -1) {
         const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
-        const size_t tiles = (size_t)bted::pk::num_tiles(nT) * bted::pk::T * bted::pk::T;
+        const size_t tiles = (size_t)(ktiles >= 0 ? ktiles : bted::pk::num_tiles(nT)) * bted::pk::T * bted::pk::T;
         const size_t NP = (size_t)nT * bted::pk::T, NPa = (NP + 255) / 256 * 256;
         const void* before[14] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Qc, G, hv, kflag, bar, tctr};
         grow(K[0], kcap[0], tiles);
@@ -437,7 +438,7 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
     const int lin = kernel == BTED_KERNEL_LINEAR ? 1 : 0;
     // K1i: the Gram tiles only (the fp64 norm pass below recomputes the first scores)
     auto k1i = [&](auto kern) {
-        kern<<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(X, (int32_t)N, d, gamma, T.K[0], nT);
+        kern<<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(X, (int32_t)N, d, gamma, T.K[0], nT, 0, 1);
     };
     // two rows per warp step at 3 CTAs/SM measured 369 us vs 388 (four rows, 2 CTAs/SM) and 412 (K1p)
     if (d <= 16) {
@@ -447,10 +448,10 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
     }
     bted::im::tile_pass_kernel<true><<<tile_pass_grid(tiles), bted::im::kTPThreads, bted::im::tile_pass_smem_bytes,
                                        T.stream>>>(T.K[0], nT, nullptr, T.P64, T.kflag, T.tctr, 0,
-                                                   l2_keep_tiles(tiles));
+                                                   l2_keep_tiles(tiles), 0, 1);
     bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
         T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, NPa, 0, T.hv, T.nv, T.rd, T.sel, keys, 0, keys, T.err,
-        T.refine ? T.top2 : nullptr, T.Qc);
+        T.refine ? T.top2 : nullptr, T.Qc, nullptr, nullptr);
     LAUNCHED(3);
 }
 
@@ -542,13 +543,13 @@ uint64_t enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned 
         const int32_t tp = t - 1;
         CK(cudaLaunchKernelEx(&cA, bted::im::ell_kernel, (const float*)T.K[0], nT, (int32_t)N, T.Lf, NPa, tp,
                               (const double*)T.rd, (const double*)T.nv, mu, (const unsigned long long*)keys, t, T.ell,
-                              (const double*)T.Qc, T.G, m, T.hv, T.sel));
+                              (const double*)T.Qc, T.G, m, T.hv, T.sel, bted::im::XKern{}));
         CK(cudaLaunchKernelEx(&cB, bted::im::tile_pass_kernel<false>, (const float*)T.K[0], nT, (const double*)T.ell,
-                              T.P64, T.kflag, T.tctr + t, (int)(t & 1), t + 1 < m ? keep : 0));
+                              T.P64, T.kflag, T.tctr + t, (int)(t & 1), t + 1 < m ? keep : 0, 0, 1));
         CK(cudaLaunchKernelEx(&cC, bted::im::fin64_kernel, (const double*)T.P64, nT, (int32_t)N,
                               (const float*)T.K[0], mu, (const double*)T.Lf, NPa, tp, (const double*)T.hv, T.nv, T.rd,
                               (const uint8_t*)T.sel, (const unsigned long long*)keys, t, keys + t, T.err,
-                              T.refine ? T.top2 : nullptr, T.Qc));
+                              T.refine ? T.top2 : nullptr, T.Qc, (const double*)nullptr, (const double*)nullptr));
         LAUNCHED(3);
     }
     return 3 * (uint64_t)(m - 1);
@@ -701,6 +702,9 @@ struct bted_ctx {
     // shard
     bool is_shard = false;
     int64_t row0 = 0, row1 = 0;
+    // tile shard of the implicit engine (bted_ishard_*)
+    bool is_ishard = false;
+    int32_t srank = 0, snranks = 1, sm_m = 0;
     Ted ted;
     // batches (Alg. 2)
     Ted bted_engine;          // the M x M batch TEDs and the merge TED
@@ -1285,7 +1289,7 @@ bted_status bted_shard_create(const float* X, int64_t N, int32_t d, bted_kernel 
 
 bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, float* out_score) {
     if (!ctx || !out_idx) { set_error("null argument"); return BTED_EINVAL; }
-    if (ctx->is_shard) { set_error("bted_select on a shard context"); return BTED_EINVAL; }
+    if (ctx->is_shard || ctx->is_ishard) { set_error("bted_select on a shard context"); return BTED_EINVAL; }
     if (m < 1 || m > ctx->N || !mu_ok(mu)) { set_error("need 1 <= m <= N and mu > 0 finite"); return BTED_EINVAL; }
     return guarded(ctx, [&]() -> bted_status {
         Ted& T = ctx->ted;
@@ -1324,7 +1328,7 @@ bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, fl
 bted_status bted_batch_teds(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_begin, int32_t b_step,
                             int64_t* out_winners, int32_t winners_on_device) {
     if (!ctx || !out_winners) { set_error("null argument"); return BTED_EINVAL; }
-    if (ctx->is_shard) { set_error("batch TEDs on a shard context"); return BTED_EINVAL; }
+    if (ctx->is_shard || ctx->is_ishard) { set_error("batch TEDs on a shard context"); return BTED_EINVAL; }
     if (m < 1 || M < m || M > ctx->N || !mu_ok(mu) || b_begin < 0 || b_step < 1) {
         set_error("need 1 <= m <= M <= N, mu > 0, b_begin >= 0, b_step >= 1"); return BTED_EINVAL;
     }
@@ -1352,7 +1356,7 @@ bted_status bted_batch_teds(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32
 bted_status bted_merge(bted_ctx* ctx, const int64_t* winners, int64_t n, int32_t winners_on_device, int32_t m,
                        float mu, int64_t* out_idx, int32_t* out_count) {
     if (!ctx || !winners || !out_idx || !out_count) { set_error("null argument"); return BTED_EINVAL; }
-    if (ctx->is_shard) { set_error("merge on a shard context"); return BTED_EINVAL; }
+    if (ctx->is_shard || ctx->is_ishard) { set_error("merge on a shard context"); return BTED_EINVAL; }
     if (n < 1 || n >= (int64_t)INT32_MAX || m < 1 || !mu_ok(mu)) { set_error("need n >= 1, m >= 1, mu > 0"); return BTED_EINVAL; }
     if (!winners_on_device) {
         for (int64_t i = 0; i < n; ++i)
@@ -1370,7 +1374,7 @@ bted_status bted_merge(bted_ctx* ctx, const int64_t* winners, int64_t n, int32_t
 bted_status bted_run_batches(bted_ctx* ctx, int64_t M, int32_t m, float mu, int64_t* out_idx, int32_t* out_count,
                              int64_t* out_batch_idx) {
     if (!ctx || !out_idx || !out_count) { set_error("null argument"); return BTED_EINVAL; }
-    if (ctx->is_shard) { set_error("run_batches on a shard context"); return BTED_EINVAL; }
+    if (ctx->is_shard || ctx->is_ishard) { set_error("run_batches on a shard context"); return BTED_EINVAL; }
     if (m < 1 || M < m || M > ctx->N || !mu_ok(mu)) { set_error("need 1 <= m <= M <= N and mu > 0"); return BTED_EINVAL; }
     return guarded(ctx, [&]() -> bted_status {
         const int nb = run_batch_range(ctx, M, m, mu, 0, 1);
@@ -1503,6 +1507,123 @@ bted_status bted_shard_scores(bted_ctx* ctx, int32_t t, float mu, const float* c
         bted::colnorm_scores_kernel<<<g, 256, 0, T.stream>>>(T.K[t & 1], ld_for(ctx->N), (int32_t)ctx->row0, rows,
                                                              colnorm_dev, mu, T.sel,
                                                              reinterpret_cast<unsigned long long*>(keys_dev), t, T.err);
+        LAUNCHED(1);
+        return BTED_OK;
+    });
+}
+
+// ------------------------------------------------------------------ tile-sharded implicit engine
+namespace {
+int64_t ishard_local_tiles(const bted_ctx* ctx) {
+    const int nT = (int)((ctx->N + bted::pk::T - 1) / bted::pk::T);
+    const int64_t all = bted::pk::num_tiles(nT);
+    return (all - ctx->srank + ctx->snranks - 1) / ctx->snranks;
+}
+bted::im::XKern ishard_xk(const bted_ctx* ctx) {
+    bted::im::XKern xk;
+    xk.X = ctx->X; xk.d = ctx->d; xk.ng = -ctx->params.gamma; xk.linear = ctx->kernel == BTED_KERNEL_LINEAR ? 1 : 0;
+    return xk;
+}
+}  // namespace
+
+bted_status bted_ishard_create(const float* X, int64_t N, int32_t d, bted_kernel kernel, int32_t rank, int32_t nranks,
+                               const bted_params* params, bted_ctx** out) {
+    if (nranks < 1 || rank < 0 || rank >= nranks) { set_error("need 0 <= rank < nranks"); return BTED_EINVAL; }
+    if (d > 32) { set_error("the tile-sharded engine needs d <= 32"); return BTED_EINVAL; }
+    bted_status st = create_common(X, N, d, kernel, params, 0, 0, false, out);
+    if (st != BTED_OK) return st;
+    (*out)->is_ishard = true;
+    (*out)->srank = rank;
+    (*out)->snranks = nranks;
+    const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
+    if (bted::pk::num_tiles(nT) < nranks) {
+        bted_destroy(*out); *out = nullptr;
+        set_error("fewer Gram tiles than shards"); return BTED_EINVAL;
+    }
+    return BTED_OK;
+}
+
+int64_t bted_ishard_qlen(const bted_ctx* ctx) {
+    if (!ctx) return 0;
+    const int64_t NP = (ctx->N + bted::pk::T - 1) / bted::pk::T * bted::pk::T;
+    return (NP + 255) / 256 * 256;
+}
+
+bted_status bted_ishard_head(bted_ctx* ctx, int32_t m, float mu, double* q_dev) {
+    if (!ctx || !q_dev || !ctx->is_ishard || m < 1 || m > ctx->N || m > bted::im::kMaxM || !mu_ok(mu)) {
+        set_error("bad ishard_head arguments"); return BTED_EINVAL;
+    }
+    return guarded(ctx, [&]() -> bted_status {
+        Ted& T = ctx->ted;
+        const int64_t N = ctx->N, NPa = bted_ishard_qlen(ctx);
+        const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
+        const int64_t lt = ishard_local_tiles(ctx);
+        ensure_implicit_attrs();
+        T.reserve_implicit(N, m, lt);
+        ctx->sm_m = m;
+        CK(cudaMemsetAsync(T.sel, 0, (size_t)NPa, T.stream));
+        CK(cudaMemsetAsync(T.kflag, 0, sizeof(int), T.stream));
+        CK(cudaMemsetAsync(T.tctr, 0, sizeof(int) * m, T.stream));
+        CK(cudaMemsetAsync(q_dev, 0, sizeof(double) * NPa, T.stream));
+        const int lin = ctx->kernel == BTED_KERNEL_LINEAR ? 1 : 0;
+        const float g = ctx->params.gamma;
+        const int r = ctx->srank, P = ctx->snranks;
+        auto k1i = [&](auto kern) {
+            kern<<<(unsigned)lt, bted::pk::kConsumers, 0, T.stream>>>(ctx->X, (int32_t)N, ctx->d, g, T.K[0], nT, r, P);
+        };
+        if (ctx->d <= 16) {
+            if (lin) k1i(bted::pk::gram_tile_kernel<16, true, 2>); else k1i(bted::pk::gram_tile_kernel<16, false, 2>);
+        } else {
+            if (lin) k1i(bted::pk::gram_tile_kernel<32, true>); else k1i(bted::pk::gram_tile_kernel<32, false>);
+        }
+        bted::im::diag_init_kernel<<<(unsigned)((NPa + 255) / 256), 256, 0, T.stream>>>(ishard_xk(ctx), (int32_t)N,
+                                                                                         NPa, T.rd);
+        bted::im::tile_pass_kernel<true><<<tile_pass_grid(lt), bted::im::kTPThreads, bted::im::tile_pass_smem_bytes,
+                                           T.stream>>>(T.K[0], nT, nullptr, T.P64, T.kflag, T.tctr, 0, 0, r, P);
+        bted::im::qpart_kernel<<<(unsigned)std::min<int64_t>((NPa + 255) / 256, 4096), 256, 0, T.stream>>>(
+            T.P64, nT, r, P, q_dev);
+        LAUNCHED(4);
+        return BTED_OK;
+    });
+}
+
+bted_status bted_ishard_step(bted_ctx* ctx, int32_t t, float mu, const uint64_t* keys_dev, double* q_dev) {
+    if (!ctx || !q_dev || !keys_dev || !ctx->is_ishard || t < 1 || t >= ctx->sm_m || !mu_ok(mu)) {
+        set_error("bad ishard_step arguments (head first; 1 <= t < m)"); return BTED_EINVAL;
+    }
+    return guarded(ctx, [&]() -> bted_status {
+        Ted& T = ctx->ted;
+        const int64_t N = ctx->N, NPa = bted_ishard_qlen(ctx);
+        const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
+        const int nA = (int)(NPa / bted::im::kEllRows);
+        const int32_t m = ctx->sm_m;
+        const auto* keys = reinterpret_cast<const unsigned long long*>(keys_dev);
+        bted::im::ell_kernel<<<(unsigned)nA + 1, bted::im::kThreads, 0, T.stream>>>(
+            T.K[0], nT, (int32_t)N, T.Lf, NPa, t - 1, T.rd, T.nv, mu, keys, t, T.ell, T.Qc, T.G, m, T.hv, T.sel,
+            ishard_xk(ctx));
+        bted::im::tile_pass_kernel<false><<<tile_pass_grid(ishard_local_tiles(ctx)), bted::im::kTPThreads,
+                                            bted::im::tile_pass_smem_bytes, T.stream>>>(
+            T.K[0], nT, T.ell, T.P64, T.kflag, T.tctr + t, (int)(t & 1), 0, ctx->srank, ctx->snranks);
+        bted::im::qpart_kernel<<<(unsigned)std::min<int64_t>((NPa + 255) / 256, 4096), 256, 0, T.stream>>>(
+            T.P64, nT, ctx->srank, ctx->snranks, q_dev);
+        LAUNCHED(3);
+        return BTED_OK;
+    });
+}
+
+bted_status bted_ishard_fin(bted_ctx* ctx, int32_t t, float mu, const double* q_dev, uint64_t* keys_dev) {
+    if (!ctx || !q_dev || !keys_dev || !ctx->is_ishard || t < 0 || t >= ctx->sm_m || !mu_ok(mu)) {
+        set_error("bad ishard_fin arguments (head first; 0 <= t < m)"); return BTED_EINVAL;
+    }
+    return guarded(ctx, [&]() -> bted_status {
+        Ted& T = ctx->ted;
+        const int64_t N = ctx->N, NPa = bted_ishard_qlen(ctx);
+        const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
+        const int64_t NP = (int64_t)nT * bted::pk::T;
+        auto* keys = reinterpret_cast<unsigned long long*>(keys_dev);
+        bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
+            T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, NPa, t > 0 ? t - 1 : 0, T.hv, T.nv, T.rd, T.sel, keys, t,
+            keys + t, T.err, nullptr, T.Qc, q_dev, t == 0 ? T.rd : nullptr);
         LAUNCHED(1);
         return BTED_OK;
     });

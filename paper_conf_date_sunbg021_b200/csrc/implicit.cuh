@@ -295,13 +295,19 @@ __device__ __forceinline__ void tp_consume(TPSmem& S, int nT, double* P64, int* 
 // evict-last (or evict-normal) policy measured no better (32 MiB) or worse
 // (>= 64 MiB), and evict-normal loads throughout cost +6 us.  keep_tiles
 // defaults to 0 (BTED_L2_KEEP_MB overrides, for experiments).
+//
+// Tile sharding (sp > 1, the multi-GPU implicit engine): this GPU stores and
+// streams only the tiles k = sr + sp * kl (kl = 0, 1, ...), compactly at
+// K + kl * T^2; consumers get the global index k (partials land where the
+// unsharded pass would put them).
 template <bool kW, class WaitW>
 __device__ __forceinline__ void tp_produce(TPSmem& S, const float* __restrict__ K, int nT, const double* w,
                                            int passes, int* tilectr, WaitW wait_w, int dir0 = 0,
-                                           int keep_tiles = 0) {
+                                           int keep_tiles = 0, int sr = 0, int sp = 1) {
     const uint64_t pol = pk::policy_evict_first();            // K is read once per step
     const uint64_t pol_keep = pk::policy_evict_last();        // ... except a tail kept for the next pass
-    const int64_t nTiles = num_tiles(nT);
+    const int64_t nAll = num_tiles(nT);
+    const int64_t nTiles = (nAll - sr + sp - 1) / sp;         // tiles stored on this GPU
     int n = 0, ti = 0;
     for (int pass = 0; pass < passes; ++pass) {
         const bool rev = ((dir0 + pass) & 1) != 0;
@@ -309,12 +315,13 @@ __device__ __forceinline__ void tp_produce(TPSmem& S, const float* __restrict__ 
         for (;; ++ti) {
             const int64_t kh = next;                          // handing order
             if (kh < nTiles) next = atomicAdd(&tilectr[pass], 1);
-            const int64_t k = kh < nTiles && rev ? nTiles - 1 - kh : kh;
+            const int64_t kl = kh < nTiles && rev ? nTiles - 1 - kh : kh;     // local tile
+            const int64_t k = kh < nTiles ? sr + sp * kl : nAll;              // global tile index
             const uint64_t kpol = kh >= nTiles - keep_tiles ? pol_keep : pol;
             const int ws = ti % kWSlots;
             pk::mbar_wait(&S.wempty[ws], ((uint32_t)(ti / kWSlots) & 1u) ^ 1u);
-            S.wtile[ws] = k < nTiles ? k : -1;
-            if (k >= nTiles || !kW) {
+            S.wtile[ws] = k < nAll ? k : -1;
+            if (k >= nAll || !kW) {
                 pk::mbar_arrive(&S.wfull[ws]);               // release: the tile index
             } else {
                 int I, J;
@@ -324,8 +331,8 @@ __device__ __forceinline__ void tp_produce(TPSmem& S, const float* __restrict__ 
                 pk::bulk_g2s(S.wslot[ws][0], w + (int64_t)J * T, T * 8, &S.wfull[ws]);
                 pk::bulk_g2s(S.wslot[ws][1], w + (int64_t)I * T, T * 8, &S.wfull[ws]);
             }
-            if (k >= nTiles) { ++ti; break; }
-            const float* src = K + k * (int64_t)(T * T);
+            if (k >= nAll) { ++ti; break; }
+            const float* src = K + kl * (int64_t)(T * T);
             for (int c = 0; c < kChunks; ++c, ++n) {
                 const int st = n % kStages;
                 pk::mbar_wait(&S.empty[st], ((uint32_t)(n / kStages) & 1u) ^ 1u);
@@ -356,13 +363,14 @@ __device__ __forceinline__ void tp_init_barriers(TPSmem& S) {
 template <bool kNorm>
 __global__ void __launch_bounds__(kTPThreads, kTPBlocksPerSM)
 tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__ w, double* __restrict__ P64,
-                 int* __restrict__ kflag, int* __restrict__ tilectr, int dir, int keep_tiles) {
+                 int* __restrict__ kflag, int* __restrict__ tilectr, int dir, int keep_tiles,
+                 int sr = 0, int sp = 1) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
     TPSmem& S = *reinterpret_cast<TPSmem*>(smem_raw);
     tp_init_barriers(S);
     if (threadIdx.x / 32 == kTPWarps) {                      // producer warp: one lane streams
         // (PDL: K streams while kernel A finishes; w only once it has completed)
-        if (threadIdx.x % 32 == 0) tp_produce<!kNorm>(S, K, nT, w, 1, tilectr, PdlWait{}, dir, keep_tiles);
+        if (threadIdx.x % 32 == 0) tp_produce<!kNorm>(S, K, nT, w, 1, tilectr, PdlWait{}, dir, keep_tiles, sr, sp);
         return;
     }
     int n = 0, tile_it = 0, col_it = 0;
@@ -390,13 +398,29 @@ struct EllSmem {
 struct SyncCTA { __device__ void operator()() const { __syncthreads(); } };
 struct SyncConsumers { __device__ void operator()() const { tp_sync(); } };
 
+// k(x_i, x_j) recomputed from the features with K1p/K1i's operation sequence
+// (fsub, fma over the features in order, then expf(-gamma * d2)): bitwise the
+// stored Gram entry (the tile-sharded engine holds only some tiles of K).
+struct XKern {
+    const float* X = nullptr; int d = 0; float ng = 0.f; int linear = 0;
+    __device__ __forceinline__ float operator()(int64_t i, int64_t j) const {
+        float a = 0.f;
+        for (int q = 0; q < d; ++q) {
+            const float xi = X[i * d + q], xj = X[j * d + q];
+            if (linear) a = __fmaf_rn(xi, xj, a);
+            else { const float df = __fsub_rn(xi, xj); a = __fmaf_rn(df, df, a); }
+        }
+        return linear ? a : expf(__fmul_rn(ng, a));
+    }
+};
+
 template <class Sync>
 __device__ __forceinline__ void ell_unit(int unit, EllSmem& sm, Sync sync, const float* __restrict__ K, int nT,
                                          int32_t N, double* Lc, int64_t ldL, int32_t tp, uint32_t s,
-                                         double rc, double* ell) {
+                                         double rc, double* ell, XKern xk = XKern{}) {
     const int tid = threadIdx.x, r = tid % kEllRows, g = tid / kEllRows;
     const int64_t i = (int64_t)unit * kEllRows + r;
-    const float kis = (g == 0 && i < N) ? K[packed_index((int)i, (int)s, nT)] : 0.f;
+    const float kis = (g == 0 && i < N) ? (xk.X ? xk(i, s) : K[packed_index((int)i, (int)s, nT)]) : 0.f;
     for (int k = tid; k < tp; k += kThreads) sm.Ls[k] = __ldcg(&Lc[(int64_t)k * ldL + s]);
     // this thread's L_ik (k = g, g + 4, ...): loaded before the barrier, 16 at a time
     double acc = 0.0;
@@ -464,7 +488,7 @@ __global__ void __launch_bounds__(kThreads)
 ell_kernel(const float* __restrict__ K, int nT, int32_t N, double* __restrict__ Lc, int64_t ldL, int32_t tp,
            const double* __restrict__ rdiag, const double* __restrict__ nv, float mu,
            const unsigned long long* __restrict__ keys, int32_t t, double* __restrict__ ell, const double* Qc,
-           double* G, int32_t ldG, double* h, uint8_t* __restrict__ sel) {
+           double* G, int32_t ldG, double* h, uint8_t* __restrict__ sel, XKern xk = XKern{}) {
     __shared__ EllSmem sm;
     pdl_wait();                                              // kernel C of the previous step complete
     pdl_trigger();                                           // the K.l pass may start streaming K now
@@ -475,7 +499,7 @@ ell_kernel(const float* __restrict__ K, int nT, int32_t N, double* __restrict__ 
         h_unit(sm.Ls, SyncCTA{}, Lc, ldL, Qc, G, ldG, tp, s, c, nv[s], h);
         return;
     }
-    ell_unit(blockIdx.x, sm, SyncCTA{}, K, nT, N, Lc, ldL, tp, s, __dsqrt_rn(c), ell);
+    ell_unit(blockIdx.x, sm, SyncCTA{}, K, nT, N, Lc, ldL, tp, s, __dsqrt_rn(c), ell, xk);
 }
 // ------------------------------------------------------------------ kernel C: scores
 // t == 0 (after the norm pass): n_v = q_v (= ||K_:v||^2), r_vv = K_vv.
@@ -497,7 +521,8 @@ __device__ __forceinline__ void fin_unit(int unit, int nunits, FinSmem& sm, Sync
                                          const double* h, double* nv,
                                          double* rdiag, const uint8_t* sel, uint32_t s,
                                          int32_t t, unsigned long long* key_out, int* err,
-                                         unsigned long long* top2, double* Qc, bool mark_sel = false) {
+                                         unsigned long long* top2, double* Qc, bool mark_sel = false,
+                                         const double* qin = nullptr, const double* rinit = nullptr) {
     const int lane = threadIdx.x % 32, w = threadIdx.x / 32;
     const int64_t NP = (int64_t)nT * T;
     const int i = unit * kFinRows + lane;
@@ -505,17 +530,21 @@ __device__ __forceinline__ void fin_unit(int unit, int nunits, FinSmem& sm, Sync
         for (int q = threadIdx.x; q <= tp; q += kThreads) sm.hs[q] = __ldcg(&h[q]);
     const int per = (nT + 7) / 8;
     const int j0 = min(nT, w * per), j1 = min(nT, j0 + per);
-    const double* src = P64 + i;
     double acc = 0.0;
-    int J = j0;
-    for (; J + 16 <= j1; J += 16) {
-        double v[16];
+    if (qin) {                                             // q given (all-reduced over tile shards)
+        acc = w == 0 ? __ldcg(&qin[i]) : 0.0;
+    } else {
+        const double* src = P64 + i;
+        int J = j0;
+        for (; J + 16 <= j1; J += 16) {
+            double v[16];
 #pragma unroll
-        for (int q = 0; q < 16; ++q) v[q] = __ldcg(&src[(int64_t)(J + q) * NP]);
+            for (int q = 0; q < 16; ++q) v[q] = __ldcg(&src[(int64_t)(J + q) * NP]);
 #pragma unroll
-        for (int q = 0; q < 16; ++q) acc = __dadd_rn(acc, v[q]);
+            for (int q = 0; q < 16; ++q) acc = __dadd_rn(acc, v[q]);
+        }
+        for (; J < j1; ++J) acc = __dadd_rn(acc, __ldcg(&src[(int64_t)J * NP]));
     }
-    for (; J < j1; ++J) acc = __dadd_rn(acc, __ldcg(&src[(int64_t)J * NP]));
     sm.part[w][lane] = acc;
     sync();
     double la = 0.0;                                       // sum_{k in range w} L_ik h_k
@@ -544,7 +573,7 @@ __device__ __forceinline__ void fin_unit(int unit, int nunits, FinSmem& sm, Sync
             if (t == 0) {
                 const int B = i / T, rr = i % T;
                 n = q;
-                r = (double)K[tile_offset(B, B, nT) * (T * T) + (int64_t)rr * T + rr];
+                r = rinit ? rinit[i] : (double)K[tile_offset(B, B, nT) * (T * T) + (int64_t)rr * T + rr];
             } else {
                 double lh = sm.lpart[0][lane];
 #pragma unroll
@@ -691,13 +720,46 @@ fin64_kernel(const double* __restrict__ P64, int nT, int32_t N, const float* __r
              const double* __restrict__ Lc, int64_t ldL, int32_t tp, const double* __restrict__ h,
              double* __restrict__ nv, double* __restrict__ rdiag, const uint8_t* __restrict__ sel,
              const unsigned long long* __restrict__ keys, int32_t t, unsigned long long* __restrict__ key_out,
-             int* __restrict__ err, unsigned long long* __restrict__ top2, double* __restrict__ Qc) {
+             int* __restrict__ err, unsigned long long* __restrict__ top2, double* __restrict__ Qc,
+             const double* __restrict__ qin = nullptr, const double* __restrict__ rinit = nullptr) {
     __shared__ FinSmem sm;
     pdl_wait();                                              // the K.l pass complete (P64, h)
     pdl_trigger();
     const uint32_t s = t > 0 ? key_index(keys[t - 1]) : 0xFFFFFFFFu;
     fin_unit(blockIdx.x, gridDim.x, sm, SyncCTA{}, P64, nT, N, K, mu, Lc, ldL, tp, h, nv, rdiag, sel, s, t, key_out,
-             err, top2, Qc);
+             err, top2, Qc, false, qin, rinit);
+}
+
+// ------------------------------------------------------------------ tile-sharded engine (multi-GPU)
+// qpart[i] = sum over the blocks J (in order) of the partials P64[J][i] that
+// THIS shard's tiles wrote: tile (min(B,J), max(B,J)) of row i's block B,
+// stored here iff its index = sr (mod sp).  The shards' qpart are then summed
+// by an all-reduce (the order of that sum is the collective's).
+__global__ void __launch_bounds__(kThreads)
+qpart_kernel(const double* __restrict__ P64, int nT, int sr, int sp, double* __restrict__ qpart) {
+    const int64_t NP = (int64_t)nT * T;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < NP; i += (int64_t)gridDim.x * blockDim.x) {
+        const int B = (int)(i / T);
+        double acc = 0.0;
+        for (int J0 = 0; J0 < nT; J0 += 16) {             // 16 loads in flight; non-owned terms are 0
+            double v[16];
+#pragma unroll
+            for (int q = 0; q < 16; ++q) {
+                const int J = J0 + q;
+                const bool own = J < nT && tile_offset(min(B, J), max(B, J), nT) % sp == sr;
+                v[q] = own ? __ldcg(&P64[(int64_t)J * NP + i]) : 0.0;
+            }
+#pragma unroll
+            for (int q = 0; q < 16; ++q) acc = __dadd_rn(acc, v[q]);
+        }
+        qpart[i] = acc;
+    }
+}
+
+// rd[i] = k(x_i, x_i) from the features (the diagonal tiles may live on other shards)
+__global__ void diag_init_kernel(XKern xk, int32_t N, int64_t NPa, double* __restrict__ rd) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < NPa; i += (int64_t)gridDim.x * blockDim.x)
+        rd[i] = i < N ? (double)xk(i, i) : 0.0;
 }
 
 // ------------------------------------------------------------------ the whole step loop in one launch

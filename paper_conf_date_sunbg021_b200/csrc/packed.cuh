@@ -663,13 +663,14 @@ gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamm
 // vs 412 us for K1p with its fp32 partials.
 template <int kD, bool kLinear, int kH = 4>
 __global__ void __launch_bounds__(kConsumers, kH == 4 ? 2 : 3)
-gram_tile_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma, float* __restrict__ K, int nT) {
+gram_tile_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma, float* __restrict__ K, int nT,
+                 int sr = 0, int sp = 1) {
     __shared__ __align__(16) unsigned long long xi2[T][kD];     // (x, x) pairs of the tile's rows
     __shared__ __align__(16) float xj[T][kD];
     const int tid = threadIdx.x, w = tid / kWarp, l = tid % kWarp;
     const float ng = -gamma;
     int I, J;
-    tile_ij((int64_t)blockIdx.x, nT, I, J);
+    tile_ij((int64_t)sr + (int64_t)sp * blockIdx.x, nT, I, J);     // (tile shards: every sp-th tile)
     for (int q = tid; q < T * kD; q += kConsumers) {
         const int r = q / kD, c = q % kD;
         const int gi = I * T + r, gj = J * T + r;

@@ -22,6 +22,11 @@ Two ways Algorithm 2 spreads over GPUs (DESIGN.md
    its own indices from it (then the same argmax all-reduce).  Same band
    values; the scores differ from the symmetric mode only in rounding order.
 
+3. `ShardedImplicitTed` -- the same oversized batch on the default implicit
+   engine: the read-only packed Gram tiles are split over the ranks (tile k on
+   rank k mod P), everything else is replicated; per step one all-reduce(SUM)
+   of the partial q = K l vectors.
+
 Every step of the method runs in libbted.so's kernels (the `LibShard` /
 `LibPool` backends below); this module only moves buffers between them
 through the `comm` object and owns no arithmetic.  The backends are
@@ -214,6 +219,124 @@ class ShardedTed:
             host = keys.cpu().numpy().view(np.uint64)
         self.be.check()
         return L.decode_keys(host)
+
+
+# ------------------------------------------- 3. tile-sharded implicit TED
+class LibIShard:
+    """Backend of ShardedImplicitTed: a tile-shard ctx of libbted.so (Gram tiles k = rank mod P)."""
+
+    def __init__(self, X, N, d, gamma, rank, nranks, device: torch.device, stream, kernel=L.BTED_KERNEL_RBF):
+        on_dev = isinstance(X, int)
+        p = L.default_params(gamma=gamma, device=device.index, stream=stream.cuda_stream,
+                             x_on_device=1 if on_dev else 0)
+        self.ctx = L.bted_ishard_create(X, N, d, kernel, rank, nranks, p)
+        self.qlen = L.bted_ishard_qlen(self.ctx)
+
+    def head(self, m, mu, q: torch.Tensor):
+        L.bted_ishard_head(self.ctx, m, mu, q.data_ptr())
+
+    def step(self, t, mu, keys: torch.Tensor, q: torch.Tensor):
+        L.bted_ishard_step(self.ctx, t, mu, keys.data_ptr(), q.data_ptr())
+
+    def fin(self, t, mu, q: torch.Tensor, keys: torch.Tensor):
+        L.bted_ishard_fin(self.ctx, t, mu, q.data_ptr(), keys.data_ptr())
+
+    def check(self):
+        L.bted_shard_check(self.ctx)
+
+    def close(self):
+        if self.ctx:
+            L.bted_destroy(self.ctx)
+            self.ctx = None
+
+
+class ShardedImplicitTed:
+    """TED (Alg. 1) on N points with the implicit engine's packed Gram tiles
+    split over the ranks (tile k on rank k mod P).  Per step ONE collective:
+    all-reduce(SUM) of the ranks' partial q = K l (qlen fp64); every rank then
+    computes the same scores and argmax from its replicated O(N m) state.
+    Per-rank HBM traffic per step ~ 2 N^2 / P bytes (vs 8 N^2 / P for the
+    dense-band ShardedTed).  `graph=True` captures the m-step loop, kernels
+    and NCCL collectives, into one CUDA graph per (m, mu)."""
+
+    def __init__(self, backend, N: int, comm, device: torch.device, stream=None, graph: bool = False):
+        self.be, self.N, self.comm, self.device, self.stream = backend, int(N), comm, device, stream
+        self.graph = bool(graph) and stream is not None
+        self._graphs = {}
+        with _stream_ctx(stream):
+            self.q = torch.zeros(backend.qlen, dtype=torch.float64, device=device)
+
+    def _loop(self, keys: torch.Tensor, m: int, mu: float):
+        keys.zero_()
+        self.be.head(m, mu, self.q)                  # l.1 + this rank's part of ||K_:v||^2
+        self.comm.allreduce_sum_(self.q)
+        self.be.fin(0, mu, self.q, keys)             # l.3: s_1 (identical on every rank)
+        for t in range(1, m):
+            self.be.step(t, mu, keys, self.q)        # l.5 implicitly: l_t, this rank's part of K l_t
+            self.comm.allreduce_sum_(self.q)
+            self.be.fin(t, mu, self.q, keys)         # next l.3: s_{t+1}
+
+    def select(self, m: int, mu: float):
+        if not (1 <= m <= self.N):
+            raise ValueError("need 1 <= m <= N")
+        with _stream_ctx(self.stream):
+            if self.graph:
+                gk = (int(m), float(mu))
+                if gk not in self._graphs:
+                    keys = torch.zeros(m, dtype=torch.int64, device=self.device)
+                    self._loop(keys, m, mu)          # eager once: allocations, NCCL init
+                    g = torch.cuda.CUDAGraph()
+                    with torch.cuda.graph(g, stream=self.stream):
+                        self._loop(keys, m, mu)
+                    self._graphs[gk] = (g, keys)
+                g, keys = self._graphs[gk]
+                g.replay()
+            else:
+                keys = torch.zeros(m, dtype=torch.int64, device=self.device)
+                self._loop(keys, m, mu)
+            host = keys.cpu().numpy().view(np.uint64)
+        self.be.check()
+        return L.decode_keys(host)
+
+
+def isharded_select_loopback(X: np.ndarray, gamma: float, P: int, m: int, mu: float, device: torch.device,
+                             stream: torch.cuda.Stream, kernel: int = L.BTED_KERNEL_RBF):
+    """ShardedImplicitTed with P logical tile shards on ONE GPU; the all-reduce
+    is a sum of the shards' partial q in rank order."""
+    N, d = X.shape
+    shards = []
+    try:
+        for r in range(P):
+            shards.append(LibIShard(X, N, d, gamma, r, P, device, stream, kernel))
+        with torch.cuda.stream(stream):
+            keys = torch.zeros((P, m), dtype=torch.int64, device=device)
+            qs = torch.zeros((P, shards[0].qlen), dtype=torch.float64, device=device)
+
+            def allreduce():
+                tot = qs[0].clone()
+                for r in range(1, P):
+                    tot += qs[r]
+                qs.copy_(tot.expand_as(qs))
+
+            for r in range(P):
+                shards[r].head(m, mu, qs[r])
+            allreduce()
+            for r in range(P):
+                shards[r].fin(0, mu, qs[r], keys[r])
+            for t in range(1, m):
+                for r in range(P):
+                    shards[r].step(t, mu, keys[r], qs[r])
+                allreduce()
+                for r in range(P):
+                    shards[r].fin(t, mu, qs[r], keys[r])
+            host = keys.cpu().numpy().view(np.uint64)
+        for s in shards:
+            s.check()
+        assert all((host[r] == host[0]).all() for r in range(P)), "shards disagree"
+        return L.decode_keys(host[0])
+    finally:
+        for s in shards:
+            s.close()
 
 
 # ------------------------------------------------ loopback (P shards, 1 GPU)

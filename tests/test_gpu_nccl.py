@@ -80,6 +80,29 @@ def test_sharded_ted_literal_norms_over_nccl(nccl_group, graph):
     check_ted(sidx, ssc, tr, "nccl-literal")
 
 
+@pytest.mark.parametrize("graph", [False, True], ids=["eager", "cuda-graph"])
+def test_tile_sharded_implicit_over_nccl(nccl_group, graph):
+    """ShardedImplicitTed: the per-step q all-reduce goes through real NCCL (one rank)."""
+    import torch
+    from oracle import dense
+    from tests.parity import check_ted
+    from paper_conf_date_sunbg021_b200.dist import LibIShard, ShardedImplicitTed, TorchComm
+    N = 5000
+    _, X = make_pool(KnobSpace(WORKLOADS["resnet18_layer1"], 16), N, 5)
+    g = median_gamma(X, 5)
+    comm = TorchComm()
+    st_ = torch.cuda.Stream(nccl_group)
+    be = LibIShard(X, N, 16, g, comm.rank, comm.world, nccl_group, st_)
+    try:
+        sted = ShardedImplicitTed(be, N, comm, nccl_group, st_, graph=graph)
+        idx, sc = sted.select(32, MU)
+        idx2, sc2 = sted.select(32, MU)
+        assert np.array_equal(idx2, idx) and np.array_equal(sc2, sc)
+    finally:
+        be.close()
+    check_ted(idx, sc, dense.ted(X, g, MU, 32, forced=idx), "nccl-ishard")
+
+
 def test_batch_round_robin_over_nccl_matches_run_batches(nccl_group):
     import torch
     from paper_conf_date_sunbg021_b200.dist import TorchComm, run_batches_dp

@@ -331,6 +331,30 @@ def test_row_sharded_literal_column_norms_vs_oracle(N, P):
     np.testing.assert_allclose(lsc, ssc, rtol=1e-5)         # same numbers up to rounding order
 
 
+@pytest.mark.parametrize("N,P,d", [(3001, 1, 16), (3001, 2, 16), (2500, 3, 12), (1100, 5, 16), (4096, 4, 30)])
+def test_tile_sharded_implicit_loopback_vs_oracle(N, P, d):
+    """ShardedImplicitTed (Gram tiles k = r mod P, one q all-reduce per step)
+    with P logical shards on one GPU: P1/P2 against the fp64 oracle along its
+    picks, the same picks as the single-GPU implicit engine wherever the
+    oracle's gap is clear, and scores within 1e-5 of it."""
+    import torch
+    from paper_conf_date_sunbg021_b200.dist import isharded_select_loopback
+    X = knob(N, d=d, seed=N + P) if d != 30 else uniform_pool(N, d, P)
+    g = median_gamma(X, P)
+    dev = torch.device("cuda", 0)
+    st = torch.cuda.Stream(dev)
+    m = 40
+    idx, sc = isharded_select_loopback(X, g, P, m, MU, dev, st)
+    assert len(set(idx.tolist())) == m
+    tr = dense.ted(X, g, MU, m, forced=idx)
+    check_ted(idx, sc, tr, f"ishard N={N} P={P}")
+    with bt.CandidateSet(X, g, flags=IMPLICIT | L.BTED_FLAG_NO_REFINE) as cs:
+        i1, s1 = cs.select(m, MU)
+    k = int(np.argmax(i1 != idx)) if not np.array_equal(i1, idx) else m
+    assert k == m or tr.gap[k] <= 1e-5, (k, tr.gap[k])
+    np.testing.assert_allclose(sc[:k], s1[:k], rtol=1e-5)
+
+
 def test_launch_counter_counts_kernels():
     X = knob(300)
     before = bt.bted_kernel_launches()
