@@ -528,7 +528,8 @@ def bench_sharded(args, X, gamma, cfg, comm, dev, world, rank):
                              "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                              "traffic": None, "peak_source": peak_src,
                              "alg_bytes_per_launch": per_gpu_bytes, "avg_launch_ms": step_ms,
-                             "note": "per-GPU step time includes the two collectives"},
+                             "note": ("per-GPU step time (Gram + head amortised) includes the q all-reduce"
+                                      if implicit else "per-GPU step time includes the two collectives")},
                 "cpu_baseline": None, "e2e": None, "gpu_launches": int(launches), "clocks": clk,
                 "final_selection_head": [int(x) for x in idx[:8]]}
         print(json.dumps(line), flush=True)

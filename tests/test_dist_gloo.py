@@ -155,6 +155,96 @@ def test_sharded_literal_column_norm_exchange_two_ranks():
     check_ted(np.array(lit[0][1]), np.array(lit[0][2]), tr, "gloo-shard-literal")
 
 
+class NumpyIShard:
+    """Test-only tile-shard backend of ShardedImplicitTed, fp64 numpy: this rank
+    owns the entries (i, j) of the 128 x 128 tiles (min(I,J), max(I,J)) whose
+    row-major upper-triangle index is rank (mod P); everything else (the factor
+    L, running norms n_v and diagonal r_vv) is replicated, as in libbted."""
+
+    T = 128
+
+    def __init__(self, X, gamma, rank, nranks):
+        X = X.astype(np.float64)
+        self.N = X.shape[0]
+        d2 = ((X[:, None, :] - X[None, :, :]) ** 2).sum(-1)
+        K = np.exp(-gamma * d2)
+        nT = -(-self.N // self.T)
+        blk = np.arange(self.N) // self.T
+        lo, hi = np.minimum.outer(blk, blk), np.maximum.outer(blk, blk)
+        toff = lo * nT - lo * (lo - 1) // 2 + (hi - lo)           # tile index of entry (i, j)
+        self.Kown = np.where(toff % nranks == rank, K, 0.0)      # this rank's share of K
+        self.diag = np.diag(K).copy()
+        self.qlen = self.N
+
+    def _put_key(self, t, keys):
+        score = np.maximum(self.n, 0.0) / (self.r + self.mu)              # as libbted's fin64
+        best = 0
+        for i in range(self.N):
+            if not self.sel[i]:
+                best = max(best, pack(score[i], i))
+        keys[t] = best
+
+    def head(self, m, mu, q):
+        self.mu, self.L = mu, []
+        self.sel = np.zeros(self.N, bool)
+        q.zero_()
+        q[: self.N] = torch.from_numpy((self.Kown * self.Kown).sum(1))       # own part of ||K_:v||^2
+
+    def fin(self, t, mu, q, keys):
+        qv = q[: self.N].numpy().astype(np.float64)
+        if t == 0:
+            self.n, self.r = qv.copy(), self.diag.copy()
+        else:
+            l = self.L[-1]
+            Lp = np.array(self.L[:-1]).T if len(self.L) > 1 else np.zeros((self.N, 0))
+            Rl = qv - Lp @ (Lp.T @ l)                              # (R l)_v = (K l)_v - L (L^T l)
+            self.n = self.n - 2 * l * Rl + l * l * (l @ l)
+            self.r = self.r - l * l
+        self._put_key(t, keys)
+
+    def step(self, t, mu, keys, q):
+        s = unpack_idx(int(keys[t - 1]))
+        self.sel[s] = True
+        Kcol = self.Kfull_col(s)
+        Lm = np.array(self.L).T if self.L else np.zeros((self.N, 0))
+        l = (Kcol - Lm @ Lm[s]) / np.sqrt(self.r[s] + mu)
+        self.L.append(l)
+        q.zero_()
+        q[: self.N] = torch.from_numpy(self.Kown @ l)                      # own part of K l (mask symmetric)
+
+    def Kfull_col(self, s):
+        return self._K[:, s]
+
+    def check(self):
+        pass
+
+
+def _ishard_worker(rank, world, port, X, gamma, m, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_date_sunbg021_b200.dist import ShardedImplicitTed, TorchComm
+    be = NumpyIShard(X, gamma, rank, world)
+    Xd = X.astype(np.float64)
+    be._K = np.exp(-gamma * ((Xd[:, None, :] - Xd[None, :, :]) ** 2).sum(-1))   # column s (replicated X)
+    st = ShardedImplicitTed(be, X.shape[0], TorchComm(), torch.device("cpu"))
+    idx, score = st.select(m, MU)
+    q.put((rank, idx.tolist(), score.tolist()))
+    dist.destroy_process_group()
+
+
+def test_tile_sharded_implicit_protocol_two_ranks():
+    """ShardedImplicitTed: one all-reduce(SUM) of the partial q per step; every
+    rank decodes the same picks, equal to one rank's and to the oracle's."""
+    _, X = make_pool(KnobSpace(WORKLOADS["resnet18_layer1"], 16), 300, 14)   # 3 blocks of 128: 6 tiles
+    g = median_gamma(X, 14)
+    m = 12
+    two = _run(2, _ishard_worker, X, g, m)
+    one = _run(1, _ishard_worker, X, g, m)
+    assert two[0][1] == two[1][1] == one[0][1]
+    tr = literal.ted(X, g, MU, m, forced=two[0][1])
+    check_ted(np.array(two[0][1]), np.array(two[0][2]), tr, "gloo-ishard")
+
+
 class NumpyPool:
     """Test-only batch backend: Alg. 2 l.1-4 / l.5-6 by the oracle."""
 
