@@ -251,6 +251,17 @@ bted_status bted_ishard_head(bted_ctx* shard, int32_t m, float mu, double* q_dev
 bted_status bted_ishard_step(bted_ctx* shard, int32_t t, float mu, const uint64_t* keys_dev, double* q_dev);
 bted_status bted_ishard_fin(bted_ctx* shard, int32_t t, float mu, const double* q_dev, uint64_t* keys_dev);
 int64_t     bted_ishard_qlen(const bted_ctx* shard);
+/* K4 near-tie refinement for the tile-sharded engine (as on one GPU, DESIGN.md
+ * "K4"): after the m-step loop, every step whose second-best fp32 score lies
+ * within 2e-5 of the best is re-scored exactly in fp64 from the (replicated)
+ * features.  *nforced = 0: the selection stands.  Otherwise forced_host[0 ..
+ * *nforced) are flagged keys (the earlier picks and the corrected one): re-run
+ * the loop with keys_dev preset to them (zeros after) and call again.  Every
+ * rank computes the same answer, so all ranks re-run together.  keys_dev:
+ * device u64 [m] of the finished loop; forced_host: host u64 [m].
+ * Errors: EINVAL, ECUDA, ESTATE. */
+bted_status bted_ishard_refine(bted_ctx* shard, int32_t m, float mu, const uint64_t* keys_dev,
+                               uint64_t* forced_host, int32_t* nforced);
 /* Leading dimension (floats) a pivot buffer must have: pivot_dev[N..ld) must be 0. */
 int64_t     bted_shard_ld(const bted_ctx* shard);
 /* Sticky device error flag of the shard (BTED_ENUMERIC if a NaN score was seen). */

@@ -75,6 +75,7 @@ _SIGS = {
     "bted_ishard_step": (ctypes.c_int, [_vp, _i32, _f32, _vp, _vp]),
     "bted_ishard_fin": (ctypes.c_int, [_vp, _i32, _f32, _vp, _vp]),
     "bted_ishard_qlen": (_i64, [_vp]),
+    "bted_ishard_refine": (ctypes.c_int, [_vp, _i32, _f32, _vp, _vp, ctypes.POINTER(_i32)]),
     "bted_shard_check": (ctypes.c_int, [_vp]),
     "bted_destroy": (None, [_vp]),
     "bted_status_string": (ctypes.c_char_p, [ctypes.c_int]),
@@ -204,6 +205,14 @@ def bted_ishard_fin(ctx: int, t: int, mu: float, q_dev: int, keys_dev: int):
     check(lib().bted_ishard_fin(ctx, int(t), float(mu), q_dev, keys_dev))
 
 
+def bted_ishard_refine(ctx: int, m: int, mu: float, keys_dev: int) -> np.ndarray:
+    """K4 for the tile-sharded engine: [] if the selection stands, else the keys to preset (u64)."""
+    forced = np.zeros(int(m), dtype=np.uint64)
+    n = _i32(0)
+    check(lib().bted_ishard_refine(ctx, int(m), float(mu), keys_dev, _ptr(forced), ctypes.byref(n)))
+    return forced[: n.value]
+
+
 def bted_ishard_qlen(ctx: int) -> int:
     return int(lib().bted_ishard_qlen(ctx))
 
@@ -300,7 +309,7 @@ def bted_reset_stats(ctx: int):
 
 def decode_keys(keys: np.ndarray):
     """Packed keys (u64) -> (index, fp32 score).  See include/bted.h."""
-    keys = np.asarray(keys, dtype=np.uint64)
+    keys = np.asarray(keys, dtype=np.uint64) & np.uint64(0x7FFFFFFFFFFFFFFF)   # K4's forced-pick flag
     idx = (np.uint64(0xFFFFFFFF) - (keys & np.uint64(0xFFFFFFFF))).astype(np.int64)
     bits = ((keys >> np.uint64(32)) - np.uint64(1)).astype(np.uint32)
     return idx, bits.view(np.float32)

@@ -1623,8 +1623,53 @@ bted_status bted_ishard_fin(bted_ctx* ctx, int32_t t, float mu, const double* q_
         auto* keys = reinterpret_cast<unsigned long long*>(keys_dev);
         bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
             T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, NPa, t > 0 ? t - 1 : 0, T.hv, T.nv, T.rd, T.sel, keys, t,
-            keys + t, T.err, nullptr, T.Qc, q_dev, t == 0 ? T.rd : nullptr);
+            keys + t, T.err, T.refine ? T.top2 : nullptr, T.Qc, q_dev, t == 0 ? T.rd : nullptr);
         LAUNCHED(1);
+        return BTED_OK;
+    });
+}
+
+bted_status bted_ishard_refine(bted_ctx* ctx, int32_t m, float mu, const uint64_t* keys_dev, uint64_t* forced_host,
+                               int32_t* nforced) {
+    if (!ctx || !keys_dev || !forced_host || !nforced || !ctx->is_ishard || m < 1 || m != ctx->sm_m || !mu_ok(mu)) {
+        set_error("bad ishard_refine arguments"); return BTED_EINVAL;
+    }
+    *nforced = 0;
+    return guarded(ctx, [&]() -> bted_status {
+        Ted& T = ctx->ted;
+        if (!T.refine) return BTED_OK;
+        cudaStream_t st = T.stream;
+        const auto* keys = reinterpret_cast<const unsigned long long*>(keys_dev);
+        CK(cudaMemsetAsync(T.nflag, 0, sizeof(int), st));
+        bted::rf::neartie_check_kernel<<<m, 256, 0, st>>>(T.top2, T.last_nC, keys, bted::rf::kTau, T.flags, T.cand,
+                                                         T.ncand, T.nflag);
+        LAUNCHED(1);
+        std::vector<unsigned long long> hk(m);
+        std::vector<int> fl(m), nc(m);
+        std::vector<uint32_t> cd((size_t)m * bted::rf::kMaxCand);
+        CK(cudaMemcpyAsync(hk.data(), keys, sizeof(unsigned long long) * m, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(fl.data(), T.flags, sizeof(int) * m, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(nc.data(), T.ncand, sizeof(int) * m, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(cd.data(), T.cand, sizeof(uint32_t) * cd.size(), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        for (int ts = 0; ts < m; ++ts) {
+            if (!fl[ts] || nc[ts] < 2) continue;
+            std::vector<uint32_t> S(ts), C;
+            for (int k = 0; k < ts; ++k) S[k] = 0xFFFFFFFFu - (uint32_t)(hk[k] & 0xFFFFFFFFull);
+            for (int c = 0; c < nc[ts]; ++c) C.push_back(cd[(size_t)ts * bted::rf::kMaxCand + c]);
+            std::sort(C.begin(), C.end());
+            uint32_t best = 0;
+            double bs = 0.0;
+            refine_step(ctx, st, ctx->X, ctx->N, ctx->d, S, C, mu, &best, &bs);
+            ctx->refined_steps++;
+            const uint32_t pick = 0xFFFFFFFFu - (uint32_t)(hk[ts] & 0xFFFFFFFFull);
+            if (best == pick) continue;
+            ctx->corrected_steps++;
+            for (int k = 0; k < ts; ++k) forced_host[k] = hk[k] | bted::rf::kForced;
+            forced_host[ts] = host_pack_key((float)bs, best) | bted::rf::kForced;
+            *nforced = ts + 1;
+            break;
+        }
         return BTED_OK;
     });
 }

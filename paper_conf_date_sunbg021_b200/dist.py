@@ -241,6 +241,9 @@ class LibIShard:
     def fin(self, t, mu, q: torch.Tensor, keys: torch.Tensor):
         L.bted_ishard_fin(self.ctx, t, mu, q.data_ptr(), keys.data_ptr())
 
+    def refine(self, m, mu, keys: torch.Tensor):
+        return L.bted_ishard_refine(self.ctx, m, mu, keys.data_ptr())
+
     def check(self):
         L.bted_shard_check(self.ctx)
 
@@ -266,8 +269,10 @@ class ShardedImplicitTed:
         with _stream_ctx(stream):
             self.q = torch.zeros(backend.qlen, dtype=torch.float64, device=device)
 
-    def _loop(self, keys: torch.Tensor, m: int, mu: float):
+    def _loop(self, keys: torch.Tensor, m: int, mu: float, preset=None):
         keys.zero_()
+        if preset is not None:                       # K4: forced picks (flagged keys win every max)
+            keys[: len(preset)].copy_(torch.from_numpy(preset.view(np.int64)))
         self.be.head(m, mu, self.q)                  # l.1 + this rank's part of ||K_:v||^2
         self.comm.allreduce_sum_(self.q)
         self.be.fin(0, mu, self.q, keys)             # l.3: s_1 (identical on every rank)
@@ -294,13 +299,21 @@ class ShardedImplicitTed:
             else:
                 keys = torch.zeros(m, dtype=torch.int64, device=self.device)
                 self._loop(keys, m, mu)
+            # K4: re-score near ties exactly; a changed pick re-runs the loop with the prefix forced
+            # (identical decision on every rank, so the collectives stay matched)
+            for _ in range(m):
+                forced = self.be.refine(m, mu, keys) if hasattr(self.be, "refine") else []
+                if len(forced) == 0:
+                    break
+                keys = torch.zeros(m, dtype=torch.int64, device=self.device)
+                self._loop(keys, m, mu, preset=forced)
             host = keys.cpu().numpy().view(np.uint64)
         self.be.check()
         return L.decode_keys(host)
 
 
 def isharded_select_loopback(X: np.ndarray, gamma: float, P: int, m: int, mu: float, device: torch.device,
-                             stream: torch.cuda.Stream, kernel: int = L.BTED_KERNEL_RBF):
+                             stream: torch.cuda.Stream, kernel: int = L.BTED_KERNEL_RBF, stats: dict | None = None):
     """ShardedImplicitTed with P logical tile shards on ONE GPU; the all-reduce
     is a sum of the shards' partial q in rank order."""
     N, d = X.shape
@@ -318,21 +331,35 @@ def isharded_select_loopback(X: np.ndarray, gamma: float, P: int, m: int, mu: fl
                     tot += qs[r]
                 qs.copy_(tot.expand_as(qs))
 
-            for r in range(P):
-                shards[r].head(m, mu, qs[r])
-            allreduce()
-            for r in range(P):
-                shards[r].fin(0, mu, qs[r], keys[r])
-            for t in range(1, m):
+            def loop(preset=None):
+                keys.zero_()
+                if preset is not None:
+                    keys[:, : len(preset)] = torch.from_numpy(preset.view(np.int64)).to(device)
                 for r in range(P):
-                    shards[r].step(t, mu, keys[r], qs[r])
+                    shards[r].head(m, mu, qs[r])
                 allreduce()
                 for r in range(P):
-                    shards[r].fin(t, mu, qs[r], keys[r])
+                    shards[r].fin(0, mu, qs[r], keys[r])
+                for t in range(1, m):
+                    for r in range(P):
+                        shards[r].step(t, mu, keys[r], qs[r])
+                    allreduce()
+                    for r in range(P):
+                        shards[r].fin(t, mu, qs[r], keys[r])
+
+            loop()
+            for _ in range(m):                                   # K4, as ShardedImplicitTed.select
+                forced = [shards[r].refine(m, mu, keys[r]) for r in range(P)]
+                assert all(np.array_equal(f, forced[0]) for f in forced), "shards disagree on K4"
+                if len(forced[0]) == 0:
+                    break
+                loop(forced[0])
             host = keys.cpu().numpy().view(np.uint64)
         for s in shards:
             s.check()
         assert all((host[r] == host[0]).all() for r in range(P)), "shards disagree"
+        if stats is not None:
+            stats.update(L.bted_get_stats(shards[0].ctx))
         return L.decode_keys(host[0])
     finally:
         for s in shards:

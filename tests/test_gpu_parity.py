@@ -355,6 +355,26 @@ def test_tile_sharded_implicit_loopback_vs_oracle(N, P, d):
     np.testing.assert_allclose(sc[:k], s1[:k], rtol=1e-5)
 
 
+@pytest.mark.parametrize("P", [2, 3])
+def test_tile_sharded_implicit_k4_exact_ties(P):
+    """Exact duplicates: the shards' q sums are not bitwise equal for the two
+    copies, so the fp32 order of tied scores is rounding; K4 (bted_ishard_refine,
+    fp64 from the replicated features) must still give the lowest index and
+    P2 at the fp64 gap GAP_K4."""
+    import torch
+    from paper_conf_date_sunbg021_b200.dist import isharded_select_loopback
+    X = knob(2500, seed=43)
+    X = np.concatenate([X, X[::5]], axis=0)                  # 500 exact duplicate pairs
+    g = median_gamma(X, 43)
+    dev = torch.device("cuda", 0)
+    st = torch.cuda.Stream(dev)
+    st_k4 = {}
+    idx, sc = isharded_select_loopback(X, g, P, 64, MU, dev, st, stats=st_k4)
+    assert st_k4["refined_steps"] > 0                        # the tied steps went through K4
+    check_ted(idx, sc, dense.ted(X, g, MU, 64, forced=idx), f"ishard-k4 P={P}", gap_exact=GAP_K4)
+    print(f"ishard K4 P={P}: refined {st_k4['refined_steps']}, corrected {st_k4['corrected_steps']}")
+
+
 def test_launch_counter_counts_kernels():
     X = knob(300)
     before = bt.bted_kernel_launches()
