@@ -19,6 +19,7 @@
 #include <cstdlib>
 #include <cstdio>
 #include <list>
+#include <mutex>
 #include <new>
 #include <string>
 #include <vector>
@@ -57,6 +58,20 @@ struct CudaError {
         if (_e != cudaSuccess) throw CudaError{_e, #expr};               \
     } while (0)
 #define LAUNCHED(n) g_launches.fetch_add((n), std::memory_order_relaxed)
+
+// Kernel attributes (dynamic smem limits, carveouts) are per device: run f once
+// per (call site, current device), thread-safe.
+template <class F>
+void once_per_device(uint64_t& mask, F&& f) {
+    static std::mutex mu;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const uint64_t bit = 1ull << (dev & 63);
+    std::lock_guard<std::mutex> lk(mu);
+    if (mask & bit) return;
+    f();
+    mask |= bit;
+}
 
 constexpr int kK1Rows = 16, kK1Threads = 256;
 constexpr int kK2Rows = 1, kK2Unroll = 4, kK2Threads = 256;
@@ -407,8 +422,8 @@ int l2_keep_tiles(int64_t tiles) {
 }
 // head: K1p (the packed Gram, read-only from now on), fp64 norm pass, scores.  (3 kernels)
 void ensure_implicit_attrs() {
-    static bool done = false;
-    if (!done) {
+    static uint64_t done = 0;
+    once_per_device(done, [] {
         CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)bted::im::tile_pass_smem_bytes));
         CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -422,8 +437,7 @@ void ensure_implicit_attrs() {
                                 (int)bted::im::tile_pass_smem_bytes));
         CK(cudaFuncSetAttribute(bted::im::ted_loop_kernel, cudaFuncAttributePreferredSharedMemoryCarveout,
                                 (int)cudaSharedmemCarveoutMaxShared));
-        done = true;
-    }
+    });
 }
 
 void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m,
@@ -605,12 +619,11 @@ void graph_run(Ted& T, const GraphKey& key, uint64_t nkernels, F&& enqueue) {
 
 // Run one TED (graph-cached unless no_graph); results stay on the device.
 void ensure_packed_attrs() {
-    static bool done = false;
-    if (!done) {
+    static uint64_t done = 0;
+    once_per_device(done, [] {
         CK(cudaFuncSetAttribute(K2P_TMA_KERNEL, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)kK2pSmem));
-        done = true;
-    }
+    });
 }
 
 // packed layout unless the caller asks for dense or d is too wide for K1p
@@ -1090,14 +1103,13 @@ bool use_small(uint32_t flags, int64_t N) { return !(flags & BTED_FLAG_NO_SMALL)
 template <int C>
 void launch_small_c(const float* X, int ninst, int32_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
                     unsigned long long* keys, int* err, cudaStream_t st) {
-    static bool attr = false;
-    if (!attr) {
+    static uint64_t attr = 0;
+    once_per_device(attr, [] {
         CK(cudaFuncSetAttribute(bted::sm::ted_cluster_kernel<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)bted::sm::kSmemBudget));
         if (C > 8) CK(cudaFuncSetAttribute(bted::sm::ted_cluster_kernel<C>,
                                            cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
-        attr = true;
-    }
+    });
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)(ninst * C));
     cfg.blockDim = dim3(bted::sm::kThreads);
