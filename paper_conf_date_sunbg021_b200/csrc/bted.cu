@@ -454,9 +454,10 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
     auto k1i = [&](auto kern) {
         kern<<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(X, (int32_t)N, d, gamma, T.K[0], nT, 0, 1);
     };
-    // two rows per warp step at 3 CTAs/SM measured 369 us vs 388 (four rows, 2 CTAs/SM) and 412 (K1p)
+    // d <= 16: two columns per lane, four rows at once, 4 CTAs/SM: 243 us at N = 16384 (B200,
+    // warm ncu) vs 371 us for gram_tile_kernel<16,·,2> and 412 us for K1p
     if (d <= 16) {
-        if (lin) k1i(bted::pk::gram_tile_kernel<16, true, 2>); else k1i(bted::pk::gram_tile_kernel<16, false, 2>);
+        if (lin) k1i(bted::pk::gram_tile2_kernel<16, true, 4>); else k1i(bted::pk::gram_tile2_kernel<16, false, 4>);
     } else {
         if (lin) k1i(bted::pk::gram_tile_kernel<32, true>); else k1i(bted::pk::gram_tile_kernel<32, false>);
     }
@@ -1584,7 +1585,7 @@ bted_status bted_ishard_head(bted_ctx* ctx, int32_t m, float mu, double* q_dev) 
             kern<<<(unsigned)lt, bted::pk::kConsumers, 0, T.stream>>>(ctx->X, (int32_t)N, ctx->d, g, T.K[0], nT, r, P);
         };
         if (ctx->d <= 16) {
-            if (lin) k1i(bted::pk::gram_tile_kernel<16, true, 2>); else k1i(bted::pk::gram_tile_kernel<16, false, 2>);
+            if (lin) k1i(bted::pk::gram_tile2_kernel<16, true, 4>); else k1i(bted::pk::gram_tile2_kernel<16, false, 4>);
         } else {
             if (lin) k1i(bted::pk::gram_tile_kernel<32, true>); else k1i(bted::pk::gram_tile_kernel<32, false>);
         }

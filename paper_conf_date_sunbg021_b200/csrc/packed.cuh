@@ -734,6 +734,74 @@ gram_tile_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma,
     }
 }
 
+// K1i variant with two columns per lane: warps 2v and 2v+1 cover rows
+// 32v .. 32v+31, lane l of warp w the columns 64 (w & 1) + 2l, +1; kH rows
+// at once.  Half the column-feature registers of
+// gram_tile_kernel (no spills at 4 CTAs/SM), 2 kH independent FFMA2 chains
+// per lane, coalesced float2 stores (256 B per warp and row).  Bitwise the
+// same values (same operand pairs, same feature order, same expf).
+template <int kD, bool kLinear, int kH>
+__global__ void __launch_bounds__(kConsumers, 4)
+gram_tile2_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma, float* __restrict__ K, int nT,
+                  int sr = 0, int sp = 1) {
+    __shared__ __align__(16) unsigned long long xi2[T][kD];     // (x, x) pairs of the tile's rows
+    __shared__ __align__(16) float xj[T][kD + 1];
+    const int tid = threadIdx.x, w = tid / kWarp, l = tid % kWarp;
+    const float ng = -gamma;
+    int I, J;
+    tile_ij((int64_t)sr + (int64_t)sp * blockIdx.x, nT, I, J);
+    for (int q = tid; q < T * kD; q += kConsumers) {
+        const int r = q / kD, c = q % kD;
+        const int gi = I * T + r, gj = J * T + r;
+        const float xv = (gi < N && c < d) ? X[(int64_t)gi * d + c] : 0.f;
+        xi2[r][c] = pack2(xv, xv);
+        xj[r][c] = (gj < N && c < d) ? X[(int64_t)gj * d + c] : 0.f;
+    }
+    __syncthreads();
+    const int c0 = 64 * (w & 1) + 2 * l;                         // this lane's two columns
+    unsigned long long y[kD];
+#pragma unroll
+    for (int q = 0; q < kD; ++q) y[q] = pack2(xj[c0][q], xj[c0 + 1][q]);
+    float* tile = K + (int64_t)blockIdx.x * (T * T);
+    const bool cv0 = J * T + c0 < N, cv1 = J * T + c0 + 1 < N;
+    const int rbase = 32 * (w >> 1);                             // warps 2v, 2v+1: rows 32v .. 32v+31
+#pragma unroll 1
+    for (int rr = 0; rr < 32; rr += kH) {
+        const int r = rbase + rr;
+        unsigned long long a[kH];
+#pragma unroll
+        for (int h = 0; h < kH; ++h) a[h] = 0ull;
+#pragma unroll
+        for (int q = 0; q < kD; q += 2) {
+#pragma unroll
+            for (int h = 0; h < kH; ++h) {
+                const ulonglong2 xx = *reinterpret_cast<const ulonglong2*>(&xi2[r + h][q]);
+                if (kLinear) {
+                    a[h] = fma2(xx.x, y[q], a[h]);
+                    a[h] = fma2(xx.y, y[q + 1], a[h]);
+                } else {
+                    unsigned long long dd = sub2(xx.x, y[q]);
+                    a[h] = fma2(dd, dd, a[h]);
+                    dd = sub2(xx.y, y[q + 1]);
+                    a[h] = fma2(dd, dd, a[h]);
+                }
+            }
+        }
+#pragma unroll
+        for (int h = 0; h < kH; ++h) {
+            float a0, a1;
+            unpack2(a[h], a0, a1);
+            const bool rv = I * T + r + h < N;
+            const float v0 = kLinear ? a0 : expf(__fmul_rn(ng, a0));
+            const float v1 = kLinear ? a1 : expf(__fmul_rn(ng, a1));
+            float2 o;
+            o.x = (rv && cv0) ? v0 : 0.f;
+            o.y = (rv && cv1) ? v1 : 0.f;
+            __stcs(reinterpret_cast<float2*>(tile + (r + h) * T + c0), o);
+        }
+    }
+}
+
 // ------------------------------------------------------------------ K2p (LDG variant)
 // One CTA (256 threads) per tile, non-persistent (the hardware scheduler
 // balances 8256+ tiles over the SMs; several CTAs per SM keep many 256-bit
