@@ -753,6 +753,13 @@ struct bted_ctx {
     double* rout = nullptr; size_t routcap = 0;
     uint32_t* ridx = nullptr; size_t ridxcap = 0;
     uint64_t refined_steps = 0, corrected_steps = 0;
+    // K4 for the cluster-kernel TEDs: per-instance top-2 keys, flags, candidates, counts, forced picks
+    unsigned long long* ktop2 = nullptr; size_t ktop2cap = 0;
+    int* kflags = nullptr; size_t kflagscap = 0;
+    uint32_t* kcand = nullptr; size_t kcandcap = 0;
+    int* kncand = nullptr; size_t kncandcap = 0;
+    int* knflag = nullptr; size_t knflagcap = 0;
+    unsigned long long* kforced = nullptr; size_t kforcedcap = 0;
     float* xall = nullptr; size_t xallcap = 0;             // [nb][M][d] gathered batches
     unsigned long long* kall = nullptr; size_t kallcap = 0; // [nb][m] keys
     // host staging (pinned)
@@ -1025,8 +1032,11 @@ void refine_step(bted_ctx* ctx, cudaStream_t st, const float* X, int64_t N, int3
     const int lin = ctx->kernel == BTED_KERNEL_LINEAR ? 1 : 0;
     bted::rf::refine_cols_kernel<<<dim3((unsigned)((N + 255) / 256), (unsigned)ncol), 256, 0, st>>>(
         X, (int32_t)N, d, (double)ctx->params.gamma, lin, ctx->rcols, ctx->rG);
-    bted::rf::refine_solve_kernel<<<1, 256, 0, st>>>(ctx->rG, (int32_t)N, ctx->rcols, t, nc, (double)mu, ctx->rA,
-                                                    ctx->rW);
+    const size_t asmem = sizeof(double) * (size_t)t * (size_t)t;
+    const bool a_in_smem = asmem <= 48 * 1024;
+    bted::rf::refine_solve_kernel<<<1, 256, a_in_smem ? asmem : 0, st>>>(ctx->rG, (int32_t)N, ctx->rcols, t, nc,
+                                                                        (double)mu, ctx->rA, ctx->rW,
+                                                                        a_in_smem ? 1 : 0);
     bted::rf::refine_resid_kernel<<<nblk, 256, 0, st>>>(ctx->rG, (int32_t)N, ctx->rcols, t, nc, ctx->rW, ctx->rpart,
                                                        ctx->rdiag);
     bted::rf::refine_pick_kernel<<<1, 32, 0, st>>>(ctx->rpart, nblk, ctx->rdiag, ctx->rcols, t, nc, (double)mu,
@@ -1103,7 +1113,8 @@ bool use_small(uint32_t flags, int64_t N) { return !(flags & BTED_FLAG_NO_SMALL)
 
 template <int C>
 void launch_small_c(const float* X, int ninst, int32_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
-                    unsigned long long* keys, int* err, cudaStream_t st) {
+                    unsigned long long* keys, int* err, cudaStream_t st, unsigned long long* top2,
+                    const unsigned long long* forced, int nforced) {
     static uint64_t attr = 0;
     once_per_device(attr, [] {
         CK(cudaFuncSetAttribute(bted::sm::ted_cluster_kernel<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1125,27 +1136,121 @@ void launch_small_c(const float* X, int ninst, int32_t N, int32_t d, float gamma
     cfg.attrs = at;
     cfg.numAttrs = 1;
     CK(cudaLaunchKernelEx(&cfg, bted::sm::ted_cluster_kernel<C>, X, N, d, gamma,
-                          (int32_t)(kernel == BTED_KERNEL_LINEAR ? 1 : 0), m, mu, keys, err, (int32_t)stage_x));
+                          (int32_t)(kernel == BTED_KERNEL_LINEAR ? 1 : 0), m, mu, keys, err, (int32_t)stage_x,
+                          top2, forced, (int32_t)nforced));
     LAUNCHED(1);
 }
 
 // ninst independent TEDs on X[inst][N][d] -> keys[inst][m]; err = a Ted's flag
-void launch_small(const float* X, int ninst, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
-                  unsigned long long* keys, int* err, cudaStream_t st) {
-    // the smallest cluster whose CTAs also hold the staged features, if the
-    // ninst clusters still fit on the SMs at once; else the smallest that fits
+// the cluster size launch_small uses for ninst TEDs of N points (K4 sizes its top-2 buffer by it)
+int small_cluster_used(int ninst, int64_t N, int32_t d) {
     int C = small_cluster_for(N);
     for (int c2 = C; c2 > 0 && c2 <= 16; c2 *= 2) {
         if ((int64_t)ninst * c2 > num_sms()) break;
         if (bted::sm::smem_core((int)N, c2) + bted::sm::smem_x((int)N, d) <= bted::sm::kSmemBudget) { C = c2; break; }
     }
+    return C;
+}
+
+void launch_small(const float* X, int ninst, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
+                  unsigned long long* keys, int* err, cudaStream_t st, unsigned long long* top2 = nullptr,
+                  const unsigned long long* forced = nullptr, int nforced = 0) {
+    // the smallest cluster whose CTAs also hold the staged features, if the
+    // ninst clusters still fit on the SMs at once; else the smallest that fits
+    const int C = small_cluster_used(ninst, N, d);
     switch (C) {
-        case 1: launch_small_c<1>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st); break;
-        case 2: launch_small_c<2>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st); break;
-        case 4: launch_small_c<4>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st); break;
-        case 8: launch_small_c<8>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st); break;
-        case 16: launch_small_c<16>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st); break;
+        case 1: launch_small_c<1>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st, top2, forced, nforced); break;
+        case 2: launch_small_c<2>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st, top2, forced, nforced); break;
+        case 4: launch_small_c<4>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st, top2, forced, nforced); break;
+        case 8: launch_small_c<8>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st, top2, forced, nforced); break;
+        case 16: launch_small_c<16>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st, top2, forced, nforced); break;
         default: throw CudaError{cudaErrorInvalidValue, "launch_small: N too large"};
+    }
+}
+
+// ---- K4 for cluster-kernel TEDs (merges, small batches, small bted_select) ----
+// Buffers for ninst instances of m steps; returns the top-2 buffer to pass to launch_small.
+unsigned long long* small_k4_reserve(bted_ctx* ctx, int ninst, int64_t N, int32_t d, int32_t m) {
+    const int nU = small_cluster_used(ninst, N, d) * bted::sm::kWarps;
+    const int nU1 = small_cluster_used(1, N, d) * bted::sm::kWarps;       // single-instance re-runs
+    grow(ctx->ktop2, ctx->ktop2cap, (size_t)ninst * m * nU * 2 + (size_t)m * nU1 * 2);   // + re-run scratch
+    grow(ctx->kflags, ctx->kflagscap, (size_t)ninst * m);
+    grow(ctx->kcand, ctx->kcandcap, (size_t)ninst * m * bted::rf::kMaxCand);
+    grow(ctx->kncand, ctx->kncandcap, (size_t)ninst * m);
+    grow(ctx->knflag, ctx->knflagcap, (size_t)ninst);
+    grow(ctx->kforced, ctx->kforcedcap, (size_t)m);
+    return ctx->ktop2;
+}
+
+// After launch_small(..., top2 = ctx->ktop2): flag near ties of every instance
+// (one check launch each, one host sync), then re-score the flagged steps of the
+// flagged instances exactly in fp64; a changed pick re-runs that instance with
+// the corrected prefix forced.  X: ninst x N x d (device); keys: ninst x m.
+void small_k4(bted_ctx* ctx, cudaStream_t st, const float* X, int ninst, int64_t N, int32_t d, int32_t m, float mu,
+              unsigned long long* keys, int* err) {
+    const int nUb = small_cluster_used(ninst, N, d) * bted::sm::kWarps;
+    const int nU1 = small_cluster_used(1, N, d) * bted::sm::kWarps;
+    const size_t kMC = bted::rf::kMaxCand;
+    unsigned long long* rerun_top2 = ctx->ktop2 + (size_t)ninst * m * nUb * 2;
+    auto check = [&](int k, const unsigned long long* t2, int nU) {
+        bted::rf::neartie_check_kernel<<<m, 256, 0, st>>>(t2, nU, keys + (size_t)k * m,
+                                                         bted::rf::kTau, ctx->kflags + (size_t)k * m,
+                                                         ctx->kcand + (size_t)k * m * kMC, ctx->kncand + (size_t)k * m,
+                                                         ctx->knflag + k);
+        LAUNCHED(1);
+    };
+    CK(cudaMemsetAsync(ctx->knflag, 0, sizeof(int) * ninst, st));
+    bted::rf::neartie_check_kernel<<<dim3(m, ninst), 256, 0, st>>>(ctx->ktop2, nUb, keys, bted::rf::kTau,
+                                                                  ctx->kflags, ctx->kcand, ctx->kncand, ctx->knflag);
+    LAUNCHED(1);
+    std::vector<int> nf(ninst);
+    CK(cudaMemcpyAsync(nf.data(), ctx->knflag, sizeof(int) * ninst, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    std::vector<unsigned long long> hk(m);
+    std::vector<int> fl(m), nc(m);
+    std::vector<uint32_t> cd((size_t)m * kMC);
+    for (int k = 0; k < ninst; ++k) {
+        if (!nf[k]) continue;
+        const float* Xk = X + (size_t)k * N * d;
+        unsigned long long* kk = keys + (size_t)k * m;
+        int checked = -1;
+        for (int rounds = 0; rounds <= m; ++rounds) {
+            CK(cudaMemcpyAsync(hk.data(), kk, sizeof(unsigned long long) * m, cudaMemcpyDeviceToHost, st));
+            CK(cudaMemcpyAsync(fl.data(), ctx->kflags + (size_t)k * m, sizeof(int) * m, cudaMemcpyDeviceToHost, st));
+            CK(cudaMemcpyAsync(nc.data(), ctx->kncand + (size_t)k * m, sizeof(int) * m, cudaMemcpyDeviceToHost, st));
+            CK(cudaMemcpyAsync(cd.data(), ctx->kcand + (size_t)k * m * kMC, sizeof(uint32_t) * cd.size(),
+                               cudaMemcpyDeviceToHost, st));
+            CK(cudaStreamSynchronize(st));
+            bool rerun = false;
+            for (int ts = checked + 1; ts < m && !rerun; ++ts) {
+                if (!fl[ts] || nc[ts] < 2) continue;
+                std::vector<uint32_t> S(ts), Cs;
+                for (int q = 0; q < ts; ++q) S[q] = 0xFFFFFFFFu - (uint32_t)(hk[q] & 0xFFFFFFFFull);
+                for (int c = 0; c < nc[ts]; ++c) Cs.push_back(cd[(size_t)ts * kMC + c]);
+                std::sort(Cs.begin(), Cs.end());
+                uint32_t best = 0;
+                double bs = 0.0;
+                refine_step(ctx, st, Xk, N, d, S, Cs, mu, &best, &bs);
+                ctx->refined_steps++;
+                checked = ts;
+                const uint32_t pick = 0xFFFFFFFFu - (uint32_t)(hk[ts] & 0xFFFFFFFFull);
+                if (best == pick) continue;
+                ctx->corrected_steps++;
+                std::vector<unsigned long long> forced(ts + 1);
+                for (int q = 0; q < ts; ++q) forced[q] = hk[q] | bted::rf::kForced;
+                forced[ts] = host_pack_key((float)bs, best) | bted::rf::kForced;
+                CK(cudaMemcpyAsync(ctx->kforced, forced.data(), sizeof(unsigned long long) * (ts + 1),
+                                   cudaMemcpyHostToDevice, st));
+                // the single-instance re-run writes its top-2 to the scratch tail
+                launch_small(Xk, 1, N, d, ctx->params.gamma, ctx->kernel, m, mu, kk, err, st, rerun_top2,
+                             ctx->kforced, ts + 1);
+                CK(cudaMemsetAsync(ctx->knflag + k, 0, sizeof(int), st));
+                check(k, rerun_top2, nU1);
+                CK(cudaStreamSynchronize(st));      // `forced` (pageable) must outlive the copy
+                rerun = true;
+            }
+            if (!rerun) break;
+        }
     }
 }
 
@@ -1171,8 +1276,10 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
             gather(ctx, st, ctx->sall + (size_t)kk * M, M, ctx->xall + (size_t)kk * M * ctx->d);
         Ted::Slot* sl = T.timing ? T.next_slot(m) : nullptr;
         if (sl) { sl->small = nb; CK(cudaEventRecord(sl->e[0], st)); }
-        launch_small(ctx->xall, nb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->kall, T.err, st);
+        unsigned long long* k4t = T.refine ? small_k4_reserve(ctx, nb, M, ctx->d, m) : nullptr;
+        launch_small(ctx->xall, nb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->kall, T.err, st, k4t);
         if (sl) CK(cudaEventRecord(sl->e[1], st));
+        if (k4t) small_k4(ctx, st, ctx->xall, nb, M, ctx->d, m, mu, ctx->kall, T.err);
         for (int kk = 0; kk < nb; ++kk) {
             bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->kall + (size_t)kk * m, m,
                                                                      ctx->sall + (size_t)kk * M,
@@ -1264,7 +1371,9 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
         // the merge is small (|X_U| <= B m): one cluster kernel runs all its steps
         Ted& T = ctx->bted_engine;
         if (!T.err) { grow(T.err, T.errcap, 1); CK(cudaMemsetAsync(T.err, 0, sizeof(int), st)); }
-        launch_small(ctx->Xb, 1, nu, ctx->d, ctx->params.gamma, ctx->kernel, mm, mu, ctx->mkeys, T.err, st);
+        unsigned long long* k4t = T.refine ? small_k4_reserve(ctx, 1, nu, ctx->d, mm) : nullptr;
+        launch_small(ctx->Xb, 1, nu, ctx->d, ctx->params.gamma, ctx->kernel, mm, mu, ctx->mkeys, T.err, st, k4t);
+        if (k4t) small_k4(ctx, st, ctx->Xb, 1, nu, ctx->d, mm, mu, ctx->mkeys, T.err);
     } else {
         // size varies with |X_U|: run it eagerly
         run_ted(ctx->bted_engine, ctx->Xb, nu, ctx->d, ctx->params.gamma, ctx->kernel, mm, mu, ctx->mkeys,
@@ -1311,8 +1420,11 @@ bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, fl
             if (!T.err) { grow(T.err, T.errcap, 1); CK(cudaMemsetAsync(T.err, 0, sizeof(int), T.stream)); }
             Ted::Slot* sl = T.timing ? T.next_slot(m) : nullptr;
             if (sl) { sl->small = 1; CK(cudaEventRecord(sl->e[0], T.stream)); }
-            launch_small(ctx->X, 1, ctx->N, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, T.keys, T.err, T.stream);
+            unsigned long long* k4t = T.refine ? small_k4_reserve(ctx, 1, ctx->N, ctx->d, m) : nullptr;
+            launch_small(ctx->X, 1, ctx->N, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, T.keys, T.err, T.stream,
+                         k4t);
             if (sl) CK(cudaEventRecord(sl->e[1], T.stream));
+            if (k4t) small_k4(ctx, T.stream, ctx->X, 1, ctx->N, ctx->d, m, mu, T.keys, T.err);
             T.last_rows = 0;                       // K lived in shared memory only
             return finish_keys(ctx, T, T.keys, m, out_idx, out_score);
         }
@@ -1767,7 +1879,8 @@ void bted_destroy(bted_ctx* ctx) {
                         ctx->u32b, ctx->count_dev, ctx->mkeys, ctx->cub_tmp, ctx->out_dev, ctx->sall,
                         ctx->xall, ctx->kall, ctx->shist, ctx->sint, ctx->scand, ctx->ssel, ctx->soff,
                         ctx->bflag, ctx->rcols, ctx->rG, ctx->rA, ctx->rW, ctx->rpart, ctx->rdiag, ctx->rout,
-                        ctx->ridx, ctx->bkeys, ctx->bsflags, ctx->bncand, ctx->bcand, ctx->sks, ctx->scnt};
+                        ctx->ridx, ctx->bkeys, ctx->bsflags, ctx->bncand, ctx->bcand, ctx->sks, ctx->scnt,
+                        ctx->ktop2, ctx->kflags, ctx->kcand, ctx->kncand, ctx->knflag, ctx->kforced};
         for (void* b : bufs) if (b) cudaFree(b);
         if (ctx->own_X && ctx->X) cudaFree(ctx->X);
         if (ctx->hkeys) cudaFreeHost(ctx->hkeys);

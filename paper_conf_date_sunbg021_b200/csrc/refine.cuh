@@ -37,6 +37,16 @@ __global__ void __launch_bounds__(256)
 neartie_check_kernel(const unsigned long long* __restrict__ top2, int nC, const unsigned long long* __restrict__ keys,
                      float tau, int* __restrict__ flags, uint32_t* __restrict__ cand, int* __restrict__ ncand,
                      int* __restrict__ nflag) {
+    // (gridDim.y > 1: one independent TED per y, m = gridDim.x steps each, arrays back to back)
+    {
+        const int64_t y = blockIdx.y, m = gridDim.x;
+        top2 += y * m * nC * 2;
+        keys += y * m;
+        flags += y * m;
+        cand += y * m * kMaxCand;
+        ncand += y * m;
+        nflag += y;
+    }
     __shared__ unsigned long long red[8];
     __shared__ int cnt;
     const int t = blockIdx.x, tid = threadIdx.x;
@@ -97,9 +107,13 @@ __global__ void refine_cols_kernel(const float* __restrict__ X, int32_t N, int32
 
 // One CTA: A = K_SS + mu I (t x t) -> Cholesky L L^T -> W[:, c] = A^-1 K_Sc for
 // the nc candidates.  cols = [S (t) | C (nc)], G from refine_cols_kernel.
+// (A lives in dynamic shared memory when the launch provides t*t doubles of it:
+// the right-looking factorisation's ~3t barriers then cost no global round trips)
 __global__ void __launch_bounds__(256)
 refine_solve_kernel(const double* __restrict__ G, int32_t N, const uint32_t* __restrict__ cols, int t, int nc,
-                    double mu, double* __restrict__ A, double* __restrict__ W) {
+                    double mu, double* __restrict__ Ag, double* __restrict__ W, int a_in_smem) {
+    extern __shared__ double As[];
+    double* A = a_in_smem ? As : Ag;
     const int tid = threadIdx.x;
     for (int e = tid; e < t * t; e += 256) {
         const int a = e / t, b = e % t;
@@ -107,9 +121,9 @@ refine_solve_kernel(const double* __restrict__ G, int32_t N, const uint32_t* __r
     }
     __syncthreads();
     for (int k = 0; k < t; ++k) {                       // right-looking Cholesky, lower triangle
-        if (tid == 0) A[k * t + k] = sqrt(A[k * t + k]);
-        __syncthreads();
-        const double dkk = A[k * t + k];
+        const double dkk = sqrt(A[k * t + k]);          // (every thread; two barriers per column)
+        __syncthreads();                                // all have read A[k][k] before it changes
+        if (tid == 0) A[k * t + k] = dkk;
         for (int i = k + 1 + tid; i < t; i += 256) A[i * t + k] /= dkk;
         __syncthreads();
         for (int e = tid; e < (t - k - 1) * (t - k - 1); e += 256) {

@@ -45,7 +45,8 @@ template <int C>
 __global__ void __launch_bounds__(kThreads, 1)
 ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float gamma, int32_t linear,
                    int32_t m, float mu, unsigned long long* __restrict__ keys_all, int* __restrict__ err,
-                   int32_t stage_x) {
+                   int32_t stage_x, unsigned long long* __restrict__ top2_all,
+                   const unsigned long long* __restrict__ forced, int32_t nforced) {
     cg::cluster_group cl = cg::this_cluster();
     const int rank = C == 1 ? 0 : (int)cl.block_rank();
     // a cluster of one CTA needs only the CTA barrier (cluster barriers also
@@ -84,6 +85,21 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
     }
     for (int q = tid; q < R; q += kThreads) sel[q] = 0;
     __syncthreads();
+    // K4 (top2_all non-null): every warp records its best two keys of each step,
+    // top2[inst][t][rank * kWarps + w][0..1] -- the input of the near-tie check
+    const int nU = C * kWarps;
+    unsigned long long* top2 = top2_all ? top2_all + (int64_t)inst * m * nU * 2 : nullptr;
+    unsigned long long second_local = 0ull;
+    auto note = [&](unsigned long long k, unsigned long long& b1, unsigned long long& b2) {
+        if (k > b1) { b2 = b1; b1 = k; } else if (k > b2) { b2 = k; }
+    };
+    auto put_top2 = [&](int t, unsigned long long b1, unsigned long long b2) {
+        if (top2 && l == 0) {
+            unsigned long long* p = top2 + ((int64_t)t * nU + rank * kWarps + w) * 2;
+            p[0] = b1;
+            p[1] = b2;
+        }
+    };
     unsigned long long best_local = 0ull;
     for (int base = w; base < nr; base += kWarps * kR) {
         float acc_norm[kR];
@@ -119,10 +135,11 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
                 if (lr >= nr) continue;
                 const int i = r0 + lr;
                 const unsigned long long k = score_key(g[h], Kb[(size_t)lr * L + i], mu, (uint32_t)i, false, err);
-                best_local = k > best_local ? k : best_local;
+                note(k, best_local, second_local);
             }
         }
     }
+    put_top2(0, best_local, second_local);
     // CTA max -> every CTA's slot[0][rank] -> cluster max
     // (one CTA: every warp reduces the kWarps slots itself after ONE barrier;
     // the slots alternate with the step parity, so the next step's writes
@@ -147,6 +164,7 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
         }
     };
     unsigned long long best = exchange(best_local, 0);
+    if (forced && 0 < nforced) best = forced[0];         // K4 re-run: preset (flagged) picks
 
     for (int t = 1; t < m; ++t) {
         if (rank == 0 && tid == 0) keys_out[t - 1] = best;
@@ -161,6 +179,7 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
         csync();                                     // every CTA holds the pivot before rows change
         const float inv_c = __frcp_rn(__fadd_rn(piv[s], mu));
         best_local = 0ull;
+        second_local = 0ull;
         for (int base = w; base < nr; base += kWarps * kR) {
             float acc_norm[kR], a[kR];
 #pragma unroll
@@ -199,11 +218,13 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
                     const int i = r0 + lr;
                     const bool masked = sel[lr] != 0 || i == s;
                     const unsigned long long k = score_key(g[h], Kb[(size_t)lr * L + i], mu, (uint32_t)i, masked, err);
-                    best_local = k > best_local ? k : best_local;
+                    note(k, best_local, second_local);
                 }
             }
         }
+        put_top2(t, best_local, second_local);
         best = exchange(best_local, t & 1);
+        if (forced && t < nforced) best = forced[t];
     }
     if (rank == 0 && tid == 0) keys_out[m - 1] = best;
     csync();                                         // no CTA exits while others may read its smem

@@ -400,7 +400,7 @@ def test_launch_counter_counts_kernels():
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3) as cs:
         cs.select(10, MU)
-    assert bt.bted_kernel_launches() - before == 1 + 1       # finite check + the whole TED in one cluster kernel
+    assert bt.bted_kernel_launches() - before == 1 + 1 + 1   # finite check + the whole TED in one cluster kernel + K4 check
 
 
 # ------------------------------------------------------------------ packed vs dense layout
@@ -609,6 +609,34 @@ def test_k4_in_batches_matches_oracle_strictly(flags):
         pos = _positions(batches[b], bidx[b])
         check_ted(pos, [], dense.ted(X[batches[b]], g, MU, m, forced=pos), f"k4-batch{b}", gap_exact=GAP_K4)
     print(f"K4 in batches: refined {st['refined_steps']}, corrected {st['corrected_steps']}, launches {launches}")
+
+
+def test_k4_cluster_kernel_exact_ties():
+    """K4 on the one-kernel cluster TED (small candidate sets: merges, paper-scale
+    batches): exact duplicates give exact fp32 ties; every flagged step is
+    re-scored in fp64 and P2 holds at the fp64 gap, for a small select, the
+    paper-scale batches and their merge."""
+    X = knob(600, seed=47)
+    X = np.concatenate([X, X[::3]], axis=0)                  # 800 points, 200 exact duplicate pairs
+    g = median_gamma(X, 47)
+    with bt.CandidateSet(X, g) as cs:                          # N = 800: the cluster kernel
+        L.bted_reset_stats(cs.ctx)
+        idx, sc = cs.select(96, MU)
+        st = L.bted_get_stats(cs.ctx)
+    assert st["refined_steps"] > 0
+    check_ted(idx, sc, dense.ted(X, g, MU, 96, forced=idx), "k4-cluster", gap_exact=GAP_K4)
+    P, M, B, m, seed = X.shape[0], 300, 4, 64, 23
+    with bt.CandidateSet(X, g, num_batches=B, seed=seed) as pool:     # batches and merge in cluster kernels
+        sel, bidx = pool.run_batches(M, m, MU)
+        sel2, _ = pool.run_batches(M, m, MU)
+    assert np.array_equal(sel, sel2)
+    batches = oracle_sample_batches(P, M, B, seed)
+    for b in range(B):
+        pos = _positions(batches[b], bidx[b])
+        check_ted(pos, [], dense.ted(X[batches[b]], g, MU, m, forced=pos), f"k4-cluster-batch{b}", gap_exact=GAP_K4)
+    XU = np.unique(bidx.reshape(-1))
+    mpos = _positions(XU, sel)
+    check_ted(mpos, [], dense.ted(X[XU], g, MU, m, forced=mpos), "k4-cluster-merge", gap_exact=GAP_K4)
 
 
 def test_large_131072_sampled_against_closed_form():
