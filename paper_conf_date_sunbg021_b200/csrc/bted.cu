@@ -760,6 +760,11 @@ struct bted_ctx {
     int* kncand = nullptr; size_t kncandcap = 0;
     int* knflag = nullptr; size_t knflagcap = 0;
     unsigned long long* kforced = nullptr; size_t kforcedcap = 0;
+    int* k4pin = nullptr; size_t k4pincap = 0;            // pinned copy of knflag (read after the next sync)
+    struct {                                              // batch K4 decided at the merge's host sync
+        bool pending = false, changed = false;
+        int ninst = 0; int64_t M = 0; int32_t m = 0; float mu = 0.f;
+    } k4b;
     float* xall = nullptr; size_t xallcap = 0;             // [nb][M][d] gathered batches
     unsigned long long* kall = nullptr; size_t kallcap = 0; // [nb][m] keys
     // host staging (pinned)
@@ -1023,7 +1028,7 @@ void refine_step(bted_ctx* ctx, cudaStream_t st, const float* X, int64_t N, int3
     grow(ctx->rG, ctx->rGcap, (size_t)ncol * N);
     grow(ctx->rA, ctx->rAcap, (size_t)std::max(1, t * t));
     grow(ctx->rW, ctx->rWcap, (size_t)bted::rf::kMaxCand * std::max(1, t));
-    const int nblk = (int)std::min<int64_t>((N + 255) / 256, 296);
+    const int nblk = (int)((N + 255) / 256);
     grow(ctx->rpart, ctx->rpartcap, (size_t)nblk * bted::rf::kMaxCand);
     grow(ctx->rdiag, ctx->rdiagcap, (size_t)bted::rf::kMaxCand);
     grow(ctx->rout, ctx->routcap, (size_t)bted::rf::kMaxCand + 1);
@@ -1032,13 +1037,15 @@ void refine_step(bted_ctx* ctx, cudaStream_t st, const float* X, int64_t N, int3
     const int lin = ctx->kernel == BTED_KERNEL_LINEAR ? 1 : 0;
     bted::rf::refine_cols_kernel<<<dim3((unsigned)((N + 255) / 256), (unsigned)ncol), 256, 0, st>>>(
         X, (int32_t)N, d, (double)ctx->params.gamma, lin, ctx->rcols, ctx->rG);
+    // A (t x t) in shared memory when it fits; with the candidates' right-hand sides too (mode 2), the
+    // triangular solves run on all threads instead of one thread per candidate
     const size_t asmem = sizeof(double) * (size_t)t * (size_t)t;
-    const bool a_in_smem = asmem <= 48 * 1024;
-    bted::rf::refine_solve_kernel<<<1, 256, a_in_smem ? asmem : 0, st>>>(ctx->rG, (int32_t)N, ctx->rcols, t, nc,
-                                                                        (double)mu, ctx->rA, ctx->rW,
-                                                                        a_in_smem ? 1 : 0);
-    bted::rf::refine_resid_kernel<<<nblk, 256, 0, st>>>(ctx->rG, (int32_t)N, ctx->rcols, t, nc, ctx->rW, ctx->rpart,
-                                                       ctx->rdiag);
+    const size_t absmem = asmem + sizeof(double) * (size_t)nc * (size_t)t;
+    const int amode = absmem <= 48 * 1024 ? 2 : asmem <= 48 * 1024 ? 1 : 0;
+    bted::rf::refine_solve_kernel<<<1, 256, amode == 2 ? absmem : amode == 1 ? asmem : 0, st>>>(
+        ctx->rG, (int32_t)N, ctx->rcols, t, nc, (double)mu, ctx->rA, ctx->rW, amode);
+    bted::rf::refine_resid2_kernel<<<dim3((unsigned)nblk, (unsigned)nc), 256, sizeof(double) * std::max(t, 1), st>>>(
+        ctx->rG, (int32_t)N, ctx->rcols, t, ctx->rW, ctx->rpart, ctx->rdiag);
     bted::rf::refine_pick_kernel<<<1, 32, 0, st>>>(ctx->rpart, nblk, ctx->rdiag, ctx->rcols, t, nc, (double)mu,
                                                   ctx->rout, ctx->ridx);
     LAUNCHED(4);
@@ -1186,11 +1193,37 @@ unsigned long long* small_k4_reserve(bted_ctx* ctx, int ninst, int64_t N, int32_
 // (one check launch each, one host sync), then re-score the flagged steps of the
 // flagged instances exactly in fp64; a changed pick re-runs that instance with
 // the corrected prefix forced.  X: ninst x N x d (device); keys: ninst x m.
-void small_k4(bted_ctx* ctx, cudaStream_t st, const float* X, int ninst, int64_t N, int32_t d, int32_t m, float mu,
-              unsigned long long* keys, int* err) {
+// Part 1 (no host sync): the batched near-tie check and an async copy of the
+// per-instance flag counts into pinned memory, read by small_k4_refine after
+// the caller's next stream synchronisation.
+void small_k4_launch(bted_ctx* ctx, cudaStream_t st, int ninst, int64_t N, int32_t d, int32_t m,
+                     const unsigned long long* keys) {
+    const int nUb = small_cluster_used(ninst, N, d) * bted::sm::kWarps;
+    if (ctx->k4pincap < (size_t)ninst) {
+        if (ctx->k4pin) cudaFreeHost(ctx->k4pin);
+        ctx->k4pin = nullptr; ctx->k4pincap = 0;
+        CK(cudaHostAlloc(&ctx->k4pin, sizeof(int) * ninst, cudaHostAllocDefault));
+        ctx->k4pincap = (size_t)ninst;
+    }
+    CK(cudaMemsetAsync(ctx->knflag, 0, sizeof(int) * ninst, st));
+    bted::rf::neartie_check_kernel<<<dim3(m, ninst), 256, 0, st>>>(ctx->ktop2, nUb, keys, bted::rf::kTau,
+                                                                  ctx->kflags, ctx->kcand, ctx->kncand, ctx->knflag);
+    LAUNCHED(1);
+    CK(cudaMemcpyAsync(ctx->k4pin, ctx->knflag, sizeof(int) * ninst, cudaMemcpyDeviceToHost, st));
+}
+
+// Part 2 (after a sync that follows small_k4_launch): re-score the flagged steps of
+// the flagged instances in fp64; a changed pick re-runs that instance alone with
+// the corrected prefix forced.  Returns true if any pick changed.
+bool small_k4_refine(bted_ctx* ctx, cudaStream_t st, const float* X, int ninst, int64_t N, int32_t d, int32_t m,
+                     float mu, unsigned long long* keys, int* err) {
+    bool any = false;
+    for (int k = 0; k < ninst; ++k) any |= ctx->k4pin[k] != 0;
+    if (!any) return false;
     const int nUb = small_cluster_used(ninst, N, d) * bted::sm::kWarps;
     const int nU1 = small_cluster_used(1, N, d) * bted::sm::kWarps;
     const size_t kMC = bted::rf::kMaxCand;
+    bool changed = false;
     unsigned long long* rerun_top2 = ctx->ktop2 + (size_t)ninst * m * nUb * 2;
     auto check = [&](int k, const unsigned long long* t2, int nU) {
         bted::rf::neartie_check_kernel<<<m, 256, 0, st>>>(t2, nU, keys + (size_t)k * m,
@@ -1199,13 +1232,7 @@ void small_k4(bted_ctx* ctx, cudaStream_t st, const float* X, int ninst, int64_t
                                                          ctx->knflag + k);
         LAUNCHED(1);
     };
-    CK(cudaMemsetAsync(ctx->knflag, 0, sizeof(int) * ninst, st));
-    bted::rf::neartie_check_kernel<<<dim3(m, ninst), 256, 0, st>>>(ctx->ktop2, nUb, keys, bted::rf::kTau,
-                                                                  ctx->kflags, ctx->kcand, ctx->kncand, ctx->knflag);
-    LAUNCHED(1);
-    std::vector<int> nf(ninst);
-    CK(cudaMemcpyAsync(nf.data(), ctx->knflag, sizeof(int) * ninst, cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
+    std::vector<int> nf(ctx->k4pin, ctx->k4pin + ninst);
     std::vector<unsigned long long> hk(m);
     std::vector<int> fl(m), nc(m);
     std::vector<uint32_t> cd((size_t)m * kMC);
@@ -1236,6 +1263,7 @@ void small_k4(bted_ctx* ctx, cudaStream_t st, const float* X, int ninst, int64_t
                 const uint32_t pick = 0xFFFFFFFFu - (uint32_t)(hk[ts] & 0xFFFFFFFFull);
                 if (best == pick) continue;
                 ctx->corrected_steps++;
+                changed = true;
                 std::vector<unsigned long long> forced(ts + 1);
                 for (int q = 0; q < ts; ++q) forced[q] = hk[q] | bted::rf::kForced;
                 forced[ts] = host_pack_key((float)bs, best) | bted::rf::kForced;
@@ -1252,11 +1280,13 @@ void small_k4(bted_ctx* ctx, cudaStream_t st, const float* X, int ninst, int64_t
             if (!rerun) break;
         }
     }
+    return changed;
 }
 
 // Alg. 2 l.1-4 for batches b_begin, b_begin+b_step, ... ; winners on device.
 int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_begin, int32_t b_step) {
     const int32_t B = ctx->params.num_batches;
+    ctx->k4b.pending = false;
     int nb = 0;
     for (int32_t b = b_begin; b < B; b += b_step) ++nb;
     grow(ctx->winners, ctx->winnerscap, (size_t)std::max(nb, 1) * m);
@@ -1279,7 +1309,11 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
         unsigned long long* k4t = T.refine ? small_k4_reserve(ctx, nb, M, ctx->d, m) : nullptr;
         launch_small(ctx->xall, nb, M, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, ctx->kall, T.err, st, k4t);
         if (sl) CK(cudaEventRecord(sl->e[1], st));
-        if (k4t) small_k4(ctx, st, ctx->xall, nb, M, ctx->d, m, mu, ctx->kall, T.err);
+        if (k4t) {                                       // decided at the caller's next host sync
+            small_k4_launch(ctx, st, nb, M, ctx->d, m, ctx->kall);
+            ctx->k4b.pending = true;
+            ctx->k4b.ninst = nb; ctx->k4b.M = M; ctx->k4b.m = m; ctx->k4b.mu = mu;
+        }
         for (int kk = 0; kk < nb; ++kk) {
             bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->kall + (size_t)kk * m, m,
                                                                      ctx->sall + (size_t)kk * M,
@@ -1362,6 +1396,20 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
     CK(cudaMemcpyAsync(&nu, ctx->count_dev, sizeof(int), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));                        // |X_U| sizes the merge TED
     ctx->bted_engine.collect();
+    if (ctx->k4b.pending) {                               // K4 of the small batch TEDs, decided here
+        ctx->k4b.pending = false;
+        auto& b = ctx->k4b;
+        if (small_k4_refine(ctx, st, ctx->xall, b.ninst, b.M, ctx->d, b.m, b.mu, ctx->kall, ctx->bted_engine.err)) {
+            for (int kk = 0; kk < b.ninst; ++kk) {
+                bted::map_winners_kernel<<<(b.m + 127) / 128, 128, 0, st>>>(ctx->kall + (size_t)kk * b.m, b.m,
+                                                                           ctx->sall + (size_t)kk * b.M,
+                                                                           ctx->winners + (size_t)kk * b.m);
+                LAUNCHED(1);
+            }
+            b.changed = true;
+            return merge_device(ctx, winners_dev, n, m, mu, out_idx, out_count);   // the union changed
+        }
+    }
     if (nu < 1) { set_error("empty union"); return BTED_ENUMERIC; }
     const int32_t mm = std::min<int32_t>(m, nu);          // reading A12
     gather(ctx, st, ctx->u32a, nu);                       // X[X_U] (A13: fresh Gram)
@@ -1373,7 +1421,20 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
         if (!T.err) { grow(T.err, T.errcap, 1); CK(cudaMemsetAsync(T.err, 0, sizeof(int), st)); }
         unsigned long long* k4t = T.refine ? small_k4_reserve(ctx, 1, nu, ctx->d, mm) : nullptr;
         launch_small(ctx->Xb, 1, nu, ctx->d, ctx->params.gamma, ctx->kernel, mm, mu, ctx->mkeys, T.err, st, k4t);
-        if (k4t) small_k4(ctx, st, ctx->Xb, 1, nu, ctx->d, mm, mu, ctx->mkeys, T.err);
+        if (k4t) {
+            small_k4_launch(ctx, st, 1, nu, ctx->d, mm, ctx->mkeys);
+            bted::map_winners_kernel<<<(mm + 127) / 128, 128, 0, st>>>(ctx->mkeys, mm, ctx->u32a, ctx->out_dev);
+            LAUNCHED(1);
+            bted_status s = finish_keys(ctx, ctx->bted_engine, ctx->mkeys, mm, out_idx, nullptr, ctx->out_dev);
+            if (s == BTED_OK && small_k4_refine(ctx, st, ctx->Xb, 1, nu, ctx->d, mm, mu, ctx->mkeys, T.err)) {
+                bted::map_winners_kernel<<<(mm + 127) / 128, 128, 0, st>>>(ctx->mkeys, mm, ctx->u32a,
+                                                                         ctx->out_dev);
+                LAUNCHED(1);
+                s = finish_keys(ctx, ctx->bted_engine, ctx->mkeys, mm, out_idx, nullptr, ctx->out_dev);
+            }
+            if (s == BTED_OK) *out_count = mm;
+            return s;
+        }
     } else {
         // size varies with |X_U|: run it eagerly
         run_ted(ctx->bted_engine, ctx->Xb, nu, ctx->d, ctx->params.gamma, ctx->kernel, mm, mu, ctx->mkeys,
@@ -1424,9 +1485,12 @@ bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, fl
             launch_small(ctx->X, 1, ctx->N, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, T.keys, T.err, T.stream,
                          k4t);
             if (sl) CK(cudaEventRecord(sl->e[1], T.stream));
-            if (k4t) small_k4(ctx, T.stream, ctx->X, 1, ctx->N, ctx->d, m, mu, T.keys, T.err);
+            if (k4t) small_k4_launch(ctx, T.stream, 1, ctx->N, ctx->d, m, T.keys);
             T.last_rows = 0;                       // K lived in shared memory only
-            return finish_keys(ctx, T, T.keys, m, out_idx, out_score);
+            bted_status s = finish_keys(ctx, T, T.keys, m, out_idx, out_score);
+            if (s == BTED_OK && k4t && small_k4_refine(ctx, T.stream, ctx->X, 1, ctx->N, ctx->d, m, mu, T.keys, T.err))
+                s = finish_keys(ctx, T, T.keys, m, out_idx, out_score);
+            return s;
         }
         T.reserve(ctx->N, ctx->N, ctx->d, m);
         const bool packed = use_packed(ctx->params.flags, ctx->d);
@@ -1468,6 +1532,21 @@ bted_status bted_batch_teds(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32
             CK(cudaMemcpyAsync(ctx->herr, ctx->bted_engine.err, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
         CK(cudaStreamSynchronize(ctx->stream));
         ctx->bted_engine.collect();
+        if (ctx->k4b.pending) {                          // K4 of small batch TEDs
+            ctx->k4b.pending = false;
+            auto& b = ctx->k4b;
+            if (small_k4_refine(ctx, ctx->stream, ctx->xall, b.ninst, b.M, ctx->d, b.m, b.mu, ctx->kall,
+                                ctx->bted_engine.err)) {
+                for (int kk = 0; kk < b.ninst; ++kk) {
+                    bted::map_winners_kernel<<<(b.m + 127) / 128, 128, 0, ctx->stream>>>(
+                        ctx->kall + (size_t)kk * b.m, b.m, ctx->sall + (size_t)kk * b.M, ctx->winners + (size_t)kk * b.m);
+                    LAUNCHED(1);
+                }
+                CK(cudaMemcpyAsync(out_winners, ctx->winners, bytes,
+                                   winners_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, ctx->stream));
+                CK(cudaStreamSynchronize(ctx->stream));
+            }
+        }
         if (take_xbad(ctx)) return BTED_EINVAL;
         if (nb > 0 && *ctx->herr) {
             CK(cudaMemsetAsync(ctx->bted_engine.err, 0, sizeof(int), ctx->stream));
@@ -1502,11 +1581,18 @@ bted_status bted_run_batches(bted_ctx* ctx, int64_t M, int32_t m, float mu, int6
     if (ctx->is_shard || ctx->is_ishard) { set_error("run_batches on a shard context"); return BTED_EINVAL; }
     if (m < 1 || M < m || M > ctx->N || !mu_ok(mu)) { set_error("need 1 <= m <= M <= N and mu > 0"); return BTED_EINVAL; }
     return guarded(ctx, [&]() -> bted_status {
+        ctx->k4b.changed = false;
         const int nb = run_batch_range(ctx, M, m, mu, 0, 1);
         if (out_batch_idx)
             CK(cudaMemcpyAsync(out_batch_idx, ctx->winners, sizeof(int64_t) * (size_t)nb * m,
                                cudaMemcpyDeviceToHost, ctx->stream));
-        return merge_device(ctx, ctx->winners, (int64_t)nb * m, m, mu, out_idx, out_count);
+        bted_status s = merge_device(ctx, ctx->winners, (int64_t)nb * m, m, mu, out_idx, out_count);
+        if (s == BTED_OK && out_batch_idx && ctx->k4b.changed) {   // batch K4 changed winners after the copy
+            CK(cudaMemcpyAsync(out_batch_idx, ctx->winners, sizeof(int64_t) * (size_t)nb * m,
+                               cudaMemcpyDeviceToHost, ctx->stream));
+            CK(cudaStreamSynchronize(ctx->stream));
+        }
+        return s;
     });
 }
 
@@ -1881,6 +1967,7 @@ void bted_destroy(bted_ctx* ctx) {
                         ctx->bflag, ctx->rcols, ctx->rG, ctx->rA, ctx->rW, ctx->rpart, ctx->rdiag, ctx->rout,
                         ctx->ridx, ctx->bkeys, ctx->bsflags, ctx->bncand, ctx->bcand, ctx->sks, ctx->scnt,
                         ctx->ktop2, ctx->kflags, ctx->kcand, ctx->kncand, ctx->knflag, ctx->kforced};
+        if (ctx->k4pin) cudaFreeHost(ctx->k4pin);
         for (void* b : bufs) if (b) cudaFree(b);
         if (ctx->own_X && ctx->X) cudaFree(ctx->X);
         if (ctx->hkeys) cudaFreeHost(ctx->hkeys);

@@ -132,6 +132,36 @@ refine_solve_kernel(const double* __restrict__ G, int32_t N, const uint32_t* __r
         }
         __syncthreads();
     }
+    if (a_in_smem == 2) {                               // all candidates at once, right-looking, in smem
+        double* B = As + (size_t)t * t;                 // [nc][t]: K_Sc -> y -> w
+        for (int e = tid; e < nc * t; e += 256) {
+            const int c = e / t, i = e % t;
+            B[e] = G[(int64_t)i * N + cols[t + c]];
+        }
+        __syncthreads();
+        for (int i = 0; i < t; ++i) {                   // L y = b
+            const double lii = A[i * t + i];
+            for (int c = tid; c < nc; c += 256) B[c * t + i] /= lii;
+            __syncthreads();
+            for (int e = tid; e < nc * (t - i - 1); e += 256) {
+                const int c = e / (t - i - 1), j = i + 1 + e % (t - i - 1);
+                B[c * t + j] -= A[j * t + i] * B[c * t + i];
+            }
+            __syncthreads();
+        }
+        for (int i = t - 1; i >= 0; --i) {              // L^T w = y
+            const double lii = A[i * t + i];
+            for (int c = tid; c < nc; c += 256) B[c * t + i] /= lii;
+            __syncthreads();
+            for (int e = tid; e < nc * i; e += 256) {
+                const int c = e / i, j = e % i;
+                B[c * t + j] -= A[i * t + j] * B[c * t + i];
+            }
+            __syncthreads();
+        }
+        for (int e = tid; e < nc * t; e += 256) W[e] = B[e];
+        return;
+    }
     for (int c = tid; c < nc; c += 256) {               // W[:, c] = L^-T L^-1 K_Sc
         double* w = W + (int64_t)c * t;
         for (int i = 0; i < t; ++i) {                   // forward
@@ -147,44 +177,32 @@ refine_solve_kernel(const double* __restrict__ G, int32_t N, const uint32_t* __r
     }
 }
 
-// r_ic = K_ic - sum_k K_{i,S_k} W[k][c]; per-CTA partial sums of r_ic^2 (rows in
-// thread order, then a fixed tree) and the residual at the candidate's own row.
+// r_ic = K_ic - sum_k K_{i,S_k} W[k][c]: per-CTA partial sums of r_ic^2 and the
+// residual at the candidate's own row.  One thread per (row, candidate): grid
+// (ceil(N / 256), nc); the candidate's W column is broadcast from shared memory.
 __global__ void __launch_bounds__(256)
-refine_resid_kernel(const double* __restrict__ G, int32_t N, const uint32_t* __restrict__ cols, int t, int nc,
-                    const double* __restrict__ W, double* __restrict__ part, double* __restrict__ diag) {
-    __shared__ double red[8][kMaxCand];
-    const int tid = threadIdx.x;
-    double acc2[kMaxCand];
-#pragma unroll
-    for (int c = 0; c < kMaxCand; ++c) acc2[c] = 0.0;
-    for (int i = blockIdx.x * 256 + tid; i < N; i += gridDim.x * 256) {
-        double r[kMaxCand];
-#pragma unroll
-        for (int c = 0; c < kMaxCand; ++c) r[c] = c < nc ? G[(int64_t)(t + c) * N + i] : 0.0;
-        for (int k = 0; k < t; ++k) {
-            const double g = G[(int64_t)k * N + i];
-#pragma unroll
-            for (int c = 0; c < kMaxCand; ++c)
-                if (c < nc) r[c] -= g * W[(int64_t)c * t + k];
-        }
-#pragma unroll
-        for (int c = 0; c < kMaxCand; ++c) {
-            if (c < nc) {
-                acc2[c] = __fma_rn(r[c], r[c], acc2[c]);
-                if ((uint32_t)i == cols[t + c]) diag[c] = r[c];
-            }
-        }
-    }
-    for (int c = 0; c < nc; ++c) {
-        double v = acc2[c];
-        for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
-        if ((tid & 31) == 0) red[tid >> 5][c] = v;
-    }
+refine_resid2_kernel(const double* __restrict__ G, int32_t N, const uint32_t* __restrict__ cols, int t,
+                     const double* __restrict__ W, double* __restrict__ part, double* __restrict__ diag) {
+    extern __shared__ double wc[];                      // [t]
+    __shared__ double red[8];
+    const int c = blockIdx.y, tid = threadIdx.x;
+    for (int k = tid; k < t; k += 256) wc[k] = W[(int64_t)c * t + k];
     __syncthreads();
-    if (tid < nc) {
+    const int i = blockIdx.x * 256 + tid;
+    double r2 = 0.0;
+    if (i < N) {
+        double r = G[(int64_t)(t + c) * N + i];
+        for (int k = 0; k < t; ++k) r -= G[(int64_t)k * N + i] * wc[k];
+        r2 = r * r;
+        if ((uint32_t)i == cols[t + c]) diag[c] = r;
+    }
+    for (int off = 16; off > 0; off >>= 1) r2 += __shfl_xor_sync(0xffffffffu, r2, off);
+    if ((tid & 31) == 0) red[tid >> 5] = r2;
+    __syncthreads();
+    if (tid == 0) {
         double v = 0.0;
-        for (int w = 0; w < 8; ++w) v += red[w][tid];
-        part[(int64_t)blockIdx.x * kMaxCand + tid] = v;
+        for (int w = 0; w < 8; ++w) v += red[w];
+        part[(int64_t)blockIdx.x * kMaxCand + c] = v;
     }
 }
 
