@@ -639,6 +639,28 @@ def test_k4_cluster_kernel_exact_ties():
     check_ted(mpos, [], dense.ted(X[XU], g, MU, m, forced=mpos), "k4-cluster-merge", gap_exact=GAP_K4)
 
 
+def test_k4_cluster_kernel_long_selections():
+    """Long selections on the cluster kernel (small N, late steps with small
+    scores and many near ties): P2 at the fp64 gap on every seed; the forced
+    re-launch path runs whenever a refined pick changes."""
+    total_refined = total_corrected = 0
+    for seed in range(6):
+        X = uniform_pool(720, 8, 700 + seed)
+        Xn = X[::4].copy()
+        Xn[:, seed % 8] += np.float32(2e-4)                  # near duplicates: fp64 gaps far below fp32 noise
+        X = np.concatenate([X, Xn], axis=0)
+        g = median_gamma(X, seed)
+        with bt.CandidateSet(X, g) as cs:
+            L.bted_reset_stats(cs.ctx)
+            idx, sc = cs.select(300, MU)
+            st = L.bted_get_stats(cs.ctx)
+        total_refined += st["refined_steps"]
+        total_corrected += st["corrected_steps"]
+        check_ted(idx, sc, dense.ted(X, g, MU, 300, forced=idx), f"k4-cluster-long-{seed}", gap_exact=GAP_K4)
+    print(f"cluster K4: refined {total_refined} steps, corrected {total_corrected}")
+    assert total_refined > 0 and total_corrected > 0         # the forced re-launch path ran (deterministic)
+
+
 def test_large_131072_sampled_against_closed_form():
     """one un-batched TED on N = 131072 (K = 34 GB per packed
     buffer), P1 at every step and sampled P2, as for 'oversized'."""
