@@ -310,22 +310,22 @@ void launch_transpose(Ted& T, const float* X, int64_t N, int32_t d) {
 }
 
 void launch_gram(Ted& T, int64_t N, int32_t d, int64_t row0, int64_t rows, float gamma, int kernel,
-                 float mu, unsigned long long* key_out) {
+                 float mu, unsigned long long* key_out, unsigned long long* top2 = nullptr) {
     const int64_t ld = ld_for(N);
     const unsigned grid = (unsigned)((rows + kK1Rows - 1) / kK1Rows);
     const size_t smem = sizeof(float) * kK1Rows * d;
     bted::gram_rownorm_kernel<kK1Rows, kK1Threads><<<grid, kK1Threads, smem, T.stream>>>(
         T.XT, ld, d, (int32_t)N, (int32_t)row0, (int32_t)rows, gamma, kernel == BTED_KERNEL_LINEAR ? 1 : 0,
-        T.K[0], mu, key_out, T.err);
+        T.K[0], mu, key_out, T.err, top2);
     LAUNCHED(1);
 }
 
 void launch_step(Ted& T, int64_t N, int64_t row0, int64_t rows, int32_t t, float mu, const float* pivot,
-                 unsigned long long* keys) {
+                 unsigned long long* keys, unsigned long long* top2 = nullptr) {
     const int64_t ld = ld_for(N);
     const unsigned grid = (unsigned)((rows + kRowsPerK2Cta - 1) / kRowsPerK2Cta);
     bted::deflate_rescore_kernel<kK2Rows, kK2Unroll, kK2Threads><<<grid, kK2Threads, 0, T.stream>>>(
-        T.K[(t - 1) & 1], T.K[t & 1], ld, (int32_t)row0, (int32_t)rows, pivot, keys, t, mu, T.sel, T.err);
+        T.K[(t - 1) & 1], T.K[t & 1], ld, (int32_t)row0, (int32_t)rows, pivot, keys, t, mu, T.sel, T.err, top2);
     LAUNCHED(1);
 }
 
@@ -576,11 +576,11 @@ void enqueue_head(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int
     launch_transpose(T, X, N, d);
     CK(cudaMemsetAsync(keys, 0, sizeof(unsigned long long) * m, T.stream));
     CK(cudaMemsetAsync(T.sel, 0, (size_t)N, T.stream));
-    launch_gram(T, N, d, 0, N, gamma, kernel, mu, keys);
+    launch_gram(T, N, d, 0, N, gamma, kernel, mu, keys, T.refine ? T.top2 : nullptr);
 }
 // Alg. 1 l.2-6 loop: m-1 fused deflate + rescore steps.  (m-1 kernels)
 void enqueue_loop(Ted& T, int64_t N, int32_t m, float mu, unsigned long long* keys) {
-    for (int32_t t = 1; t < m; ++t) launch_step(T, N, 0, N, t, mu, nullptr, keys);
+    for (int32_t t = 1; t < m; ++t) launch_step(T, N, 0, N, t, mu, nullptr, keys, T.refine ? T.top2 : nullptr);
 }
 
 template <class F>
@@ -649,6 +649,11 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
         T.last_nT = (int32_t)((N + bted::pk::T - 1) / bted::pk::T);
     } else {
         T.reserve(N, N, d, m);
+        if (T.refine) {                    // K4 on the dense engine: top-2 keys of every K2 CTA
+            const void* top2_before = T.top2;
+            T.reserve_refine((int64_t)((N + kRowsPerK2Cta - 1) / kRowsPerK2Cta) * 32, m);
+            if (T.top2 != top2_before) { for (auto& g : T.graphs) cudaGraphExecDestroy(g.second); T.graphs.clear(); }
+        }
     }
     T.last_packed = packed;
     T.last_rows = N;
@@ -687,7 +692,7 @@ void run_ted(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kern
         }
     }
     if (sl) CK(cudaEventRecord(sl->e[2], T.stream));
-    if (packed && T.refine && nflag_dst) {
+    if (T.refine && nflag_dst) {
         // K4 check; its per-step flags/candidates go to T's buffers or, for a batch
         // TED of Alg. 2, to that batch's own slice (refined later without a re-run)
         bted::rf::neartie_check_kernel<<<m, 256, 0, T.stream>>>(T.top2, T.last_nC, keys, bted::rf::kTau,
@@ -1324,7 +1329,7 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
     }
     Ted& T = ctx->bted_engine;
     const bool packed = use_packed(ctx->params.flags, ctx->d);
-    const bool k4 = packed && T.refine;
+    const bool k4 = T.refine;
     const size_t nC = (size_t)bted::rf::kMaxCand;
     if (k4) {
         grow(ctx->bflag, ctx->bflagcap, (size_t)nb);
@@ -1494,14 +1499,14 @@ bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, fl
         }
         T.reserve(ctx->N, ctx->N, ctx->d, m);
         const bool packed = use_packed(ctx->params.flags, ctx->d);
-        if (packed && T.refine) {
+        if (T.refine) {
             T.reserve_refine(((ctx->N + bted::pk::T - 1) / bted::pk::T) * bted::pk::T, m);
             CK(cudaMemsetAsync(T.nflag, 0, sizeof(int), T.stream));
         }
         run_ted(T, ctx->X, ctx->N, ctx->d, ctx->params.gamma, ctx->kernel, m, mu, T.keys,
-                (ctx->params.flags & BTED_FLAG_NO_GRAPH) != 0, true, packed, packed ? T.nflag : nullptr);
+                (ctx->params.flags & BTED_FLAG_NO_GRAPH) != 0, true, packed, T.refine ? T.nflag : nullptr);
         std::vector<float> fixed(m, -1.f);
-        if (packed && T.refine) {
+        if (T.refine) {
             int nf = 0;
             CK(cudaMemcpyAsync(&nf, T.nflag, sizeof(int), cudaMemcpyDeviceToHost, T.stream));
             CK(cudaStreamSynchronize(T.stream));

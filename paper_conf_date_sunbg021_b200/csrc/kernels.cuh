@@ -83,18 +83,41 @@ __device__ __forceinline__ unsigned long long score_key(float g, float diag, flo
     return masked ? 0ull : pack_key(sc, idx);
 }
 
-// CTA-wide max of one key per thread, then one atomicMax into *dst.
+// CTA-wide max of one key per thread, then one atomicMax into *dst.  With
+// top2 (K4 near-tie check, refine.cuh) the CTA's two best keys are also
+// written to top2[0..1] (keys are distinct: they carry the row index).
+__device__ __forceinline__ void top2_merge(unsigned long long& b1, unsigned long long& b2, unsigned long long c1,
+                                           unsigned long long c2) {
+    const unsigned long long hi = b1 > c1 ? b1 : c1, lo = b1 > c1 ? c1 : b1;
+    const unsigned long long s2 = b2 > c2 ? b2 : c2;
+    b1 = hi;
+    b2 = lo > s2 ? lo : s2;
+}
 template <int kThreads>
-__device__ __forceinline__ void cta_key_max_to(unsigned long long key, unsigned long long* dst) {
-    __shared__ unsigned long long red[kThreads / kWarp];
-    key = warp_max_u64(key);
+__device__ __forceinline__ void cta_key_max_to(unsigned long long key, unsigned long long* dst,
+                                               unsigned long long* top2 = nullptr) {
+    __shared__ unsigned long long red[kThreads / kWarp][2];
+    unsigned long long b1 = key, b2 = 0ull;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+        const unsigned long long c1 = __shfl_xor_sync(0xffffffffu, b1, off);
+        const unsigned long long c2 = __shfl_xor_sync(0xffffffffu, b2, off);
+        top2_merge(b1, b2, c1, c2);
+    }
     const int w = threadIdx.x / kWarp, l = threadIdx.x % kWarp;
-    if (l == 0) red[w] = key;
+    if (l == 0) { red[w][0] = b1; red[w][1] = b2; }
     __syncthreads();
     if (w == 0) {
-        unsigned long long v = l < kThreads / kWarp ? red[l] : 0ull;
-        v = warp_max_u64(v);
-        if (l == 0 && v != 0ull) atomicMax(dst, v);
+        unsigned long long v1 = l < kThreads / kWarp ? red[l][0] : 0ull;
+        unsigned long long v2 = l < kThreads / kWarp ? red[l][1] : 0ull;
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) {
+            const unsigned long long c1 = __shfl_xor_sync(0xffffffffu, v1, off);
+            const unsigned long long c2 = __shfl_xor_sync(0xffffffffu, v2, off);
+            top2_merge(v1, v2, c1, c2);
+        }
+        if (l == 0 && v1 != 0ull) atomicMax(dst, v1);
+        if (l == 0 && top2) { top2[0] = v1; top2[1] = v2; }
     }
 }
 
@@ -117,7 +140,8 @@ __global__ void __launch_bounds__(kThreads)
 gram_rownorm_kernel(const float* __restrict__ XT, int64_t ld, int32_t d, int32_t N,
                     int32_t row0, int32_t nrows, float gamma, int32_t linear,
                     float* __restrict__ K, float mu,
-                    unsigned long long* __restrict__ key_out, int* __restrict__ err) {
+                    unsigned long long* __restrict__ key_out, int* __restrict__ err,
+                    unsigned long long* __restrict__ top2 = nullptr) {
     extern __shared__ float xi[];                       // [kRows][d]
     __shared__ float red[kThreads / kWarp][kRows];
     const int lrow0 = blockIdx.x * kRows;               // local row of this CTA
@@ -199,7 +223,9 @@ gram_rownorm_kernel(const float* __restrict__ XT, int64_t ld, int32_t d, int32_t
             key = score_key(g, diag, mu, (uint32_t)(row0 + lr), false, err);
         }
     }
-    cta_key_max_to<kThreads>(key, key_out);
+    // (top2 at step 0 is laid out like K2's: CTA b of K1 covers K2's CTAs 2b, 2b+1)
+    if (top2 && threadIdx.x == 0) top2[4 * (int64_t)blockIdx.x + 2] = top2[4 * (int64_t)blockIdx.x + 3] = 0ull;
+    cta_key_max_to<kThreads>(key, key_out, top2 ? top2 + 4 * (int64_t)blockIdx.x : nullptr);
 }
 
 // ---------------------------------------------------------------------------
@@ -241,7 +267,8 @@ __global__ void __launch_bounds__(kThreads)
 deflate_rescore_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, int64_t ld,
                        int32_t row0, int32_t nrows, const float* __restrict__ pivot_ext,
                        unsigned long long* __restrict__ keys, int32_t t, float mu,
-                       uint8_t* __restrict__ sel, int* __restrict__ err) {
+                       uint8_t* __restrict__ sel, int* __restrict__ err,
+                       unsigned long long* __restrict__ top2 = nullptr) {
     constexpr int kWarps = kThreads / kWarp;
     const uint32_t s = key_index(keys[t - 1]);
     const float* __restrict__ p = pivot_ext ? pivot_ext : Kin + (int64_t)((int32_t)s - row0) * ld;
@@ -316,7 +343,7 @@ deflate_rescore_kernel(const float* __restrict__ Kin, float* __restrict__ Kout, 
             key = score_key(g, diag, mu, (uint32_t)i, masked, err);
         }
     }
-    cta_key_max_to<kThreads>(key, keys + t);
+    cta_key_max_to<kThreads>(key, keys + t, top2 ? top2 + ((int64_t)t * gridDim.x + blockIdx.x) * 2 : nullptr);
 }
 
 // ---------------------------------------------------------------------------

@@ -106,11 +106,9 @@ def test_one_deflation_step_vs_fp64_and_selected_column(flags):
 
 # ------------------------------------------------------------------ TED parity
 def k4_on(flags, N):
-    """K4 near-tie refinement runs on the packed / implicit engines (not dense,
-    not the small-N cluster kernel)."""
-    if flags & L.BTED_FLAG_DENSE or flags & L.BTED_FLAG_NO_REFINE:
-        return False
-    return bool(flags & L.BTED_FLAG_NO_SMALL) or N > 940
+    """K4 near-tie refinement runs on every single-GPU engine (packed, implicit,
+    dense and the small-N cluster kernel) unless BTED_FLAG_NO_REFINE."""
+    return not (flags & L.BTED_FLAG_NO_REFINE)
 
 
 def _ted_parity(X, g, m, label, use_dense=True, flags=0):
@@ -380,7 +378,7 @@ def test_launch_counter_counts_kernels():
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3, flags=DENSE) as cs:
         cs.select(10, MU)
-    assert bt.bted_kernel_launches() - before == 1 + 11      # finite check + transpose + K1 + 9 x K2
+    assert bt.bted_kernel_launches() - before == 1 + 11 + 1  # finite check + transpose + K1 + 9 x K2 + K4 check
     before = bt.bted_kernel_launches()
     with bt.CandidateSet(X, 0.3, flags=PACKED) as cs:
         cs.select(10, MU)
@@ -567,7 +565,7 @@ def test_k4_resolves_exact_ties_and_counts():
     check_ted(idx, sc, tr, "k4-dups", gap_exact=GAP_K4)
 
 
-@pytest.mark.parametrize("flags", [PACKED, IMPLICIT], ids=["packed", "implicit"])
+@pytest.mark.parametrize("flags", [PACKED, IMPLICIT, DENSE], ids=["packed", "implicit", "dense"])
 def test_k4_strict_parity_on_long_selections(flags):
     """Long selections (small late scores, many near ties): every pick equals
     the fp64 oracle's argmax wherever the oracle's gap exceeds 1e-9."""
@@ -586,7 +584,7 @@ def test_k4_strict_parity_on_long_selections(flags):
     print(f"K4: refined {total_refined} steps, corrected {total_corrected}")
 
 
-@pytest.mark.parametrize("flags", [PACKED, IMPLICIT], ids=["packed", "implicit"])
+@pytest.mark.parametrize("flags", [PACKED, IMPLICIT, DENSE], ids=["packed", "implicit", "dense"])
 def test_k4_in_batches_matches_oracle_strictly(flags):
     """Alg. 2 batch TEDs keep their own K4 state (keys, flags, candidates per
     batch); the flagged steps are refined after all batches without re-running
