@@ -58,9 +58,11 @@ typedef enum {
 
 /* flags */
 #define BTED_FLAG_NO_GRAPH 1u   /* launch the m-step loop eagerly (debug / profiling) */
-#define BTED_FLAG_DENSE    4u   /* store K densely (N x ld, 8 N^2 bytes per step) instead of the
-                                   default packed upper-triangular tiles (4 N^2 bytes per step;
-                                   used when d <= 32).  Shard contexts are always dense. */
+#define BTED_FLAG_DENSE    4u   /* literal deflation on a dense K (N x ld, 8 N^2 bytes per step)
+                                   instead of the packed upper-triangular tiles (used when
+                                   d <= 32; default engine: BTED_FLAG_IMPLICIT below, 2 N^2 bytes
+                                   per step).  Also used when d > 32.  Row-shard contexts
+                                   (bted_shard_*) are always dense. */
 #define BTED_FLAG_NO_SMALL 8u   /* never use the one-kernel cluster TED for small candidate sets
                                    (N <= ~940: K in distributed shared memory)               */
 #define BTED_FLAG_TMA     16u   /* packed layout: stream K through the persistent TMA ring
@@ -79,7 +81,8 @@ typedef enum {
                                    default three kernels per step (factor column, K.l pass, scores) */
 #define BTED_FLAG_NO_REFINE 128u /* disable K4: near ties (fp32 scores within 2e-5 of the best) are
                                    otherwise re-scored exactly in fp64 from the features and the
-                                   exact argmax taken (packed / implicit engines)               */
+                                   exact argmax taken (every single-GPU engine and the tile-sharded
+                                   engine; not the row-shard API)                               */
 #define BTED_FLAG_TIMING   2u   /* record CUDA events around K1 and the K2 loop of every batch
                                    TED on the ctx stream; read with bted_get_stats()          */
 
