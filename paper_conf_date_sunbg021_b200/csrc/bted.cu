@@ -1073,10 +1073,43 @@ inline unsigned long long host_pack_key(float score, uint32_t idx) {
 // the TED is re-run with the corrected prefix forced.  On return `keys` on
 // the device holds the final picks (forced ones flagged kForced) and
 // scores_out[t] (nullable) the fp32 score of each pick.
+// K4 host scan (shared by every engine): the first flagged step after `checked`
+// (with >= 2 candidates) is re-scored exactly; returns true with `forced` =
+// the flagged keys of steps 0..ts (the corrected pick last) if the exact argmax
+// differs from the GPU's pick, false once no flagged step is left.  hk, fl,
+// nc, cd: the TED's keys, flags, candidate counts and candidates (host copies).
+bool k4_next_correction(bted_ctx* ctx, cudaStream_t st, const float* X, int64_t N, int32_t d, int32_t m, float mu,
+                        const std::vector<unsigned long long>& hk, const std::vector<int>& fl,
+                        const std::vector<int>& nc, const std::vector<uint32_t>& cd, int& checked,
+                        std::vector<unsigned long long>& forced, double* corrected_score = nullptr) {
+    const size_t kMC = bted::rf::kMaxCand;
+    for (int ts = checked + 1; ts < m; ++ts) {
+        if (!fl[ts] || nc[ts] < 2) continue;
+        std::vector<uint32_t> S(ts), C;
+        for (int k = 0; k < ts; ++k) S[k] = 0xFFFFFFFFu - (uint32_t)(hk[k] & 0xFFFFFFFFull);
+        for (int c = 0; c < nc[ts]; ++c) C.push_back(cd[(size_t)ts * kMC + c]);
+        std::sort(C.begin(), C.end());
+        uint32_t best = 0;
+        double bs = 0.0;
+        refine_step(ctx, st, X, N, d, S, C, mu, &best, &bs);
+        ctx->refined_steps++;
+        checked = ts;
+        const uint32_t pick = 0xFFFFFFFFu - (uint32_t)(hk[ts] & 0xFFFFFFFFull);
+        if (best == pick) continue;
+        ctx->corrected_steps++;
+        forced.assign(ts + 1, 0ull);
+        for (int k = 0; k < ts; ++k) forced[k] = hk[k] | bted::rf::kForced;
+        forced[ts] = host_pack_key((float)bs, best) | bted::rf::kForced;
+        if (corrected_score) *corrected_score = bs;
+        return true;
+    }
+    return false;
+}
+
 void refine_ted(bted_ctx* ctx, Ted& T, const float* X, int64_t N, int32_t d, int32_t m, float mu,
                 unsigned long long* keys, float* scores_out) {
     cudaStream_t st = T.stream;
-    std::vector<unsigned long long> hk(m);
+    std::vector<unsigned long long> hk(m), forced;
     std::vector<int> fl(m), nc(m);
     std::vector<uint32_t> cd((size_t)m * bted::rf::kMaxCand);
     int checked = -1;
@@ -1086,30 +1119,13 @@ void refine_ted(bted_ctx* ctx, Ted& T, const float* X, int64_t N, int32_t d, int
         CK(cudaMemcpyAsync(nc.data(), T.ncand, sizeof(int) * m, cudaMemcpyDeviceToHost, st));
         CK(cudaMemcpyAsync(cd.data(), T.cand, sizeof(uint32_t) * cd.size(), cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
-        int ts = -1;
-        for (int t = checked + 1; t < m; ++t)
-            if (fl[t] && nc[t] >= 2) { ts = t; break; }
-        if (ts < 0) break;
-        std::vector<uint32_t> S(ts), C;
-        for (int k = 0; k < ts; ++k) S[k] = 0xFFFFFFFFu - (uint32_t)(hk[k] & 0xFFFFFFFFull);
-        for (int c = 0; c < nc[ts]; ++c) C.push_back(cd[(size_t)ts * bted::rf::kMaxCand + c]);
-        std::sort(C.begin(), C.end());
-        uint32_t best = 0;
         double bs = 0.0;
-        refine_step(ctx, st, X, N, d, S, C, mu, &best, &bs);
-        ctx->refined_steps++;
-        const uint32_t pick = 0xFFFFFFFFu - (uint32_t)(hk[ts] & 0xFFFFFFFFull);
-        checked = ts;
-        if (best == pick) continue;
-        // corrected pick: re-run with picks 0..ts forced
-        ctx->corrected_steps++;
-        std::vector<unsigned long long> forced(ts + 1);
-        for (int k = 0; k < ts; ++k) forced[k] = hk[k] | bted::rf::kForced;
-        forced[ts] = host_pack_key((float)bs, best) | bted::rf::kForced;
-        if (scores_out) scores_out[ts] = (float)bs;
+        if (!k4_next_correction(ctx, st, X, N, d, m, mu, hk, fl, nc, cd, checked, forced, &bs)) break;
+        if (scores_out) scores_out[checked] = (float)bs;
+        // corrected pick: re-run (same engine as the TED) with picks 0..ts forced
         CK(cudaMemsetAsync(T.nflag, 0, sizeof(int), st));
-        run_ted(T, X, N, d, ctx->params.gamma, ctx->kernel, m, mu, keys, true, false, true, T.nflag, forced.data(),
-                ts + 1);
+        run_ted(T, X, N, d, ctx->params.gamma, ctx->kernel, m, mu, keys, true, false, T.last_packed, T.nflag,
+                forced.data(), (int)forced.size());
         CK(cudaStreamSynchronize(st));      // `forced` (pageable) must outlive the copy
     }
 }
@@ -1238,7 +1254,7 @@ bool small_k4_refine(bted_ctx* ctx, cudaStream_t st, const float* X, int ninst, 
         LAUNCHED(1);
     };
     std::vector<int> nf(ctx->k4pin, ctx->k4pin + ninst);
-    std::vector<unsigned long long> hk(m);
+    std::vector<unsigned long long> hk(m), forced;
     std::vector<int> fl(m), nc(m);
     std::vector<uint32_t> cd((size_t)m * kMC);
     for (int k = 0; k < ninst; ++k) {
@@ -1253,36 +1269,16 @@ bool small_k4_refine(bted_ctx* ctx, cudaStream_t st, const float* X, int ninst, 
             CK(cudaMemcpyAsync(cd.data(), ctx->kcand + (size_t)k * m * kMC, sizeof(uint32_t) * cd.size(),
                                cudaMemcpyDeviceToHost, st));
             CK(cudaStreamSynchronize(st));
-            bool rerun = false;
-            for (int ts = checked + 1; ts < m && !rerun; ++ts) {
-                if (!fl[ts] || nc[ts] < 2) continue;
-                std::vector<uint32_t> S(ts), Cs;
-                for (int q = 0; q < ts; ++q) S[q] = 0xFFFFFFFFu - (uint32_t)(hk[q] & 0xFFFFFFFFull);
-                for (int c = 0; c < nc[ts]; ++c) Cs.push_back(cd[(size_t)ts * kMC + c]);
-                std::sort(Cs.begin(), Cs.end());
-                uint32_t best = 0;
-                double bs = 0.0;
-                refine_step(ctx, st, Xk, N, d, S, Cs, mu, &best, &bs);
-                ctx->refined_steps++;
-                checked = ts;
-                const uint32_t pick = 0xFFFFFFFFu - (uint32_t)(hk[ts] & 0xFFFFFFFFull);
-                if (best == pick) continue;
-                ctx->corrected_steps++;
-                changed = true;
-                std::vector<unsigned long long> forced(ts + 1);
-                for (int q = 0; q < ts; ++q) forced[q] = hk[q] | bted::rf::kForced;
-                forced[ts] = host_pack_key((float)bs, best) | bted::rf::kForced;
-                CK(cudaMemcpyAsync(ctx->kforced, forced.data(), sizeof(unsigned long long) * (ts + 1),
-                                   cudaMemcpyHostToDevice, st));
-                // the single-instance re-run writes its top-2 to the scratch tail
-                launch_small(Xk, 1, N, d, ctx->params.gamma, ctx->kernel, m, mu, kk, err, st, rerun_top2,
-                             ctx->kforced, ts + 1);
-                CK(cudaMemsetAsync(ctx->knflag + k, 0, sizeof(int), st));
-                check(k, rerun_top2, nU1);
-                CK(cudaStreamSynchronize(st));      // `forced` (pageable) must outlive the copy
-                rerun = true;
-            }
-            if (!rerun) break;
+            if (!k4_next_correction(ctx, st, Xk, N, d, m, mu, hk, fl, nc, cd, checked, forced)) break;
+            changed = true;
+            CK(cudaMemcpyAsync(ctx->kforced, forced.data(), sizeof(unsigned long long) * forced.size(),
+                               cudaMemcpyHostToDevice, st));
+            // the single-instance re-run writes its top-2 to the scratch tail
+            launch_small(Xk, 1, N, d, ctx->params.gamma, ctx->kernel, m, mu, kk, err, st, rerun_top2, ctx->kforced,
+                         (int)forced.size());
+            CK(cudaMemsetAsync(ctx->knflag + k, 0, sizeof(int), st));
+            check(k, rerun_top2, nU1);
+            CK(cudaStreamSynchronize(st));      // `forced` (pageable) must outlive the copy
         }
     }
     return changed;
@@ -1868,23 +1864,11 @@ bted_status bted_ishard_refine(bted_ctx* ctx, int32_t m, float mu, const uint64_
         CK(cudaMemcpyAsync(nc.data(), T.ncand, sizeof(int) * m, cudaMemcpyDeviceToHost, st));
         CK(cudaMemcpyAsync(cd.data(), T.cand, sizeof(uint32_t) * cd.size(), cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
-        for (int ts = 0; ts < m; ++ts) {
-            if (!fl[ts] || nc[ts] < 2) continue;
-            std::vector<uint32_t> S(ts), C;
-            for (int k = 0; k < ts; ++k) S[k] = 0xFFFFFFFFu - (uint32_t)(hk[k] & 0xFFFFFFFFull);
-            for (int c = 0; c < nc[ts]; ++c) C.push_back(cd[(size_t)ts * bted::rf::kMaxCand + c]);
-            std::sort(C.begin(), C.end());
-            uint32_t best = 0;
-            double bs = 0.0;
-            refine_step(ctx, st, ctx->X, ctx->N, ctx->d, S, C, mu, &best, &bs);
-            ctx->refined_steps++;
-            const uint32_t pick = 0xFFFFFFFFu - (uint32_t)(hk[ts] & 0xFFFFFFFFull);
-            if (best == pick) continue;
-            ctx->corrected_steps++;
-            for (int k = 0; k < ts; ++k) forced_host[k] = hk[k] | bted::rf::kForced;
-            forced_host[ts] = host_pack_key((float)bs, best) | bted::rf::kForced;
-            *nforced = ts + 1;
-            break;
+        std::vector<unsigned long long> forced;
+        int checked = -1;
+        if (k4_next_correction(ctx, st, ctx->X, ctx->N, ctx->d, m, mu, hk, fl, nc, cd, checked, forced)) {
+            for (size_t q = 0; q < forced.size(); ++q) forced_host[q] = forced[q];
+            *nforced = (int32_t)forced.size();
         }
         return BTED_OK;
     });
