@@ -81,8 +81,8 @@ typedef enum {
                                    default three kernels per step (factor column, K.l pass, scores) */
 #define BTED_FLAG_NO_REFINE 128u /* disable K4: near ties (fp32 scores within 2e-5 of the best) are
                                    otherwise re-scored exactly in fp64 from the features and the
-                                   exact argmax taken (every single-GPU engine and the tile-sharded
-                                   engine; not the row-shard API)                               */
+                                   exact argmax taken (every single-GPU engine, the tile-sharded
+                                   engine and the row-shard API's symmetric mode)               */
 #define BTED_FLAG_TIMING   2u   /* record CUDA events around K1 and the K2 loop of every batch
                                    TED on the ctx stream; read with bted_get_stats()          */
 
@@ -265,6 +265,23 @@ int64_t     bted_ishard_qlen(const bted_ctx* shard);
  * Errors: EINVAL, ECUDA, ESTATE. */
 bted_status bted_ishard_refine(bted_ctx* shard, int32_t m, float mu, const uint64_t* keys_dev,
                                uint64_t* forced_host, int32_t* nforced);
+/*
+ * K4 near-tie refinement for the row-sharded TED (symmetric norm mode; steps
+ * t < 256): after the loop, bted_shard_nearties lists this band's candidates of
+ * every step whose fp32 score lies within 2e-5 of the global pick keys[t]
+ * (cand_dev: device u32 [m][32], ncand_dev: device i32 [m]); the caller
+ * all-gathers both over the ranks and calls bted_shard_refine with the host
+ * copies (cand_all [nranks][m][32], ncand_all [nranks][m]): the first step
+ * whose exact fp64 argmax (from the replicated features) differs from the pick
+ * gives forced_host[0 .. *nforced) (flagged keys; 0 = the selection stands).
+ * Every rank computes the same answer; re-run the loop with keys preset to
+ * them (zeros after) and repeat.  Errors: EINVAL, ECUDA, ESTATE.
+ */
+bted_status bted_shard_nearties(bted_ctx* shard, int32_t m, const uint64_t* keys_dev, uint32_t* cand_dev,
+                                int32_t* ncand_dev);
+bted_status bted_shard_refine(bted_ctx* shard, int32_t m, float mu, const uint64_t* keys_dev,
+                              const uint32_t* cand_all, const int32_t* ncand_all, int32_t nranks,
+                              uint64_t* forced_host, int32_t* nforced);
 /* Leading dimension (floats) a pivot buffer must have: pivot_dev[N..ld) must be 0. */
 int64_t     bted_shard_ld(const bted_ctx* shard);
 /* Sticky device error flag of the shard (BTED_ENUMERIC if a NaN score was seen). */

@@ -69,6 +69,8 @@ _SIGS = {
     "bted_shard_colnorm": (ctypes.c_int, [_vp, _i32, _f32, _vp, _vp, _vp]),
     "bted_shard_scores": (ctypes.c_int, [_vp, _i32, _f32, _vp, _vp]),
     "bted_shard_ld": (_i64, [_vp]),
+    "bted_shard_nearties": (ctypes.c_int, [_vp, _i32, _vp, _vp, _vp]),
+    "bted_shard_refine": (ctypes.c_int, [_vp, _i32, _f32, _vp, _vp, _vp, _i32, _vp, ctypes.POINTER(_i32)]),
     "bted_ishard_create": (ctypes.c_int, [_vp, _i64, _i32, ctypes.c_int, _i32, _i32, ctypes.POINTER(bted_params),
                                           ctypes.POINTER(_vp)]),
     "bted_ishard_head": (ctypes.c_int, [_vp, _i32, _f32, _vp]),
@@ -235,6 +237,22 @@ def bted_shard_colnorm(ctx: int, t: int, mu: float, pivot_dev, keys_dev, colnorm
 
 def bted_shard_scores(ctx: int, t: int, mu: float, colnorm_dev: int, keys_dev: int):
     check(lib().bted_shard_scores(ctx, int(t), float(mu), colnorm_dev, keys_dev))
+
+
+def bted_shard_nearties(ctx: int, m: int, keys_dev: int, cand_dev: int, ncand_dev: int):
+    check(lib().bted_shard_nearties(ctx, int(m), keys_dev, cand_dev, ncand_dev))
+
+
+def bted_shard_refine(ctx: int, m: int, mu: float, keys_dev: int, cand_all: np.ndarray, ncand_all: np.ndarray,
+                      nranks: int) -> np.ndarray:
+    """K4 for the row-sharded TED: [] if the selection stands, else the keys to preset (u64)."""
+    cand_all = np.ascontiguousarray(cand_all, dtype=np.uint32)
+    ncand_all = np.ascontiguousarray(ncand_all, dtype=np.int32)
+    forced = np.zeros(int(m), dtype=np.uint64)
+    n = _i32(0)
+    check(lib().bted_shard_refine(ctx, int(m), float(mu), keys_dev, _ptr(cand_all), _ptr(ncand_all), int(nranks),
+                                  _ptr(forced), ctypes.byref(n)))
+    return forced[: n.value]
 
 
 def bted_shard_ld(ctx: int) -> int:

@@ -1648,8 +1648,10 @@ bted_status bted_shard_gram(bted_ctx* ctx, float mu, uint64_t* keys_dev) {
         T.last_buf = 0;
         launch_transpose(T, ctx->X, ctx->N, ctx->d);
         CK(cudaMemsetAsync(T.sel, 0, (size_t)rows, T.stream));
+        // K4: per-CTA top-2 keys of the first kMaxM steps (bted_shard_nearties / bted_shard_refine)
+        if (T.refine) T.reserve_refine((rows + kRowsPerK2Cta - 1) / kRowsPerK2Cta * 32, bted::im::kMaxM);
         launch_gram(T, ctx->N, ctx->d, ctx->row0, rows, ctx->params.gamma, ctx->kernel, mu,
-                    reinterpret_cast<unsigned long long*>(keys_dev));
+                    reinterpret_cast<unsigned long long*>(keys_dev), T.refine ? T.top2 : nullptr);
         return BTED_OK;
     });
 }
@@ -1661,7 +1663,8 @@ bted_status bted_shard_step(bted_ctx* ctx, int32_t t, float mu, const float* piv
     return guarded(ctx, [&]() -> bted_status {
         Ted& T = ctx->ted;
         const int64_t rows = ctx->row1 - ctx->row0;
-        launch_step(T, ctx->N, ctx->row0, rows, t, mu, pivot_dev, reinterpret_cast<unsigned long long*>(keys_dev));
+        launch_step(T, ctx->N, ctx->row0, rows, t, mu, pivot_dev, reinterpret_cast<unsigned long long*>(keys_dev),
+                    (T.refine && T.top2 && t < bted::im::kMaxM) ? T.top2 : nullptr);
         T.last_buf = t & 1;
         return BTED_OK;
     });
@@ -1868,6 +1871,63 @@ bted_status bted_ishard_refine(bted_ctx* ctx, int32_t m, float mu, const uint64_
         int checked = -1;
         if (k4_next_correction(ctx, st, ctx->X, ctx->N, ctx->d, m, mu, hk, fl, nc, cd, checked, forced)) {
             for (size_t q = 0; q < forced.size(); ++q) forced_host[q] = forced[q];
+            *nforced = (int32_t)forced.size();
+        }
+        return BTED_OK;
+    });
+}
+
+bted_status bted_shard_nearties(bted_ctx* ctx, int32_t m, const uint64_t* keys_dev, uint32_t* cand_dev,
+                                int32_t* ncand_dev) {
+    if (!ctx || !keys_dev || !cand_dev || !ncand_dev || !ctx->is_shard || m < 1) {
+        set_error("bad shard_nearties arguments"); return BTED_EINVAL;
+    }
+    return guarded(ctx, [&]() -> bted_status {
+        Ted& T = ctx->ted;
+        const int mm = std::min<int32_t>(m, bted::im::kMaxM);
+        CK(cudaMemsetAsync(ncand_dev, 0, sizeof(int32_t) * m, T.stream));
+        if (!T.refine || !T.top2) return BTED_OK;
+        bted::rf::shard_neartie_kernel<<<mm, 256, 0, T.stream>>>(
+            T.top2, T.last_nC, reinterpret_cast<const unsigned long long*>(keys_dev), bted::rf::kTau, cand_dev,
+            reinterpret_cast<int*>(ncand_dev));
+        LAUNCHED(1);
+        return BTED_OK;
+    });
+}
+
+bted_status bted_shard_refine(bted_ctx* ctx, int32_t m, float mu, const uint64_t* keys_dev, const uint32_t* cand_all,
+                              const int32_t* ncand_all, int32_t nranks, uint64_t* forced_host, int32_t* nforced) {
+    if (!ctx || !keys_dev || !cand_all || !ncand_all || !forced_host || !nforced || !ctx->is_shard || m < 1 ||
+        nranks < 1 || !mu_ok(mu)) {
+        set_error("bad shard_refine arguments"); return BTED_EINVAL;
+    }
+    *nforced = 0;
+    return guarded(ctx, [&]() -> bted_status {
+        Ted& T = ctx->ted;
+        if (!T.refine) return BTED_OK;
+        const size_t kMC = bted::rf::kMaxCand;
+        std::vector<unsigned long long> hk(m), forced;
+        CK(cudaMemcpyAsync(hk.data(), keys_dev, sizeof(unsigned long long) * m, cudaMemcpyDeviceToHost, T.stream));
+        CK(cudaStreamSynchronize(T.stream));
+        // every rank's band candidates of each step, merged (sorted, unique, at most kMaxCand)
+        std::vector<int> fl(m, 0), nc(m, 0);
+        std::vector<uint32_t> cd((size_t)m * kMC);
+        for (int t = 0; t < m; ++t) {
+            std::vector<uint32_t> c;
+            for (int r = 0; r < nranks; ++r) {
+                const int n = std::min<int>(ncand_all[(size_t)r * m + t], (int)kMC);
+                for (int q = 0; q < n; ++q) c.push_back(cand_all[((size_t)r * m + t) * kMC + q]);
+            }
+            std::sort(c.begin(), c.end());
+            c.erase(std::unique(c.begin(), c.end()), c.end());
+            if (c.size() > kMC) c.resize(kMC);
+            fl[t] = c.size() >= 2;
+            nc[t] = (int)c.size();
+            std::copy(c.begin(), c.end(), cd.begin() + (size_t)t * kMC);
+        }
+        int checked = -1;
+        if (k4_next_correction(ctx, T.stream, ctx->X, ctx->N, ctx->d, m, mu, hk, fl, nc, cd, checked, forced)) {
+            std::copy(forced.begin(), forced.end(), forced_host);
             *nforced = (int32_t)forced.size();
         }
         return BTED_OK;

@@ -89,6 +89,32 @@ neartie_check_kernel(const unsigned long long* __restrict__ top2, int nC, const 
     }
 }
 
+// Row-shard K4 (bted_shard_nearties): per step t, this band's candidates within
+// tau of the GLOBAL pick keys[t] (already all-reduced), from the band's per-CTA
+// top-2 keys; a forced (preset) step lists none.  One CTA per step.
+__global__ void __launch_bounds__(256)
+shard_neartie_kernel(const unsigned long long* __restrict__ top2, int nC, const unsigned long long* __restrict__ keys,
+                     float tau, uint32_t* __restrict__ cand, int* __restrict__ ncand) {
+    __shared__ int cnt;
+    const int t = blockIdx.x, tid = threadIdx.x;
+    const unsigned long long kt = keys[t];
+    if (tid == 0) cnt = 0;
+    __syncthreads();
+    if (!(kt & kForced) && kt != 0ull) {
+        const float lim = key_score(kt) * (1.f - tau);
+        const unsigned long long* p = top2 + (int64_t)t * nC * 2;
+        for (int q = tid; q < 2 * nC; q += 256) {
+            const unsigned long long k = p[q];
+            if (k != 0ull && key_score(k) >= lim) {
+                const int pos = atomicAdd(&cnt, 1);
+                if (pos < kMaxCand) cand[(int64_t)t * kMaxCand + pos] = key_index(k);
+            }
+        }
+    }
+    __syncthreads();
+    if (tid == 0) ncand[t] = min(cnt, kMaxCand);
+}
+
 // G[j][i] = k(x_i, x_{cols[j]}) in fp64 (direct difference; reading A1), i < N.
 __global__ void refine_cols_kernel(const float* __restrict__ X, int32_t N, int32_t d, double gamma, int32_t linear,
                                    const uint32_t* __restrict__ cols, double* __restrict__ G) {

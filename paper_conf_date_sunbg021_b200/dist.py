@@ -127,6 +127,12 @@ class LibShard:
     def step(self, t, mu, pivot: torch.Tensor, keys: torch.Tensor):
         L.bted_shard_step(self.ctx, t, mu, pivot.data_ptr(), keys.data_ptr())
 
+    def nearties(self, m, keys: torch.Tensor, cand: torch.Tensor, ncand: torch.Tensor):
+        L.bted_shard_nearties(self.ctx, m, keys.data_ptr(), cand.data_ptr(), ncand.data_ptr())
+
+    def refine(self, m, mu, keys: torch.Tensor, cand_all: np.ndarray, ncand_all: np.ndarray, nranks: int):
+        return L.bted_shard_refine(self.ctx, m, mu, keys.data_ptr(), cand_all, ncand_all, nranks)
+
     def colnorm(self, t, mu, pivot, keys, colnorm: torch.Tensor):
         L.bted_shard_colnorm(self.ctx, t, mu, pivot.data_ptr() if pivot is not None else None,
                              keys.data_ptr() if keys is not None else None, colnorm.data_ptr())
@@ -184,11 +190,13 @@ class ShardedTed:
             self.be.scores(t, mu, self.cn, keys)
             self.comm.allreduce_max_(keys[t:t + 1])               # s_{t+1}
 
-    def _loop(self, keys: torch.Tensor, m: int, mu: float):
+    def _loop(self, keys: torch.Tensor, m: int, mu: float, preset=None):
         if self.norm_mode == "literal":
             return self._loop_literal(keys, m, mu)
         P = self.comm.world
         keys.zero_()
+        if preset is not None:                                    # K4: forced picks win every max
+            keys[: len(preset)].copy_(torch.from_numpy(preset.view(np.int64)))
         self.be.gram(mu, keys)                                    # l.1 + first l.3 on the band
         self.comm.allreduce_max_(keys[0:1])                       # global argmax s_1 (8 B)
         gathered = self.pivot[: P * self.bandB]
@@ -216,9 +224,27 @@ class ShardedTed:
             else:
                 keys = torch.zeros(m, dtype=torch.int64, device=self.device)
                 self._loop(keys, m, mu)
+            if self.norm_mode == "symmetric" and hasattr(self.be, "nearties"):
+                for _ in range(m):                                # K4 (identical decision on every rank)
+                    forced = self._k4(keys, m, mu)
+                    if len(forced) == 0:
+                        break
+                    keys = torch.zeros(m, dtype=torch.int64, device=self.device)
+                    self._loop(keys, m, mu, preset=forced)
             host = keys.cpu().numpy().view(np.uint64)
         self.be.check()
         return L.decode_keys(host)
+
+    def _k4(self, keys: torch.Tensor, m: int, mu: float):
+        P = self.comm.world
+        cand = torch.zeros((m, 32), dtype=torch.int32, device=self.device)
+        ncand = torch.zeros(m, dtype=torch.int32, device=self.device)
+        self.be.nearties(m, keys, cand, ncand)
+        cand_all = torch.empty((P * m, 32), dtype=torch.int32, device=self.device)
+        ncand_all = torch.empty(P * m, dtype=torch.int32, device=self.device)
+        self.comm.allgather_(cand_all, cand)
+        self.comm.allgather_(ncand_all, ncand)
+        return self.be.refine(m, mu, keys, cand_all.cpu().numpy().view(np.uint32), ncand_all.cpu().numpy(), P)
 
 
 # ------------------------------------------- 3. tile-sharded implicit TED
@@ -369,7 +395,7 @@ def isharded_select_loopback(X: np.ndarray, gamma: float, P: int, m: int, mu: fl
 # ------------------------------------------------ loopback (P shards, 1 GPU)
 def sharded_select_loopback(X: np.ndarray, gamma: float, P: int, m: int, mu: float, device: torch.device,
                             stream: torch.cuda.Stream, kernel: int = L.BTED_KERNEL_RBF,
-                            norm_mode: str = "symmetric"):
+                            norm_mode: str = "symmetric", stats: dict | None = None):
     """The ShardedTed exchange with P logical shards on ONE GPU; the
     collectives are emulated by a device copy, a max and (literal norm mode)
     a sum over the shards in rank order.  Exercises the sharded kernels and
@@ -397,30 +423,50 @@ def sharded_select_loopback(X: np.ndarray, gamma: float, P: int, m: int, mu: flo
                 for r in range(P):
                     shards[r].scores(t, mu, tot, keys[r])
 
-            for r in range(P):
-                if literal:
-                    shards[r].gram(mu, scratch[r])
-                    shards[r].colnorm(0, mu, None, None, cn[r])
-                else:
-                    shards[r].gram(mu, keys[r])
-            if literal:
-                scores(0)
-            keys[:, 0] = keys[:, 0].max()
-            for t in range(1, m):
-                for r in range(P):
-                    shards[r].pivot_column(t - 1, keys[r], cols[r])
-                pivot[: P * Bw].copy_(cols.reshape(-1))
+            def rerun(preset=None):
+                keys.zero_()
+                if preset is not None:
+                    keys[:, : len(preset)] = torch.from_numpy(preset.view(np.int64)).to(device)
                 for r in range(P):
                     if literal:
-                        shards[r].colnorm(t, mu, pivot, keys[r], cn[r])
+                        shards[r].gram(mu, scratch[r])
+                        shards[r].colnorm(0, mu, None, None, cn[r])
                     else:
-                        shards[r].step(t, mu, pivot, keys[r])
+                        shards[r].gram(mu, keys[r])
                 if literal:
-                    scores(t)
-                keys[:, t] = keys[:, t].max()
+                    scores(0)
+                keys[:, 0] = keys[:, 0].max()
+                for t in range(1, m):
+                    for r in range(P):
+                        shards[r].pivot_column(t - 1, keys[r], cols[r])
+                    pivot[: P * Bw].copy_(cols.reshape(-1))
+                    for r in range(P):
+                        if literal:
+                            shards[r].colnorm(t, mu, pivot, keys[r], cn[r])
+                        else:
+                            shards[r].step(t, mu, pivot, keys[r])
+                    if literal:
+                        scores(t)
+                    keys[:, t] = keys[:, t].max()
+
+            rerun()
+            if not literal:                                       # K4, as ShardedTed.select
+                for _ in range(m):
+                    cand = torch.zeros((P, m, 32), dtype=torch.int32, device=device)
+                    ncand = torch.zeros((P, m), dtype=torch.int32, device=device)
+                    for r in range(P):
+                        shards[r].nearties(m, keys[r], cand[r], ncand[r])
+                    ca, na = cand.cpu().numpy().view(np.uint32), ncand.cpu().numpy()
+                    forced = [shards[r].refine(m, mu, keys[r], ca, na, P) for r in range(P)]
+                    assert all(np.array_equal(f, forced[0]) for f in forced), "shards disagree on K4"
+                    if len(forced[0]) == 0:
+                        break
+                    rerun(forced[0])
             host = keys[0].cpu().numpy().view(np.uint64)
         for s in shards:
             s.check()
+        if stats is not None:
+            stats.update(L.bted_get_stats(shards[0].ctx))
         return L.decode_keys(host)
     finally:
         for s in shards:

@@ -373,6 +373,26 @@ def test_tile_sharded_implicit_k4_exact_ties(P):
     print(f"ishard K4 P={P}: refined {st_k4['refined_steps']}, corrected {st_k4['corrected_steps']}")
 
 
+@pytest.mark.parametrize("P", [1, 2, 3])
+def test_row_sharded_k4_exact_ties(P):
+    """Row bands (symmetric mode) with K4: near-tie candidates of every band,
+    gathered over the shards, re-scored in fp64; P2 at the fp64 gap."""
+    import torch
+    from paper_conf_date_sunbg021_b200.dist import sharded_select_loopback
+    X = uniform_pool(1800, 8, 53)
+    Xn = X[::4].copy()
+    Xn[:, 1] += np.float32(2e-4)                             # near duplicates: fp64 gaps below fp32 noise
+    X = np.concatenate([X, Xn], axis=0)
+    g = median_gamma(X, 53)
+    dev = torch.device("cuda", 0)
+    st = torch.cuda.Stream(dev)
+    k4 = {}
+    idx, sc = sharded_select_loopback(X, g, P, 200, MU, dev, st, stats=k4)
+    assert k4["refined_steps"] > 0
+    check_ted(idx, sc, dense.ted(X, g, MU, 200, forced=idx), f"rowshard-k4 P={P}", gap_exact=GAP_K4)
+    print(f"row-shard K4 P={P}: refined {k4['refined_steps']}, corrected {k4['corrected_steps']}")
+
+
 def test_launch_counter_counts_kernels():
     X = knob(300)
     before = bt.bted_kernel_launches()
