@@ -266,8 +266,9 @@ int64_t     bted_ishard_qlen(const bted_ctx* shard);
 bted_status bted_ishard_refine(bted_ctx* shard, int32_t m, float mu, const uint64_t* keys_dev,
                                uint64_t* forced_host, int32_t* nforced);
 /*
- * K4 near-tie refinement for the row-sharded TED (symmetric norm mode; steps
- * t < 256): after the loop, bted_shard_nearties lists this band's candidates of
+ * K4 near-tie refinement for the row-sharded TED (both norm modes: the
+ * band's top-2 keys come from bted_shard_gram/step, or from bted_shard_scores
+ * in the literal mode; steps t < 256): after the loop, bted_shard_nearties lists this band's candidates of
  * every step whose fp32 score lies within 2e-5 of the global pick keys[t]
  * (cand_dev: device u32 [m][32], ncand_dev: device i32 [m]); the caller
  * all-gathers both over the ranks and calls bted_shard_refine with the host

@@ -1718,10 +1718,18 @@ bted_status bted_shard_scores(bted_ctx* ctx, int32_t t, float mu, const float* c
     return guarded(ctx, [&]() -> bted_status {
         Ted& T = ctx->ted;
         const int32_t rows = (int32_t)(ctx->row1 - ctx->row0);
-        const unsigned g = (unsigned)std::min<int64_t>((rows + 255) / 256, 1184);
+        unsigned g = (unsigned)std::min<int64_t>((rows + 255) / 256, 1184);
+        // K4: one CTA per top-2 slot pair of the step (T.last_nC, set by bted_shard_gram),
+        // so bted_shard_nearties reads the literal mode's keys like the symmetric mode's
+        unsigned long long* top2 = nullptr;
+        if (T.refine && T.top2 && t < bted::im::kMaxM && T.last_nC > 0) {
+            g = (unsigned)T.last_nC;
+            top2 = T.top2 + (int64_t)t * T.last_nC * 2;
+        }
         bted::colnorm_scores_kernel<<<g, 256, 0, T.stream>>>(T.K[t & 1], ld_for(ctx->N), (int32_t)ctx->row0, rows,
                                                              colnorm_dev, mu, T.sel,
-                                                             reinterpret_cast<unsigned long long*>(keys_dev), t, T.err);
+                                                             reinterpret_cast<unsigned long long*>(keys_dev), t, T.err,
+                                                             top2);
         LAUNCHED(1);
         return BTED_OK;
     });

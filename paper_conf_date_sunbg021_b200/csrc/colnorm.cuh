@@ -115,15 +115,19 @@ __global__ void colnorm_reduce_kernel(const float* __restrict__ partial, int32_t
 __global__ void __launch_bounds__(256)
 colnorm_scores_kernel(const float* __restrict__ K, int64_t ld, int32_t row0, int32_t nrows,
                       const float* __restrict__ colnorm, float mu, const uint8_t* __restrict__ sel,
-                      unsigned long long* __restrict__ keys, int32_t t, int* __restrict__ err) {
-    unsigned long long best = 0ull;
+                      unsigned long long* __restrict__ keys, int32_t t, int* __restrict__ err,
+                      unsigned long long* __restrict__ top2 = nullptr) {
+    unsigned long long best = 0ull, second = 0ull;           // this thread's two best keys (K4)
     for (int lr = blockIdx.x * blockDim.x + threadIdx.x; lr < nrows; lr += gridDim.x * blockDim.x) {
         const int32_t i = row0 + lr;
         const unsigned long long k =
             score_key(colnorm[i], K[(int64_t)lr * ld + i], mu, (uint32_t)i, sel[lr] != 0, err);
+        second = k > best ? best : (k > second ? k : second);
         best = k > best ? k : best;
     }
-    cta_key_max_to<256>(best, keys + t);
+    // top2 (K4): this CTA's two best keys at top2[2 * blockIdx.x], the layout
+    // bted_shard_nearties reads (one slot pair per CTA of the step)
+    cta_key_max_to<256>(best, keys + t, top2 ? top2 + 2 * (int64_t)blockIdx.x : nullptr, second);
 }
 
 }  // namespace bted

@@ -85,7 +85,8 @@ __device__ __forceinline__ unsigned long long score_key(float g, float diag, flo
 
 // CTA-wide max of one key per thread, then one atomicMax into *dst.  With
 // top2 (K4 near-tie check, refine.cuh) the CTA's two best keys are also
-// written to top2[0..1] (keys are distinct: they carry the row index).
+// written to top2[0..1] (keys are distinct: they carry the row index); key2 is
+// a thread's second-best key when it scored several rows (else 0).
 __device__ __forceinline__ void top2_merge(unsigned long long& b1, unsigned long long& b2, unsigned long long c1,
                                            unsigned long long c2) {
     const unsigned long long hi = b1 > c1 ? b1 : c1, lo = b1 > c1 ? c1 : b1;
@@ -95,9 +96,10 @@ __device__ __forceinline__ void top2_merge(unsigned long long& b1, unsigned long
 }
 template <int kThreads>
 __device__ __forceinline__ void cta_key_max_to(unsigned long long key, unsigned long long* dst,
-                                               unsigned long long* top2 = nullptr) {
+                                               unsigned long long* top2 = nullptr,
+                                               unsigned long long key2 = 0ull) {
     __shared__ unsigned long long red[kThreads / kWarp][2];
-    unsigned long long b1 = key, b2 = 0ull;
+    unsigned long long b1 = key, b2 = key2;
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) {
         const unsigned long long c1 = __shfl_xor_sync(0xffffffffu, b1, off);

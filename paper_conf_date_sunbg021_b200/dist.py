@@ -173,9 +173,11 @@ class ShardedTed:
                 self.cn = torch.zeros(width, dtype=torch.float32, device=device)
                 self.scratch = torch.zeros(1, dtype=torch.int64, device=device)
 
-    def _loop_literal(self, keys: torch.Tensor, m: int, mu: float):
+    def _loop_literal(self, keys: torch.Tensor, m: int, mu: float, preset=None):
         P = self.comm.world
         keys.zero_()
+        if preset is not None:                                    # K4: forced picks win every max
+            keys[: len(preset)].copy_(torch.from_numpy(preset.view(np.int64)))
         self.be.gram(mu, self.scratch)                            # l.1 on the band
         self.be.colnorm(0, mu, None, None, self.cn)               # band part of every column norm
         self.comm.allreduce_sum_(self.cn)                         # ||K_v||^2 (N floats)
@@ -192,7 +194,7 @@ class ShardedTed:
 
     def _loop(self, keys: torch.Tensor, m: int, mu: float, preset=None):
         if self.norm_mode == "literal":
-            return self._loop_literal(keys, m, mu)
+            return self._loop_literal(keys, m, mu, preset)
         P = self.comm.world
         keys.zero_()
         if preset is not None:                                    # K4: forced picks win every max
@@ -224,7 +226,7 @@ class ShardedTed:
             else:
                 keys = torch.zeros(m, dtype=torch.int64, device=self.device)
                 self._loop(keys, m, mu)
-            if self.norm_mode == "symmetric" and hasattr(self.be, "nearties"):
+            if hasattr(self.be, "nearties"):
                 for _ in range(m):                                # K4 (identical decision on every rank)
                     forced = self._k4(keys, m, mu)
                     if len(forced) == 0:
@@ -450,18 +452,18 @@ def sharded_select_loopback(X: np.ndarray, gamma: float, P: int, m: int, mu: flo
                     keys[:, t] = keys[:, t].max()
 
             rerun()
-            if not literal:                                       # K4, as ShardedTed.select
-                for _ in range(m):
-                    cand = torch.zeros((P, m, 32), dtype=torch.int32, device=device)
-                    ncand = torch.zeros((P, m), dtype=torch.int32, device=device)
-                    for r in range(P):
-                        shards[r].nearties(m, keys[r], cand[r], ncand[r])
-                    ca, na = cand.cpu().numpy().view(np.uint32), ncand.cpu().numpy()
-                    forced = [shards[r].refine(m, mu, keys[r], ca, na, P) for r in range(P)]
-                    assert all(np.array_equal(f, forced[0]) for f in forced), "shards disagree on K4"
-                    if len(forced[0]) == 0:
-                        break
-                    rerun(forced[0])
+            # K4, as ShardedTed.select (both norm modes)
+            for _ in range(m):
+                cand = torch.zeros((P, m, 32), dtype=torch.int32, device=device)
+                ncand = torch.zeros((P, m), dtype=torch.int32, device=device)
+                for r in range(P):
+                    shards[r].nearties(m, keys[r], cand[r], ncand[r])
+                ca, na = cand.cpu().numpy().view(np.uint32), ncand.cpu().numpy()
+                forced = [shards[r].refine(m, mu, keys[r], ca, na, P) for r in range(P)]
+                assert all(np.array_equal(f, forced[0]) for f in forced), "shards disagree on K4"
+                if len(forced[0]) == 0:
+                    break
+                rerun(forced[0])
             host = keys[0].cpu().numpy().view(np.uint64)
         for s in shards:
             s.check()

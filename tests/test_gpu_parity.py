@@ -323,7 +323,7 @@ def test_row_sharded_literal_column_norms_vs_oracle(N, P):
     m = 24
     lidx, lsc = sharded_select_loopback(X, g, P, m, MU, dev, st, norm_mode="literal")
     tr = literal.ted(X, g, MU, m, forced=lidx.tolist())
-    check_ted(lidx, lsc, tr, f"literal-colnorm N={N} P={P}")
+    check_ted(lidx, lsc, tr, f"literal-colnorm N={N} P={P}", gap_exact=GAP_K4)
     sidx, ssc = sharded_select_loopback(X, g, P, m, MU, dev, st)
     assert len(set(lidx.tolist())) == m
     np.testing.assert_allclose(lsc, ssc, rtol=1e-5)         # same numbers up to rounding order
@@ -373,10 +373,12 @@ def test_tile_sharded_implicit_k4_exact_ties(P):
     print(f"ishard K4 P={P}: refined {st_k4['refined_steps']}, corrected {st_k4['corrected_steps']}")
 
 
+@pytest.mark.parametrize("norm_mode", ["symmetric", "literal"])
 @pytest.mark.parametrize("P", [1, 2, 3])
-def test_row_sharded_k4_exact_ties(P):
-    """Row bands (symmetric mode) with K4: near-tie candidates of every band,
-    gathered over the shards, re-scored in fp64; P2 at the fp64 gap."""
+def test_row_sharded_k4_exact_ties(P, norm_mode):
+    """Row bands (symmetric mode, and the literal column-norm ablation) with K4:
+    near-tie candidates of every band, gathered over the shards, re-scored in
+    fp64; P2 at the fp64 gap."""
     import torch
     from paper_conf_date_sunbg021_b200.dist import sharded_select_loopback
     X = uniform_pool(1800, 8, 53)
@@ -387,10 +389,10 @@ def test_row_sharded_k4_exact_ties(P):
     dev = torch.device("cuda", 0)
     st = torch.cuda.Stream(dev)
     k4 = {}
-    idx, sc = sharded_select_loopback(X, g, P, 200, MU, dev, st, stats=k4)
+    idx, sc = sharded_select_loopback(X, g, P, 200, MU, dev, st, norm_mode=norm_mode, stats=k4)
     assert k4["refined_steps"] > 0
-    check_ted(idx, sc, dense.ted(X, g, MU, 200, forced=idx), f"rowshard-k4 P={P}", gap_exact=GAP_K4)
-    print(f"row-shard K4 P={P}: refined {k4['refined_steps']}, corrected {k4['corrected_steps']}")
+    check_ted(idx, sc, dense.ted(X, g, MU, 200, forced=idx), f"rowshard-k4-{norm_mode} P={P}", gap_exact=GAP_K4)
+    print(f"row-shard K4 {norm_mode} P={P}: refined {k4['refined_steps']}, corrected {k4['corrected_steps']}")
 
 
 def test_launch_counter_counts_kernels():
