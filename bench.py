@@ -469,7 +469,6 @@ def bench_sharded(args, X, gamma, cfg, comm, dev, world, rank):
     import torch
     import paper_conf_date_sunbg021_b200 as bt
     from paper_conf_date_sunbg021_b200.dist import LibShard, ShardedTed, band
-    from oracle.sampling import sample_batches  # noqa: F401  (not used on the timed path)
     mu = float(np.float32(cfg["mu"]))
     M, m = cfg["M"], cfg["m"]
     # the batch V_0 = the first draw of Alg. 2 l.2, gathered on every rank by the library
