@@ -463,9 +463,12 @@ def bench_wholemodel(args, comm, dev, world, rank, local):
 
 
 def bench_sharded(args, X, gamma, cfg, comm, dev, world, rank):
-    """config 'oversized' on N > 1 GPUs: ONE batch of M points, K row-sharded
-    (dense bands) over the ranks; per step an 8-byte MAX all-reduce of the
-    packed argmax key and an all-gather of column s (= row s) -- dist.ShardedTed."""
+    """config 'oversized' on N > 1 GPUs: ONE batch of M points over the ranks.
+    Default (--shard-engine implicit): the packed Gram tiles split k mod P, one
+    all-reduce(SUM) of q = K l per step -- dist.ShardedImplicitTed.  With
+    --shard-engine dense: K row-sharded in bands, per step an 8-byte MAX
+    all-reduce of the packed argmax key and an all-gather of column s (= row s)
+    -- dist.ShardedTed (--norm-mode literal adds the column-norm all-reduce)."""
     import torch
     import paper_conf_date_sunbg021_b200 as bt
     from paper_conf_date_sunbg021_b200.dist import LibShard, ShardedTed, band
