@@ -73,3 +73,24 @@ def test_decode_keys_roundtrip():
         (np.uint64(0xFFFFFFFF) - idx.astype(np.uint64))
     i2, s2 = L.decode_keys(keys)
     assert np.array_equal(i2, idx) and np.array_equal(s2, score)
+
+
+def test_product_path_shares_nothing_with_the_oracle():
+    """The product package (Python binding + CUDA sources) never imports, links
+    or includes anything under oracle/, and the oracle never imports the product
+    package: the two meet only through synth/ inputs and the tests."""
+    pkg = os.path.join(ROOT, "paper_conf_date_sunbg021_b200")
+    bad = []
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                src = open(os.path.join(dirpath, f)).read()
+                if re.search(r"^\s*(from|import)\s+oracle\b|#include\s+[\"<][^\">]*oracle|ted_oracle", src, flags=re.M):
+                    bad.append(f)
+    for f in os.listdir(os.path.join(ROOT, "oracle")):
+        if f.endswith((".py", ".c")):
+            src = open(os.path.join(ROOT, "oracle", f)).read()
+            if re.search(r"^\s*(from|import)\s+paper_conf_date_sunbg021_b200\b|#include\s+[\"<][^\">]*"
+                         r"(paper_conf_date_sunbg021_b200|bted)|libbted", src, flags=re.M):
+                bad.append("oracle/" + f)
+    assert not bad, bad
