@@ -7,11 +7,17 @@
 //
 //   CTA r of a cluster of C owns rows [r*R, r*R+R) of K (dense, ld = N
 //   rounded to 4) in its own smem.  Per step: every CTA copies the pivot row
-//   from its owner's smem (DSMEM), cluster barrier, deflates its rows
+//   from its owner's smem (DSMEM), CTA barrier, deflates its UNSELECTED rows
 //   (k - (a_i p_j)/c with the same instruction as K2 -> bitwise the same
 //   elements), computes the new row norms, scores and its masked argmax
 //   key, writes the key into every CTA's slot (DSMEM), cluster barrier,
-//   each CTA reduces the C keys -> next pivot.  2 cluster barriers per step.
+//   each CTA reduces the C keys -> next pivot.  1 cluster barrier per step.
+//   Selected rows are left as they are: after s is picked, no later pivot,
+//   multiplier a_i = K_is (read from the pivot copy) or unmasked score reads
+//   row s (its entries K_sj live on as K_js in the unselected rows j), so
+//   their values cannot change any result -- and the owner never writes row s
+//   again, so the remote pivot reads need no cluster barrier before the
+//   deflation (they finish before the reader's next exchange barrier).
 //
 // Several TEDs (the B batches) run as independent clusters of one launch.
 #pragma once
@@ -176,16 +182,19 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
         for (int j4 = tid; j4 < L / 4; j4 += kThreads)
             reinterpret_cast<float4*>(piv)[j4] = reinterpret_cast<const float4*>(src)[j4];
         if (owner == rank && tid == 0) sel[s - r0] = 1;
-        csync();                                     // every CTA holds the pivot before rows change
+        __syncthreads();                             // this CTA's pivot copy and sel[] (row s is never
+                                                     // written again, so remote readers need no barrier)
         const float inv_c = __frcp_rn(__fadd_rn(piv[s], mu));
         best_local = 0ull;
         second_local = 0ull;
         for (int base = w; base < nr; base += kWarps * kR) {
             float acc_norm[kR], a[kR];
+            bool act[kR];                            // unselected rows only (selected: see the header)
 #pragma unroll
             for (int h = 0; h < kR; ++h) {
                 const int lr = base + h * kWarps;
                 acc_norm[h] = 0.f;
+                act[h] = lr < nr && sel[lr] == 0;
                 a[h] = lr < nr ? piv[r0 + lr] : 0.f;   // K[i][s] = K[s][i]
             }
             for (int j4 = l; j4 < L / 4; j4 += 32) {
@@ -193,7 +202,7 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
 #pragma unroll
                 for (int h = 0; h < kR; ++h) {
                     const int lr = base + h * kWarps;
-                    if (lr >= nr) continue;
+                    if (!act[h]) continue;
                     float4* row = reinterpret_cast<float4*>(Kb + (size_t)lr * L);
                     float4 kv = row[j4];
                     kv.x = deflate1(kv.x, a[h], pv.x, inv_c);
