@@ -7,17 +7,19 @@
 //
 //   CTA r of a cluster of C owns rows [r*R, r*R+R) of K (dense, ld = N
 //   rounded to 4) in its own smem.  Per step: every CTA copies the pivot row
-//   from its owner's smem (DSMEM), CTA barrier, deflates its UNSELECTED rows
-//   (k - (a_i p_j)/c with the same instruction as K2 -> bitwise the same
-//   elements), computes the new row norms, scores and its masked argmax
-//   key, writes the key into every CTA's slot (DSMEM), cluster barrier,
-//   each CTA reduces the C keys -> next pivot.  1 cluster barrier per step.
-//   Selected rows are left as they are: after s is picked, no later pivot,
+//   from its owner's smem (DSMEM), CTA barrier, deflates its rows except
+//   the pivot row s itself (k - (a_i p_j)/c with the same instruction as K2
+//   -> bitwise the same elements), computes the new row norms, scores and its
+//   masked argmax key, writes the key into every CTA's slot (DSMEM), cluster
+//   barrier, each CTA reduces the C keys -> next pivot.  1 cluster barrier
+//   per step.  Row s may miss its update: after s is picked no later pivot,
 //   multiplier a_i = K_is (read from the pivot copy) or unmasked score reads
-//   row s (its entries K_sj live on as K_js in the unselected rows j), so
-//   their values cannot change any result -- and the owner never writes row s
-//   again, so the remote pivot reads need no cluster barrier before the
-//   deflation (they finish before the reader's next exchange barrier).
+//   row s (its entries K_sj live on as K_js in the unselected rows j), so its
+//   values cannot change any result -- and since the owner does not write row
+//   s in the step that reads it remotely, those reads need no cluster barrier
+//   before the deflation (they finish before the reader's exchange barrier,
+//   which the owner passes before it next writes row s).  With C = 1 there
+//   are no remote readers and every row is updated.
 //
 // Several TEDs (the B batches) run as independent clusters of one launch.
 #pragma once
@@ -189,12 +191,12 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
         second_local = 0ull;
         for (int base = w; base < nr; base += kWarps * kR) {
             float acc_norm[kR], a[kR];
-            bool act[kR];                            // unselected rows only (selected: see the header)
+            bool act[kR];                            // all rows but the pivot row (see the header)
 #pragma unroll
             for (int h = 0; h < kR; ++h) {
                 const int lr = base + h * kWarps;
                 acc_norm[h] = 0.f;
-                act[h] = lr < nr && sel[lr] == 0;
+                act[h] = lr < nr && (C == 1 || r0 + lr != s);   // the pivot row: read remotely now
                 a[h] = lr < nr ? piv[r0 + lr] : 0.f;   // K[i][s] = K[s][i]
             }
             for (int j4 = l; j4 < L / 4; j4 += 32) {
