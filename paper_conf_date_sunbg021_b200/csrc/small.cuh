@@ -102,6 +102,11 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
         if (k > b1) { b2 = b1; b1 = k; } else if (k > b2) { b2 = k; }
     };
     auto put_top2 = [&](int t, unsigned long long b1, unsigned long long b2) {
+        if (top2) {                                            // lanes 0..kR-1 hold partial top-2s
+#pragma unroll
+            for (int off = 1; off < kR; off <<= 1)
+                top2_merge(b1, b2, __shfl_xor_sync(0xffffffffu, b1, off), __shfl_xor_sync(0xffffffffu, b2, off));
+        }
         if (top2 && l == 0) {
             unsigned long long* p = top2 + ((int64_t)t * nU + rank * kWarps + w) * 2;
             p[0] = b1;
@@ -221,14 +226,15 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
             float g[kR];
 #pragma unroll
             for (int h = 0; h < kR; ++h) g[h] = warp_sum(acc_norm[h]);
-            if (l == 0) {
+            if (l < kR) {                            // lane h scores row h of the group
+                float gl = g[0];
 #pragma unroll
-                for (int h = 0; h < kR; ++h) {
-                    const int lr = base + h * kWarps;
-                    if (lr >= nr) continue;
+                for (int h = 1; h < kR; ++h) gl = l == h ? g[h] : gl;
+                const int lr = base + l * kWarps;
+                if (lr < nr) {
                     const int i = r0 + lr;
                     const bool masked = sel[lr] != 0 || i == s;
-                    const unsigned long long k = score_key(g[h], Kb[(size_t)lr * L + i], mu, (uint32_t)i, masked, err);
+                    const unsigned long long k = score_key(gl, Kb[(size_t)lr * L + i], mu, (uint32_t)i, masked, err);
                     note(k, best_local, second_local);
                 }
             }
