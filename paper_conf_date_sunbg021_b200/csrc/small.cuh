@@ -158,11 +158,23 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
     // the slots alternate with the step parity, so the next step's writes
     // cannot race this step's reads)
     auto exchange = [&](unsigned long long key, int parity) -> unsigned long long {
-        key = warp_max_u64(key);
+        // only lanes 0..kR-1 ever hold a key (the scoring lanes), so two
+        // butterfly levels bring the warp's max to lane 0
+        static_assert(kR <= 4 && kWarps <= 32 && (kWarps & (kWarps - 1)) == 0, "exchange levels");
+#pragma unroll
+        for (int off = 1; off < 4; off <<= 1) {
+            const unsigned long long o = __shfl_xor_sync(0xffffffffu, key, off);
+            key = o > key ? o : key;
+        }
         unsigned long long* wr = wred + parity * kWarps;
         if (l == 0) wr[w] = key;
         __syncthreads();
-        unsigned long long v = warp_max_u64(l < kWarps ? wr[l] : 0ull);
+        unsigned long long v = wr[l % kWarps];            // every lane: max of the kWarps slots
+#pragma unroll
+        for (int off = kWarps / 2; off > 0; off >>= 1) {
+            const unsigned long long o = __shfl_xor_sync(0xffffffffu, v, off);
+            v = o > v ? o : v;
+        }
         if constexpr (C == 1) {
             return v;
         } else {
