@@ -39,6 +39,28 @@ constexpr size_t kSmemBudget = 220 * 1024;
 __host__ __device__ __forceinline__ int ldk_for(int N) { return (N + 3) / 4 * 4; }
 __host__ __device__ __forceinline__ int rows_per(int N, int C) { return (N + C - 1) / C; }
 constexpr int kR = 4;                  // rows per warp iteration (independent reduction chains)
+constexpr int kLanePerRow = 32 / kR;   // after warp_sum4: lanes [8h, 8h + 8) hold row h's sum
+static_assert(kR == 4, "warp_sum4 reduces four rows");
+
+// Sums of four per-lane values over the warp with 6 shuffles instead of 4 x 5:
+// the first two levels (offsets 16, 8) each hand half of the still-open rows
+// to the partner, the last three are plain butterflies.  Every row sees the
+// xor-butterfly tree of warp_sum (offsets 16, 8, 4, 2, 1; fp32 add is
+// commutative), so each result is bitwise warp_sum's.  Returns row
+// (l >> 4) * 2 + ((l >> 3) & 1)'s sum, i.e. row l / 8.
+__device__ __forceinline__ float warp_sum4(const float (&v)[4], int l) {
+    const bool up16 = (l & 16) != 0, up8 = (l & 8) != 0;
+    // offset 16: lower lanes keep rows 0, 1; upper lanes keep rows 2, 3
+    const float s0 = up16 ? v[0] : v[2], s1 = up16 ? v[1] : v[3];
+    const float r0 = __shfl_xor_sync(0xffffffffu, s0, 16), r1 = __shfl_xor_sync(0xffffffffu, s1, 16);
+    const float a = __fadd_rn(up16 ? v[2] : v[0], r0), b = __fadd_rn(up16 ? v[3] : v[1], r1);
+    // offset 8: keep the even row (lower) or the odd row (upper)
+    const float r = __shfl_xor_sync(0xffffffffu, up8 ? a : b, 8);
+    float c = __fadd_rn(up8 ? b : a, r);
+#pragma unroll
+    for (int off = 4; off > 0; off >>= 1) c = __fadd_rn(c, __shfl_xor_sync(0xffffffffu, c, off));
+    return c;
+}
 // dynamic smem of one CTA: band + pivot row + key slots + warp keys + sel
 __host__ __device__ __forceinline__ size_t smem_core(int N, int C) {
     const size_t R = (size_t)rows_per(N, C), L = (size_t)ldk_for(N);
@@ -102,9 +124,9 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
         if (k > b1) { b2 = b1; b1 = k; } else if (k > b2) { b2 = k; }
     };
     auto put_top2 = [&](int t, unsigned long long b1, unsigned long long b2) {
-        if (top2) {                                            // lanes 0..kR-1 hold partial top-2s
+        if (top2) {                                            // lanes 0, 8, 16, 24 hold partial top-2s
 #pragma unroll
-            for (int off = 1; off < kR; off <<= 1)
+            for (int off = kLanePerRow; off < 32; off <<= 1)
                 top2_merge(b1, b2, __shfl_xor_sync(0xffffffffu, b1, off), __shfl_xor_sync(0xffffffffu, b2, off));
         }
         if (top2 && l == 0) {
@@ -158,11 +180,11 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
     // the slots alternate with the step parity, so the next step's writes
     // cannot race this step's reads)
     auto exchange = [&](unsigned long long key, int parity) -> unsigned long long {
-        // only lanes 0..kR-1 ever hold a key (the scoring lanes), so two
+        // only the scoring lanes 0, 8, 16, 24 ever hold a key, so two
         // butterfly levels bring the warp's max to lane 0
-        static_assert(kR <= 4 && kWarps <= 32 && (kWarps & (kWarps - 1)) == 0, "exchange levels");
+        static_assert(kWarps <= 32 && (kWarps & (kWarps - 1)) == 0, "exchange levels");
 #pragma unroll
-        for (int off = 1; off < 4; off <<= 1) {
+        for (int off = kLanePerRow; off < 32; off <<= 1) {
             const unsigned long long o = __shfl_xor_sync(0xffffffffu, key, off);
             key = o > key ? o : key;
         }
@@ -235,14 +257,9 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
                     acc_norm[h] = __fmaf_rn(kv.w, kv.w, acc_norm[h]);
                 }
             }
-            float g[kR];
-#pragma unroll
-            for (int h = 0; h < kR; ++h) g[h] = warp_sum(acc_norm[h]);
-            if (l < kR) {                            // lane h scores row h of the group
-                float gl = g[0];
-#pragma unroll
-                for (int h = 1; h < kR; ++h) gl = l == h ? g[h] : gl;
-                const int lr = base + l * kWarps;
+            const float gl = warp_sum4(acc_norm, l);  // row l / 8 of the group (kLanePerRow)
+            if ((l & (kLanePerRow - 1)) == 0) {      // lane 8h scores row h of the group
+                const int lr = base + (l / kLanePerRow) * kWarps;
                 if (lr < nr) {
                     const int i = r0 + lr;
                     const bool masked = sel[lr] != 0 || i == s;
