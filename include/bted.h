@@ -320,6 +320,10 @@ typedef struct {
     double   small_ms;       /* their device time                              */
     uint64_t refined_steps;  /* K4: near-tie steps re-scored exactly in fp64   */
     uint64_t corrected_steps;/* K4: of those, steps whose pick changed         */
+    uint64_t full_refined_steps; /* K4: of the refined steps, those whose candidate list
+                                    could be incomplete (a score unit's second key in the
+                                    window, or > 32 candidates): ALL unselected points
+                                    were re-scored in fp64                          */
 } bted_stats;
 bted_status bted_get_stats(bted_ctx* ctx, bted_stats* out);
 bted_status bted_reset_stats(bted_ctx* ctx);

@@ -48,7 +48,8 @@ class bted_stats(ctypes.Structure):
     _fields_ = [("teds", ctypes.c_uint64), ("k2_launches", ctypes.c_uint64),
                 ("k1_ms", ctypes.c_double), ("k2_ms", ctypes.c_double),
                 ("small_teds", ctypes.c_uint64), ("small_ms", ctypes.c_double),
-                ("refined_steps", ctypes.c_uint64), ("corrected_steps", ctypes.c_uint64)]
+                ("refined_steps", ctypes.c_uint64), ("corrected_steps", ctypes.c_uint64),
+                ("full_refined_steps", ctypes.c_uint64)]
 
 
 _lib = None
@@ -280,11 +281,22 @@ def bted_debug_copy_K(ctx: int, which: int, rows: int, ld: int) -> np.ndarray:
     return out
 
 
-def bted_update(ctx: int, X, x_on_device: bool = False):
-    """X: int pointer (host pinned or device), or a host np.float32 array
-    (then copied synchronously enough: the array is referenced only during
-    the call, so it is first pinned by the caller or kept alive)."""
-    ptr = X if isinstance(X, int) else _ptr(X)
+_UPDATE_KEEP: dict = {}
+
+
+def bted_update(ctx: int, X, x_on_device: bool = False, shape=None):
+    """X: int pointer (host pinned or device; the caller guarantees N x d fp32),
+    or a host array, which must be N x d (shape = the ctx's (N, d), checked when
+    given) and is converted to C-contiguous fp32.  The H2D copy is asynchronous:
+    the converted array is kept referenced until the next update of this ctx."""
+    if isinstance(X, int):
+        ptr = X
+    else:
+        A = np.ascontiguousarray(X, dtype=np.float32)
+        if A.ndim != 2 or (shape is not None and tuple(A.shape) != tuple(shape)):
+            raise ValueError(f"bted_update: X has shape {A.shape}, the context holds {shape}")
+        _UPDATE_KEEP[ctx] = A            # alive until the copy has run (next update / call)
+        ptr = _ptr(A)
     check(lib().bted_update(ctx, ptr, 1 if x_on_device else 0))
 
 
@@ -318,7 +330,7 @@ def bted_get_stats(ctx: int) -> dict:
     check(lib().bted_get_stats(ctx, ctypes.byref(st)))
     return dict(teds=st.teds, k2_launches=st.k2_launches, k1_ms=st.k1_ms, k2_ms=st.k2_ms,
                 small_teds=st.small_teds, small_ms=st.small_ms, refined_steps=st.refined_steps,
-                corrected_steps=st.corrected_steps)
+                corrected_steps=st.corrected_steps, full_refined_steps=st.full_refined_steps)
 
 
 def bted_reset_stats(ctx: int):

@@ -756,6 +756,10 @@ struct bted_ctx {
     double* rpart = nullptr; size_t rpartcap = 0;
     double* rdiag = nullptr; size_t rdiagcap = 0;
     double* rout = nullptr; size_t routcap = 0;
+    double* rWt = nullptr; size_t rWtcap = 0;             // full re-scoring: W^T (t x N), scores, selected mask
+    double* rsc = nullptr; size_t rsccap = 0;
+    uint8_t* rmask = nullptr; size_t rmaskcap = 0;
+    uint64_t full_refined_steps = 0;
     uint32_t* ridx = nullptr; size_t ridxcap = 0;
     uint64_t refined_steps = 0, corrected_steps = 0;
     // K4 for the cluster-kernel TEDs: per-instance top-2 keys, flags, candidates, counts, forced picks
@@ -851,6 +855,11 @@ bted_status finish_keys(bted_ctx* ctx, Ted& T, const unsigned long long* keys_de
     CK(cudaStreamSynchronize(T.stream));
     T.collect();
     if (ctx->xbad && take_xbad(ctx)) return BTED_EINVAL;
+    if (*ctx->herr & bted::kSampleOverflow) {
+        CK(cudaMemsetAsync(T.err, 0, sizeof(int), T.stream));
+        set_error("batch sampler: candidate bin overflow (internal limit kCandCap)");
+        return BTED_ENUMERIC;
+    }
     if (*ctx->herr & 4) {
         CK(cudaMemsetAsync(T.err, 0, sizeof(int), T.stream));
         set_error("persistent TED loop: grid barrier timed out (CTAs not co-resident)");
@@ -977,36 +986,41 @@ int bits_for(uint64_t maxval) {
 // out[k][0..M) = sorted V_{b_begin + k b_step}, by radix select (sample.cuh).
 void sample_batches_dev(bted_ctx* ctx, cudaStream_t st, int64_t P, int64_t M, int32_t b_begin, int32_t b_step,
                         int nb, uint64_t seed, uint32_t* out) {
-    grow(ctx->shist, ctx->shistcap, (size_t)nb * bted::kSelBins);
-    grow(ctx->sint, ctx->sintcap, (size_t)4 * nb + 1);
+    grow(ctx->shist, ctx->shistcap, (size_t)2 * nb * bted::kSelBins);
+    grow(ctx->sint, ctx->sintcap, (size_t)5 * nb + 1);
     grow(ctx->scand, ctx->scandcap, (size_t)nb * bted::kCandCap);
-    int* bstar = ctx->sint;
-    int* below = ctx->sint + nb;
-    unsigned* nsel = reinterpret_cast<unsigned*>(ctx->sint + 2 * nb);
-    unsigned* ncand = reinterpret_cast<unsigned*>(ctx->sint + 3 * nb);
-    CK(cudaMemsetAsync(ctx->shist, 0, sizeof(unsigned) * nb * bted::kSelBins, st));
-    CK(cudaMemsetAsync(nsel, 0, sizeof(unsigned) * 2 * nb, st));
-    const unsigned gx = (unsigned)std::max<int64_t>(1, std::min<int64_t>((P + 1023) / 1024, 64));
-    bted::sel_hist_kernel<<<dim3(gx, nb), 256, 0, st>>>((uint64_t)P, seed, b_begin, b_step, ctx->shist);
-    bted::sel_thresh_kernel<<<nb, 1024, 0, st>>>(ctx->shist, M, bstar, below);
-    bted::sel_collect_kernel<<<dim3(gx, nb), 256, 0, st>>>((uint64_t)P, seed, b_begin, b_step, M, bstar, nullptr,
-                                                            nsel, ctx->scand, ncand);
+    unsigned* hist0 = ctx->shist;
+    unsigned* hist1 = ctx->shist + (size_t)nb * bted::kSelBins;
+    int* bstar0 = ctx->sint;
+    int* below0 = ctx->sint + nb;
+    int* bstar1 = ctx->sint + 2 * nb;
+    int* below1 = ctx->sint + 3 * nb;
+    unsigned* ncand = reinterpret_cast<unsigned*>(ctx->sint + 4 * nb);
     if (!ctx->bted_engine.err) {
         grow(ctx->bted_engine.err, ctx->bted_engine.errcap, 1);
         CK(cudaMemsetAsync(ctx->bted_engine.err, 0, sizeof(int), st));
     }
+    CK(cudaMemsetAsync(ctx->shist, 0, sizeof(unsigned) * 2 * nb * bted::kSelBins, st));
+    CK(cudaMemsetAsync(ncand, 0, sizeof(unsigned) * nb, st));
+    const unsigned gx = (unsigned)std::max<int64_t>(1, std::min<int64_t>((P + 1023) / 1024, 64));
+    // two 12-bit radix levels: the candidate bin holds ~P / 2^24 keys
+    bted::sel_hist_kernel<<<dim3(gx, nb), 256, 0, st>>>((uint64_t)P, seed, b_begin, b_step, nullptr, hist0);
+    bted::sel_thresh_kernel<<<nb, 1024, 0, st>>>(hist0, M, nullptr, bstar0, below0);
+    bted::sel_hist_kernel<<<dim3(gx, nb), 256, 0, st>>>((uint64_t)P, seed, b_begin, b_step, bstar0, hist1);
+    bted::sel_thresh_kernel<<<nb, 1024, 0, st>>>(hist1, M, below0, bstar1, below1);
+    bted::sel_collect_kernel<<<dim3(gx, nb), 256, 0, st>>>((uint64_t)P, seed, b_begin, b_step, bstar0, bstar1,
+                                                            ctx->scand, ncand);
     // k* per batch, then the ordered compaction (V_b ascending, no sort)
     const int G = (int)((P + bted::kCmpChunk - 1) / bted::kCmpChunk);
     grow(ctx->sks, ctx->skscap, (size_t)nb);
     grow(ctx->scnt, ctx->scntcap, (size_t)nb * G);
-    bted::sel_finish_kernel<<<nb, 1024, 0, st>>>(M, below, ctx->scand, ncand, nullptr, ctx->bted_engine.err,
-                                                 ctx->sks);
+    bted::sel_finish_kernel<<<nb, 1024, 0, st>>>(M, below1, ctx->scand, ncand, ctx->bted_engine.err, ctx->sks);
     bted::sel_count_kernel<<<dim3(G, nb), bted::kCmpThreads, 0, st>>>((uint64_t)P, seed, b_begin, b_step, ctx->sks,
-                                                                     ctx->scnt);
+                                                                     ctx->scnt, ctx->bted_engine.err);
     bted::sel_scan_kernel<<<nb, 1024, 0, st>>>(ctx->scnt, G);
     bted::sel_write_kernel<<<dim3(G, nb), bted::kCmpThreads, 0, st>>>((uint64_t)P, seed, b_begin, b_step, ctx->sks,
-                                                                     ctx->scnt, M, out);
-    LAUNCHED(7);
+                                                                     ctx->scnt, M, out, ctx->bted_engine.err);
+    LAUNCHED(9);
 }
 
 void gather(bted_ctx* ctx, cudaStream_t st, const uint32_t* idx, int64_t M, float* dst = nullptr) {
@@ -1061,6 +1075,52 @@ void refine_step(bted_ctx* ctx, cudaStream_t st, const float* X, int64_t N, int3
     *best_score = sc;
 }
 
+// fp64 closed-form scores of ALL points after the picks S (refine.cuh, kFlagFull:
+// the near-tie candidate list of a step may be incomplete); returns the exact
+// argmax over the unselected points (ties: lowest index) and its score.
+void refine_full(bted_ctx* ctx, cudaStream_t st, const float* X, int64_t N, int32_t d,
+                 const std::vector<uint32_t>& S, float mu, uint32_t* best, double* best_score) {
+    const int t = (int)S.size();
+    grow(ctx->rcols, ctx->rcolscap, (size_t)std::max(t, 1));
+    grow(ctx->rG, ctx->rGcap, (size_t)std::max(t, 1) * N);
+    grow(ctx->rA, ctx->rAcap, (size_t)std::max(1, t * t));
+    grow(ctx->rWt, ctx->rWtcap, (size_t)std::max(t, 1) * N);
+    grow(ctx->rsc, ctx->rsccap, (size_t)N);
+    grow(ctx->rmask, ctx->rmaskcap, (size_t)N);
+    grow(ctx->rout, ctx->routcap, (size_t)bted::rf::kMaxCand + 1);
+    grow(ctx->ridx, ctx->ridxcap, 1);
+    std::vector<uint8_t> mask((size_t)N, 0);
+    for (uint32_t s : S) mask[s] = 1;
+    CK(cudaMemcpyAsync(ctx->rmask, mask.data(), (size_t)N, cudaMemcpyHostToDevice, st));
+    const int lin = ctx->kernel == BTED_KERNEL_LINEAR ? 1 : 0;
+    if (t > 0) {
+        CK(cudaMemcpyAsync(ctx->rcols, S.data(), sizeof(uint32_t) * t, cudaMemcpyHostToDevice, st));
+        bted::rf::refine_cols_kernel<<<dim3((unsigned)((N + 255) / 256), (unsigned)t), 256, 0, st>>>(
+            X, (int32_t)N, d, (double)ctx->params.gamma, lin, ctx->rcols, ctx->rG);
+        bted::rf::refine_chol_kernel<<<1, 256, 0, st>>>(ctx->rG, (int32_t)N, ctx->rcols, t, (double)mu, ctx->rA);
+        bted::rf::refine_solve_all_kernel<<<(unsigned)((N + 255) / 256), 256, 0, st>>>(ctx->rG, (int32_t)N, t,
+                                                                                      ctx->rA, ctx->rWt);
+        LAUNCHED(3);
+    }
+    const size_t wsmem = sizeof(double) * (size_t)std::max(t, 1) * bted::rf::kAllCand;
+    static uint64_t attr = 0;
+    once_per_device(attr, [] {
+        CK(cudaFuncSetAttribute(bted::rf::refine_all_scores_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)(sizeof(double) * bted::im::kMaxM * bted::rf::kAllCand)));
+    });
+    bted::rf::refine_all_scores_kernel<<<(unsigned)((N + bted::rf::kAllCand - 1) / bted::rf::kAllCand), 256, wsmem,
+                                         st>>>(X, (int32_t)N, d, (double)ctx->params.gamma, lin, ctx->rG, t,
+                                               ctx->rWt, ctx->rmask, (double)mu, ctx->rsc);
+    bted::rf::refine_all_pick_kernel<<<1, 1024, 0, st>>>(ctx->rsc, (int32_t)N, ctx->rout + bted::rf::kMaxCand,
+                                                        ctx->ridx);
+    LAUNCHED(2);
+    double sc = 0.0;
+    CK(cudaMemcpyAsync(best, ctx->ridx, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&sc, ctx->rout + bted::rf::kMaxCand, sizeof(double), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    *best_score = sc;
+}
+
 inline unsigned long long host_pack_key(float score, uint32_t idx) {
     uint32_t b;
     std::memcpy(&b, &score, 4);
@@ -1084,14 +1144,20 @@ bool k4_next_correction(bted_ctx* ctx, cudaStream_t st, const float* X, int64_t 
                         std::vector<unsigned long long>& forced, double* corrected_score = nullptr) {
     const size_t kMC = bted::rf::kMaxCand;
     for (int ts = checked + 1; ts < m; ++ts) {
-        if (!fl[ts] || nc[ts] < 2) continue;
+        const bool full = fl[ts] == bted::rf::kFlagFull;
+        if (!fl[ts] || (!full && nc[ts] < 2)) continue;
         std::vector<uint32_t> S(ts), C;
         for (int k = 0; k < ts; ++k) S[k] = 0xFFFFFFFFu - (uint32_t)(hk[k] & 0xFFFFFFFFull);
-        for (int c = 0; c < nc[ts]; ++c) C.push_back(cd[(size_t)ts * kMC + c]);
-        std::sort(C.begin(), C.end());
         uint32_t best = 0;
         double bs = 0.0;
-        refine_step(ctx, st, X, N, d, S, C, mu, &best, &bs);
+        if (full) {                      // the candidate list may be incomplete: every unselected point
+            refine_full(ctx, st, X, N, d, S, mu, &best, &bs);
+            ctx->full_refined_steps++;
+        } else {
+            for (int c = 0; c < nc[ts]; ++c) C.push_back(cd[(size_t)ts * kMC + c]);
+            std::sort(C.begin(), C.end());
+            refine_step(ctx, st, X, N, d, S, C, mu, &best, &bs);
+        }
         ctx->refined_steps++;
         checked = ts;
         const uint32_t pick = 0xFFFFFFFFu - (uint32_t)(hk[ts] & 0xFFFFFFFFull);
@@ -1380,7 +1446,11 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
     grow(ctx->u32b, ctx->u32bcap, (size_t)n);
     grow(ctx->count_dev, ctx->countcap, 1);
     const unsigned g = (unsigned)std::min<int64_t>((n + 255) / 256, 1024);
-    bted::i64_to_u32_kernel<<<g, 256, 0, st>>>(winners_dev, n, ctx->u32a);
+    if (!ctx->bted_engine.err) {
+        grow(ctx->bted_engine.err, ctx->bted_engine.errcap, 1);
+        CK(cudaMemsetAsync(ctx->bted_engine.err, 0, sizeof(int), st));
+    }
+    bted::i64_to_u32_kernel<<<g, 256, 0, st>>>(winners_dev, n, ctx->N, ctx->u32a, ctx->bted_engine.err);
     LAUNCHED(1);
     size_t need = 0, need2 = 0;
     const int nbits = 32;   // padding (0xFFFFFFFF) must sort last
@@ -1395,7 +1465,13 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
     LAUNCHED(1);
     int nu = 0;
     CK(cudaMemcpyAsync(&nu, ctx->count_dev, sizeof(int), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(ctx->herr, ctx->bted_engine.err, sizeof(int), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));                        // |X_U| sizes the merge TED
+    if (*ctx->herr & bted::kBadWinner) {
+        CK(cudaMemsetAsync(ctx->bted_engine.err, 0, sizeof(int), st));
+        set_error("winner index out of range (>= N)");
+        return BTED_EINVAL;
+    }
     ctx->bted_engine.collect();
     if (ctx->k4b.pending) {                               // K4 of the small batch TEDs, decided here
         ctx->k4b.pending = false;
@@ -1493,7 +1569,10 @@ bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, fl
                 s = finish_keys(ctx, T, T.keys, m, out_idx, out_score);
             return s;
         }
-        T.reserve(ctx->N, ctx->N, ctx->d, m);
+        // engine buffers are sized inside run_ted (the implicit engine needs ~2 N^2
+        // bytes, the dense one 8 N^2): only the keys and K4 scratch here
+        grow(T.keys, T.keyscap, (size_t)m);
+        if (!T.err) { grow(T.err, T.errcap, 1); CK(cudaMemsetAsync(T.err, 0, sizeof(int), T.stream)); }
         const bool packed = use_packed(ctx->params.flags, ctx->d);
         if (T.refine) {
             T.reserve_refine(((ctx->N + bted::pk::T - 1) / bted::pk::T) * bted::pk::T, m);
@@ -1551,7 +1630,8 @@ bted_status bted_batch_teds(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32
         if (take_xbad(ctx)) return BTED_EINVAL;
         if (nb > 0 && *ctx->herr) {
             CK(cudaMemsetAsync(ctx->bted_engine.err, 0, sizeof(int), ctx->stream));
-            set_error("non-finite score during a batch TED");
+            set_error((*ctx->herr & bted::kSampleOverflow) ? "batch sampler: candidate bin overflow (internal limit kCandCap)"
+                                                         : "non-finite score during a batch TED");
             return BTED_ENUMERIC;
         }
         return BTED_OK;
@@ -1922,14 +2002,17 @@ bted_status bted_shard_refine(bted_ctx* ctx, int32_t m, float mu, const uint64_t
         std::vector<uint32_t> cd((size_t)m * kMC);
         for (int t = 0; t < m; ++t) {
             std::vector<uint32_t> c;
+            bool incomplete = false;
             for (int r = 0; r < nranks; ++r) {
-                const int n = std::min<int>(ncand_all[(size_t)r * m + t], (int)kMC);
+                const int n0 = ncand_all[(size_t)r * m + t];
+                if (n0 < 0) { incomplete = true; continue; }           // the band's list may miss candidates
+                const int n = std::min<int>(n0, (int)kMC);
                 for (int q = 0; q < n; ++q) c.push_back(cand_all[((size_t)r * m + t) * kMC + q]);
             }
             std::sort(c.begin(), c.end());
             c.erase(std::unique(c.begin(), c.end()), c.end());
-            if (c.size() > kMC) c.resize(kMC);
-            fl[t] = c.size() >= 2;
+            if (c.size() > kMC) { incomplete = true; c.resize(kMC); }
+            fl[t] = incomplete ? bted::rf::kFlagFull : c.size() >= 2 ? bted::rf::kFlagNear : 0;
             nc[t] = (int)c.size();
             std::copy(c.begin(), c.end(), cd.begin() + (size_t)t * kMC);
         }
@@ -1999,6 +2082,7 @@ bted_status bted_get_stats(bted_ctx* ctx, bted_stats* out) {
     out->small_ms = a.small_ms + b.small_ms;
     out->refined_steps = ctx->refined_steps;
     out->corrected_steps = ctx->corrected_steps;
+    out->full_refined_steps = ctx->full_refined_steps;
     return BTED_OK;
 }
 
@@ -2006,7 +2090,7 @@ bted_status bted_reset_stats(bted_ctx* ctx) {
     if (!ctx) { set_error("null argument"); return BTED_EINVAL; }
     ctx->ted.stats = Stats{};
     ctx->bted_engine.stats = Stats{};
-    ctx->refined_steps = ctx->corrected_steps = 0;
+    ctx->refined_steps = ctx->corrected_steps = ctx->full_refined_steps = 0;
     return BTED_OK;
 }
 
@@ -2022,7 +2106,7 @@ void bted_destroy(bted_ctx* ctx) {
                         ctx->u32b, ctx->count_dev, ctx->mkeys, ctx->cub_tmp, ctx->out_dev, ctx->sall,
                         ctx->xall, ctx->kall, ctx->shist, ctx->sint, ctx->scand, ctx->ssel, ctx->soff,
                         ctx->bflag, ctx->rcols, ctx->rG, ctx->rA, ctx->rW, ctx->rpart, ctx->rdiag, ctx->rout,
-                        ctx->ridx, ctx->bkeys, ctx->bsflags, ctx->bncand, ctx->bcand, ctx->sks, ctx->scnt,
+                        ctx->ridx, ctx->rWt, ctx->rsc, ctx->rmask, ctx->bkeys, ctx->bsflags, ctx->bncand, ctx->bcand, ctx->sks, ctx->scnt,
                         ctx->ktop2, ctx->kflags, ctx->kcand, ctx->kncand, ctx->knflag, ctx->kforced};
         if (ctx->k4pin) cudaFreeHost(ctx->k4pin);
         for (void* b : bufs) if (b) cudaFree(b);

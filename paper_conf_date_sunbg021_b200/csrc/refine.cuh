@@ -15,6 +15,17 @@
 //
 // and takes the exact argmax (ties: lowest index).  If it differs from the
 // GPU's pick, the TED is re-run with the corrected prefix forced.
+//
+// Completeness.  Each score unit (a CTA, a fin unit of 32 rows, a cluster
+// warp) reports only its best two keys.  The candidate list of a step is
+// complete -- it holds EVERY unselected point whose fp32 score is within tau
+// of the best -- exactly when no unit's second key lies in the window (then
+// that unit has no third one either) and at most kMaxCand keys do.  The GPU's
+// own pick, the maximum of all unit keys, is then always on the list.  A step
+// whose list may be incomplete is flagged kFlagFull: the host re-scores ALL
+// unselected points in fp64 (refine_all_* below: the same closed form, every
+// candidate) and takes that argmax, so the decision never depends on which
+// candidates a unit happened to report.
 #pragma once
 #include <cstdint>
 #include <cuda_runtime.h>
@@ -26,13 +37,16 @@ namespace rf {
 constexpr float kTau = 2e-5f;          // near-tie window, relative (>= 8x the measured fp32 error)
 constexpr int kMaxCand = 32;
 constexpr unsigned long long kForced = 1ull << 63;   // key flag of a forced (preset) pick
+constexpr int kFlagNear = 1;           // near tie, complete candidate list
+constexpr int kFlagFull = 2;           // near tie, list may be incomplete: re-score every unselected point
 
 __device__ __forceinline__ float key_score(unsigned long long k) {
     return __uint_as_float((uint32_t)(k >> 32) - 1u);
 }
 
-// Per step t (one CTA each): reduce the finalize CTAs' (top1, top2) keys; flag
-// a near tie and list the candidates within tau of the best.
+// Per step t (one CTA each): reduce the score units' (top1, top2) keys; flag a
+// near tie and list the candidates within tau of the best (kFlagNear), or flag
+// kFlagFull when the list may be incomplete (see the header).
 __global__ void __launch_bounds__(256)
 neartie_check_kernel(const unsigned long long* __restrict__ top2, int nC, const unsigned long long* __restrict__ keys,
                      float tau, int* __restrict__ flags, uint32_t* __restrict__ cand, int* __restrict__ ncand,
@@ -48,7 +62,7 @@ neartie_check_kernel(const unsigned long long* __restrict__ top2, int nC, const 
         nflag += y;
     }
     __shared__ unsigned long long red[8];
-    __shared__ int cnt;
+    __shared__ int cnt, over;
     const int t = blockIdx.x, tid = threadIdx.x;
     const unsigned long long kt = keys[t];
     if (kt & kForced) { if (tid == 0) { flags[t] = 0; ncand[t] = 0; } return; }
@@ -57,7 +71,7 @@ neartie_check_kernel(const unsigned long long* __restrict__ top2, int nC, const 
     for (int q = tid; q < 2 * nC; q += 256) m1 = p[q] > m1 ? p[q] : m1;
     m1 = warp_max_u64(m1);
     if ((tid & 31) == 0) red[tid >> 5] = m1;
-    if (tid == 0) cnt = 0;
+    if (tid == 0) { cnt = 0; over = 0; }
     __syncthreads();
     unsigned long long best = 0ull;
     for (int q = 0; q < 8; ++q) best = red[q] > best ? red[q] : best;
@@ -76,6 +90,7 @@ neartie_check_kernel(const unsigned long long* __restrict__ top2, int nC, const 
         for (int q = tid; q < 2 * nC; q += 256) {
             const unsigned long long k = p[q];
             if (k != 0ull && key_score(k) >= lim) {
+                if (q & 1) over = 1;                    // a unit's SECOND key in the window: it may hold a third
                 const int pos = atomicAdd(&cnt, 1);
                 if (pos < kMaxCand) cand[(int64_t)t * kMaxCand + pos] = key_index(k);
             }
@@ -83,7 +98,8 @@ neartie_check_kernel(const unsigned long long* __restrict__ top2, int nC, const 
     }
     __syncthreads();
     if (tid == 0) {
-        flags[t] = near ? 1 : 0;
+        const bool full = near && (over || cnt > kMaxCand);
+        flags[t] = near ? (full ? kFlagFull : kFlagNear) : 0;
         ncand[t] = near ? min(cnt, kMaxCand) : 0;
         if (near) atomicAdd(nflag, 1);
     }
@@ -91,14 +107,16 @@ neartie_check_kernel(const unsigned long long* __restrict__ top2, int nC, const 
 
 // Row-shard K4 (bted_shard_nearties): per step t, this band's candidates within
 // tau of the GLOBAL pick keys[t] (already all-reduced), from the band's per-CTA
-// top-2 keys; a forced (preset) step lists none.  One CTA per step.
+// top-2 keys; a forced (preset) step lists none.  ncand[t] = -1 when the band's
+// list may be incomplete (a CTA's second key in the window, or > kMaxCand).
+// One CTA per step.
 __global__ void __launch_bounds__(256)
 shard_neartie_kernel(const unsigned long long* __restrict__ top2, int nC, const unsigned long long* __restrict__ keys,
                      float tau, uint32_t* __restrict__ cand, int* __restrict__ ncand) {
-    __shared__ int cnt;
+    __shared__ int cnt, over;
     const int t = blockIdx.x, tid = threadIdx.x;
     const unsigned long long kt = keys[t];
-    if (tid == 0) cnt = 0;
+    if (tid == 0) { cnt = 0; over = 0; }
     __syncthreads();
     if (!(kt & kForced) && kt != 0ull) {
         const float lim = key_score(kt) * (1.f - tau);
@@ -106,13 +124,14 @@ shard_neartie_kernel(const unsigned long long* __restrict__ top2, int nC, const 
         for (int q = tid; q < 2 * nC; q += 256) {
             const unsigned long long k = p[q];
             if (k != 0ull && key_score(k) >= lim) {
+                if (q & 1) over = 1;
                 const int pos = atomicAdd(&cnt, 1);
                 if (pos < kMaxCand) cand[(int64_t)t * kMaxCand + pos] = key_index(k);
             }
         }
     }
     __syncthreads();
-    if (tid == 0) ncand[t] = min(cnt, kMaxCand);
+    if (tid == 0) ncand[t] = (over || cnt > kMaxCand) ? -1 : cnt;
 }
 
 // G[j][i] = k(x_i, x_{cols[j]}) in fp64 (direct difference; reading A1), i < N.
@@ -249,6 +268,156 @@ __global__ void refine_pick_kernel(const double* __restrict__ part, int nblocks,
     }
     out_idx[0] = bi;
     out_score[kMaxCand] = bs;
+}
+
+// ------------------------------------------------------------------ full re-scoring (kFlagFull)
+// Exact fp64 scores of EVERY point after the picks S (|S| = t), the closed form
+// of pin C2 for all candidates at once:
+//   W = (K_SS + mu I)^-1 K_S:            (t x N; Cholesky of K_SS + mu I)
+//   r_ic = K_ic - sum_k K_{i,S_k} W_kc,   score_c = sum_i r_ic^2 / (r_cc + mu)
+// K_ic recomputed from the features in fp64 (as refine_cols_kernel).  Every
+// candidate's sum runs in a fixed order, so exact duplicates score bitwise
+// equal and tie to the lowest index.  Cost ~N^2 (t + d) fp64 FMAs: a rare path.
+
+// one CTA: Ag (t x t, global) <- Cholesky factor (lower) of K_SS + mu I, G = K_:S [t][N]
+__global__ void __launch_bounds__(256)
+refine_chol_kernel(const double* __restrict__ G, int32_t N, const uint32_t* __restrict__ S, int t, double mu,
+                   double* __restrict__ A) {
+    const int tid = threadIdx.x;
+    for (int e = tid; e < t * t; e += 256) {
+        const int a = e / t, b = e % t;
+        A[e] = G[(int64_t)a * N + S[b]] + (a == b ? mu : 0.0);
+    }
+    __syncthreads();
+    for (int k = 0; k < t; ++k) {                       // right-looking, lower triangle
+        const double dkk = sqrt(A[k * t + k]);
+        __syncthreads();
+        if (tid == 0) A[k * t + k] = dkk;
+        for (int i = k + 1 + tid; i < t; i += 256) A[i * t + k] /= dkk;
+        __syncthreads();
+        for (int e = tid; e < (t - k - 1) * (t - k - 1); e += 256) {
+            const int i = k + 1 + e / (t - k - 1), j = k + 1 + e % (t - k - 1);
+            if (j <= i) A[i * t + j] -= A[i * t + k] * A[j * t + k];
+        }
+        __syncthreads();
+    }
+}
+
+// one thread per column c: Wt[:, c] = L^-T L^-1 K_{S,c}  (Wt is t x N, c contiguous)
+__global__ void __launch_bounds__(256)
+refine_solve_all_kernel(const double* __restrict__ G, int32_t N, int t, const double* __restrict__ A,
+                        double* __restrict__ Wt) {
+    const int c = blockIdx.x * 256 + threadIdx.x;
+    if (c >= N) return;
+    for (int i = 0; i < t; ++i) {                       // forward: L y = K_Sc
+        double v = G[(int64_t)i * N + c];
+        for (int k = 0; k < i; ++k) v -= __ldg(&A[i * t + k]) * Wt[(int64_t)k * N + c];
+        Wt[(int64_t)i * N + c] = v / __ldg(&A[i * t + i]);
+    }
+    for (int i = t - 1; i >= 0; --i) {                  // backward: L^T w = y
+        double v = Wt[(int64_t)i * N + c];
+        for (int k = i + 1; k < t; ++k) v -= __ldg(&A[k * t + i]) * Wt[(int64_t)k * N + c];
+        Wt[(int64_t)i * N + c] = v / __ldg(&A[i * t + i]);
+    }
+}
+
+constexpr int kAllCand = 16;            // candidates per CTA of refine_all_scores_kernel
+constexpr int kAllMaxD = 64;
+
+// CTA b: candidates c = 16b .. 16b+15 over all rows i (fixed order per
+// candidate: thread-strided rows, then a fixed warp/CTA tree).  score[c] =
+// fp64 exact score, or -1 for selected / padding candidates.
+__global__ void __launch_bounds__(256)
+refine_all_scores_kernel(const float* __restrict__ X, int32_t N, int32_t d, double gamma, int32_t linear,
+                         const double* __restrict__ G, int t, const double* __restrict__ Wt,
+                         const uint8_t* __restrict__ selmask, double mu, double* __restrict__ score) {
+    extern __shared__ double wsm[];                     // [t][kAllCand]
+    __shared__ float xc[kAllCand][kAllMaxD];
+    __shared__ double red[8][kAllCand];
+    __shared__ double rcc[kAllCand];
+    const int tid = threadIdx.x, c0 = blockIdx.x * kAllCand;
+    for (int e = tid; e < t * kAllCand; e += 256) {
+        const int k = e / kAllCand, c = e % kAllCand;
+        wsm[e] = c0 + c < N ? Wt[(int64_t)k * N + c0 + c] : 0.0;
+    }
+    for (int e = tid; e < kAllCand * d; e += 256) {
+        const int c = e / d, k = e % d;
+        xc[c][k] = c0 + c < N ? X[(int64_t)(c0 + c) * d + k] : 0.f;
+    }
+    if (tid < kAllCand) rcc[tid] = 0.0;
+    __syncthreads();
+    double ss[kAllCand];
+#pragma unroll
+    for (int c = 0; c < kAllCand; ++c) ss[c] = 0.0;
+    for (int i = tid; i < N; i += 256) {
+        double kv[kAllCand];
+#pragma unroll
+        for (int c = 0; c < kAllCand; ++c) kv[c] = 0.0;
+        for (int k = 0; k < d; ++k) {
+            const double xi = (double)X[(int64_t)i * d + k];
+#pragma unroll
+            for (int c = 0; c < kAllCand; ++c) {
+                if (linear) kv[c] = __fma_rn(xi, (double)xc[c][k], kv[c]);
+                else { const double df = xi - (double)xc[c][k]; kv[c] = __fma_rn(df, df, kv[c]); }
+            }
+        }
+        if (!linear) {
+#pragma unroll
+            for (int c = 0; c < kAllCand; ++c) kv[c] = exp(-gamma * kv[c]);
+        }
+        for (int k = 0; k < t; ++k) {
+            const double g = G[(int64_t)k * N + i];
+#pragma unroll
+            for (int c = 0; c < kAllCand; ++c) kv[c] = __fma_rn(-g, wsm[k * kAllCand + c], kv[c]);
+        }
+#pragma unroll
+        for (int c = 0; c < kAllCand; ++c) {
+            ss[c] = __fma_rn(kv[c], kv[c], ss[c]);
+            if (i == c0 + c) rcc[c] = kv[c];            // r_cc: the candidate's own row
+        }
+    }
+#pragma unroll
+    for (int c = 0; c < kAllCand; ++c) {
+        double v = ss[c];
+        for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+        if ((tid & 31) == 0) red[tid >> 5][c] = v;
+    }
+    __syncthreads();
+    if (tid < kAllCand) {
+        const int c = c0 + tid;
+        if (c < N) {
+            double n = 0.0;
+            for (int w = 0; w < 8; ++w) n += red[w][tid];
+            score[c] = selmask[c] ? -1.0 : n / (rcc[tid] + mu);
+        }
+    }
+}
+
+// one CTA: the exact argmax of score[0..N) (score >= 0; ties: lowest index)
+__global__ void __launch_bounds__(1024)
+refine_all_pick_kernel(const double* __restrict__ score, int32_t N, double* __restrict__ out_score,
+                       uint32_t* __restrict__ out_idx) {
+    __shared__ double bs[32];
+    __shared__ uint32_t bi[32];
+    double b = -1.0;
+    uint32_t ib = 0xFFFFFFFFu;
+    for (int c = threadIdx.x; c < N; c += 1024) {       // ascending c per thread: strict > keeps the lowest
+        const double v = score[c];
+        if (v > b) { b = v; ib = (uint32_t)c; }
+    }
+    for (int off = 16; off > 0; off >>= 1) {
+        const double ob = __shfl_xor_sync(0xffffffffu, b, off);
+        const uint32_t oi = __shfl_xor_sync(0xffffffffu, ib, off);
+        if (ob > b || (ob == b && oi < ib)) { b = ob; ib = oi; }
+    }
+    if ((threadIdx.x & 31) == 0) { bs[threadIdx.x >> 5] = b; bi[threadIdx.x >> 5] = ib; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int w = 1; w < 32; ++w)
+            if (bs[w] > b || (bs[w] == b && bi[w] < ib)) { b = bs[w]; ib = bi[w]; }
+        *out_score = b;
+        *out_idx = ib;
+    }
 }
 
 }  // namespace rf

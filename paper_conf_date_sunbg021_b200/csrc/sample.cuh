@@ -37,10 +37,16 @@ __global__ void map_winners_kernel(const unsigned long long* __restrict__ keys, 
     }
 }
 
-// negative entries are padding: they map to 0xFFFFFFFF, which sorts last
-__global__ void i64_to_u32_kernel(const int64_t* __restrict__ in, int64_t n, uint32_t* __restrict__ out) {
-    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
-        out[j] = in[j] < 0 ? 0xFFFFFFFFu : (uint32_t)in[j];
+// negative entries are padding: they map to 0xFFFFFFFF, which sorts last;
+// an entry >= N (a bad device-side winner list) is dropped and flags kBadWinner
+constexpr int kBadWinner = 16;
+__global__ void i64_to_u32_kernel(const int64_t* __restrict__ in, int64_t n, int64_t N, uint32_t* __restrict__ out,
+                                  int* __restrict__ err) {
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t v = in[j];
+        if (v >= N) atomicOr(err, kBadWinner);
+        out[j] = (v < 0 || v >= N) ? 0xFFFFFFFFu : (uint32_t)v;
+    }
 }
 
 // drop the padding value from the end of the unique list
@@ -66,15 +72,21 @@ __global__ void finite_check_kernel(const float* __restrict__ X, int64_t n, int*
 // ---------------------------------------------------------------------------
 // Batch draws by radix SELECT instead of a full sort (all batches at once).
 // V_b = the M smallest key_b(i); key order = (hash32, i).  hash32 is computed on
-// the fly, nothing of size P is stored:
-//   sel_hist     histogram of the top 12 bits of hash32 per batch
-//   sel_thresh   the bin b* holding the M-th smallest key, count `below` before it
-//   sel_collect  indices in bins < b* (all selected), keys in bin b* (candidates)
-//   sel_finish   sort the candidates (bitonic, smem): the M-th smallest key k*
+// the fly, nothing of size P is stored.  Two radix levels of 12 bits each:
+//   sel_hist (lvl 0)  histogram of hash32 bits 31..20 per batch
+//   sel_thresh        the bin b0* holding the M-th smallest key, count before it
+//   sel_hist (lvl 1)  histogram of bits 19..8 of the keys inside bin b0*
+//   sel_thresh        the sub-bin b1* holding it, count before it (cumulative)
+//   sel_collect       keys whose top 24 bits are (b0*, b1*): the candidates
+//   sel_finish        sort the candidates (bitonic, smem): the M-th smallest key k*
 //   sel_count / sel_scan / sel_write   ordered compaction of {i : key_b(i) <= k*}:
 //                each V_b comes out in ascending index order, no sort.
+// The candidate bin holds ~P/2^24 keys (<= 128 on average for P < 2^31), far
+// below kCandCap.  Should it ever overflow, sel_finish sets kSampleOverflow in
+// the error word and the compaction kernels write nothing (kstar never read).
 constexpr int kSelBins = 4096;
 constexpr int kCandCap = 4096;
+constexpr int kSampleOverflow = 8;     // error-word bit of a sampler candidate overflow
 
 __device__ __forceinline__ uint64_t batch_hash_seed(uint64_t seed, int32_t b) {
     return splitmix64(seed + (uint64_t)b * kBatchStride);
@@ -95,27 +107,37 @@ __device__ __forceinline__ unsigned warp_agg_inc(unsigned* ctr, bool pred) {
     return base + (unsigned)__popc(m & ((1u << lane) - 1u));
 }
 
+// level 0 (bstar == nullptr): histogram of h >> 20; level 1: histogram of
+// (h >> 8) & 0xFFF over the keys with h >> 20 == bstar[k]
 __global__ void sel_hist_kernel(uint64_t P, uint64_t seed, int32_t b_begin, int32_t b_step,
-                                unsigned* __restrict__ hist) {
+                                const int* __restrict__ bstar, unsigned* __restrict__ hist) {
     __shared__ unsigned h[kSelBins];
     const int k = blockIdx.y;
     const uint64_t hb = batch_hash_seed(seed, b_begin + k * b_step);
+    const unsigned b0 = bstar ? (unsigned)bstar[k] : 0u;
     for (int q = threadIdx.x; q < kSelBins; q += blockDim.x) h[q] = 0u;
     __syncthreads();
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < P; i += (uint64_t)gridDim.x * blockDim.x)
-        atomicAdd(&h[hash32_of(hb, i) >> 20], 1u);
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < P; i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t x = hash32_of(hb, i);
+        if (!bstar) atomicAdd(&h[x >> 20], 1u);
+        else if ((x >> 20) == b0) atomicAdd(&h[(x >> 8) & 0xFFFu], 1u);
+    }
     __syncthreads();
     for (int q = threadIdx.x; q < kSelBins; q += blockDim.x)
         if (h[q]) atomicAdd(&hist[(int64_t)k * kSelBins + q], h[q]);
 }
 
 // one CTA (1024 threads) per batch: inclusive scan of the 4096 bins, first bin
-// whose cumulative count reaches M
+// whose cumulative count reaches the rank M - below_in[k] (below_in nullable = 0);
+// below_out[k] = below_in[k] + the count of the bins before it
 __global__ void __launch_bounds__(1024)
-sel_thresh_kernel(const unsigned* __restrict__ hist, int64_t M, int* __restrict__ bstar, int* __restrict__ below) {
+sel_thresh_kernel(const unsigned* __restrict__ hist, int64_t M, const int* __restrict__ below_in,
+                  int* __restrict__ bstar, int* __restrict__ below_out) {
     __shared__ unsigned part[1024];
     const int k = blockIdx.x, tid = threadIdx.x;
     const unsigned* hk = hist + (int64_t)k * kSelBins;
+    const unsigned base = below_in ? (unsigned)below_in[k] : 0u;
+    const unsigned need = (unsigned)M - base;
     unsigned v[4], s = 0;
 #pragma unroll
     for (int q = 0; q < 4; ++q) { v[q] = hk[4 * tid + q]; s += v[q]; }
@@ -130,18 +152,18 @@ sel_thresh_kernel(const unsigned* __restrict__ hist, int64_t M, int* __restrict_
     unsigned c = tid ? part[tid - 1] : 0u;                // count before this thread's 4 bins
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
-        if (c < (unsigned)M && c + v[q] >= (unsigned)M) { bstar[k] = 4 * tid + q; below[k] = (int)c; }
+        if (c < need && c + v[q] >= need) { bstar[k] = 4 * tid + q; below_out[k] = (int)(base + c); }
         c += v[q];
     }
 }
 
-__global__ void sel_collect_kernel(uint64_t P, uint64_t seed, int32_t b_begin, int32_t b_step, int64_t M,
-                                   const int* __restrict__ bstar, uint32_t* __restrict__ sel,
-                                   unsigned* __restrict__ nsel, uint64_t* __restrict__ cand,
-                                   unsigned* __restrict__ ncand) {
+// the candidates: keys whose top 24 hash bits are (b0*, b1*)
+__global__ void sel_collect_kernel(uint64_t P, uint64_t seed, int32_t b_begin, int32_t b_step,
+                                   const int* __restrict__ bstar0, const int* __restrict__ bstar1,
+                                   uint64_t* __restrict__ cand, unsigned* __restrict__ ncand) {
     const int k = blockIdx.y;
     const uint64_t hb = batch_hash_seed(seed, b_begin + k * b_step);
-    const unsigned bs = (unsigned)bstar[k];
+    const unsigned top = ((unsigned)bstar0[k] << 12) | (unsigned)bstar1[k];
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     const uint64_t first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const uint64_t iters = (P + stride - 1) / stride;      // uniform per warp: ballots stay converged
@@ -149,27 +171,25 @@ __global__ void sel_collect_kernel(uint64_t P, uint64_t seed, int32_t b_begin, i
         const uint64_t i = first + it * stride;
         const bool in = i < P;
         const uint32_t h = in ? hash32_of(hb, i) : 0xFFFFFFFFu;
-        const unsigned bin = h >> 20;
-        const bool is_sel = in && bin < bs, is_cand = in && bin == bs;
-        if (sel) {
-            const unsigned ps = warp_agg_inc(nsel + k, is_sel);
-            if (is_sel) sel[(int64_t)k * M + ps] = (uint32_t)i;
-        }
+        const bool is_cand = in && (h >> 8) == top;
         const unsigned pc = warp_agg_inc(ncand + k, is_cand);
         if (is_cand && pc < (unsigned)kCandCap) cand[(int64_t)k * kCandCap + pc] = ((uint64_t)h << 32) | i;
     }
 }
 
-// one CTA (1024 threads) per batch: bitonic sort of the candidates in smem
-// (kstar non-null: only record the M-th smallest key per batch for the ordered compaction)
+// one CTA (1024 threads) per batch: bitonic sort of the candidates in smem, then
+// kstar[k] = the M-th smallest key of the batch (rank M - below[k] among them)
 __global__ void __launch_bounds__(1024)
 sel_finish_kernel(int64_t M, const int* __restrict__ below, const uint64_t* __restrict__ cand,
-                  const unsigned* __restrict__ ncand, uint32_t* __restrict__ sel, int* __restrict__ err,
-                  uint64_t* __restrict__ kstar = nullptr) {
+                  const unsigned* __restrict__ ncand, int* __restrict__ err, uint64_t* __restrict__ kstar) {
     __shared__ uint64_t s[kCandCap];
     const int k = blockIdx.x, tid = threadIdx.x;
     const unsigned n = ncand[k];
-    if (n > (unsigned)kCandCap) { if (tid == 0) atomicOr(err, 4); return; }
+    const int need = (int)M - below[k];
+    if (n > (unsigned)kCandCap || need < 1 || need > (int)n) {
+        if (tid == 0) { atomicOr(err, kSampleOverflow); kstar[k] = 0ull; }
+        return;
+    }
     int np = 1;
     while (np < (int)n) np <<= 1;
     for (int q = tid; q < np; q += 1024) s[q] = q < (int)n ? cand[(int64_t)k * kCandCap + q] : ~0ull;
@@ -186,13 +206,7 @@ sel_finish_kernel(int64_t M, const int* __restrict__ below, const uint64_t* __re
             }
             __syncthreads();
         }
-    const int b0 = below[k];
-    const int need = (int)M - b0;
-    if (kstar) {
-        if (tid == 0) kstar[k] = s[need - 1];             // the M-th smallest key of the batch
-        return;
-    }
-    for (int q = tid; q < need; q += 1024) sel[(int64_t)k * M + b0 + q] = (uint32_t)(s[q] & 0xFFFFFFFFull);
+    if (tid == 0) kstar[k] = s[need - 1];
 }
 
 // ---------------------------------------------------------------------------
@@ -207,9 +221,10 @@ __device__ __forceinline__ bool sel_pred(uint64_t hb, uint64_t i, uint64_t P, ui
 
 __global__ void __launch_bounds__(kCmpThreads)
 sel_count_kernel(uint64_t P, uint64_t seed, int32_t b_begin, int32_t b_step, const uint64_t* __restrict__ kstar,
-                 unsigned* __restrict__ cnt) {
+                 unsigned* __restrict__ cnt, const int* __restrict__ err) {
     __shared__ unsigned red[kCmpThreads / 32];
     const int k = blockIdx.y, G = gridDim.x;
+    if (*err & kSampleOverflow) { if (threadIdx.x == 0) cnt[(int64_t)k * G + blockIdx.x] = 0u; return; }
     const uint64_t hb = batch_hash_seed(seed, b_begin + k * b_step), ks = kstar[k];
     const uint64_t base = (uint64_t)blockIdx.x * kCmpChunk;
     unsigned c = 0;
@@ -251,9 +266,10 @@ __global__ void __launch_bounds__(1024) sel_scan_kernel(unsigned* __restrict__ c
 
 __global__ void __launch_bounds__(kCmpThreads)
 sel_write_kernel(uint64_t P, uint64_t seed, int32_t b_begin, int32_t b_step, const uint64_t* __restrict__ kstar,
-                 const unsigned* __restrict__ off, int64_t M, uint32_t* __restrict__ out) {
+                 const unsigned* __restrict__ off, int64_t M, uint32_t* __restrict__ out, const int* __restrict__ err) {
     __shared__ unsigned wcount[kCmpThreads / 32];
     const int k = blockIdx.y, G = gridDim.x, w = threadIdx.x / 32, l = threadIdx.x % 32;
+    if (*err & kSampleOverflow) return;
     const uint64_t hb = batch_hash_seed(seed, b_begin + k * b_step), ks = kstar[k];
     const uint64_t base = (uint64_t)blockIdx.x * kCmpChunk;
     unsigned pos = off[(int64_t)k * G + blockIdx.x];
@@ -270,15 +286,11 @@ sel_write_kernel(uint64_t P, uint64_t seed, int32_t b_begin, int32_t b_step, con
             before += ww < w ? wcount[ww] : 0u;
             tot += wcount[ww];
         }
-        if (p) o[pos + before + __popc(m & ((1u << l) - 1u))] = (uint32_t)i;
+        const unsigned at = pos + before + __popc(m & ((1u << l) - 1u));
+        if (p && at < (unsigned)M) o[at] = (uint32_t)i;
         pos += tot;
         __syncthreads();
     }
-}
-
-__global__ void seg_offsets_kernel(int nb, int64_t M, int* __restrict__ off) {
-    const int q = blockIdx.x * blockDim.x + threadIdx.x;
-    if (q <= nb) off[q] = (int)(q * M);
 }
 
 }  // namespace bted

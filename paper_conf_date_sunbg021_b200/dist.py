@@ -82,6 +82,10 @@ class LibPool:
         self.ctx = ctx
 
     def batch_teds(self, M, m, mu, b_begin, b_step, out: torch.Tensor):
+        if out.is_cuda:
+            # `out` was written (e.g. filled with -1) on torch's current stream; the
+            # library writes the winners on the ctx's own stream: order the two
+            torch.cuda.current_stream(out.device).synchronize()
         L.bted_batch_teds(self.ctx, M, m, mu, b_begin, b_step, out.data_ptr(), winners_on_device=out.is_cuda)
 
     def merge(self, winners: torch.Tensor, m, mu):
