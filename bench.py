@@ -414,7 +414,7 @@ def bench_wholemodel(args, comm, dev, world, rank, local):
     M, m, B = cfg["M"], cfg["m"], cfg["B"]
     nodes = whole_model_nodes()
     mine = [k for k in range(len(nodes)) if k % world == rank]
-    pools = whole_model_pools(nodes=[nodes[k] for k in mine])
+    pools = whole_model_pools(which=mine)
     stream = torch.cuda.Stream(dev)
     ctxs = []
     for (wl, X, g), k in zip(pools, mine):

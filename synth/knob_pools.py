@@ -242,15 +242,17 @@ CONFIGS = {
 MU = 0.1
 
 
-def whole_model_pools(pool: int = 1 << 20, d: int = 16, nodes=None):
+def whole_model_pools(pool: int = 1 << 20, d: int = 16, which=None):
     """[(node, X fp32 [P_node, d], gamma)] for the 'wholemodel' config: the first
     20 unique conv workloads of ResNet-50 and of MobileNet-v2, pool P =
-    min(pool, |D|) each, seed = 5000 + node index."""
+    min(pool, |D|) each, seed = 5000 + node index.
+    which: the node indices (into whole_model_nodes()) to build; default all."""
+    nodes = whole_model_nodes()
     out = []
-    for k, wl in enumerate(whole_model_nodes() if nodes is None else nodes):
-        space = KnobSpace(wl, d)
+    for k in (range(len(nodes)) if which is None else which):
+        space = KnobSpace(nodes[k], d)
         _, X = make_pool(space, pool, 5000 + k)
-        out.append((wl, X, median_gamma(X, 5000 + k)))
+        out.append((nodes[k], X, median_gamma(X, 5000 + k)))
     return out
 
 
