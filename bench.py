@@ -132,7 +132,20 @@ class Clocks:
 def oracle_points_per_s(Xb: np.ndarray, gamma: float, mu: float, m: int, budget_s: float):
     """The fp64 oracle (oracle/ted_dense.c, all host cores) on one full batch:
     Gram + as many of the m greedy steps as fit in ~budget_s; the m-step TED
-    time is extrapolated from the measured per-step time."""
+    time is extrapolated from the measured per-step time.  Batches above
+    32768 points use the matrix-free O2 oracle (oracle/ted_matfree.c): a 1-step
+    and a 3-step run, the per-step time from their difference."""
+    if Xb.shape[0] > 32768:
+        from oracle import matfree
+        t0 = time.perf_counter()
+        matfree.ted(Xb, gamma, mu, 1)
+        t1 = time.perf_counter() - t0
+        t0 = time.perf_counter()
+        matfree.ted(Xb, gamma, mu, 3)
+        t3 = time.perf_counter() - t0
+        per = max((t3 - t1) / 2, 1e-9)
+        t_ted = t1 + (m - 1) * per
+        return m / t_ted, t1, per, 3, matfree.num_threads()
     from oracle import dense
     t0 = time.perf_counter()
     K = dense.gram(Xb, gamma)
@@ -379,9 +392,10 @@ def bench_ours(args):
         from oracle.sampling import sample_batches
         V = sample_batches(P, M, 1, cfg["seed"])[0]
         v, tg, ts, n, cores = oracle_points_per_s(X[V], gamma, mu, m, args.cpu_budget_s)
+        which = "matrix-free O2 C/OpenMP oracle" if M > 32768 else "dense C/OpenMP oracle"
         cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
                "sample": (f"batch 0 (N={M}): fp64 Gram ({tg:.2f} s) + {n} of {m} greedy steps "
-                          f"({ts:.3f} s/step) with the dense C/OpenMP oracle; points/s of the full "
+                          f"({ts:.3f} s/step) with the {which}; points/s of the full "
                           f"{m}-step TED extrapolated from those")}
 
     pool.close()
@@ -560,11 +574,29 @@ def bench_sharded(args, X, gamma, cfg, comm, dev, world, rank):
     torch.distributed.destroy_process_group()
 
 
+def spawn_ranks(n: int) -> int:
+    """`python bench.py --gpus N` outside torchrun: re-launch this command as N
+    ranks (one process per GPU) under torch.distributed.run on 127.0.0.1."""
+    import socket
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
 def main():
     args = parse()
     if args.warmup < 3:
         print("warning: --warmup < 3 violates the timing rules; using 3", file=sys.stderr)
         args.warmup = 3
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(spawn_ranks(args.gpus))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world != args.gpus:
+        sys.exit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world} (launch one rank per GPU)")
     if args.impl == "reference":
         bench_reference(args)
     else:

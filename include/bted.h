@@ -51,7 +51,8 @@ typedef enum {
     BTED_EINVAL = 1,         /* invalid argument (see each call)                    */
     BTED_ENOMEM = 2,         /* device or host allocation failed                    */
     BTED_ECUDA = 3,          /* CUDA runtime error / no usable device               */
-    BTED_ENCCL = 4,          /* reserved for collective failures                    */
+    BTED_ENCCL = 4,          /* multi-GPU exchange failed: an NCCL error, or a peer
+                                that stopped publishing (flag wait / collective timeout) */
     BTED_ENUMERIC = 5,       /* NaN score or non-positive k(v,v)+mu during a run    */
     BTED_ESTATE = 6          /* context poisoned by an earlier CUDA error           */
 } bted_status;
@@ -83,6 +84,14 @@ typedef enum {
                                    otherwise re-scored exactly in fp64 from the features and the
                                    exact argmax taken (every single-GPU engine, the tile-sharded
                                    engine and the row-shard API's symmetric mode)               */
+#define BTED_FLAG_LOOPBACK 512u /* num_devices > 1: run the G (P) device shards / replicas as
+                                   logical devices all on `device` (one stream): the
+                                   multi-GPU control flow and exchange on one GPU (tests) */
+#define BTED_FLAG_NCCL   1024u  /* bted_select with P > 1: exchange through NCCL collectives
+                                   (ncclCommInitAll over the P devices, libnccl.so.2 loaded at
+                                   run time) instead of the default peer-memory exchange;
+                                   NCCL failures and a stalled collective (BTED_NCCL_TIMEOUT_S,
+                                   default 300 s; ncclCommGetAsyncError polled) -> BTED_ENCCL */
 #define BTED_FLAG_TIMING   2u   /* record CUDA events around K1 and the K2 loop of every batch
                                    TED on the ctx stream; read with bted_get_stats()          */
 
@@ -93,11 +102,24 @@ typedef struct {
     uint64_t  seed;          /* batch sampling seed (Alg. 2 l.2, reading A10)          */
     int32_t   x_on_device;   /* 1: X is a device pointer on `device` (adopted, not copied) */
     uint32_t  flags;         /* BTED_FLAG_*                                           */
-    uintptr_t stream;        /* cudaStream_t to run on; 0 = a stream owned by the ctx  */
+    uintptr_t stream;        /* cudaStream_t to run on; 0 = a stream owned by the ctx
+                                (num_devices > 1: the stream of `device` only)         */
+    int32_t   num_devices;   /* G = P >= 1 GPUs [device, device + G) driven by this ctx
+                                (SURVEY 8(e)); 1 = single GPU.  bted_run_batches runs
+                                batch b on device b mod G (no exchange until the
+                                merge, which runs on `device`); bted_select row- or
+                                tile-shards the ONE candidate set over the P GPUs
+                                (see "Multi-GPU" below).  X is replicated.          */
+    int32_t   norm_mode;     /* bted_select with P > 1 and BTED_FLAG_DENSE (row bands):
+                                0 = local row norms (K bit-symmetric: row norm =
+                                column norm, no norm exchange), 1 = the literal
+                                all-reduce of every band's partial COLUMN norms
+                                (north_star wording; an ablation).  Ignored by the
+                                default tile-sharded implicit engine.               */
 } bted_params;
 
 /* Fill *p with defaults: gamma 1, device -1, num_batches 1, seed 0, host X,
- * flags 0, own stream. */
+ * flags 0, own stream, num_devices 1, norm_mode 0. */
 void bted_default_params(bted_params* p);
 
 /*

@@ -22,6 +22,8 @@ BTED_FLAG_IMPLICIT = 32
 BTED_FLAG_LITERAL = 64
 BTED_FLAG_NO_REFINE = 128
 BTED_FLAG_PERSISTENT_LOOP = 256
+BTED_FLAG_LOOPBACK = 512
+BTED_FLAG_NCCL = 1024
 STATUS = {0: "BTED_OK", 1: "BTED_EINVAL", 2: "BTED_ENOMEM", 3: "BTED_ECUDA", 4: "BTED_ENCCL",
           5: "BTED_ENUMERIC", 6: "BTED_ESTATE"}
 
@@ -41,6 +43,8 @@ class bted_params(ctypes.Structure):
         ("x_on_device", ctypes.c_int32),
         ("flags", ctypes.c_uint32),
         ("stream", ctypes.c_size_t),
+        ("num_devices", ctypes.c_int32),
+        ("norm_mode", ctypes.c_int32),
     ]
 
 
@@ -119,11 +123,13 @@ def _ptr(a: np.ndarray) -> int:
     return a.ctypes.data
 
 
-def default_params(gamma=1.0, device=-1, num_batches=1, seed=0, x_on_device=0, flags=0, stream=0) -> bted_params:
+def default_params(gamma=1.0, device=-1, num_batches=1, seed=0, x_on_device=0, flags=0, stream=0,
+                   num_devices=1, norm_mode=0) -> bted_params:
     p = bted_params()
     lib().bted_default_params(ctypes.byref(p))
     p.gamma, p.device, p.num_batches, p.seed = float(gamma), int(device), int(num_batches), int(seed)
     p.x_on_device, p.flags, p.stream = int(x_on_device), int(flags), int(stream)
+    p.num_devices, p.norm_mode = int(num_devices), int(norm_mode)
     return p
 
 

@@ -9,6 +9,8 @@
 // m packed keys at the end (no per-step host round trip).
 #include <cub/cub.cuh>
 #include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nccl.h>            // types only: libnccl.so.2 is loaded at run time (BTED_FLAG_NCCL)
 
 #include <algorithm>
 #include <atomic>
@@ -22,6 +24,8 @@
 #include <mutex>
 #include <new>
 #include <string>
+#include <thread>
+#include <chrono>
 #include <vector>
 
 #include "../../include/bted.h"
@@ -32,6 +36,7 @@
 #include "implicit.cuh"
 #include "refine.cuh"
 #include "colnorm.cuh"
+#include "xchg.cuh"
 
 namespace {
 
@@ -50,6 +55,9 @@ void set_error(const char* fmt, ...) {
 struct CudaError {
     cudaError_t e;
     const char* what;
+};
+struct NcclError {            // a failed or stalled collective (BTED_FLAG_NCCL) -> BTED_ENCCL
+    std::string what;
 };
 
 #define CK(expr)                                                         \
@@ -780,6 +788,7 @@ struct bted_ctx {
     unsigned long long* hkeys = nullptr; size_t hkeyscap = 0;
     int* herr = nullptr;
     int* xbad = nullptr;      // device: non-finite feature seen by finite_check_kernel
+    struct MultiDev* md = nullptr;   // num_devices > 1: the per-device shards / replicas
 };
 
 namespace {
@@ -818,6 +827,11 @@ bted_status guarded(bted_ctx* ctx, F&& f) {
         set_error("CUDA error %s (%s) in %s", cudaGetErrorName(e.e), cudaGetErrorString(e.e), e.what);
         cudaGetLastError();
         return e.e == cudaErrorMemoryAllocation ? BTED_ENOMEM : BTED_ECUDA;
+    } catch (const NcclError& e) {
+        ctx->poisoned = true;
+        set_error("%s", e.what.c_str());
+        cudaGetLastError();
+        return BTED_ENCCL;
     } catch (const std::bad_alloc&) {
         set_error("host allocation failed");
         return BTED_ENOMEM;
@@ -855,6 +869,12 @@ bted_status finish_keys(bted_ctx* ctx, Ted& T, const unsigned long long* keys_de
     CK(cudaStreamSynchronize(T.stream));
     T.collect();
     if (ctx->xbad && take_xbad(ctx)) return BTED_EINVAL;
+    if (*ctx->herr & bted::im::kErrPeerTimeout) {
+        CK(cudaMemsetAsync(T.err, 0, sizeof(int), T.stream));
+        ctx->poisoned = true;
+        set_error("multi-GPU exchange: a peer device never published its step (20 s flag wait)");
+        return BTED_ENCCL;
+    }
     if (*ctx->herr & bted::kSampleOverflow) {
         CK(cudaMemsetAsync(T.err, 0, sizeof(int), T.stream));
         set_error("batch sampler: candidate bin overflow (internal limit kCandCap)");
@@ -889,6 +909,8 @@ bted_status validate_params(const bted_params* p, bted_kernel kernel) {
         set_error("gamma must be > 0 and finite"); return BTED_EINVAL;
     }
     if (p->num_batches < 1) { set_error("num_batches must be >= 1"); return BTED_EINVAL; }
+    if (p->num_devices < 0) { set_error("num_devices must be >= 1"); return BTED_EINVAL; }
+    if (p->norm_mode != 0 && p->norm_mode != 1) { set_error("norm_mode must be 0 or 1"); return BTED_EINVAL; }
     return BTED_OK;
 }
 
@@ -1438,6 +1460,37 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
     return nb;
 }
 
+// After run_batch_range: wait for the batch TEDs, resolve the small-batch K4
+// deferred to this sync (ctx->winners updated), check the error words.
+bted_status batch_range_finish(bted_ctx* ctx, int nb) {
+    *ctx->herr = 0;
+    if (nb > 0)
+        CK(cudaMemcpyAsync(ctx->herr, ctx->bted_engine.err, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    ctx->bted_engine.collect();
+    if (ctx->k4b.pending) {                          // K4 of small batch TEDs
+        ctx->k4b.pending = false;
+        auto& b = ctx->k4b;
+        if (small_k4_refine(ctx, ctx->stream, ctx->xall, b.ninst, b.M, ctx->d, b.m, b.mu, ctx->kall,
+                            ctx->bted_engine.err)) {
+            for (int kk = 0; kk < b.ninst; ++kk) {
+                bted::map_winners_kernel<<<(b.m + 127) / 128, 128, 0, ctx->stream>>>(
+                    ctx->kall + (size_t)kk * b.m, b.m, ctx->sall + (size_t)kk * b.M, ctx->winners + (size_t)kk * b.m);
+                LAUNCHED(1);
+            }
+            CK(cudaStreamSynchronize(ctx->stream));
+        }
+    }
+    if (take_xbad(ctx)) return BTED_EINVAL;
+    if (nb > 0 && *ctx->herr) {
+        CK(cudaMemsetAsync(ctx->bted_engine.err, 0, sizeof(int), ctx->stream));
+        set_error((*ctx->herr & bted::kSampleOverflow) ? "batch sampler: candidate bin overflow (internal limit kCandCap)"
+                                                     : "non-finite score during a batch TED");
+        return BTED_ENUMERIC;
+    }
+    return BTED_OK;
+}
+
 // Alg. 2 l.5-6 on device winners[0..n): returns count, out_idx host [count].
 bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, int32_t m, float mu,
                          int64_t* out_idx, int32_t* out_count) {
@@ -1526,6 +1579,833 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
 
 }  // namespace
 
+// ------------------------------------------------------------------ row-sharded dense bands (internal)
+namespace {
+void shard_gram_enqueue(bted_ctx* ctx, float mu, uint64_t* keys_dev) {
+    Ted& T = ctx->ted;
+    const int64_t rows = ctx->row1 - ctx->row0;
+    T.reserve(rows, ctx->N, ctx->d, 2);
+    T.last_rows = rows;
+    T.last_ld = ld_for(ctx->N);
+    T.last_buf = 0;
+    launch_transpose(T, ctx->X, ctx->N, ctx->d);
+    CK(cudaMemsetAsync(T.sel, 0, (size_t)rows, T.stream));
+    // K4: per-CTA top-2 keys of the first kMaxM steps (bted_shard_nearties / bted_shard_refine)
+    if (T.refine) T.reserve_refine((rows + kRowsPerK2Cta - 1) / kRowsPerK2Cta * 32, bted::im::kMaxM);
+    launch_gram(T, ctx->N, ctx->d, ctx->row0, rows, ctx->params.gamma, ctx->kernel, mu,
+                reinterpret_cast<unsigned long long*>(keys_dev), T.refine ? T.top2 : nullptr);
+}
+
+void shard_step_enqueue(bted_ctx* ctx, int32_t t, float mu, const float* pivot_dev, uint64_t* keys_dev) {
+    Ted& T = ctx->ted;
+    const int64_t rows = ctx->row1 - ctx->row0;
+    launch_step(T, ctx->N, ctx->row0, rows, t, mu, pivot_dev, reinterpret_cast<unsigned long long*>(keys_dev),
+                (T.refine && T.top2 && t < bted::im::kMaxM) ? T.top2 : nullptr);
+    T.last_buf = t & 1;
+}
+
+void shard_pivot_enqueue(bted_ctx* ctx, int32_t t, const uint64_t* keys_dev, float* col_dev) {
+    Ted& T = ctx->ted;
+    const int32_t rows = (int32_t)(ctx->row1 - ctx->row0);
+    const unsigned g = (unsigned)std::min<int64_t>((rows + 255) / 256, 1024);
+    bted::pivot_column_kernel<<<g, 256, 0, T.stream>>>(T.K[t & 1], ld_for(ctx->N), rows,
+                                                       reinterpret_cast<const unsigned long long*>(keys_dev), t,
+                                                       col_dev);
+    LAUNCHED(1);
+}
+
+void shard_colnorm_enqueue(bted_ctx* ctx, int32_t t, float mu, const float* pivot_dev,
+                           const uint64_t* keys_dev, float* colnorm_dev) {
+    Ted& T = ctx->ted;
+    const int64_t ld = ld_for(ctx->N);
+    const int32_t rows = (int32_t)(ctx->row1 - ctx->row0);
+    const int32_t nchunks = (rows + bted::kColChunk - 1) / bted::kColChunk;
+    grow(T.P, T.pcap, (size_t)nchunks * (size_t)ld);
+    const dim3 grid((unsigned)((ld + 255) / 256), (unsigned)nchunks);
+    const auto* keys = reinterpret_cast<const unsigned long long*>(keys_dev);
+    if (t == 0)
+        bted::deflate_colnorm_kernel<false><<<grid, bted::kColThreads, 0, T.stream>>>(
+            T.K[0], nullptr, ld, (int32_t)ctx->row0, rows, nullptr, nullptr, 0, mu, T.sel, T.P);
+    else
+        bted::deflate_colnorm_kernel<true><<<grid, bted::kColThreads, 0, T.stream>>>(
+            T.K[(t - 1) & 1], T.K[t & 1], ld, (int32_t)ctx->row0, rows, pivot_dev, keys, t, mu, T.sel, T.P);
+    const unsigned g2 = (unsigned)std::min<int64_t>((ld + 255) / 256, 2048);
+    bted::colnorm_reduce_kernel<<<g2, 256, 0, T.stream>>>(T.P, nchunks, ld, colnorm_dev);
+    LAUNCHED(2);
+    T.last_buf = t & 1;
+}
+
+void shard_scores_enqueue(bted_ctx* ctx, int32_t t, float mu, const float* colnorm_dev, uint64_t* keys_dev) {
+    Ted& T = ctx->ted;
+    const int32_t rows = (int32_t)(ctx->row1 - ctx->row0);
+    unsigned g = (unsigned)std::min<int64_t>((rows + 255) / 256, 1184);
+    // K4: one CTA per top-2 slot pair of the step (T.last_nC, set by bted_shard_gram),
+    // so bted_shard_nearties reads the literal mode's keys like the symmetric mode's
+    unsigned long long* top2 = nullptr;
+    if (T.refine && T.top2 && t < bted::im::kMaxM && T.last_nC > 0) {
+        g = (unsigned)T.last_nC;
+        top2 = T.top2 + (int64_t)t * T.last_nC * 2;
+    }
+    bted::colnorm_scores_kernel<<<g, 256, 0, T.stream>>>(T.K[t & 1], ld_for(ctx->N), (int32_t)ctx->row0, rows,
+                                                         colnorm_dev, mu, T.sel,
+                                                         reinterpret_cast<unsigned long long*>(keys_dev), t, T.err,
+                                                         top2);
+    LAUNCHED(1);
+}
+// K4 for row bands: every band's candidates within tau of the global pick
+// (cand_all / ncand_all: host, [nranks][m][kMaxCand] / [nranks][m]; -1 = that
+// band's list may be incomplete), merged, then the usual decision on this shard.
+bool shard_k4_decide(bted_ctx* ctx, int32_t m, float mu, const unsigned long long* keys_dev, const uint32_t* cand_all,
+                     const int32_t* ncand_all, int32_t nranks, std::vector<unsigned long long>& forced) {
+    Ted& T = ctx->ted;
+    forced.clear();
+    if (!T.refine) return false;
+    const size_t kMC = bted::rf::kMaxCand;
+    std::vector<unsigned long long> hk(m);
+    CK(cudaMemcpyAsync(hk.data(), keys_dev, sizeof(unsigned long long) * m, cudaMemcpyDeviceToHost, T.stream));
+    CK(cudaStreamSynchronize(T.stream));
+    std::vector<int> fl(m, 0), nc(m, 0);
+    std::vector<uint32_t> cd((size_t)m * kMC);
+    for (int t = 0; t < m; ++t) {
+        std::vector<uint32_t> c;
+        bool incomplete = false;
+        for (int r = 0; r < nranks; ++r) {
+            const int n0 = ncand_all[(size_t)r * m + t];
+            if (n0 < 0) { incomplete = true; continue; }           // the band's list may miss candidates
+            const int n = std::min<int>(n0, (int)kMC);
+            for (int q = 0; q < n; ++q) c.push_back(cand_all[((size_t)r * m + t) * kMC + q]);
+        }
+        std::sort(c.begin(), c.end());
+        c.erase(std::unique(c.begin(), c.end()), c.end());
+        if (c.size() > kMC) { incomplete = true; c.resize(kMC); }
+        fl[t] = incomplete ? bted::rf::kFlagFull : c.size() >= 2 ? bted::rf::kFlagNear : 0;
+        nc[t] = (int)c.size();
+        std::copy(c.begin(), c.end(), cd.begin() + (size_t)t * kMC);
+    }
+    int checked = -1;
+    return k4_next_correction(ctx, T.stream, ctx->X, ctx->N, ctx->d, m, mu, hk, fl, nc, cd, checked, forced);
+}
+}  // namespace
+
+// ------------------------------------------------------------------ tile-sharded implicit engine
+namespace {
+int64_t ishard_local_tiles(const bted_ctx* ctx) {
+    const int nT = (int)((ctx->N + bted::pk::T - 1) / bted::pk::T);
+    const int64_t all = bted::pk::num_tiles(nT);
+    return (all - ctx->srank + ctx->snranks - 1) / ctx->snranks;
+}
+bted::im::XKern ishard_xk(const bted_ctx* ctx) {
+    bted::im::XKern xk;
+    xk.X = ctx->X; xk.d = ctx->d; xk.ng = -ctx->params.gamma; xk.linear = ctx->kernel == BTED_KERNEL_LINEAR ? 1 : 0;
+    return xk;
+}
+int64_t ishard_qlen_of(int64_t N) {
+    const int64_t NP = (N + bted::pk::T - 1) / bted::pk::T * bted::pk::T;
+    return (NP + 255) / 256 * 256;
+}
+
+// Alg. 1 l.1 + this shard's part of ||K_:v||^2 into q_dev (on the ctx's device / stream)
+void ishard_head_enqueue(bted_ctx* ctx, int32_t m, double* q_dev) {
+    Ted& T = ctx->ted;
+    const int64_t N = ctx->N, NPa = ishard_qlen_of(N);
+    const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
+    const int64_t lt = ishard_local_tiles(ctx);
+    ensure_implicit_attrs();
+    T.reserve_implicit(N, m, lt);
+    ctx->sm_m = m;
+    CK(cudaMemsetAsync(T.sel, 0, (size_t)NPa, T.stream));
+    CK(cudaMemsetAsync(T.kflag, 0, sizeof(int), T.stream));
+    CK(cudaMemsetAsync(T.tctr, 0, sizeof(int) * m, T.stream));
+    CK(cudaMemsetAsync(q_dev, 0, sizeof(double) * NPa, T.stream));
+    const int lin = ctx->kernel == BTED_KERNEL_LINEAR ? 1 : 0;
+    const float g = ctx->params.gamma;
+    const int r = ctx->srank, P = ctx->snranks;
+    auto k1i = [&](auto kern) {
+        kern<<<(unsigned)lt, bted::pk::kConsumers, 0, T.stream>>>(ctx->X, (int32_t)N, ctx->d, g, T.K[0], nT, r, P);
+    };
+    if (ctx->d <= 16) {
+        if (lin) k1i(bted::pk::gram_tile2_kernel<16, true, 4>); else k1i(bted::pk::gram_tile2_kernel<16, false, 4>);
+    } else {
+        if (lin) k1i(bted::pk::gram_tile_kernel<32, true>); else k1i(bted::pk::gram_tile_kernel<32, false>);
+    }
+    bted::im::diag_init_kernel<<<(unsigned)((NPa + 255) / 256), 256, 0, T.stream>>>(ishard_xk(ctx), (int32_t)N,
+                                                                                     NPa, T.rd);
+    bted::im::tile_pass_kernel<true><<<tile_pass_grid(lt), bted::im::kTPThreads, bted::im::tile_pass_smem_bytes,
+                                       T.stream>>>(T.K[0], nT, nullptr, T.P64, T.kflag, T.tctr, 0, 0, r, P);
+    bted::im::qpart_kernel<<<(unsigned)std::min<int64_t>((NPa + 255) / 256, 4096), 256, 0, T.stream>>>(
+        T.P64, nT, r, P, q_dev);
+    LAUNCHED(4);
+}
+
+// step t: the new factor column l_t (from keys[t-1]) and this shard's part of K l_t into q_dev
+void ishard_step_enqueue(bted_ctx* ctx, int32_t t, float mu, const unsigned long long* keys, double* q_dev) {
+    Ted& T = ctx->ted;
+    const int64_t N = ctx->N, NPa = ishard_qlen_of(N);
+    const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
+    const int nA = (int)(NPa / bted::im::kEllRows);
+    const int32_t m = ctx->sm_m;
+    bted::im::ell_kernel<<<(unsigned)nA + 1, bted::im::kThreads, 0, T.stream>>>(
+        T.K[0], nT, (int32_t)N, T.Lf, NPa, t - 1, T.rd, T.nv, mu, keys, t, T.ell, T.Qc, T.G, m, T.hv, T.sel,
+        ishard_xk(ctx));
+    bted::im::tile_pass_kernel<false><<<tile_pass_grid(ishard_local_tiles(ctx)), bted::im::kTPThreads,
+                                        bted::im::tile_pass_smem_bytes, T.stream>>>(
+        T.K[0], nT, T.ell, T.P64, T.kflag, T.tctr + t, (int)(t & 1), 0, ctx->srank, ctx->snranks);
+    bted::im::qpart_kernel<<<(unsigned)std::min<int64_t>((NPa + 255) / 256, 4096), 256, 0, T.stream>>>(
+        T.P64, nT, ctx->srank, ctx->snranks, q_dev);
+    LAUNCHED(3);
+}
+
+// scores of step t from the summed q (q_dev) or, with pq, from the devices' partials
+void ishard_fin_enqueue(bted_ctx* ctx, int32_t t, float mu, const double* q_dev, unsigned long long* keys,
+                        const bted::im::PeerQ* pq = nullptr) {
+    Ted& T = ctx->ted;
+    const int64_t N = ctx->N, NPa = ishard_qlen_of(N);
+    const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
+    const int64_t NP = (int64_t)nT * bted::pk::T;
+    if (pq)
+        bted::im::fin64_peer_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
+            *pq, nT, (int32_t)N, T.K[0], mu, T.Lf, NPa, t > 0 ? t - 1 : 0, T.hv, T.nv, T.rd, T.sel, keys, t,
+            keys + t, T.err, T.refine ? T.top2 : nullptr, T.Qc, t == 0 ? T.rd : nullptr);
+    else
+        bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
+            T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, NPa, t > 0 ? t - 1 : 0, T.hv, T.nv, T.rd, T.sel, keys, t,
+            keys + t, T.err, T.refine ? T.top2 : nullptr, T.Qc, q_dev, t == 0 ? T.rd : nullptr);
+    LAUNCHED(1);
+}
+
+// K4 on a tile shard (all shards hold the same keys and reach the same decision):
+// true with `forced` = the corrected prefix if a refined pick changes
+bool ishard_k4(bted_ctx* ctx, int32_t m, float mu, const unsigned long long* keys,
+               std::vector<unsigned long long>& forced) {
+    Ted& T = ctx->ted;
+    forced.clear();
+    if (!T.refine) return false;
+    cudaStream_t st = T.stream;
+    CK(cudaMemsetAsync(T.nflag, 0, sizeof(int), st));
+    bted::rf::neartie_check_kernel<<<m, 256, 0, st>>>(T.top2, T.last_nC, keys, bted::rf::kTau, T.flags, T.cand,
+                                                     T.ncand, T.nflag);
+    LAUNCHED(1);
+    std::vector<unsigned long long> hk(m);
+    std::vector<int> fl(m), nc(m);
+    std::vector<uint32_t> cd((size_t)m * bted::rf::kMaxCand);
+    CK(cudaMemcpyAsync(hk.data(), keys, sizeof(unsigned long long) * m, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(fl.data(), T.flags, sizeof(int) * m, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(nc.data(), T.ncand, sizeof(int) * m, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(cd.data(), T.cand, sizeof(uint32_t) * cd.size(), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    int checked = -1;
+    return k4_next_correction(ctx, st, ctx->X, ctx->N, ctx->d, m, mu, hk, fl, nc, cd, checked, forced);
+}
+}  // namespace
+
+// ------------------------------------------------------------------ multi-GPU (num_devices > 1)
+// One ctx drives G = P devices [device, device + G) from one process (SURVEY
+// 8(e)): bted_run_batches sends batch b to device b mod G (replica ctxs, one
+// host thread each: the batches are independent, Alg. 2 l.1-4);
+// bted_select tile-shards one candidate set (the implicit engine's packed Gram
+// tiles k = p mod P on device p; X and the O(N m) fp64 state replicated).  Per
+// step the only exchange is the sum of the P partial q = K l vectors: by
+// default each device publishes its partial (a release flag in its memory)
+// and every device's score kernel (fin64_peer_kernel) sums all P partials
+// through peer loads in rank order -- the all-reduce fused into its consumer,
+// bitwise the same on every device; BTED_FLAG_NCCL uses ncclAllReduce instead.
+// BTED_FLAG_LOOPBACK runs the P shards / G replicas as logical devices on one
+// GPU and one stream (the same control flow and kernels; tests).
+namespace {
+
+struct NcclApi {
+    bool ok = false;
+    std::string why;
+    ncclResult_t (*CommInitAll)(ncclComm_t*, int, const int*) = nullptr;
+    ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                              cudaStream_t) = nullptr;
+    ncclResult_t (*GroupStart)() = nullptr;
+    ncclResult_t (*GroupEnd)() = nullptr;
+    ncclResult_t (*CommGetAsyncError)(ncclComm_t, ncclResult_t*) = nullptr;
+    ncclResult_t (*CommAbort)(ncclComm_t) = nullptr;
+    ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+    const char* (*GetErrorString)(ncclResult_t) = nullptr;
+};
+// libnccl.so.2 at run time: the process's already-loaded NCCL (e.g. torch's) if any
+NcclApi& nccl_api() {
+    static NcclApi a;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) { a.why = std::string("dlopen(libnccl.so.2): ") + dlerror(); return; }
+        auto sym = [&](auto& f, const char* name) { f = reinterpret_cast<std::remove_reference_t<decltype(f)>>(dlsym(h, name)); return f != nullptr; };
+        a.ok = sym(a.CommInitAll, "ncclCommInitAll") && sym(a.AllReduce, "ncclAllReduce") &&
+               sym(a.GroupStart, "ncclGroupStart") && sym(a.GroupEnd, "ncclGroupEnd") &&
+               sym(a.CommGetAsyncError, "ncclCommGetAsyncError") && sym(a.CommAbort, "ncclCommAbort") &&
+               sym(a.CommDestroy, "ncclCommDestroy") && sym(a.GetErrorString, "ncclGetErrorString");
+        if (!a.ok) a.why = "libnccl.so.2 lacks a required symbol";
+    });
+    return a;
+}
+#define NK(expr)                                                                          \
+    do {                                                                                  \
+        ncclResult_t _r = (expr);                                                         \
+        if (_r != ncclSuccess)                                                            \
+            throw NcclError{std::string("NCCL ") + nccl_api().GetErrorString(_r) + " in " + #expr}; \
+    } while (0)
+
+}  // namespace
+
+struct MultiDev {
+    int P = 1;
+    bool loopback = false, use_nccl = false;
+    std::vector<int> dev;
+    std::vector<bted_ctx*> sub;                    // select: tile shards (rank p on dev[p])
+    std::vector<bted_ctx*> rep;                    // run_batches: replicas on dev[1..G) (rep[0] unused: the ctx)
+    std::vector<double*> qbuf;                     // [P] 2 qlen fp64 (ping-pong by step parity) on dev[p]
+    std::vector<double*> qsum;                     // [P] NCCL: the all-reduced q
+    std::vector<unsigned long long*> flag;         // [P] publish counters on dev[p]
+    std::vector<ncclComm_t> comms;
+    int64_t qlen = 0;
+    unsigned long long seq = 0;                    // last published counter value
+    unsigned long long timeout_ns = 20000000000ull;   // peer flag wait (BTED_PEER_TIMEOUT_MS)
+    int drop_publish = -1;                         // debug (BTED_DEBUG_DROP_PUBLISH): never publish on dev p
+    int64_t* wall = nullptr; size_t wallcap = 0;   // all batches' winners on dev[0]
+    // row bands (BTED_FLAG_DENSE): shard ctxs and their exchange buffers, all on dev[p]
+    std::vector<bted_ctx*> band;
+    std::vector<unsigned long long*> bkeys;        // [m] keys (band max, then the global max)
+    std::vector<float*> col, piv, cn, cns;          // column slice [Bw], pivot [W], partial / summed norms [ld]
+    std::vector<unsigned long long*> scratch;
+    std::vector<uint32_t*> cand;
+    std::vector<int*> ncand;
+    int64_t Bw = 0, W = 0, ld = 0;
+    int32_t band_m = 0;
+};
+
+namespace {
+
+// the shards / replicas and their exchange buffers (re-created lazily, e.g. after bted_update)
+void md_drop_replicas(MultiDev* md) {
+    for (int p = 0; p < (int)md->band.size(); ++p) {
+        DeviceGuard dg(md->dev[p]);
+        for (void* q : {(void*)md->bkeys[p], (void*)md->col[p], (void*)md->piv[p], (void*)md->cn[p],
+                        (void*)md->cns[p], (void*)md->scratch[p], (void*)md->cand[p], (void*)md->ncand[p]})
+            if (q) cudaFree(q);
+        bted_destroy(md->band[p]);
+    }
+    md->band.clear(); md->bkeys.clear(); md->col.clear(); md->piv.clear(); md->cn.clear(); md->cns.clear();
+    md->scratch.clear(); md->cand.clear(); md->ncand.clear();
+    md->band_m = 0;
+    for (auto* c : md->sub) bted_destroy(c);
+    for (auto* c : md->rep) if (c) bted_destroy(c);
+    md->sub.clear();
+    md->rep.clear();
+    for (int p = 0; p < (int)md->qbuf.size(); ++p) {
+        DeviceGuard dg(md->dev[p]);
+        if (md->qbuf[p]) cudaFree(md->qbuf[p]);
+        if (p < (int)md->qsum.size() && md->qsum[p]) cudaFree(md->qsum[p]);
+        if (md->flag[p]) cudaFree(md->flag[p]);
+    }
+    md->qbuf.clear();
+    md->qsum.clear();
+    md->flag.clear();
+    md->seq = 0;
+    if (!md->comms.empty() && nccl_api().ok)
+        for (auto c : md->comms) nccl_api().CommDestroy(c);
+    md->comms.clear();
+}
+
+void md_release(MultiDev* md) {
+    if (!md) return;
+    md_drop_replicas(md);
+    if (md->wall) { DeviceGuard dg(md->dev[0]); cudaFree(md->wall); }
+    delete md;
+}
+
+// the ctx's G devices: validated, peer access enabled between every pair
+bted_status md_init(bted_ctx* ctx) {
+    const int G = std::max(1, ctx->params.num_devices);
+    auto* md = new MultiDev();
+    md->P = G;
+    md->loopback = (ctx->params.flags & BTED_FLAG_LOOPBACK) != 0;
+    md->use_nccl = (ctx->params.flags & BTED_FLAG_NCCL) != 0;
+    if (const char* e = std::getenv("BTED_PEER_TIMEOUT_MS")) md->timeout_ns = (unsigned long long)(std::atof(e) * 1e6);
+    if (const char* e = std::getenv("BTED_DEBUG_DROP_PUBLISH")) md->drop_publish = std::atoi(e);
+    ctx->md = md;
+    if (G > bted::im::kMaxDev) { set_error("num_devices must be <= %d", bted::im::kMaxDev); return BTED_EINVAL; }
+    if (md->loopback && md->use_nccl) { set_error("BTED_FLAG_NCCL needs distinct devices (not LOOPBACK)"); return BTED_EINVAL; }
+    int ndev = 0;
+    CK(cudaGetDeviceCount(&ndev));
+    for (int p = 0; p < G; ++p) md->dev.push_back(md->loopback ? ctx->device : ctx->device + p);
+    if (!md->loopback && ctx->device + G > ndev) {
+        set_error("num_devices %d from device %d: only %d devices visible", G, ctx->device, ndev);
+        return BTED_EINVAL;
+    }
+    if (!md->loopback) {
+        for (int a = 0; a < G; ++a) {
+            DeviceGuard dg(md->dev[a]);
+            for (int b = 0; b < G; ++b) {
+                if (a == b) continue;
+                int can = 0;
+                CK(cudaDeviceCanAccessPeer(&can, md->dev[a], md->dev[b]));
+                if (!can && !md->use_nccl) {
+                    set_error("device %d cannot access device %d (no P2P): use BTED_FLAG_NCCL", md->dev[a], md->dev[b]);
+                    return BTED_ECUDA;
+                }
+                if (can) {
+                    cudaError_t e = cudaDeviceEnablePeerAccess(md->dev[b], 0);
+                    if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) CK(e);
+                    cudaGetLastError();
+                }
+            }
+        }
+    }
+    return BTED_OK;
+}
+
+// a ctx on dev[p] with its own copy of X (loopback: adopts the ctx's X and shares its stream)
+bted_ctx* md_replica(bted_ctx* ctx, int p) {
+    MultiDev& md = *ctx->md;
+    bted_params q = ctx->params;
+    q.device = md.dev[p];
+    q.num_devices = 1;
+    q.flags &= ~(uint32_t)(BTED_FLAG_LOOPBACK | BTED_FLAG_NCCL);
+    float* X = ctx->X;
+    bool own = false;
+    if (md.loopback) {
+        q.stream = reinterpret_cast<uintptr_t>(ctx->stream);
+    } else {
+        q.stream = 0;
+        DeviceGuard dg(md.dev[p]);
+        CK(cudaMalloc(&X, sizeof(float) * ctx->N * ctx->d));
+        CK(cudaMemcpyPeer(X, md.dev[p], ctx->X, ctx->device, sizeof(float) * ctx->N * ctx->d));
+        own = true;
+    }
+    q.x_on_device = 1;
+    bted_ctx* r = nullptr;
+    const bted_status st = create_common(X, ctx->N, ctx->d, ctx->kernel, &q, 0, ctx->N, false, &r);
+    if (st != BTED_OK) {
+        if (own) { DeviceGuard dg(md.dev[p]); cudaFree(X); }
+        throw CudaError{cudaErrorUnknown, "replica context creation"};
+    }
+    r->own_X = own;
+    return r;
+}
+
+void md_sync_all(MultiDev& md, const std::vector<bted_ctx*>& cs) {
+    for (size_t p = 0; p < cs.size(); ++p) {
+        DeviceGuard dg(md.dev[p]);
+        CK(cudaStreamSynchronize(cs[p]->stream));
+    }
+}
+
+// NCCL: wait for every stream with a deadline, polling the communicators' async errors
+void md_nccl_wait(MultiDev& md) {
+    double limit = 300.0;
+    if (const char* e = std::getenv("BTED_NCCL_TIMEOUT_S")) limit = std::atof(e);
+    const auto t0 = std::chrono::steady_clock::now();
+    for (;;) {
+        bool done = true;
+        for (int p = 0; p < md.P; ++p) {
+            DeviceGuard dg(md.dev[p]);
+            const cudaError_t q = cudaStreamQuery(md.sub[p]->stream);
+            if (q == cudaErrorNotReady) done = false;
+            else if (q != cudaSuccess) CK(q);
+            ncclResult_t ar = ncclSuccess;
+            NK(nccl_api().CommGetAsyncError(md.comms[p], &ar));
+            if (ar != ncclSuccess) {
+                for (auto c : md.comms) nccl_api().CommAbort(c);
+                md.comms.clear();
+                throw NcclError{std::string("NCCL async error: ") + nccl_api().GetErrorString(ar)};
+            }
+        }
+        if (done) return;
+        const double el = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+        if (el > limit) {
+            for (auto c : md.comms) nccl_api().CommAbort(c);
+            md.comms.clear();
+            throw NcclError{"NCCL collective did not complete within BTED_NCCL_TIMEOUT_S; communicators aborted"};
+        }
+        std::this_thread::sleep_for(std::chrono::microseconds(200));
+    }
+}
+
+// TED(V, mu, m) tile-sharded over the P devices; keys of every shard end identical.
+void md_select_loop(bted_ctx* ctx, int32_t m, float mu, const std::vector<unsigned long long>* forced) {
+    MultiDev& md = *ctx->md;
+    const int P = md.P;
+    const int64_t NPa = md.qlen;
+    auto pq_of = [&](int slot, unsigned long long expect) {
+        bted::im::PeerQ pq{};
+        pq.P = P;
+        pq.expect = expect;
+        pq.timeout_ns = md.timeout_ns;
+        for (int p = 0; p < P; ++p) { pq.q[p] = md.qbuf[p] + (size_t)slot * NPa; pq.flag[p] = md.flag[p]; }
+        return pq;
+    };
+    auto exchange = [&](int slot) {                 // after every device enqueued its partial into `slot`
+        if (md.use_nccl) {
+            NK(nccl_api().GroupStart());
+            for (int p = 0; p < P; ++p)
+                NK(nccl_api().AllReduce(md.qbuf[p] + (size_t)slot * NPa, md.qsum[p], (size_t)NPa, ncclFloat64, ncclSum,
+                                        md.comms[p], md.sub[p]->stream));
+            NK(nccl_api().GroupEnd());
+            return 0ull;
+        }
+        const unsigned long long e = ++md.seq;
+        for (int p = 0; p < P; ++p) {
+            if (p == md.drop_publish) continue;         // debug: a device that stopped (tests the timeout)
+            DeviceGuard dg(md.dev[p]);
+            bted::im::publish_kernel<<<1, 1, 0, md.sub[p]->stream>>>(md.flag[p], e);
+            LAUNCHED(1);
+        }
+        return e;
+    };
+    auto fin = [&](int32_t t, int slot, unsigned long long e) {
+        const bted::im::PeerQ pq = pq_of(slot, e);
+        for (int p = 0; p < P; ++p) {
+            DeviceGuard dg(md.dev[p]);
+            bted_ctx* c = md.sub[p];
+            ishard_fin_enqueue(c, t, mu, md.use_nccl ? md.qsum[p] : nullptr, c->ted.keys, md.use_nccl ? nullptr : &pq);
+        }
+    };
+    for (int p = 0; p < P; ++p) {
+        DeviceGuard dg(md.dev[p]);
+        bted_ctx* c = md.sub[p];
+        CK(cudaMemsetAsync(c->ted.keys, 0, sizeof(unsigned long long) * m, c->stream));
+        if (forced && !forced->empty())
+            CK(cudaMemcpyAsync(c->ted.keys, forced->data(), sizeof(unsigned long long) * forced->size(),
+                               cudaMemcpyHostToDevice, c->stream));
+        ishard_head_enqueue(c, m, md.qbuf[p]);                     // slot 0
+    }
+    fin(0, 0, exchange(0));
+    for (int32_t t = 1; t < m; ++t) {
+        const int slot = t & 1;
+        for (int p = 0; p < P; ++p) {
+            DeviceGuard dg(md.dev[p]);
+            bted_ctx* c = md.sub[p];
+            ishard_step_enqueue(c, t, mu, c->ted.keys, md.qbuf[p] + (size_t)slot * NPa);
+        }
+        fin(t, slot, exchange(slot));
+    }
+    if (md.use_nccl) md_nccl_wait(md);
+    else md_sync_all(md, md.sub);
+}
+
+bted_status md_select_bands(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, float* out_score);
+
+bted_status md_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, float* out_score) {
+    MultiDev& md = *ctx->md;
+    const int P = md.P;
+    if (ctx->d > 32) { set_error("multi-GPU select needs d <= 32"); return BTED_EINVAL; }
+    if (m > bted::im::kMaxM) { set_error("multi-GPU select needs m <= %d", bted::im::kMaxM); return BTED_EINVAL; }
+    if ((ctx->params.flags & BTED_FLAG_DENSE) || ctx->params.norm_mode == 1)
+        return md_select_bands(ctx, m, mu, out_idx, out_score);
+    const int nT = (int)((ctx->N + bted::pk::T - 1) / bted::pk::T);
+    if (bted::pk::num_tiles(nT) < P) { set_error("fewer Gram tiles than devices"); return BTED_EINVAL; }
+    if (md.sub.empty()) {
+        md.qlen = ishard_qlen_of(ctx->N);
+        for (int p = 0; p < P; ++p) {
+            bted_ctx* c = md_replica(ctx, p);
+            c->is_ishard = true;
+            c->srank = p;
+            c->snranks = P;
+            md.sub.push_back(c);
+            DeviceGuard dg(md.dev[p]);
+            double* q = nullptr;
+            unsigned long long* f = nullptr;
+            CK(cudaMalloc(&q, sizeof(double) * 2 * md.qlen));
+            CK(cudaMalloc(&f, sizeof(unsigned long long)));
+            CK(cudaMemset(f, 0, sizeof(unsigned long long)));
+            md.qbuf.push_back(q);
+            md.flag.push_back(f);
+            if (md.use_nccl) {
+                double* r = nullptr;
+                CK(cudaMalloc(&r, sizeof(double) * md.qlen));
+                md.qsum.push_back(r);
+            }
+        }
+        if (md.use_nccl) {
+            if (!nccl_api().ok) throw NcclError{"BTED_FLAG_NCCL: " + nccl_api().why};
+            md.comms.resize(P);
+            NK(nccl_api().CommInitAll(md.comms.data(), P, md.dev.data()));
+        }
+    }
+    for (int p = 0; p < P; ++p) {
+        DeviceGuard dg(md.dev[p]);
+        grow(md.sub[p]->ted.keys, md.sub[p]->ted.keyscap, (size_t)m);
+    }
+    md_select_loop(ctx, m, mu, nullptr);
+    // K4: every shard holds the same keys and features; shard 0 decides, all re-run
+    std::vector<float> fixed(m, -1.f);
+    bted_ctx* c0 = md.sub[0];
+    for (int rounds = 0; rounds <= m; ++rounds) {
+        std::vector<unsigned long long> forced;
+        DeviceGuard dg(md.dev[0]);
+        if (!ishard_k4(c0, m, mu, c0->ted.keys, forced)) break;
+        md_select_loop(ctx, m, mu, &forced);
+    }
+    for (int p = 1; p < P; ++p) {                 // a peer's numeric error / stall surfaces here
+        DeviceGuard dg(md.dev[p]);
+        CK(cudaMemcpy(ctx->herr, md.sub[p]->ted.err, sizeof(int), cudaMemcpyDeviceToHost));
+        if (*ctx->herr & bted::im::kErrPeerTimeout) {
+            ctx->poisoned = true;
+            set_error("multi-GPU exchange: a peer device never published its step (20 s flag wait)");
+            return BTED_ENCCL;
+        }
+        if (*ctx->herr) { set_error("non-finite score on device %d", md.dev[p]); return BTED_ENUMERIC; }
+    }
+    DeviceGuard dg(md.dev[0]);
+    const bted_status st = finish_keys(c0, c0->ted, c0->ted.keys, m, out_idx, out_score);
+    if (st != BTED_OK && c0->poisoned) ctx->poisoned = true;
+    return st;
+}
+
+// Row bands over the P devices (BTED_FLAG_DENSE): band p = rows [p Bw, (p+1) Bw)
+// of the dense K on dev[p].  Per step (Alg. 1 l.3-5): the pivot column slices
+// are published and gathered into every device's pivot row (bit-symmetry: column
+// s = row s), the band deflates and scores, the band maxima are published and
+// max-reduced.  norm_mode 1 (literal) adds the published partial column norms,
+// summed in rank order.  Bitwise the same as a dense single-GPU select in the
+// symmetric mode (every row's arithmetic depends on N only).
+void md_band_setup(bted_ctx* ctx, int32_t m) {
+    MultiDev& md = *ctx->md;
+    const int P = md.P;
+    if (!md.band.empty() && md.band_m >= m) return;
+    md_drop_replicas(&md);                       // (re)build: the keys / candidate buffers are sized by m
+    const int64_t N = ctx->N;
+    md.Bw = (N + P - 1) / P;
+    md.ld = ld_for(N);
+    md.W = std::max<int64_t>(md.ld, (int64_t)P * md.Bw);
+    for (int p = 0; p < P; ++p) {
+        bted_params q = ctx->params;
+        q.device = md.dev[p];
+        q.num_devices = 1;
+        q.flags &= ~(uint32_t)(BTED_FLAG_LOOPBACK | BTED_FLAG_NCCL);
+        float* X = ctx->X;
+        bool own = false;
+        DeviceGuard dg(md.dev[p]);
+        if (md.loopback) {
+            q.stream = reinterpret_cast<uintptr_t>(ctx->stream);
+        } else {
+            q.stream = 0;
+            CK(cudaMalloc(&X, sizeof(float) * N * ctx->d));
+            CK(cudaMemcpyPeer(X, md.dev[p], ctx->X, ctx->device, sizeof(float) * N * ctx->d));
+            own = true;
+        }
+        q.x_on_device = 1;
+        const int64_t r0 = std::min<int64_t>(N, p * md.Bw), r1 = std::min<int64_t>(N, (p + 1) * md.Bw);
+        if (r0 >= r1) throw CudaError{cudaErrorInvalidValue, "row bands: more devices than rows"};
+        bted_ctx* c = nullptr;
+        if (create_common(X, N, ctx->d, ctx->kernel, &q, r0, r1, true, &c) != BTED_OK) {
+            if (own) cudaFree(X);
+            throw CudaError{cudaErrorUnknown, "band context creation"};
+        }
+        c->own_X = own;
+        md.band.push_back(c);
+        unsigned long long* k = nullptr; float* a = nullptr; float* b = nullptr; float* e = nullptr; float* f = nullptr;
+        unsigned long long* sc = nullptr; uint32_t* cd = nullptr; int* nc = nullptr;
+        CK(cudaMalloc(&k, sizeof(unsigned long long) * m));
+        CK(cudaMalloc(&a, sizeof(float) * md.Bw));
+        CK(cudaMemset(a, 0, sizeof(float) * md.Bw));
+        CK(cudaMalloc(&b, sizeof(float) * md.W));
+        CK(cudaMemset(b, 0, sizeof(float) * md.W));
+        CK(cudaMalloc(&e, sizeof(float) * md.W));
+        CK(cudaMemset(e, 0, sizeof(float) * md.W));
+        CK(cudaMalloc(&f, sizeof(float) * md.W));
+        CK(cudaMemset(f, 0, sizeof(float) * md.W));
+        CK(cudaMalloc(&sc, sizeof(unsigned long long)));
+        CK(cudaMalloc(&cd, sizeof(uint32_t) * m * bted::rf::kMaxCand));
+        CK(cudaMalloc(&nc, sizeof(int) * m));
+        md.bkeys.push_back(k); md.col.push_back(a); md.piv.push_back(b); md.cn.push_back(e); md.cns.push_back(f);
+        md.scratch.push_back(sc); md.cand.push_back(cd); md.ncand.push_back(nc);
+        if (md.flag.size() < (size_t)P) {
+            unsigned long long* fl = nullptr;
+            CK(cudaMalloc(&fl, sizeof(unsigned long long)));
+            CK(cudaMemset(fl, 0, sizeof(unsigned long long)));
+            md.flag.push_back(fl);
+            md.qbuf.push_back(nullptr);
+        }
+    }
+    md.band_m = m;
+}
+
+void md_band_loop(bted_ctx* ctx, int32_t m, float mu, bool literal, const std::vector<unsigned long long>* forced) {
+    MultiDev& md = *ctx->md;
+    const int P = md.P;
+    auto peers = [&](auto bufs, unsigned long long e) {
+        bted::xg::Peers pk{};
+        pk.P = P;
+        pk.expect = e;
+        pk.timeout_ns = md.timeout_ns;
+        for (int p = 0; p < P; ++p) { pk.buf[p] = bufs[p]; pk.flag[p] = md.flag[p]; }
+        return pk;
+    };
+    auto publish = [&]() {
+        const unsigned long long e = ++md.seq;
+        for (int p = 0; p < P; ++p) {
+            if (p == md.drop_publish) continue;
+            DeviceGuard dg(md.dev[p]);
+            bted::im::publish_kernel<<<1, 1, 0, md.band[p]->stream>>>(md.flag[p], e);
+            LAUNCHED(1);
+        }
+        return e;
+    };
+    auto keymax = [&](int32_t t, unsigned long long e) {
+        const bted::xg::Peers pk = peers(md.bkeys, e);
+        for (int p = 0; p < P; ++p) {
+            DeviceGuard dg(md.dev[p]);
+            bted::xg::keymax_kernel<<<1, 32, 0, md.band[p]->stream>>>(pk, t, md.bkeys[p], md.band[p]->ted.err);
+            LAUNCHED(1);
+        }
+    };
+    auto sum_scores = [&](int32_t t, unsigned long long e) {
+        const bted::xg::Peers pk = peers(md.cn, e);
+        for (int p = 0; p < P; ++p) {
+            DeviceGuard dg(md.dev[p]);
+            bted_ctx* c = md.band[p];
+            bted::xg::sum_colnorm_kernel<<<(unsigned)std::min<int64_t>((md.ld + 255) / 256, 1024), 256, 0, c->stream>>>(
+                pk, md.ld, md.cns[p], c->ted.err);
+            LAUNCHED(1);
+            shard_scores_enqueue(c, t, mu, md.cns[p], reinterpret_cast<uint64_t*>(md.bkeys[p]));
+        }
+    };
+    for (int p = 0; p < P; ++p) {
+        DeviceGuard dg(md.dev[p]);
+        bted_ctx* c = md.band[p];
+        CK(cudaMemsetAsync(md.bkeys[p], 0, sizeof(unsigned long long) * m, c->stream));
+        if (forced && !forced->empty())
+            CK(cudaMemcpyAsync(md.bkeys[p], forced->data(), sizeof(unsigned long long) * forced->size(),
+                               cudaMemcpyHostToDevice, c->stream));
+        if (literal) {
+            shard_gram_enqueue(c, mu, reinterpret_cast<uint64_t*>(md.scratch[p]));
+            shard_colnorm_enqueue(c, 0, mu, nullptr, nullptr, md.cn[p]);
+        } else {
+            shard_gram_enqueue(c, mu, reinterpret_cast<uint64_t*>(md.bkeys[p]));
+        }
+    }
+    unsigned long long e = publish();
+    if (literal) { sum_scores(0, e); e = publish(); }
+    keymax(0, e);
+    for (int32_t t = 1; t < m; ++t) {
+        for (int p = 0; p < P; ++p) {
+            DeviceGuard dg(md.dev[p]);
+            shard_pivot_enqueue(md.band[p], t - 1, reinterpret_cast<uint64_t*>(md.bkeys[p]), md.col[p]);
+        }
+        e = publish();
+        const bted::xg::Peers pc = peers(md.col, e);
+        for (int p = 0; p < P; ++p) {
+            DeviceGuard dg(md.dev[p]);
+            bted_ctx* c = md.band[p];
+            bted::xg::gather_pivot_kernel<<<(unsigned)std::min<int64_t>((md.W + 255) / 256, 1024), 256, 0, c->stream>>>(
+                pc, md.Bw, ctx->N, md.W, md.piv[p], c->ted.err);
+            LAUNCHED(1);
+            if (literal) shard_colnorm_enqueue(c, t, mu, md.piv[p], reinterpret_cast<uint64_t*>(md.bkeys[p]), md.cn[p]);
+            else shard_step_enqueue(c, t, mu, md.piv[p], reinterpret_cast<uint64_t*>(md.bkeys[p]));
+        }
+        e = publish();
+        if (literal) { sum_scores(t, e); e = publish(); }
+        keymax(t, e);
+    }
+    std::vector<bted_ctx*> cs(md.band.begin(), md.band.end());
+    md_sync_all(md, cs);
+}
+
+bted_status md_select_bands(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, float* out_score) {
+    MultiDev& md = *ctx->md;
+    const int P = md.P;
+    const bool literal = ctx->params.norm_mode == 1;
+    if (md.use_nccl) { set_error("row bands exchange through peer memory (BTED_FLAG_NCCL: tile-sharded engine only)"); return BTED_EINVAL; }
+    if (ctx->N < P) { set_error("row bands: more devices than rows"); return BTED_EINVAL; }
+    md_band_setup(ctx, m);
+    md_band_loop(ctx, m, mu, literal, nullptr);
+    bted_ctx* c0 = md.band[0];
+    const size_t kMC = bted::rf::kMaxCand;
+    const int mm = std::min<int32_t>(m, bted::im::kMaxM);
+    for (int rounds = 0; c0->ted.refine && rounds <= m; ++rounds) {    // K4 over the bands' candidates
+        std::vector<uint32_t> ca((size_t)P * m * kMC, 0u);
+        std::vector<int32_t> na((size_t)P * m, 0);
+        for (int p = 0; p < P; ++p) {
+            DeviceGuard dg(md.dev[p]);
+            bted_ctx* c = md.band[p];
+            CK(cudaMemsetAsync(md.ncand[p], 0, sizeof(int) * m, c->stream));
+            if (c->ted.top2) {
+                bted::rf::shard_neartie_kernel<<<mm, 256, 0, c->stream>>>(c->ted.top2, c->ted.last_nC, md.bkeys[p],
+                                                                        bted::rf::kTau, md.cand[p], md.ncand[p]);
+                LAUNCHED(1);
+            }
+            CK(cudaMemcpyAsync(ca.data() + (size_t)p * m * kMC, md.cand[p], sizeof(uint32_t) * m * kMC,
+                               cudaMemcpyDeviceToHost, c->stream));
+            CK(cudaMemcpyAsync(na.data() + (size_t)p * m, md.ncand[p], sizeof(int) * m, cudaMemcpyDeviceToHost,
+                               c->stream));
+            CK(cudaStreamSynchronize(c->stream));
+        }
+        std::vector<unsigned long long> forced;
+        DeviceGuard dg(md.dev[0]);
+        if (!shard_k4_decide(c0, m, mu, md.bkeys[0], ca.data(), na.data(), P, forced)) break;
+        md_band_loop(ctx, m, mu, literal, &forced);
+    }
+    for (int p = 1; p < P; ++p) {
+        DeviceGuard dg(md.dev[p]);
+        CK(cudaMemcpy(ctx->herr, md.band[p]->ted.err, sizeof(int), cudaMemcpyDeviceToHost));
+        if (*ctx->herr & bted::im::kErrPeerTimeout) {
+            ctx->poisoned = true;
+            set_error("multi-GPU exchange: a peer device never published its step (flag wait timed out)");
+            return BTED_ENCCL;
+        }
+        if (*ctx->herr) { set_error("non-finite score on device %d", md.dev[p]); return BTED_ENUMERIC; }
+    }
+    DeviceGuard dg(md.dev[0]);
+    const bted_status st = finish_keys(c0, c0->ted, md.bkeys[0], m, out_idx, out_score);
+    if (st != BTED_OK && c0->poisoned) ctx->poisoned = true;
+    return st;
+}
+
+// Alg. 2 with batch b on device b mod G: one host thread per device runs its
+// batches (replica ctx; device 0 = this ctx), then the merge on device 0.
+bted_status md_run_batches(bted_ctx* ctx, int64_t M, int32_t m, float mu, int64_t* out_idx, int32_t* out_count,
+                           int64_t* out_batch_idx) {
+    MultiDev& md = *ctx->md;
+    const int G = md.P, B = ctx->params.num_batches;
+    if (md.rep.empty()) {
+        md.rep.assign(G, nullptr);
+        for (int p = 1; p < G; ++p) md.rep[p] = md_replica(ctx, p);
+    }
+    std::vector<bted_status> st(G, BTED_OK);
+    std::vector<std::string> msg(G);
+    std::vector<int> nbs(G, 0);
+    auto work = [&](int p) {
+        bted_ctx* c = p == 0 ? ctx : md.rep[p];
+        st[p] = guarded(c, [&]() -> bted_status {
+            nbs[p] = run_batch_range(c, M, m, mu, p, G);
+            return batch_range_finish(c, nbs[p]);
+        });
+        if (st[p] != BTED_OK) msg[p] = bted_last_error();
+    };
+    if (md.loopback) {
+        for (int p = 0; p < G; ++p) work(p);       // one stream: the replicas run in turn
+    } else {
+        std::vector<std::thread> th;
+        for (int p = 1; p < G; ++p) th.emplace_back(work, p);
+        work(0);
+        for (auto& t : th) t.join();
+    }
+    for (int p = 0; p < G; ++p)
+        if (st[p] != BTED_OK) { set_error("device %d: %s", md.dev[p], msg[p].c_str()); return st[p]; }
+    // l.5 exchange: every batch's winners to device 0, in batch order (b = p + k G)
+    grow(md.wall, md.wallcap, (size_t)B * m);
+    for (int p = 0; p < G; ++p) {
+        bted_ctx* c = p == 0 ? ctx : md.rep[p];
+        for (int k = 0; k < nbs[p]; ++k) {
+            const int b = p + k * G;
+            CK(cudaMemcpyPeerAsync(md.wall + (size_t)b * m, md.dev[0], c->winners + (size_t)k * m, md.dev[p],
+                                   sizeof(int64_t) * m, ctx->stream));
+        }
+    }
+    if (out_batch_idx) {
+        CK(cudaMemcpyAsync(out_batch_idx, md.wall, sizeof(int64_t) * (size_t)B * m, cudaMemcpyDeviceToHost,
+                           ctx->stream));
+    }
+    return merge_device(ctx, md.wall, (int64_t)B * m, m, mu, out_idx, out_count);
+}
+
+}  // namespace
+
 // ======================================================================= ABI
 extern "C" {
 
@@ -1535,11 +2415,22 @@ void bted_default_params(bted_params* p) {
     p->gamma = 1.0f;
     p->device = -1;
     p->num_batches = 1;
+    p->num_devices = 1;
+    p->norm_mode = 0;
 }
 
 bted_status bted_create(const float* X, int64_t N, int32_t d, bted_kernel kernel, const bted_params* params,
                         bted_ctx** out) {
-    return create_common(X, N, d, kernel, params, 0, N, false, out);
+    bted_status st = create_common(X, N, d, kernel, params, 0, N, false, out);
+    if (st != BTED_OK || (params->num_devices <= 1 && !(params->flags & BTED_FLAG_NCCL))) return st;
+    st = guarded(*out, [&]() { return md_init(*out); });
+    if (st != BTED_OK) {
+        const std::string why = bted_last_error();
+        bted_destroy(*out);
+        *out = nullptr;
+        set_error("%s", why.c_str());
+    }
+    return st;
 }
 
 bted_status bted_shard_create(const float* X, int64_t N, int32_t d, bted_kernel kernel, int64_t row0,
@@ -1551,6 +2442,7 @@ bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, fl
     if (!ctx || !out_idx) { set_error("null argument"); return BTED_EINVAL; }
     if (ctx->is_shard || ctx->is_ishard) { set_error("bted_select on a shard context"); return BTED_EINVAL; }
     if (m < 1 || m > ctx->N || !mu_ok(mu)) { set_error("need 1 <= m <= N and mu > 0 finite"); return BTED_EINVAL; }
+    if (ctx->md) return guarded(ctx, [&]() { return md_select(ctx, m, mu, out_idx, out_score); });
     return guarded(ctx, [&]() -> bted_status {
         Ted& T = ctx->ted;
         if (use_small(ctx->params.flags, ctx->N)) {
@@ -1603,36 +2495,11 @@ bted_status bted_batch_teds(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32
     }
     return guarded(ctx, [&]() -> bted_status {
         const int nb = run_batch_range(ctx, M, m, mu, b_begin, b_step);
-        const size_t bytes = sizeof(int64_t) * (size_t)nb * m;
-        if (nb > 0)
-            CK(cudaMemcpyAsync(out_winners, ctx->winners, bytes,
+        if (bted_status s = batch_range_finish(ctx, nb)) return s;
+        if (nb > 0) {
+            CK(cudaMemcpyAsync(out_winners, ctx->winners, sizeof(int64_t) * (size_t)nb * m,
                                winners_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, ctx->stream));
-        *ctx->herr = 0;
-        if (nb > 0)
-            CK(cudaMemcpyAsync(ctx->herr, ctx->bted_engine.err, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
-        CK(cudaStreamSynchronize(ctx->stream));
-        ctx->bted_engine.collect();
-        if (ctx->k4b.pending) {                          // K4 of small batch TEDs
-            ctx->k4b.pending = false;
-            auto& b = ctx->k4b;
-            if (small_k4_refine(ctx, ctx->stream, ctx->xall, b.ninst, b.M, ctx->d, b.m, b.mu, ctx->kall,
-                                ctx->bted_engine.err)) {
-                for (int kk = 0; kk < b.ninst; ++kk) {
-                    bted::map_winners_kernel<<<(b.m + 127) / 128, 128, 0, ctx->stream>>>(
-                        ctx->kall + (size_t)kk * b.m, b.m, ctx->sall + (size_t)kk * b.M, ctx->winners + (size_t)kk * b.m);
-                    LAUNCHED(1);
-                }
-                CK(cudaMemcpyAsync(out_winners, ctx->winners, bytes,
-                                   winners_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, ctx->stream));
-                CK(cudaStreamSynchronize(ctx->stream));
-            }
-        }
-        if (take_xbad(ctx)) return BTED_EINVAL;
-        if (nb > 0 && *ctx->herr) {
-            CK(cudaMemsetAsync(ctx->bted_engine.err, 0, sizeof(int), ctx->stream));
-            set_error((*ctx->herr & bted::kSampleOverflow) ? "batch sampler: candidate bin overflow (internal limit kCandCap)"
-                                                         : "non-finite score during a batch TED");
-            return BTED_ENUMERIC;
+            CK(cudaStreamSynchronize(ctx->stream));
         }
         return BTED_OK;
     });
@@ -1661,6 +2528,8 @@ bted_status bted_run_batches(bted_ctx* ctx, int64_t M, int32_t m, float mu, int6
     if (!ctx || !out_idx || !out_count) { set_error("null argument"); return BTED_EINVAL; }
     if (ctx->is_shard || ctx->is_ishard) { set_error("run_batches on a shard context"); return BTED_EINVAL; }
     if (m < 1 || M < m || M > ctx->N || !mu_ok(mu)) { set_error("need 1 <= m <= M <= N and mu > 0"); return BTED_EINVAL; }
+    if (ctx->md)
+        return guarded(ctx, [&]() { return md_run_batches(ctx, M, m, mu, out_idx, out_count, out_batch_idx); });
     return guarded(ctx, [&]() -> bted_status {
         ctx->k4b.changed = false;
         const int nb = run_batch_range(ctx, M, m, mu, 0, 1);
@@ -1720,18 +2589,7 @@ bted_status bted_sample_batches(int64_t P, int64_t M, int32_t B, uint64_t seed, 
 bted_status bted_shard_gram(bted_ctx* ctx, float mu, uint64_t* keys_dev) {
     if (!ctx || !keys_dev || !ctx->is_shard || !mu_ok(mu)) { set_error("bad shard_gram arguments"); return BTED_EINVAL; }
     return guarded(ctx, [&]() -> bted_status {
-        Ted& T = ctx->ted;
-        const int64_t rows = ctx->row1 - ctx->row0;
-        T.reserve(rows, ctx->N, ctx->d, 2);
-        T.last_rows = rows;
-        T.last_ld = ld_for(ctx->N);
-        T.last_buf = 0;
-        launch_transpose(T, ctx->X, ctx->N, ctx->d);
-        CK(cudaMemsetAsync(T.sel, 0, (size_t)rows, T.stream));
-        // K4: per-CTA top-2 keys of the first kMaxM steps (bted_shard_nearties / bted_shard_refine)
-        if (T.refine) T.reserve_refine((rows + kRowsPerK2Cta - 1) / kRowsPerK2Cta * 32, bted::im::kMaxM);
-        launch_gram(T, ctx->N, ctx->d, ctx->row0, rows, ctx->params.gamma, ctx->kernel, mu,
-                    reinterpret_cast<unsigned long long*>(keys_dev), T.refine ? T.top2 : nullptr);
+        shard_gram_enqueue(ctx, mu, keys_dev);
         return BTED_OK;
     });
 }
@@ -1741,11 +2599,7 @@ bted_status bted_shard_step(bted_ctx* ctx, int32_t t, float mu, const float* piv
         set_error("bad shard_step arguments"); return BTED_EINVAL;
     }
     return guarded(ctx, [&]() -> bted_status {
-        Ted& T = ctx->ted;
-        const int64_t rows = ctx->row1 - ctx->row0;
-        launch_step(T, ctx->N, ctx->row0, rows, t, mu, pivot_dev, reinterpret_cast<unsigned long long*>(keys_dev),
-                    (T.refine && T.top2 && t < bted::im::kMaxM) ? T.top2 : nullptr);
-        T.last_buf = t & 1;
+        shard_step_enqueue(ctx, t, mu, pivot_dev, keys_dev);
         return BTED_OK;
     });
 }
@@ -1753,13 +2607,7 @@ bted_status bted_shard_step(bted_ctx* ctx, int32_t t, float mu, const float* piv
 bted_status bted_shard_pivot_column(bted_ctx* ctx, int32_t t, const uint64_t* keys_dev, float* col_dev) {
     if (!ctx || !keys_dev || !col_dev || !ctx->is_shard || t < 0) { set_error("bad pivot_column arguments"); return BTED_EINVAL; }
     return guarded(ctx, [&]() -> bted_status {
-        Ted& T = ctx->ted;
-        const int32_t rows = (int32_t)(ctx->row1 - ctx->row0);
-        const unsigned g = (unsigned)std::min<int64_t>((rows + 255) / 256, 1024);
-        bted::pivot_column_kernel<<<g, 256, 0, T.stream>>>(T.K[t & 1], ld_for(ctx->N), rows,
-                                                           reinterpret_cast<const unsigned long long*>(keys_dev), t,
-                                                           col_dev);
-        LAUNCHED(1);
+        shard_pivot_enqueue(ctx, t, keys_dev, col_dev);
         return BTED_OK;
     });
 }
@@ -1770,23 +2618,7 @@ bted_status bted_shard_colnorm(bted_ctx* ctx, int32_t t, float mu, const float* 
         set_error("bad shard_colnorm arguments"); return BTED_EINVAL;
     }
     return guarded(ctx, [&]() -> bted_status {
-        Ted& T = ctx->ted;
-        const int64_t ld = ld_for(ctx->N);
-        const int32_t rows = (int32_t)(ctx->row1 - ctx->row0);
-        const int32_t nchunks = (rows + bted::kColChunk - 1) / bted::kColChunk;
-        grow(T.P, T.pcap, (size_t)nchunks * (size_t)ld);
-        const dim3 grid((unsigned)((ld + 255) / 256), (unsigned)nchunks);
-        const auto* keys = reinterpret_cast<const unsigned long long*>(keys_dev);
-        if (t == 0)
-            bted::deflate_colnorm_kernel<false><<<grid, bted::kColThreads, 0, T.stream>>>(
-                T.K[0], nullptr, ld, (int32_t)ctx->row0, rows, nullptr, nullptr, 0, mu, T.sel, T.P);
-        else
-            bted::deflate_colnorm_kernel<true><<<grid, bted::kColThreads, 0, T.stream>>>(
-                T.K[(t - 1) & 1], T.K[t & 1], ld, (int32_t)ctx->row0, rows, pivot_dev, keys, t, mu, T.sel, T.P);
-        const unsigned g2 = (unsigned)std::min<int64_t>((ld + 255) / 256, 2048);
-        bted::colnorm_reduce_kernel<<<g2, 256, 0, T.stream>>>(T.P, nchunks, ld, colnorm_dev);
-        LAUNCHED(2);
-        T.last_buf = t & 1;
+        shard_colnorm_enqueue(ctx, t, mu, pivot_dev, keys_dev, colnorm_dev);
         return BTED_OK;
     });
 }
@@ -1796,39 +2628,12 @@ bted_status bted_shard_scores(bted_ctx* ctx, int32_t t, float mu, const float* c
         set_error("bad shard_scores arguments"); return BTED_EINVAL;
     }
     return guarded(ctx, [&]() -> bted_status {
-        Ted& T = ctx->ted;
-        const int32_t rows = (int32_t)(ctx->row1 - ctx->row0);
-        unsigned g = (unsigned)std::min<int64_t>((rows + 255) / 256, 1184);
-        // K4: one CTA per top-2 slot pair of the step (T.last_nC, set by bted_shard_gram),
-        // so bted_shard_nearties reads the literal mode's keys like the symmetric mode's
-        unsigned long long* top2 = nullptr;
-        if (T.refine && T.top2 && t < bted::im::kMaxM && T.last_nC > 0) {
-            g = (unsigned)T.last_nC;
-            top2 = T.top2 + (int64_t)t * T.last_nC * 2;
-        }
-        bted::colnorm_scores_kernel<<<g, 256, 0, T.stream>>>(T.K[t & 1], ld_for(ctx->N), (int32_t)ctx->row0, rows,
-                                                             colnorm_dev, mu, T.sel,
-                                                             reinterpret_cast<unsigned long long*>(keys_dev), t, T.err,
-                                                             top2);
-        LAUNCHED(1);
+        shard_scores_enqueue(ctx, t, mu, colnorm_dev, keys_dev);
         return BTED_OK;
     });
 }
 
 // ------------------------------------------------------------------ tile-sharded implicit engine
-namespace {
-int64_t ishard_local_tiles(const bted_ctx* ctx) {
-    const int nT = (int)((ctx->N + bted::pk::T - 1) / bted::pk::T);
-    const int64_t all = bted::pk::num_tiles(nT);
-    return (all - ctx->srank + ctx->snranks - 1) / ctx->snranks;
-}
-bted::im::XKern ishard_xk(const bted_ctx* ctx) {
-    bted::im::XKern xk;
-    xk.X = ctx->X; xk.d = ctx->d; xk.ng = -ctx->params.gamma; xk.linear = ctx->kernel == BTED_KERNEL_LINEAR ? 1 : 0;
-    return xk;
-}
-}  // namespace
-
 bted_status bted_ishard_create(const float* X, int64_t N, int32_t d, bted_kernel kernel, int32_t rank, int32_t nranks,
                                const bted_params* params, bted_ctx** out) {
     if (nranks < 1 || rank < 0 || rank >= nranks) { set_error("need 0 <= rank < nranks"); return BTED_EINVAL; }
@@ -1848,8 +2653,7 @@ bted_status bted_ishard_create(const float* X, int64_t N, int32_t d, bted_kernel
 
 int64_t bted_ishard_qlen(const bted_ctx* ctx) {
     if (!ctx) return 0;
-    const int64_t NP = (ctx->N + bted::pk::T - 1) / bted::pk::T * bted::pk::T;
-    return (NP + 255) / 256 * 256;
+    return ishard_qlen_of(ctx->N);
 }
 
 bted_status bted_ishard_head(bted_ctx* ctx, int32_t m, float mu, double* q_dev) {
@@ -1857,35 +2661,7 @@ bted_status bted_ishard_head(bted_ctx* ctx, int32_t m, float mu, double* q_dev) 
         set_error("bad ishard_head arguments"); return BTED_EINVAL;
     }
     return guarded(ctx, [&]() -> bted_status {
-        Ted& T = ctx->ted;
-        const int64_t N = ctx->N, NPa = bted_ishard_qlen(ctx);
-        const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
-        const int64_t lt = ishard_local_tiles(ctx);
-        ensure_implicit_attrs();
-        T.reserve_implicit(N, m, lt);
-        ctx->sm_m = m;
-        CK(cudaMemsetAsync(T.sel, 0, (size_t)NPa, T.stream));
-        CK(cudaMemsetAsync(T.kflag, 0, sizeof(int), T.stream));
-        CK(cudaMemsetAsync(T.tctr, 0, sizeof(int) * m, T.stream));
-        CK(cudaMemsetAsync(q_dev, 0, sizeof(double) * NPa, T.stream));
-        const int lin = ctx->kernel == BTED_KERNEL_LINEAR ? 1 : 0;
-        const float g = ctx->params.gamma;
-        const int r = ctx->srank, P = ctx->snranks;
-        auto k1i = [&](auto kern) {
-            kern<<<(unsigned)lt, bted::pk::kConsumers, 0, T.stream>>>(ctx->X, (int32_t)N, ctx->d, g, T.K[0], nT, r, P);
-        };
-        if (ctx->d <= 16) {
-            if (lin) k1i(bted::pk::gram_tile2_kernel<16, true, 4>); else k1i(bted::pk::gram_tile2_kernel<16, false, 4>);
-        } else {
-            if (lin) k1i(bted::pk::gram_tile_kernel<32, true>); else k1i(bted::pk::gram_tile_kernel<32, false>);
-        }
-        bted::im::diag_init_kernel<<<(unsigned)((NPa + 255) / 256), 256, 0, T.stream>>>(ishard_xk(ctx), (int32_t)N,
-                                                                                         NPa, T.rd);
-        bted::im::tile_pass_kernel<true><<<tile_pass_grid(lt), bted::im::kTPThreads, bted::im::tile_pass_smem_bytes,
-                                           T.stream>>>(T.K[0], nT, nullptr, T.P64, T.kflag, T.tctr, 0, 0, r, P);
-        bted::im::qpart_kernel<<<(unsigned)std::min<int64_t>((NPa + 255) / 256, 4096), 256, 0, T.stream>>>(
-            T.P64, nT, r, P, q_dev);
-        LAUNCHED(4);
+        ishard_head_enqueue(ctx, m, q_dev);
         return BTED_OK;
     });
 }
@@ -1895,21 +2671,7 @@ bted_status bted_ishard_step(bted_ctx* ctx, int32_t t, float mu, const uint64_t*
         set_error("bad ishard_step arguments (head first; 1 <= t < m)"); return BTED_EINVAL;
     }
     return guarded(ctx, [&]() -> bted_status {
-        Ted& T = ctx->ted;
-        const int64_t N = ctx->N, NPa = bted_ishard_qlen(ctx);
-        const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
-        const int nA = (int)(NPa / bted::im::kEllRows);
-        const int32_t m = ctx->sm_m;
-        const auto* keys = reinterpret_cast<const unsigned long long*>(keys_dev);
-        bted::im::ell_kernel<<<(unsigned)nA + 1, bted::im::kThreads, 0, T.stream>>>(
-            T.K[0], nT, (int32_t)N, T.Lf, NPa, t - 1, T.rd, T.nv, mu, keys, t, T.ell, T.Qc, T.G, m, T.hv, T.sel,
-            ishard_xk(ctx));
-        bted::im::tile_pass_kernel<false><<<tile_pass_grid(ishard_local_tiles(ctx)), bted::im::kTPThreads,
-                                            bted::im::tile_pass_smem_bytes, T.stream>>>(
-            T.K[0], nT, T.ell, T.P64, T.kflag, T.tctr + t, (int)(t & 1), 0, ctx->srank, ctx->snranks);
-        bted::im::qpart_kernel<<<(unsigned)std::min<int64_t>((NPa + 255) / 256, 4096), 256, 0, T.stream>>>(
-            T.P64, nT, ctx->srank, ctx->snranks, q_dev);
-        LAUNCHED(3);
+        ishard_step_enqueue(ctx, t, mu, reinterpret_cast<const unsigned long long*>(keys_dev), q_dev);
         return BTED_OK;
     });
 }
@@ -1919,15 +2681,7 @@ bted_status bted_ishard_fin(bted_ctx* ctx, int32_t t, float mu, const double* q_
         set_error("bad ishard_fin arguments (head first; 0 <= t < m)"); return BTED_EINVAL;
     }
     return guarded(ctx, [&]() -> bted_status {
-        Ted& T = ctx->ted;
-        const int64_t N = ctx->N, NPa = bted_ishard_qlen(ctx);
-        const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
-        const int64_t NP = (int64_t)nT * bted::pk::T;
-        auto* keys = reinterpret_cast<unsigned long long*>(keys_dev);
-        bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
-            T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, NPa, t > 0 ? t - 1 : 0, T.hv, T.nv, T.rd, T.sel, keys, t,
-            keys + t, T.err, T.refine ? T.top2 : nullptr, T.Qc, q_dev, t == 0 ? T.rd : nullptr);
-        LAUNCHED(1);
+        ishard_fin_enqueue(ctx, t, mu, q_dev, reinterpret_cast<unsigned long long*>(keys_dev));
         return BTED_OK;
     });
 }
@@ -1939,25 +2693,8 @@ bted_status bted_ishard_refine(bted_ctx* ctx, int32_t m, float mu, const uint64_
     }
     *nforced = 0;
     return guarded(ctx, [&]() -> bted_status {
-        Ted& T = ctx->ted;
-        if (!T.refine) return BTED_OK;
-        cudaStream_t st = T.stream;
-        const auto* keys = reinterpret_cast<const unsigned long long*>(keys_dev);
-        CK(cudaMemsetAsync(T.nflag, 0, sizeof(int), st));
-        bted::rf::neartie_check_kernel<<<m, 256, 0, st>>>(T.top2, T.last_nC, keys, bted::rf::kTau, T.flags, T.cand,
-                                                         T.ncand, T.nflag);
-        LAUNCHED(1);
-        std::vector<unsigned long long> hk(m);
-        std::vector<int> fl(m), nc(m);
-        std::vector<uint32_t> cd((size_t)m * bted::rf::kMaxCand);
-        CK(cudaMemcpyAsync(hk.data(), keys, sizeof(unsigned long long) * m, cudaMemcpyDeviceToHost, st));
-        CK(cudaMemcpyAsync(fl.data(), T.flags, sizeof(int) * m, cudaMemcpyDeviceToHost, st));
-        CK(cudaMemcpyAsync(nc.data(), T.ncand, sizeof(int) * m, cudaMemcpyDeviceToHost, st));
-        CK(cudaMemcpyAsync(cd.data(), T.cand, sizeof(uint32_t) * cd.size(), cudaMemcpyDeviceToHost, st));
-        CK(cudaStreamSynchronize(st));
         std::vector<unsigned long long> forced;
-        int checked = -1;
-        if (k4_next_correction(ctx, st, ctx->X, ctx->N, ctx->d, m, mu, hk, fl, nc, cd, checked, forced)) {
+        if (ishard_k4(ctx, m, mu, reinterpret_cast<const unsigned long long*>(keys_dev), forced)) {
             for (size_t q = 0; q < forced.size(); ++q) forced_host[q] = forced[q];
             *nforced = (int32_t)forced.size();
         }
@@ -1991,33 +2728,9 @@ bted_status bted_shard_refine(bted_ctx* ctx, int32_t m, float mu, const uint64_t
     }
     *nforced = 0;
     return guarded(ctx, [&]() -> bted_status {
-        Ted& T = ctx->ted;
-        if (!T.refine) return BTED_OK;
-        const size_t kMC = bted::rf::kMaxCand;
-        std::vector<unsigned long long> hk(m), forced;
-        CK(cudaMemcpyAsync(hk.data(), keys_dev, sizeof(unsigned long long) * m, cudaMemcpyDeviceToHost, T.stream));
-        CK(cudaStreamSynchronize(T.stream));
-        // every rank's band candidates of each step, merged (sorted, unique, at most kMaxCand)
-        std::vector<int> fl(m, 0), nc(m, 0);
-        std::vector<uint32_t> cd((size_t)m * kMC);
-        for (int t = 0; t < m; ++t) {
-            std::vector<uint32_t> c;
-            bool incomplete = false;
-            for (int r = 0; r < nranks; ++r) {
-                const int n0 = ncand_all[(size_t)r * m + t];
-                if (n0 < 0) { incomplete = true; continue; }           // the band's list may miss candidates
-                const int n = std::min<int>(n0, (int)kMC);
-                for (int q = 0; q < n; ++q) c.push_back(cand_all[((size_t)r * m + t) * kMC + q]);
-            }
-            std::sort(c.begin(), c.end());
-            c.erase(std::unique(c.begin(), c.end()), c.end());
-            if (c.size() > kMC) { incomplete = true; c.resize(kMC); }
-            fl[t] = incomplete ? bted::rf::kFlagFull : c.size() >= 2 ? bted::rf::kFlagNear : 0;
-            nc[t] = (int)c.size();
-            std::copy(c.begin(), c.end(), cd.begin() + (size_t)t * kMC);
-        }
-        int checked = -1;
-        if (k4_next_correction(ctx, T.stream, ctx->X, ctx->N, ctx->d, m, mu, hk, fl, nc, cd, checked, forced)) {
+        std::vector<unsigned long long> forced;
+        if (shard_k4_decide(ctx, m, mu, reinterpret_cast<const unsigned long long*>(keys_dev), cand_all, ncand_all,
+                            nranks, forced)) {
             std::copy(forced.begin(), forced.end(), forced_host);
             *nforced = (int32_t)forced.size();
         }
@@ -2050,6 +2763,10 @@ bted_status bted_update(bted_ctx* ctx, const float* X, int32_t x_on_device) {
         // the caller must keep a host X alive until the next call returns.  The
         // finiteness check runs on the device; a bad X fails the next call (EINVAL).
         launch_finite_check(ctx);
+        if (ctx->md) {                       // the devices' copies are rebuilt from the new X on next use
+            CK(cudaStreamSynchronize(ctx->stream));
+            md_drop_replicas(ctx->md);
+        }
         return BTED_OK;
     });
 }
@@ -2072,31 +2789,48 @@ void bted_host_free(void* p) {
 
 bted_status bted_get_stats(bted_ctx* ctx, bted_stats* out) {
     if (!ctx || !out) { set_error("null argument"); return BTED_EINVAL; }
-    const Stats& a = ctx->ted.stats;
-    const Stats& b = ctx->bted_engine.stats;
-    out->teds = a.teds + b.teds;
-    out->k2_launches = a.k2_launches + b.k2_launches;
-    out->k1_ms = a.k1_ms + b.k1_ms;
-    out->k2_ms = a.k2_ms + b.k2_ms;
-    out->small_teds = a.small_teds + b.small_teds;
-    out->small_ms = a.small_ms + b.small_ms;
-    out->refined_steps = ctx->refined_steps;
-    out->corrected_steps = ctx->corrected_steps;
-    out->full_refined_steps = ctx->full_refined_steps;
+    std::memset(out, 0, sizeof *out);
+    std::vector<bted_ctx*> all{ctx};
+    if (ctx->md) {                                 // multi-GPU: the replicas' batches + shard 0's K4
+        for (auto* c : ctx->md->rep) if (c) all.push_back(c);
+        if (!ctx->md->sub.empty()) all.push_back(ctx->md->sub[0]);
+    }
+    for (bted_ctx* c : all) {
+        for (const Stats* a : {&c->ted.stats, &c->bted_engine.stats}) {
+            out->teds += a->teds;
+            out->k2_launches += a->k2_launches;
+            out->k1_ms += a->k1_ms;
+            out->k2_ms += a->k2_ms;
+            out->small_teds += a->small_teds;
+            out->small_ms += a->small_ms;
+        }
+        out->refined_steps += c->refined_steps;
+        out->corrected_steps += c->corrected_steps;
+        out->full_refined_steps += c->full_refined_steps;
+    }
     return BTED_OK;
 }
 
 bted_status bted_reset_stats(bted_ctx* ctx) {
     if (!ctx) { set_error("null argument"); return BTED_EINVAL; }
-    ctx->ted.stats = Stats{};
-    ctx->bted_engine.stats = Stats{};
-    ctx->refined_steps = ctx->corrected_steps = ctx->full_refined_steps = 0;
+    std::vector<bted_ctx*> all{ctx};
+    if (ctx->md) {
+        for (auto* c : ctx->md->rep) if (c) all.push_back(c);
+        for (auto* c : ctx->md->sub) all.push_back(c);
+    }
+    for (bted_ctx* c : all) {
+        c->ted.stats = Stats{};
+        c->bted_engine.stats = Stats{};
+        c->refined_steps = c->corrected_steps = c->full_refined_steps = 0;
+    }
     return BTED_OK;
 }
 
 // ------------------------------------------------------------------ misc
 void bted_destroy(bted_ctx* ctx) {
     if (!ctx) return;
+    md_release(ctx->md);
+    ctx->md = nullptr;
     {
         DeviceGuard dg(ctx->device);
         if (ctx->stream) cudaStreamSynchronize(ctx->stream);

@@ -507,6 +507,60 @@ ell_kernel(const float* __restrict__ K, int nT, int32_t N, double* __restrict__ 
 // r_vv -= l_v^2.  Score n_v / (r_vv + mu) rounded to fp32, masked, packed key.
 // Unit = 32 rows (lanes) x 8 warps; warp w sums the J-range and the k-range
 // w of its rows, the 8 partial sums are added in warp order.
+// In-library multi-GPU exchange (bted_select with num_devices = P > 1): the P
+// devices' partial q = K l live in their own memory; every device's score
+// kernel waits for all P "published" flags and sums the P partials itself,
+// in rank order, through peer (NVLink) loads -- the all-reduce fused into its
+// consumer, bitwise identical on every device and independent of P's layout.
+constexpr int kMaxDev = 16;
+constexpr int kErrPeerTimeout = 32;           // error-word bit: a peer never published (ENCCL)
+struct PeerQ {
+    const double* q[kMaxDev];                 // device p's partial q of this step
+    const unsigned long long* flag[kMaxDev];  // device p's publish counter
+    int P;
+    unsigned long long expect;                // this step's counter value
+    unsigned long long timeout_ns;            // give up (kErrPeerTimeout) after this long
+    __device__ __forceinline__ double sum(int64_t i) const {
+        double a = __ldcv(&q[0][i]);
+        for (int p = 1; p < P; ++p) a = __dadd_rn(a, __ldcv(&q[p][i]));
+        return a;
+    }
+};
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+// thread 0 of the CTA waits until every device published `expect` (timeout ->
+// kErrPeerTimeout, after which no later wait of this device blocks), then the
+// CTA proceeds
+__device__ __forceinline__ void wait_peers(const PeerQ& pq, int* err) {
+    if (threadIdx.x == 0) {
+        const unsigned long long t0 = globaltimer_ns();
+        for (int p = 0; p < pq.P; ++p) {
+            while (ld_acquire_sys(pq.flag[p]) < pq.expect) {
+                if ((*(volatile int*)err & kErrPeerTimeout) || globaltimer_ns() - t0 > pq.timeout_ns) {
+                    atomicOr(err, kErrPeerTimeout);
+                    break;
+                }
+                __nanosleep(64);
+            }
+        }
+    }
+    __syncthreads();
+}
+// after the producers of this stream's step completed: make their writes
+// visible system-wide, then publish the step counter
+__global__ void publish_kernel(unsigned long long* flag, unsigned long long v) {
+    __threadfence_system();
+    asm volatile("st.release.sys.global.u64 [%0], %1;" :: "l"(flag), "l"(v) : "memory");
+}
+
 constexpr int kFinRows = 32;
 struct FinSmem {
     double part[8][kFinRows];
@@ -522,7 +576,8 @@ __device__ __forceinline__ void fin_unit(int unit, int nunits, FinSmem& sm, Sync
                                          double* rdiag, const uint8_t* sel, uint32_t s,
                                          int32_t t, unsigned long long* key_out, int* err,
                                          unsigned long long* top2, double* Qc, bool mark_sel = false,
-                                         const double* qin = nullptr, const double* rinit = nullptr) {
+                                         const double* qin = nullptr, const double* rinit = nullptr,
+                                         const PeerQ* pq = nullptr) {
     const int lane = threadIdx.x % 32, w = threadIdx.x / 32;
     const int64_t NP = (int64_t)nT * T;
     const int i = unit * kFinRows + lane;
@@ -531,7 +586,9 @@ __device__ __forceinline__ void fin_unit(int unit, int nunits, FinSmem& sm, Sync
     const int per = (nT + 7) / 8;
     const int j0 = min(nT, w * per), j1 = min(nT, j0 + per);
     double acc = 0.0;
-    if (qin) {                                             // q given (all-reduced over tile shards)
+    if (pq) {                                              // q = sum of the devices' partials (rank order)
+        acc = w == 0 ? pq->sum(i) : 0.0;
+    } else if (qin) {                                      // q given (all-reduced over tile shards)
         acc = w == 0 ? __ldcg(&qin[i]) : 0.0;
     } else {
         const double* src = P64 + i;
@@ -728,6 +785,22 @@ fin64_kernel(const double* __restrict__ P64, int nT, int32_t N, const float* __r
     const uint32_t s = t > 0 ? key_index(keys[t - 1]) : 0xFFFFFFFFu;
     fin_unit(blockIdx.x, gridDim.x, sm, SyncCTA{}, P64, nT, N, K, mu, Lc, ldL, tp, h, nv, rdiag, sel, s, t, key_out,
              err, top2, Qc, false, qin, rinit);
+}
+
+// fin64 of the in-library multi-GPU engine: waits for the P partial q of this
+// step (PeerQ), sums them while scoring
+__global__ void __launch_bounds__(kThreads)
+fin64_peer_kernel(PeerQ pq, int nT, int32_t N, const float* __restrict__ K, float mu,
+                  const double* __restrict__ Lc, int64_t ldL, int32_t tp, const double* __restrict__ h,
+                  double* __restrict__ nv, double* __restrict__ rdiag, const uint8_t* __restrict__ sel,
+                  const unsigned long long* __restrict__ keys, int32_t t, unsigned long long* __restrict__ key_out,
+                  int* __restrict__ err, unsigned long long* __restrict__ top2, double* __restrict__ Qc,
+                  const double* __restrict__ rinit) {
+    __shared__ FinSmem sm;
+    wait_peers(pq, err);
+    const uint32_t s = t > 0 ? key_index(keys[t - 1]) : 0xFFFFFFFFu;
+    fin_unit(blockIdx.x, gridDim.x, sm, SyncCTA{}, nullptr, nT, N, K, mu, Lc, ldL, tp, h, nv, rdiag, sel, s, t,
+             key_out, err, top2, Qc, false, nullptr, rinit, &pq);
 }
 
 // ------------------------------------------------------------------ tile-sharded engine (multi-GPU)

@@ -94,3 +94,30 @@ def test_product_path_shares_nothing_with_the_oracle():
                          r"(paper_conf_date_sunbg021_b200|bted)|libbted", src, flags=re.M):
                 bad.append("oracle/" + f)
     assert not bad, bad
+
+
+def test_params_struct_layout_matches_header(tmp_path):
+    """The ctypes mirror of bted_params has the header's field offsets and size
+    (compiled against include/bted.h by gcc)."""
+    fields = [f for f, _ in L.bted_params._fields_]
+    src = tmp_path / "layout.c"
+    src.write_text('#include <stddef.h>\n#include <stdio.h>\n#include "bted.h"\nint main(void){\n'
+                   + "".join(f'printf("{f} %zu\\n", offsetof(bted_params, {f}));\n' for f in fields)
+                   + 'printf("SIZE %zu\\n", sizeof(bted_params)); return 0; }\n')
+    exe = tmp_path / "layout"
+    assert os.system(f"gcc -I{os.path.join(ROOT, 'include')} {src} -o {exe}") == 0
+    out = dict(line.split() for line in os.popen(str(exe)).read().splitlines())
+    for f in fields:
+        assert int(out[f]) == getattr(L.bted_params, f).offset, f
+    assert int(out["SIZE"]) == ctypes.sizeof(L.bted_params)
+    p = L.default_params()
+    assert p.num_devices == 1 and p.norm_mode == 0
+
+
+def test_multi_device_params_validated_before_device():
+    with pytest.raises(bt.BtedError) as e:
+        bt.CandidateSet(np.zeros((4, 2), np.float32), 1.0, norm_mode=2)
+    assert e.value.status == 1
+    with pytest.raises(bt.BtedError) as e:
+        bt.CandidateSet(np.zeros((4, 2), np.float32), 1.0, num_devices=-1)
+    assert e.value.status == 1
