@@ -35,7 +35,13 @@
  * When the caller grants cache_bytes >= 8 N^2 (host RAM permitting), the
  * values k(x_i, x_j) computed in the first pass are kept and re-read by the
  * later passes instead of being recomputed -- the same numbers, so the result
- * is bitwise the same; it only trades memory for the m recomputations.
+ * is bitwise the same; it only trades memory for the m recomputations.  With
+ * between 4 N (N + 1) and 8 N^2 bytes only the upper triangle j >= i is kept
+ * (K is symmetric) and the mat-vec K l runs over it once: row i adds
+ * K_ij l_j (j >= i) in order and scatters K_ij l_i into a per-thread copy of
+ * the result for j > i; the copies are added in thread order (a fixed order
+ * for a fixed thread count; the sums differ from the row order only in
+ * rounding).
  */
 #include <math.h>
 #include <stdint.h>
@@ -84,8 +90,16 @@ int matfree_ted(const float* Xf, int64_t N, int32_t d, double gamma, int32_t lin
                 double* gap_out, double* all_scores, int64_t cache_bytes) {
     if (N < 1 || d < 1 || m < 1 || m > N || !(mu > 0)) return -1;
     double* Kc = NULL;                                             /* optional cache of the N^2 values */
+    double* Ku = NULL;                                             /* or of the upper triangle, row-packed */
+    double* qt = NULL;                                             /* per-thread scatter targets (Ku) */
+    int nthr = matfree_num_threads();
     if (cache_bytes > 0 && (double)N * (double)N * 8.0 <= (double)cache_bytes)
         Kc = (double*)malloc(sizeof(double) * (size_t)N * (size_t)N);
+    else if (cache_bytes > 0 && (double)N * (double)(N + 1) * 4.0 + 8.0 * nthr * N <= (double)cache_bytes) {
+        Ku = (double*)malloc(sizeof(double) * (size_t)N * (size_t)(N + 1) / 2);
+        qt = Ku ? (double*)malloc(sizeof(double) * (size_t)nthr * (size_t)N) : NULL;
+        if (!qt) { free(Ku); Ku = NULL; }
+    }
     double* X = (double*)malloc(sizeof(double) * (size_t)N * d);
     double* L = (double*)calloc((size_t)N * m, sizeof(double));    /* column t at L + t N */
     double* A = (double*)calloc((size_t)N * m, sizeof(double));    /* A = K L, same layout */
@@ -103,9 +117,11 @@ int matfree_ted(const float* Xf, int64_t N, int32_t d, double gamma, int32_t lin
     #pragma omp parallel for schedule(static)
     for (int64_t v = 0; v < N; ++v) {
         double s = 0.0;
+        double* up = Ku ? Ku + (size_t)v * N - (size_t)v * (v - 1) / 2 - (size_t)v : NULL;   /* up[j], j >= v */
         for (int64_t i = 0; i < N; ++i) {
             const double k = kij(X, d, v, i, gamma, linear);
             if (Kc) Kc[(size_t)v * N + i] = k;
+            if (up && i >= v) up[i] = k;
             s += k * k;
         }
         g[v] = s;
@@ -154,22 +170,54 @@ int matfree_ted(const float* Xf, int64_t N, int32_t d, double gamma, int32_t lin
         double* l = L + (size_t)t * N;
         #pragma omp parallel for schedule(static)
         for (int64_t i = 0; i < N; ++i) {
-            double v = Kc ? Kc[(size_t)i * N + s] : kij(X, d, i, s, gamma, linear);
+            double v = Kc ? Kc[(size_t)i * N + s]
+                     : Ku ? Ku[(size_t)(i < s ? i : s) * N - (size_t)(i < s ? i : s) * ((i < s ? i : s) - 1) / 2
+                               - (size_t)(i < s ? i : s) + (size_t)(i < s ? s : i)]
+                          : kij(X, d, i, s, gamma, linear);
             for (int32_t a = 0; a < t; ++a) v -= L[(size_t)a * N + i] * L[(size_t)a * N + s];
             l[i] = v / rt;
         }
         /* A gains K l (rows of K recomputed); C gains L^T l */
         double* Al = A + (size_t)t * N;
-        #pragma omp parallel for schedule(static)
-        for (int64_t i = 0; i < N; ++i) {
-            double acc = 0.0;
-            if (Kc) {
-                const double* row = Kc + (size_t)i * N;
-                for (int64_t j = 0; j < N; ++j) acc += row[j] * l[j];
-            } else {
-                for (int64_t j = 0; j < N; ++j) acc += kij(X, d, i, j, gamma, linear) * l[j];
+        if (Ku) {                                          /* upper triangle: row sums + scattered columns */
+            memset(qt, 0, sizeof(double) * (size_t)nthr * (size_t)N);
+            #pragma omp parallel num_threads(nthr)
+            {
+#ifdef _OPENMP
+                double* q = qt + (size_t)omp_get_thread_num() * N;
+#else
+                double* q = qt;
+#endif
+                #pragma omp for schedule(static, 16)
+                for (int64_t i = 0; i < N; ++i) {
+                    const double* up = Ku + (size_t)i * N - (size_t)i * (i - 1) / 2 - (size_t)i;
+                    const double li = l[i];
+                    double acc = 0.0;
+                    for (int64_t j = i; j < N; ++j) {
+                        acc += up[j] * l[j];
+                        if (j > i) q[j] += up[j] * li;
+                    }
+                    Al[i] = acc;
+                }
             }
-            Al[i] = acc;
+            #pragma omp parallel for schedule(static)
+            for (int64_t i = 0; i < N; ++i) {
+                double a = Al[i];
+                for (int th = 0; th < nthr; ++th) a += qt[(size_t)th * N + i];
+                Al[i] = a;
+            }
+        } else {
+            #pragma omp parallel for schedule(static)
+            for (int64_t i = 0; i < N; ++i) {
+                double acc = 0.0;
+                if (Kc) {
+                    const double* row = Kc + (size_t)i * N;
+                    for (int64_t j = 0; j < N; ++j) acc += row[j] * l[j];
+                } else {
+                    for (int64_t j = 0; j < N; ++j) acc += kij(X, d, i, j, gamma, linear) * l[j];
+                }
+                Al[i] = acc;
+            }
         }
         for (int32_t a = 0; a <= t; ++a) {
             double c = 0.0;
@@ -179,6 +227,6 @@ int matfree_ted(const float* Xf, int64_t N, int32_t d, double gamma, int32_t lin
         }
     }
 done:
-    free(Kc); free(X); free(L); free(A); free(C); free(g); free(kd); free(score); free(sel);
+    free(Kc); free(Ku); free(qt); free(X); free(L); free(A); free(C); free(g); free(kd); free(score); free(sel);
     return rc;
 }

@@ -113,3 +113,20 @@ def test_resnet18_bench_batch_with_near_ties():
         print(f"near-tie resnet18 {name}: K4 refined {st['refined_steps']} (full {st['full_refined_steps']}), "
               f"corrected {st['corrected_steps']}, oracle gaps <= 1e-5: {near} of {m}")
         assert st["refined_steps"] >= m // 2, "K4 did not fire on most steps"
+
+
+@pytest.mark.slow
+def test_large_n131072_tile_sharded_4_devices_full_protocol_o2():
+    """the un-batched TED on N = 131072,
+    tile-sharded over P = 4 devices through the C ABI (num_devices = 4, logical
+    devices on the one GPU: the same kernels and peer exchange), P1 on every
+    pick and P2 at every step against the O2 oracle (upper-triangle cache,
+    68.7 GB of host RAM)."""
+    X, g, cfg = config_pool("large")
+    V = oracle_sample_batches(X.shape[0], cfg["M"], 1, cfg["seed"])[0]
+    Xb = X[V]
+    m = cfg["m"]
+    with bt.CandidateSet(Xb, g, num_devices=4, flags=L.BTED_FLAG_LOOPBACK) as cs:
+        idx, sc = cs.select(m, MU)
+    tr = matfree.ted(Xb, g, MU, m, forced=idx)
+    check_ted(idx, sc, tr, "large-131072-4shards-o2", gap_exact=GAP_K4)

@@ -161,7 +161,7 @@ def test_select_row_bands_over_devices_bit_identical_to_dense(N, P):
     assert np.array_equal(i2, idx) and np.array_equal(s2.view(np.uint32), sc.view(np.uint32))
 
 
-@pytest.mark.parametrize("P", [1, 3])
+@pytest.mark.parametrize("P", [2, 3])
 def test_select_row_bands_literal_column_norms_equal_driver(P):
     """norm_mode = 1: the bands' partial column norms summed (rank order) every
     step -- bitwise dist.ShardedTed's literal mode on the loopback driver, and
@@ -170,7 +170,7 @@ def test_select_row_bands_literal_column_norms_equal_driver(P):
     from paper_conf_date_sunbg021_b200.dist import sharded_select_loopback
     X = knob(3001, seed=3001 + 7 * P)
     g = median_gamma(X, P)
-    num = max(P, 2)                                          # num_devices = 1 would not build the multi-device ctx
+    num = P
     with bt.CandidateSet(X, g, flags=L.BTED_FLAG_DENSE | LOOP, num_devices=num, norm_mode=1) as many:
         idx, sc = many.select(24, MU)
     dev = torch.device("cuda", 0)

@@ -363,3 +363,20 @@ def test_matfree_oracle_cache_is_bitwise_and_forcing_works():
     lit = ted(X, g, MU, 40, forced=forced)
     assert f.idx == forced and f.argmax == lit.argmax
     np.testing.assert_allclose(f.score, lit.score, rtol=5e-11)
+
+
+def test_matfree_upper_triangle_cache_agrees():
+    """O2 with only the upper triangle of K cached (the N = 131072 mode): the
+    mat-vec adds the mirrored half from per-thread copies -- the same numbers up
+    to rounding order: same picks, every score within 1e-10 of the row order."""
+    from oracle import matfree
+    X = knob_X(900, seed=13)
+    g = median_gamma(X, 13)
+    N = X.shape[0]
+    a = matfree.ted(X, g, MU, 48, keep_scores=True, cache_bytes=0)
+    tri = N * (N + 1) * 4 + 8 * matfree.num_threads() * N
+    c = matfree.ted(X, g, MU, 48, keep_scores=True, cache_bytes=tri)
+    assert a.idx == c.idx and a.argmax == c.argmax
+    A, C = np.array(a.scores), np.array(c.scores)
+    fin = np.isfinite(A)
+    assert np.max(np.abs(A[fin] - C[fin]) / np.abs(A[fin])) < 1e-10
