@@ -92,6 +92,10 @@ typedef enum {
                                    run time) instead of the default peer-memory exchange;
                                    NCCL failures and a stalled collective (BTED_NCCL_TIMEOUT_S,
                                    default 300 s; ncclCommGetAsyncError polled) -> BTED_ENCCL */
+#define BTED_FLAG_NO_TC_GRAM 2048u /* implicit engine: build the Gram on CUDA cores (direct-difference
+                                   form) instead of the tensor cores (centred expansion, bf16x3
+                                   tcgen05.mma with the accumulator in TMEM; the default for the
+                                   RBF kernel with d <= 16) */
 #define BTED_FLAG_TIMING   2u   /* record CUDA events around K1 and the K2 loop of every batch
                                    TED on the ctx stream; read with bted_get_stats()          */
 

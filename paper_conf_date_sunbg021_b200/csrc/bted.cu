@@ -11,6 +11,7 @@
 #include <cuda_runtime.h>
 #include <dlfcn.h>
 #include <nccl.h>            // types only: libnccl.so.2 is loaded at run time (BTED_FLAG_NCCL)
+#include <nvtx3/nvToolsExt.h> // header-only NVTX ranges (free unless a profiler attaches)
 
 #include <algorithm>
 #include <atomic>
@@ -37,8 +38,15 @@
 #include "refine.cuh"
 #include "colnorm.cuh"
 #include "xchg.cuh"
+#include "gram_tc.cuh"
 
 namespace {
+
+// NVTX range for timelines (nsys / ncu --nvtx): the BTED call, its phases, K4
+struct Nvtx {
+    explicit Nvtx(const char* name) { nvtxRangePushA(name); }
+    ~Nvtx() { nvtxRangePop(); }
+};
 
 thread_local std::string g_last_error;
 std::atomic<uint64_t> g_launches{0};
@@ -146,6 +154,11 @@ struct Ted {
     int* kflag = nullptr; size_t kflagcap = 0;   // K has a non-positive-normal entry (exact conversion)
     int* bar = nullptr; size_t barcap = 0;       // dependency counters of the persistent loop kernel
     int* tctr = nullptr; size_t tctrcap = 0;     // per-pass tile counters of the K.l passes [m]
+    uint8_t* opA = nullptr; size_t opAcap = 0;   // K1 on tensor cores (gram_tc.cuh): operand blocks,
+    uint8_t* opB = nullptr; size_t opBcap = 0;   //   row norms of the centred features, the centre
+    float* xnrm = nullptr; size_t xnrmcap = 0;
+    float* xctr = nullptr; size_t xctrcap = 0;
+    bool gram_tc = true;                         // implicit head: K1 on tensor cores (else CUDA cores)
     bool split = true;                           // implicit: three kernels per step (else BTED_FLAG_PERSISTENT_LOOP)
     bool implicit = false;
     // K4 near-tie refinement (refine.cuh): per-CTA top-2 keys of every step, flags, candidates
@@ -189,6 +202,8 @@ struct Ted {
         if (err) cudaFree(err);
         if (P) cudaFree(P);
         for (double* q : {P64, Lf, ell, nv, rd, Qc, G, hv}) if (q) cudaFree(q);
+        for (void* q : {(void*)opA, (void*)opB, (void*)xnrm, (void*)xctr}) if (q) cudaFree(q);
+        opA = opB = nullptr; xnrm = xctr = nullptr;
         P64 = Lf = ell = nv = rd = Qc = G = hv = nullptr;
         if (kflag) cudaFree(kflag);
         kflag = nullptr;
@@ -210,7 +225,7 @@ struct Ted {
         const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
         const size_t tiles = (size_t)(ktiles >= 0 ? ktiles : bted::pk::num_tiles(nT)) * bted::pk::T * bted::pk::T;
         const size_t NP = (size_t)nT * bted::pk::T, NPa = (NP + 255) / 256 * 256;
-        const void* before[14] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Qc, G, hv, kflag, bar, tctr};
+        const void* before[18] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Qc, G, hv, kflag, bar, tctr, opA, opB, xnrm, xctr};
         grow(K[0], kcap[0], tiles);
         grow(sel, selcap, NPa);
         grow(keys, keyscap, (size_t)std::max(m, 1));
@@ -222,13 +237,19 @@ struct Ted {
         grow(Qc, qccap, NPa * (size_t)m);
         grow(G, gcap, (size_t)m * (size_t)m);
         grow(hv, hvcap, (size_t)m + 1);
+        if (gram_tc) {
+            grow(opA, opAcap, (size_t)nT * bted::tc::kBlockBytes);
+            grow(opB, opBcap, (size_t)nT * bted::tc::kBlockBytes);
+            grow(xnrm, xnrmcap, NP);
+            grow(xctr, xctrcap, (size_t)bted::tc::kD);
+        }
         grow(kflag, kflagcap, 1);
         grow(bar, barcap, (size_t)bted::im::loop_sync_ints(NPa / bted::im::kEllRows, m));
         grow(tctr, tctrcap, (size_t)std::max(m, 1));
         if (!err) { grow(err, errcap, 1); CK(cudaMemsetAsync(err, 0, sizeof(int), stream)); }
         const void* top2_before = top2;
         reserve_refine((int64_t)NP, m);
-        const void* after[14] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Qc, G, hv, kflag, bar, tctr};
+        const void* after[18] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Qc, G, hv, kflag, bar, tctr, opA, opB, xnrm, xctr};
         if (top2 != top2_before) { for (auto& g : graphs) cudaGraphExecDestroy(g.second); graphs.clear(); }
         if (std::memcmp(before, after, sizeof before) != 0) {
             for (auto& g : graphs) cudaGraphExecDestroy(g.second);
@@ -448,6 +469,14 @@ void ensure_implicit_attrs() {
     });
 }
 
+void ensure_gram_tc_attrs() {
+    static uint64_t done = 0;
+    once_per_device(done, [] {
+        CK(cudaFuncSetAttribute(bted::tc::gram_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)bted::tc::kSmemBytes));
+    });
+}
+
 void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m,
                            float mu, unsigned long long* keys) {
     const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
@@ -462,9 +491,19 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
     auto k1i = [&](auto kern) {
         kern<<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(X, (int32_t)N, d, gamma, T.K[0], nT, 0, 1);
     };
-    // d <= 16: two columns per lane, four rows at once, 4 CTAs/SM: 243 us at N = 16384 (B200,
-    // warm ncu) vs 371 us for gram_tile_kernel<16,·,2> and 412 us for K1p
-    if (d <= 16) {
+    // d <= 16 (RBF): the tensor-core Gram (gram_tc.cuh: centred expansion, bf16x3 tcgen05.mma,
+    // TMEM accumulator); else / BTED_FLAG_NO_TC_GRAM: the CUDA-core direct form -- two columns
+    // per lane, four rows at once, 4 CTAs/SM: 243 us at N = 16384 (B200, warm ncu)
+    if (d <= 16 && !lin && T.gram_tc) {
+        ensure_gram_tc_attrs();
+        bted::tc::center_kernel<<<1, bted::tc::kThreads, 0, T.stream>>>(X, (int32_t)N, d, T.xctr);
+        bted::tc::prep_kernel<<<(unsigned)((NP + bted::tc::kThreads - 1) / bted::tc::kThreads), bted::tc::kThreads, 0,
+                                T.stream>>>(X, (int32_t)N, d, nT, T.xctr, T.opA, T.opB, T.xnrm);
+        const unsigned g = (unsigned)std::min<int64_t>(tiles, (int64_t)3 * num_sms());
+        bted::tc::gram_tc_kernel<<<g, bted::tc::kThreads, bted::tc::kSmemBytes, T.stream>>>(
+            T.opA, T.opB, T.xnrm, (int32_t)N, gamma, T.K[0], nT);
+        LAUNCHED(2);
+    } else if (d <= 16) {
         if (lin) k1i(bted::pk::gram_tile2_kernel<16, true, 4>); else k1i(bted::pk::gram_tile2_kernel<16, false, 4>);
     } else {
         if (lin) k1i(bted::pk::gram_tile_kernel<32, true>); else k1i(bted::pk::gram_tile_kernel<32, false>);
@@ -962,6 +1001,7 @@ bted_status create_common(const float* X, int64_t N, int32_t d, bted_kernel kern
         ctx->ted.implicit = ctx->bted_engine.implicit = (params->flags & BTED_FLAG_LITERAL) == 0;
         ctx->ted.refine = ctx->bted_engine.refine = (params->flags & BTED_FLAG_NO_REFINE) == 0;
         ctx->ted.split = ctx->bted_engine.split = (params->flags & BTED_FLAG_PERSISTENT_LOOP) == 0;
+        ctx->ted.gram_tc = ctx->bted_engine.gram_tc = (params->flags & BTED_FLAG_NO_TC_GRAM) == 0;
         CK(cudaMallocHost(&ctx->herr, sizeof(int)));
         if (params->x_on_device) {
             ctx->X = const_cast<float*>(X);
@@ -1008,6 +1048,7 @@ int bits_for(uint64_t maxval) {
 // out[k][0..M) = sorted V_{b_begin + k b_step}, by radix select (sample.cuh).
 void sample_batches_dev(bted_ctx* ctx, cudaStream_t st, int64_t P, int64_t M, int32_t b_begin, int32_t b_step,
                         int nb, uint64_t seed, uint32_t* out) {
+    Nvtx nvtx_("bted sample (Alg. 2 l.2)");
     grow(ctx->shist, ctx->shistcap, (size_t)2 * nb * bted::kSelBins);
     grow(ctx->sint, ctx->sintcap, (size_t)5 * nb + 1);
     grow(ctx->scand, ctx->scandcap, (size_t)nb * bted::kCandCap);
@@ -1196,6 +1237,7 @@ bool k4_next_correction(bted_ctx* ctx, cudaStream_t st, const float* X, int64_t 
 
 void refine_ted(bted_ctx* ctx, Ted& T, const float* X, int64_t N, int32_t d, int32_t m, float mu,
                 unsigned long long* keys, float* scores_out) {
+    Nvtx nvtx_("bted K4 refine");
     cudaStream_t st = T.stream;
     std::vector<unsigned long long> hk(m), forced;
     std::vector<int> fl(m), nc(m);
@@ -1374,6 +1416,7 @@ bool small_k4_refine(bted_ctx* ctx, cudaStream_t st, const float* X, int ninst, 
 
 // Alg. 2 l.1-4 for batches b_begin, b_begin+b_step, ... ; winners on device.
 int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_begin, int32_t b_step) {
+    Nvtx nvtx_("bted batch TEDs (Alg. 2 l.1-4)");
     const int32_t B = ctx->params.num_batches;
     ctx->k4b.pending = false;
     int nb = 0;
@@ -1494,6 +1537,7 @@ bted_status batch_range_finish(bted_ctx* ctx, int nb) {
 // Alg. 2 l.5-6 on device winners[0..n): returns count, out_idx host [count].
 bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, int32_t m, float mu,
                          int64_t* out_idx, int32_t* out_count) {
+    Nvtx nvtx_("bted union + merge (Alg. 2 l.5-6)");
     cudaStream_t st = ctx->stream;
     grow(ctx->u32a, ctx->u32acap, (size_t)n);
     grow(ctx->u32b, ctx->u32bcap, (size_t)n);
@@ -2090,6 +2134,7 @@ void md_select_loop(bted_ctx* ctx, int32_t m, float mu, const std::vector<unsign
 bted_status md_select_bands(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, float* out_score);
 
 bted_status md_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, float* out_score) {
+    Nvtx nvtx_("bted multi-GPU select");
     MultiDev& md = *ctx->md;
     const int P = md.P;
     if (ctx->d > 32) { set_error("multi-GPU select needs d <= 32"); return BTED_EINVAL; }
@@ -2360,6 +2405,7 @@ bted_status md_select_bands(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx
 // batches (replica ctx; device 0 = this ctx), then the merge on device 0.
 bted_status md_run_batches(bted_ctx* ctx, int64_t M, int32_t m, float mu, int64_t* out_idx, int32_t* out_count,
                            int64_t* out_batch_idx) {
+    Nvtx nvtx_("bted multi-GPU run_batches");
     MultiDev& md = *ctx->md;
     const int G = md.P, B = ctx->params.num_batches;
     if (md.rep.empty()) {
@@ -2439,6 +2485,7 @@ bted_status bted_shard_create(const float* X, int64_t N, int32_t d, bted_kernel 
 }
 
 bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, float* out_score) {
+    Nvtx nvtx_("bted_select (Alg. 1)");
     if (!ctx || !out_idx) { set_error("null argument"); return BTED_EINVAL; }
     if (ctx->is_shard || ctx->is_ishard) { set_error("bted_select on a shard context"); return BTED_EINVAL; }
     if (m < 1 || m > ctx->N || !mu_ok(mu)) { set_error("need 1 <= m <= N and mu > 0 finite"); return BTED_EINVAL; }
@@ -2525,6 +2572,7 @@ bted_status bted_merge(bted_ctx* ctx, const int64_t* winners, int64_t n, int32_t
 
 bted_status bted_run_batches(bted_ctx* ctx, int64_t M, int32_t m, float mu, int64_t* out_idx, int32_t* out_count,
                              int64_t* out_batch_idx) {
+    Nvtx nvtx_("bted_run_batches (Alg. 2)");
     if (!ctx || !out_idx || !out_count) { set_error("null argument"); return BTED_EINVAL; }
     if (ctx->is_shard || ctx->is_ishard) { set_error("run_batches on a shard context"); return BTED_EINVAL; }
     if (m < 1 || M < m || M > ctx->N || !mu_ok(mu)) { set_error("need 1 <= m <= M <= N and mu > 0"); return BTED_EINVAL; }

@@ -44,10 +44,12 @@ def ld_of(N):
 # ------------------------------------------------------------------ K1 Gram
 @pytest.mark.parametrize("N,d,pool", [(1000, 16, "knob"), (777, 16, "uniform"), (300, 12, "knob"), (515, 30, "uniform")])
 def test_implicit_gram_bitwise_equals_k1p(N, d, pool):
-    """K1i (the implicit head's Gram-only kernel) writes bitwise the tiles K1p writes."""
+    """K1i on CUDA cores (the implicit head's Gram-only kernel, BTED_FLAG_NO_TC_GRAM) writes
+    bitwise the tiles K1p writes."""
     X = knob(N, d=d) if pool == "knob" else uniform_pool(N, d, 4)
     g = median_gamma(X, 2)
-    with bt.CandidateSet(X, g, flags=IMPLICIT) as ci, bt.CandidateSet(X, g, flags=PACKED) as cp:
+    with bt.CandidateSet(X, g, flags=IMPLICIT | L.BTED_FLAG_NO_TC_GRAM) as ci, \
+            bt.CandidateSet(X, g, flags=PACKED) as cp:
         ci.select(5, MU)
         cp.select(1, MU)
         assert np.array_equal(ci.debug_K(N), cp.debug_K(N))
@@ -77,6 +79,34 @@ def test_gram_entries_bitsymmetric_and_within_ulp_bound(N, pool, flags):
     # first pick = argmax of fp64 first scores (C1 + l.3)
     s64 = (K64 * K64).sum(0) / (1.0 + MU)
     assert abs(float(sc[0]) - s64[idx[0]]) <= 1e-5 * s64[idx[0]]
+
+
+@pytest.mark.parametrize("N,d,pool", [(1000, 16, "knob"), (777, 16, "uniform"), (300, 12, "knob"),
+                                      (4099, 16, "knob"), (129, 8, "uniform"), (2000, 16, "knob-dups")])
+def test_tensor_core_gram_c1_bound(N, d, pool):
+    """K1 on the tensor cores (gram_tc.cuh: centred expansion, bf16x3 tcgen05.mma):
+    every entry within pin C1's 6 ulp * (1 + gamma d^2) of fp64, bit-symmetric,
+    K_ii = 1, zero padding, exact duplicates give bitwise-equal rows."""
+    if pool == "knob-dups":
+        X = knob(N // 2, seed=8)
+        X = np.concatenate([X, X], axis=0)
+    else:
+        X = knob(N, d=d) if pool == "knob" else uniform_pool(N, d, 4)
+    g = median_gamma(X, 2)
+    with bt.CandidateSet(X, g, flags=IMPLICIT) as cs:
+        cs.select(2, MU)
+        K = cs.debug_K(N)
+    K32 = K[:, :N].astype(np.float64)
+    assert np.all(K[:, N:] == 0.0)
+    assert np.array_equal(K[:, :N], K[:, :N].T)
+    assert np.all(np.diag(K) == 1.0)
+    d2 = cdist(X.astype(np.float64), X.astype(np.float64), "sqeuclidean")
+    K64 = np.exp(-float(g) * d2)
+    ratio = np.abs(K32 - K64) / (ulp32(K64) * (1.0 + float(g) * d2))
+    print(f"TC Gram N={N} d={d} {pool}: max {ratio.max():.2f} ulp*(1+g d2)")
+    assert ratio.max() <= 6.0
+    if pool == "knob-dups":
+        assert np.array_equal(K[: N // 2, :N], K[N // 2:, :N][:, np.r_[N // 2:N, 0:N // 2]])
 
 
 # ------------------------------------------------------------------ K2 step
