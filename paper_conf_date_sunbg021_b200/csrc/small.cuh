@@ -115,6 +115,9 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
     }
     for (int q = tid; q < R; q += kThreads) sel[q] = 0;
     __syncthreads();
+    // every CTA of the cluster has started (its shared memory exists) before the
+    // first remote (DSMEM) write of the key exchange
+    if constexpr (C > 1) cl.sync();
     // K4 (top2_all non-null): every warp records its best two keys of each step,
     // top2[inst][t][rank * kWarps + w][0..1] -- the input of the near-tie check
     const int nU = C * kWarps;
@@ -163,6 +166,7 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
         float g[kR];
 #pragma unroll
         for (int h = 0; h < kR; ++h) g[h] = warp_sum(acc_norm[h]);
+        __syncwarp();                                      // the diagonal entry was written by another lane
         if (l == 0) {
 #pragma unroll
             for (int h = 0; h < kR; ++h) {
@@ -258,6 +262,7 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
                 }
             }
             const float gl = warp_sum4(acc_norm, l);  // row l / 8 of the group (kLanePerRow)
+            __syncwarp();                            // the diagonal entry was written by another lane
             if ((l & (kLanePerRow - 1)) == 0) {      // lane 8h scores row h of the group
                 const int lr = base + (l / kLanePerRow) * kWarps;
                 if (lr < nr) {
