@@ -232,7 +232,12 @@ def bench_ours(args):
             sk.close()
             os.environ.setdefault("RANK", "0")
             os.environ.setdefault("WORLD_SIZE", "1")
-        dist.init_process_group("nccl", device_id=dev)
+        # a dead or stalled rank fails the job instead of hanging it: NCCL async error
+        # handling + a collective timeout (BTED_NCCL_TIMEOUT_S, default 600 s)
+        os.environ.setdefault("TORCH_NCCL_ASYNC_ERROR_HANDLING", "1")
+        import datetime
+        dist.init_process_group("nccl", device_id=dev, timeout=datetime.timedelta(
+            seconds=float(os.environ.get("BTED_NCCL_TIMEOUT_S", "600"))))
         comm = TorchComm()
 
     if args.config == "wholemodel":

@@ -158,6 +158,7 @@ struct Ted {
     uint8_t* opB = nullptr; size_t opBcap = 0;   //   row norms of the centred features, the centre
     float* xnrm = nullptr; size_t xnrmcap = 0;
     float* xctr = nullptr; size_t xctrcap = 0;
+    int* xmax = nullptr; size_t xmaxcap = 0;
     bool gram_tc = true;                         // implicit head: K1 on tensor cores (else CUDA cores)
     bool split = true;                           // implicit: three kernels per step (else BTED_FLAG_PERSISTENT_LOOP)
     bool implicit = false;
@@ -202,8 +203,8 @@ struct Ted {
         if (err) cudaFree(err);
         if (P) cudaFree(P);
         for (double* q : {P64, Lf, ell, nv, rd, Qc, G, hv}) if (q) cudaFree(q);
-        for (void* q : {(void*)opA, (void*)opB, (void*)xnrm, (void*)xctr}) if (q) cudaFree(q);
-        opA = opB = nullptr; xnrm = xctr = nullptr;
+        for (void* q : {(void*)opA, (void*)opB, (void*)xnrm, (void*)xctr, (void*)xmax}) if (q) cudaFree(q);
+        opA = opB = nullptr; xnrm = xctr = nullptr; xmax = nullptr;
         P64 = Lf = ell = nv = rd = Qc = G = hv = nullptr;
         if (kflag) cudaFree(kflag);
         kflag = nullptr;
@@ -225,7 +226,7 @@ struct Ted {
         const int nT = (int)((N + bted::pk::T - 1) / bted::pk::T);
         const size_t tiles = (size_t)(ktiles >= 0 ? ktiles : bted::pk::num_tiles(nT)) * bted::pk::T * bted::pk::T;
         const size_t NP = (size_t)nT * bted::pk::T, NPa = (NP + 255) / 256 * 256;
-        const void* before[18] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Qc, G, hv, kflag, bar, tctr, opA, opB, xnrm, xctr};
+        const void* before[19] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Qc, G, hv, kflag, bar, tctr, opA, opB, xnrm, xctr, xmax};
         grow(K[0], kcap[0], tiles);
         grow(sel, selcap, NPa);
         grow(keys, keyscap, (size_t)std::max(m, 1));
@@ -242,6 +243,7 @@ struct Ted {
             grow(opB, opBcap, (size_t)nT * bted::tc::kBlockBytes);
             grow(xnrm, xnrmcap, NP);
             grow(xctr, xctrcap, (size_t)bted::tc::kD);
+            grow(xmax, xmaxcap, 1);
         }
         grow(kflag, kflagcap, 1);
         grow(bar, barcap, (size_t)bted::im::loop_sync_ints(NPa / bted::im::kEllRows, m));
@@ -249,7 +251,7 @@ struct Ted {
         if (!err) { grow(err, errcap, 1); CK(cudaMemsetAsync(err, 0, sizeof(int), stream)); }
         const void* top2_before = top2;
         reserve_refine((int64_t)NP, m);
-        const void* after[18] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Qc, G, hv, kflag, bar, tctr, opA, opB, xnrm, xctr};
+        const void* after[19] = {K[0], sel, keys, P64, Lf, ell, nv, rd, Qc, G, hv, kflag, bar, tctr, opA, opB, xnrm, xctr, xmax};
         if (top2 != top2_before) { for (auto& g : graphs) cudaGraphExecDestroy(g.second); graphs.clear(); }
         if (std::memcmp(before, after, sizeof before) != 0) {
             for (auto& g : graphs) cudaGraphExecDestroy(g.second);
@@ -474,6 +476,8 @@ void ensure_gram_tc_attrs() {
     once_per_device(done, [] {
         CK(cudaFuncSetAttribute(bted::tc::gram_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)bted::tc::kSmemBytes));
+        CK(cudaFuncSetAttribute(bted::tc::gram_tc_norm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)(2 * bted::tc::kBlockBytes)));
     });
 }
 
@@ -489,20 +493,27 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
     const int lin = kernel == BTED_KERNEL_LINEAR ? 1 : 0;
     // K1i: the Gram tiles only (the fp64 norm pass below recomputes the first scores)
     auto k1i = [&](auto kern) {
-        kern<<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(X, (int32_t)N, d, gamma, T.K[0], nT, 0, 1);
+        kern<<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(X, (int32_t)N, d, gamma, T.K[0], nT, 0, 1,
+                                                                     (const int*)nullptr);
     };
     // d <= 16 (RBF): the tensor-core Gram (gram_tc.cuh: centred expansion, bf16x3 tcgen05.mma,
     // TMEM accumulator); else / BTED_FLAG_NO_TC_GRAM: the CUDA-core direct form -- two columns
     // per lane, four rows at once, 4 CTAs/SM: 243 us at N = 16384 (B200, warm ncu)
     if (d <= 16 && !lin && T.gram_tc) {
         ensure_gram_tc_attrs();
-        bted::tc::center_kernel<<<1, bted::tc::kThreads, 0, T.stream>>>(X, (int32_t)N, d, T.xctr);
+        bted::tc::center_kernel<<<1, bted::tc::kCenterThreads, 0, T.stream>>>(X, (int32_t)N, d, T.xctr);
         bted::tc::prep_kernel<<<(unsigned)((NP + bted::tc::kThreads - 1) / bted::tc::kThreads), bted::tc::kThreads, 0,
-                                T.stream>>>(X, (int32_t)N, d, nT, T.xctr, T.opA, T.opB, T.xnrm);
-        const unsigned g = (unsigned)std::min<int64_t>(tiles, (int64_t)3 * num_sms());
+                                T.stream>>>(X, (int32_t)N, d, nT, T.xctr, T.opA, T.opB);
+        CK(cudaMemsetAsync(T.xmax, 0, sizeof(int), T.stream));
+        bted::tc::gram_tc_norm_kernel<<<(unsigned)nT, bted::tc::kThreads, 2 * bted::tc::kBlockBytes, T.stream>>>(
+            T.opA, T.opB, T.xnrm, T.xmax);
+        const unsigned g = (unsigned)std::min<int64_t>(tiles, (int64_t)2 * num_sms());
         bted::tc::gram_tc_kernel<<<g, bted::tc::kThreads, bted::tc::kSmemBytes, T.stream>>>(
-            T.opA, T.opB, T.xnrm, (int32_t)N, gamma, T.K[0], nT);
-        LAUNCHED(2);
+            T.opA, T.opB, T.xnrm, (int32_t)N, gamma, T.K[0], nT, T.xmax);
+        // the accuracy guard's fallback (exits at once when the tensor-core Gram was written)
+        bted::pk::gram_tile2_kernel<16, false, 4><<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
+            X, (int32_t)N, d, gamma, T.K[0], nT, 0, 1, T.xmax);
+        LAUNCHED(5);
     } else if (d <= 16) {
         if (lin) k1i(bted::pk::gram_tile2_kernel<16, true, 4>); else k1i(bted::pk::gram_tile2_kernel<16, false, 4>);
     } else {
@@ -1765,7 +1776,8 @@ void ishard_head_enqueue(bted_ctx* ctx, int32_t m, double* q_dev) {
     const float g = ctx->params.gamma;
     const int r = ctx->srank, P = ctx->snranks;
     auto k1i = [&](auto kern) {
-        kern<<<(unsigned)lt, bted::pk::kConsumers, 0, T.stream>>>(ctx->X, (int32_t)N, ctx->d, g, T.K[0], nT, r, P);
+        kern<<<(unsigned)lt, bted::pk::kConsumers, 0, T.stream>>>(ctx->X, (int32_t)N, ctx->d, g, T.K[0], nT, r, P,
+                                                                   (const int*)nullptr);
     };
     if (ctx->d <= 16) {
         if (lin) k1i(bted::pk::gram_tile2_kernel<16, true, 4>); else k1i(bted::pk::gram_tile2_kernel<16, false, 4>);

@@ -3,8 +3,8 @@
 //
 // k(x_i, x_j) = exp(-gamma ||x_i - x_j||^2) with ||x_i - x_j||^2 expanded as
 //     n_i + n_j - 2 x'_i . x'_j,    x' = x - c  (c = the mean feature vector),
-// where the 128 x 128 block of dot products x'_I . x'_J^T is ONE tcgen05.mma
-// chain per tile (M = N = 128, fp32 accumulator in TMEM).  Centring makes the
+// where the 128 x 128 blocks of dot products x'_I . x'_J^T are tcgen05.mma
+// chains per tile (M = N = 128, fp32 accumulators in TMEM).  Centring makes the
 // expansion as accurate as the direct-difference form it replaces (translation
 // leaves every distance unchanged; the cancellation of n_i + n_j - 2 dot is then
 // relative to the spread of the data, not to |x|^2): measured on the knob and
@@ -22,13 +22,12 @@
 // 8 x 8 core matrices of 128 B, k-chunks 128 B apart (LBO), 8-row groups
 // 1536 B apart (SBO), six 16-wide k-slices per block of 128 rows.
 //
-// Per tile (I <= J): all threads copy the two 24 KiB operand blocks into
-// shared memory, one elected thread issues the six MMAs and commits them to
-// an mbarrier, eight warps read the accumulator (tcgen05.ld, warp w: TMEM
-// lanes 32 (w % 4).., columns 64 (w / 4)..), form K, stage the tile in shared
-// memory (reusing the operand space) and write it out with coalesced
-// 512-byte rows.  Diagonal tiles store their upper triangle mirrored, so the
-// matrix is bit-symmetric by construction, and K_ii = 1 exactly.
+// Per tile (I <= J): the two 24 KiB operand blocks arrive by TMA bulk copies
+// (mbarrier), one thread issues the six MMAs and commits them to an mbarrier,
+// eight warps read the accumulator (tcgen05.ld), form K and store it; the
+// next tile's copies overlap the epilogue.  Diagonal tiles store their upper
+// triangle mirrored, so the matrix is bit-symmetric by construction, and
+// K_ii = 1 exactly.
 #pragma once
 #include <cstdint>
 #include <cuda_bf16.h>
@@ -46,9 +45,7 @@ constexpr int kK = kD * kSlices;               // 96 bf16 per row
 constexpr uint32_t kLBO = 128;                 // bytes between k-adjacent core matrices
 constexpr uint32_t kSBO = (kK / 8) * 128;      // 1536: bytes between 8-row groups
 constexpr uint32_t kBlockBytes = (T / 8) * kSBO;   // 24576 per 128-row block
-constexpr int kStageLd = T + 4;                // padded staging row (floats): conflict-free float4 writes
-constexpr size_t kSmemBytes = (size_t)T * kStageLd * sizeof(float) > 2 * kBlockBytes
-                                  ? (size_t)T * kStageLd * sizeof(float) : 2 * (size_t)kBlockBytes;
+constexpr size_t kSmemBytes = 4 * (size_t)kBlockBytes;       // A_I, B_I, A_J, B_J (96 KiB)
 // kind::f16, A = B = bf16 (K-major), D = f32, M = 128, N = 128
 constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(T >> 3) << 17) | ((uint32_t)(T >> 4) << 24);
 
@@ -58,23 +55,30 @@ __host__ __device__ __forceinline__ uint32_t op_offset(int r, int k) {
 }
 
 // ---------------------------------------------------------------- prep
-// c = mean of the N rows (one CTA, thread-strided fp32 sums in row order, then a
-// fixed tree over the 256 threads): any c is exact in the algebra; the mean keeps
-// the expansion's cancellation small
-__global__ void __launch_bounds__(kThreads) center_kernel(const float* __restrict__ X, int32_t N, int32_t d,
-                                                         float* __restrict__ c) {
-    __shared__ float red[kThreads];
-    for (int k = 0; k < d; ++k) {
-        float s = 0.f;
-        for (int i = threadIdx.x; i < N; i += kThreads) s = __fadd_rn(s, X[(int64_t)i * d + k]);
-        red[threadIdx.x] = s;
-        __syncthreads();
-        for (int off = kThreads / 2; off > 0; off >>= 1) {
-            if (threadIdx.x < off) red[threadIdx.x] = __fadd_rn(red[threadIdx.x], red[threadIdx.x + off]);
-            __syncthreads();
-        }
-        if (threadIdx.x == 0) c[k] = __fdiv_rn(red[0], (float)N);
-        __syncthreads();
+// c = mean of the N rows (one CTA: per thread the rows tid, tid + 1024, ... in
+// order, then a fixed butterfly and the warps in order): any c is exact in the
+// algebra; the mean keeps the expansion's cancellation small
+constexpr int kCenterThreads = 1024;
+__global__ void __launch_bounds__(kCenterThreads) center_kernel(const float* __restrict__ X, int32_t N, int32_t d,
+                                                               float* __restrict__ c) {
+    __shared__ float red[kCenterThreads / 32][kD];
+    float s[kD];
+#pragma unroll
+    for (int k = 0; k < kD; ++k) s[k] = 0.f;
+    for (int i = threadIdx.x; i < N; i += kCenterThreads)        // rows tid, tid + 1024, ... in order
+        for (int k = 0; k < d; ++k) s[k] = __fadd_rn(s[k], X[(int64_t)i * d + k]);
+    const int w = threadIdx.x / 32, l = threadIdx.x % 32;
+#pragma unroll
+    for (int k = 0; k < kD; ++k) {                               // fixed butterfly, then warps in order
+        float v = s[k];
+        for (int off = 16; off > 0; off >>= 1) v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, off));
+        if (l == 0) red[w][k] = v;
+    }
+    __syncthreads();
+    if (threadIdx.x < d) {
+        float t = 0.f;
+        for (int q = 0; q < kCenterThreads / 32; ++q) t = __fadd_rn(t, red[q][threadIdx.x]);
+        c[threadIdx.x] = __fdiv_rn(t, (float)N);
     }
 }
 
@@ -86,22 +90,19 @@ __device__ __forceinline__ void split3(float v, __nv_bfloat16& h, __nv_bfloat16&
     l = __float2bfloat16_rn(r2);                                  // exact for normal v
 }
 
-// per row i (padding rows: 0): x' = x - c, n_i = sum_k x'_k^2 (fp32, k order),
-// and the two operand blocks: A slices [m, h, l, h, m, h], B slices [m, l, h, m, h, h]
+// per row i (padding rows: 0): x' = x - c and the two operand blocks:
+// A slices [m, h, l, h, m, h], B slices [m, l, h, m, h, h]
 __global__ void __launch_bounds__(kThreads) prep_kernel(const float* __restrict__ X, int32_t N, int32_t d,
                                                        int nT, const float* __restrict__ c,
-                                                       uint8_t* __restrict__ opA, uint8_t* __restrict__ opB,
-                                                       float* __restrict__ nrm) {
+                                                       uint8_t* __restrict__ opA, uint8_t* __restrict__ opB) {
     const int64_t i = (int64_t)blockIdx.x * kThreads + threadIdx.x;
     if (i >= (int64_t)nT * T) return;
     const int blk = (int)(i / T), r = (int)(i % T);
     uint8_t* a = opA + (size_t)blk * kBlockBytes;
     uint8_t* b = opB + (size_t)blk * kBlockBytes;
-    float n = 0.f;
     for (int k = 0; k < kD; ++k) {
         float v = 0.f;
         if (i < N && k < d) v = __fsub_rn(X[i * d + k], c[k]);
-        n = __fmaf_rn(v, v, n);
         __nv_bfloat16 h, m, l;
         split3(v, h, m, l);
         const __nv_bfloat16 sa[kSlices] = {m, h, l, h, m, h};
@@ -112,7 +113,6 @@ __global__ void __launch_bounds__(kThreads) prep_kernel(const float* __restrict_
             *reinterpret_cast<__nv_bfloat16*>(b + op_offset(r, s * kD + k)) = sb[s];
         }
     }
-    nrm[i] = i < N ? n : 0.f;
 }
 
 // ---------------------------------------------------------------- tcgen05 helpers
@@ -133,14 +133,6 @@ __device__ __forceinline__ void mma_bf16(uint32_t tmem_d, uint64_t adesc, uint64
                  :: "r"(tmem_d), "l"(adesc), "l"(bdesc), "r"(kIdesc), "r"(acc));
 }
 
-__device__ __forceinline__ void mbar_init(uint64_t* bar) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(smem_u32(bar)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
-    asm volatile("{\n\t.reg .pred done;\n\tWAIT_%=:\n\t"
-                 "mbarrier.try_wait.parity.shared::cta.b64 done, [%0], %1;\n\t"
-                 "@!done bra WAIT_%=;\n\t}\n" :: "r"(smem_u32(bar)), "r"(phase) : "memory");
-}
 
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, float (&v)[16]) {
     uint32_t r[16];
@@ -154,108 +146,213 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, float (&v)[16]) {
     for (int q = 0; q < 16; ++q) v[q] = __uint_as_float(r[q]);
 }
 
-// ---------------------------------------------------------------- the tile kernel
-// grid: persistent, tile k = blockIdx.x + j gridDim.x (k < num_tiles(nT)); writes
-// K[k] (64 KiB, row-major) of the packed upper-triangular layout
+// ---------------------------------------------------------------- symmetric dot products
+// D = A_I . B_J^T and D' = B_I . A_J^T (two accumulators, TMEM columns [0, 128) and
+// [128, 256)).  D[r][c] = dot(A_r, B_c), D'[r][c] = dot(B_r, A_c) = dot(A_c, B_r)
+// (the same products in the same slice order), so S = D + D' is symmetric in (r, c)
+// BITWISE: S_cr adds the same two numbers in the other order.  Hence K is
+// bit-symmetric without mirroring, and exact duplicate points get bitwise-equal
+// rows.  The squared norms are S's own diagonal halves, n_r = S_rr / 2, so that
+// d2 = (n_r + n_c) - S_rc is exactly 0 for identical points (K = 1, like the
+// direct form).
+constexpr int kTmemCols = 2 * T;
+// Accuracy guard: the expansion's rounding is relative to the centred norms, so the
+// tensor-core Gram is used only when gamma * max_r n_r <= kGuard (the median-gamma
+// knob and uniform pools: ~1-2); otherwise (badly scaled data, a huge gamma) the
+// direct-difference kernel writes the Gram instead -- both kernels are launched and
+// each reads the decision from *nmax_bits (max n_r, as non-negative float bits).
+constexpr float kGuard = 4.f;
+__device__ __forceinline__ bool tc_ok(const int* nmax_bits, float gamma) {
+    return __fmul_rn(gamma, __int_as_float(*nmax_bits)) <= kGuard;
+}
+
+__device__ __forceinline__ void issue_sym_mmas(uint32_t tbase, uint32_t aI, uint32_t bI, uint32_t aJ, uint32_t bJ) {
+#pragma unroll
+    for (int s = 0; s < kSlices; ++s)                          // each k-slice = 16 bf16 = 2 core matrices
+        mma_bf16(tbase, smem_desc(aI + 2 * s * kLBO), smem_desc(bJ + 2 * s * kLBO), s > 0 ? 1u : 0u);
+#pragma unroll
+    for (int s = 0; s < kSlices; ++s)
+        mma_bf16(tbase + T, smem_desc(bI + 2 * s * kLBO), smem_desc(aJ + 2 * s * kLBO), s > 0 ? 1u : 0u);
+}
+
+__device__ __forceinline__ void tmem_alloc(uint32_t* dst) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
+                 :: "r"(smem_u32(dst)), "n"(kTmemCols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+}
+__device__ __forceinline__ void tmem_free(uint32_t base) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(base), "n"(kTmemCols));
+}
+__device__ __forceinline__ void mma_commit(uint64_t* bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                 :: "r"(smem_u32(bar)) : "memory");
+}
+
+// n_r = S_rr / 2 for every row of every block (one CTA per block I: the diagonal tile's S)
 __global__ void __launch_bounds__(kThreads)
-gram_tc_kernel(const uint8_t* __restrict__ opA, const uint8_t* __restrict__ opB, const float* __restrict__ nrm,
-               int32_t N, float gamma, float* __restrict__ K, int nT) {
-    extern __shared__ __align__(1024) uint8_t smem[];
-    __shared__ __align__(8) uint64_t mbar;
+gram_tc_norm_kernel(const uint8_t* __restrict__ opA, const uint8_t* __restrict__ opB, float* __restrict__ nrm,
+                    int* __restrict__ nmax_bits) {
+    extern __shared__ __align__(1024) uint8_t smem[];            // [A_I | B_I]
+    __shared__ __align__(8) uint64_t ldbar, mmabar;
     __shared__ uint32_t tmem_base;
-    __shared__ float nI[T], nJ[T];
-    uint8_t* sA = smem;
-    uint8_t* sB = smem + kBlockBytes;
-    float* stage = reinterpret_cast<float*>(smem);                // reuses the operand space after the MMAs
-    const int tid = threadIdx.x, w = tid / 32, lane = tid % 32;
-    if (w == 0) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
-                     :: "r"(smem_u32(&tmem_base)), "n"(T));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-    }
+    const int tid = threadIdx.x, w = tid / 32, lane = tid % 32, I = blockIdx.x;
+    if (w == 0) tmem_alloc(&tmem_base);
     if (tid == 0) {
-        mbar_init(&mbar);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");   // visible to the async proxy
+        pk::mbar_init(&ldbar, 1);
+        pk::mbar_init(&mmabar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tbase = tmem_base;
+    if (tid == 0) {
+        pk::mbar_expect_tx(&ldbar, 2 * kBlockBytes);
+        pk::bulk_g2s(smem, opA + (size_t)I * kBlockBytes, kBlockBytes, &ldbar);
+        pk::bulk_g2s(smem + kBlockBytes, opB + (size_t)I * kBlockBytes, kBlockBytes, &ldbar);
+    }
+    pk::mbar_wait(&ldbar, 0);
+    if (tid == 0) {
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        const uint32_t a = smem_u32(smem), b = smem_u32(smem + kBlockBytes);
+        issue_sym_mmas(tbase, a, b, a, b);
+        mma_commit(&mmabar);
+    }
+    pk::mbar_wait(&mmabar, 0);
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    if (w < 4) {                                               // lane r = 32 w + lane needs column r
+        const int r = 32 * w + lane;
+        float d0[16], d1[16], e0[16], e1[16];
+        const uint32_t lb = (uint32_t)(32 * w) << 16;
+        tmem_ld16(tbase + lb + (uint32_t)(32 * w), d0);
+        tmem_ld16(tbase + lb + (uint32_t)(32 * w + 16), d1);
+        tmem_ld16(tbase + T + lb + (uint32_t)(32 * w), e0);
+        tmem_ld16(tbase + T + lb + (uint32_t)(32 * w + 16), e1);
+        float dv = 0.f, ev = 0.f;
+#pragma unroll
+        for (int q = 0; q < 16; ++q) {
+            if (lane == q) { dv = d0[q]; ev = e0[q]; }
+            if (lane == 16 + q) { dv = d1[q]; ev = e1[q]; }
+        }
+        const float n = __fmul_rn(0.5f, __fadd_rn(dv, ev));
+        nrm[(int64_t)I * T + r] = n;
+        atomicMax(nmax_bits, __float_as_int(fmaxf(n, 0.f)));
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (w == 0) tmem_free(tbase);
+}
+
+// ---------------------------------------------------------------- the tile kernel
+// Persistent: CTA b owns the contiguous tile range [b per, (b+1) per) of the packed
+// upper triangle (row-major over I <= J), so consecutive tiles share the row block I
+// (its two operand blocks are reloaded only when I changes).  As soon as a tile's
+// MMAs completed, the operand copies of the next tile are issued (cp.async.bulk),
+// overlapping this tile's epilogue.  Epilogue: warp w reads TMEM lanes 32 (w % 4)
+// .. +31 (tile rows), columns 64 (w / 4) .. +63 of D and D', forms K and stores each
+// row segment with 16-byte streaming stores; tiles on the ragged edge zero the
+// padding.
+__device__ __forceinline__ void st_cs4(float* p, float a, float b, float c, float d) {
+    __stcs(reinterpret_cast<float4*>(p), make_float4(a, b, c, d));
+}
+
+__global__ void __launch_bounds__(kThreads, 2)
+gram_tc_kernel(const uint8_t* __restrict__ opA, const uint8_t* __restrict__ opB, const float* __restrict__ nrm,
+               int32_t N, float gamma, float* __restrict__ K, int nT, const int* __restrict__ nmax_bits) {
+    if (!tc_ok(nmax_bits, gamma)) return;                         // the direct-form kernel writes K
+    extern __shared__ __align__(1024) uint8_t smem[];            // [A_I | B_I | A_J | B_J]
+    __shared__ __align__(8) uint64_t ldbar;
+    __shared__ __align__(8) uint64_t mmabar;
+    __shared__ uint32_t tmem_base;
+    __shared__ __align__(16) float nIs[2][T];
+    __shared__ __align__(16) float nJs[2][T];
+    const int tid = threadIdx.x, w = tid / 32, lane = tid % 32;
+    const int64_t ntiles = pk::num_tiles(nT);
+    const int64_t per = (ntiles + gridDim.x - 1) / gridDim.x;
+    const int64_t k0 = (int64_t)blockIdx.x * per, k1 = k0 + per < ntiles ? k0 + per : ntiles;
+    if (w == 0) tmem_alloc(&tmem_base);
+    if (tid == 0) {
+        pk::mbar_init(&ldbar, 1);
+        pk::mbar_init(&mmabar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
     __syncthreads();
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     const uint32_t tbase = tmem_base;
     const float ng = -gamma;
-    const int64_t ntiles = pk::num_tiles(nT);
-    uint32_t phase = 0;
-    for (int64_t k = blockIdx.x; k < ntiles; k += gridDim.x) {
-        int I, J;
-        pk::tile_ij(k, nT, I, J);
-        // operands: 2 x 24 KiB from the prepared blocks (L2-resident)
-        const uint4* ga = reinterpret_cast<const uint4*>(opA + (size_t)I * kBlockBytes);
-        const uint4* gb = reinterpret_cast<const uint4*>(opB + (size_t)J * kBlockBytes);
-        uint4* la = reinterpret_cast<uint4*>(sA);
-        uint4* lb = reinterpret_cast<uint4*>(sB);
-        for (int q = tid; q < (int)(kBlockBytes / 16); q += kThreads) {
-            la[q] = __ldg(&ga[q]);
-            lb[q] = __ldg(&gb[q]);
+    int I = 0, J = 0, loadedI = -1;
+    if (k0 < k1) pk::tile_ij(k0, nT, I, J);
+    // thread 0: the copies of tile (I, J); norms into slot b
+    auto issue = [&](int I_, int J_, int b) {
+        const bool newI = I_ != loadedI;
+        pk::mbar_expect_tx(&ldbar, (newI ? 2 * kBlockBytes : 0u) + 2 * kBlockBytes + 2u * T * 4u);
+        if (newI) {
+            pk::bulk_g2s(smem, opA + (size_t)I_ * kBlockBytes, kBlockBytes, &ldbar);
+            pk::bulk_g2s(smem + kBlockBytes, opB + (size_t)I_ * kBlockBytes, kBlockBytes, &ldbar);
         }
-        if (tid < T) { nI[tid] = nrm[(int64_t)I * T + tid]; nJ[tid] = nrm[(int64_t)J * T + tid]; }
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic smem writes -> tensor core reads
-        __syncthreads();
+        pk::bulk_g2s(smem + 2 * kBlockBytes, opA + (size_t)J_ * kBlockBytes, kBlockBytes, &ldbar);
+        pk::bulk_g2s(smem + 3 * kBlockBytes, opB + (size_t)J_ * kBlockBytes, kBlockBytes, &ldbar);
+        pk::bulk_g2s(nIs[b], nrm + (int64_t)I_ * T, T * 4u, &ldbar);
+        pk::bulk_g2s(nJs[b], nrm + (int64_t)J_ * T, T * 4u, &ldbar);
+        loadedI = I_;
+    };
+    if (tid == 0 && k0 < k1) issue(I, J, 0);
+    uint32_t ldph = 0u, mph = 0u;
+    for (int64_t k = k0; k < k1; ++k) {
+        const int b = (int)((k - k0) & 1);
+        pk::mbar_wait(&ldbar, ldph);
+        ldph ^= 1u;
         if (tid == 0) {
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-            const uint32_t a0 = smem_u32(sA), b0 = smem_u32(sB);
-#pragma unroll
-            for (int s = 0; s < kSlices; ++s)                      // each k-slice = 16 bf16 = 2 core matrices
-                mma_bf16(tbase, smem_desc(a0 + 2 * s * kLBO), smem_desc(b0 + 2 * s * kLBO), s > 0 ? 1u : 0u);
-            asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
-                         :: "r"(smem_u32(&mbar)) : "memory");
+            issue_sym_mmas(tbase, smem_u32(smem), smem_u32(smem + kBlockBytes), smem_u32(smem + 2 * kBlockBytes),
+                           smem_u32(smem + 3 * kBlockBytes));
+            mma_commit(&mmabar);
         }
-        mbar_wait(&mbar, phase);
-        phase ^= 1u;
+        pk::mbar_wait(&mmabar, mph);
+        mph ^= 1u;
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        // epilogue: warp w reads TMEM lanes 32 (w % 4) .. +31 (tile rows), columns 64 (w / 4) .. +63
+        int In = I, Jn = J + 1;                                    // the next tile of the range
+        if (Jn == nT) { ++In; Jn = In; }
+        if (tid == 0 && k + 1 < k1) issue(In, Jn, b ^ 1);          // operands free: overlaps the epilogue
+        // epilogue
         const int r = 32 * (w & 3) + lane;
         const int cbase = 64 * (w >> 2);
-        const int gi = I * T + r;
-        const float ni = nI[r];
+        const float ni = nIs[b][r];
+        const float* nj = nJs[b];
+        const bool edge = (I + 1) * T > N || (J + 1) * T > N;
+        const bool rowv = I * T + r < N;
+        float* trow = K + k * (int64_t)(T * T) + (size_t)r * T;
+        const uint32_t lb = (uint32_t)(32 * (w & 3)) << 16;
 #pragma unroll 1
         for (int cc = 0; cc < 64; cc += 16) {
-            float v[16];
-            tmem_ld16(tbase + ((uint32_t)(32 * (w & 3)) << 16) + (uint32_t)(cbase + cc), v);
+            const int c0 = cbase + cc;
+            float dv[16], ev[16];
+            tmem_ld16(tbase + lb + (uint32_t)c0, dv);
+            tmem_ld16(tbase + T + lb + (uint32_t)c0, ev);
             float o[16];
 #pragma unroll
             for (int q = 0; q < 16; ++q) {
-                const int cj = cbase + cc + q;
-                const int gj = J * T + cj;
-                float d2 = __fmaf_rn(-2.f, v[q], __fadd_rn(ni, nJ[cj]));
-                d2 = d2 > 0.f ? d2 : 0.f;
-                const float kv = gi == gj ? 1.f : expf(__fmul_rn(ng, d2));
-                o[q] = (gi < N && gj < N) ? kv : 0.f;
+                float d2 = __fsub_rn(__fadd_rn(ni, nj[c0 + q]), __fadd_rn(dv[q], ev[q]));
+                d2 = fmaxf(d2, 0.f);
+                o[q] = expf(__fmul_rn(ng, d2));
             }
-            float4* dst = reinterpret_cast<float4*>(stage + (size_t)r * kStageLd + cbase + cc);
+            if (edge) {
 #pragma unroll
-            for (int q = 0; q < 4; ++q) dst[q] = make_float4(o[4 * q], o[4 * q + 1], o[4 * q + 2], o[4 * q + 3]);
+                for (int q = 0; q < 16; ++q)
+                    if (!rowv || J * T + c0 + q >= N) o[q] = 0.f;
+            }
+#pragma unroll
+            for (int q = 0; q < 16; q += 4) st_cs4(trow + c0 + q, o[q], o[q + 1], o[q + 2], o[q + 3]);
         }
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-        __syncthreads();
-        // coalesced store: warp w writes rows w, w + 8, ...; diagonal tiles mirror the upper triangle
-        float* tile = K + k * (int64_t)(T * T);
-        for (int row = w; row < T; row += kThreads / 32) {
-            const float* srow = stage + (size_t)row * kStageLd;
-            float4 o = *reinterpret_cast<const float4*>(srow + 4 * lane);
-            if (I == J) {
-                float* oc = &o.x;
-#pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                    const int col = 4 * lane + q;
-                    if (col < row) oc[q] = stage[(size_t)col * kStageLd + row];
-                }
-            }
-            __stcs(reinterpret_cast<float4*>(tile + (size_t)row * T) + lane, o);
-        }
-        __syncthreads();                                           // staging / operand space reused next tile
+        __syncthreads();                                           // TMEM read out: the next MMA may write it
+        I = In;
+        J = Jn;
     }
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
     __syncthreads();
-    if (w == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(tbase), "n"(T));
+    if (w == 0) tmem_free(tbase);
 }
 
 }  // namespace tc

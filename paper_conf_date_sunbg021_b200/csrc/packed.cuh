@@ -664,7 +664,7 @@ gram_packed_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamm
 template <int kD, bool kLinear, int kH = 4>
 __global__ void __launch_bounds__(kConsumers, kH == 4 ? 2 : 3)
 gram_tile_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma, float* __restrict__ K, int nT,
-                 int sr = 0, int sp = 1) {
+                 int sr = 0, int sp = 1, const int* __restrict__ = nullptr) {
     __shared__ __align__(16) unsigned long long xi2[T][kD];     // (x, x) pairs of the tile's rows
     __shared__ __align__(16) float xj[T][kD];
     const int tid = threadIdx.x, w = tid / kWarp, l = tid % kWarp;
@@ -743,7 +743,10 @@ gram_tile_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma,
 template <int kD, bool kLinear, int kH>
 __global__ void __launch_bounds__(kConsumers, 4)
 gram_tile2_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma, float* __restrict__ K, int nT,
-                  int sr = 0, int sp = 1) {
+                  int sr = 0, int sp = 1, const int* __restrict__ tc_nmax_bits = nullptr) {
+    // (the implicit head launches this kernel after the tensor-core one: it writes K only
+    // when the tensor-core kernel's accuracy guard declined, gram_tc.cuh kGuard)
+    if (tc_nmax_bits && __fmul_rn(gamma, __int_as_float(*tc_nmax_bits)) <= 4.f) return;
     __shared__ __align__(16) unsigned long long xi2[T][kD];     // (x, x) pairs of the tile's rows
     __shared__ __align__(16) float xj[T][kD + 1];
     const int tid = threadIdx.x, w = tid / kWarp, l = tid % kWarp;

@@ -105,8 +105,20 @@ def test_tensor_core_gram_c1_bound(N, d, pool):
     ratio = np.abs(K32 - K64) / (ulp32(K64) * (1.0 + float(g) * d2))
     print(f"TC Gram N={N} d={d} {pool}: max {ratio.max():.2f} ulp*(1+g d2)")
     assert ratio.max() <= 6.0
-    if pool == "knob-dups":
+    if pool == "knob-dups":                                  # S = D + D' is symmetric bitwise: twins tie
         assert np.array_equal(K[: N // 2, :N], K[N // 2:, :N][:, np.r_[N // 2:N, 0:N // 2]])
+
+
+def test_tensor_core_gram_guard_falls_back_on_badly_scaled_data():
+    """gamma * max |x - c|^2 far above the guard (points 100 apart, gamma = 1):
+    the expansion would cancel catastrophically, so the direct-difference kernel
+    writes the Gram -- exactly the identity here."""
+    N = 3000
+    X = (np.arange(N, dtype=np.float32) * 100.0)[:, None]
+    with bt.CandidateSet(X, 1.0, flags=IMPLICIT) as cs:
+        cs.select(2, MU)
+        K = cs.debug_K(N)
+    assert np.array_equal(K[:, :N], np.eye(N, dtype=np.float32))
 
 
 # ------------------------------------------------------------------ K2 step
