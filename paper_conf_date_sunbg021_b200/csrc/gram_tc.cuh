@@ -45,7 +45,7 @@ constexpr int kK = kD * kSlices;               // 96 bf16 per row
 constexpr uint32_t kLBO = 128;                 // bytes between k-adjacent core matrices
 constexpr uint32_t kSBO = (kK / 8) * 128;      // 1536: bytes between 8-row groups
 constexpr uint32_t kBlockBytes = (T / 8) * kSBO;   // 24576 per 128-row block
-constexpr size_t kSmemBytes = 4 * (size_t)kBlockBytes;       // A_I, B_I, A_J, B_J (96 KiB)
+
 // kind::f16, A = B = bf16 (K-major), D = f32, M = 128, N = 128
 constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(T >> 3) << 17) | ((uint32_t)(T >> 4) << 24);
 
@@ -55,31 +55,45 @@ __host__ __device__ __forceinline__ uint32_t op_offset(int r, int k) {
 }
 
 // ---------------------------------------------------------------- prep
-// c = mean of the N rows (one CTA: per thread the rows tid, tid + 1024, ... in
-// order, then a fixed butterfly and the warps in order): any c is exact in the
-// algebra; the mean keeps the expansion's cancellation small
-constexpr int kCenterThreads = 1024;
-__global__ void __launch_bounds__(kCenterThreads) center_kernel(const float* __restrict__ X, int32_t N, int32_t d,
-                                                               float* __restrict__ c) {
+// c = mean of the N rows (fixed-order partial sums: deterministic): any c is exact
+// in the algebra; the mean keeps the expansion's cancellation small
+constexpr int kCenterThreads = 256;
+constexpr int kCenterBlocks = 64;
+// pass 1: CTA b sums rows b*256 + tid, + 64*256, ... (in order) per thread, then a
+// fixed tree over its threads -> part[b][k]
+__global__ void __launch_bounds__(kCenterThreads) center_part_kernel(const float* __restrict__ X, int32_t N, int32_t d,
+                                                                    float* __restrict__ part) {
     __shared__ float red[kCenterThreads / 32][kD];
     float s[kD];
 #pragma unroll
     for (int k = 0; k < kD; ++k) s[k] = 0.f;
-    for (int i = threadIdx.x; i < N; i += kCenterThreads)        // rows tid, tid + 1024, ... in order
-        for (int k = 0; k < d; ++k) s[k] = __fadd_rn(s[k], X[(int64_t)i * d + k]);
+    for (int64_t i = (int64_t)blockIdx.x * kCenterThreads + threadIdx.x; i < N;
+         i += (int64_t)kCenterBlocks * kCenterThreads) {
+#pragma unroll
+        for (int k = 0; k < kD; ++k)
+            if (k < d) s[k] = __fadd_rn(s[k], X[i * d + k]);
+    }
     const int w = threadIdx.x / 32, l = threadIdx.x % 32;
 #pragma unroll
-    for (int k = 0; k < kD; ++k) {                               // fixed butterfly, then warps in order
+    for (int k = 0; k < kD; ++k) {
         float v = s[k];
         for (int off = 16; off > 0; off >>= 1) v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, off));
         if (l == 0) red[w][k] = v;
     }
     __syncthreads();
-    if (threadIdx.x < d) {
+    if (threadIdx.x < kD) {
         float t = 0.f;
         for (int q = 0; q < kCenterThreads / 32; ++q) t = __fadd_rn(t, red[q][threadIdx.x]);
-        c[threadIdx.x] = __fdiv_rn(t, (float)N);
+        part[blockIdx.x * kD + threadIdx.x] = t;
     }
+}
+// pass 2: c_k = (sum of the 64 partials in order) / N
+__global__ void center_kernel(const float* __restrict__ part, int32_t N, int32_t d, float* __restrict__ c) {
+    const int k = threadIdx.x;
+    if (k >= d) return;
+    float t = 0.f;
+    for (int b = 0; b < kCenterBlocks; ++b) t = __fadd_rn(t, part[b * kD + k]);
+    c[k] = __fdiv_rn(t, (float)N);
 }
 
 __device__ __forceinline__ void split3(float v, __nv_bfloat16& h, __nv_bfloat16& m, __nv_bfloat16& l) {
@@ -100,19 +114,26 @@ __global__ void __launch_bounds__(kThreads) prep_kernel(const float* __restrict_
     const int blk = (int)(i / T), r = (int)(i % T);
     uint8_t* a = opA + (size_t)blk * kBlockBytes;
     uint8_t* b = opB + (size_t)blk * kBlockBytes;
+    __nv_bfloat16 h[kD], m[kD], l[kD];
+#pragma unroll
     for (int k = 0; k < kD; ++k) {
         float v = 0.f;
         if (i < N && k < d) v = __fsub_rn(X[i * d + k], c[k]);
-        __nv_bfloat16 h, m, l;
-        split3(v, h, m, l);
-        const __nv_bfloat16 sa[kSlices] = {m, h, l, h, m, h};
-        const __nv_bfloat16 sb[kSlices] = {m, l, h, m, h, h};
-#pragma unroll
-        for (int s = 0; s < kSlices; ++s) {
-            *reinterpret_cast<__nv_bfloat16*>(a + op_offset(r, s * kD + k)) = sa[s];
-            *reinterpret_cast<__nv_bfloat16*>(b + op_offset(r, s * kD + k)) = sb[s];
-        }
+        split3(v, h[k], m[k], l[k]);
     }
+    // slice s of a row = 16 bf16 = two 16-byte core-matrix rows (features 0-7, 8-15)
+    auto put = [&](uint8_t* base, int s, const __nv_bfloat16 (&v)[kD]) {
+#pragma unroll
+        for (int kc = 0; kc < 2; ++kc) {
+            uint4 q;
+            __nv_bfloat16* e = reinterpret_cast<__nv_bfloat16*>(&q);
+#pragma unroll
+            for (int x = 0; x < 8; ++x) e[x] = v[8 * kc + x];
+            *reinterpret_cast<uint4*>(base + op_offset(r, s * kD + 8 * kc)) = q;
+        }
+    };
+    put(a, 0, m); put(a, 1, h); put(a, 2, l); put(a, 3, h); put(a, 4, m); put(a, 5, h);   // A: m h l h m h
+    put(b, 0, m); put(b, 1, l); put(b, 2, h); put(b, 3, m); put(b, 4, h); put(b, 5, h);   // B: m l h m h h
 }
 
 // ---------------------------------------------------------------- tcgen05 helpers
@@ -244,28 +265,31 @@ gram_tc_norm_kernel(const uint8_t* __restrict__ opA, const uint8_t* __restrict__
 }
 
 // ---------------------------------------------------------------- the tile kernel
-// Persistent: CTA b owns the contiguous tile range [b per, (b+1) per) of the packed
-// upper triangle (row-major over I <= J), so consecutive tiles share the row block I
-// (its two operand blocks are reloaded only when I changes).  As soon as a tile's
-// MMAs completed, the operand copies of the next tile are issued (cp.async.bulk),
-// overlapping this tile's epilogue.  Epilogue: warp w reads TMEM lanes 32 (w % 4)
-// .. +31 (tile rows), columns 64 (w / 4) .. +63 of D and D', forms K and stores each
-// row segment with 16-byte streaming stores; tiles on the ragged edge zero the
-// padding.
-__device__ __forceinline__ void st_cs4(float* p, float a, float b, float c, float d) {
-    __stcs(reinterpret_cast<float4*>(p), make_float4(a, b, c, d));
-}
+// Persistent, 512 threads: CTA b owns the contiguous tile range [b per, (b+1) per)
+// of the packed upper triangle (row-major over I <= J), so consecutive tiles share
+// the row block I (its two operand blocks are reloaded only when I changes).  As
+// soon as a tile's MMAs completed, the operand copies of the next tile are issued
+// (cp.async.bulk), overlapping this tile's epilogue.  Epilogue: warp w reads TMEM
+// lanes 32 (w % 4) .. +31 (tile rows), columns 32 (w / 4) .. +31 of D and D', forms
+// K into a padded staging tile in shared memory, and the CTA then writes the
+// tile with coalesced 512-byte row stores (16-byte accesses per lane); tiles on the
+// ragged edge zero the padding.
+constexpr int kTcThreads = 512;
+constexpr int kStageLd = T + 4;                                  // conflict-free float4 staging rows
+constexpr size_t kStageBytes = (size_t)T * kStageLd * sizeof(float);
+constexpr size_t kTileSmemBytes = 4 * (size_t)kBlockBytes + kStageBytes;   // 96 KiB + 66 KiB
 
-__global__ void __launch_bounds__(kThreads, 2)
+__global__ void __launch_bounds__(kTcThreads, 1)
 gram_tc_kernel(const uint8_t* __restrict__ opA, const uint8_t* __restrict__ opB, const float* __restrict__ nrm,
                int32_t N, float gamma, float* __restrict__ K, int nT, const int* __restrict__ nmax_bits) {
     if (!tc_ok(nmax_bits, gamma)) return;                         // the direct-form kernel writes K
-    extern __shared__ __align__(1024) uint8_t smem[];            // [A_I | B_I | A_J | B_J]
+    extern __shared__ __align__(1024) uint8_t smem[];            // [A_I | B_I | A_J | B_J | stage]
     __shared__ __align__(8) uint64_t ldbar;
     __shared__ __align__(8) uint64_t mmabar;
     __shared__ uint32_t tmem_base;
     __shared__ __align__(16) float nIs[2][T];
     __shared__ __align__(16) float nJs[2][T];
+    float* stage = reinterpret_cast<float*>(smem + 4 * kBlockBytes);
     const int tid = threadIdx.x, w = tid / 32, lane = tid % 32;
     const int64_t ntiles = pk::num_tiles(nT);
     const int64_t per = (ntiles + gridDim.x - 1) / gridDim.x;
@@ -297,56 +321,69 @@ gram_tc_kernel(const uint8_t* __restrict__ opA, const uint8_t* __restrict__ opB,
         pk::bulk_g2s(nJs[b], nrm + (int64_t)J_ * T, T * 4u, &ldbar);
         loadedI = I_;
     };
-    if (tid == 0 && k0 < k1) issue(I, J, 0);
     uint32_t ldph = 0u, mph = 0u;
-    for (int64_t k = k0; k < k1; ++k) {
-        const int b = (int)((k - k0) & 1);
+    // software pipeline per tile k: [MMA(k) done] -> copies of k+1 issued -> TMEM read-out of k
+    // -> MMA(k+1) issued (async) -> the stores of k overlap it
+    auto mma = [&]() {
         pk::mbar_wait(&ldbar, ldph);
         ldph ^= 1u;
-        if (tid == 0) {
-            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-            issue_sym_mmas(tbase, smem_u32(smem), smem_u32(smem + kBlockBytes), smem_u32(smem + 2 * kBlockBytes),
-                           smem_u32(smem + 3 * kBlockBytes));
-            mma_commit(&mmabar);
-        }
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        issue_sym_mmas(tbase, smem_u32(smem), smem_u32(smem + kBlockBytes), smem_u32(smem + 2 * kBlockBytes),
+                       smem_u32(smem + 3 * kBlockBytes));
+        mma_commit(&mmabar);
+    };
+    if (tid == 0 && k0 < k1) { issue(I, J, 0); mma(); }
+    for (int64_t k = k0; k < k1; ++k) {
+        const int b = (int)((k - k0) & 1);
         pk::mbar_wait(&mmabar, mph);
         mph ^= 1u;
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         int In = I, Jn = J + 1;                                    // the next tile of the range
         if (Jn == nT) { ++In; Jn = In; }
-        if (tid == 0 && k + 1 < k1) issue(In, Jn, b ^ 1);          // operands free: overlaps the epilogue
-        // epilogue
-        const int r = 32 * (w & 3) + lane;
-        const int cbase = 64 * (w >> 2);
-        const float ni = nIs[b][r];
-        const float* nj = nJs[b];
-        const bool edge = (I + 1) * T > N || (J + 1) * T > N;
-        const bool rowv = I * T + r < N;
-        float* trow = K + k * (int64_t)(T * T) + (size_t)r * T;
-        const uint32_t lb = (uint32_t)(32 * (w & 3)) << 16;
-#pragma unroll 1
-        for (int cc = 0; cc < 64; cc += 16) {
-            const int c0 = cbase + cc;
-            float dv[16], ev[16];
-            tmem_ld16(tbase + lb + (uint32_t)c0, dv);
-            tmem_ld16(tbase + T + lb + (uint32_t)c0, ev);
-            float o[16];
+        if (tid == 0 && k + 1 < k1) issue(In, Jn, b ^ 1);          // operands free after MMA(k)
+        // epilogue part 1: TMEM -> K values -> staging
+        {
+            const int r = 32 * (w & 3) + lane;
+            const int cbase = 32 * (w >> 2);
+            const float ni = nIs[b][r];
+            const float* nj = nJs[b];
+            const bool edge = (I + 1) * T > N || (J + 1) * T > N;
+            const bool rowv = I * T + r < N;
+            const uint32_t lb = (uint32_t)(32 * (w & 3)) << 16;
 #pragma unroll
-            for (int q = 0; q < 16; ++q) {
-                float d2 = __fsub_rn(__fadd_rn(ni, nj[c0 + q]), __fadd_rn(dv[q], ev[q]));
-                d2 = fmaxf(d2, 0.f);
-                o[q] = expf(__fmul_rn(ng, d2));
+            for (int cc = 0; cc < 32; cc += 16) {
+                const int c0 = cbase + cc;
+                float dv[16], ev[16];
+                tmem_ld16(tbase + lb + (uint32_t)c0, dv);
+                tmem_ld16(tbase + T + lb + (uint32_t)c0, ev);
+                float o[16];
+#pragma unroll
+                for (int q = 0; q < 16; ++q) {
+                    float d2 = __fsub_rn(__fadd_rn(ni, nj[c0 + q]), __fadd_rn(dv[q], ev[q]));
+                    d2 = fmaxf(d2, 0.f);
+                    o[q] = expf(__fmul_rn(ng, d2));
+                }
+                if (edge) {
+#pragma unroll
+                    for (int q = 0; q < 16; ++q)
+                        if (!rowv || J * T + c0 + q >= N) o[q] = 0.f;
+                }
+                float4* dst = reinterpret_cast<float4*>(stage + (size_t)r * kStageLd + c0);
+#pragma unroll
+                for (int q = 0; q < 4; ++q) dst[q] = make_float4(o[4 * q], o[4 * q + 1], o[4 * q + 2], o[4 * q + 3]);
             }
-            if (edge) {
-#pragma unroll
-                for (int q = 0; q < 16; ++q)
-                    if (!rowv || J * T + c0 + q >= N) o[q] = 0.f;
-            }
-#pragma unroll
-            for (int q = 0; q < 16; q += 4) st_cs4(trow + c0 + q, o[q], o[q + 1], o[q + 2], o[q + 3]);
         }
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-        __syncthreads();                                           // TMEM read out: the next MMA may write it
+        __syncthreads();                                           // TMEM read out; the staged tile complete
+        if (tid == 0 && k + 1 < k1) mma();                         // MMA(k+1) overlaps the stores below
+        // epilogue part 2: coalesced 512-byte rows (warp w: rows w, w + 16, ...)
+        float* tile = K + k * (int64_t)(T * T);
+#pragma unroll 2
+        for (int row = w; row < T; row += kTcThreads / 32) {
+            const float4 v = *reinterpret_cast<const float4*>(stage + (size_t)row * kStageLd + 4 * lane);
+            __stcs(reinterpret_cast<float4*>(tile + (size_t)row * T) + lane, v);
+        }
+        __syncthreads();                                           // the staging tile is reused next tile
         I = In;
         J = Jn;
     }
