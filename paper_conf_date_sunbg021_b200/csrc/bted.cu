@@ -240,7 +240,6 @@ struct Ted {
         grow(hv, hvcap, (size_t)m + 1);
         if (gram_tc) {
             grow(opA, opAcap, (size_t)nT * bted::tc::kBlockBytes);
-            grow(opB, opBcap, (size_t)nT * bted::tc::kBlockBytes);
             grow(xnrm, xnrmcap, NP);
             grow(xctr, xctrcap, (size_t)bted::tc::kD * (1 + bted::tc::kCenterBlocks));
             grow(xmax, xmaxcap, 1);
@@ -477,7 +476,7 @@ void ensure_gram_tc_attrs() {
         CK(cudaFuncSetAttribute(bted::tc::gram_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)bted::tc::kTileSmemBytes));
         CK(cudaFuncSetAttribute(bted::tc::gram_tc_norm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)(2 * bted::tc::kBlockBytes)));
+                                (int)bted::tc::kBlockBytes));
     });
 }
 
@@ -505,13 +504,13 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
             X, (int32_t)N, d, T.xctr + bted::tc::kD);
         bted::tc::center_kernel<<<1, 32, 0, T.stream>>>(T.xctr + bted::tc::kD, (int32_t)N, d, T.xctr);
         bted::tc::prep_kernel<<<(unsigned)((NP + bted::tc::kThreads - 1) / bted::tc::kThreads), bted::tc::kThreads, 0,
-                                T.stream>>>(X, (int32_t)N, d, nT, T.xctr, T.opA, T.opB);
+                                T.stream>>>(X, (int32_t)N, d, nT, T.xctr, T.opA);
         CK(cudaMemsetAsync(T.xmax, 0, sizeof(int), T.stream));
-        bted::tc::gram_tc_norm_kernel<<<(unsigned)nT, bted::tc::kThreads, 2 * bted::tc::kBlockBytes, T.stream>>>(
-            T.opA, T.opB, T.xnrm, T.xmax);
-        const unsigned g = (unsigned)std::min<int64_t>(tiles, (int64_t)num_sms());
+        bted::tc::gram_tc_norm_kernel<<<(unsigned)nT, bted::tc::kThreads, bted::tc::kBlockBytes, T.stream>>>(
+            T.opA, T.xnrm, T.xmax);
+        const unsigned g = (unsigned)std::min<int64_t>(tiles, (int64_t)2 * num_sms());
         bted::tc::gram_tc_kernel<<<g, bted::tc::kTcThreads, bted::tc::kTileSmemBytes, T.stream>>>(
-            T.opA, T.opB, T.xnrm, (int32_t)N, gamma, T.K[0], nT, T.xmax);
+            T.opA, T.xnrm, (int32_t)N, gamma, T.K[0], nT, T.xmax);
         // the accuracy guard's fallback (exits at once when the tensor-core Gram was written)
         bted::pk::gram_tile2_kernel<16, false, 4><<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
             X, (int32_t)N, d, gamma, T.K[0], nT, 0, 1, T.xmax);

@@ -104,16 +104,15 @@ __device__ __forceinline__ void split3(float v, __nv_bfloat16& h, __nv_bfloat16&
     l = __float2bfloat16_rn(r2);                                  // exact for normal v
 }
 
-// per row i (padding rows: 0): x' = x - c and the two operand blocks:
-// A slices [m, h, l, h, m, h], B slices [m, l, h, m, h, h]
+// per row i (padding rows: 0): x' = x - c and its operand row, slices
+// [m, h, l, h, m, h] (the B arrangement is the same block with permuted slices)
 __global__ void __launch_bounds__(kThreads) prep_kernel(const float* __restrict__ X, int32_t N, int32_t d,
                                                        int nT, const float* __restrict__ c,
-                                                       uint8_t* __restrict__ opA, uint8_t* __restrict__ opB) {
+                                                       uint8_t* __restrict__ opA) {
     const int64_t i = (int64_t)blockIdx.x * kThreads + threadIdx.x;
     if (i >= (int64_t)nT * T) return;
     const int blk = (int)(i / T), r = (int)(i % T);
     uint8_t* a = opA + (size_t)blk * kBlockBytes;
-    uint8_t* b = opB + (size_t)blk * kBlockBytes;
     __nv_bfloat16 h[kD], m[kD], l[kD];
 #pragma unroll
     for (int k = 0; k < kD; ++k) {
@@ -133,11 +132,17 @@ __global__ void __launch_bounds__(kThreads) prep_kernel(const float* __restrict_
         }
     };
     put(a, 0, m); put(a, 1, h); put(a, 2, l); put(a, 3, h); put(a, 4, m); put(a, 5, h);   // A: m h l h m h
-    put(b, 0, m); put(b, 1, l); put(b, 2, h); put(b, 3, m); put(b, 4, h); put(b, 5, h);   // B: m l h m h h
 }
 
 // ---------------------------------------------------------------- tcgen05 helpers
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+// 2^x on the SFU (MUFU.EX2); the rounding of the scaled argument -g log2(e) d2 adds a
+// relative error ~ g d2 ulp, inside pin C1's (1 + g d2) factor
+__device__ __forceinline__ float ex2_approx(float x) {
+    float y;
+    asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
 
 __device__ __forceinline__ uint64_t smem_desc(uint32_t saddr) {
     uint64_t desc = 0;
@@ -187,13 +192,17 @@ __device__ __forceinline__ bool tc_ok(const int* nmax_bits, float gamma) {
     return __fmul_rn(gamma, __int_as_float(*nmax_bits)) <= kGuard;
 }
 
-__device__ __forceinline__ void issue_sym_mmas(uint32_t tbase, uint32_t aI, uint32_t bI, uint32_t aJ, uint32_t bJ) {
+// The B arrangement [m, l, h, m, h, h] is the A arrangement [m, h, l, h, m, h] with
+// its slices permuted (kPerm), so only A blocks are stored: B's slice s is A's
+// slice kPerm[s], addressed through the descriptor's start offset.
+__device__ __forceinline__ uint32_t perm_slice(int s) { return s == 1 ? 2u : s == 2 ? 1u : s == 3 ? 4u : s == 4 ? 3u : (uint32_t)s; }
+__device__ __forceinline__ void issue_sym_mmas(uint32_t tbase, uint32_t aI, uint32_t aJ) {
 #pragma unroll
-    for (int s = 0; s < kSlices; ++s)                          // each k-slice = 16 bf16 = 2 core matrices
-        mma_bf16(tbase, smem_desc(aI + 2 * s * kLBO), smem_desc(bJ + 2 * s * kLBO), s > 0 ? 1u : 0u);
+    for (int s = 0; s < kSlices; ++s)                          // D = A_I . B_J^T
+        mma_bf16(tbase, smem_desc(aI + 2 * s * kLBO), smem_desc(aJ + 2 * perm_slice(s) * kLBO), s > 0 ? 1u : 0u);
 #pragma unroll
-    for (int s = 0; s < kSlices; ++s)
-        mma_bf16(tbase + T, smem_desc(bI + 2 * s * kLBO), smem_desc(aJ + 2 * s * kLBO), s > 0 ? 1u : 0u);
+    for (int s = 0; s < kSlices; ++s)                          // D' = B_I . A_J^T
+        mma_bf16(tbase + T, smem_desc(aI + 2 * perm_slice(s) * kLBO), smem_desc(aJ + 2 * s * kLBO), s > 0 ? 1u : 0u);
 }
 
 __device__ __forceinline__ void tmem_alloc(uint32_t* dst) {
@@ -211,9 +220,8 @@ __device__ __forceinline__ void mma_commit(uint64_t* bar) {
 
 // n_r = S_rr / 2 for every row of every block (one CTA per block I: the diagonal tile's S)
 __global__ void __launch_bounds__(kThreads)
-gram_tc_norm_kernel(const uint8_t* __restrict__ opA, const uint8_t* __restrict__ opB, float* __restrict__ nrm,
-                    int* __restrict__ nmax_bits) {
-    extern __shared__ __align__(1024) uint8_t smem[];            // [A_I | B_I]
+gram_tc_norm_kernel(const uint8_t* __restrict__ opA, float* __restrict__ nrm, int* __restrict__ nmax_bits) {
+    extern __shared__ __align__(1024) uint8_t smem[];            // [A_I]
     __shared__ __align__(8) uint64_t ldbar, mmabar;
     __shared__ uint32_t tmem_base;
     const int tid = threadIdx.x, w = tid / 32, lane = tid % 32, I = blockIdx.x;
@@ -228,15 +236,14 @@ gram_tc_norm_kernel(const uint8_t* __restrict__ opA, const uint8_t* __restrict__
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     const uint32_t tbase = tmem_base;
     if (tid == 0) {
-        pk::mbar_expect_tx(&ldbar, 2 * kBlockBytes);
+        pk::mbar_expect_tx(&ldbar, kBlockBytes);
         pk::bulk_g2s(smem, opA + (size_t)I * kBlockBytes, kBlockBytes, &ldbar);
-        pk::bulk_g2s(smem + kBlockBytes, opB + (size_t)I * kBlockBytes, kBlockBytes, &ldbar);
     }
     pk::mbar_wait(&ldbar, 0);
     if (tid == 0) {
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        const uint32_t a = smem_u32(smem), b = smem_u32(smem + kBlockBytes);
-        issue_sym_mmas(tbase, a, b, a, b);
+        const uint32_t a = smem_u32(smem);
+        issue_sym_mmas(tbase, a, a);
         mma_commit(&mmabar);
     }
     pk::mbar_wait(&mmabar, 0);
@@ -265,31 +272,34 @@ gram_tc_norm_kernel(const uint8_t* __restrict__ opA, const uint8_t* __restrict__
 }
 
 // ---------------------------------------------------------------- the tile kernel
-// Persistent, 512 threads: CTA b owns the contiguous tile range [b per, (b+1) per)
-// of the packed upper triangle (row-major over I <= J), so consecutive tiles share
-// the row block I (its two operand blocks are reloaded only when I changes).  As
-// soon as a tile's MMAs completed, the operand copies of the next tile are issued
-// (cp.async.bulk), overlapping this tile's epilogue.  Epilogue: warp w reads TMEM
-// lanes 32 (w % 4) .. +31 (tile rows), columns 32 (w / 4) .. +31 of D and D', forms
-// K into a padded staging tile in shared memory, and the CTA then writes the
-// tile with coalesced 512-byte row stores (16-byte accesses per lane); tiles on the
-// ragged edge zero the padding.
-constexpr int kTcThreads = 512;
-constexpr int kStageLd = T + 4;                                  // conflict-free float4 staging rows
+// Persistent, two CTAs (256 threads each) per SM: CTA b owns the contiguous tile
+// range [b per, (b+1) per) of the packed upper triangle (row-major over I <= J), so
+// consecutive tiles share the row block I (its operand block is reloaded only when
+// I changes).  As soon as a tile's MMAs completed, the operand copies of the next
+// tile are issued (cp.async.bulk), overlapping this tile's epilogue; the next
+// tile's MMAs are issued as soon as the accumulators are read out, overlapping the
+// last stores.  Epilogue, in two column halves: warp w reads TMEM lanes 32 (w % 4)
+// .. +31 (tile rows) and 32 of the columns 64 (w / 4) .. +63 of D and D', forms K
+// into a padded staging buffer (128 rows x 64 columns), and the CTA writes the half
+// tile with coalesced 128-byte row segments; tiles on the ragged edge zero the
+// padding.  The other CTA on the SM computes while this one stores.
+constexpr int kTcThreads = 256;
+constexpr int kStageCols = 64;
+constexpr int kStageLd = kStageCols + 4;                         // conflict-free float4 staging rows
 constexpr size_t kStageBytes = (size_t)T * kStageLd * sizeof(float);
-constexpr size_t kTileSmemBytes = 4 * (size_t)kBlockBytes + kStageBytes;   // 96 KiB + 66 KiB
+constexpr size_t kTileSmemBytes = 2 * (size_t)kBlockBytes + kStageBytes;   // 48 KiB + 34 KiB
 
-__global__ void __launch_bounds__(kTcThreads, 1)
-gram_tc_kernel(const uint8_t* __restrict__ opA, const uint8_t* __restrict__ opB, const float* __restrict__ nrm,
+__global__ void __launch_bounds__(kTcThreads, 2)
+gram_tc_kernel(const uint8_t* __restrict__ opA, const float* __restrict__ nrm,
                int32_t N, float gamma, float* __restrict__ K, int nT, const int* __restrict__ nmax_bits) {
     if (!tc_ok(nmax_bits, gamma)) return;                         // the direct-form kernel writes K
-    extern __shared__ __align__(1024) uint8_t smem[];            // [A_I | B_I | A_J | B_J | stage]
+    extern __shared__ __align__(1024) uint8_t smem[];            // [A_I | A_J | stage]
     __shared__ __align__(8) uint64_t ldbar;
     __shared__ __align__(8) uint64_t mmabar;
     __shared__ uint32_t tmem_base;
     __shared__ __align__(16) float nIs[2][T];
     __shared__ __align__(16) float nJs[2][T];
-    float* stage = reinterpret_cast<float*>(smem + 4 * kBlockBytes);
+    float* stage = reinterpret_cast<float*>(smem + 2 * kBlockBytes);
     const int tid = threadIdx.x, w = tid / 32, lane = tid % 32;
     const int64_t ntiles = pk::num_tiles(nT);
     const int64_t per = (ntiles + gridDim.x - 1) / gridDim.x;
@@ -304,35 +314,31 @@ gram_tc_kernel(const uint8_t* __restrict__ opA, const uint8_t* __restrict__ opB,
     __syncthreads();
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     const uint32_t tbase = tmem_base;
-    const float ng = -gamma;
+    const float ngl2e = __fmul_rn(-gamma, 1.4426950408889634f);   // exp(-g d2) = 2^(-g log2(e) d2)
     int I = 0, J = 0, loadedI = -1;
     if (k0 < k1) pk::tile_ij(k0, nT, I, J);
     // thread 0: the copies of tile (I, J); norms into slot b
     auto issue = [&](int I_, int J_, int b) {
         const bool newI = I_ != loadedI;
-        pk::mbar_expect_tx(&ldbar, (newI ? 2 * kBlockBytes : 0u) + 2 * kBlockBytes + 2u * T * 4u);
-        if (newI) {
-            pk::bulk_g2s(smem, opA + (size_t)I_ * kBlockBytes, kBlockBytes, &ldbar);
-            pk::bulk_g2s(smem + kBlockBytes, opB + (size_t)I_ * kBlockBytes, kBlockBytes, &ldbar);
-        }
-        pk::bulk_g2s(smem + 2 * kBlockBytes, opA + (size_t)J_ * kBlockBytes, kBlockBytes, &ldbar);
-        pk::bulk_g2s(smem + 3 * kBlockBytes, opB + (size_t)J_ * kBlockBytes, kBlockBytes, &ldbar);
+        pk::mbar_expect_tx(&ldbar, (newI ? kBlockBytes : 0u) + kBlockBytes + 2u * T * 4u);
+        if (newI) pk::bulk_g2s(smem, opA + (size_t)I_ * kBlockBytes, kBlockBytes, &ldbar);
+        pk::bulk_g2s(smem + kBlockBytes, opA + (size_t)J_ * kBlockBytes, kBlockBytes, &ldbar);
         pk::bulk_g2s(nIs[b], nrm + (int64_t)I_ * T, T * 4u, &ldbar);
         pk::bulk_g2s(nJs[b], nrm + (int64_t)J_ * T, T * 4u, &ldbar);
         loadedI = I_;
     };
     uint32_t ldph = 0u, mph = 0u;
-    // software pipeline per tile k: [MMA(k) done] -> copies of k+1 issued -> TMEM read-out of k
-    // -> MMA(k+1) issued (async) -> the stores of k overlap it
     auto mma = [&]() {
         pk::mbar_wait(&ldbar, ldph);
         ldph ^= 1u;
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        issue_sym_mmas(tbase, smem_u32(smem), smem_u32(smem + kBlockBytes), smem_u32(smem + 2 * kBlockBytes),
-                       smem_u32(smem + 3 * kBlockBytes));
+        issue_sym_mmas(tbase, smem_u32(smem), smem_u32(smem + kBlockBytes));
         mma_commit(&mmabar);
     };
     if (tid == 0 && k0 < k1) { issue(I, J, 0); mma(); }
+    const int q4 = w & 3, hh = w >> 2;                             // TMEM lane quarter, column half
+    const int r = 32 * q4 + lane;
+    const uint32_t lb = (uint32_t)(32 * q4) << 16;
     for (int64_t k = k0; k < k1; ++k) {
         const int b = (int)((k - k0) & 1);
         pk::mbar_wait(&mmabar, mph);
@@ -341,49 +347,53 @@ gram_tc_kernel(const uint8_t* __restrict__ opA, const uint8_t* __restrict__ opB,
         int In = I, Jn = J + 1;                                    // the next tile of the range
         if (Jn == nT) { ++In; Jn = In; }
         if (tid == 0 && k + 1 < k1) issue(In, Jn, b ^ 1);          // operands free after MMA(k)
-        // epilogue part 1: TMEM -> K values -> staging
-        {
-            const int r = 32 * (w & 3) + lane;
-            const int cbase = 32 * (w >> 2);
-            const float ni = nIs[b][r];
-            const float* nj = nJs[b];
-            const bool edge = (I + 1) * T > N || (J + 1) * T > N;
-            const bool rowv = I * T + r < N;
-            const uint32_t lb = (uint32_t)(32 * (w & 3)) << 16;
-#pragma unroll
-            for (int cc = 0; cc < 32; cc += 16) {
-                const int c0 = cbase + cc;
-                float dv[16], ev[16];
-                tmem_ld16(tbase + lb + (uint32_t)c0, dv);
-                tmem_ld16(tbase + T + lb + (uint32_t)c0, ev);
-                float o[16];
-#pragma unroll
-                for (int q = 0; q < 16; ++q) {
-                    float d2 = __fsub_rn(__fadd_rn(ni, nj[c0 + q]), __fadd_rn(dv[q], ev[q]));
-                    d2 = fmaxf(d2, 0.f);
-                    o[q] = expf(__fmul_rn(ng, d2));
-                }
-                if (edge) {
-#pragma unroll
-                    for (int q = 0; q < 16; ++q)
-                        if (!rowv || J * T + c0 + q >= N) o[q] = 0.f;
-                }
-                float4* dst = reinterpret_cast<float4*>(stage + (size_t)r * kStageLd + c0);
-#pragma unroll
-                for (int q = 0; q < 4; ++q) dst[q] = make_float4(o[4 * q], o[4 * q + 1], o[4 * q + 2], o[4 * q + 3]);
-            }
-        }
-        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-        __syncthreads();                                           // TMEM read out; the staged tile complete
-        if (tid == 0 && k + 1 < k1) mma();                         // MMA(k+1) overlaps the stores below
-        // epilogue part 2: coalesced 512-byte rows (warp w: rows w, w + 16, ...)
+        const float ni = nIs[b][r];
+        const float* nj = nJs[b];
+        const bool edge = (I + 1) * T > N || (J + 1) * T > N;
+        const bool rowv = I * T + r < N;
         float* tile = K + k * (int64_t)(T * T);
+#pragma unroll 1
+        for (int half = 0; half < 2; ++half) {
+            // part 1: 32 columns per warp, TMEM -> K values -> staging columns 32 hh .. +31
+            {
+                const int c0 = 64 * hh + 32 * half;                // tile column
+                float* srow = stage + (size_t)r * kStageLd + 32 * hh;
+#pragma unroll
+                for (int cc = 0; cc < 32; cc += 16) {
+                    float dv[16], ev[16];
+                    tmem_ld16(tbase + lb + (uint32_t)(c0 + cc), dv);
+                    tmem_ld16(tbase + T + lb + (uint32_t)(c0 + cc), ev);
+                    float o[16];
+#pragma unroll
+                    for (int q = 0; q < 16; ++q) {
+                        float d2 = __fsub_rn(__fadd_rn(ni, nj[c0 + cc + q]), __fadd_rn(dv[q], ev[q]));
+                        d2 = fmaxf(d2, 0.f);
+                        o[q] = ex2_approx(__fmul_rn(ngl2e, d2));
+                    }
+                    if (edge) {
+#pragma unroll
+                        for (int q = 0; q < 16; ++q)
+                            if (!rowv || J * T + c0 + cc + q >= N) o[q] = 0.f;
+                    }
+                    float4* dst = reinterpret_cast<float4*>(srow + cc);
+#pragma unroll
+                    for (int q = 0; q < 4; ++q)
+                        dst[q] = make_float4(o[4 * q], o[4 * q + 1], o[4 * q + 2], o[4 * q + 3]);
+                }
+            }
+            if (half == 1) asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+            __syncthreads();                                       // staging half complete (half 1: TMEM read out)
+            if (half == 1 && tid == 0 && k + 1 < k1) mma();        // MMA(k+1) overlaps the stores below
+            // part 2: rows in pairs per warp instruction: lanes 0-15 row 2i, 16-31 row 2i+1;
+            // lane group g = lane % 16: segment g / 8 (tile columns 64 (g / 8) + 32 half ..), 16 B each
 #pragma unroll 2
-        for (int row = w; row < T; row += kTcThreads / 32) {
-            const float4 v = *reinterpret_cast<const float4*>(stage + (size_t)row * kStageLd + 4 * lane);
-            __stcs(reinterpret_cast<float4*>(tile + (size_t)row * T) + lane, v);
+            for (int row0 = 2 * w; row0 < T; row0 += 2 * (kTcThreads / 32)) {
+                const int row = row0 + (lane >> 4), g = lane & 15, seg = g >> 3, e = (g & 7) * 4;
+                const float4 v = *reinterpret_cast<const float4*>(stage + (size_t)row * kStageLd + 32 * seg + e);
+                __stcs(reinterpret_cast<float4*>(tile + (size_t)row * T + 64 * seg + 32 * half + e), v);
+            }
+            __syncthreads();                                       // the staging half is reused
         }
-        __syncthreads();                                           // the staging tile is reused next tile
         I = In;
         J = Jn;
     }
