@@ -833,6 +833,11 @@ struct bted_ctx {
         bool pending = false, changed = false;
         int ninst = 0; int64_t M = 0; int32_t m = 0; float mu = 0.f;
     } k4b;
+    struct {                                              // the same for the large (non-cluster) batch TEDs
+        bool pending = false;
+        int nb = 0; int64_t M = 0; int32_t m = 0; float mu = 0.f;
+    } k4big;
+    int* bfpin = nullptr; size_t bfpincap = 0;            // pinned copy of bflag
     float* xall = nullptr; size_t xallcap = 0;             // [nb][M][d] gathered batches
     unsigned long long* kall = nullptr; size_t kallcap = 0; // [nb][m] keys
     // host staging (pinned)
@@ -1364,6 +1369,7 @@ void small_k4_launch(bted_ctx* ctx, cudaStream_t st, int ninst, int64_t N, int32
     const int nUb = small_cluster_used(ninst, N, d) * bted::sm::kWarps;
     if (ctx->k4pincap < (size_t)ninst) {
         if (ctx->k4pin) cudaFreeHost(ctx->k4pin);
+        if (ctx->bfpin) cudaFreeHost(ctx->bfpin);
         ctx->k4pin = nullptr; ctx->k4pincap = 0;
         CK(cudaHostAlloc(&ctx->k4pin, sizeof(int) * ninst, cudaHostAllocDefault));
         ctx->k4pincap = (size_t)ninst;
@@ -1431,6 +1437,7 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
     Nvtx nvtx_("bted batch TEDs (Alg. 2 l.1-4)");
     const int32_t B = ctx->params.num_batches;
     ctx->k4b.pending = false;
+    ctx->k4big.pending = false;
     int nb = 0;
     for (int32_t b = b_begin; b < B; b += b_step) ++nb;
     grow(ctx->winners, ctx->winnerscap, (size_t)std::max(nb, 1) * m);
@@ -1491,28 +1498,52 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
         LAUNCHED(1);
     }
     if (k4) {
-        // K4: the near-tie steps of each flagged batch TED are re-scored exactly
-        // from its kept keys/flags/candidates; a TED is re-run only if a pick changes
-        std::vector<int> bf(nb);
-        CK(cudaMemcpyAsync(bf.data(), ctx->bflag, sizeof(int) * nb, cudaMemcpyDeviceToHost, st));
-        CK(cudaStreamSynchronize(st));
-        for (int k = 0; k < nb; ++k) {
-            if (!bf[k]) continue;
-            const uint32_t* idx = ctx->sall + (size_t)k * M;
-            gather(ctx, st, idx, M);
-            CK(cudaMemcpyAsync(ctx->mkeys, ctx->bkeys + (size_t)k * m, sizeof(unsigned long long) * m,
-                               cudaMemcpyDeviceToDevice, st));
-            CK(cudaMemcpyAsync(T.flags, ctx->bsflags + (size_t)k * m, sizeof(int) * m, cudaMemcpyDeviceToDevice, st));
-            CK(cudaMemcpyAsync(T.ncand, ctx->bncand + (size_t)k * m, sizeof(int) * m, cudaMemcpyDeviceToDevice, st));
-            CK(cudaMemcpyAsync(T.cand, ctx->bcand + (size_t)k * m * nC, sizeof(uint32_t) * m * nC,
-                               cudaMemcpyDeviceToDevice, st));
-            refine_ted(ctx, T, ctx->Xb, M, ctx->d, m, mu, ctx->mkeys, nullptr);
-            bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->mkeys, m, idx,
-                                                                     ctx->winners + (size_t)k * m);
-            LAUNCHED(1);
+        // K4 of the batch TEDs, decided at the caller's next host sync (big_k4_resolve):
+        // the per-batch near-tie counts go to pinned memory, no sync here
+        if (ctx->bfpincap < (size_t)nb) {
+            if (ctx->bfpin) cudaFreeHost(ctx->bfpin);
+            ctx->bfpin = nullptr; ctx->bfpincap = 0;
+            CK(cudaHostAlloc(&ctx->bfpin, sizeof(int) * nb, cudaHostAllocDefault));
+            ctx->bfpincap = (size_t)nb;
         }
+        CK(cudaMemcpyAsync(ctx->bfpin, ctx->bflag, sizeof(int) * nb, cudaMemcpyDeviceToHost, st));
+        ctx->k4big.pending = true;
+        ctx->k4big.nb = nb; ctx->k4big.M = M; ctx->k4big.m = m; ctx->k4big.mu = mu;
     }
     return nb;
+}
+
+// K4 of the large batch TEDs (after a host sync that follows run_batch_range): the
+// near-tie steps of each flagged batch TED are re-scored exactly from its kept
+// keys/flags/candidates; a TED is re-run only if a pick changes.  Returns true if
+// any batch's winners changed (the union must then be redone).
+bool big_k4_resolve(bted_ctx* ctx) {
+    if (!ctx->k4big.pending) return false;
+    ctx->k4big.pending = false;
+    const int nb = ctx->k4big.nb;
+    const int64_t M = ctx->k4big.M;
+    const int32_t m = ctx->k4big.m;
+    const float mu = ctx->k4big.mu;
+    Ted& T = ctx->bted_engine;
+    cudaStream_t st = ctx->stream;
+    const size_t nC = (size_t)bted::rf::kMaxCand;
+    const uint64_t corrected0 = ctx->corrected_steps;
+    for (int k = 0; k < nb; ++k) {
+        if (!ctx->bfpin[k]) continue;
+        const uint32_t* idx = ctx->sall + (size_t)k * M;
+        gather(ctx, st, idx, M);
+        CK(cudaMemcpyAsync(ctx->mkeys, ctx->bkeys + (size_t)k * m, sizeof(unsigned long long) * m,
+                           cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(T.flags, ctx->bsflags + (size_t)k * m, sizeof(int) * m, cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(T.ncand, ctx->bncand + (size_t)k * m, sizeof(int) * m, cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(T.cand, ctx->bcand + (size_t)k * m * nC, sizeof(uint32_t) * m * nC,
+                           cudaMemcpyDeviceToDevice, st));
+        refine_ted(ctx, T, ctx->Xb, M, ctx->d, m, mu, ctx->mkeys, nullptr);
+        bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->mkeys, m, idx, ctx->winners + (size_t)k * m);
+        LAUNCHED(1);
+    }
+    CK(cudaStreamSynchronize(st));
+    return ctx->corrected_steps != corrected0;
 }
 
 // After run_batch_range: wait for the batch TEDs, resolve the small-batch K4
@@ -1523,6 +1554,7 @@ bted_status batch_range_finish(bted_ctx* ctx, int nb) {
         CK(cudaMemcpyAsync(ctx->herr, ctx->bted_engine.err, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     ctx->bted_engine.collect();
+    big_k4_resolve(ctx);                             // K4 of large batch TEDs (winners updated in place)
     if (ctx->k4b.pending) {                          // K4 of small batch TEDs
         ctx->k4b.pending = false;
         auto& b = ctx->k4b;
@@ -1547,8 +1579,10 @@ bted_status batch_range_finish(bted_ctx* ctx, int nb) {
 }
 
 // Alg. 2 l.5-6 on device winners[0..n): returns count, out_idx host [count].
+// distinct: the n winners are known to be n distinct valid indices (one batch TED's
+// picks), so |X_U| = n without a host round trip
 bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, int32_t m, float mu,
-                         int64_t* out_idx, int32_t* out_count) {
+                         int64_t* out_idx, int32_t* out_count, bool distinct = false) {
     Nvtx nvtx_("bted union + merge (Alg. 2 l.5-6)");
     cudaStream_t st = ctx->stream;
     grow(ctx->u32a, ctx->u32acap, (size_t)n);
@@ -1559,20 +1593,27 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
         grow(ctx->bted_engine.err, ctx->bted_engine.errcap, 1);
         CK(cudaMemsetAsync(ctx->bted_engine.err, 0, sizeof(int), st));
     }
-    bted::i64_to_u32_kernel<<<g, 256, 0, st>>>(winners_dev, n, ctx->N, ctx->u32a, ctx->bted_engine.err);
-    LAUNCHED(1);
-    size_t need = 0, need2 = 0;
-    const int nbits = 32;   // padding (0xFFFFFFFF) must sort last
-    CK(cub::DeviceRadixSort::SortKeys(nullptr, need, ctx->u32a, ctx->u32b, (int)n, 0, nbits, st));
-    CK(cub::DeviceSelect::Unique(nullptr, need2, ctx->u32b, ctx->u32a, ctx->count_dev, (int)n, st));
-    cub_reserve(ctx, std::max(need, need2));
-    size_t cap = ctx->cub_cap;
-    CK(cub::DeviceRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->u32a, ctx->u32b, (int)n, 0, nbits, st));
-    cap = ctx->cub_cap;
-    CK(cub::DeviceSelect::Unique(ctx->cub_tmp, cap, ctx->u32b, ctx->u32a, ctx->count_dev, (int)n, st));
-    bted::drop_pad_kernel<<<1, 1, 0, st>>>(ctx->u32a, ctx->count_dev);
-    LAUNCHED(1);
-    int nu = 0;
+    if (n <= bted::kUnionMax) {                           // one CTA: sort + unique + drop padding
+        bted::union_small_kernel<<<1, bted::kUnionThreads, 0, st>>>(winners_dev, (int)n, ctx->N, ctx->u32a,
+                                                                    ctx->count_dev, ctx->bted_engine.err);
+        LAUNCHED(1);
+    } else {
+        bted::i64_to_u32_kernel<<<g, 256, 0, st>>>(winners_dev, n, ctx->N, ctx->u32a, ctx->bted_engine.err);
+        LAUNCHED(1);
+        size_t need = 0, need2 = 0;
+        const int nbits = 32;   // padding (0xFFFFFFFF) must sort last
+        CK(cub::DeviceRadixSort::SortKeys(nullptr, need, ctx->u32a, ctx->u32b, (int)n, 0, nbits, st));
+        CK(cub::DeviceSelect::Unique(nullptr, need2, ctx->u32b, ctx->u32a, ctx->count_dev, (int)n, st));
+        cub_reserve(ctx, std::max(need, need2));
+        size_t cap = ctx->cub_cap;
+        CK(cub::DeviceRadixSort::SortKeys(ctx->cub_tmp, cap, ctx->u32a, ctx->u32b, (int)n, 0, nbits, st));
+        cap = ctx->cub_cap;
+        CK(cub::DeviceSelect::Unique(ctx->cub_tmp, cap, ctx->u32b, ctx->u32a, ctx->count_dev, (int)n, st));
+        bted::drop_pad_kernel<<<1, 1, 0, st>>>(ctx->u32a, ctx->count_dev);
+        LAUNCHED(1);
+    }
+    int nu = (int)n;
+    if (!distinct || ctx->k4b.pending || n > bted::kUnionMax) {
     CK(cudaMemcpyAsync(&nu, ctx->count_dev, sizeof(int), cudaMemcpyDeviceToHost, st));
     CK(cudaMemcpyAsync(ctx->herr, ctx->bted_engine.err, sizeof(int), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));                        // |X_U| sizes the merge TED
@@ -1582,6 +1623,10 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
         return BTED_EINVAL;
     }
     ctx->bted_engine.collect();
+    if (big_k4_resolve(ctx)) {                            // K4 of the large batch TEDs, decided here
+        ctx->k4b.changed = true;
+        return merge_device(ctx, winners_dev, n, m, mu, out_idx, out_count, distinct);   // the union changed
+    }
     if (ctx->k4b.pending) {                               // K4 of the small batch TEDs, decided here
         ctx->k4b.pending = false;
         auto& b = ctx->k4b;
@@ -1593,8 +1638,9 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
                 LAUNCHED(1);
             }
             b.changed = true;
-            return merge_device(ctx, winners_dev, n, m, mu, out_idx, out_count);   // the union changed
+            return merge_device(ctx, winners_dev, n, m, mu, out_idx, out_count, distinct);   // the union changed
         }
+    }
     }
     if (nu < 1) { set_error("empty union"); return BTED_ENUMERIC; }
     const int32_t mm = std::min<int32_t>(m, nu);          // reading A12
@@ -1612,6 +1658,10 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
             bted::map_winners_kernel<<<(mm + 127) / 128, 128, 0, st>>>(ctx->mkeys, mm, ctx->u32a, ctx->out_dev);
             LAUNCHED(1);
             bted_status s = finish_keys(ctx, ctx->bted_engine, ctx->mkeys, mm, out_idx, nullptr, ctx->out_dev);
+            if (s == BTED_OK && big_k4_resolve(ctx)) {    // (fast path) a batch pick changed: redo l.5-6
+                ctx->k4b.changed = true;
+                return merge_device(ctx, winners_dev, n, m, mu, out_idx, out_count, distinct);
+            }
             if (s == BTED_OK && small_k4_refine(ctx, st, ctx->Xb, 1, nu, ctx->d, mm, mu, ctx->mkeys, T.err)) {
                 bted::map_winners_kernel<<<(mm + 127) / 128, 128, 0, st>>>(ctx->mkeys, mm, ctx->u32a,
                                                                          ctx->out_dev);
@@ -1629,6 +1679,10 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
     bted::map_winners_kernel<<<(mm + 127) / 128, 128, 0, st>>>(ctx->mkeys, mm, ctx->u32a, ctx->out_dev);
     LAUNCHED(1);
     bted_status s = finish_keys(ctx, ctx->bted_engine, ctx->mkeys, mm, out_idx, nullptr, ctx->out_dev);
+    if (s == BTED_OK && big_k4_resolve(ctx)) {            // (fast path) a batch pick changed: redo l.5-6
+        ctx->k4b.changed = true;
+        return merge_device(ctx, winners_dev, n, m, mu, out_idx, out_count, distinct);
+    }
     if (s == BTED_OK) *out_count = mm;
     return s;
 }
@@ -2460,7 +2514,7 @@ bted_status md_run_batches(bted_ctx* ctx, int64_t M, int32_t m, float mu, int64_
         CK(cudaMemcpyAsync(out_batch_idx, md.wall, sizeof(int64_t) * (size_t)B * m, cudaMemcpyDeviceToHost,
                            ctx->stream));
     }
-    return merge_device(ctx, md.wall, (int64_t)B * m, m, mu, out_idx, out_count);
+    return merge_device(ctx, md.wall, (int64_t)B * m, m, mu, out_idx, out_count, B == 1);
 }
 
 }  // namespace
@@ -2597,7 +2651,7 @@ bted_status bted_run_batches(bted_ctx* ctx, int64_t M, int32_t m, float mu, int6
         if (out_batch_idx)
             CK(cudaMemcpyAsync(out_batch_idx, ctx->winners, sizeof(int64_t) * (size_t)nb * m,
                                cudaMemcpyDeviceToHost, ctx->stream));
-        bted_status s = merge_device(ctx, ctx->winners, (int64_t)nb * m, m, mu, out_idx, out_count);
+        bted_status s = merge_device(ctx, ctx->winners, (int64_t)nb * m, m, mu, out_idx, out_count, nb == 1);
         if (s == BTED_OK && out_batch_idx && ctx->k4b.changed) {   // batch K4 changed winners after the copy
             CK(cudaMemcpyAsync(out_batch_idx, ctx->winners, sizeof(int64_t) * (size_t)nb * m,
                                cudaMemcpyDeviceToHost, ctx->stream));
@@ -2904,6 +2958,7 @@ void bted_destroy(bted_ctx* ctx) {
                         ctx->ridx, ctx->rWt, ctx->rsc, ctx->rmask, ctx->bkeys, ctx->bsflags, ctx->bncand, ctx->bcand, ctx->sks, ctx->scnt,
                         ctx->ktop2, ctx->kflags, ctx->kcand, ctx->kncand, ctx->knflag, ctx->kforced};
         if (ctx->k4pin) cudaFreeHost(ctx->k4pin);
+        if (ctx->bfpin) cudaFreeHost(ctx->bfpin);
         for (void* b : bufs) if (b) cudaFree(b);
         if (ctx->own_X && ctx->X) cudaFree(ctx->X);
         if (ctx->hkeys) cudaFreeHost(ctx->hkeys);

@@ -49,6 +49,74 @@ __global__ void i64_to_u32_kernel(const int64_t* __restrict__ in, int64_t n, int
     }
 }
 
+// Alg. 2 l.5 for up to kUnionMax winners in ONE CTA (replaces the radix sort + unique
+// + drop-padding launches): X_U = sorted unique(winners), negative entries are padding,
+// entries >= N flag kBadWinner and are dropped.  Bitonic sort in shared memory, then a
+// block-wide scan compacts the first occurrence of every index.
+constexpr int kUnionMax = 4096;
+constexpr int kUnionThreads = 1024;
+__global__ void __launch_bounds__(kUnionThreads)
+union_small_kernel(const int64_t* __restrict__ w, int n, int64_t N, uint32_t* __restrict__ out,
+                   int* __restrict__ count, int* __restrict__ err) {
+    __shared__ uint32_t key[kUnionMax];
+    __shared__ int wsum[kUnionThreads / 32];
+    const int tid = threadIdx.x;
+    int np = 1;
+    while (np < n) np <<= 1;
+    for (int i = tid; i < np; i += kUnionThreads) {
+        uint32_t k = 0xFFFFFFFFu;
+        if (i < n) {
+            const int64_t v = w[i];
+            if (v >= N) atomicOr(err, 16);                  // kBadWinner
+            if (v >= 0 && v < N) k = (uint32_t)v;
+        }
+        key[i] = k;
+    }
+    __syncthreads();
+    for (int size = 2; size <= np; size <<= 1)
+        for (int stride = size >> 1; stride > 0; stride >>= 1) {
+            for (int q = tid; q < np; q += kUnionThreads) {
+                const int p = q ^ stride;
+                if (p > q) {
+                    const bool up = (q & size) == 0;
+                    const uint32_t a = key[q], c = key[p];
+                    if ((a > c) == up) { key[q] = c; key[p] = a; }
+                }
+            }
+            __syncthreads();
+        }
+    // each thread owns 4 consecutive slots: keep = first occurrence and not padding
+    uint32_t kv[4];
+    int keep[4], cnt = 0;
+#pragma unroll
+    for (int x = 0; x < 4; ++x) {
+        const int i = 4 * tid + x;
+        kv[x] = i < np ? key[i] : 0xFFFFFFFFu;
+        keep[x] = i < np && kv[x] != 0xFFFFFFFFu && (i == 0 || key[i - 1] != kv[x]);
+        cnt += keep[x];
+    }
+    // exclusive scan of cnt over the block (warp shuffles, then the warp totals in order)
+    const int lane = tid & 31, wi = tid >> 5;
+    int incl = cnt;
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        const int o = __shfl_up_sync(0xffffffffu, incl, off);
+        if (lane >= off) incl += o;
+    }
+    if (lane == 31) wsum[wi] = incl;
+    __syncthreads();
+    int base = 0, total = 0;
+    for (int q = 0; q < kUnionThreads / 32; ++q) {
+        if (q < wi) base += wsum[q];
+        total += wsum[q];
+    }
+    int pos = base + incl - cnt;
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+        if (keep[x]) out[pos++] = kv[x];
+    if (tid == 0) *count = total;
+}
+
 // drop the padding value from the end of the unique list
 __global__ void drop_pad_kernel(const uint32_t* __restrict__ uniq, int* __restrict__ count) {
     const int c = *count;
