@@ -512,7 +512,8 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
         bted::tc::gram_tc_kernel<<<g, bted::tc::kTcThreads, bted::tc::kTileSmemBytes, T.stream>>>(
             T.opA, T.xnrm, (int32_t)N, gamma, T.K[0], nT, T.xmax);
         // the accuracy guard's fallback (exits at once when the tensor-core Gram was written)
-        bted::pk::gram_tile2_kernel<16, false, 4><<<(unsigned)tiles, bted::pk::kConsumers, 0, T.stream>>>(
+        bted::pk::gram_tile2_kernel<16, false, 4><<<(unsigned)std::min<int64_t>(tiles, (int64_t)4 * num_sms()),
+                                                     bted::pk::kConsumers, 0, T.stream>>>(
             X, (int32_t)N, d, gamma, T.K[0], nT, 0, 1, T.xmax);
         LAUNCHED(6);
     } else if (d <= 16) {
@@ -1333,6 +1334,20 @@ void launch_small(const float* X, int ninst, int64_t N, int32_t d, float gamma, 
     // the smallest cluster whose CTAs also hold the staged features, if the
     // ninst clusters still fit on the SMs at once; else the smallest that fits
     const int C = small_cluster_used(ninst, N, d);
+    if (N <= 128 && d <= 32) {
+        // tiny TEDs (e.g. the one-batch merge of m = 64 points): one CTA per instance, rows in
+        // registers; top-2 keys in the cluster kernel's unit layout (nU units, unit 0 used)
+        const int nU = C * bted::sm::kWarps;
+        const int32_t lin = kernel == BTED_KERNEL_LINEAR ? 1 : 0;
+        if (N <= 64)
+            bted::sm::ted_tiny_kernel<64><<<ninst, 64, 0, st>>>(X, (int32_t)N, d, gamma, lin, m, mu, keys, err, top2,
+                                                                nU, forced, nforced);
+        else
+            bted::sm::ted_tiny_kernel<128><<<ninst, 128, 0, st>>>(X, (int32_t)N, d, gamma, lin, m, mu, keys, err, top2,
+                                                                  nU, forced, nforced);
+        LAUNCHED(1);
+        return;
+    }
     switch (C) {
         case 1: launch_small_c<1>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st, top2, forced, nforced); break;
         case 2: launch_small_c<2>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st, top2, forced, nforced); break;
@@ -1369,7 +1384,6 @@ void small_k4_launch(bted_ctx* ctx, cudaStream_t st, int ninst, int64_t N, int32
     const int nUb = small_cluster_used(ninst, N, d) * bted::sm::kWarps;
     if (ctx->k4pincap < (size_t)ninst) {
         if (ctx->k4pin) cudaFreeHost(ctx->k4pin);
-        if (ctx->bfpin) cudaFreeHost(ctx->bfpin);
         ctx->k4pin = nullptr; ctx->k4pincap = 0;
         CK(cudaHostAlloc(&ctx->k4pin, sizeof(int) * ninst, cudaHostAllocDefault));
         ctx->k4pincap = (size_t)ninst;

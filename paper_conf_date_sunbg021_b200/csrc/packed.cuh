@@ -751,8 +751,11 @@ gram_tile2_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma
     __shared__ __align__(16) float xj[T][kD + 1];
     const int tid = threadIdx.x, w = tid / kWarp, l = tid % kWarp;
     const float ng = -gamma;
+    // tiles kl = blockIdx.x, + gridDim.x, ... of this shard (one per CTA when the grid covers them all)
+    const int64_t nloc = (num_tiles(nT) - sr + sp - 1) / sp;
+    for (int64_t kl = blockIdx.x; kl < nloc; kl += gridDim.x) {
     int I, J;
-    tile_ij((int64_t)sr + (int64_t)sp * blockIdx.x, nT, I, J);
+    tile_ij((int64_t)sr + (int64_t)sp * kl, nT, I, J);
     for (int q = tid; q < T * kD; q += kConsumers) {
         const int r = q / kD, c = q % kD;
         const int gi = I * T + r, gj = J * T + r;
@@ -765,7 +768,7 @@ gram_tile2_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma
     unsigned long long y[kD];
 #pragma unroll
     for (int q = 0; q < kD; ++q) y[q] = pack2(xj[c0][q], xj[c0 + 1][q]);
-    float* tile = K + (int64_t)blockIdx.x * (T * T);
+    float* tile = K + kl * (T * T);
     const bool cv0 = J * T + c0 < N, cv1 = J * T + c0 + 1 < N;
     const int rbase = 32 * (w >> 1);                             // warps 2v, 2v+1: rows 32v .. 32v+31
 #pragma unroll 1
@@ -802,6 +805,8 @@ gram_tile2_kernel(const float* __restrict__ X, int32_t N, int32_t d, float gamma
             o.y = (rv && cv1) ? v1 : 0.f;
             __stcs(reinterpret_cast<float2*>(tile + (r + h) * T + c0), o);
         }
+    }
+    __syncthreads();                                             // xi2 / xj are refilled for the next tile
     }
 }
 
