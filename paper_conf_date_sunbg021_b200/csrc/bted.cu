@@ -1334,20 +1334,6 @@ void launch_small(const float* X, int ninst, int64_t N, int32_t d, float gamma, 
     // the smallest cluster whose CTAs also hold the staged features, if the
     // ninst clusters still fit on the SMs at once; else the smallest that fits
     const int C = small_cluster_used(ninst, N, d);
-    if (N <= 128 && d <= 32) {
-        // tiny TEDs (e.g. the one-batch merge of m = 64 points): one CTA per instance, rows in
-        // registers; top-2 keys in the cluster kernel's unit layout (nU units, unit 0 used)
-        const int nU = C * bted::sm::kWarps;
-        const int32_t lin = kernel == BTED_KERNEL_LINEAR ? 1 : 0;
-        if (N <= 64)
-            bted::sm::ted_tiny_kernel<64><<<ninst, 64, 0, st>>>(X, (int32_t)N, d, gamma, lin, m, mu, keys, err, top2,
-                                                                nU, forced, nforced);
-        else
-            bted::sm::ted_tiny_kernel<128><<<ninst, 128, 0, st>>>(X, (int32_t)N, d, gamma, lin, m, mu, keys, err, top2,
-                                                                  nU, forced, nforced);
-        LAUNCHED(1);
-        return;
-    }
     switch (C) {
         case 1: launch_small_c<1>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st, top2, forced, nforced); break;
         case 2: launch_small_c<2>(X, ninst, (int32_t)N, d, gamma, kernel, m, mu, keys, err, st, top2, forced, nforced); break;

@@ -284,107 +284,3 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
 }  // namespace sm
 }  // namespace bted
 
-namespace bted {
-namespace sm {
-
-// ------------------------------------------------------------------ tiny TEDs (N <= 128)
-// The merge TED of a one-batch BTED (|X_U| = m = 64 points) and other tiny
-// candidate sets: one CTA of kCols threads per instance, thread i owns row i of
-// K in registers (Alg. 1 on N <= kCols points).  Per step: the pivot row goes
-// through shared memory (one barrier), every thread deflates its own row (the
-// K2 instruction, deflate1), sums its squared entries in column order (two
-// interleaved chains, combined in a fixed order: the same for every row, so
-// exact duplicates score bitwise equal), scores, and the CTA's masked argmax
-// (ties: lowest index) is a warp max + one barrier.  No cluster, no DSMEM; the
-// Gram entries are those of the cluster kernel (same operation sequence).
-// K4: unit 0 of top2[inst][t][nU] holds the CTA's best two keys, the other
-// units stay 0 (the layout of the cluster kernel's warps, so the same check).
-template <int kCols>
-__global__ void __launch_bounds__(kCols)
-ted_tiny_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float gamma, int32_t linear, int32_t m,
-                float mu, unsigned long long* __restrict__ keys_all, int* __restrict__ err,
-                unsigned long long* __restrict__ top2_all, int32_t nU, const unsigned long long* __restrict__ forced,
-                int32_t nforced) {
-    constexpr int kW = kCols / 32;
-    __shared__ float Xs[kCols * 33];                  // features, row stride d | 1 (d <= 32)
-    __shared__ float piv[kCols];
-    __shared__ unsigned long long wb1[kW], wb2[kW];
-    const int inst = blockIdx.x, i = threadIdx.x, l = i % 32, w = i / 32;
-    const float* __restrict__ X = Xall + (int64_t)inst * N * d;
-    unsigned long long* keys_out = keys_all + (int64_t)inst * m;
-    unsigned long long* top2 = top2_all ? top2_all + (int64_t)inst * m * nU * 2 : nullptr;
-    const int xs = d | 1;
-    for (int q = i; q < N * d; q += kCols) Xs[(q / d) * xs + q % d] = X[q];
-    if (top2) for (int q = i; q < m * nU * 2; q += kCols) top2[q] = 0ull;
-    __syncthreads();
-    const bool valid = i < N;
-    const float ng = -gamma;
-    float row[kCols];
-#pragma unroll
-    for (int j = 0; j < kCols; ++j) {
-        float v = 0.f;
-        if (valid && j < N) {
-            float a = 0.f;
-            for (int k = 0; k < d; ++k) {
-                const float xi = Xs[i * xs + k], xj = Xs[j * xs + k];
-                if (linear) a = __fmaf_rn(xi, xj, a);
-                else { const float df = __fsub_rn(xi, xj); a = __fmaf_rn(df, df, a); }
-            }
-            v = linear ? a : expf(__fmul_rn(ng, a));
-        }
-        row[j] = v;
-    }
-    bool sel = false;
-    // the CTA's best two keys of this thread's row score; returns the best (ties: lowest index)
-    auto argmax = [&](unsigned long long key, int t) -> unsigned long long {
-        unsigned long long b1 = key, b2 = 0ull;
-#pragma unroll
-        for (int off = 16; off > 0; off >>= 1)
-            top2_merge(b1, b2, __shfl_xor_sync(0xffffffffu, b1, off), __shfl_xor_sync(0xffffffffu, b2, off));
-        if (l == 0) { wb1[w] = b1; wb2[w] = b2; }
-        __syncthreads();
-        unsigned long long c1 = wb1[0], c2 = wb2[0];
-#pragma unroll
-        for (int q = 1; q < kW; ++q) top2_merge(c1, c2, wb1[q], wb2[q]);
-        if (top2 && i == 0) { top2[(int64_t)t * nU * 2] = c1; top2[(int64_t)t * nU * 2 + 1] = c2; }
-        return c1;
-    };
-    auto score = [&](int t) -> unsigned long long {
-        float g0 = 0.f, g1 = 0.f;                         // two chains: even / odd columns, then g0 + g1
-#pragma unroll
-        for (int j = 0; j < kCols; j += 2) {
-            g0 = __fmaf_rn(row[j], row[j], g0);
-            g1 = __fmaf_rn(row[j + 1], row[j + 1], g1);
-        }
-        const float g = __fadd_rn(g0, g1);
-        float kii = 0.f;
-#pragma unroll
-        for (int j = 0; j < kCols; ++j) if (j == i) kii = row[j];
-        const unsigned long long k = valid ? score_key(g, kii, mu, (uint32_t)i, sel, err) : 0ull;
-        return argmax(k, t);
-    };
-    unsigned long long best = score(0);
-    if (forced && 0 < nforced) best = forced[0];          // K4 re-run: preset (flagged) picks
-    for (int t = 1; t < m; ++t) {
-        if (i == 0) keys_out[t - 1] = best;
-        if (best == 0ull) { if (i == 0) atomicOr(err, 2); return; }
-        const int s = (int)key_index(best);
-        if (i == s) {
-            sel = true;
-#pragma unroll
-            for (int j = 0; j < kCols; ++j) piv[j] = row[j];
-        }
-        __syncthreads();                                  // pivot row published (wb1/wb2 free as well)
-        const float a = valid ? piv[i] : 0.f;             // K[i][s] = K[s][i] (bit-symmetric)
-        const float inv_c = __frcp_rn(__fadd_rn(piv[s], mu));
-#pragma unroll
-        for (int j = 0; j < kCols; ++j) row[j] = deflate1(row[j], a, piv[j], inv_c);
-        __syncthreads();                                  // everyone read piv before the next pivot write
-        best = score(t);
-        if (forced && t < nforced) best = forced[t];
-    }
-    if (i == 0) keys_out[m - 1] = best;
-}
-
-}  // namespace sm
-}  // namespace bted
