@@ -2556,7 +2556,11 @@ bted_status bted_select(bted_ctx* ctx, int32_t m, float mu, int64_t* out_idx, fl
     if (!ctx || !out_idx) { set_error("null argument"); return BTED_EINVAL; }
     if (ctx->is_shard || ctx->is_ishard) { set_error("bted_select on a shard context"); return BTED_EINVAL; }
     if (m < 1 || m > ctx->N || !mu_ok(mu)) { set_error("need 1 <= m <= N and mu > 0 finite"); return BTED_EINVAL; }
-    if (ctx->md) return guarded(ctx, [&]() { return md_select(ctx, m, mu, out_idx, out_score); });
+    // several devices: shard the candidate set -- unless it is small enough for the one-kernel
+    // cluster TED (nothing to gain from sharding) or has fewer Gram tiles / rows than devices
+    if (ctx->md && !use_small(ctx->params.flags, ctx->N) &&
+        bted::pk::num_tiles((int)((ctx->N + bted::pk::T - 1) / bted::pk::T)) >= ctx->md->P && ctx->N >= ctx->md->P)
+        return guarded(ctx, [&]() { return md_select(ctx, m, mu, out_idx, out_score); });
     return guarded(ctx, [&]() -> bted_status {
         Ted& T = ctx->ted;
         if (use_small(ctx->params.flags, ctx->N)) {

@@ -188,3 +188,16 @@ def test_select_row_bands_k4_near_ties():
         idx, sc = many.select(120, MU)
         st = L.bted_get_stats(many.ctx)
     check_ted(idx, sc, dense.ted(X, g, MU, 120, forced=idx), "bands-k4", gap_exact=GAP_K4)
+
+
+def test_small_candidate_sets_are_not_sharded():
+    """A candidate set the one-kernel cluster TED handles (N <= ~940), or one with
+    fewer Gram tiles than devices, runs on the first device alone: bitwise the
+    single-device selection."""
+    for N in (300, 900):
+        X = knob(N, seed=N)
+        g = median_gamma(X, N)
+        with bt.CandidateSet(X, g) as one, bt.CandidateSet(X, g, num_devices=4, flags=LOOP) as many:
+            a, sa = one.select(32, MU)
+            b, sb = many.select(32, MU)
+        assert np.array_equal(a, b) and np.array_equal(sa.view(np.uint32), sb.view(np.uint32))
