@@ -136,6 +136,27 @@ __global__ void __launch_bounds__(kThreads) prep_kernel(const float* __restrict_
 
 // ---------------------------------------------------------------- tcgen05 helpers
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+// paired fp32 arithmetic (one instruction for two IEEE round-to-nearest operations)
+__device__ __forceinline__ unsigned long long f2pack(float lo, float hi) {
+    return ((unsigned long long)__float_as_uint(hi) << 32) | __float_as_uint(lo);
+}
+__device__ __forceinline__ float f2lo(unsigned long long v) { return __uint_as_float((uint32_t)v); }
+__device__ __forceinline__ float f2hi(unsigned long long v) { return __uint_as_float((uint32_t)(v >> 32)); }
+__device__ __forceinline__ unsigned long long f2add(unsigned long long a, unsigned long long b) {
+    unsigned long long d;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+    return d;
+}
+__device__ __forceinline__ unsigned long long f2sub(unsigned long long a, unsigned long long b) {
+    unsigned long long d;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+    return d;
+}
+__device__ __forceinline__ unsigned long long f2mul(unsigned long long a, unsigned long long b) {
+    unsigned long long d;
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+    return d;
+}
 // 2^x on the SFU (MUFU.EX2); the rounding of the scaled argument -g log2(e) d2 adds a
 // relative error ~ g d2 ulp, inside pin C1's (1 + g d2) factor
 __device__ __forceinline__ float ex2_approx(float x) {
@@ -363,12 +384,18 @@ gram_tc_kernel(const uint8_t* __restrict__ opA, const float* __restrict__ nrm,
                     float dv[16], ev[16];
                     tmem_ld16(tbase + lb + (uint32_t)(c0 + cc), dv);
                     tmem_ld16(tbase + T + lb + (uint32_t)(c0 + cc), ev);
+                    // d2 = (n_r + n_c) - (D + D'), two columns per f32x2 instruction (the same IEEE
+                    // operations as the scalar form, so S and the norms keep their symmetry)
                     float o[16];
+                    const unsigned long long ni2 = f2pack(ni, ni), g2 = f2pack(ngl2e, ngl2e);
 #pragma unroll
-                    for (int q = 0; q < 16; ++q) {
-                        float d2 = __fsub_rn(__fadd_rn(ni, nj[c0 + cc + q]), __fadd_rn(dv[q], ev[q]));
-                        d2 = fmaxf(d2, 0.f);
-                        o[q] = ex2_approx(__fmul_rn(ngl2e, d2));
+                    for (int q = 0; q < 16; q += 2) {
+                        const float2 njq = *reinterpret_cast<const float2*>(&nj[c0 + cc + q]);
+                        const unsigned long long sd = f2add(f2pack(dv[q], dv[q + 1]), f2pack(ev[q], ev[q + 1]));
+                        const unsigned long long d2 = f2sub(f2add(ni2, f2pack(njq.x, njq.y)), sd);
+                        const unsigned long long y = f2mul(g2, f2pack(fmaxf(f2lo(d2), 0.f), fmaxf(f2hi(d2), 0.f)));
+                        o[q] = ex2_approx(f2lo(y));
+                        o[q + 1] = ex2_approx(f2hi(y));
                     }
                     if (edge) {
 #pragma unroll
