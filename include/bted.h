@@ -208,6 +208,35 @@ bted_status bted_merge(bted_ctx* pool, const int64_t* winners, int64_t n,
 bted_status bted_sample_batches(int64_t P, int64_t M, int32_t B, uint64_t seed,
                                 int64_t* out);
 
+/* ---------------- Multi-GPU through one context (params.num_devices = G > 1) -------
+ * SURVEY 8(e), PAPER.md:150 ("stimulate the parallelism") and Alg. 2.
+ * One process drives GPUs [device, device + G) (BTED_FLAG_LOOPBACK: G logical
+ * devices on `device`, one stream -- the same kernels and exchange protocol);
+ * X is replicated on every device; peer access is enabled between them (without
+ * P2P only BTED_FLAG_NCCL works).
+ *   bted_run_batches: batch b of Alg. 2 runs on device b mod G (one host thread
+ *     per device, no exchange), the m winners of every batch are copied to
+ *     `device` (l.5) and the union + merge TED run there.  Results are bitwise
+ *     those of one device.
+ *   bted_select: the candidate set is sharded over P = G devices --
+ *     default: the implicit engine's packed Gram tiles k = p (mod P) on device p;
+ *       per step each device publishes its partial q = K l (a release counter in
+ *       its memory) and every device's score kernel sums the P partials in rank
+ *       order through peer loads (bitwise the same on every device);
+ *     BTED_FLAG_DENSE: row bands of the dense K; per step the pivot column slices
+ *       are gathered, the band maxima max-reduced, and with norm_mode = 1 the
+ *       bands' partial column norms summed (the literal column-norm exchange);
+ *     BTED_FLAG_NCCL: the q exchange through ncclAllReduce (libnccl.so.2 loaded at
+ *       run time; ncclCommInitAll over the P devices).
+ *     Candidate sets small enough for the one-kernel cluster TED, or with fewer
+ *     Gram tiles (rows) than devices, run on `device` alone.
+ *   Errors: BTED_ENCCL (the ctx is then poisoned) when an NCCL call or async error
+ *   fails, a collective exceeds BTED_NCCL_TIMEOUT_S (default 300 s; the
+ *   communicators are aborted), or a device stops publishing its step (the other
+ *   devices' waits time out after BTED_PEER_TIMEOUT_MS, default 20000 ms).
+ *   bted_batch_teds / bted_merge / bted_shard_* / bted_ishard_* use `device` only.
+ */
+
 /* ---------------- row-sharded TED (one oversized batch over P GPUs) -------------
  * A shard context owns rows [row0, row1) of the N x N matrix K of the full
  * candidate set X (X is replicated: N x d).  The per-step exchange is done by
