@@ -360,15 +360,19 @@ void launch_step(Ted& T, int64_t N, int64_t row0, int64_t rows, int32_t t, float
 }
 
 // ---- packed layout (packed.cuh) ----
-int g_num_sms = 0;
+// (lazily initialised process-wide constants are atomics: the multi-GPU run_batches
+// calls them from one host thread per device)
+std::atomic<int> g_num_sms{0};
 int num_sms() {
-    if (!g_num_sms) {
+    int n = g_num_sms.load(std::memory_order_relaxed);
+    if (!n) {
         int dev = 0;
         cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
-        if (g_num_sms <= 0) g_num_sms = 148;
+        if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
+        cudaGetLastError();
+        g_num_sms.store(n, std::memory_order_relaxed);
     }
-    return g_num_sms;
+    return n;
 }
 // K2p configurations (scripts/k2p_variants.cu, profiles/r1/k2p_variants_*.txt):
 // default = one CTA per tile with 256-bit loads (k2p_ldg<4>, measured 6.40 /
@@ -435,7 +439,8 @@ unsigned tile_pass_grid(int64_t tiles) {
 // BTED_L2_KEEP_MB overrides.
 constexpr double kL2KeepFrac = 0.0;
 int l2_keep_tiles(int64_t tiles) {
-    static int64_t bytes = -1;
+    static std::atomic<int64_t> cached{-1};
+    int64_t bytes = cached.load(std::memory_order_relaxed);
     if (bytes < 0) {
         if (const char* e = std::getenv("BTED_L2_KEEP_MB")) {
             bytes = (int64_t)(std::atof(e) * 1048576.0);
@@ -446,6 +451,7 @@ int l2_keep_tiles(int64_t tiles) {
             cudaGetLastError();
             bytes = (int64_t)(kL2KeepFrac * l2);
         }
+        cached.store(bytes, std::memory_order_relaxed);
     }
     const int64_t tile_bytes = (int64_t)bted::pk::T * bted::pk::T * 4;
     return (int)std::min<int64_t>(tiles, std::max<int64_t>(0, bytes / tile_bytes));
@@ -538,7 +544,8 @@ bool capturing(cudaStream_t st) {
 // Grid of the persistent loop kernel: every CTA must be resident at once (grid
 // barriers), so the grid is the measured occupancy x SMs (0: cannot run).
 int loop_kernel_grid() {
-    static int g = -1;
+    static std::atomic<int> cached{-1};
+    int g = cached.load(std::memory_order_relaxed);
     if (g < 0) {
         int nb = 0;
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, bted::im::ted_loop_kernel, bted::im::kTPThreads,
@@ -546,6 +553,7 @@ int loop_kernel_grid() {
             nb = 0;
         cudaGetLastError();
         g = std::min(nb, bted::im::kTPBlocksPerSM) * num_sms();
+        cached.store(g, std::memory_order_relaxed);
     }
     return g;
 }

@@ -744,3 +744,19 @@ def test_large_131072_sampled_against_closed_form():
             cand = np.array([c for c in cand if c not in set(idx[:t].tolist())])
             assert cf.scores(cand).max() <= s64 * (1 + 1e-6)
         cf.add(idx[t])
+
+
+@pytest.mark.parametrize("B", [64, 70], ids=["one-cta-union-4096", "cub-union-4480"])
+def test_union_of_many_batches_both_paths(B):
+    """Alg. 2 l.5 with B * m winners at the one-CTA union's limit (4096) and above
+    it (the CUB sort + unique path): X_U is exactly the sorted unique winners and
+    the merge TED passes P2 against the oracle on a fresh Gram of X_U."""
+    P, M, m, seed = 20000, 256, 64, 31
+    X = knob(P, seed=12)
+    g = median_gamma(X, 12)
+    with bt.CandidateSet(X, g, num_batches=B, seed=seed) as pool:
+        sel, bidx = pool.run_batches(M, m, MU)
+    XU = np.unique(bidx.reshape(-1))
+    assert len(sel) == m and set(sel.tolist()) <= set(XU.tolist())
+    mpos = _positions(XU, sel)
+    check_ted(mpos, [], dense.ted(X[XU], g, MU, m, forced=mpos), f"union-{B}", gap_exact=GAP_K4)
