@@ -181,6 +181,17 @@ __device__ __forceinline__ void mma_bf16(uint32_t tmem_d, uint64_t adesc, uint64
 }
 
 
+// tcgen05.ld of 16 consecutive columns without the wait (several loads share one
+// tcgen05.wait::ld); the registers are valid only after tmem_wait_ld()
+__device__ __forceinline__ void tmem_ld16_async(uint32_t taddr, uint32_t (&r)[16]) {
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x16.b32 "
+                 "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+                   "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+                 : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, float (&v)[16]) {
     uint32_t r[16];
     asm volatile("tcgen05.ld.sync.aligned.32x32b.x16.b32 "
@@ -381,9 +392,13 @@ gram_tc_kernel(const uint8_t* __restrict__ opA, const float* __restrict__ nrm,
                 float* srow = stage + (size_t)r * kStageLd + 32 * hh;
 #pragma unroll
                 for (int cc = 0; cc < 32; cc += 16) {
+                    uint32_t du[16], eu[16];
+                    tmem_ld16_async(tbase + lb + (uint32_t)(c0 + cc), du);
+                    tmem_ld16_async(tbase + T + lb + (uint32_t)(c0 + cc), eu);
+                    tmem_wait_ld();                              // one wait for both accumulators
                     float dv[16], ev[16];
-                    tmem_ld16(tbase + lb + (uint32_t)(c0 + cc), dv);
-                    tmem_ld16(tbase + T + lb + (uint32_t)(c0 + cc), ev);
+#pragma unroll
+                    for (int q = 0; q < 16; ++q) { dv[q] = __uint_as_float(du[q]); ev[q] = __uint_as_float(eu[q]); }
                     // d2 = (n_r + n_c) - (D + D'), two columns per f32x2 instruction (the same IEEE
                     // operations as the scalar form, so S and the norms keep their symmetry)
                     float o[16];
