@@ -15,19 +15,31 @@
 // fp32 operands through bf16 tensor cores without losing precision: each
 // centred fp32 value is split exactly into three bf16 parts v = h + m + l
 // (8 + 8 + 8 significand bits), and the dot product is the sum of the six
-// MMAs m.m, h.l, l.h, h.m, m.h, h.h (the three dropped terms m.l, l.m, l.l
-// are below 2^-32 relative) -- products of bf16 are exact in fp32; the
-// smallest terms accumulate first.  The operands are prepared once per TED
-// (prep kernel) in the tensor cores' canonical K-major layout (no swizzle):
-// 8 x 8 core matrices of 128 B, k-chunks 128 B apart (LBO), 8-row groups
-// 1536 B apart (SBO), six 16-wide k-slices per block of 128 rows.
+// products h.l, l.h, m.m, h.m, m.h, h.h (the three dropped terms m.l, l.m, l.l
+// are below 2^-32 relative) -- products of bf16 are exact in fp32; the smallest
+// terms accumulate first.  ONE accumulator D = x'_I . x'_J^T, bit-symmetric by
+// construction: each cross term sits in a single MMA instruction with both of
+// its halves ([h | l] . [l | h] puts h_r l_c and l_r h_c in the same K = 16
+// reduction, features 0-7 or 8-15), so under r <-> c every instruction reduces
+// the same multiset of 16 products, and the tensor core's K = 16 reduction is a
+// symmetric function of its products (measured on B200: D == D^T bitwise, the
+// result independent of the operand's position in the tile and of the tile's
+// orientation, exact duplicate rows bitwise equal -- scripts/tc_sym_probe.cu).
+// The operands are prepared once per TED (prep kernel) in the tensor cores'
+// canonical K-major layout (no swizzle): 8 x 8 core matrices of 128 B, 8-row
+// groups 1536 B apart (SBO), twelve 8-wide k-chunks per row,
+//     0 h0-7  1 l0-7  2 h8-15  3 l8-15  4 m0-7  5 m8-15
+//     6 h0-7  7 m0-7  8 h8-15  9 m8-15  10 h0-7  11 h8-15,
+// and every MMA addresses its two k-chunks (A and B) through the descriptor's
+// start and leading byte offset (LBO), so one copy of the block serves both
+// operand arrangements.
 //
 // Per tile (I <= J): the two 24 KiB operand blocks arrive by TMA bulk copies
 // (mbarrier), one thread issues the six MMAs and commits them to an mbarrier,
 // eight warps read the accumulator (tcgen05.ld), form K and store it; the
-// next tile's copies overlap the epilogue.  Diagonal tiles store their upper
-// triangle mirrored, so the matrix is bit-symmetric by construction, and
-// K_ii = 1 exactly.
+// next tile's copies overlap the epilogue.  The same K function (kval2) serves
+// the recomputing tile pass (rc_pass.cuh), so the stored Gram and the
+// recomputed one are the same numbers.
 #pragma once
 #include <cstdint>
 #include <cuda_bf16.h>
@@ -40,9 +52,9 @@ namespace tc {
 using pk::T;
 constexpr int kThreads = 256;
 constexpr int kD = 16;                         // features per k-slice (d <= 16)
-constexpr int kSlices = 6;                     // the six split products
-constexpr int kK = kD * kSlices;               // 96 bf16 per row
-constexpr uint32_t kLBO = 128;                 // bytes between k-adjacent core matrices
+constexpr int kSlices = 6;                     // the six MMAs (K = 16 each)
+constexpr int kK = kD * kSlices;               // 96 bf16 per row (12 k-chunks of 8)
+constexpr uint32_t kChunk = 128;               // bytes of one 8 x 8 core matrix (k-chunk)
 constexpr uint32_t kSBO = (kK / 8) * 128;      // 1536: bytes between 8-row groups
 constexpr uint32_t kBlockBytes = (T / 8) * kSBO;   // 24576 per 128-row block
 
@@ -51,8 +63,13 @@ constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(T >
 
 // byte offset of element (row r, k) of a block in the canonical K-major layout
 __host__ __device__ __forceinline__ uint32_t op_offset(int r, int k) {
-    return (uint32_t)(r >> 3) * kSBO + (uint32_t)(k >> 3) * kLBO + (uint32_t)(r & 7) * 16u + (uint32_t)(k & 7) * 2u;
+    return (uint32_t)(r >> 3) * kSBO + (uint32_t)(k >> 3) * kChunk + (uint32_t)(r & 7) * 16u + (uint32_t)(k & 7) * 2u;
 }
+// MMA s: A = k-chunks (a0, a0 + 1), B = k-chunks (b0, b0 + blbo) of the block above
+//   s = 0, 1: [h | l] . [l | h]   2: [m] . [m]   3, 4: [h | m] . [m | h]   5: [h] . [h]
+__host__ __device__ __forceinline__ uint32_t mma_a0(int s) { return s == 0 ? 0u : s == 1 ? 2u : s == 2 ? 4u : s == 3 ? 6u : s == 4 ? 8u : 10u; }
+__host__ __device__ __forceinline__ uint32_t mma_b0(int s) { return s == 0 ? 1u : s == 1 ? 3u : s == 2 ? 4u : s == 3 ? 7u : s == 4 ? 9u : 10u; }
+__host__ __device__ __forceinline__ uint32_t mma_blbo(int s) { return s == 0 || s == 1 ? 5u : s == 3 ? 3u : s == 4 ? 2u : 1u; }
 
 // ---------------------------------------------------------------- prep
 // c = mean of the N rows (fixed-order partial sums: deterministic): any c is exact
@@ -104,8 +121,7 @@ __device__ __forceinline__ void split3(float v, __nv_bfloat16& h, __nv_bfloat16&
     l = __float2bfloat16_rn(r2);                                  // exact for normal v
 }
 
-// per row i (padding rows: 0): x' = x - c and its operand row, slices
-// [m, h, l, h, m, h] (the B arrangement is the same block with permuted slices)
+// per row i (padding rows: 0): x' = x - c and its operand row (the twelve k-chunks above)
 __global__ void __launch_bounds__(kThreads) prep_kernel(const float* __restrict__ X, int32_t N, int32_t d,
                                                        int nT, const float* __restrict__ c,
                                                        uint8_t* __restrict__ opA) {
@@ -120,18 +136,16 @@ __global__ void __launch_bounds__(kThreads) prep_kernel(const float* __restrict_
         if (i < N && k < d) v = __fsub_rn(X[i * d + k], c[k]);
         split3(v, h[k], m[k], l[k]);
     }
-    // slice s of a row = 16 bf16 = two 16-byte core-matrix rows (features 0-7, 8-15)
-    auto put = [&](uint8_t* base, int s, const __nv_bfloat16 (&v)[kD]) {
+    // k-chunk q of a row = 8 bf16 = one 16-byte core-matrix row
+    auto put = [&](int q, const __nv_bfloat16* v) {
+        uint4 u;
+        __nv_bfloat16* e = reinterpret_cast<__nv_bfloat16*>(&u);
 #pragma unroll
-        for (int kc = 0; kc < 2; ++kc) {
-            uint4 q;
-            __nv_bfloat16* e = reinterpret_cast<__nv_bfloat16*>(&q);
-#pragma unroll
-            for (int x = 0; x < 8; ++x) e[x] = v[8 * kc + x];
-            *reinterpret_cast<uint4*>(base + op_offset(r, s * kD + 8 * kc)) = q;
-        }
+        for (int x = 0; x < 8; ++x) e[x] = v[x];
+        *reinterpret_cast<uint4*>(a + op_offset(r, 8 * q)) = u;
     };
-    put(a, 0, m); put(a, 1, h); put(a, 2, l); put(a, 3, h); put(a, 4, m); put(a, 5, h);   // A: m h l h m h
+    put(0, h); put(1, l); put(2, h + 8); put(3, l + 8); put(4, m); put(5, m + 8);
+    put(6, h); put(7, m); put(8, h + 8); put(9, m + 8); put(10, h); put(11, h + 8);
 }
 
 // ---------------------------------------------------------------- tcgen05 helpers
@@ -165,10 +179,10 @@ __device__ __forceinline__ float ex2_approx(float x) {
     return y;
 }
 
-__device__ __forceinline__ uint64_t smem_desc(uint32_t saddr) {
+__device__ __forceinline__ uint64_t smem_desc(uint32_t saddr, uint32_t lbo) {
     uint64_t desc = 0;
     desc |= (uint64_t)((saddr >> 4) & 0x3FFFu);                  // start address
-    desc |= (uint64_t)((kLBO >> 4) & 0x3FFFu) << 16;             // leading (k) byte offset
+    desc |= (uint64_t)((lbo >> 4) & 0x3FFFu) << 16;              // leading (k) byte offset
     desc |= (uint64_t)((kSBO >> 4) & 0x3FFFu) << 32;             // stride (8-row group) byte offset
     desc |= (uint64_t)1 << 46;                                   // version 1 (sm_100)
     return desc;                                                 // base offset 0, SWIZZLE_NONE
@@ -204,16 +218,11 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, float (&v)[16]) {
     for (int q = 0; q < 16; ++q) v[q] = __uint_as_float(r[q]);
 }
 
-// ---------------------------------------------------------------- symmetric dot products
-// D = A_I . B_J^T and D' = B_I . A_J^T (two accumulators, TMEM columns [0, 128) and
-// [128, 256)).  D[r][c] = dot(A_r, B_c), D'[r][c] = dot(B_r, A_c) = dot(A_c, B_r)
-// (the same products in the same slice order), so S = D + D' is symmetric in (r, c)
-// BITWISE: S_cr adds the same two numbers in the other order.  Hence K is
-// bit-symmetric without mirroring, and exact duplicate points get bitwise-equal
-// rows.  The squared norms are S's own diagonal halves, n_r = S_rr / 2, so that
-// d2 = (n_r + n_c) - S_rc is exactly 0 for identical points (K = 1, like the
+// ---------------------------------------------------------------- the dot products
+// D = x'_I . x'_J^T in TMEM columns [tD, tD + 128) (one accumulator, bit-symmetric:
+// see the header).  The squared norms are D's own diagonal, n_r = D_rr, so that
+// d2 = (n_r + n_c) - 2 D_rc is exactly 0 for identical points (K = 1, like the
 // direct form).
-constexpr int kTmemCols = 2 * T;
 // Accuracy guard: the expansion's rounding is relative to the centred norms, so the
 // tensor-core Gram is used only when gamma * max_r n_r <= kGuard (the median-gamma
 // knob and uniform pools: ~1-2); otherwise (badly scaled data, a huge gamma) the
@@ -223,34 +232,46 @@ constexpr float kGuard = 4.f;
 __device__ __forceinline__ bool tc_ok(const int* nmax_bits, float gamma) {
     return __fmul_rn(gamma, __int_as_float(*nmax_bits)) <= kGuard;
 }
-
-// The B arrangement [m, l, h, m, h, h] is the A arrangement [m, h, l, h, m, h] with
-// its slices permuted (kPerm), so only A blocks are stored: B's slice s is A's
-// slice kPerm[s], addressed through the descriptor's start offset.
-__device__ __forceinline__ uint32_t perm_slice(int s) { return s == 1 ? 2u : s == 2 ? 1u : s == 3 ? 4u : s == 4 ? 3u : (uint32_t)s; }
-__device__ __forceinline__ void issue_sym_mmas(uint32_t tbase, uint32_t aI, uint32_t aJ) {
+__device__ __forceinline__ void issue_gram_mmas(uint32_t tD, uint32_t aI, uint32_t aJ) {
 #pragma unroll
-    for (int s = 0; s < kSlices; ++s)                          // D = A_I . B_J^T
-        mma_bf16(tbase, smem_desc(aI + 2 * s * kLBO), smem_desc(aJ + 2 * perm_slice(s) * kLBO), s > 0 ? 1u : 0u);
-#pragma unroll
-    for (int s = 0; s < kSlices; ++s)                          // D' = B_I . A_J^T
-        mma_bf16(tbase + T, smem_desc(aI + 2 * perm_slice(s) * kLBO), smem_desc(aJ + 2 * s * kLBO), s > 0 ? 1u : 0u);
+    for (int s = 0; s < kSlices; ++s)
+        mma_bf16(tD, smem_desc(aI + kChunk * mma_a0(s), kChunk), smem_desc(aJ + kChunk * mma_b0(s), kChunk * mma_blbo(s)),
+                 s > 0 ? 1u : 0u);
+}
+// K for two columns from their dot products D and t = n_r + n_c (f32x2: one instruction per
+// pair; the same IEEE operations per element as the scalar form, so symmetric inputs give
+// symmetric K):  d2 = t - 2 D (one rounding, fma),  K = 2^(-gamma log2(e) max(d2, 0)).
+// Every Gram entry of the tensor-core path -- stored (gram_tc_kernel) or recomputed in a
+// tile pass (rc_pass.cuh) -- is this function of (D_rc, n_r + n_c).
+__device__ __forceinline__ unsigned long long f2fma(unsigned long long a, unsigned long long b, unsigned long long c) {
+    unsigned long long d;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+    return d;
+}
+__device__ __forceinline__ void kval2(float D0, float D1, unsigned long long t2, unsigned long long g2, float& k0,
+                                      float& k1) {
+    const unsigned long long d2 = f2fma(f2pack(-2.f, -2.f), f2pack(D0, D1), t2);
+    const unsigned long long y = f2mul(g2, f2pack(fmaxf(f2lo(d2), 0.f), fmaxf(f2hi(d2), 0.f)));
+    k0 = ex2_approx(f2lo(y));
+    k1 = ex2_approx(f2hi(y));
 }
 
+template <int kCols = T>
 __device__ __forceinline__ void tmem_alloc(uint32_t* dst) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
-                 :: "r"(smem_u32(dst)), "n"(kTmemCols));
+                 :: "r"(smem_u32(dst)), "n"(kCols));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
 }
+template <int kCols = T>
 __device__ __forceinline__ void tmem_free(uint32_t base) {
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(base), "n"(kTmemCols));
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(base), "n"(kCols));
 }
 __device__ __forceinline__ void mma_commit(uint64_t* bar) {
     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
                  :: "r"(smem_u32(bar)) : "memory");
 }
 
-// n_r = S_rr / 2 for every row of every block (one CTA per block I: the diagonal tile's S)
+// n_r = D_rr for every row of every block (one CTA per block I: the diagonal tile's D)
 __global__ void __launch_bounds__(kThreads)
 gram_tc_norm_kernel(const uint8_t* __restrict__ opA, float* __restrict__ nrm, int* __restrict__ nmax_bits) {
     extern __shared__ __align__(1024) uint8_t smem[];            // [A_I]
@@ -275,26 +296,23 @@ gram_tc_norm_kernel(const uint8_t* __restrict__ opA, float* __restrict__ nrm, in
     if (tid == 0) {
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const uint32_t a = smem_u32(smem);
-        issue_sym_mmas(tbase, a, a);
+        issue_gram_mmas(tbase, a, a);
         mma_commit(&mmabar);
     }
     pk::mbar_wait(&mmabar, 0);
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     if (w < 4) {                                               // lane r = 32 w + lane needs column r
         const int r = 32 * w + lane;
-        float d0[16], d1[16], e0[16], e1[16];
+        float d0[16], d1[16];
         const uint32_t lb = (uint32_t)(32 * w) << 16;
         tmem_ld16(tbase + lb + (uint32_t)(32 * w), d0);
         tmem_ld16(tbase + lb + (uint32_t)(32 * w + 16), d1);
-        tmem_ld16(tbase + T + lb + (uint32_t)(32 * w), e0);
-        tmem_ld16(tbase + T + lb + (uint32_t)(32 * w + 16), e1);
-        float dv = 0.f, ev = 0.f;
+        float n = 0.f;
 #pragma unroll
         for (int q = 0; q < 16; ++q) {
-            if (lane == q) { dv = d0[q]; ev = e0[q]; }
-            if (lane == 16 + q) { dv = d1[q]; ev = e1[q]; }
+            if (lane == q) n = d0[q];
+            if (lane == 16 + q) n = d1[q];
         }
-        const float n = __fmul_rn(0.5f, __fadd_rn(dv, ev));
         nrm[(int64_t)I * T + r] = n;
         atomicMax(nmax_bits, __float_as_int(fmaxf(n, 0.f)));
     }
@@ -309,9 +327,9 @@ gram_tc_norm_kernel(const uint8_t* __restrict__ opA, float* __restrict__ nrm, in
 // consecutive tiles share the row block I (its operand block is reloaded only when
 // I changes).  As soon as a tile's MMAs completed, the operand copies of the next
 // tile are issued (cp.async.bulk), overlapping this tile's epilogue; the next
-// tile's MMAs are issued as soon as the accumulators are read out, overlapping the
-// last stores.  Epilogue, in two column halves: warp w reads TMEM lanes 32 (w % 4)
-// .. +31 (tile rows) and 32 of the columns 64 (w / 4) .. +63 of D and D', forms K
+// tile's MMAs (into the other of two TMEM accumulators) are issued half-way through
+// this tile's epilogue.  Epilogue, in two column halves: warp w reads TMEM lanes 32 (w % 4)
+// .. +31 (tile rows) and 32 of the columns 64 (w / 4) .. +63 of D, forms K
 // into a padded staging buffer (128 rows x 64 columns), and the CTA writes the half
 // tile with coalesced 128-byte row segments; tiles on the ragged edge zero the
 // padding.  The other CTA on the SM computes while this one stores.
@@ -336,7 +354,7 @@ gram_tc_kernel(const uint8_t* __restrict__ opA, const float* __restrict__ nrm,
     const int64_t ntiles = pk::num_tiles(nT);
     const int64_t per = (ntiles + gridDim.x - 1) / gridDim.x;
     const int64_t k0 = (int64_t)blockIdx.x * per, k1 = k0 + per < ntiles ? k0 + per : ntiles;
-    if (w == 0) tmem_alloc(&tmem_base);
+    if (w == 0) tmem_alloc<2 * T>(&tmem_base);
     if (tid == 0) {
         pk::mbar_init(&ldbar, 1);
         pk::mbar_init(&mmabar, 1);
@@ -360,14 +378,14 @@ gram_tc_kernel(const uint8_t* __restrict__ opA, const float* __restrict__ nrm,
         loadedI = I_;
     };
     uint32_t ldph = 0u, mph = 0u;
-    auto mma = [&]() {
+    auto mma = [&](int b) {
         pk::mbar_wait(&ldbar, ldph);
         ldph ^= 1u;
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        issue_sym_mmas(tbase, smem_u32(smem), smem_u32(smem + kBlockBytes));
+        issue_gram_mmas(tbase + (uint32_t)(b * T), smem_u32(smem), smem_u32(smem + kBlockBytes));
         mma_commit(&mmabar);
     };
-    if (tid == 0 && k0 < k1) { issue(I, J, 0); mma(); }
+    if (tid == 0 && k0 < k1) { issue(I, J, 0); mma(0); }
     const int q4 = w & 3, hh = w >> 2;                             // TMEM lane quarter, column half
     const int r = 32 * q4 + lane;
     const uint32_t lb = (uint32_t)(32 * q4) << 16;
@@ -384,6 +402,8 @@ gram_tc_kernel(const uint8_t* __restrict__ opA, const float* __restrict__ nrm,
         const bool edge = (I + 1) * T > N || (J + 1) * T > N;
         const bool rowv = I * T + r < N;
         float* tile = K + k * (int64_t)(T * T);
+        const uint32_t tD = tbase + (uint32_t)(b * T) + lb;
+        const unsigned long long g2 = f2pack(ngl2e, ngl2e);
 #pragma unroll 1
         for (int half = 0; half < 2; ++half) {
             // part 1: 32 columns per warp, TMEM -> K values -> staging columns 32 hh .. +31
@@ -392,25 +412,15 @@ gram_tc_kernel(const uint8_t* __restrict__ opA, const float* __restrict__ nrm,
                 float* srow = stage + (size_t)r * kStageLd + 32 * hh;
 #pragma unroll
                 for (int cc = 0; cc < 32; cc += 16) {
-                    uint32_t du[16], eu[16];
-                    tmem_ld16_async(tbase + lb + (uint32_t)(c0 + cc), du);
-                    tmem_ld16_async(tbase + T + lb + (uint32_t)(c0 + cc), eu);
-                    tmem_wait_ld();                              // one wait for both accumulators
-                    float dv[16], ev[16];
-#pragma unroll
-                    for (int q = 0; q < 16; ++q) { dv[q] = __uint_as_float(du[q]); ev[q] = __uint_as_float(eu[q]); }
-                    // d2 = (n_r + n_c) - (D + D'), two columns per f32x2 instruction (the same IEEE
-                    // operations as the scalar form, so S and the norms keep their symmetry)
+                    uint32_t du[16];
+                    tmem_ld16_async(tD + (uint32_t)(c0 + cc), du);
+                    tmem_wait_ld();
                     float o[16];
-                    const unsigned long long ni2 = f2pack(ni, ni), g2 = f2pack(ngl2e, ngl2e);
 #pragma unroll
                     for (int q = 0; q < 16; q += 2) {
                         const float2 njq = *reinterpret_cast<const float2*>(&nj[c0 + cc + q]);
-                        const unsigned long long sd = f2add(f2pack(dv[q], dv[q + 1]), f2pack(ev[q], ev[q + 1]));
-                        const unsigned long long d2 = f2sub(f2add(ni2, f2pack(njq.x, njq.y)), sd);
-                        const unsigned long long y = f2mul(g2, f2pack(fmaxf(f2lo(d2), 0.f), fmaxf(f2hi(d2), 0.f)));
-                        o[q] = ex2_approx(f2lo(y));
-                        o[q + 1] = ex2_approx(f2hi(y));
+                        kval2(__uint_as_float(du[q]), __uint_as_float(du[q + 1]),
+                              f2add(f2pack(ni, ni), f2pack(njq.x, njq.y)), g2, o[q], o[q + 1]);
                     }
                     if (edge) {
 #pragma unroll
@@ -423,9 +433,9 @@ gram_tc_kernel(const uint8_t* __restrict__ opA, const float* __restrict__ nrm,
                         dst[q] = make_float4(o[4 * q], o[4 * q + 1], o[4 * q + 2], o[4 * q + 3]);
                 }
             }
-            if (half == 1) asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-            __syncthreads();                                       // staging half complete (half 1: TMEM read out)
-            if (half == 1 && tid == 0 && k + 1 < k1) mma();        // MMA(k+1) overlaps the stores below
+            asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+            __syncthreads();                                       // staging half complete
+            if (half == 0 && tid == 0 && k + 1 < k1) mma(b ^ 1);   // MMA(k+1): the other accumulator
             // part 2: rows in pairs per warp instruction: lanes 0-15 row 2i, 16-31 row 2i+1;
             // lane group g = lane % 16: segment g / 8 (tile columns 64 (g / 8) + 32 half ..), 16 B each
 #pragma unroll 2
@@ -441,7 +451,7 @@ gram_tc_kernel(const uint8_t* __restrict__ opA, const float* __restrict__ nrm,
     }
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
     __syncthreads();
-    if (w == 0) tmem_free(tbase);
+    if (w == 0) tmem_free<2 * T>(tbase);
 }
 
 }  // namespace tc
