@@ -96,6 +96,11 @@ typedef enum {
                                    form) instead of the tensor cores (centred expansion, bf16x3
                                    tcgen05.mma with the accumulator in TMEM; the default for the
                                    RBF kernel with d <= 16) */
+#define BTED_FLAG_RECOMPUTE 4096u /* implicit engine with the tensor-core Gram: every K.l pass rebuilds
+                                   the Gram tiles on the tensor cores (rc_pass.cuh) instead of
+                                   streaming the stored Gram from HBM; bitwise the same results.
+                                   Off by default: on B200 it is issue-bound at ~121 us per pass at
+                                   N = 16384 vs 84 us for the HBM-bound streaming pass */
 #define BTED_FLAG_TIMING   2u   /* record CUDA events around K1 and the K2 loop of every batch
                                    TED on the ctx stream; read with bted_get_stats()          */
 

@@ -25,6 +25,7 @@ BTED_FLAG_PERSISTENT_LOOP = 256
 BTED_FLAG_LOOPBACK = 512
 BTED_FLAG_NCCL = 1024
 BTED_FLAG_NO_TC_GRAM = 2048
+BTED_FLAG_RECOMPUTE = 4096
 STATUS = {0: "BTED_OK", 1: "BTED_EINVAL", 2: "BTED_ENOMEM", 3: "BTED_ECUDA", 4: "BTED_ENCCL",
           5: "BTED_ENUMERIC", 6: "BTED_ESTATE"}
 

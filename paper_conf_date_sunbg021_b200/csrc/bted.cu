@@ -39,6 +39,7 @@
 #include "colnorm.cuh"
 #include "xchg.cuh"
 #include "gram_tc.cuh"
+#include "rc_pass.cuh"
 
 namespace {
 
@@ -160,6 +161,9 @@ struct Ted {
     float* xctr = nullptr; size_t xctrcap = 0;
     int* xmax = nullptr; size_t xmaxcap = 0;
     bool gram_tc = true;                         // implicit head: K1 on tensor cores (else CUDA cores)
+    bool rc = false;                             // K.l passes recompute the tensor-core Gram (rc_pass.cuh)
+    bool rc_on = false;                          //   ... for the TED being enqueued (set by its head)
+    float rc_gamma = 0.f;
     bool split = true;                           // implicit: three kernels per step (else BTED_FLAG_PERSISTENT_LOOP)
     bool implicit = false;
     // K4 near-tie refinement (refine.cuh): per-CTA top-2 keys of every step, flags, candidates
@@ -240,6 +244,7 @@ struct Ted {
         grow(hv, hvcap, (size_t)m + 1);
         if (gram_tc) {
             grow(opA, opAcap, (size_t)nT * bted::tc::kBlockBytes);
+            if (rc) grow(opB, opBcap, (size_t)nT * bted::tc::kBlockBytes);   // row-permuted copy (rc_pass.cuh)
             grow(xnrm, xnrmcap, NP);
             grow(xctr, xctrcap, (size_t)bted::tc::kD * (1 + bted::tc::kCenterBlocks));
             grow(xmax, xmaxcap, 1);
@@ -483,8 +488,14 @@ void ensure_gram_tc_attrs() {
                                 (int)bted::tc::kTileSmemBytes));
         CK(cudaFuncSetAttribute(bted::tc::gram_tc_norm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)bted::tc::kBlockBytes));
+        CK(cudaFuncSetAttribute(bted::rc::rc_pass_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)bted::rc::kSmemBytes));
+        CK(cudaFuncSetAttribute(bted::rc::rc_pass_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)bted::rc::kSmemBytes));
     });
 }
+// the recomputing K.l pass: one CTA per SM (never more than the tiles)
+unsigned rc_pass_grid(int64_t tiles) { return (unsigned)std::min<int64_t>(tiles, (int64_t)num_sms()); }
 
 void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m,
                            float mu, unsigned long long* keys) {
@@ -510,7 +521,7 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
             X, (int32_t)N, d, T.xctr + bted::tc::kD);
         bted::tc::center_kernel<<<1, 32, 0, T.stream>>>(T.xctr + bted::tc::kD, (int32_t)N, d, T.xctr);
         bted::tc::prep_kernel<<<(unsigned)((NP + bted::tc::kThreads - 1) / bted::tc::kThreads), bted::tc::kThreads, 0,
-                                T.stream>>>(X, (int32_t)N, d, nT, T.xctr, T.opA);
+                                T.stream>>>(X, (int32_t)N, d, nT, T.xctr, T.opA, T.rc ? T.opB : nullptr);
         CK(cudaMemsetAsync(T.xmax, 0, sizeof(int), T.stream));
         bted::tc::gram_tc_norm_kernel<<<(unsigned)nT, bted::tc::kThreads, bted::tc::kBlockBytes, T.stream>>>(
             T.opA, T.xnrm, T.xmax);
@@ -527,9 +538,16 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
     } else {
         if (lin) k1i(bted::pk::gram_tile_kernel<32, true>); else k1i(bted::pk::gram_tile_kernel<32, false>);
     }
-    bted::im::tile_pass_kernel<true><<<tile_pass_grid(tiles), bted::im::kTPThreads, bted::im::tile_pass_smem_bytes,
-                                       T.stream>>>(T.K[0], nT, nullptr, T.P64, T.kflag, T.tctr, 0,
-                                                   l2_keep_tiles(tiles), 0, 1);
+    T.rc_on = d <= 16 && !lin && T.gram_tc && T.rc;
+    T.rc_gamma = gamma;
+    if (T.rc_on) {         // the norm pass on recomputed tiles (the stored Gram if the guard failed)
+        bted::rc::rc_pass_kernel<true><<<rc_pass_grid(tiles), bted::rc::kThreads, bted::rc::kSmemBytes, T.stream>>>(
+            T.opB, T.opA, T.xnrm, T.xmax, gamma, (int32_t)N, T.K[0], nT, nullptr, T.P64, T.kflag);
+    } else {
+        bted::im::tile_pass_kernel<true><<<tile_pass_grid(tiles), bted::im::kTPThreads,
+                                           bted::im::tile_pass_smem_bytes, T.stream>>>(
+            T.K[0], nT, nullptr, T.P64, T.kflag, T.tctr, 0, l2_keep_tiles(tiles), 0, 1);
+    }
     bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
         T.P64, nT, (int32_t)N, T.K[0], mu, T.Lf, NPa, 0, T.hv, T.nv, T.rd, T.sel, keys, 0, keys, T.err,
         T.refine ? T.top2 : nullptr, T.Qc, nullptr, nullptr);
@@ -619,7 +637,9 @@ uint64_t enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned 
         return c;
     };
     const cudaLaunchConfig_t cA = cfg_of((unsigned)nA + 1, bted::im::kThreads, 0);      // + the h CTA
-    const cudaLaunchConfig_t cB = cfg_of(tile_pass_grid(tiles), bted::im::kTPThreads, bted::im::tile_pass_smem_bytes);
+    const cudaLaunchConfig_t cB = T.rc_on ? cfg_of(rc_pass_grid(tiles), bted::rc::kThreads, bted::rc::kSmemBytes)
+                                          : cfg_of(tile_pass_grid(tiles), bted::im::kTPThreads,
+                                                   bted::im::tile_pass_smem_bytes);
     const cudaLaunchConfig_t cC = cfg_of((unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0);
     const int keep = l2_keep_tiles(tiles);
     for (int32_t t = 1; t < m; ++t) {
@@ -627,8 +647,14 @@ uint64_t enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned 
         CK(cudaLaunchKernelEx(&cA, bted::im::ell_kernel, (const float*)T.K[0], nT, (int32_t)N, T.Lf, NPa, tp,
                               (const double*)T.rd, (const double*)T.nv, mu, (const unsigned long long*)keys, t, T.ell,
                               (const double*)T.Qc, T.G, m, T.hv, T.sel, bted::im::XKern{}));
-        CK(cudaLaunchKernelEx(&cB, bted::im::tile_pass_kernel<false>, (const float*)T.K[0], nT, (const double*)T.ell,
-                              T.P64, T.kflag, T.tctr + t, (int)(t & 1), t + 1 < m ? keep : 0, 0, 1));
+        if (T.rc_on)
+            CK(cudaLaunchKernelEx(&cB, bted::rc::rc_pass_kernel<false>, (const uint8_t*)T.opB, (const uint8_t*)T.opA,
+                                  (const float*)T.xnrm, (const int*)T.xmax, T.rc_gamma, (int32_t)N,
+                                  (const float*)T.K[0], nT, (const double*)T.ell, T.P64, T.kflag));
+        else
+            CK(cudaLaunchKernelEx(&cB, bted::im::tile_pass_kernel<false>, (const float*)T.K[0], nT,
+                                  (const double*)T.ell, T.P64, T.kflag, T.tctr + t, (int)(t & 1),
+                                  t + 1 < m ? keep : 0, 0, 1));
         CK(cudaLaunchKernelEx(&cC, bted::im::fin64_kernel, (const double*)T.P64, nT, (int32_t)N,
                               (const float*)T.K[0], mu, (const double*)T.Lf, NPa, tp, (const double*)T.hv, T.nv, T.rd,
                               (const uint8_t*)T.sel, (const unsigned long long*)keys, t, keys + t, T.err,
@@ -1028,6 +1054,7 @@ bted_status create_common(const float* X, int64_t N, int32_t d, bted_kernel kern
         ctx->ted.refine = ctx->bted_engine.refine = (params->flags & BTED_FLAG_NO_REFINE) == 0;
         ctx->ted.split = ctx->bted_engine.split = (params->flags & BTED_FLAG_PERSISTENT_LOOP) == 0;
         ctx->ted.gram_tc = ctx->bted_engine.gram_tc = (params->flags & BTED_FLAG_NO_TC_GRAM) == 0;
+        ctx->ted.rc = ctx->bted_engine.rc = (params->flags & BTED_FLAG_RECOMPUTE) != 0;
         CK(cudaMallocHost(&ctx->herr, sizeof(int)));
         if (params->x_on_device) {
             ctx->X = const_cast<float*>(X);

@@ -122,9 +122,14 @@ __device__ __forceinline__ void split3(float v, __nv_bfloat16& h, __nv_bfloat16&
 }
 
 // per row i (padding rows: 0): x' = x - c and its operand row (the twelve k-chunks above)
+// opP (optional): a second copy with the rows of every block permuted for the
+// recomputing pass (rc_pass.cuh): tile row r = 16a + 4qd + r' sits at row (TMEM lane)
+// 32qd + 4a + r', so that a TMEM lane quarter holds every fourth 4-row group.
+__host__ __device__ __forceinline__ int rc_lane_of_row(int r) { return 32 * ((r & 15) >> 2) + 4 * (r >> 4) + (r & 3); }
+__host__ __device__ __forceinline__ int rc_row_of_lane(int L) { return 16 * ((L & 31) >> 2) + 4 * (L >> 5) + (L & 3); }
 __global__ void __launch_bounds__(kThreads) prep_kernel(const float* __restrict__ X, int32_t N, int32_t d,
                                                        int nT, const float* __restrict__ c,
-                                                       uint8_t* __restrict__ opA) {
+                                                       uint8_t* __restrict__ opA, uint8_t* __restrict__ opP = nullptr) {
     const int64_t i = (int64_t)blockIdx.x * kThreads + threadIdx.x;
     if (i >= (int64_t)nT * T) return;
     const int blk = (int)(i / T), r = (int)(i % T);
@@ -137,12 +142,15 @@ __global__ void __launch_bounds__(kThreads) prep_kernel(const float* __restrict_
         split3(v, h[k], m[k], l[k]);
     }
     // k-chunk q of a row = 8 bf16 = one 16-byte core-matrix row
+    uint8_t* ap = opP ? opP + (size_t)blk * kBlockBytes : nullptr;
+    const int rp = rc_lane_of_row(r);
     auto put = [&](int q, const __nv_bfloat16* v) {
         uint4 u;
         __nv_bfloat16* e = reinterpret_cast<__nv_bfloat16*>(&u);
 #pragma unroll
         for (int x = 0; x < 8; ++x) e[x] = v[x];
         *reinterpret_cast<uint4*>(a + op_offset(r, 8 * q)) = u;
+        if (ap) *reinterpret_cast<uint4*>(ap + op_offset(rp, 8 * q)) = u;
     };
     put(0, h); put(1, l); put(2, h + 8); put(3, l + 8); put(4, m); put(5, m + 8);
     put(6, h); put(7, m); put(8, h + 8); put(9, m + 8); put(10, h); put(11, h + 8);

@@ -133,8 +133,11 @@ __device__ __forceinline__ void tp_store(double* p, double v, uint64_t keep) {
 // tree is handed to warps 0-3 through an mbarrier and finished one chunk into
 // the next tile (no CTA-wide barrier per tile).  n / tile_it / col_it carry the
 // ring, w-slot and column-buffer phases across calls.
-template <bool kNorm, bool kExact, int kAbl = 0>
-__device__ __forceinline__ void tp_consume(TPSmem& S, int nT, double* P64, int* __restrict__ kflag, int& n,
+// Sm: the shared-memory struct (TPSmem, or rc_pass.cuh's RCSmem: the same members),
+// kSt its ring depth; kSwz: the ring chunks are stored with 16-byte granule g of
+// row r at g ^ (r & 7) (written row-per-lane by the recomputing epilogue).
+template <bool kNorm, bool kExact, int kAbl = 0, class Sm = TPSmem, int kSt = kStages, bool kSwz = false>
+__device__ __forceinline__ void tp_consume(Sm& S, int nT, double* P64, int* __restrict__ kflag, int& n,
                                            int& tile_it, int& col_it) {
     double sink = 0.0;
     const int tid = threadIdx.x, wq = tid / 32, l = tid % 32;
@@ -147,8 +150,8 @@ __device__ __forceinline__ void tp_consume(TPSmem& S, int nT, double* P64, int* 
     int cit = 0;
     double* rptr = P64;                                       // the pending chunk's 4 row partials
     double* cptr = P64;                                       // the pending tile's column partials
-    int st = n % kStages;                                     // ring slot and phase of chunk n
-    uint32_t ph = (uint32_t)(n / kStages) & 1u;
+    int st = n % kSt;                                         // ring slot and phase of chunk n
+    uint32_t ph = (uint32_t)(n / kSt) & 1u;
     auto row_finish = [&]() {
         if (!rpend) return;
         rpend = false;
@@ -211,7 +214,7 @@ __device__ __forceinline__ void tp_consume(TPSmem& S, int nT, double* P64, int* 
         for (int c = 0; c < kChunks; ++c, ++n) {
             const int stc = st;
             pk::mbar_wait(&S.full[stc], ph);
-            if (++st == kStages) { st = 0; ph ^= 1u; }
+            if (++st == kSt) { st = 0; ph ^= 1u; }
             if (kAbl & 8) {
 #pragma unroll
                 for (int r = 0; r < 4; ++r) {
@@ -227,7 +230,8 @@ __device__ __forceinline__ void tp_consume(TPSmem& S, int nT, double* P64, int* 
             double g[4], cg[4];
 #pragma unroll
             for (int r = 0; r < 4; ++r) {
-                const float4 kv = *reinterpret_cast<const float4*>(&S.ring[stc][(4 * wq + r) * T + 4 * l]);
+                const int row = 4 * wq + r;
+                const float4 kv = *reinterpret_cast<const float4*>(&S.ring[stc][row * T + 4 * (kSwz ? l ^ (row & 7) : l)]);
                 const float f32[4] = {kv.x, kv.y, kv.z, kv.w};
                 double kd[4];
 #pragma unroll
@@ -300,8 +304,8 @@ __device__ __forceinline__ void tp_consume(TPSmem& S, int nT, double* P64, int* 
 // streams only the tiles k = sr + sp * kl (kl = 0, 1, ...), compactly at
 // K + kl * T^2; consumers get the global index k (partials land where the
 // unsharded pass would put them).
-template <bool kW, class WaitW>
-__device__ __forceinline__ void tp_produce(TPSmem& S, const float* __restrict__ K, int nT, const double* w,
+template <bool kW, class WaitW, class Sm = TPSmem, int kSt = kStages>
+__device__ __forceinline__ void tp_produce(Sm& S, const float* __restrict__ K, int nT, const double* w,
                                            int passes, int* tilectr, WaitW wait_w, int dir0 = 0,
                                            int keep_tiles = 0, int sr = 0, int sp = 1) {
     const uint64_t pol = pk::policy_evict_first();            // K is read once per step
@@ -334,8 +338,8 @@ __device__ __forceinline__ void tp_produce(TPSmem& S, const float* __restrict__ 
             if (k >= nAll) { ++ti; break; }
             const float* src = K + kl * (int64_t)(T * T);
             for (int c = 0; c < kChunks; ++c, ++n) {
-                const int st = n % kStages;
-                pk::mbar_wait(&S.empty[st], ((uint32_t)(n / kStages) & 1u) ^ 1u);
+                const int st = n % kSt;
+                pk::mbar_wait(&S.empty[st], ((uint32_t)(n / kSt) & 1u) ^ 1u);
                 pk::mbar_expect_tx(&S.full[st], kChunkBytes);
                 pk::bulk_g2s_hint(S.ring[st], src + c * kChunkFloats, kChunkBytes, &S.full[st], kpol);
             }
