@@ -37,6 +37,9 @@ CASES = {
     "dense4096": lambda: sel(4096, 8, NS | L.BTED_FLAG_DENSE),
     "k4full2048": lambda: bt.CandidateSet((np.arange(2048, dtype=np.float32) * 100)[:, None], 1.0,
                                           flags=NS).select(4, MU),
+    "recompute4096": lambda: sel(4096, 8, NS | L.BTED_FLAG_RECOMPUTE),       # rc_pass.cuh (TMEM, tcgen05)
+    "recompute_guard": lambda: bt.CandidateSet((np.arange(2048, dtype=np.float32) * 100)[:, None], 1.0,
+                                               flags=NS | L.BTED_FLAG_RECOMPUTE).select(4, MU),
     "tileshard3": lambda: sel(3001, 8, L.BTED_FLAG_LOOPBACK, num_devices=3),
     "rowbands2": lambda: sel(3001, 8, L.BTED_FLAG_LOOPBACK | L.BTED_FLAG_DENSE, num_devices=2),
     "bands_literal2": lambda: sel(3001, 8, L.BTED_FLAG_LOOPBACK | L.BTED_FLAG_DENSE, num_devices=2, norm_mode=1),
