@@ -461,19 +461,40 @@ int l2_keep_tiles(int64_t tiles) {
     const int64_t tile_bytes = (int64_t)bted::pk::T * bted::pk::T * 4;
     return (int)std::min<int64_t>(tiles, std::max<int64_t>(0, bytes / tile_bytes));
 }
+// The K.l pass's fp64 partials (nT x NP doubles, rewritten every step and read by kernel C) are stored
+// with an L2 evict-last hint when they take at most kP64KeepFrac of L2: they then never reach DRAM,
+// whose reads the pass needs (B200, N = 16384, scripts/tp_ablate.cu: 86.9 -> 80.3 us per pass).
+// BTED_P64_KEEP = 0 / 1 overrides.
+constexpr double kP64KeepFrac = 0.25;
+bool keep_partials(int nT) {
+    static std::atomic<int64_t> cached{-1};
+    int64_t lim = cached.load(std::memory_order_relaxed);
+    if (lim < 0) {
+        if (const char* e = std::getenv("BTED_P64_KEEP")) {
+            lim = std::atoi(e) ? INT64_MAX : 0;
+        } else {
+            int dev = 0, l2 = 0;
+            cudaGetDevice(&dev);
+            if (cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev) != cudaSuccess) l2 = 0;
+            cudaGetLastError();
+            lim = (int64_t)(kP64KeepFrac * l2);
+        }
+        cached.store(lim, std::memory_order_relaxed);
+    }
+    return (int64_t)nT * nT * bted::pk::T * 8 <= lim;
+}
 // head: K1p (the packed Gram, read-only from now on), fp64 norm pass, scores.  (3 kernels)
 void ensure_implicit_attrs() {
     static uint64_t done = 0;
     once_per_device(done, [] {
-        CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)bted::im::tile_pass_smem_bytes));
-        CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)bted::im::tile_pass_smem_bytes));
         // two persistent CTAs per SM need the maximum shared-memory carveout
-        CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<true>, cudaFuncAttributePreferredSharedMemoryCarveout,
-                                (int)cudaSharedmemCarveoutMaxShared));
-        CK(cudaFuncSetAttribute(bted::im::tile_pass_kernel<false>, cudaFuncAttributePreferredSharedMemoryCarveout,
-                                (int)cudaSharedmemCarveoutMaxShared));
+        for (const void* f : {(const void*)bted::im::tile_pass_kernel<true, false>,
+                              (const void*)bted::im::tile_pass_kernel<false, false>,
+                              (const void*)bted::im::tile_pass_kernel<true, true>,
+                              (const void*)bted::im::tile_pass_kernel<false, true>}) {
+            CK(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bted::im::tile_pass_smem_bytes));
+            CK(cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared));
+        }
         CK(cudaFuncSetAttribute(bted::im::ted_loop_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)bted::im::tile_pass_smem_bytes));
         CK(cudaFuncSetAttribute(bted::im::ted_loop_kernel, cudaFuncAttributePreferredSharedMemoryCarveout,
@@ -544,8 +565,8 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
         bted::rc::rc_pass_kernel<true><<<rc_pass_grid(tiles), bted::rc::kThreads, bted::rc::kSmemBytes, T.stream>>>(
             T.opB, T.opA, T.xnrm, T.xmax, gamma, (int32_t)N, T.K[0], nT, nullptr, T.P64, T.kflag);
     } else {
-        bted::im::tile_pass_kernel<true><<<tile_pass_grid(tiles), bted::im::kTPThreads,
-                                           bted::im::tile_pass_smem_bytes, T.stream>>>(
+        auto normk = keep_partials(nT) ? bted::im::tile_pass_kernel<true, true> : bted::im::tile_pass_kernel<true, false>;
+        normk<<<tile_pass_grid(tiles), bted::im::kTPThreads, bted::im::tile_pass_smem_bytes, T.stream>>>(
             T.K[0], nT, nullptr, T.P64, T.kflag, T.tctr, 0, l2_keep_tiles(tiles), 0, 1);
     }
     bted::im::fin64_kernel<<<(unsigned)(NP / bted::im::kFinRows), bted::im::kThreads, 0, T.stream>>>(
@@ -652,7 +673,9 @@ uint64_t enqueue_loop_implicit(Ted& T, int64_t N, int32_t m, float mu, unsigned 
                                   (const float*)T.xnrm, (const int*)T.xmax, T.rc_gamma, (int32_t)N,
                                   (const float*)T.K[0], nT, (const double*)T.ell, T.P64, T.kflag));
         else
-            CK(cudaLaunchKernelEx(&cB, bted::im::tile_pass_kernel<false>, (const float*)T.K[0], nT,
+            CK(cudaLaunchKernelEx(&cB, keep_partials(nT) ? bted::im::tile_pass_kernel<false, true>
+                                                         : bted::im::tile_pass_kernel<false, false>,
+                                  (const float*)T.K[0], nT,
                                   (const double*)T.ell, T.P64, T.kflag, T.tctr + t, (int)(t & 1),
                                   t + 1 < m ? keep : 0, 0, 1));
         CK(cudaLaunchKernelEx(&cC, bted::im::fin64_kernel, (const double*)T.P64, nT, (int32_t)N,

@@ -116,15 +116,16 @@ __device__ __forceinline__ bool not_pos_normal(float x) {
     return __float_as_uint(x) - 0x00800000u >= 0x7F000000u;
 }
 
-// partial stores: streaming (.cs) by default -- measured faster for the pass
-// than L2 evict-last or plain stores (scripts/tp_ablate.cu, profiles/)
+// partial stores: streaming (.cs), or L2 evict-last (kAbl & 64: tile_pass_kernel's kKeepP, chosen by
+// the library when the partial buffer fits well inside L2 -- then they never reach DRAM;
+// profiles/r2/partials_l2)
 template <int kAbl>
 __device__ __forceinline__ void tp_store(double* p, double v, uint64_t keep) {
     if (kAbl & 16) *p = v;
     else if (kAbl & 64) st_f64_hint(p, v, keep);
     else __stcs(p, v);
 }
-// kAbl (scripts/tp_ablate.cu only; 0 in the library): 1 = no partial stores,
+// kAbl (scripts/tp_ablate.cu; the library uses 0 and 64): 1 = no partial stores,
 // 8 = no arithmetic at all (LDS + release: the streaming ceiling), 16 = plain
 // partial stores (no L2 hint), 64 = L2 evict-last partial stores
 //
@@ -281,7 +282,7 @@ __device__ __forceinline__ void tp_consume(Sm& S, int nT, double* P64, int* __re
     row_finish();
     col_finish();
     if (kNorm && odd_value) atomicOr(kflag, 1);
-    if (kAbl && sink == 1.2345) P64[0] = sink;
+    if ((kAbl & ~64) && sink == 1.2345) P64[0] = sink;
 }
 
 // Producer lane: `passes` passes over the tiles, grabbed one at a time from
@@ -364,7 +365,9 @@ __device__ __forceinline__ void tp_init_barriers(TPSmem& S) {
 
 // Kernel B (norm pass when kNorm): q = K w into per-tile partials P64.
 // tilectr: this launch's tile counter (zeroed).
-template <bool kNorm>
+// kKeepP: store the partials with an L2 evict-last hint (they stay in L2 for kernel C and are
+// overwritten by the next pass, never written back) -- for partial buffers well inside L2.
+template <bool kNorm, bool kKeepP = false>
 __global__ void __launch_bounds__(kTPThreads, kTPBlocksPerSM)
 tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__ w, double* __restrict__ P64,
                  int* __restrict__ kflag, int* __restrict__ tilectr, int dir, int keep_tiles,
@@ -378,12 +381,13 @@ tile_pass_kernel(const float* __restrict__ K, int nT, const double* __restrict__
         return;
     }
     int n = 0, tile_it = 0, col_it = 0;
+    constexpr int kSt = kKeepP ? 64 : 0;                      // tp_store: evict-last / streaming
     if (kNorm) {
-        tp_consume<true, true>(S, nT, P64, kflag, n, tile_it, col_it);
+        tp_consume<true, true, kSt>(S, nT, P64, kflag, n, tile_it, col_it);
         return;
     }
-    if (*kflag) tp_consume<false, true>(S, nT, P64, kflag, n, tile_it, col_it);
-    else tp_consume<false, false>(S, nT, P64, kflag, n, tile_it, col_it);
+    if (*kflag) tp_consume<false, true, kSt>(S, nT, P64, kflag, n, tile_it, col_it);
+    else tp_consume<false, false, kSt>(S, nT, P64, kflag, n, tile_it, col_it);
     pdl_trigger();                                           // kernel C may launch as CTAs drain
 }
 

@@ -69,13 +69,21 @@ __global__ void __launch_bounds__(64) bulk_read(const float* __restrict__ a, siz
     }
 }
 
-int main() {
+__global__ void fill_rand(float* a, size_t n) {
+    for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x)
+        a[i] = 0.25f + 0.5f * (float)((i * 2654435761u) % 1000003) / 1000003.f;
+}
+
+int main(int argc, char** argv) {
+    const bool rnd = argc > 1 && argv[1][0] == 'r';         // "r": non-zero pseudo-random data
     int sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
     const size_t bytes = (size_t)1 << 30;                     // 1 GiB, >> L2
     float* a; float* out;
     cudaMalloc(&a, bytes); cudaMalloc(&out, 4);
     cudaMemset(a, 0, bytes);
+    if (rnd) fill_rand<<<1184, 256>>>(a, bytes / 4);
+    printf("data: %s\n", rnd ? "pseudo-random floats in [0.25, 0.75)" : "zeros");
     cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
     auto timeit = [&](const char* name, auto launch) {
         launch(); cudaDeviceSynchronize();
