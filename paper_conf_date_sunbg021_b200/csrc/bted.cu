@@ -1386,9 +1386,34 @@ int small_cluster_used(int ninst, int64_t N, int32_t d) {
     return C;
 }
 
+// TEDs of at most 64 points run in one 256-thread CTA each (small.cuh ted_tiny_kernel);
+// BTED_NO_TINY_TED=1 sends them to the cluster kernel instead (A/B only)
+bool use_tiny_ted(int64_t N) {
+    static const bool off = [] { const char* e = std::getenv("BTED_NO_TINY_TED"); return e && std::atoi(e); }();
+    return !off && N >= 1 && N <= bted::sm::kTinyMaxN;
+}
+// score units per TED instance of launch_small (K4's top-2 layout)
+int small_units(int ninst, int64_t N, int32_t d) {
+    return use_tiny_ted(N) ? bted::sm::kTinyUnits : small_cluster_used(ninst, N, d) * bted::sm::kWarps;
+}
+
 void launch_small(const float* X, int ninst, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
                   unsigned long long* keys, int* err, cudaStream_t st, unsigned long long* top2 = nullptr,
                   const unsigned long long* forced = nullptr, int nforced = 0) {
+    if (use_tiny_ted(N)) {
+        const size_t smem = bted::sm::tiny_smem_bytes((int)N, d);
+        static uint64_t attr = 0;
+        once_per_device(attr, [] {
+            CK(cudaFuncSetAttribute(bted::sm::ted_tiny_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    (int)(200 * 1024)));
+        });
+        if (smem > (size_t)200 * 1024) throw CudaError{cudaErrorInvalidValue, "launch_small: d too large"};
+        bted::sm::ted_tiny_kernel<<<(unsigned)ninst, bted::sm::kTinyThreads, smem, st>>>(
+            X, (int32_t)N, d, gamma, (int32_t)(kernel == BTED_KERNEL_LINEAR ? 1 : 0), m, mu, keys, err, top2, forced,
+            (int32_t)nforced);
+        LAUNCHED(1);
+        return;
+    }
     // the smallest cluster whose CTAs also hold the staged features, if the
     // ninst clusters still fit on the SMs at once; else the smallest that fits
     const int C = small_cluster_used(ninst, N, d);
@@ -1405,8 +1430,8 @@ void launch_small(const float* X, int ninst, int64_t N, int32_t d, float gamma, 
 // ---- K4 for cluster-kernel TEDs (merges, small batches, small bted_select) ----
 // Buffers for ninst instances of m steps; returns the top-2 buffer to pass to launch_small.
 unsigned long long* small_k4_reserve(bted_ctx* ctx, int ninst, int64_t N, int32_t d, int32_t m) {
-    const int nU = small_cluster_used(ninst, N, d) * bted::sm::kWarps;
-    const int nU1 = small_cluster_used(1, N, d) * bted::sm::kWarps;       // single-instance re-runs
+    const int nU = small_units(ninst, N, d);
+    const int nU1 = small_units(1, N, d);                                  // single-instance re-runs
     grow(ctx->ktop2, ctx->ktop2cap, (size_t)ninst * m * nU * 2 + (size_t)m * nU1 * 2);   // + re-run scratch
     grow(ctx->kflags, ctx->kflagscap, (size_t)ninst * m);
     grow(ctx->kcand, ctx->kcandcap, (size_t)ninst * m * bted::rf::kMaxCand);
@@ -1425,7 +1450,7 @@ unsigned long long* small_k4_reserve(bted_ctx* ctx, int ninst, int64_t N, int32_
 // the caller's next stream synchronisation.
 void small_k4_launch(bted_ctx* ctx, cudaStream_t st, int ninst, int64_t N, int32_t d, int32_t m,
                      const unsigned long long* keys) {
-    const int nUb = small_cluster_used(ninst, N, d) * bted::sm::kWarps;
+    const int nUb = small_units(ninst, N, d);
     if (ctx->k4pincap < (size_t)ninst) {
         if (ctx->k4pin) cudaFreeHost(ctx->k4pin);
         ctx->k4pin = nullptr; ctx->k4pincap = 0;
@@ -1447,8 +1472,8 @@ bool small_k4_refine(bted_ctx* ctx, cudaStream_t st, const float* X, int ninst, 
     bool any = false;
     for (int k = 0; k < ninst; ++k) any |= ctx->k4pin[k] != 0;
     if (!any) return false;
-    const int nUb = small_cluster_used(ninst, N, d) * bted::sm::kWarps;
-    const int nU1 = small_cluster_used(1, N, d) * bted::sm::kWarps;
+    const int nUb = small_units(ninst, N, d);
+    const int nU1 = small_units(1, N, d);
     const size_t kMC = bted::rf::kMaxCand;
     bool changed = false;
     unsigned long long* rerun_top2 = ctx->ktop2 + (size_t)ninst * m * nUb * 2;

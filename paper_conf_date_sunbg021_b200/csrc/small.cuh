@@ -281,6 +281,141 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
     csync();                                         // no CTA exits while others may read its smem
 }
 
+// ---------------------------------------------------------------- N <= 64: one small CTA per TED
+// The |X_U| <= B m point merge of Alg. 2 l.6 at the bench's B m = 64,
+// and any other TED of at most 64 points.  A whole TED is 64 dependent steps of very
+// little work each, so the step's latency chain is the cost: the 512-thread cluster
+// kernel spends ~1.5 us per step in shuffle trees and CTA barriers.  Here 256 threads
+// hold K in registers, thread (q, j) = (tid / 64, tid % 64) the 16 entries of column j
+// in rows 16q .. 16q + 15 (K is symmetric: a column is a row, and its squared norm is
+// the row norm of Alg. 1 l.3).  Per step, three CTA barriers:
+//   the four threads of column s publish it to shared memory | every thread deflates
+//   its 16 entries with deflate1 (the instruction every engine uses: K stays bitwise
+//   symmetric) and writes its partial sum of squares | the 64 threads of quarter 0 add
+//   the four partials ((p0 + p1) + (p2 + p3)), score their column, and the two warps'
+//   argmax (redux.sync on the score bits, then on the index bits) meet in shared memory.
+// Fixed summation orders throughout (partials: four interleaved accumulators, then
+// (a0 + a1) + (a2 + a3)), so exact duplicate points have identical columns, norms and
+// scores and tie to the lowest index.  The diagonal entry of column j is carried by its
+// quarter-0 thread and updated with the same deflate1 operands as the matrix entry.
+// K4: every column is a score unit (nU = 64; top2_all[inst][t][j] = {key, 0}).
+constexpr int kTinyMaxN = 64;
+constexpr int kTinyThreads = 256;
+constexpr int kTinyRows = kTinyMaxN / 4;          // entries per thread
+constexpr int kTinyUnits = kTinyMaxN;
+__host__ __device__ __forceinline__ size_t tiny_smem_bytes(int N, int d) {
+    return 16 + (size_t)(kTinyMaxN + 4 * kTinyMaxN + (size_t)N * (size_t)(d | 1)) * sizeof(float);
+}
+__global__ void __launch_bounds__(kTinyThreads, 1)
+ted_tiny_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float gamma, int32_t linear, int32_t m,
+                float mu, unsigned long long* __restrict__ keys_all, int* __restrict__ err,
+                unsigned long long* __restrict__ top2_all, const unsigned long long* __restrict__ forced,
+                int32_t nforced) {
+    extern __shared__ __align__(16) unsigned char tsm[];
+    unsigned long long* wbest = reinterpret_cast<unsigned long long*>(tsm);     // [2] the two warps' keys
+    float* piv = reinterpret_cast<float*>(tsm + 16);                            // [64] pivot column
+    float* part = piv + kTinyMaxN;                                              // [4][64] partial norms
+    float* Xs = part + 4 * kTinyMaxN;                                           // [N][d | 1] features
+    const int tid = threadIdx.x, j = tid % kTinyMaxN, q = tid / kTinyMaxN, l = tid % 32, w = tid / 32;
+    const int inst = blockIdx.x;
+    const float* X = Xall + (int64_t)inst * N * d;
+    unsigned long long* keys_out = keys_all + (int64_t)inst * m;
+    unsigned long long* top2 = top2_all ? top2_all + (int64_t)inst * m * kTinyUnits * 2 : nullptr;
+    const int xs = d | 1;
+    for (int p = tid; p < N * d; p += kTinyThreads) Xs[(p / d) * xs + p % d] = X[p];
+    __syncthreads();
+    const bool vj = j < N;
+    const float ng = -gamma;
+    // l.1: K_ij exactly as the cluster kernel forms it (row i, column j; k ascending)
+    float c[kTinyRows];
+    {
+        float a[kTinyRows];
+#pragma unroll
+        for (int r = 0; r < kTinyRows; ++r) a[r] = 0.f;
+        for (int k = 0; k < d; ++k) {
+            const float xj = vj ? Xs[j * xs + k] : 0.f;
+#pragma unroll
+            for (int r = 0; r < kTinyRows; ++r) {
+                const int i = q * kTinyRows + r;
+                const float xi = i < N ? Xs[i * xs + k] : 0.f;
+                if (linear) a[r] = __fmaf_rn(xi, xj, a[r]);
+                else { const float df = __fsub_rn(xi, xj); a[r] = __fmaf_rn(df, df, a[r]); }
+            }
+        }
+#pragma unroll
+        for (int r = 0; r < kTinyRows; ++r)
+            c[r] = (q * kTinyRows + r < N && vj) ? (linear ? a[r] : expf(__fmul_rn(ng, a[r]))) : 0.f;
+    }
+    float dg = 0.f;                                         // K_jj (quarter-0 threads)
+    if (q == 0 && vj) {
+        float a = 0.f;
+        for (int k = 0; k < d; ++k) {
+            const float xj = Xs[j * xs + k];
+            if (linear) a = __fmaf_rn(xj, xj, a);
+            else { const float df = __fsub_rn(xj, xj); a = __fmaf_rn(df, df, a); }
+        }
+        dg = linear ? a : expf(__fmul_rn(ng, a));
+    }
+    bool selj = false;
+    auto put_partial = [&]() {
+        float a[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+        for (int r = 0; r < kTinyRows; ++r) a[r & 3] = __fmaf_rn(c[r], c[r], a[r & 3]);
+        part[q * kTinyMaxN + j] = __fadd_rn(__fadd_rn(a[0], a[1]), __fadd_rn(a[2], a[3]));
+    };
+    // after the partials' barrier: quarter 0 scores its columns, the CTA's argmax key
+    auto argmax = [&](int t) -> unsigned long long {
+        if (q == 0) {
+            const float n = __fadd_rn(__fadd_rn(part[j], part[kTinyMaxN + j]),
+                                      __fadd_rn(part[2 * kTinyMaxN + j], part[3 * kTinyMaxN + j]));
+            const unsigned long long key = vj ? score_key(n, dg, mu, (uint32_t)j, selj, err) : 0ull;
+            if (top2) {
+                unsigned long long* p = top2 + ((int64_t)t * kTinyUnits + j) * 2;
+                p[0] = key;
+                p[1] = 0ull;
+            }
+            const uint32_t hi = (uint32_t)(key >> 32);
+            const uint32_t mh = __reduce_max_sync(0xffffffffu, hi);
+            const uint32_t ml = __reduce_max_sync(0xffffffffu, hi == mh ? (uint32_t)key : 0u);
+            if (l == 0) wbest[w] = ((unsigned long long)mh << 32) | ml;
+        }
+        __syncthreads();
+        return wbest[0] > wbest[1] ? wbest[0] : wbest[1];
+    };
+    put_partial();
+    __syncthreads();
+    unsigned long long best = argmax(0);
+    if (forced && 0 < nforced) best = forced[0];             // K4 re-run: preset (flagged) picks
+    for (int t = 1; t < m; ++t) {
+        if (tid == 0) keys_out[t - 1] = best;
+        if (best == 0ull) { if (tid == 0) atomicOr(err, 2); break; }
+        const int s = (int)key_index(best);
+        selj |= j == s;
+        if (j == s) {                                       // column s, rows 16q ..: publish
+#pragma unroll
+            for (int r = 0; r < kTinyRows; r += 4)
+                *reinterpret_cast<float4*>(&piv[q * kTinyRows + r]) = make_float4(c[r], c[r + 1], c[r + 2], c[r + 3]);
+        }
+        __syncthreads();
+        const float inv_c = __frcp_rn(__fadd_rn(piv[s], mu));   // 1 / (K_ss + mu)
+        const float pj = piv[j];                                // K_sj
+#pragma unroll
+        for (int r = 0; r < kTinyRows; r += 4) {
+            const float4 a = *reinterpret_cast<const float4*>(&piv[q * kTinyRows + r]);   // K_is
+            c[r] = deflate1(c[r], a.x, pj, inv_c);
+            c[r + 1] = deflate1(c[r + 1], a.y, pj, inv_c);
+            c[r + 2] = deflate1(c[r + 2], a.z, pj, inv_c);
+            c[r + 3] = deflate1(c[r + 3], a.w, pj, inv_c);
+        }
+        if (q == 0) dg = deflate1(dg, pj, pj, inv_c);
+        put_partial();
+        __syncthreads();
+        best = argmax(t);
+        if (forced && t < nforced) best = forced[t];
+    }
+    if (tid == 0) keys_out[m - 1] = best;
+}
+
 }  // namespace sm
 }  // namespace bted
 

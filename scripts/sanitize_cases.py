@@ -28,6 +28,8 @@ def sel(N, m, flags=0, **kw):
 
 CASES = {
     "toy": lambda: sel(256, 16),                                        # cluster kernel, C = 1
+    "tiny64": lambda: sel(64, 64),                                      # ted_tiny_kernel (N <= 64)
+    "tiny33": lambda: sel(33, 20),
     "cluster500": lambda: sel(500, 16),
     "cluster940": lambda: sel(940, 16),
     "implicit4096": lambda: sel(4096, 8, NS),
@@ -55,6 +57,15 @@ def run_batches():
 
 
 CASES["batches"] = run_batches
+
+
+def run_tiny_batches():
+    X, g = knob(5000, 7)
+    with bt.CandidateSet(X, g, num_batches=5, seed=2) as pool:            # 5 tiny batch TEDs, merge of <= 100
+        pool.run_batches(50, 20, MU)
+
+
+CASES["tinybatches"] = run_tiny_batches
 
 if __name__ == "__main__":
     for name in sys.argv[1:]:
