@@ -38,6 +38,7 @@
 #include "refine.cuh"
 #include "colnorm.cuh"
 #include "xchg.cuh"
+#include <cudaTypedefs.h>
 #include "gram_tc.cuh"
 #include "rc_pass.cuh"
 
@@ -507,6 +508,8 @@ void ensure_gram_tc_attrs() {
     once_per_device(done, [] {
         CK(cudaFuncSetAttribute(bted::tc::gram_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)bted::tc::kTileSmemBytes));
+        CK(cudaFuncSetAttribute(bted::tc::gram_tc_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)bted::tc::kTmaSmemBytes));
         CK(cudaFuncSetAttribute(bted::tc::gram_tc_norm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)bted::tc::kBlockBytes));
         CK(cudaFuncSetAttribute(bted::rc::rc_pass_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -517,6 +520,34 @@ void ensure_gram_tc_attrs() {
 }
 // the recomputing K.l pass: one CTA per SM (never more than the tiles)
 unsigned rc_pass_grid(int64_t tiles) { return (unsigned)std::min<int64_t>(tiles, (int64_t)num_sms()); }
+
+// The packed Gram as a 2-D fp32 tensor [tiles * 128 rows][128 columns] for the tensor-core Gram's
+// TMA stores (gram_tc.cuh gram_tc_tma_kernel: boxes of 32 columns x 128 rows, 128-byte swizzle).
+// cuTensorMapEncodeTiled comes from the driver through the runtime (no libcuda link).
+bool k_tensor_map(CUtensorMap* map, float* K, int64_t tiles) {
+    static PFN_cuTensorMapEncodeTiled_v12000 encode = [] {
+        void* fn = nullptr;
+        cudaDriverEntryPointQueryResult q{};
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess)
+            fn = nullptr;
+        cudaGetLastError();
+        return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+    }();
+    if (!encode) return false;
+    const cuuint64_t dims[2] = {(cuuint64_t)bted::pk::T, (cuuint64_t)tiles * bted::pk::T};
+    const cuuint64_t strides[1] = {(cuuint64_t)bted::pk::T * sizeof(float)};
+    const cuuint32_t box[2] = {(cuuint32_t)bted::tc::kBoxCols, (cuuint32_t)bted::pk::T};
+    const cuuint32_t estr[2] = {1, 1};
+    return encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, K, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                  CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+// BTED_GRAM_STG=1: the tensor-core Gram with the threads' own stores (A/B only)
+bool gram_tma_stores() {
+    static const bool off = [] { const char* e = std::getenv("BTED_GRAM_STG"); return e && std::atoi(e); }();
+    return !off;
+}
 
 void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float gamma, int kernel, int32_t m,
                            float mu, unsigned long long* keys) {
@@ -547,8 +578,13 @@ void enqueue_head_implicit(Ted& T, const float* X, int64_t N, int32_t d, float g
         bted::tc::gram_tc_norm_kernel<<<(unsigned)nT, bted::tc::kThreads, bted::tc::kBlockBytes, T.stream>>>(
             T.opA, T.xnrm, T.xmax);
         const unsigned g = (unsigned)std::min<int64_t>(tiles, (int64_t)2 * num_sms());
-        bted::tc::gram_tc_kernel<<<g, bted::tc::kTcThreads, bted::tc::kTileSmemBytes, T.stream>>>(
-            T.opA, T.xnrm, (int32_t)N, gamma, T.K[0], nT, T.xmax);
+        CUtensorMap kmap;
+        if (gram_tma_stores() && k_tensor_map(&kmap, T.K[0], tiles))
+            bted::tc::gram_tc_tma_kernel<<<g, bted::tc::kWsThreads, bted::tc::kTmaSmemBytes, T.stream>>>(
+                T.opA, T.xnrm, (int32_t)N, gamma, nT, T.xmax, kmap);
+        else
+            bted::tc::gram_tc_kernel<<<g, bted::tc::kTcThreads, bted::tc::kTileSmemBytes, T.stream>>>(
+                T.opA, T.xnrm, (int32_t)N, gamma, T.K[0], nT, T.xmax);
         // the accuracy guard's fallback (exits at once when the tensor-core Gram was written)
         bted::pk::gram_tile2_kernel<16, false, 4><<<(unsigned)std::min<int64_t>(tiles, (int64_t)4 * num_sms()),
                                                      bted::pk::kConsumers, 0, T.stream>>>(

@@ -42,6 +42,7 @@
 // recomputed one are the same numbers.
 #pragma once
 #include <cstdint>
+#include <cuda.h>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include "packed.cuh"
@@ -456,6 +457,167 @@ gram_tc_kernel(const uint8_t* __restrict__ opA, const float* __restrict__ nrm,
         }
         I = In;
         J = Jn;
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (w == 0) tmem_free<2 * T>(tbase);
+}
+
+// ---------------------------------------------------------------- the tile kernel, warp-specialised
+// Same tiles, same K values (the same kval2 on the same accumulator), restructured so
+// the epilogue never waits on a copy or an MMA issue:
+//   * a PRODUCER warp (warp 8, one lane) issues the operand copies (cp.async.bulk) and the
+//     six MMAs of every tile: MMA(t) into TMEM accumulator t % 2 once the epilogue has
+//     released it (acc_free) and tile t's operands have landed; then the copies of tile
+//     t + 1 into operand slot (t + 1) % 2 (A_J and the norms are double-buffered; the A_I
+//     block is reloaded, after MMA(t) completed, only when the row block changes);
+//   * eight EPILOGUE warps read the accumulator (tcgen05.ld), form K (kval2) into two
+//     16 KiB boxes [128 rows][32 floats] per half tile in the 128-byte swizzled layout the
+//     tensor map names (16-byte chunk c of row r at chunk c ^ (r % 8): conflict-free for a
+//     warp writing 32 consecutive rows), and one thread stores the boxes with
+//     cp.async.bulk.tensor (TMA); a box is rewritten only after its bulk group READ it.
+// tmap: K as a 2-D fp32 tensor [tiles * 128 rows][128 columns], box 32 x 128, SWIZZLE_128B.
+constexpr int kBoxCols = 32;
+constexpr size_t kBoxBytes = (size_t)T * kBoxCols * sizeof(float);          // 16 KiB
+constexpr int kWsThreads = kTcThreads + 32;                                  // + the producer warp
+constexpr size_t kTmaSmemBytes = 3 * (size_t)kBlockBytes + 2 * kBoxBytes;    // A_I, A_J x 2, 2 boxes: 104 KiB
+
+__device__ __forceinline__ void tma_store_2d(const void* tmap, const void* src, int c0, int c1) {
+    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];"
+                 :: "l"(reinterpret_cast<uint64_t>(tmap)), "r"(c0), "r"(c1), "r"(smem_u32(src)) : "memory");
+}
+__device__ __forceinline__ void epi_sync() {                   // named barrier 1: the 8 epilogue warps
+    asm volatile("bar.sync 1, %0;" :: "n"(kTcThreads) : "memory");
+}
+
+__global__ void __launch_bounds__(kWsThreads, 2)
+gram_tc_tma_kernel(const uint8_t* __restrict__ opA, const float* __restrict__ nrm, int32_t N, float gamma, int nT,
+                   const int* __restrict__ nmax_bits, const __grid_constant__ CUtensorMap tmap) {
+    if (!tc_ok(nmax_bits, gamma)) return;                         // the direct-form kernel writes K
+    extern __shared__ __align__(1024) uint8_t smem[];            // [A_I | A_J 0 | A_J 1 | box 0 | box 1]
+    __shared__ __align__(8) uint64_t ldbar[2], mmabar[2], freebar[2];
+    __shared__ uint32_t tmem_base;
+    __shared__ __align__(16) float nIs[2][T];
+    __shared__ __align__(16) float nJs[2][T];
+    uint8_t* const aI = smem;
+    uint8_t* const box = smem + 3 * kBlockBytes;
+    const int tid = threadIdx.x, w = tid / 32, lane = tid % 32;
+    const int64_t ntiles = pk::num_tiles(nT);
+    const int64_t per = (ntiles + gridDim.x - 1) / gridDim.x;
+    const int64_t k0 = (int64_t)blockIdx.x * per, k1 = k0 + per < ntiles ? k0 + per : ntiles;
+    const int cnt = k0 < k1 ? (int)(k1 - k0) : 0;
+    if (w == 0) tmem_alloc<2 * T>(&tmem_base);
+    if (tid == 0) {
+        for (int q = 0; q < 2; ++q) {
+            pk::mbar_init(&ldbar[q], 1);
+            pk::mbar_init(&mmabar[q], 1);
+            pk::mbar_init(&freebar[q], 1);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tbase = tmem_base;
+
+    if (w == kTcThreads / 32) {                                   // ---- producer warp
+        if (lane == 0 && cnt > 0) {
+            int I = 0, J = 0, loadedI = -1;
+            pk::tile_ij(k0, nT, I, J);
+            // copies of tile (I_, J_) into operand slot s (A_I only when the row block changes)
+            auto load = [&](int I_, int J_, int s) {
+                const bool newI = I_ != loadedI;
+                pk::mbar_expect_tx(&ldbar[s], (newI ? kBlockBytes : 0u) + kBlockBytes + 2u * T * 4u);
+                if (newI) pk::bulk_g2s(aI, opA + (size_t)I_ * kBlockBytes, kBlockBytes, &ldbar[s]);
+                pk::bulk_g2s(smem + (1 + s) * kBlockBytes, opA + (size_t)J_ * kBlockBytes, kBlockBytes, &ldbar[s]);
+                pk::bulk_g2s(nIs[s], nrm + (int64_t)I_ * T, T * 4u, &ldbar[s]);
+                pk::bulk_g2s(nJs[s], nrm + (int64_t)J_ * T, T * 4u, &ldbar[s]);
+                loadedI = I_;
+            };
+            load(I, J, 0);
+            for (int it = 0; it < cnt; ++it) {
+                const int s = it & 1;
+                // MMA(it): accumulator s released by epilogue(it - 2), operands of tile it landed
+                if (it >= 2) pk::mbar_wait(&freebar[s], (uint32_t)((it - 2) >> 1) & 1u);
+                pk::mbar_wait(&ldbar[s], (uint32_t)(it >> 1) & 1u);
+                asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+                issue_gram_mmas(tbase + (uint32_t)(s * T), smem_u32(aI), smem_u32(smem + (1 + s) * kBlockBytes));
+                mma_commit(&mmabar[s]);
+                if (it + 1 < cnt) {                               // copies of tile it + 1 into slot s ^ 1
+                    int In = I, Jn = J + 1;
+                    if (Jn == nT) { ++In; Jn = In; }
+                    // slot s ^ 1 (A_J, norms) was last read by epilogue(it - 1); A_I by MMA(it)
+                    if (it >= 1) pk::mbar_wait(&freebar[s ^ 1], (uint32_t)((it - 1) >> 1) & 1u);
+                    if (In != loadedI) pk::mbar_wait(&mmabar[s], (uint32_t)(it >> 1) & 1u);
+                    load(In, Jn, s ^ 1);
+                    I = In;
+                    J = Jn;
+                }
+            }
+        }
+    } else {                                                      // ---- epilogue warps
+        const float ngl2e = __fmul_rn(-gamma, 1.4426950408889634f);   // exp(-g d2) = 2^(-g log2(e) d2)
+        const unsigned long long g2 = f2pack(ngl2e, ngl2e);
+        const int q4 = w & 3, hh = w >> 2;                         // TMEM lane quarter, box (column half)
+        const int r = 32 * q4 + lane;
+        const uint32_t lb = (uint32_t)(32 * q4) << 16;
+        uint8_t* const myrow = box + hh * kBoxBytes + (size_t)r * (kBoxCols * 4);
+        int I = 0, J = 0;
+        if (cnt > 0) pk::tile_ij(k0, nT, I, J);
+        for (int it = 0; it < cnt; ++it) {
+            const int s = it & 1;
+            const int64_t k = k0 + it;
+            pk::mbar_wait(&mmabar[s], (uint32_t)(it >> 1) & 1u);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            const float ni = nIs[s][r];
+            const float* nj = nJs[s];
+            const bool edge = (I + 1) * T > N || (J + 1) * T > N;
+            const bool rowv = I * T + r < N;
+            const uint32_t tD = tbase + (uint32_t)(s * T) + lb;
+#pragma unroll 1
+            for (int half = 0; half < 2; ++half) {
+                // the boxes are free once the previous half's stores have read them
+                if (tid == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+                epi_sync();
+                const int c0 = 64 * hh + 32 * half;                // tile column of box hh's column 0
+#pragma unroll
+                for (int cc = 0; cc < 32; cc += 16) {
+                    uint32_t du[16];
+                    tmem_ld16_async(tD + (uint32_t)(c0 + cc), du);
+                    tmem_wait_ld();
+                    float o[16];
+#pragma unroll
+                    for (int q = 0; q < 16; q += 2) {
+                        const float2 njq = *reinterpret_cast<const float2*>(&nj[c0 + cc + q]);
+                        kval2(__uint_as_float(du[q]), __uint_as_float(du[q + 1]),
+                              f2add(f2pack(ni, ni), f2pack(njq.x, njq.y)), g2, o[q], o[q + 1]);
+                    }
+                    if (edge) {
+#pragma unroll
+                        for (int q = 0; q < 16; ++q)
+                            if (!rowv || J * T + c0 + cc + q >= N) o[q] = 0.f;
+                    }
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {                  // 16-byte chunk cc/4 + q, swizzled
+                        const int ch = (cc >> 2) + q;
+                        *reinterpret_cast<float4*>(myrow + ((ch ^ (r & 7)) << 4)) =
+                            make_float4(o[4 * q], o[4 * q + 1], o[4 * q + 2], o[4 * q + 3]);
+                    }
+                }
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic writes -> async proxy
+                asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+                epi_sync();                                        // both boxes complete
+                if (tid == 0) {
+                    if (half == 1) pk::mbar_arrive(&freebar[s]);   // accumulator s and norm slot s read
+                    const int row = (int)(k * T);
+                    tma_store_2d(&tmap, box, 32 * half, row);
+                    tma_store_2d(&tmap, box + kBoxBytes, 64 + 32 * half, row);
+                    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+                }
+            }
+            if (++J == nT) { ++I; J = I; }
+        }
+        if (tid == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
     }
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
     __syncthreads();
