@@ -11,6 +11,6 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:"til
     -o $OUT/prof_imp python bench.py --config $CFG --steps 1 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_imp.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"gram_tc|prep_kernel|center_kernel" -s 3 -c 3 \
     -o $OUT/prof_gram python bench.py --config $CFG --steps 1 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_gram.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:"ted_cluster" -s 3 -c 1 \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"ted_cluster|ted_tiny" -s 3 -c 1 \
     -o $OUT/prof_merge python bench.py --config $CFG --steps 1 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_merge.log 2>&1
 ls -la $OUT
