@@ -430,10 +430,18 @@ struct XKern {
     }
 };
 
-template <class Sync>
+// this thread's first 16 factor entries L_ik (k = g, g + 4, ...; they do not depend on the pick s)
+__device__ __forceinline__ void ell_rows(int unit, const double* Lc, int64_t ldL, int32_t tp, double (&a)[16]) {
+    const int r = threadIdx.x % kEllRows, g = threadIdx.x / kEllRows;
+    const int64_t i = (int64_t)unit * kEllRows + r;
+#pragma unroll
+    for (int q = 0; q < 16; ++q) a[q] = (g + 4 * q < tp) ? __ldcg(&Lc[(int64_t)(g + 4 * q) * ldL + i]) : 0.0;
+}
+// kPre: a[] was loaded by ell_rows already (ell_kernel does it before waiting for the pick)
+template <class Sync, bool kPre = false>
 __device__ __forceinline__ void ell_unit(int unit, EllSmem& sm, Sync sync, const float* __restrict__ K, int nT,
                                          int32_t N, double* Lc, int64_t ldL, int32_t tp, uint32_t s,
-                                         double rc, double* ell, XKern xk = XKern{}) {
+                                         double rc, double* ell, XKern xk, double (&a)[16]) {
     const int tid = threadIdx.x, r = tid % kEllRows, g = tid / kEllRows;
     const int64_t i = (int64_t)unit * kEllRows + r;
     const float kis = (g == 0 && i < N) ? (xk.X ? xk(i, s) : K[packed_index((int)i, (int)s, nT)]) : 0.f;
@@ -441,10 +449,8 @@ __device__ __forceinline__ void ell_unit(int unit, EllSmem& sm, Sync sync, const
     // this thread's L_ik (k = g, g + 4, ...): loaded before the barrier, 16 at a time
     double acc = 0.0;
     int k = g;
-    double a[16];
     int na = 0;
-#pragma unroll
-    for (int q = 0; q < 16; ++q) a[q] = (g + 4 * q < tp) ? __ldcg(&Lc[(int64_t)(g + 4 * q) * ldL + i]) : 0.0;
+    if (!kPre) ell_rows(unit, Lc, ldL, tp, a);
     sync();
 #pragma unroll
     for (int q = 0; q < 16; ++q)
@@ -506,16 +512,20 @@ ell_kernel(const float* __restrict__ K, int nT, int32_t N, double* __restrict__ 
            const unsigned long long* __restrict__ keys, int32_t t, double* __restrict__ ell, const double* Qc,
            double* G, int32_t ldG, double* h, uint8_t* __restrict__ sel, XKern xk = XKern{}) {
     __shared__ EllSmem sm;
+    // the factor rows (written by earlier, completed steps) before waiting for this step's pick
+    double a[16];
+    const bool hcta = blockIdx.x == gridDim.x - 1;
+    if (!hcta) ell_rows(blockIdx.x, Lc, ldL, tp, a);
     pdl_wait();                                              // kernel C of the previous step complete
     pdl_trigger();                                           // the K.l pass may start streaming K now
     const uint32_t s = key_index(keys[t - 1]);
     if (blockIdx.x == 0 && threadIdx.x == 0) sel[s] = 1;
     const double c = __dadd_rn(rdiag[s], (double)mu);
-    if (blockIdx.x == gridDim.x - 1) {
+    if (hcta) {
         h_unit(sm.Ls, SyncCTA{}, Lc, ldL, Qc, G, ldG, tp, s, c, nv[s], h);
         return;
     }
-    ell_unit(blockIdx.x, sm, SyncCTA{}, K, nT, N, Lc, ldL, tp, s, __dsqrt_rn(c), ell, xk);
+    ell_unit<SyncCTA, true>(blockIdx.x, sm, SyncCTA{}, K, nT, N, Lc, ldL, tp, s, __dsqrt_rn(c), ell, xk, a);
 }
 // ------------------------------------------------------------------ kernel C: scores
 // t == 0 (after the norm pass): n_v = q_v (= ||K_:v||^2), r_vv = K_vv.
@@ -584,7 +594,9 @@ struct FinSmem {
     double hs[kMaxM + 1];
 };
 
-template <class Sync>
+struct NoWaitFn { __device__ void operator()() const {} };
+struct PdlWaitFn { __device__ void operator()() const { pdl_wait(); pdl_trigger(); } };
+template <class Sync, class WaitP = NoWaitFn>
 __device__ __forceinline__ void fin_unit(int unit, int nunits, FinSmem& sm, Sync sync, const double* P64,
                                          int nT, int32_t N, const float* __restrict__ K, float mu,
                                          const double* Lc, int64_t ldL, int32_t tp,
@@ -593,12 +605,31 @@ __device__ __forceinline__ void fin_unit(int unit, int nunits, FinSmem& sm, Sync
                                          int32_t t, unsigned long long* key_out, int* err,
                                          unsigned long long* top2, double* Qc, bool mark_sel = false,
                                          const double* qin = nullptr, const double* rinit = nullptr,
-                                         const PeerQ* pq = nullptr) {
+                                         const PeerQ* pq = nullptr, WaitP wait_partials = WaitP{}) {
     const int lane = threadIdx.x % 32, w = threadIdx.x / 32;
     const int64_t NP = (int64_t)nT * T;
     const int i = unit * kFinRows + lane;
     if (t > 0)
         for (int q = threadIdx.x; q <= tp; q += kThreads) sm.hs[q] = __ldcg(&h[q]);
+    // sum_{k in range w} L_ik h_k: inputs of this step's kernel A (complete), not of the K.l pass --
+    // computed before wait_partials (fin64_kernel: the PDL wait for the pass)
+    sync();
+    double la = 0.0;
+    if (t > 0) {
+        const int kper = (tp + 7) / 8;
+        const int k0 = min(tp, w * kper), k1 = min(tp, k0 + kper);
+        int k = k0;
+        for (; k + 8 <= k1; k += 8) {
+            double a[8];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) a[q] = __ldcg(&Lc[(int64_t)(k + q) * ldL + i]);
+#pragma unroll
+            for (int q = 0; q < 8; ++q) la = __fma_rn(a[q], sm.hs[k + q], la);
+        }
+        for (; k < k1; ++k) la = __fma_rn(__ldcg(&Lc[(int64_t)k * ldL + i]), sm.hs[k], la);
+    }
+    sm.lpart[w][lane] = la;
+    wait_partials();
     const int per = (nT + 7) / 8;
     const int j0 = min(nT, w * per), j1 = min(nT, j0 + per);
     double acc = 0.0;
@@ -619,22 +650,6 @@ __device__ __forceinline__ void fin_unit(int unit, int nunits, FinSmem& sm, Sync
         for (; J < j1; ++J) acc = __dadd_rn(acc, __ldcg(&src[(int64_t)J * NP]));
     }
     sm.part[w][lane] = acc;
-    sync();
-    double la = 0.0;                                       // sum_{k in range w} L_ik h_k
-    if (t > 0) {
-        const int kper = (tp + 7) / 8;
-        const int k0 = min(tp, w * kper), k1 = min(tp, k0 + kper);
-        int k = k0;
-        for (; k + 8 <= k1; k += 8) {
-            double a[8];
-#pragma unroll
-            for (int q = 0; q < 8; ++q) a[q] = __ldcg(&Lc[(int64_t)(k + q) * ldL + i]);
-#pragma unroll
-            for (int q = 0; q < 8; ++q) la = __fma_rn(a[q], sm.hs[k + q], la);
-        }
-        for (; k < k1; ++k) la = __fma_rn(__ldcg(&Lc[(int64_t)k * ldL + i]), sm.hs[k], la);
-    }
-    sm.lpart[w][lane] = la;
     sync();
     if (w == 0) {
         unsigned long long key = 0ull;
@@ -796,11 +811,11 @@ fin64_kernel(const double* __restrict__ P64, int nT, int32_t N, const float* __r
              int* __restrict__ err, unsigned long long* __restrict__ top2, double* __restrict__ Qc,
              const double* __restrict__ qin = nullptr, const double* __restrict__ rinit = nullptr) {
     __shared__ FinSmem sm;
-    pdl_wait();                                              // the K.l pass complete (P64, h)
-    pdl_trigger();
+    // keys[t-1], h, L, n_v, r_vv come from kernels that completed before the K.l pass of this step
+    // started consuming; only P64 needs the PDL wait for the pass (inside fin_unit, after L h)
     const uint32_t s = t > 0 ? key_index(keys[t - 1]) : 0xFFFFFFFFu;
     fin_unit(blockIdx.x, gridDim.x, sm, SyncCTA{}, P64, nT, N, K, mu, Lc, ldL, tp, h, nv, rdiag, sel, s, t, key_out,
-             err, top2, Qc, false, qin, rinit);
+             err, top2, Qc, false, qin, rinit, nullptr, PdlWaitFn{});
 }
 
 // fin64 of the in-library multi-GPU engine: waits for the P partial q of this
@@ -939,7 +954,8 @@ __device__ __forceinline__ void loop_consumers(TPSmem& S, const LoopArgs& a) {
         }
         const double rc = __dsqrt_rn(c);
         for (int u = blockIdx.x; u < nEll; u += gridDim.x) {
-            ell_unit(u, es, SyncConsumers{}, a.K, a.nT, a.N, a.Lc, a.ldL, tp, s, rc, a.ell);
+            double ar[16];
+            ell_unit(u, es, SyncConsumers{}, a.K, a.nT, a.N, a.Lc, a.ldL, tp, s, rc, a.ell, XKern{}, ar);
             if (threadIdx.x == 0) {
                 __threadfence();
                 asm volatile("st.release.gpu.global.s32 [%0], %1;" :: "l"(unit_flag + u), "r"(t) : "memory");
