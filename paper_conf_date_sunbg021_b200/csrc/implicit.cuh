@@ -811,8 +811,10 @@ fin64_kernel(const double* __restrict__ P64, int nT, int32_t N, const float* __r
              int* __restrict__ err, unsigned long long* __restrict__ top2, double* __restrict__ Qc,
              const double* __restrict__ qin = nullptr, const double* __restrict__ rinit = nullptr) {
     __shared__ FinSmem sm;
-    // keys[t-1], h, L, n_v, r_vv come from kernels that completed before the K.l pass of this step
-    // started consuming; only P64 needs the PDL wait for the pass (inside fin_unit, after L h)
+    // keys[t-1], h and L come from kernels that completed before any CTA of this step's K.l pass
+    // let this grid launch (the pass triggers only after its own wait for kernel A: tile_pass_kernel
+    // when its consumers finish -- at least one CTA has a tile --, rc_pass_kernel right after its
+    // producer's wait); only P64 needs the PDL wait for the pass (inside fin_unit, after L h)
     const uint32_t s = t > 0 ? key_index(keys[t - 1]) : 0xFFFFFFFFu;
     fin_unit(blockIdx.x, gridDim.x, sm, SyncCTA{}, P64, nT, N, K, mu, Lc, ldL, tp, h, nv, rdiag, sel, s, t, key_out,
              err, top2, Qc, false, qin, rinit, nullptr, PdlWaitFn{});

@@ -331,7 +331,12 @@ rc_pass_kernel(const uint8_t* __restrict__ opP, const uint8_t* __restrict__ opA,
             }
             next(wI_, wJ_);
         };
-        if (!kNorm && cnt > 0) im::pdl_wait();                 // l of this step written (previous kernel)
+        if (!kNorm && cnt > 0) {
+            im::pdl_wait();                                    // l of this step written (previous kernel)
+            // this CTA may let kernel C launch only now: worker groups without a tile finish at
+            // once, and kernel C reads this step's h and L before its own wait for the partials
+            im::pdl_trigger();
+        }
         for (int t = 0; t < kSlots && t < cnt; ++t) issue_w(t);
         for (int it = 0; it < cnt; ++it) {
             const int s = it % kSlots, b = it & 1;
@@ -362,7 +367,6 @@ rc_pass_kernel(const uint8_t* __restrict__ opP, const uint8_t* __restrict__ opA,
         else if (*kflag) rc_work<false, true, false>(S, nrm, gamma, N, K, nT, k0, cnt, P64, kflag);
         else rc_work<false, false, false>(S, nrm, gamma, N, K, nT, k0, cnt, P64, kflag);
     }
-    if (!kNorm) im::pdl_trigger();
     if (tc) {
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         asm volatile("bar.sync 4, %0;" :: "n"(kWorkWarps * 32) : "memory");   // every worker done with TMEM
