@@ -1572,8 +1572,7 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
         grow(ctx->xall, ctx->xallcap, (size_t)nb * M * ctx->d);
         grow(ctx->kall, ctx->kallcap, (size_t)nb * m);
         Ted& T = ctx->bted_engine;
-        for (int kk = 0; kk < nb; ++kk)
-            gather(ctx, st, ctx->sall + (size_t)kk * M, M, ctx->xall + (size_t)kk * M * ctx->d);
+        gather(ctx, st, ctx->sall, (int64_t)nb * M, ctx->xall);   // all batches: [nb][M] -> [nb][M][d]
         Ted::Slot* sl = T.timing ? T.next_slot(m) : nullptr;
         if (sl) { sl->small = nb; CK(cudaEventRecord(sl->e[0], st)); }
         unsigned long long* k4t = T.refine ? small_k4_reserve(ctx, nb, M, ctx->d, m) : nullptr;
@@ -1584,12 +1583,9 @@ int run_batch_range(bted_ctx* ctx, int64_t M, int32_t m, float mu, int32_t b_beg
             ctx->k4b.pending = true;
             ctx->k4b.ninst = nb; ctx->k4b.M = M; ctx->k4b.m = m; ctx->k4b.mu = mu;
         }
-        for (int kk = 0; kk < nb; ++kk) {
-            bted::map_winners_kernel<<<(m + 127) / 128, 128, 0, st>>>(ctx->kall + (size_t)kk * m, m,
-                                                                     ctx->sall + (size_t)kk * M,
-                                                                     ctx->winners + (size_t)kk * m);
-            LAUNCHED(1);
-        }
+        bted::map_winners_batched_kernel<<<dim3((m + 127) / 128, nb), 128, 0, st>>>(ctx->kall, m, ctx->sall, M,
+                                                                                    ctx->winners);
+        LAUNCHED(1);
         return nb;
     }
     Ted& T = ctx->bted_engine;
@@ -1679,11 +1675,9 @@ bted_status batch_range_finish(bted_ctx* ctx, int nb) {
         auto& b = ctx->k4b;
         if (small_k4_refine(ctx, ctx->stream, ctx->xall, b.ninst, b.M, ctx->d, b.m, b.mu, ctx->kall,
                             ctx->bted_engine.err)) {
-            for (int kk = 0; kk < b.ninst; ++kk) {
-                bted::map_winners_kernel<<<(b.m + 127) / 128, 128, 0, ctx->stream>>>(
-                    ctx->kall + (size_t)kk * b.m, b.m, ctx->sall + (size_t)kk * b.M, ctx->winners + (size_t)kk * b.m);
-                LAUNCHED(1);
-            }
+            bted::map_winners_batched_kernel<<<dim3((b.m + 127) / 128, b.ninst), 128, 0, ctx->stream>>>(
+                ctx->kall, b.m, ctx->sall, b.M, ctx->winners);
+            LAUNCHED(1);
             CK(cudaStreamSynchronize(ctx->stream));
         }
     }
@@ -1750,12 +1744,9 @@ bted_status merge_device(bted_ctx* ctx, const int64_t* winners_dev, int64_t n, i
         ctx->k4b.pending = false;
         auto& b = ctx->k4b;
         if (small_k4_refine(ctx, st, ctx->xall, b.ninst, b.M, ctx->d, b.m, b.mu, ctx->kall, ctx->bted_engine.err)) {
-            for (int kk = 0; kk < b.ninst; ++kk) {
-                bted::map_winners_kernel<<<(b.m + 127) / 128, 128, 0, st>>>(ctx->kall + (size_t)kk * b.m, b.m,
-                                                                           ctx->sall + (size_t)kk * b.M,
-                                                                           ctx->winners + (size_t)kk * b.m);
-                LAUNCHED(1);
-            }
+            bted::map_winners_batched_kernel<<<dim3((b.m + 127) / 128, b.ninst), 128, 0, st>>>(
+                ctx->kall, b.m, ctx->sall, b.M, ctx->winners);
+            LAUNCHED(1);
             b.changed = true;
             return merge_device(ctx, winners_dev, n, m, mu, out_idx, out_count, distinct);   // the union changed
         }

@@ -37,6 +37,18 @@ __global__ void map_winners_kernel(const unsigned long long* __restrict__ keys, 
     }
 }
 
+// the same for nb batches at once (blockIdx.y = batch): keys [nb][m], pool_idx [nb][M], out [nb][m]
+__global__ void map_winners_batched_kernel(const unsigned long long* __restrict__ keys, int32_t m,
+                                           const uint32_t* __restrict__ pool_idx, int64_t M,
+                                           int64_t* __restrict__ out) {
+    const int t = blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t b = blockIdx.y;
+    if (t < m) {
+        const uint32_t pos = 0xFFFFFFFFu - (uint32_t)(keys[b * m + t] & 0xFFFFFFFFull);
+        out[b * m + t] = (int64_t)pool_idx[b * M + pos];
+    }
+}
+
 // negative entries are padding: they map to 0xFFFFFFFF, which sorts last;
 // an entry >= N (a bad device-side winner list) is dropped and flags kBadWinner
 constexpr int kBadWinner = 16;

@@ -12,4 +12,4 @@ for r in $(seq 1 $REPS); do
   done
 done
 cp /tmp/libbted_new.so $LIB
-for f in $OUT/*.json; do python -c "import json; d=json.load(open('$f')); print('$f', round(d['value'],1), round(d['ms_per_step'],3), round(d['roofline']['avg_launch_ms']*1e3,2), d['clocks']['sm_mhz'])" 2>&1 | tail -1; done | tee $OUT/summary.txt
+for f in $OUT/*.json; do python -c "import json; d=json.load(open('$f')); print('$f', round(d['value'],1), round(d['ms_per_step'],3), round((d['roofline'].get('avg_launch_ms') or 0)*1e3,2), d['clocks']['sm_mhz'])" 2>&1 | tail -1; done | tee $OUT/summary.txt
