@@ -1424,26 +1424,27 @@ int small_cluster_used(int ninst, int64_t N, int32_t d) {
 
 // TEDs of at most 64 points run in one 256-thread CTA each (small.cuh ted_tiny_kernel);
 // BTED_NO_TINY_TED=1 sends them to the cluster kernel instead (A/B only)
-bool use_tiny_ted(int64_t N) {
+constexpr size_t kTinySmemMax = 200 * 1024;
+bool use_tiny_ted(int64_t N, int32_t d) {
     static const bool off = [] { const char* e = std::getenv("BTED_NO_TINY_TED"); return e && std::atoi(e); }();
-    return !off && N >= 1 && N <= bted::sm::kTinyMaxN;
+    // (the staged features must fit: otherwise the cluster kernel, which reads them from global memory)
+    return !off && N >= 1 && N <= bted::sm::kTinyMaxN && bted::sm::tiny_smem_bytes((int)N, d) <= kTinySmemMax;
 }
 // score units per TED instance of launch_small (K4's top-2 layout)
 int small_units(int ninst, int64_t N, int32_t d) {
-    return use_tiny_ted(N) ? bted::sm::kTinyUnits : small_cluster_used(ninst, N, d) * bted::sm::kWarps;
+    return use_tiny_ted(N, d) ? bted::sm::kTinyUnits : small_cluster_used(ninst, N, d) * bted::sm::kWarps;
 }
 
 void launch_small(const float* X, int ninst, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
                   unsigned long long* keys, int* err, cudaStream_t st, unsigned long long* top2 = nullptr,
                   const unsigned long long* forced = nullptr, int nforced = 0) {
-    if (use_tiny_ted(N)) {
+    if (use_tiny_ted(N, d)) {
         const size_t smem = bted::sm::tiny_smem_bytes((int)N, d);
         static uint64_t attr = 0;
         once_per_device(attr, [] {
             CK(cudaFuncSetAttribute(bted::sm::ted_tiny_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    (int)(200 * 1024)));
+                                    (int)kTinySmemMax));
         });
-        if (smem > (size_t)200 * 1024) throw CudaError{cudaErrorInvalidValue, "launch_small: d too large"};
         bted::sm::ted_tiny_kernel<<<(unsigned)ninst, bted::sm::kTinyThreads, smem, st>>>(
             X, (int32_t)N, d, gamma, (int32_t)(kernel == BTED_KERNEL_LINEAR ? 1 : 0), m, mu, keys, err, top2, forced,
             (int32_t)nforced);

@@ -115,3 +115,12 @@ def test_tiny_ted_is_deterministic_across_calls_and_contexts():
         ia2, sa2 = a.select(64, MU)
     assert np.array_equal(ia, ib) and np.array_equal(sa.view(np.uint32), sb.view(np.uint32))
     assert np.array_equal(ia, ia2) and np.array_equal(sa.view(np.uint32), sa2.view(np.uint32))
+
+
+def test_tiny_ted_widest_features():
+    """d = 64, the widest bted_create accepts, at N = 64 (the features staged in shared memory)."""
+    X = uniform_pool(64, 64, 77)
+    g = median_gamma(X, 77)
+    with bt.CandidateSet(X, g) as cs:
+        idx, sc = cs.select(48, MU)
+    check_ted(idx, sc, literal.ted(X, g, MU, 48, forced=idx), "tiny-d64")
