@@ -492,8 +492,10 @@ __device__ __forceinline__ void h_unit(double* Ls, Sync sync, const double* Lc, 
         double hk;
         if (k < tp) {
             double acc = 0.0;
-            const double* Gk = G + (int64_t)k * ldG;
-            for (int j = 0; j < tp; ++j) acc = __fma_rn(__ldcg(&Gk[j]), Ls[j], acc);
+            // G is symmetric by construction (row and column tp are both written with h below), so
+            // G[j][k] = G[k][j]: the threads k of one j read consecutive addresses (coalesced);
+            // the same values in the same order as a row walk
+            for (int j = 0; j < tp; ++j) acc = __fma_rn(__ldcg(&G[(int64_t)j * ldG + k]), Ls[j], acc);
             hk = __ddiv_rn(__dsub_rn(__ldcg(&Qc[(int64_t)k * ldL + s]), acc), rc);
             G[(int64_t)tp * ldG + k] = hk;
         } else {
