@@ -1422,7 +1422,7 @@ int small_cluster_used(int ninst, int64_t N, int32_t d) {
     return C;
 }
 
-// TEDs of at most 64 points run in one 256-thread CTA each (small.cuh ted_tiny_kernel);
+// TEDs of at most 128 points run in one CTA each (small.cuh ted_tiny_kernel<64 / 128>);
 // BTED_NO_TINY_TED=1 sends them to the cluster kernel instead (A/B only)
 constexpr size_t kTinySmemMax = 200 * 1024;
 bool use_tiny_ted(int64_t N, int32_t d) {
@@ -1432,7 +1432,7 @@ bool use_tiny_ted(int64_t N, int32_t d) {
 }
 // score units per TED instance of launch_small (K4's top-2 layout)
 int small_units(int ninst, int64_t N, int32_t d) {
-    return use_tiny_ted(N, d) ? bted::sm::kTinyUnits : small_cluster_used(ninst, N, d) * bted::sm::kWarps;
+    return use_tiny_ted(N, d) ? bted::sm::tiny_max_for((int)N) : small_cluster_used(ninst, N, d) * bted::sm::kWarps;
 }
 
 void launch_small(const float* X, int ninst, int64_t N, int32_t d, float gamma, int kernel, int32_t m, float mu,
@@ -1442,10 +1442,14 @@ void launch_small(const float* X, int ninst, int64_t N, int32_t d, float gamma, 
         const size_t smem = bted::sm::tiny_smem_bytes((int)N, d);
         static uint64_t attr = 0;
         once_per_device(attr, [] {
-            CK(cudaFuncSetAttribute(bted::sm::ted_tiny_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+            CK(cudaFuncSetAttribute(bted::sm::ted_tiny_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    (int)kTinySmemMax));
+            CK(cudaFuncSetAttribute(bted::sm::ted_tiny_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     (int)kTinySmemMax));
         });
-        bted::sm::ted_tiny_kernel<<<(unsigned)ninst, bted::sm::kTinyThreads, smem, st>>>(
+        const int kmax = bted::sm::tiny_max_for((int)N);
+        auto tk = kmax == 64 ? bted::sm::ted_tiny_kernel<64> : bted::sm::ted_tiny_kernel<128>;
+        tk<<<(unsigned)ninst, (unsigned)(4 * kmax), smem, st>>>(
             X, (int32_t)N, d, gamma, (int32_t)(kernel == BTED_KERNEL_LINEAR ? 1 : 0), m, mu, keys, err, top2, forced,
             (int32_t)nforced);
         LAUNCHED(1);

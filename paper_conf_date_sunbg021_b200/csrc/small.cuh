@@ -281,42 +281,45 @@ ted_cluster_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float g
     csync();                                         // no CTA exits while others may read its smem
 }
 
-// ---------------------------------------------------------------- N <= 64: one small CTA per TED
+// ---------------------------------------------------------------- N <= 128: one small CTA per TED
 // The |X_U| <= B m point merge of Alg. 2 l.6 at the bench's B m = 64,
-// and any other TED of at most 64 points.  A whole TED is 64 dependent steps of very
+// and any other TED of at most 128 points.  A whole TED is 64 dependent steps of very
 // little work each, so the step's latency chain is the cost: the 512-thread cluster
-// kernel spends ~1.5 us per step in shuffle trees and CTA barriers.  Here 256 threads
-// hold K in registers, thread (q, j) = (tid / 64, tid % 64) the 16 entries of column j
-// in rows 16q .. 16q + 15 (K is symmetric: a column is a row, and its squared norm is
+// kernel spends ~1.5 us per step in shuffle trees and CTA barriers.  Here 4 kMax threads
+// hold K in registers, thread (q, j) = (tid / kMax, tid % kMax) the kMax/4 entries of
+// column j in rows q kMax/4 .. (K is symmetric: a column is a row, and its squared norm is
 // the row norm of Alg. 1 l.3).  Per step, three CTA barriers:
 //   the four threads of column s publish it to shared memory | every thread deflates
 //   its 16 entries with deflate1 (the instruction every engine uses: K stays bitwise
-//   symmetric) and writes its partial sum of squares | the 64 threads of quarter 0 add
+//   symmetric) and writes its partial sum of squares | the kMax threads of quarter 0 add
 //   the four partials ((p0 + p1) + (p2 + p3)), score their column, and the two warps'
 //   argmax (redux.sync on the score bits, then on the index bits) meet in shared memory.
 // Fixed summation orders throughout (partials: four interleaved accumulators, then
 // (a0 + a1) + (a2 + a3)), so exact duplicate points have identical columns, norms and
 // scores and tie to the lowest index.  The diagonal entry of column j is carried by its
 // quarter-0 thread and updated with the same deflate1 operands as the matrix entry.
-// K4: every column is a score unit (nU = 64; top2_all[inst][t][j] = {key, 0}).
-constexpr int kTinyMaxN = 64;
-constexpr int kTinyThreads = 256;
-constexpr int kTinyRows = kTinyMaxN / 4;          // entries per thread
-constexpr int kTinyUnits = kTinyMaxN;
+// K4: every column is a score unit (nU = kMax; top2_all[inst][t][j] = {key, 0}).
+// Two sizes: kMax = 64 (256 threads, 16 entries each) and kMax = 128 (512 threads, 32 entries each:
+// e.g. the merge of two 64-point batches).  Units (K4) = kMax, one per column.
+constexpr int kTinyMaxN = 128;                     // the largest N the tiny kernels take
+__host__ __device__ __forceinline__ int tiny_max_for(int N) { return N <= 64 ? 64 : 128; }
 __host__ __device__ __forceinline__ size_t tiny_smem_bytes(int N, int d) {
-    return 16 + (size_t)(kTinyMaxN + 4 * kTinyMaxN + (size_t)N * (size_t)(d | 1)) * sizeof(float);
+    const int kMax = tiny_max_for(N);
+    return 64 + (size_t)(kMax + 4 * kMax + (size_t)N * (size_t)(d | 1)) * sizeof(float);
 }
-__global__ void __launch_bounds__(kTinyThreads, 1)
+template <int kMax>
+__global__ void __launch_bounds__(4 * kMax, 1)
 ted_tiny_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float gamma, int32_t linear, int32_t m,
                 float mu, unsigned long long* __restrict__ keys_all, int* __restrict__ err,
                 unsigned long long* __restrict__ top2_all, const unsigned long long* __restrict__ forced,
                 int32_t nforced) {
+    constexpr int kTinyThreads = 4 * kMax, kTinyRows = kMax / 4, kTinyUnits = kMax, kW0 = kMax / 32;
     extern __shared__ __align__(16) unsigned char tsm[];
-    unsigned long long* wbest = reinterpret_cast<unsigned long long*>(tsm);     // [2] the two warps' keys
-    float* piv = reinterpret_cast<float*>(tsm + 16);                            // [64] pivot column
-    float* part = piv + kTinyMaxN;                                              // [4][64] partial norms
-    float* Xs = part + 4 * kTinyMaxN;                                           // [N][d | 1] features
-    const int tid = threadIdx.x, j = tid % kTinyMaxN, q = tid / kTinyMaxN, l = tid % 32, w = tid / 32;
+    unsigned long long* wbest = reinterpret_cast<unsigned long long*>(tsm);     // [kMax / 32] quarter-0 warps' keys
+    float* piv = reinterpret_cast<float*>(tsm + 64);                            // [kMax] pivot column
+    float* part = piv + kMax;                                                   // [4][kMax] partial norms
+    float* Xs = part + 4 * kMax;                                                // [N][d | 1] features
+    const int tid = threadIdx.x, j = tid % kMax, q = tid / kMax, l = tid % 32, w = tid / 32;
     const int inst = blockIdx.x;
     const float* X = Xall + (int64_t)inst * N * d;
     unsigned long long* keys_out = keys_all + (int64_t)inst * m;
@@ -361,13 +364,13 @@ ted_tiny_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float gamm
         float a[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
         for (int r = 0; r < kTinyRows; ++r) a[r & 3] = __fmaf_rn(c[r], c[r], a[r & 3]);
-        part[q * kTinyMaxN + j] = __fadd_rn(__fadd_rn(a[0], a[1]), __fadd_rn(a[2], a[3]));
+        part[q * kMax + j] = __fadd_rn(__fadd_rn(a[0], a[1]), __fadd_rn(a[2], a[3]));
     };
     // after the partials' barrier: quarter 0 scores its columns, the CTA's argmax key
     auto argmax = [&](int t) -> unsigned long long {
         if (q == 0) {
-            const float n = __fadd_rn(__fadd_rn(part[j], part[kTinyMaxN + j]),
-                                      __fadd_rn(part[2 * kTinyMaxN + j], part[3 * kTinyMaxN + j]));
+            const float n = __fadd_rn(__fadd_rn(part[j], part[kMax + j]),
+                                      __fadd_rn(part[2 * kMax + j], part[3 * kMax + j]));
             const unsigned long long key = vj ? score_key(n, dg, mu, (uint32_t)j, selj, err) : 0ull;
             if (top2) {
                 unsigned long long* p = top2 + ((int64_t)t * kTinyUnits + j) * 2;
@@ -380,7 +383,10 @@ ted_tiny_kernel(const float* __restrict__ Xall, int32_t N, int32_t d, float gamm
             if (l == 0) wbest[w] = ((unsigned long long)mh << 32) | ml;
         }
         __syncthreads();
-        return wbest[0] > wbest[1] ? wbest[0] : wbest[1];
+        unsigned long long bb = wbest[0];
+#pragma unroll
+        for (int q2 = 1; q2 < kW0; ++q2) bb = wbest[q2] > bb ? wbest[q2] : bb;
+        return bb;
     };
     put_partial();
     __syncthreads();

@@ -24,7 +24,7 @@ def _gpu(need_gpu):
 
 
 @pytest.mark.parametrize("name,flags", ENGINES, ids=[e[0] for e in ENGINES])
-@pytest.mark.parametrize("N,m", [(64, 64), (500, 32), (1000, 24), (4099, 40)])
+@pytest.mark.parametrize("N,m", [(64, 64), (128, 64), (500, 32), (1000, 24), (4099, 40)])
 def test_repeated_selects_are_bitwise_identical(name, flags, N, m):
     _, X = make_pool(KnobSpace(WORKLOADS["resnet18_layer1"], 16), N, 3)
     g = median_gamma(X, 2)

@@ -1,6 +1,6 @@
-"""The one-CTA TED for candidate sets of at most 64 points (small.cuh
-ted_tiny_kernel): the merge TED of Alg. 2 l.6 at the bench's
-B m = 64, and every select / batch TED with N <= 64.  Against the fp64 oracle on
+"""The one-CTA TED for candidate sets of at most 128 points (small.cuh
+ted_tiny_kernel<64 / 128>): the merge TED of Alg. 2 l.6 at the bench's
+B m = 64 (and 128 for two batches), and every select / batch TED with N <= 128.  Against the fp64 oracle on
 the same seeded inputs (tests/parity.py protocol: P1 on every pick, P2 at the
 fp64 gap, with K4 at GAP_K4 where ties are exact)."""
 import numpy as np
@@ -27,7 +27,7 @@ def knob(N, d=16, seed=3, wl="resnet18_layer1"):
     return X
 
 
-@pytest.mark.parametrize("N", [1, 2, 7, 16, 31, 32, 33, 48, 63, 64])
+@pytest.mark.parametrize("N", [1, 2, 7, 16, 31, 32, 33, 48, 63, 64, 65, 97, 127, 128])
 @pytest.mark.parametrize("pool", ["knob", "uniform"])
 def test_tiny_ted_matches_oracle(N, pool):
     """Every N of the kernel's range (one and two columns per thread quarter,
@@ -58,37 +58,40 @@ def test_tiny_ted_linear_kernel():
     check_ted(idx, sc, tr, "tiny-linear")
 
 
-def test_tiny_ted_exact_duplicates_tie_to_lowest_index():
-    """32 points, each twice (rows i and i + 32 identical): exact fp32 ties on every
+@pytest.mark.parametrize("half", [32, 64])
+def test_tiny_ted_exact_duplicates_tie_to_lowest_index(half):
+    """half points, each twice (rows i and i + half identical): exact fp32 ties on every
     step; K4 re-scores them in fp64 and the lower index of a pair is always taken
     first (reading A5); P2 at the fp64 gap."""
-    base = knob(32, seed=91)
+    base = knob(half, seed=91)
     X = np.concatenate([base, base], axis=0)
+    n = 2 * half
     g = median_gamma(X, 91)
     with bt.CandidateSet(X, g) as cs:
         L.bted_reset_stats(cs.ctx)
-        idx, sc = cs.select(64, MU)
+        idx, sc = cs.select(n, MU)
         st = L.bted_get_stats(cs.ctx)
-    assert sorted(idx.tolist()) == list(range(64))
+    assert sorted(idx.tolist()) == list(range(n))
     pos = {int(v): t for t, v in enumerate(idx)}
-    for i in range(32):
-        assert pos[i] < pos[i + 32], (i, pos[i], pos[i + 32])
+    for i in range(half):
+        assert pos[i] < pos[i + half], (i, pos[i], pos[i + half])
     assert st["refined_steps"] > 0
-    check_ted(idx, sc, dense.ted(X, g, MU, 64, forced=idx), "tiny-dups", gap_exact=GAP_K4)
+    check_ted(idx, sc, dense.ted(X, g, MU, n, forced=idx), f"tiny-dups-{n}", gap_exact=GAP_K4)
 
 
-def test_tiny_ted_far_apart_points_pick_in_index_order():
+@pytest.mark.parametrize("N", [64, 128])
+def test_tiny_ted_far_apart_points_pick_in_index_order(N):
     """K = I (points 100 apart, gamma = 1): every score ties exactly; the picks are
     0, 1, ..., m-1 (pin C9 + reading A5)."""
-    X = (np.arange(64, dtype=np.float32) * 100.0).reshape(64, 1)
+    X = (np.arange(N, dtype=np.float32) * 100.0).reshape(N, 1)
     with bt.CandidateSet(X, 1.0) as cs:
-        idx, _ = cs.select(64, MU)
-    assert idx.tolist() == list(range(64))
+        idx, _ = cs.select(N, MU)
+    assert idx.tolist() == list(range(N))
 
 
 def test_tiny_ted_batches_and_their_merge():
     """Alg. 2 with batches of M = 50 (each batch TED in the tiny kernel, six
-    instances in one launch) and the 120-point merge in the cluster kernel."""
+    instances in one launch) and the 120-point merge (tiny kernel, 128-point size)."""
     P, M, B, m, seed = 4000, 50, 6, 20, 31
     X = knob(P, seed=seed)
     g = median_gamma(X, seed)
@@ -106,13 +109,14 @@ def test_tiny_ted_batches_and_their_merge():
     check_ted(mpos, [], literal.ted(X[XU], g, MU, m, forced=mpos), "tiny-batches-merge")
 
 
-def test_tiny_ted_is_deterministic_across_calls_and_contexts():
-    X = knob(64, seed=5)
+@pytest.mark.parametrize("N", [64, 128])
+def test_tiny_ted_is_deterministic_across_calls_and_contexts(N):
+    X = knob(N, seed=5)
     g = median_gamma(X, 5)
     with bt.CandidateSet(X, g) as a, bt.CandidateSet(X, g) as b:
-        ia, sa = a.select(64, MU)
-        ib, sb = b.select(64, MU)
-        ia2, sa2 = a.select(64, MU)
+        ia, sa = a.select(N, MU)
+        ib, sb = b.select(N, MU)
+        ia2, sa2 = a.select(N, MU)
     assert np.array_equal(ia, ib) and np.array_equal(sa.view(np.uint32), sb.view(np.uint32))
     assert np.array_equal(ia, ia2) and np.array_equal(sa.view(np.uint32), sa2.view(np.uint32))
 
