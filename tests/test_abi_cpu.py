@@ -121,3 +121,16 @@ def test_multi_device_params_validated_before_device():
     with pytest.raises(bt.BtedError) as e:
         bt.CandidateSet(np.zeros((4, 2), np.float32), 1.0, num_devices=-1)
     assert e.value.status == 1
+
+
+def test_update_checks_host_arrays_before_the_call():
+    """bted_update's binding: a host array of the wrong shape is rejected in Python,
+    before any pointer reaches the library; the accepted array is converted to C-contiguous fp32."""
+    with pytest.raises(ValueError):
+        L.bted_update(0, np.zeros((5, 3), np.float32), shape=(4, 3))
+    with pytest.raises(ValueError):
+        L.bted_update(0, np.zeros((12,), np.float32), shape=(4, 3))
+    # a null context with a well-formed array reaches the library, which refuses it (EINVAL)
+    with pytest.raises(bt.BtedError) as e:
+        L.bted_update(0, np.zeros((4, 3), np.float64).T.copy().T, shape=(4, 3))
+    assert e.value.status == 1
