@@ -91,6 +91,7 @@ struct TPSmem {
     double colstage[2][kTPWarps][T];                          // double-buffered per tile
     double wslot[kWSlots][2][T];                              // [slot][0: w on block J, 1: w on block I]
     int64_t wtile[kWSlots];                                   // the slot's tile index (-1: end of pass)
+    int wI[kWSlots], wJ[kWSlots];                             // ... and its block coordinates (I <= J)
     double red[kTPWarps];
     double rowx[kTPWarps][4][kRowxLd];                        // per-warp row-group transposes
     uint64_t full[kStages], empty[kStages];
@@ -202,8 +203,7 @@ __device__ __forceinline__ void tp_consume(Sm& S, int nT, double* P64, int* __re
             ++tile_it;
             break;
         }
-        int I, J;
-        tile_ij(k, nT, I, J);
+        const int I = S.wI[ws], J = S.wJ[ws];                 // published by the producer with k
         const bool offdiag = I != J;
         double wc[4];                                         // w on the lane's 4 columns
         if (!kNorm) {
@@ -334,11 +334,15 @@ __device__ __forceinline__ void tp_produce(Sm& S, const float* __restrict__ K, i
             const int ws = ti % kWSlots;
             pk::mbar_wait(&S.wempty[ws], ((uint32_t)(ti / kWSlots) & 1u) ^ 1u);
             S.wtile[ws] = k < nAll ? k : -1;
+            int I = 0, J = 0;
+            if (k < nAll) {                                   // the coordinates once, for every consumer
+                tile_ij(k, nT, I, J);
+                S.wI[ws] = I;
+                S.wJ[ws] = J;
+            }
             if (k >= nAll || !kW) {
                 pk::mbar_arrive(&S.wfull[ws]);               // release: the tile index
             } else {
-                int I, J;
-                tile_ij(k, nT, I, J);
                 wait_w(pass, I, J);
                 pk::mbar_expect_tx(&S.wfull[ws], 2 * T * 8);
                 pk::bulk_g2s(S.wslot[ws][0], w + (int64_t)J * T, T * 8, &S.wfull[ws]);
